@@ -1,0 +1,227 @@
+/*
+ * oracle.c -- TEST INFRASTRUCTURE ONLY.  The plain, slow, obviously-correct CPU
+ * oracle for the tridiagonal solve A x = d (Sec. II.A, Eq 1).
+ *
+ * Only tests/, __graft_entry__.smoke() and bench.py's cpu_baseline / --impl
+ * reference legs may load this library.  It shares no code, header, table or
+ * helper with the CUDA path (paper_conf_icpp_kimwch11_b200/), and it never
+ * includes include/tri.h.
+ *
+ * Build: gcc -O2 -ffp-contract=off -fno-fast-math (no FMA contraction, IEEE
+ * division), so the arithmetic is exactly the textbook operation sequence.
+ *
+ * What the method computes: the method (tiled PCR + p-Thomas) is a DIRECT
+ * solver -- PCR steps are row operations that preserve the solution (P:205,
+ * P:253) and Thomas is Gaussian elimination specialised to tridiagonal A.
+ * So the oracle is the plain definition of the result: x = A^{-1} d per system,
+ * computed by
+ *   - oracle_thomas:   Thomas algorithm exactly as Eqs 2-4, fp64;
+ *   - oracle_dense_ge: textbook dense Gaussian elimination with partial pivoting
+ *                      on the assembled n x n matrix (independent code path);
+ *   - oracle_pcr_step: one PCR forward-reduction step, Eqs 5-6 at
+ *                      stride sigma (reading X3/X4), used by tests of
+ *                      the PCR stage and by the k-step reduced-system checks;
+ *   - oracle_residual: relative residual ||Ax-d||_inf/||d||_inf and normwise
+ *                      backward error, accumulated in long double.
+ * Pins (tests/test_oracle.py): exact rational brute force, dense GE, LAPACK
+ * dgtsv, Poisson closed form, integer-manufactured exact solutions, residual
+ * invariant, paper Figs 3/4/6 index structure.
+ *
+ * Conventions: arrays have length n, 0-based.  a[0] and c[n-1] lie outside A
+ * (Eq 1 is 1-based with no a_1, c_n; reading X1) and are IGNORED
+ * (read as 0), whatever they hold.
+ */
+#include <stdint.h>
+#include <stdlib.h>
+#include <string.h>
+#include <math.h>
+#include <pthread.h>
+
+/* ---- Thomas algorithm, Eqs 2-4; reading X2 for the garbled text --
+ *   c'_1 = c_1/b_1,  c'_i = c_i / (b_i - c'_{i-1} a_i),            i = 2..n-1  (Eq 2)
+ *   d'_1 = d_1/b_1,  d'_i = (d_i - d'_{i-1} a_i)/(b_i - c'_{i-1} a_i), i = 2..n (Eq 3)
+ *   x_n = d'_n,      x_i = d'_i - c'_i x_{i+1},                   i = n-1..1  (Eq 4)
+ * cp and dp are caller-provided work arrays of length n.                      */
+void oracle_thomas(int64_t n, const double* a, const double* b, const double* c,
+                   const double* d, double* x, double* cp, double* dp) {
+    if (n < 1) return;
+    if (n == 1) { x[0] = d[0] / b[0]; return; }
+    cp[0] = c[0] / b[0];
+    dp[0] = d[0] / b[0];
+    for (int64_t i = 1; i < n; ++i) {
+        double den = b[i] - cp[i - 1] * a[i];
+        if (i < n - 1) cp[i] = c[i] / den;
+        dp[i] = (d[i] - dp[i - 1] * a[i]) / den;
+    }
+    x[n - 1] = dp[n - 1];
+    for (int64_t i = n - 2; i >= 0; --i) x[i] = dp[i] - cp[i] * x[i + 1];
+}
+
+/* ---- Dense Gaussian elimination with partial pivoting (textbook) ----------
+ * M is n x n row-major (overwritten), r is the rhs (overwritten), x the result.
+ * Independent of the tridiagonal structure: used as brute force for n <= 64. */
+int oracle_dense_ge(int64_t n, double* M, double* r, double* x) {
+    for (int64_t k = 0; k < n; ++k) {
+        int64_t p = k;
+        for (int64_t i = k + 1; i < n; ++i)
+            if (fabs(M[i * n + k]) > fabs(M[p * n + k])) p = i;
+        if (M[p * n + k] == 0.0) return 1;
+        if (p != k) {
+            for (int64_t j = 0; j < n; ++j) {
+                double t = M[k * n + j]; M[k * n + j] = M[p * n + j]; M[p * n + j] = t;
+            }
+            double t = r[k]; r[k] = r[p]; r[p] = t;
+        }
+        for (int64_t i = k + 1; i < n; ++i) {
+            double l = M[i * n + k] / M[k * n + k];
+            for (int64_t j = k; j < n; ++j) M[i * n + j] -= l * M[k * n + j];
+            r[i] -= l * r[k];
+        }
+    }
+    for (int64_t i = n - 1; i >= 0; --i) {
+        double s = r[i];
+        for (int64_t j = i + 1; j < n; ++j) s -= M[i * n + j] * x[j];
+        x[i] = s / M[i * n + i];
+    }
+    return 0;
+}
+
+/* Assemble the dense n x n matrix of Eq 1 from (a, b, c); a[0], c[n-1] ignored. */
+void oracle_assemble(int64_t n, const double* a, const double* b, const double* c, double* M) {
+    memset(M, 0, (size_t)(n * n) * sizeof(double));
+    for (int64_t i = 0; i < n; ++i) {
+        if (i > 0) M[i * n + i - 1] = a[i];
+        M[i * n + i] = b[i];
+        if (i < n - 1) M[i * n + i + 1] = c[i];
+    }
+}
+
+/* ---- One PCR forward-reduction step at stride s, Eqs 5-6 -------
+ *   k1 = a_i / b_{i-s},  k2 = c_i / b_{i+s}
+ *   a'_i = -a_{i-s} k1,  b'_i = b_i - c_{i-s} k1 - a_{i+s} k2
+ *   c'_i = -c_{i+s} k2,  d'_i = d_i - d_{i-s} k1 - d_{i+s} k2
+ * The paper writes the step for stride 1; PCR applies it with stride 2^j at step
+ * j (Fig 4; reading X3).  Neighbours outside [0, n) are identity rows
+ * a = c = d = 0, b = 1 (reading X4).  Inputs must already have a[0] = c[n-1] = 0
+ * semantics; this function reads a[i] for i < s as given, so callers pass arrays
+ * with a[0] = c[n-1] = 0 (oracle_pcr_k does this). */
+void oracle_pcr_step(int64_t n, int64_t s, const double* a, const double* b, const double* c,
+                     const double* d, double* a2, double* b2, double* c2, double* d2) {
+    for (int64_t i = 0; i < n; ++i) {
+        double am = 0.0, bm = 1.0, cm = 0.0, dm = 0.0; /* row i-s */
+        double ap = 0.0, bp = 1.0, cp = 0.0, dp = 0.0; /* row i+s */
+        if (i - s >= 0) { am = a[i - s]; bm = b[i - s]; cm = c[i - s]; dm = d[i - s]; }
+        if (i + s < n) { ap = a[i + s]; bp = b[i + s]; cp = c[i + s]; dp = d[i + s]; }
+        double k1 = a[i] / bm;
+        double k2 = c[i] / bp;
+        a2[i] = -am * k1;
+        b2[i] = b[i] - cm * k1 - ap * k2;
+        c2[i] = -cp * k2;
+        d2[i] = d[i] - dm * k1 - dp * k2;
+    }
+}
+
+/* k PCR steps (strides 1, 2, ..., 2^{k-1}) on one system; outputs may alias
+ * nothing.  Work arrays: 4n doubles. a[0], c[n-1] are zeroed first (X1). */
+void oracle_pcr_k(int64_t n, int k, const double* a, const double* b, const double* c,
+                  const double* d, double* ao, double* bo, double* co, double* dout, double* work) {
+    double *ta = work, *tb = work + n, *tc = work + 2 * n, *td = work + 3 * n;
+    memcpy(ao, a, (size_t)n * sizeof(double));
+    memcpy(bo, b, (size_t)n * sizeof(double));
+    memcpy(co, c, (size_t)n * sizeof(double));
+    memcpy(dout, d, (size_t)n * sizeof(double));
+    ao[0] = 0.0; co[n - 1] = 0.0;
+    for (int j = 0; j < k; ++j) {
+        int64_t s = (int64_t)1 << j;
+        oracle_pcr_step(n, s, ao, bo, co, dout, ta, tb, tc, td);
+        memcpy(ao, ta, (size_t)n * sizeof(double));
+        memcpy(bo, tb, (size_t)n * sizeof(double));
+        memcpy(co, tc, (size_t)n * sizeof(double));
+        memcpy(dout, td, (size_t)n * sizeof(double));
+    }
+}
+
+/* ---- residuals, accumulated in long double (x86 80-bit) --------------------
+ * out[0] = ||A x - d||_inf / ||d||_inf
+ * out[1] = ||A x - d||_inf / || |A||x| + |d| ||_inf   (normwise backward error) */
+void oracle_residual(int64_t n, const double* a, const double* b, const double* c,
+                     const double* d, const double* x, double* out) {
+    long double rmax = 0.0L, dmax = 0.0L, smax = 0.0L;
+    for (int64_t i = 0; i < n; ++i) {
+        long double r = (long double)b[i] * x[i] - d[i];
+        long double s = fabsl((long double)b[i] * x[i]) + fabsl((long double)d[i]);
+        if (i > 0) { r += (long double)a[i] * x[i - 1]; s += fabsl((long double)a[i] * x[i - 1]); }
+        if (i < n - 1) { r += (long double)c[i] * x[i + 1]; s += fabsl((long double)c[i] * x[i + 1]); }
+        if (fabsl(r) > rmax) rmax = fabsl(r);
+        if (fabsl((long double)d[i]) > dmax) dmax = fabsl((long double)d[i]);
+        if (s > smax) smax = s;
+    }
+    out[0] = dmax > 0 ? (double)(rmax / dmax) : (double)rmax;
+    out[1] = smax > 0 ? (double)(rmax / smax) : (double)rmax;
+}
+
+/* ---- batch driver: threads over independent systems (the paper's MKL
+ * threading policy).  Reads a, b, c, d of dtype (0 f32 / 1 f64) in
+ * layout (0 contiguous [q*n+i], 1 interleaved [i*m+q]); upcasts f32 exactly to
+ * f64; writes x (f64) in the same layout.  Optional resid (2*m doubles) gets
+ * oracle_residual per system.  Systems [q_begin, q_end) only (for bounded
+ * samples); nthreads <= 0 means 1.                                            */
+typedef struct {
+    int64_t n, m, q_begin, q_end;
+    int dtype, layout;
+    const void *a, *b, *c, *d;
+    double* x;
+    double* resid;
+    int64_t next;
+    pthread_mutex_t mu;
+} batch_t;
+
+static double ld_elem(const void* p, int dtype, int64_t idx) {
+    return dtype == 1 ? ((const double*)p)[idx] : (double)((const float*)p)[idx];
+}
+
+static void* batch_worker(void* arg) {
+    batch_t* B = (batch_t*)arg;
+    const int64_t n = B->n;
+    double* buf = (double*)malloc((size_t)(7 * n) * sizeof(double));
+    double *a = buf, *b = buf + n, *c = buf + 2 * n, *d = buf + 3 * n, *x = buf + 4 * n;
+    double *cp = buf + 5 * n, *dp = buf + 6 * n;
+    for (;;) {
+        pthread_mutex_lock(&B->mu);
+        int64_t q = B->next++;
+        pthread_mutex_unlock(&B->mu);
+        if (q >= B->q_end) break;
+        for (int64_t i = 0; i < n; ++i) {
+            int64_t idx = B->layout == 0 ? q * n + i : i * B->m + q;
+            a[i] = ld_elem(B->a, B->dtype, idx);
+            b[i] = ld_elem(B->b, B->dtype, idx);
+            c[i] = ld_elem(B->c, B->dtype, idx);
+            d[i] = ld_elem(B->d, B->dtype, idx);
+        }
+        a[0] = 0.0;     /* reading X1: outside A, ignored */
+        c[n - 1] = 0.0;
+        oracle_thomas(n, a, b, c, d, x, cp, dp);
+        for (int64_t i = 0; i < n; ++i) {
+            int64_t idx = B->layout == 0 ? q * n + i : i * B->m + q;
+            B->x[idx] = x[i];
+        }
+        if (B->resid) oracle_residual(n, a, b, c, d, x, B->resid + 2 * q);
+    }
+    free(buf);
+    return NULL;
+}
+
+int oracle_solve_batch(int64_t n, int64_t m, int dtype, int layout, const void* a, const void* b,
+                       const void* c, const void* d, double* x, double* resid, int64_t q_begin,
+                       int64_t q_end, int nthreads) {
+    if (n < 1 || m < 1 || q_begin < 0 || q_end > m || q_begin > q_end) return 1;
+    if (nthreads < 1) nthreads = 1;
+    batch_t B = {n, m, q_begin, q_end, dtype, layout, a, b, c, d, x, resid, q_begin};
+    pthread_mutex_init(&B.mu, NULL);
+    pthread_t* th = (pthread_t*)malloc(sizeof(pthread_t) * (size_t)nthreads);
+    for (int t = 0; t < nthreads; ++t) pthread_create(&th[t], NULL, batch_worker, &B);
+    for (int t = 0; t < nthreads; ++t) pthread_join(th[t], NULL);
+    free(th);
+    pthread_mutex_destroy(&B.mu);
+    return 0;
+}
