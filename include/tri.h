@@ -1,0 +1,137 @@
+/*
+ * tri.h -- C ABI of the B200 (sm_100a) hybrid tridiagonal solver.
+ *
+ * Operation (Sec. II.A, Eq 1): for each of m independent
+ * systems q, solve A_q x_q = d_q where A_q is n x n tridiagonal with
+ * sub-diagonal a (a_2..a_n), diagonal b (b_1..b_n) and super-diagonal c
+ * (c_1..c_{n-1}).  Method (Sec. III): k steps of tiled parallel
+ * cyclic reduction (Eqs 5-6 at stride 2^j) split every
+ * system into 2^k interleaved independent subsystems, then thread-level
+ * parallel Thomas (Eqs 2-4) solves each subsystem with one
+ * thread.  The transition point k is chosen at plan time from n, m, the dtype
+ * and the SM count; tri_plan_set_k overrides it.
+ *
+ * Conventions common to every call:
+ *   - Element (system q, row i), 0 <= q < m, 0 <= i < n, lives at
+ *       TRI_LAYOUT_CONTIGUOUS :  [q*n + i]   (system-major)
+ *       TRI_LAYOUT_INTERLEAVED:  [i*m + q]   (the paper's interleave)
+ *     in each of a, b, c, d, x; every array holds n*m elements of the dtype.
+ *   - a[q][0] and c[q][n-1] lie outside A (Eq 1) and are IGNORED (read as 0,
+ *     whatever they hold, including NaN) -- DESIGN.md reading X1.
+ *   - No pivoting: the precondition is diagonal dominance (or SPD); numerical
+ *     breakdown is not detected (reading X6).
+ *   - No exceptions cross the ABI; every fallible call returns a tri_status.
+ *   - All device pointers must be 16-byte aligned device allocations on the
+ *     plan's device; x must not overlap a, b, c or d.
+ *   - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).
+ *     tri_solve is stream-ordered and asynchronous.
+ *   - Determinism: a given (plan, inputs) gives bitwise-identical x every run.
+ */
+#ifndef TRI_H
+#define TRI_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#if defined(__GNUC__)
+#define TRI_API __attribute__((visibility("default")))
+#else
+#define TRI_API
+#endif
+
+typedef enum { TRI_F32 = 0, TRI_F64 = 1 } tri_dtype;
+
+typedef enum {
+    TRI_LAYOUT_CONTIGUOUS = 0,  /* element i of system q at [q*n + i] */
+    TRI_LAYOUT_INTERLEAVED = 1  /* element i of system q at [i*m + q] */
+} tri_layout;
+
+typedef enum {
+    TRI_OK = 0,
+    TRI_ERR_INVALID_ARG = 1, /* bad n, m, dtype, layout, k, variant, NULL pointer */
+    TRI_ERR_ALIGNMENT = 2,   /* a device pointer not 16-byte aligned */
+    TRI_ERR_ALIAS = 3,       /* x overlaps a, b, c or d */
+    TRI_ERR_DEVICE = 4,      /* no CUDA device / not sm_100 / pointer not on the plan's device */
+    TRI_ERR_OOM = 5,         /* scratch or staging allocation failed */
+    TRI_ERR_CUDA = 6         /* a CUDA runtime call or kernel launch failed */
+} tri_status;
+
+/* Kernel variants; the planner picks one, tests may force. */
+typedef enum {
+    TRI_VARIANT_AUTO = 0,   /* only as an argument of tri_plan_set_variant */
+    TRI_VARIANT_ONCHIP = 1, /* whole system(s) in one CTA's smem: PCR + Thomas (Fig 11a/c) */
+    TRI_VARIANT_SPLIT = 2,  /* tiled-PCR pass (sliding window, Figs 8-10) -> scratch, then p-Thomas */
+    TRI_VARIANT_FUSED = 3   /* streaming tiled PCR feeding p-Thomas in one kernel (Sec. III.C) */
+} tri_variant;
+
+typedef struct tri_plan_s* tri_plan_t;
+
+/* Create a plan for m systems of size n on the CURRENT CUDA device.
+ * n >= 1, m >= 1, n*m <= 2^40.  Chooses k and the variant, allocates the
+ * plan-owned device scratch.  Returns NULL on failure; tri_last_status() says
+ * why (TRI_ERR_INVALID_ARG, TRI_ERR_DEVICE, TRI_ERR_OOM, TRI_ERR_CUDA). */
+TRI_API tri_plan_t tri_plan(int64_t n, int64_t m, tri_dtype dtype, tri_layout layout);
+
+/* Thread-local status of the last tri_plan call on this thread. */
+TRI_API tri_status tri_last_status(void);
+
+/* Solve: read a, b, c, d (device, read-only), write x (device).  Asynchronous
+ * on `stream`.  At most one tri_solve per plan may be in flight (the plan's
+ * scratch is reused); use one plan per concurrent stream. */
+TRI_API tri_status tri_solve(tri_plan_t plan, const void* a, const void* b, const void* c, const void* d,
+                     void* x, void* stream);
+
+/* End-to-end solve through HOST buffers: copies a, b, c, d host->device into
+ * plan-owned staging, solves, copies x device->host, all on `stream`, then
+ * synchronises `stream`.  Host buffers should be pinned for full bandwidth.
+ * Returns after x is in host memory. */
+TRI_API tri_status tri_solve_host(tri_plan_t plan, const void* a, const void* b, const void* c,
+                          const void* d, void* x, void* stream);
+
+/* Run only the tiled-PCR stage (k steps, Eqs 5-6 at strides 1..2^{k-1}) and
+ * write the reduced system, rows normalised to unit diagonal (a/b, 1, c/b,
+ * d/b; reading X17), into ao, co, do_ in the plan's layout.  For
+ * tests of SURVEY 8(a) row A2.  Same pointer rules as tri_solve. */
+TRI_API tri_status tri_debug_pcr(tri_plan_t plan, const void* a, const void* b, const void* c,
+                         const void* d, void* ao, void* co, void* do_, void* stream);
+
+/* Release the plan and its scratch.  NULL-safe.  Must not race a solve. */
+TRI_API void tri_destroy(tri_plan_t plan);
+
+/* Plan introspection and overrides. */
+TRI_API int tri_plan_k(tri_plan_t plan);                     /* chosen transition point k, -1 if NULL */
+TRI_API int tri_plan_variant(tri_plan_t plan);               /* tri_variant in use, -1 if NULL */
+TRI_API int tri_plan_launches(tri_plan_t plan);              /* kernels launched per tri_solve */
+TRI_API int64_t tri_plan_scratch_bytes(tri_plan_t plan);     /* plan-owned device scratch */
+/* 0 <= k <= floor(log2 n) and k <= the variant's limit, else TRI_ERR_INVALID_ARG. */
+TRI_API tri_status tri_plan_set_k(tri_plan_t plan, int k);
+/* Force a variant (TRI_VARIANT_AUTO re-runs the planner); re-plans k if the
+ * current k is invalid for it; may reallocate scratch (TRI_ERR_OOM). */
+TRI_API tri_status tri_plan_set_variant(tri_plan_t plan, tri_variant v);
+/* Human-readable one-line plan description into buf (NUL-terminated). */
+TRI_API void tri_plan_describe(tri_plan_t plan, char* buf, int buflen);
+
+TRI_API const char* tri_status_str(tri_status s);
+
+/* ---- pure host helpers (no device needed; unit-testable on CPU) ---------- */
+/* Eq 8: redundant loads per tile boundary f(k) = sum_{i<k} 2^i. */
+TRI_API int64_t tri_halo_f(int k);
+/* Eq 9: redundant eliminations g(k) = k f(k) - sum_{i<=k} f(i). */
+TRI_API int64_t tri_halo_g(int k);
+/* The planner's heuristic (Sec. III.D, re-derived for B200 in
+ * DESIGN.md): transition point k for (n, m, dtype, layout) on sm_count SMs. */
+TRI_API int tri_choose_k(int64_t n, int64_t m, tri_dtype dtype, tri_layout layout, int sm_count);
+/* The planner's variant choice for the same arguments (a tri_variant). */
+TRI_API int tri_choose_variant(int64_t n, int64_t m, tri_dtype dtype, tri_layout layout, int sm_count);
+/* Contiguous shard of m systems for rank r of G (multi-GPU):
+ * q0 = r*ceil(m/G) clipped to m, mr = min(ceil(m/G), m - q0). */
+TRI_API void tri_shard_range(int64_t m, int G, int r, int64_t* q0, int64_t* mr);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* TRI_H */

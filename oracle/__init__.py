@@ -54,6 +54,9 @@ def _load():
         lib.oracle_solve_batch.argtypes = [_I64, _I64, ctypes.c_int, ctypes.c_int, _P, _P, _P, _P, _P, _P,
                                            _I64, _I64, ctypes.c_int]
         lib.oracle_solve_batch.restype = ctypes.c_int
+        lib.oracle_residual_batch.argtypes = [_I64, _I64, ctypes.c_int, ctypes.c_int, _P, _P, _P, _P, _P, _P,
+                                              ctypes.c_int]
+        lib.oracle_residual_batch.restype = ctypes.c_int
         _lib = lib
     return _lib
 
@@ -142,3 +145,20 @@ def solve_batch(n, m, a, b, c, d, layout=0, want_resid=False, q_begin=0, q_end=N
     if rc != 0:
         raise ValueError("oracle_solve_batch: bad arguments")
     return (x, res.reshape(m, 2)) if want_resid else x
+
+
+def residual_batch(n, m, a, b, c, d, x, layout=0, nthreads=None):
+    """Per-system (relative residual, backward error) of a given solution x
+    (any float dtype; upcast to f64) -> array of shape (m, 2)."""
+    assert a.dtype == b.dtype == c.dtype == d.dtype
+    dt = 1 if a.dtype == np.float64 else 0
+    if nthreads is None:
+        nthreads = len(os.sched_getaffinity(0))
+    xx = np.ascontiguousarray(x, dtype=np.float64)
+    out = np.zeros(2 * m, np.float64)
+    arrs = [np.ascontiguousarray(t) for t in (a, b, c, d)]
+    rc = _load().oracle_residual_batch(int(n), int(m), dt, int(layout), *map(_p, arrs), _p(xx), _p(out),
+                                       int(nthreads))
+    if rc != 0:
+        raise ValueError("oracle_residual_batch: bad arguments")
+    return out.reshape(m, 2)

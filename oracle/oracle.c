@@ -225,3 +225,54 @@ int oracle_solve_batch(int64_t n, int64_t m, int dtype, int layout, const void* 
     pthread_mutex_destroy(&B.mu);
     return 0;
 }
+
+/* ---- residuals of a GIVEN solution (e.g. the GPU's x, upcast to f64) for every
+ * system of a batch: out[2q] = relative residual, out[2q+1] = backward error of
+ * system q (oracle_residual; a[0], c[n-1] ignored).  Threads over systems.     */
+typedef struct {
+    int64_t n, m;
+    int dtype, layout;
+    const void *a, *b, *c, *d;
+    const double* x;
+    double* out;
+    int64_t next;
+    pthread_mutex_t mu;
+} rbatch_t;
+
+static void* rbatch_worker(void* arg) {
+    rbatch_t* B = (rbatch_t*)arg;
+    const int64_t n = B->n;
+    double* buf = (double*)malloc((size_t)(5 * n) * sizeof(double));
+    double *a = buf, *b = buf + n, *c = buf + 2 * n, *d = buf + 3 * n, *x = buf + 4 * n;
+    for (;;) {
+        pthread_mutex_lock(&B->mu);
+        int64_t q = B->next++;
+        pthread_mutex_unlock(&B->mu);
+        if (q >= B->m) break;
+        for (int64_t i = 0; i < n; ++i) {
+            int64_t idx = B->layout == 0 ? q * n + i : i * B->m + q;
+            a[i] = ld_elem(B->a, B->dtype, idx);
+            b[i] = ld_elem(B->b, B->dtype, idx);
+            c[i] = ld_elem(B->c, B->dtype, idx);
+            d[i] = ld_elem(B->d, B->dtype, idx);
+            x[i] = B->x[idx];
+        }
+        oracle_residual(n, a, b, c, d, x, B->out + 2 * q);
+    }
+    free(buf);
+    return NULL;
+}
+
+int oracle_residual_batch(int64_t n, int64_t m, int dtype, int layout, const void* a, const void* b,
+                          const void* c, const void* d, const double* x, double* out, int nthreads) {
+    if (n < 1 || m < 1) return 1;
+    if (nthreads < 1) nthreads = 1;
+    rbatch_t B = {n, m, dtype, layout, a, b, c, d, x, out, 0};
+    pthread_mutex_init(&B.mu, NULL);
+    pthread_t* th = (pthread_t*)malloc(sizeof(pthread_t) * (size_t)nthreads);
+    for (int t = 0; t < nthreads; ++t) pthread_create(&th[t], NULL, rbatch_worker, &B);
+    for (int t = 0; t < nthreads; ++t) pthread_join(th[t], NULL);
+    free(th);
+    pthread_mutex_destroy(&B.mu);
+    return 0;
+}

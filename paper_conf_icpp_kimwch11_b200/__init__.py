@@ -1,0 +1,219 @@
+"""B200-native hybrid tridiagonal solver (tiled PCR + p-Thomas; Kim, Wu, Chang,
+Hwu, "A Scalable Tridiagonal Solver for GPUs", ICPP 2011).
+
+Thin Python binding over the C ABI in include/tri.h (libtri.so, sm_100a).
+Argument marshalling only: every step of the solve runs in the CUDA kernels.
+There is no CPU fallback -- if libtri.so is missing or cannot load, importing
+the binding raises.  PyTorch supplies device memory, streams and process
+groups (plumbing only).
+"""
+import ctypes
+import os
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(HERE, "libtri.so")
+
+F32, F64 = 0, 1
+CONTIGUOUS, INTERLEAVED = 0, 1
+VARIANT_AUTO, VARIANT_ONCHIP, VARIANT_SPLIT, VARIANT_FUSED = 0, 1, 2, 3
+VARIANT_NAMES = {1: "onchip", 2: "split", 3: "fused"}
+STATUS = {0: "TRI_OK", 1: "TRI_ERR_INVALID_ARG", 2: "TRI_ERR_ALIGNMENT", 3: "TRI_ERR_ALIAS",
+          4: "TRI_ERR_DEVICE", 5: "TRI_ERR_OOM", 6: "TRI_ERR_CUDA"}
+
+
+class TriError(RuntimeError):
+    def __init__(self, status, what=""):
+        self.status = status
+        super().__init__(f"{what}: {STATUS.get(status, status)}")
+
+
+_lib = None
+_P = ctypes.c_void_p
+_I64 = ctypes.c_int64
+_I = ctypes.c_int
+
+
+def lib():
+    """Load libtri.so (raises OSError if it is missing: no fallback)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise OSError(f"{LIB_PATH} not built; run __graft_entry__.build() "
+                          "(python paper_conf_icpp_kimwch11_b200/_build.py)")
+        L = ctypes.CDLL(LIB_PATH)
+        sig = {
+            "tri_plan": (_P, [_I64, _I64, _I, _I]),
+            "tri_last_status": (_I, []),
+            "tri_solve": (_I, [_P] * 7),
+            "tri_solve_host": (_I, [_P] * 7),
+            "tri_debug_pcr": (_I, [_P] * 9),
+            "tri_destroy": (None, [_P]),
+            "tri_plan_k": (_I, [_P]),
+            "tri_plan_variant": (_I, [_P]),
+            "tri_plan_launches": (_I, [_P]),
+            "tri_plan_scratch_bytes": (_I64, [_P]),
+            "tri_plan_set_k": (_I, [_P, _I]),
+            "tri_plan_set_variant": (_I, [_P, _I]),
+            "tri_plan_describe": (None, [_P, ctypes.c_char_p, _I]),
+            "tri_status_str": (ctypes.c_char_p, [_I]),
+            "tri_halo_f": (_I64, [_I]),
+            "tri_halo_g": (_I64, [_I]),
+            "tri_choose_k": (_I, [_I64, _I64, _I, _I, _I]),
+            "tri_choose_variant": (_I, [_I64, _I64, _I, _I, _I]),
+            "tri_shard_range": (None, [_I64, _I, _I, ctypes.POINTER(_I64), ctypes.POINTER(_I64)]),
+        }
+        for name, (res, args) in sig.items():
+            fn = getattr(L, name)
+            fn.restype = res
+            fn.argtypes = args
+        _lib = L
+    return _lib
+
+
+def halo_f(k):
+    """Eq 8."""
+    return lib().tri_halo_f(k)
+
+
+def halo_g(k):
+    """Eq 9."""
+    return lib().tri_halo_g(k)
+
+
+def choose_k(n, m, dtype=F64, layout=CONTIGUOUS, sm_count=148):
+    return lib().tri_choose_k(n, m, dtype, layout, sm_count)
+
+
+def choose_variant(n, m, dtype=F64, layout=CONTIGUOUS, sm_count=148):
+    return lib().tri_choose_variant(n, m, dtype, layout, sm_count)
+
+
+def shard_range(m, G, r):
+    """Contiguous system range (q0, m_r) of rank r among G (no collective in the solve)."""
+    q0, mr = _I64(), _I64()
+    lib().tri_shard_range(m, G, r, ctypes.byref(q0), ctypes.byref(mr))
+    return q0.value, mr.value
+
+
+def _dtype_code(dtype):
+    import torch
+    if dtype in (F64, "f64", torch.float64):
+        return F64
+    if dtype in (F32, "f32", torch.float32):
+        return F32
+    raise ValueError(f"unsupported dtype {dtype}")
+
+
+class Plan:
+    """Plan(n, m, dtype, layout) -> .solve(a, b, c, d, out=x) on CUDA tensors.
+
+    Wraps tri_plan / tri_solve (include/tri.h).  The plan is bound to the CUDA
+    device current at construction and owns its scratch."""
+
+    def __init__(self, n, m, dtype=F64, layout=CONTIGUOUS):
+        import torch
+        self.n, self.m = int(n), int(m)
+        self.dtype_code = _dtype_code(dtype)
+        self.torch_dtype = torch.float64 if self.dtype_code == F64 else torch.float32
+        self.layout = int(layout)
+        h = lib().tri_plan(self.n, self.m, self.dtype_code, self.layout)
+        if not h:
+            raise TriError(lib().tri_last_status(), "tri_plan")
+        self._h = ctypes.c_void_p(h)
+        self.device = torch.cuda.current_device()
+
+    def __del__(self):
+        h = getattr(self, "_h", None)
+        if h is not None and _lib is not None:
+            _lib.tri_destroy(h)
+            self._h = None
+
+    @property
+    def k(self):
+        return lib().tri_plan_k(self._h)
+
+    @k.setter
+    def k(self, value):
+        st = lib().tri_plan_set_k(self._h, int(value))
+        if st != 0:
+            raise TriError(st, f"tri_plan_set_k({value})")
+
+    @property
+    def variant(self):
+        return lib().tri_plan_variant(self._h)
+
+    @variant.setter
+    def variant(self, v):
+        st = lib().tri_plan_set_variant(self._h, int(v))
+        if st != 0:
+            raise TriError(st, f"tri_plan_set_variant({v})")
+
+    @property
+    def launches(self):
+        return lib().tri_plan_launches(self._h)
+
+    @property
+    def scratch_bytes(self):
+        return lib().tri_plan_scratch_bytes(self._h)
+
+    def describe(self):
+        buf = ctypes.create_string_buffer(512)
+        lib().tri_plan_describe(self._h, buf, 512)
+        return buf.value.decode()
+
+    def _check(self, *ts):
+        for t in ts:
+            if not t.is_cuda or t.dtype != self.torch_dtype or t.numel() != self.n * self.m \
+                    or not t.is_contiguous():
+                raise ValueError(f"expected contiguous CUDA {self.torch_dtype} tensor of {self.n * self.m} "
+                                 f"elements, got {t.dtype} {tuple(t.shape)} on {t.device}")
+
+    def solve(self, a, b, c, d, out=None, stream=None):
+        import torch
+        if out is None:
+            out = torch.empty_like(b)
+        self._check(a, b, c, d, out)
+        s = stream if stream is not None else torch.cuda.current_stream()
+        st = lib().tri_solve(self._h, a.data_ptr(), b.data_ptr(), c.data_ptr(), d.data_ptr(),
+                             out.data_ptr(), s.cuda_stream)
+        if st != 0:
+            raise TriError(st, "tri_solve")
+        return out
+
+    def solve_raw(self, a, b, c, d, x, stream=0):
+        """tri_solve on raw device pointers (ints); returns the status code."""
+        return lib().tri_solve(self._h, a, b, c, d, x, stream)
+
+    def solve_host(self, a, b, c, d, out, stream=None):
+        """End-to-end through host buffers (tri_solve_host): a..d, out are
+        host tensors/arrays (pinned for bandwidth); copies are inside the call."""
+        import torch
+
+        def ptr(t):
+            return t.data_ptr() if isinstance(t, torch.Tensor) else t.ctypes.data
+        s = stream if stream is not None else torch.cuda.current_stream()
+        st = lib().tri_solve_host(self._h, ptr(a), ptr(b), ptr(c), ptr(d), ptr(out), s.cuda_stream)
+        if st != 0:
+            raise TriError(st, "tri_solve_host")
+        return out
+
+    def debug_pcr(self, a, b, c, d, stream=None):
+        """Only the PCR stage: returns the k-step reduced system normalised to
+        unit diagonal, (A, C, D) = (a'/b', c'/b', d'/b'), in the plan's layout."""
+        import torch
+        self._check(a, b, c, d)
+        outs = [torch.empty_like(b) for _ in range(3)]
+        s = stream if stream is not None else torch.cuda.current_stream()
+        st = lib().tri_debug_pcr(self._h, a.data_ptr(), b.data_ptr(), c.data_ptr(), d.data_ptr(),
+                                 *[o.data_ptr() for o in outs], s.cuda_stream)
+        if st != 0:
+            raise TriError(st, "tri_debug_pcr")
+        return tuple(outs)
+
+
+def solve(a, b, c, d, n, m, layout=CONTIGUOUS, out=None, k=None):
+    """One-shot convenience: plan + solve on CUDA tensors."""
+    p = Plan(n, m, b.dtype, layout)
+    if k is not None:
+        p.k = k
+    return p.solve(a, b, c, d, out=out)

@@ -1,0 +1,467 @@
+// tri_api.cu -- the C ABI of include/tri.h: planner (transition point k and
+// variant, Sec. III.D, re-derived for B200 in DESIGN.md),
+// argument validation, scratch ownership and kernel dispatch.
+//
+// Build: nvcc -gencode arch=compute_100a,code=sm_100a -shared (see _build.py).
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdint>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+
+#include "tri.h"
+#include "common.cuh"
+#include "k_onchip.cuh"
+#include "k_tiled_pcr.cuh"
+#include "k_pthomas.cuh"
+
+using namespace tri;
+
+namespace {
+
+thread_local tri_status g_last = TRI_OK;
+
+constexpr int ONCHIP_THREADS = 512;
+constexpr int SPLIT_KMAX = 10;  // deepest k one sliding-window pass holds in smem (T = 256)
+constexpr int64_t MAX_ELEMS = int64_t(1) << 40;
+
+int floor_log2(int64_t v) {
+    int r = -1;
+    while (v > 0) { v >>= 1; ++r; }
+    return r;
+}
+int ceil_log2(int64_t v) {
+    int r = 0;
+    while ((int64_t(1) << r) < v) ++r;
+    return r;
+}
+int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
+size_t esize(tri_dtype t) { return t == TRI_F64 ? 8 : 4; }
+
+// ---- pure host planner ------------------------------------------------------
+// Rows of (normalised, 3-array) system data one ONCHIP CTA holds: sized for
+// 3 resident CTAs per SM (72 KiB each) so loads of one CTA overlap compute of
+// another.
+int64_t onchip_rows_budget(tri_dtype t) { return t == TRI_F64 ? 3072 : 6144; }
+
+int onchip_G(int64_t n, int64_t m, tri_dtype t, int sms) {
+    int64_t G = std::max<int64_t>(1, std::min<int64_t>(onchip_rows_budget(t) / n, m));
+    // keep >= 2 CTAs per SM when the batch allows it (wave balance, H6)
+    if (cdiv(m, G) < 2 * (int64_t)sms) G = std::max<int64_t>(1, cdiv(m, 2 * (int64_t)sms));
+    G = std::min<int64_t>(G, std::max<int64_t>(1, onchip_rows_budget(t) / n));
+    return (int)G;
+}
+
+tri_variant choose_variant(int64_t n, int64_t m, tri_dtype t, tri_layout, int) {
+    return n <= onchip_rows_budget(t) ? TRI_VARIANT_ONCHIP : TRI_VARIANT_SPLIT;
+}
+
+// Paper rule: M > P => k = 0; M <= P => the largest k with 2^k M <= P,
+// P the machine's effective parallelism.  B200: P_eff = SMs x chains per SM
+// needed to cover the Thomas recurrence latency.
+int choose_k_for(tri_variant v, int64_t n, int64_t m, tri_dtype t, tri_layout layout, int sms) {
+    const int kmax_n = floor_log2(n);
+    if (v == TRI_VARIANT_ONCHIP) {
+        const int G = onchip_G(n, m, t, sms);
+        int k = ceil_log2(cdiv(64, G));
+        return std::min(k, kmax_n);
+    }
+    const int64_t P = (int64_t)sms * 64;
+    int k = m >= P ? 0 : ceil_log2(cdiv(P, m));
+    return std::min(std::min(k, kmax_n), SPLIT_KMAX);
+}
+
+int kmax_for(tri_variant v, int64_t n) {
+    const int kn = floor_log2(n);
+    return v == TRI_VARIANT_SPLIT ? std::min(kn, SPLIT_KMAX) : kn;
+}
+
+}  // namespace
+
+struct tri_plan_s {
+    int64_t n, m;
+    tri_dtype dtype;
+    tri_layout layout;
+    int device, sms;
+    int k;
+    tri_variant variant;
+    int G, P, rpt;            // ONCHIP geometry
+    int64_t n_pad, L, C;      // SPLIT: chain length, chains
+    int64_t region, nreg;     // SPLIT: tiled-PCR regions per system
+    void* scratch;
+    size_t scratch_bytes;
+    void* stage;              // tri_solve_host staging (5 arrays), lazily allocated
+    size_t stage_bytes;
+};
+
+namespace {
+
+// ---- per-plan geometry -----------------------------------------------------
+void plan_geometry(tri_plan_s* p) {
+    const int64_t n = p->n, m = p->m;
+    if (p->variant == TRI_VARIANT_ONCHIP) {
+        p->G = onchip_G(n, m, p->dtype, p->sms);
+        // pad the per-system smem stride so the p-Thomas walk (lanes = chains,
+        // chain r of system g at g*P + r + j 2^k) hits distinct banks
+        const int S = 1 << p->k;
+        const int mod = p->dtype == TRI_F64 ? 16 : 32;
+        int P = (int)n;
+        if (S < 32) while ((P % mod) != (S % mod)) ++P;
+        p->P = P;
+        const int64_t rows = (int64_t)p->G * n;
+        int rpt = 1;
+        while ((int64_t)rpt * ONCHIP_THREADS < rows) rpt *= 2;
+        p->rpt = rpt;
+        p->n_pad = n; p->L = 0; p->C = 0; p->region = 0; p->nreg = 0;
+    } else {
+        const int S = 1 << p->k;
+        p->L = cdiv(n, S);
+        p->n_pad = p->L * S;
+        p->C = m * S;
+        if (p->k > 0) {
+            const int64_t target = 3 * (int64_t)p->sms;
+            int64_t nreg = std::max<int64_t>(1, cdiv(target, m));
+            // regions no shorter than 4 f(k) + T so halos stay a small fraction
+            const int64_t minreg = 4 * halo_f(p->k) + TPCR_T;
+            nreg = std::max<int64_t>(1, std::min<int64_t>(nreg, p->n_pad / minreg));
+            p->region = cdiv(p->n_pad, nreg);
+            p->nreg = cdiv(p->n_pad, p->region);
+        } else {
+            p->region = 0; p->nreg = 0;
+        }
+        p->G = 0; p->P = 0; p->rpt = 0;
+    }
+}
+
+size_t scratch_need(const tri_plan_s* p) {
+    if (p->variant != TRI_VARIANT_SPLIT) return 0;
+    const size_t s = esize(p->dtype);
+    const size_t chain_elems = (size_t)p->C * (size_t)p->L;
+    // k > 0: normalised reduced rows (3 arrays) + c', d' (2 arrays); k = 0: c', d'
+    return (p->k > 0 ? 5 : 2) * chain_elems * s;
+}
+
+tri_status ensure_scratch(tri_plan_s* p) {
+    const size_t need = scratch_need(p);
+    if (need <= p->scratch_bytes) return TRI_OK;
+    if (p->scratch) cudaFree(p->scratch);
+    p->scratch = nullptr;
+    p->scratch_bytes = 0;
+    if (cudaMalloc(&p->scratch, need) != cudaSuccess) {
+        cudaGetLastError();
+        return TRI_ERR_OOM;
+    }
+    p->scratch_bytes = need;
+    return TRI_OK;
+}
+
+int tiled_smem_layout(int k, int* off, int* mask) {
+    int total = 0;
+    for (int j = 0; j < k; ++j) {
+        int need = TPCR_T + 2 * (1 << j);
+        int rs = 1;
+        while (rs < need) rs *= 2;
+        off[j] = total;
+        mask[j] = rs - 1;
+        total += rs;
+    }
+    return total;
+}
+
+// ---- launches ---------------------------------------------------------------
+template <typename T, int RPT>
+cudaError_t launch_onchip_rpt(const tri_plan_s* p, OnchipArgs<T> a, cudaStream_t st) {
+    const size_t smem = (size_t)3 * p->G * p->P * sizeof(T);
+    cudaError_t e = cudaFuncSetAttribute(k_onchip<T, RPT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    const int64_t grid = cdiv(p->m, p->G);
+    k_onchip<T, RPT><<<(unsigned)grid, ONCHIP_THREADS, smem, st>>>(a);
+    return cudaGetLastError();
+}
+
+template <typename T>
+cudaError_t launch_onchip(const tri_plan_s* p, const void* a, const void* b, const void* c, const void* d,
+                          void* x, void* ao, void* co, void* do_, int mode, cudaStream_t st) {
+    OnchipArgs<T> A;
+    A.a = (const T*)a; A.b = (const T*)b; A.c = (const T*)c; A.d = (const T*)d;
+    A.x = (T*)x; A.ao = (T*)ao; A.co = (T*)co; A.do_ = (T*)do_;
+    A.n = p->n; A.m = p->m; A.layout = p->layout; A.k = p->k; A.G = p->G; A.P = p->P; A.mode = mode;
+    switch (p->rpt) {
+        case 1: return launch_onchip_rpt<T, 1>(p, A, st);
+        case 2: return launch_onchip_rpt<T, 2>(p, A, st);
+        case 4: return launch_onchip_rpt<T, 4>(p, A, st);
+        case 8: return launch_onchip_rpt<T, 8>(p, A, st);
+        case 16: return launch_onchip_rpt<T, 16>(p, A, st);
+        default: return cudaErrorInvalidValue;
+    }
+}
+
+template <typename T>
+cudaError_t launch_tiled(const tri_plan_s* p, const void* a, const void* b, const void* c, const void* d,
+                         void* oA, void* oC, void* oD, int mode, cudaStream_t st) {
+    TiledArgs<T> A;
+    A.a = (const T*)a; A.b = (const T*)b; A.c = (const T*)c; A.d = (const T*)d;
+    A.oA = (T*)oA; A.oC = (T*)oC; A.oD = (T*)oD;
+    A.n = p->n; A.m = p->m; A.n_pad = p->n_pad; A.region = p->region; A.nreg = p->nreg; A.C = p->C;
+    A.layout = p->layout; A.k = p->k; A.mode = mode;
+    A.ring_total = tiled_smem_layout(p->k, A.ring_off, A.ring_mask);
+    const size_t smem = (size_t)3 * A.ring_total * sizeof(T);
+    cudaError_t e = cudaFuncSetAttribute(k_tiled_pcr<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    const int64_t grid = p->m * p->nreg;
+    k_tiled_pcr<T><<<(unsigned)grid, TPCR_T, smem, st>>>(A);
+    return cudaGetLastError();
+}
+
+template <typename T>
+cudaError_t launch_split(const tri_plan_s* p, const void* a, const void* b, const void* c, const void* d,
+                         void* x, cudaStream_t st) {
+    const size_t ce = (size_t)p->C * (size_t)p->L;
+    T* base = (T*)p->scratch;
+    PThomasArgs<T> A;
+    A.a = (const T*)a; A.b = (const T*)b; A.c = (const T*)c; A.d = (const T*)d;
+    A.x = (T*)x;
+    A.n = p->n; A.m = p->m; A.C = p->C; A.L = p->L; A.layout = p->layout; A.k = p->k;
+    if (p->k > 0) {
+        T *rA = base, *rC = base + ce, *rD = base + 2 * ce;
+        cudaError_t e = launch_tiled<T>(p, a, b, c, d, rA, rC, rD, 0, st);
+        if (e != cudaSuccess) return e;
+        A.iA = rA; A.iC = rC; A.iD = rD;
+        A.cps = base + 3 * ce; A.dps = base + 4 * ce;
+        k_pthomas<T, 0><<<(unsigned)cdiv(p->C, 128), 128, 0, st>>>(A);
+    } else {
+        A.iA = A.iC = A.iD = nullptr;
+        A.cps = base; A.dps = base + ce;
+        if (p->layout == TRI_LAYOUT_INTERLEAVED)
+            k_pthomas<T, 1><<<(unsigned)cdiv(p->C, 128), 128, 0, st>>>(A);
+        else
+            k_pthomas_contig<T><<<(unsigned)cdiv(p->m, PT2_CH), PT2_CH, 0, st>>>(A);
+    }
+    return cudaGetLastError();
+}
+
+tri_status check_ptrs(const tri_plan_s* p, const void* const* in, int nin, const void* const* out, int nout) {
+    const size_t bytes = (size_t)p->n * (size_t)p->m * esize(p->dtype);
+    for (int i = 0; i < nin + nout; ++i) {
+        const void* q = i < nin ? in[i] : out[i - nin];
+        if (!q) return TRI_ERR_INVALID_ARG;
+        if (((uintptr_t)q & 15) != 0) return TRI_ERR_ALIGNMENT;
+        cudaPointerAttributes at;
+        if (cudaPointerGetAttributes(&at, q) != cudaSuccess) { cudaGetLastError(); return TRI_ERR_DEVICE; }
+        if ((at.type != cudaMemoryTypeDevice && at.type != cudaMemoryTypeManaged) || at.device != p->device)
+            return TRI_ERR_DEVICE;
+    }
+    for (int o = 0; o < nout; ++o) {
+        const uintptr_t x0 = (uintptr_t)out[o], x1 = x0 + bytes;
+        for (int i = 0; i < nin; ++i) {
+            const uintptr_t a0 = (uintptr_t)in[i], a1 = a0 + bytes;
+            if (x0 < a1 && a0 < x1) return TRI_ERR_ALIAS;
+        }
+        for (int o2 = 0; o2 < o; ++o2) {
+            const uintptr_t y0 = (uintptr_t)out[o2], y1 = y0 + bytes;
+            if (x0 < y1 && y0 < x1) return TRI_ERR_ALIAS;
+        }
+    }
+    return TRI_OK;
+}
+
+tri_status current_device_ok(int* dev, int* sms) {
+    int count = 0;
+    if (cudaGetDeviceCount(&count) != cudaSuccess || count == 0) { cudaGetLastError(); return TRI_ERR_DEVICE; }
+    if (cudaGetDevice(dev) != cudaSuccess) { cudaGetLastError(); return TRI_ERR_DEVICE; }
+    int major = 0, minor = 0;
+    cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, *dev);
+    cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, *dev);
+    cudaDeviceGetAttribute(sms, cudaDevAttrMultiProcessorCount, *dev);
+    if (major != 10 || minor != 0) return TRI_ERR_DEVICE;  // kernels are sm_100a only
+    return TRI_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+int64_t tri_halo_f(int k) { return k < 0 || k > 62 ? -1 : halo_f(k); }
+
+int64_t tri_halo_g(int k) {
+    if (k < 0 || k > 40) return -1;
+    int64_t s = 0;
+    for (int i = 0; i <= k; ++i) s += halo_f(i);
+    return (int64_t)k * halo_f(k) - s;
+}
+
+int tri_choose_variant(int64_t n, int64_t m, tri_dtype dtype, tri_layout layout, int sm_count) {
+    if (n < 1 || m < 1 || sm_count < 1) return -1;
+    return (int)choose_variant(n, m, dtype, layout, sm_count);
+}
+
+int tri_choose_k(int64_t n, int64_t m, tri_dtype dtype, tri_layout layout, int sm_count) {
+    if (n < 1 || m < 1 || sm_count < 1) return -1;
+    return choose_k_for(choose_variant(n, m, dtype, layout, sm_count), n, m, dtype, layout, sm_count);
+}
+
+void tri_shard_range(int64_t m, int G, int r, int64_t* q0, int64_t* mr) {
+    if (G < 1 || r < 0 || r >= G || m < 0) { if (q0) *q0 = 0; if (mr) *mr = 0; return; }
+    const int64_t per = cdiv(m, G);
+    const int64_t s = std::min<int64_t>((int64_t)r * per, m);
+    if (q0) *q0 = s;
+    if (mr) *mr = std::min<int64_t>(per, m - s);
+}
+
+const char* tri_status_str(tri_status s) {
+    switch (s) {
+        case TRI_OK: return "TRI_OK";
+        case TRI_ERR_INVALID_ARG: return "TRI_ERR_INVALID_ARG";
+        case TRI_ERR_ALIGNMENT: return "TRI_ERR_ALIGNMENT";
+        case TRI_ERR_ALIAS: return "TRI_ERR_ALIAS";
+        case TRI_ERR_DEVICE: return "TRI_ERR_DEVICE";
+        case TRI_ERR_OOM: return "TRI_ERR_OOM";
+        case TRI_ERR_CUDA: return "TRI_ERR_CUDA";
+    }
+    return "TRI_ERR_UNKNOWN";
+}
+
+tri_status tri_last_status(void) { return g_last; }
+
+tri_plan_t tri_plan(int64_t n, int64_t m, tri_dtype dtype, tri_layout layout) {
+    if (n < 1 || m < 1 || (dtype != TRI_F32 && dtype != TRI_F64) ||
+        (layout != TRI_LAYOUT_CONTIGUOUS && layout != TRI_LAYOUT_INTERLEAVED) || n > MAX_ELEMS / m) {
+        g_last = TRI_ERR_INVALID_ARG;
+        return nullptr;
+    }
+    int dev = 0, sms = 0;
+    tri_status st = current_device_ok(&dev, &sms);
+    if (st != TRI_OK) { g_last = st; return nullptr; }
+    tri_plan_s* p = new tri_plan_s();
+    p->n = n; p->m = m; p->dtype = dtype; p->layout = layout; p->device = dev; p->sms = sms;
+    p->variant = choose_variant(n, m, dtype, layout, sms);
+    p->k = choose_k_for(p->variant, n, m, dtype, layout, sms);
+    plan_geometry(p);
+    st = ensure_scratch(p);
+    if (st != TRI_OK) { delete p; g_last = st; return nullptr; }
+    g_last = TRI_OK;
+    return p;
+}
+
+void tri_destroy(tri_plan_t p) {
+    if (!p) return;
+    if (p->scratch) cudaFree(p->scratch);
+    if (p->stage) cudaFree(p->stage);
+    delete p;
+}
+
+int tri_plan_k(tri_plan_t p) { return p ? p->k : -1; }
+int tri_plan_variant(tri_plan_t p) { return p ? (int)p->variant : -1; }
+int64_t tri_plan_scratch_bytes(tri_plan_t p) { return p ? (int64_t)p->scratch_bytes : -1; }
+
+int tri_plan_launches(tri_plan_t p) {
+    if (!p) return -1;
+    if (p->variant == TRI_VARIANT_SPLIT) return p->k > 0 ? 2 : 1;
+    return 1;
+}
+
+tri_status tri_plan_set_k(tri_plan_t p, int k) {
+    if (!p || k < 0 || k > kmax_for(p->variant, p->n)) return TRI_ERR_INVALID_ARG;
+    const int old = p->k;
+    p->k = k;
+    plan_geometry(p);
+    tri_status st = ensure_scratch(p);
+    if (st != TRI_OK) { p->k = old; plan_geometry(p); }
+    return st;
+}
+
+tri_status tri_plan_set_variant(tri_plan_t p, tri_variant v) {
+    if (!p) return TRI_ERR_INVALID_ARG;
+    if (v == TRI_VARIANT_AUTO) v = choose_variant(p->n, p->m, p->dtype, p->layout, p->sms);
+    if (v == TRI_VARIANT_ONCHIP && p->n > onchip_rows_budget(p->dtype)) return TRI_ERR_INVALID_ARG;
+    if (v != TRI_VARIANT_ONCHIP && v != TRI_VARIANT_SPLIT) return TRI_ERR_INVALID_ARG;
+    const tri_variant ov = p->variant;
+    const int ok = p->k;
+    p->variant = v;
+    p->k = choose_k_for(v, p->n, p->m, p->dtype, p->layout, p->sms);
+    plan_geometry(p);
+    tri_status st = ensure_scratch(p);
+    if (st != TRI_OK) { p->variant = ov; p->k = ok; plan_geometry(p); }
+    return st;
+}
+
+void tri_plan_describe(tri_plan_t p, char* buf, int len) {
+    if (!buf || len <= 0) return;
+    if (!p) { snprintf(buf, len, "null plan"); return; }
+    static const char* vn[] = {"auto", "onchip", "split", "fused"};
+    snprintf(buf, len,
+             "n=%lld m=%lld dtype=%s layout=%s variant=%s k=%d G=%d P=%d rpt=%d L=%lld C=%lld region=%lld nreg=%lld "
+             "scratch=%zu sms=%d",
+             (long long)p->n, (long long)p->m, p->dtype == TRI_F64 ? "f64" : "f32",
+             p->layout == TRI_LAYOUT_CONTIGUOUS ? "contiguous" : "interleaved", vn[p->variant], p->k, p->G, p->P,
+             p->rpt, (long long)p->L, (long long)p->C, (long long)p->region, (long long)p->nreg, p->scratch_bytes,
+             p->sms);
+}
+
+tri_status tri_solve(tri_plan_t p, const void* a, const void* b, const void* c, const void* d, void* x,
+                     void* stream) {
+    if (!p) return TRI_ERR_INVALID_ARG;
+    const void* in[4] = {a, b, c, d};
+    const void* out[1] = {x};
+    tri_status st = check_ptrs(p, in, 4, out, 1);
+    if (st != TRI_OK) return st;
+    cudaStream_t s = (cudaStream_t)stream;
+    cudaError_t e;
+    if (p->variant == TRI_VARIANT_ONCHIP) {
+        e = p->dtype == TRI_F64 ? launch_onchip<double>(p, a, b, c, d, x, nullptr, nullptr, nullptr, 0, s)
+                                : launch_onchip<float>(p, a, b, c, d, x, nullptr, nullptr, nullptr, 0, s);
+    } else {
+        e = p->dtype == TRI_F64 ? launch_split<double>(p, a, b, c, d, x, s) : launch_split<float>(p, a, b, c, d, x, s);
+    }
+    return e == cudaSuccess ? TRI_OK : TRI_ERR_CUDA;
+}
+
+tri_status tri_debug_pcr(tri_plan_t p, const void* a, const void* b, const void* c, const void* d, void* ao,
+                         void* co, void* do_, void* stream) {
+    if (!p) return TRI_ERR_INVALID_ARG;
+    const void* in[4] = {a, b, c, d};
+    const void* out[3] = {ao, co, do_};
+    tri_status st = check_ptrs(p, in, 4, out, 3);
+    if (st != TRI_OK) return st;
+    cudaStream_t s = (cudaStream_t)stream;
+    cudaError_t e;
+    if (p->variant == TRI_VARIANT_ONCHIP) {
+        e = p->dtype == TRI_F64 ? launch_onchip<double>(p, a, b, c, d, nullptr, ao, co, do_, 1, s)
+                                : launch_onchip<float>(p, a, b, c, d, nullptr, ao, co, do_, 1, s);
+    } else {
+        if (p->k == 0) return TRI_ERR_INVALID_ARG;  // no PCR stage to show
+        e = p->dtype == TRI_F64 ? launch_tiled<double>(p, a, b, c, d, ao, co, do_, 1, s)
+                                : launch_tiled<float>(p, a, b, c, d, ao, co, do_, 1, s);
+    }
+    return e == cudaSuccess ? TRI_OK : TRI_ERR_CUDA;
+}
+
+tri_status tri_solve_host(tri_plan_t p, const void* a, const void* b, const void* c, const void* d, void* x,
+                          void* stream) {
+    if (!p || !a || !b || !c || !d || !x) return TRI_ERR_INVALID_ARG;
+    const size_t bytes = (size_t)p->n * (size_t)p->m * esize(p->dtype);
+    const size_t need = 5 * ((bytes + 255) / 256 * 256);
+    if (p->stage_bytes < need) {
+        if (p->stage) cudaFree(p->stage);
+        p->stage = nullptr;
+        p->stage_bytes = 0;
+        if (cudaMalloc(&p->stage, need) != cudaSuccess) { cudaGetLastError(); return TRI_ERR_OOM; }
+        p->stage_bytes = need;
+    }
+    const size_t slot = need / 5;
+    char* base = (char*)p->stage;
+    void* dv[5] = {base, base + slot, base + 2 * slot, base + 3 * slot, base + 4 * slot};
+    const void* hv[4] = {a, b, c, d};
+    cudaStream_t s = (cudaStream_t)stream;
+    for (int i = 0; i < 4; ++i)
+        if (cudaMemcpyAsync(dv[i], hv[i], bytes, cudaMemcpyHostToDevice, s) != cudaSuccess) return TRI_ERR_CUDA;
+    tri_status st = tri_solve(p, dv[0], dv[1], dv[2], dv[3], dv[4], stream);
+    if (st != TRI_OK) return st;
+    if (cudaMemcpyAsync(x, dv[4], bytes, cudaMemcpyDeviceToHost, s) != cudaSuccess) return TRI_ERR_CUDA;
+    if (cudaStreamSynchronize(s) != cudaSuccess) return TRI_ERR_CUDA;
+    return TRI_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,109 @@
+"""CPU tests of the C-ABI library: it loads without a GPU, exports every symbol
+include/tri.h declares, and its pure host logic (halo formulas Eqs 8-9, the
+transition heuristic, shard ranges, status strings) is right.  No compute calls."""
+import ctypes
+import os
+import re
+
+import pytest
+
+import paper_conf_icpp_kimwch11_b200 as tri
+from paper_conf_icpp_kimwch11_b200 import _build
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def L():
+    _build.build()
+    return tri.lib()
+
+
+def declared_symbols():
+    hdr = open(os.path.join(ROOT, "include", "tri.h")).read()
+    return sorted(set(re.findall(r"^TRI_API\s+[\w\s\*]+?\b(tri_\w+)\(", hdr, re.M)))
+
+
+def test_header_declares_the_north_star_calls():
+    syms = declared_symbols()
+    for s in ("tri_plan", "tri_solve", "tri_destroy", "tri_plan_k", "tri_plan_set_k", "tri_status_str",
+              "tri_last_status", "tri_solve_host"):
+        assert s in syms
+
+
+def test_library_exports_every_declared_symbol(L):
+    for s in declared_symbols():
+        assert hasattr(L, s), s
+    # nothing else leaks (visibility=hidden): nm -D lists exactly the tri_ ABI
+    import subprocess
+    out = subprocess.run(["nm", "-D", "--defined-only", tri.LIB_PATH], capture_output=True, text=True).stdout
+    exported = sorted(set(re.findall(r"\bT (tri_\w+)", out)))
+    assert exported == declared_symbols()
+
+
+def test_halo_formulas_match_paper_definitions(L):
+    rows = [list(map(int, ln.split())) for ln in open(os.path.join(ROOT, "tests/golden/halo_eq8_eq9.txt"))
+            if ln.strip() and not ln.startswith("#")]
+    for k, f, g, cache in rows:
+        assert tri.halo_f(k) == f          # Eq 8
+        assert tri.halo_g(k) == g          # Eq 9
+        assert 3 * tri.halo_f(k) == cache <= 3 * 2 ** k   # Table I
+    # closed forms noted in SURVEY A7
+    for k in range(0, 21):
+        assert tri.halo_g(k) == (k - 2) * 2 ** k + 2
+
+
+def test_status_strings(L):
+    for code, name in tri.STATUS.items():
+        assert L.tri_status_str(code).decode() == name
+
+
+def test_plan_without_gpu_fails_cleanly(L):
+    import torch
+    if torch.cuda.is_available():
+        pytest.skip("GPU present")
+    assert not L.tri_plan(1024, 4, tri.F64, tri.CONTIGUOUS)
+    assert L.tri_last_status() == 4  # TRI_ERR_DEVICE
+    assert not L.tri_plan(0, 4, tri.F64, tri.CONTIGUOUS)
+    assert L.tri_last_status() == 1  # TRI_ERR_INVALID_ARG
+    assert not L.tri_plan(16, 4, 7, tri.CONTIGUOUS)
+    assert L.tri_last_status() == 1
+    assert not L.tri_plan(16, 4, tri.F64, 9)
+    assert L.tri_last_status() == 1
+    assert L.tri_plan_k(None) == -1
+    L.tri_destroy(None)  # NULL-safe
+    with pytest.raises(tri.TriError):
+        tri.Plan(16, 4)
+
+
+@pytest.mark.parametrize("dtype", [tri.F64, tri.F32])
+@pytest.mark.parametrize("layout", [tri.CONTIGUOUS, tri.INTERLEAVED])
+@pytest.mark.parametrize("n", [1, 2, 7, 256, 1024, 5000, 16384, 1 << 24])
+def test_heuristic_k_valid_and_nonincreasing_in_m(L, dtype, layout, n):
+    """Table III shape: k never grows as M grows; k <= floor(log2 n)."""
+    prev = None
+    for m in [1, 2, 16, 32, 100, 512, 1024, 4096, 16384, 1 << 20]:
+        k = tri.choose_k(n, m, dtype, layout, 148)
+        v = tri.choose_variant(n, m, dtype, layout, 148)
+        assert v in (tri.VARIANT_ONCHIP, tri.VARIANT_SPLIT)
+        assert 0 <= k <= max(0, n.bit_length() - 1)
+        if prev is not None and v == prev[1]:
+            assert k <= prev[0], (n, m, k, prev)
+        prev = (k, v)
+
+
+def test_heuristic_paper_rule_extremes(L):
+    """with M > P (plenty of systems) go straight to p-Thomas (k = 0);
+    a single huge system gets deep PCR."""
+    assert tri.choose_k(16384, 16384, tri.F64, tri.CONTIGUOUS, 148) == 0
+    assert tri.choose_k(1 << 24, 1, tri.F64, tri.CONTIGUOUS, 148) >= 8
+
+
+@pytest.mark.parametrize("m,G", [(16384, 1), (16384, 8), (10, 4), (3, 8), (1, 2), (1000, 7)])
+def test_shard_range_partitions(L, m, G):
+    covered = []
+    for r in range(G):
+        q0, mr = tri.shard_range(m, G, r)
+        assert mr >= 0
+        covered += list(range(q0, q0 + mr))
+    assert covered == list(range(m))

@@ -324,3 +324,14 @@ def test_pcr_step_exact_rational():
                         (c2[i], new[i + 2 * s] if i + 2 * s < n else F(0)),
                         (d2[i], new[n])):
             assert abs(F(val) - ex) <= 4 * U * max(abs(ex), F(1))
+
+
+def test_residual_batch_matches_single():
+    n, m = 33, 9
+    a, b, c, d = trigen.generate(n, m, "f32", trigen.INTERLEAVED, "dd")
+    x = oracle.solve_batch(n, m, a, b, c, d, layout=1)
+    xp = x * (1 + 1e-7 * np.cos(np.arange(n * m)))
+    rb = oracle.residual_batch(n, m, a, b, c, d, xp, layout=1)
+    for q in (0, 4, 8):
+        sl = lambda t: t.reshape(n, m)[:, q].astype(np.float64)
+        assert tuple(rb[q]) == oracle.residual(sl(a), sl(b), sl(c), sl(d), sl(xp))

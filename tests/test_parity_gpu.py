@@ -1,0 +1,236 @@
+"""GPU parity: the CUDA path (through the C ABI) vs the CPU oracle, element by
+element on the same seeded inputs, with the north-star tolerances
+(fp64: max rel err <= 1e-10 and rel residual <= 1e-12; fp32: rel err <= 1e-4).
+Shapes span several tiles, ragged tails, every variant, both layouts and every
+forced transition point k."""
+import numpy as np
+import pytest
+
+import oracle
+from tests._helpers import check_parity, gen, gpu_solve, to_dev
+
+pytestmark = pytest.mark.gpu
+
+tri = pytest.importorskip("paper_conf_icpp_kimwch11_b200")
+ONCHIP, SPLIT = tri.VARIANT_ONCHIP, tri.VARIANT_SPLIT
+
+
+# ------------------------------------------------------------------ auto plan
+@pytest.mark.parametrize("dtype", ["f64", "f32"])
+@pytest.mark.parametrize("layout", [0, 1])
+@pytest.mark.parametrize("n,m", [(1, 1), (1, 9), (2, 3), (5, 1), (17, 33), (64, 129), (255, 3), (1000, 37),
+                                 (1024, 1), (1024, 300), (3000, 3), (5003, 2), (8191, 5), (20000, 3),
+                                 (65536 + 37, 1)])
+def test_auto_plan_parity(cuda_ok, dtype, layout, n, m):
+    arrs = gen(n, m, dtype, layout)
+    x, plan = gpu_solve(n, m, arrs, dtype, layout)
+    check_parity(n, m, arrs, x, dtype, layout)
+
+
+@pytest.mark.parametrize("family,eps", [("weak", 1e-2), ("weak", 1e-3), ("integer", 0.0)])
+@pytest.mark.parametrize("n,m", [(1024, 64), (333, 17), (40000, 2)])
+def test_families_fp64(cuda_ok, family, eps, n, m):
+    arrs = gen(n, m, "f64", 0, family, eps=eps)
+    x, _ = gpu_solve(n, m, arrs, "f64", 0)
+    check_parity(n, m, arrs, x, "f64", 0)
+
+
+@pytest.mark.parametrize("family", ["dd", "weak"])
+def test_families_fp32(cuda_ok, family):
+    n, m = 256, 4096
+    arrs = gen(n, m, "f32", 0, family, eps=1e-2)
+    x, _ = gpu_solve(n, m, arrs, "f32", 0)
+    check_parity(n, m, arrs, x, "f32", 0)
+
+
+# ------------------------------------------------------------------ forced k
+@pytest.mark.parametrize("dtype", ["f64", "f32"])
+@pytest.mark.parametrize("layout", [0, 1])
+@pytest.mark.parametrize("n,m", [(1024, 5), (777, 3), (2048, 1)])
+def test_onchip_every_k(cuda_ok, dtype, layout, n, m):
+    """k-independence: every forced k in [0, floor(log2 n)]."""
+    arrs = gen(n, m, dtype, layout, "weak", eps=1e-2)
+    xo = oracle.solve_batch(n, m, *arrs, layout=layout)
+    plan = None
+    for k in range(0, int(np.log2(n)) + 1):
+        x, plan = gpu_solve(n, m, arrs, dtype, layout, k=k, variant=ONCHIP, plan=plan)
+        check_parity(n, m, arrs, x, dtype, layout, x_oracle=xo)
+
+
+@pytest.mark.parametrize("dtype", ["f64", "f32"])
+@pytest.mark.parametrize("layout", [0, 1])
+@pytest.mark.parametrize("n,m", [(10007, 3), (4099, 1), (70001, 1)])
+def test_split_every_k(cuda_ok, dtype, layout, n, m):
+    arrs = gen(n, m, dtype, layout, "weak", eps=1e-2)
+    xo = oracle.solve_batch(n, m, *arrs, layout=layout)
+    plan = None
+    for k in range(0, min(int(np.log2(n)), 10) + 1):
+        x, plan = gpu_solve(n, m, arrs, dtype, layout, k=k, variant=SPLIT, plan=plan)
+        check_parity(n, m, arrs, x, dtype, layout, x_oracle=xo)
+
+
+def test_split_on_small_systems(cuda_ok):
+    """The streaming variant must also handle systems shorter than a tile."""
+    for n, m in [(1, 4), (3, 7), (100, 9), (600, 2)]:
+        arrs = gen(n, m, "f64", 0)
+        for k in range(0, int(np.log2(n)) + 1):
+            x, _ = gpu_solve(n, m, arrs, "f64", 0, k=k, variant=SPLIT)
+            check_parity(n, m, arrs, x, "f64", 0)
+
+
+# ------------------------------------------------------------------ PCR stage (row A2)
+@pytest.mark.parametrize("variant,n,m,k", [(ONCHIP, 1024, 3, 3), (ONCHIP, 500, 2, 5), (SPLIT, 9000, 2, 4),
+                                           (SPLIT, 20001, 1, 8), (SPLIT, 5000, 3, 1)])
+def test_pcr_stage_matches_oracle(cuda_ok, variant, n, m, k):
+    """The reduced system after k PCR steps (Eqs 5-6) vs the oracle's plain PCR,
+    normalised to unit diagonal, and satisfied by the oracle solution."""
+    arrs = gen(n, m, "f64", 0, "weak", eps=1e-2)
+    plan = tri.Plan(n, m, tri.F64, 0)
+    plan.variant = variant
+    plan.k = k
+    A, C, D = (t.cpu().numpy() for t in plan.debug_pcr(*to_dev(*arrs)))
+    xo = oracle.solve_batch(n, m, *arrs)
+    s = 1 << k
+    for q in range(m):
+        sl = slice(q * n, (q + 1) * n)
+        ao, bo, co, do = oracle.pcr_k(*(t[sl] for t in arrs), k)
+        An, Cn, Dn = ao / bo, co / bo, do / bo
+        for got, ref in ((A[sl], An), (C[sl], Cn), (D[sl], Dn)):
+            assert np.max(np.abs(got - ref)) <= 1e-12 * max(1.0, np.max(np.abs(ref)))
+        # invariant: A_i x_{i-s} + x_i + C_i x_{i+s} - D_i = 0
+        x = xo[sl]
+        xm = np.concatenate([np.zeros(s), x[:-s]]) if s < n else np.zeros(n)
+        xp = np.concatenate([x[s:], np.zeros(s)]) if s < n else np.zeros(n)
+        r = A[sl] * xm + x + C[sl] * xp - D[sl]
+        assert np.max(np.abs(r)) <= 1e-13 * np.max(np.abs(D[sl]))
+
+
+# ------------------------------------------------------------------ edge cases / API
+@pytest.mark.parametrize("variant,n,m", [(ONCHIP, 1024, 4), (SPLIT, 9000, 2), (SPLIT, 3000, 130)])
+@pytest.mark.parametrize("layout", [0, 1])
+def test_ignored_entries_nan(cuda_ok, variant, n, m, layout):
+    """a[q][0] and c[q][n-1] lie outside A (Eq 1, reading X1): NaN there must
+    not change x (bitwise)."""
+    import torch
+    arrs = gen(n, m, "f64", layout)
+    plan = tri.Plan(n, m, tri.F64, layout)
+    plan.variant = variant
+    a, b, c, d = to_dev(*arrs)
+    x1 = plan.solve(a, b, c, d).clone()
+    a2, c2 = a.clone(), c.clone()
+    if layout == 0:
+        a2.view(m, n)[:, 0] = float("nan")
+        c2.view(m, n)[:, -1] = float("nan")
+    else:
+        a2.view(n, m)[0, :] = float("nan")
+        c2.view(n, m)[-1, :] = float("nan")
+    x2 = plan.solve(a2, b, c2, d)
+    assert torch.equal(x1, x2)
+
+
+def test_determinism_and_plan_reuse(cuda_ok):
+    import torch
+    for n, m in [(1024, 300), (16384, 64), (100000, 1)]:
+        arrs = gen(n, m, "f64", 0)
+        plan = tri.Plan(n, m, tri.F64, 0)
+        a, b, c, d = to_dev(*arrs)
+        x1 = plan.solve(a, b, c, d).clone()
+        for _ in range(3):
+            assert torch.equal(plan.solve(a, b, c, d), x1)
+
+
+def test_batch_invariance(cuda_ok):
+    """Identical systems give identical x (bitwise) wherever they sit."""
+    import torch
+    n, m = 700, 40
+    a, b, c, d = gen(n, 1, "f64", 0)
+    rep = [np.tile(t, m) for t in (a, b, c, d)]
+    for variant in (ONCHIP, SPLIT):
+        x, _ = gpu_solve(n, m, rep, "f64", 0, variant=variant)
+        xs = x.reshape(m, n)
+        assert np.all(xs == xs[0])
+
+
+def test_power_of_two_row_scaling_bitwise(cuda_ok):
+    """Scaling row i by 2^p_i leaves x unchanged bitwise; scaling d by 2^p scales
+    x by 2^p bitwise (every rounding step is scale-covariant)."""
+    n, m = 3000, 8
+    a, b, c, d = gen(n, m, "f64", 0, "weak", eps=1e-2)
+    rng = np.random.default_rng(0)
+    p = 2.0 ** rng.integers(-20, 20, n * m)
+    for variant, k in ((ONCHIP, 3), (SPLIT, 0), (SPLIT, 4)):
+        x0, _ = gpu_solve(n, m, (a, b, c, d), "f64", 0, variant=variant, k=k)
+        x1, _ = gpu_solve(n, m, (a * p, b * p, c * p, d * p), "f64", 0, variant=variant, k=k)
+        assert np.array_equal(x0, x1)
+        x2, _ = gpu_solve(n, m, (a, b, c, d * 1024.0), "f64", 0, variant=variant, k=k)
+        assert np.array_equal(x2, x0 * 1024.0)
+
+
+def test_flip(cuda_ok):
+    """Reversing the rows and swapping a and c reverses x (within tolerance)."""
+    n, m = 5000, 4
+    a, b, c, d = gen(n, m, "f64", 0)
+    rev = lambda t: t.reshape(m, n)[:, ::-1].copy().ravel()
+    x0, _ = gpu_solve(n, m, (a, b, c, d), "f64", 0)
+    x1, _ = gpu_solve(n, m, (rev(c), rev(b), rev(a), rev(d)), "f64", 0)
+    assert np.max(np.abs(rev(x1) - x0) / np.abs(x0)) <= 1e-12
+
+
+def test_api_errors(cuda_ok):
+    import torch
+    n, m = 1024, 4
+    plan = tri.Plan(n, m, tri.F64, 0)
+    a, b, c, d = to_dev(*gen(n, m, "f64", 0))
+    x = torch.empty_like(b)
+    L = tri.lib()
+    h = plan._h
+    assert L.tri_solve(h, a.data_ptr(), b.data_ptr(), c.data_ptr(), d.data_ptr(), x.data_ptr(), None) == 0
+    assert L.tri_solve(h, None, b.data_ptr(), c.data_ptr(), d.data_ptr(), x.data_ptr(), None) == 1
+    assert L.tri_solve(h, a.data_ptr() + 8, b.data_ptr(), c.data_ptr(), d.data_ptr(), x.data_ptr(), None) == 2
+    assert L.tri_solve(h, a.data_ptr(), b.data_ptr(), c.data_ptr(), d.data_ptr(), d.data_ptr(), None) == 3
+    big = torch.empty(2 * n * m, dtype=torch.float64, device="cuda")
+    assert L.tri_solve(h, big.data_ptr(), b.data_ptr(), c.data_ptr(), d.data_ptr(),
+                       big.data_ptr() + 8 * (n * m // 2), None) == 3  # partial overlap
+    host = np.zeros(n * m)
+    assert L.tri_solve(h, a.data_ptr(), b.data_ptr(), c.data_ptr(), d.data_ptr(), host.ctypes.data, None) == 4
+    assert L.tri_plan_set_k(h, 11) == 1          # k > floor(log2 1024)
+    assert L.tri_plan_set_k(h, -1) == 1
+    assert L.tri_plan_set_variant(h, 9) == 1
+    p1 = tri.Plan(1, 5, tri.F64, 0)
+    with pytest.raises(tri.TriError):
+        p1.k = 1                                  # n = 1: only k = 0
+    with pytest.raises(tri.TriError):
+        tri.Plan(0, 5)
+    ps = tri.Plan(100000, 1, tri.F64, 0)
+    with pytest.raises(tri.TriError):
+        ps.variant = ONCHIP                       # does not fit one CTA
+
+
+def test_concurrent_plans_two_streams(cuda_ok):
+    import torch
+    n, m = 20000, 8
+    arrs = gen(n, m, "f64", 0)
+    xo = oracle.solve_batch(n, m, *arrs)
+    a, b, c, d = to_dev(*arrs)
+    s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+    p1, p2 = tri.Plan(n, m, tri.F64, 0), tri.Plan(n, m, tri.F64, 0)
+    p2.k = 3
+    torch.cuda.synchronize()
+    x1, x2 = torch.empty_like(b), torch.empty_like(b)
+    for _ in range(3):
+        p1.solve(a, b, c, d, out=x1, stream=s1)
+        p2.solve(a, b, c, d, out=x2, stream=s2)
+    torch.cuda.synchronize()
+    for x in (x1, x2):
+        assert np.max(np.abs(x.cpu().numpy() - xo) / np.abs(xo)) <= 1e-10
+
+
+def test_solve_host(cuda_ok):
+    import torch
+    n, m = 4096, 16
+    arrs = gen(n, m, "f64", 0)
+    plan = tri.Plan(n, m, tri.F64, 0)
+    pin = [torch.from_numpy(t).pin_memory() for t in arrs]
+    out = torch.empty(n * m, dtype=torch.float64).pin_memory()
+    plan.solve_host(*pin, out)
+    check_parity(n, m, arrs, out.numpy(), "f64", 0)
