@@ -1,0 +1,339 @@
+#!/usr/bin/env python
+"""Benchmark of the hybrid tridiagonal solve (tiled PCR + p-Thomas) on B200.
+
+Contract (driver): `python bench.py --gpus N --steps K --warmup W` prints ONE
+JSON line on rank 0.  A "step" is one pass of the whole hot path (one tri_solve
+of the full batch).  Default workload = BASELINE config 5 (fp64, m = 16384
+systems of n = 16384, contiguous), the config the metric's 1/2/4/8-GPU figures
+are quoted on; other configs via --config.  Inputs are synthetic (trigen,
+seeded), generated on the host and resident in HBM before the timed region.
+
+N > 1 (torchrun, one rank per GPU, NCCL): the m systems are sharded into
+contiguous ranges (no collective inside the solve); time = max over ranks.
+
+--impl reference times the CPU oracle (plain sequential Thomas, oracle/) on a
+bounded sample of the same workload -- the tier's reference arm.
+"""
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+CONFIGS = {
+    # name: (n, m, dtype, layout, description)  -- BASELINE.json configs[0..4]
+    "c1": (1024, 1, "f64", 0, "single fp64 diagonally dominant system n=1024"),
+    "c2": (1024, 1024, "f64", 1, "batched fp64 m=1024 systems of n=1024, interleaved"),
+    "c3": (1 << 24, 1, "f64", 0, "single large fp64 system n=2^24"),
+    "c4": (256, 1 << 20, "f32", 0, "many small fp32 systems m=2^20, n=256, contiguous"),
+    "c5": (16384, 16384, "f64", 0, "batched fp64 m=16384 systems of n=16384, contiguous"),
+}
+METRIC = "Munknowns/s fp64/fp32 and % of HBM roofline at 1/2/4/8 B200"
+FALLBACK_HBM_GBS = 6650.0  # /opt/skills/guides/B200_PROFILING.md fallback
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="c5", choices=sorted(CONFIGS))
+    ap.add_argument("--layout", type=int, default=None, help="override layout (0 contiguous, 1 interleaved)")
+    ap.add_argument("--family", default="dd")
+    ap.add_argument("--k", type=int, default=None, help="force the transition point k")
+    ap.add_argument("--variant", type=int, default=None, help="force variant (1 onchip, 2 split, 3 fused)")
+    ap.add_argument("--scaling", default="strong", choices=["strong", "weak"],
+                    help="strong: the config's m is split over ranks; weak: every rank solves the full m")
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-check", action="store_true")
+    return ap.parse_args()
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as fh:
+            j = json.load(fh)
+        return float(j["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy test)"
+    return FALLBACK_HBM_GBS, "fallback (B200_PROFILING.md)"
+
+
+class ClockSampler:
+    """Polls NVML (SM clock, throttle reasons) every 10 ms during the timed region."""
+
+    REASONS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap",
+               0x8: "hw_slowdown", 0x10: "sync_boost", 0x20: "sw_thermal_slowdown",
+               0x40: "hw_thermal_slowdown", 0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting"}
+
+    def __init__(self, index):
+        self.samples, self.reasons, self.ok = [], set(), False
+        self._stop = threading.Event()
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.ok = True
+        except Exception:
+            self.max_mhz = None
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                r = self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                for bit, name in self.REASONS.items():
+                    if r & bit and name != "gpu_idle":
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            time.sleep(0.01)
+
+    def __enter__(self):
+        if self.ok:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *exc):
+        if self.ok:
+            self._stop.set()
+            self.t.join()
+
+    def summary(self):
+        if not self.ok or not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons), "samples": 0}
+        return {"sm_mhz": float(statistics.median(self.samples)), "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+def dist_env():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return world, rank, local
+
+
+def cpu_oracle_time(n, mr, arrs, layout, budget_s=20.0):
+    """Time the oracle (as it stands) on the host cores over a bounded sample."""
+    import oracle
+    cores = len(os.sched_getaffinity(0))
+    # sample: whole systems, as many as fit ~budget_s at ~50 Munk/s/core
+    est_rate = 50e6 * cores
+    qs = int(max(1, min(mr, budget_s * est_rate / n)))
+    if layout == 1 and qs < mr:
+        qs = mr  # interleaved sample would read strided rows; use the full (small) batch
+    t0 = time.perf_counter()
+    oracle.solve_batch(n, mr, *arrs, layout=layout, q_begin=0, q_end=qs, nthreads=cores)
+    dt = time.perf_counter() - t0
+    return {"value": n * qs / dt / 1e6, "unit": "Munknowns/s", "cores": cores, "kind": "oracle",
+            "sample": f"{qs} of {mr} systems x n={n} (whole systems, {dt:.2f} s, {cores} threads over systems)"}
+
+
+def run_reference(args):
+    """--impl reference: the CPU oracle on the box's host cores."""
+    world, rank, _ = dist_env()
+    n, m, dt, layout, desc = CONFIGS[args.config]
+    if args.layout is not None:
+        layout = args.layout
+    if rank != 0:
+        return  # rank 0 alone runs and prints it
+    import oracle
+    import trigen
+    cores = len(os.sched_getaffinity(0))
+    # bounded sample per step: ~10 s of CPU work across all steps
+    total_budget = 60.0
+    per_step = total_budget / max(1, args.steps + args.warmup)
+    qs = int(max(1, min(m, per_step * 50e6 * cores / n)))
+    if layout == 1:
+        qs = m
+    arrs = trigen.generate(n, qs, dt, layout, args.family, seed=trigen.SEED_BASE + int(args.config[1]))
+    for _ in range(args.warmup):
+        oracle.solve_batch(n, qs, *arrs, layout=layout, nthreads=cores)
+    times = []
+    for _ in range(args.steps):
+        t0 = time.perf_counter()
+        oracle.solve_batch(n, qs, *arrs, layout=layout, nthreads=cores)
+        times.append(time.perf_counter() - t0)
+    t = sum(times) / len(times)
+    v = n * qs / t / 1e6
+    out = {"metric": METRIC, "value": v, "unit": "Munknowns/s", "impl": "reference", "n_gpus": args.gpus,
+           "steps": args.steps, "warmup": args.warmup, "ms_per_step": t * 1e3, "higher_is_better": True,
+           "scaling": args.scaling, "vs_baseline": None, "dtype": dt, "data": "synthetic",
+           "config": {"workload": args.config, "desc": desc, "n": n, "m": m, "layout": layout,
+                      "family": args.family},
+           "cpu_baseline": {"value": v, "unit": "Munknowns/s", "cores": cores, "kind": "oracle",
+                            "sample": f"{qs} of {m} systems x n={n} per step (whole systems)"},
+           "e2e": {"value": v, "unit": "Munknowns/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(out), flush=True)
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        run_reference(args)
+        return
+    import torch
+    import torch.distributed as dist
+
+    import trigen
+    import paper_conf_icpp_kimwch11_b200 as tri
+
+    world, rank, local = dist_env()
+    if world > 1:
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    else:
+        torch.cuda.set_device(0)
+    dev = torch.device("cuda", torch.cuda.current_device())
+
+    n, m, dt, layout, desc = CONFIGS[args.config]
+    if args.layout is not None:
+        layout = args.layout
+    s = 8 if dt == "f64" else 4
+    tdt = torch.float64 if dt == "f64" else torch.float32
+    if args.scaling == "strong":
+        q0, mr = tri.shard_range(m, world, rank)
+    else:
+        q0, mr = rank * m, m
+    m_all = m if args.scaling == "strong" else m * world
+    seed = trigen.SEED_BASE + int(args.config[1])
+
+    # ---- inputs: seeded host generation of this rank's shard, then resident in HBM
+    pin = not args.no_e2e
+    host = [torch.empty(n * mr, dtype=tdt, pin_memory=pin) for _ in range(4)]
+    trigen.generate(n, mr, dt, layout, args.family, seed=seed, q0=q0, out=[t.numpy() for t in host])
+    a, b, c, d = (t.to(dev, non_blocking=False) for t in host)
+    x = torch.empty_like(b)
+    plan = tri.Plan(n, mr, tri.F64 if dt == "f64" else tri.F32, layout)
+    if args.variant is not None:
+        plan.variant = args.variant
+    if args.k is not None:
+        plan.k = args.k
+    stream = torch.cuda.current_stream()
+    n_unknowns = n * mr
+
+    # L2 policy: flush between timed steps when this rank's working set could sit in L2
+    l2 = torch.cuda.get_device_properties(dev).L2_cache_size
+    ws = 5 * n_unknowns * s + plan.scratch_bytes
+    flush = ws < 4 * l2
+    flush_buf = torch.empty(2 * l2 // 4 + 1024, dtype=torch.int32, device=dev) if flush else None
+
+    for _ in range(args.warmup):
+        plan.solve(a, b, c, d, out=x, stream=stream)
+    torch.cuda.synchronize()
+
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(dev.index) as clk:
+        for i in range(args.steps):
+            if flush:
+                flush_buf.add_(1)  # writes 2x L2 worth of bytes outside the timed interval
+            ev[i][0].record(stream)
+            plan.solve(a, b, c, d, out=x, stream=stream)
+            ev[i][1].record(stream)
+        torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    step_ms = [e0.elapsed_time(e1) for e0, e1 in ev]
+    t_step = sum(step_ms) / len(step_ms)
+    t_max = torch.tensor([t_step], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t_max, op=dist.ReduceOp.MAX)
+    t_step_max = float(t_max.item())
+    value = m_all * n / (t_step_max * 1e-3) / 1e6  # whole-job Munknowns/s
+
+    # ---- sampled parity vs the oracle (rank 0's shard, a few whole systems)
+    parity = None
+    if not args.no_check and rank == 0:
+        import oracle
+        xs = x.cpu().numpy()
+        qs = sorted(set([0, mr // 3, mr // 2, mr - 1]))
+        errs = []
+        for qq in qs:
+            sa = trigen.generate(n, 1, dt, 0, args.family, seed=seed, q0=q0 + qq)
+            xo = oracle.solve_batch(n, 1, *sa)
+            xg = xs.reshape(mr, n)[qq] if layout == 0 else xs.reshape(n, mr)[:, qq]
+            errs.append(float(np.max(np.abs(xg.astype(np.float64) - xo) / np.abs(xo))))
+        parity = {"systems": len(qs), "max_rel_err": max(errs)}
+
+    # ---- end to end through the C ABI with HOST buffers (copies inside the timed region)
+    e2e = None
+    if not args.no_e2e:
+        xh = torch.empty(n * mr, dtype=tdt, pin_memory=True)
+        plan.solve_host(*host, xh, stream=stream)  # warm (allocates staging)
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        for _ in range(args.e2e_steps):
+            plan.solve_host(*host, xh, stream=stream)  # synchronises its stream
+        te = (time.perf_counter() - t0) / args.e2e_steps
+        tt = torch.tensor([te], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        te = float(tt.item())
+        e2e = {"value": m_all * n / te / 1e6, "unit": "Munknowns/s",
+               "h2d_bytes_per_step": 4 * n_unknowns * s, "d2h_bytes_per_step": n_unknowns * s,
+               "steps": args.e2e_steps, "ms_per_step": te * 1e3,
+               "how": "tri_solve_host: pinned host a,b,c,d -> device, solve, x -> pinned host, per step"}
+        del xh
+
+    # ---- CPU oracle baseline (rank 0 at N=1 only)
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu:
+        cpu = cpu_oracle_time(n, mr, [t.numpy() for t in host], layout)
+
+    if rank != 0:
+        dist.destroy_process_group()
+        return
+    peak, peak_src = measured_peaks()
+    algo_bytes = 5 * n_unknowns * s          # compulsory 5 arrays per unknown
+    achieved = algo_bytes / (t_step * 1e-3) / 1e9
+    traffic = None
+    tf = os.path.join(ROOT, "profiles", f"traffic_{args.config}.json")
+    if os.path.exists(tf):
+        with open(tf) as fh:
+            tj = json.load(fh)
+        if tj.get("n") == n and tj.get("m") == mr and tj.get("k") == plan.k:
+            traffic = tj.get("dram_bytes_per_launch")
+    out = {
+        "metric": METRIC, "value": value, "unit": "Munknowns/s", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": t_step_max, "higher_is_better": True, "scaling": args.scaling,
+        "vs_baseline": None, "dtype": dt, "data": "synthetic",
+        "config": {"workload": args.config, "desc": desc, "n": n, "m": m, "m_per_rank": mr, "layout": layout,
+                   "family": args.family, "parallelism": f"dp{world} (contiguous system shards, no collective)",
+                   "l2": "flushed between timed steps" if flush else
+                         f"inputs larger than L2 ({ws / 2**30:.1f} GiB working set vs {l2 / 2**20:.0f} MiB L2)",
+                   "plan": plan.describe()},
+        "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+                     "traffic": traffic, "peak_source": peak_src,
+                     "algorithmic_bytes_per_launch": algo_bytes,
+                     "kernel": "whole solve (%d launch%s)" % (plan.launches, "" if plan.launches == 1 else "es")},
+        "clocks": clk.summary(),
+        "e2e": e2e,
+        "gpu_launches": args.steps * plan.launches,
+        "cpu_baseline": cpu,
+        "parity": parity,
+        "step_ms_min": min(step_ms), "step_ms_median": statistics.median(step_ms),
+    }
+    print(json.dumps(out), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -123,67 +123,104 @@ __global__ void __launch_bounds__(128) k_pthomas(PThomasArgs<T> p) {
     }
 }
 
-// MODE 2: contiguous raw input, k = 0, staged through shared memory.
-constexpr int PT2_CH = 128;  // systems (threads) per CTA
+// MODE 2: contiguous raw input, k = 0.  A CTA of CH threads owns CH consecutive
+// systems.  An S-stage cp.async ring stages R-row tiles, smem layout
+// [stage][array][system][R + pad] (80-byte system stride: conflict-free 16-byte
+// reads), so each thread walks its own system's rows out of shared memory.
 template <typename T>
 struct PT2Cfg {
-    static constexpr int R = 64 / sizeof(T);  // rows per tile: one 64-byte segment per system
+    static constexpr int R = 64 / sizeof(T);      // rows per tile: one 64-byte segment per system
+    static constexpr int EPC = 16 / sizeof(T);    // elements per 16-byte chunk
+    static constexpr int SROW = R + EPC;          // padded per-system stride (80 bytes)
 };
+constexpr int PT2_S = 5;  // pipeline stages
+constexpr int PT2_UB = 16;  // backward-sweep prefetch depth (rows)
 
-template <typename T>
-__global__ void __launch_bounds__(PT2_CH) k_pthomas_contig(PThomasArgs<T> p) {
-    constexpr int R = PT2Cfg<T>::R;
-    constexpr int W = PT2_CH + 1;  // padded row of the transposed tile
-    __shared__ T tile[4][R][W];  // [array][row][system]
+template <typename T, int CH>
+__host__ __device__ constexpr int pt2_smem_bytes() {
+    return PT2_S * 4 * CH * PT2Cfg<T>::SROW * (int)sizeof(T);
+}
+
+template <typename T, int CH, bool VEC16>
+__global__ void __launch_bounds__(CH) k_pthomas_contig(PThomasArgs<T> p) {
+    constexpr int R = PT2Cfg<T>::R, EPC = PT2Cfg<T>::EPC, SROW = PT2Cfg<T>::SROW;
+    constexpr int STAGE = 4 * CH * SROW;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    T* sm = reinterpret_cast<T*>(smem_raw);
     const int tid = threadIdx.x;
-    const int64_t q0 = (int64_t)blockIdx.x * PT2_CH;
-    const int G = (int)imin64(PT2_CH, p.m - q0);
+    const int64_t q0 = (int64_t)blockIdx.x * CH;
+    const int G = (int)imin64(CH, p.m - q0);
     const int64_t n = p.n;
     const int64_t ntile = (n + R - 1) / R;
+    auto src = [&](int arr) { return arr == 0 ? p.a : arr == 1 ? p.b : arr == 2 ? p.c : p.d; };
+
+    auto issue = [&](int64_t t) {
+        T* st = sm + (int)(t % PT2_S) * STAGE;
+        if (VEC16) {
+            constexpr int CPS = R / EPC;  // 16-byte chunks per system segment
+#pragma unroll 4
+            for (int e = tid; e < 4 * CH * CPS; e += CH) {
+                const int arr = e / (CH * CPS);
+                const int rem = e - arr * CH * CPS;
+                const int g = rem / CPS, ck = rem - (rem / CPS) * CPS;
+                const int64_t i = t * R + ck * EPC;
+                int bytes = 0;
+                const T* gp = src(arr);
+                if (g < G && i < n) {
+                    bytes = (int)imin64(EPC, n - i) * (int)sizeof(T);
+                    gp = src(arr) + (q0 + g) * n + i;
+                }
+                cp_async_16(st + (arr * CH + g) * SROW + ck * EPC, gp, bytes);
+            }
+        } else {
+#pragma unroll 4
+            for (int e = tid; e < 4 * CH * R; e += CH) {
+                const int arr = e / (CH * R);
+                const int rem = e - arr * CH * R;
+                const int g = rem / R, u = rem - (rem / R) * R;
+                const int64_t i = t * R + u;
+                int bytes = 0;
+                const T* gp = src(arr);
+                if (g < G && i < n) {
+                    bytes = (int)sizeof(T);
+                    gp = src(arr) + (q0 + g) * n + i;
+                }
+                if (sizeof(T) == 8) cp_async_8(st + (arr * CH + g) * SROW + u, gp, bytes);
+                else cp_async_4(st + (arr * CH + g) * SROW + u, gp, bytes);
+            }
+        }
+    };
+
+#pragma unroll
+    for (int s = 0; s < PT2_S - 1; ++s) {
+        if (s < ntile) issue(s);
+        cp_async_commit();
+    }
     const int64_t ch = q0 + tid;
     const bool active = tid < G;
-
-    // cooperative loader: element e of a tile = (system e / R, row e % R)
-    auto load_tile = [&](int64_t t, T (&reg)[4][R]) {
-#pragma unroll
-        for (int u = 0; u < R; ++u) {
-            const int e = tid + u * PT2_CH;
-            const int g = e / R, rr = e % R;
-            const int64_t i = t * R + rr;
-            T av = T(0), bv = T(1), cv = T(0), dv = T(0);
-            if (g < G && i < n) {
-                const int64_t gi = (q0 + g) * n + i;
-                av = i > 0 ? ldg_stream(p.a + gi) : T(0);
-                bv = ldg_stream(p.b + gi);
-                cv = i < n - 1 ? ldg_stream(p.c + gi) : T(0);
-                dv = ldg_stream(p.d + gi);
-            }
-            reg[0][u] = av; reg[1][u] = bv; reg[2][u] = cv; reg[3][u] = dv;
-        }
-    };
-    auto store_tile = [&](const T (&reg)[4][R]) {
-#pragma unroll
-        for (int u = 0; u < R; ++u) {
-            const int e = tid + u * PT2_CH;
-            const int g = e / R, rr = e % R;
-#pragma unroll
-            for (int v = 0; v < 4; ++v) tile[v][rr][g] = reg[v][u];
-        }
-    };
-
     T cp = T(0), dp = T(0);
-    T reg[4][R];
-    load_tile(0, reg);
-    store_tile(reg);
-    __syncthreads();
     for (int64_t t = 0; t < ntile; ++t) {
-        if (t + 1 < ntile) load_tile(t + 1, reg);  // in flight while we compute
+        cp_async_wait<PT2_S - 2>();
+        __syncthreads();  // tile t visible to all; stage (t-1) % S free
+        if (t + PT2_S - 1 < ntile) issue(t + PT2_S - 1);
+        cp_async_commit();
         if (active) {
+            const T* st = sm + (int)(t % PT2_S) * STAGE + tid * SROW;
+            T v[4][R];
+#pragma unroll
+            for (int arr = 0; arr < 4; ++arr)
+#pragma unroll
+                for (int c = 0; c < R / EPC; ++c) {
+                    const int4 w = *reinterpret_cast<const int4*>(st + arr * CH * SROW + c * EPC);
+                    const T* wt = reinterpret_cast<const T*>(&w);
+#pragma unroll
+                    for (int e = 0; e < EPC; ++e) v[arr][c * EPC + e] = wt[e];
+                }
 #pragma unroll
             for (int u = 0; u < R; ++u) {
                 const int64_t j = t * R + u;
                 if (j < n) {
-                    Row4<T> row{tile[0][u][tid], tile[1][u][tid], tile[2][u][tid], tile[3][u][tid]};
+                    Row4<T> row{j > 0 ? v[0][u] : T(0), v[1][u], j < n - 1 ? v[2][u] : T(0), v[3][u]};
                     thomas_fwd(row, cp, dp);
                     const int64_t idx = j * p.C + ch;
                     p.cps[idx] = cp;
@@ -191,37 +228,32 @@ __global__ void __launch_bounds__(PT2_CH) k_pthomas_contig(PThomasArgs<T> p) {
                 }
             }
         }
-        __syncthreads();
-        if (t + 1 < ntile) {
-            store_tile(reg);
-            __syncthreads();
+    }
+    cp_async_wait<0>();
+    if (!active) return;
+    // backward sweep (Eq 4) with a PT2_UB-row register prefetch; x stored directly
+    T* xq = p.x + ch * n;
+    T xv = dp;
+    xq[n - 1] = xv;
+    int64_t j = n - 2;
+    for (; j >= PT2_UB - 1; j -= PT2_UB) {
+        T cs[PT2_UB], ds[PT2_UB];
+#pragma unroll
+        for (int u = 0; u < PT2_UB; ++u) {
+            const int64_t idx = (j - u) * p.C + ch;
+            cs[u] = p.cps[idx];
+            ds[u] = p.dps[idx];
+        }
+#pragma unroll
+        for (int u = 0; u < PT2_UB; ++u) {
+            xv = fma(-cs[u], xv, ds[u]);
+            xq[j - u] = xv;
         }
     }
-    // backward sweep, tile by tile from the end; x staged in tile[0][0]
-    T xv = dp;
-    for (int64_t t = ntile - 1; t >= 0; --t) {
-        if (active) {
-#pragma unroll
-            for (int u = R - 1; u >= 0; --u) {
-                const int64_t j = t * R + u;
-                if (j < n) {
-                    if (j < n - 1) {
-                        const int64_t idx = j * p.C + ch;
-                        xv = fma(-p.cps[idx], xv, p.dps[idx]);
-                    }
-                    tile[0][u][tid] = xv;
-                }
-            }
-        }
-        __syncthreads();
-#pragma unroll
-        for (int u = 0; u < R; ++u) {
-            const int e = tid + u * PT2_CH;
-            const int g = e / R, rr = e % R;
-            const int64_t i = t * R + rr;
-            if (g < G && i < n) __stcs(p.x + (q0 + g) * n + i, tile[0][rr][g]);
-        }
-        __syncthreads();
+    for (; j >= 0; --j) {
+        const int64_t idx = j * p.C + ch;
+        xv = fma(-p.cps[idx], xv, p.dps[idx]);
+        xq[j] = xv;
     }
 }
 

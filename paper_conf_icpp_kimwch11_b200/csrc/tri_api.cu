@@ -215,6 +215,16 @@ cudaError_t launch_tiled(const tri_plan_s* p, const void* a, const void* b, cons
     return cudaGetLastError();
 }
 
+template <typename T, int CH>
+cudaError_t launch_contig(const tri_plan_s* p, const PThomasArgs<T>& A, bool vec, cudaStream_t st) {
+    constexpr int smem = pt2_smem_bytes<T, CH>();
+    auto kern = vec ? k_pthomas_contig<T, CH, true> : k_pthomas_contig<T, CH, false>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e != cudaSuccess) return e;
+    kern<<<(unsigned)cdiv(p->m, CH), CH, smem, st>>>(A);
+    return cudaGetLastError();
+}
+
 template <typename T>
 cudaError_t launch_split(const tri_plan_s* p, const void* a, const void* b, const void* c, const void* d,
                          void* x, cudaStream_t st) {
@@ -234,10 +244,14 @@ cudaError_t launch_split(const tri_plan_s* p, const void* a, const void* b, cons
     } else {
         A.iA = A.iC = A.iD = nullptr;
         A.cps = base; A.dps = base + ce;
-        if (p->layout == TRI_LAYOUT_INTERLEAVED)
+        if (p->layout == TRI_LAYOUT_INTERLEAVED) {
             k_pthomas<T, 1><<<(unsigned)cdiv(p->C, 128), 128, 0, st>>>(A);
-        else
-            k_pthomas_contig<T><<<(unsigned)cdiv(p->m, PT2_CH), PT2_CH, 0, st>>>(A);
+        } else {
+            const bool vec = ((p->n * (int64_t)sizeof(T)) % 16) == 0 && ((uintptr_t)a % 16) == 0;
+            // 16 systems per CTA when the batch is thin (finer balance over the SMs)
+            const bool thin = cdiv(p->m, 32) < 6 * (int64_t)p->sms;
+            return thin ? launch_contig<T, 16>(p, A, vec, st) : launch_contig<T, 32>(p, A, vec, st);
+        }
     }
     return cudaGetLastError();
 }
