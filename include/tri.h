@@ -98,6 +98,15 @@ TRI_API tri_status tri_solve_host(tri_plan_t plan, const void* a, const void* b,
 TRI_API tri_status tri_debug_pcr(tri_plan_t plan, const void* a, const void* b, const void* c,
                          const void* d, void* ao, void* co, void* do_, void* stream);
 
+/* Diagnostics: when dev_counters (device memory, 9 x uint64, zeroed by the
+ * caller) is non-NULL, the fused kernel accumulates per-role clock64() cycle
+ * counters into it: [0] forward warp waiting for PCR rows, [1] forward warp
+ * total, [2] forward warp waiting for free storage, [3] forward warp storing,
+ * [4] PCR warps waiting for handoff slots, [5] PCR warps total, [6] back
+ * substitution warp total, [7] back substitution waiting for forward sweeps.
+ * Process-wide; NULL disables (default). */
+TRI_API void tri_debug_set_profile(void* dev_counters);
+
 /* Release the plan and its scratch.  NULL-safe.  Must not race a solve. */
 TRI_API void tri_destroy(tri_plan_t plan);
 

@@ -61,6 +61,7 @@ def lib():
             "tri_choose_k": (_I, [_I64, _I64, _I, _I, _I]),
             "tri_choose_variant": (_I, [_I64, _I64, _I, _I, _I]),
             "tri_shard_range": (None, [_I64, _I, _I, ctypes.POINTER(_I64), ctypes.POINTER(_I64)]),
+            "tri_debug_set_profile": (None, [_P]),
         }
         for name, (res, args) in sig.items():
             fn = getattr(L, name)

@@ -16,12 +16,15 @@
 #include "k_onchip.cuh"
 #include "k_tiled_pcr.cuh"
 #include "k_pthomas.cuh"
+#include "k_fused.cuh"
 
 using namespace tri;
 
 namespace {
 
 thread_local tri_status g_last = TRI_OK;
+void* g_fused_prof = nullptr;  // tri_debug_set_profile: device counters for the fused kernel
+int g_fused_dbg_mode = 0;     // TRI_FUSED_DBG_MODE (diagnostics only)
 
 constexpr int ONCHIP_THREADS = 512;
 constexpr int SPLIT_KMAX = 10;  // deepest k one sliding-window pass holds in smem (T = 256)
@@ -54,8 +57,16 @@ int onchip_G(int64_t n, int64_t m, tri_dtype t, int sms) {
     return (int)G;
 }
 
-tri_variant choose_variant(int64_t n, int64_t m, tri_dtype t, tri_layout, int) {
-    return n <= onchip_rows_budget(t) ? TRI_VARIANT_ONCHIP : TRI_VARIANT_SPLIT;
+// FUSED needs the contiguous layout (or m = 1) and enough systems to give
+// every SM its own (one system per CTA at a time).
+bool fused_ok(int64_t n, int64_t m, tri_layout layout) {
+    return (layout == TRI_LAYOUT_CONTIGUOUS || m == 1) && n >= 2 * FU_W;
+}
+
+tri_variant choose_variant(int64_t n, int64_t m, tri_dtype t, tri_layout layout, int sms) {
+    if (n <= onchip_rows_budget(t)) return TRI_VARIANT_ONCHIP;
+    if (fused_ok(n, m, layout) && m >= sms) return TRI_VARIANT_FUSED;
+    return TRI_VARIANT_SPLIT;
 }
 
 // Paper rule: M > P => k = 0; M <= P => the largest k with 2^k M <= P,
@@ -68,6 +79,7 @@ int choose_k_for(tri_variant v, int64_t n, int64_t m, tri_dtype t, tri_layout la
         int k = ceil_log2(cdiv(64, G));
         return std::min(k, kmax_n);
     }
+    if (v == TRI_VARIANT_FUSED) return FU_K;
     const int64_t P = (int64_t)sms * 64;
     int k = m >= P ? 0 : ceil_log2(cdiv(P, m));
     return std::min(std::min(k, kmax_n), SPLIT_KMAX);
@@ -75,8 +87,10 @@ int choose_k_for(tri_variant v, int64_t n, int64_t m, tri_dtype t, tri_layout la
 
 int kmax_for(tri_variant v, int64_t n) {
     const int kn = floor_log2(n);
+    if (v == TRI_VARIANT_FUSED) return FU_K;
     return v == TRI_VARIANT_SPLIT ? std::min(kn, SPLIT_KMAX) : kn;
 }
+int kmin_for(tri_variant v) { return v == TRI_VARIANT_FUSED ? FU_K : 0; }
 
 }  // namespace
 
@@ -90,6 +104,10 @@ struct tri_plan_s {
     int G, P, rpt;            // ONCHIP geometry
     int64_t n_pad, L, C;      // SPLIT: chain length, chains
     int64_t region, nreg;     // SPLIT: tiled-PCR regions per system
+    int fu_grid, fu_son;      // FUSED: persistent CTAs, on-chip positions per chain
+    bool fu_vec;              // FUSED: staged 8-row-aligned path
+    int64_t fu_nc;            // FUSED: windows per system
+    size_t smem_optin;
     void* scratch;
     size_t scratch_bytes;
     void* stage;              // tri_solve_host staging (5 arrays), lazily allocated
@@ -133,9 +151,25 @@ void plan_geometry(tri_plan_s* p) {
         }
         p->G = 0; p->P = 0; p->rpt = 0;
     }
+    if (p->variant == TRI_VARIANT_FUSED) {
+        const size_t s = esize(p->dtype);
+        p->L = cdiv(n, FU_S);
+        p->n_pad = p->L * FU_S;
+        p->C = m * FU_S;
+        p->fu_nc = cdiv(p->n_pad, FU_V);
+        p->fu_grid = (int)std::min<int64_t>(m, p->sms);
+        const bool vec = (n % 8) == 0;  // the staged (cp.async) path; pointers checked at launch
+        p->fu_vec = vec;
+        const int fixed = (p->dtype == TRI_F64 ? fused_fixed_smem<double>() : fused_fixed_smem<float>()) +
+                          (vec ? (p->dtype == TRI_F64 ? fused_stage_smem<double>() : fused_stage_smem<float>()) : 0);
+        const int64_t avail = ((int64_t)p->smem_optin - fixed) / (int64_t)(FU_S * 2 * s);
+        p->fu_son = (int)std::max<int64_t>(0, std::min<int64_t>(p->L, avail));
+    }
 }
 
 size_t scratch_need(const tri_plan_s* p) {
+    if (p->variant == TRI_VARIANT_FUSED)
+        return (size_t)p->fu_grid * 2 * (size_t)std::max<int64_t>(0, p->L - p->fu_son) * FU_S * 2 * esize(p->dtype);
     if (p->variant != TRI_VARIANT_SPLIT) return 0;
     const size_t s = esize(p->dtype);
     const size_t chain_elems = (size_t)p->C * (size_t)p->L;
@@ -212,6 +246,26 @@ cudaError_t launch_tiled(const tri_plan_s* p, const void* a, const void* b, cons
     if (e != cudaSuccess) return e;
     const int64_t grid = p->m * p->nreg;
     k_tiled_pcr<T><<<(unsigned)grid, TPCR_T, smem, st>>>(A);
+    return cudaGetLastError();
+}
+
+template <typename T>
+cudaError_t launch_fused(const tri_plan_s* p, const void* a, const void* b, const void* c, const void* d, void* x,
+                         cudaStream_t st, void* dA = nullptr, void* dC = nullptr, void* dD = nullptr) {
+    FusedArgs<T> A;
+    A.dA = (T*)dA; A.dC = (T*)dC; A.dD = (T*)dD;
+    A.prof = (unsigned long long*)g_fused_prof;
+    A.dbg_mode = g_fused_dbg_mode;
+    A.a = (const T*)a; A.b = (const T*)b; A.c = (const T*)c; A.d = (const T*)d; A.x = (T*)x;
+    A.spill = (T*)p->scratch;
+    A.n = p->n; A.m = p->m; A.L = p->L; A.NC = p->fu_nc; A.S_on = p->fu_son;
+    const bool vec = p->fu_vec && ((uintptr_t)a | (uintptr_t)b | (uintptr_t)c | (uintptr_t)d) % 16 == 0;
+    const size_t smem = (size_t)fused_fixed_smem<T>() + (vec ? (size_t)fused_stage_smem<T>() : 0) +
+                        (size_t)p->fu_son * FU_S * 2 * sizeof(T);
+    auto kern = vec ? k_fused<T, true> : k_fused<T, false>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    kern<<<p->fu_grid, FU_THREADS, smem, st>>>(A);
     return cudaGetLastError();
 }
 
@@ -339,6 +393,12 @@ const char* tri_status_str(tri_status s) {
 
 tri_status tri_last_status(void) { return g_last; }
 
+void tri_debug_set_profile(void* dev_counters) {
+    g_fused_prof = dev_counters;
+    const char* e = getenv("TRI_FUSED_DBG_MODE");
+    g_fused_dbg_mode = e ? atoi(e) : 0;
+}
+
 tri_plan_t tri_plan(int64_t n, int64_t m, tri_dtype dtype, tri_layout layout) {
     if (n < 1 || m < 1 || (dtype != TRI_F32 && dtype != TRI_F64) ||
         (layout != TRI_LAYOUT_CONTIGUOUS && layout != TRI_LAYOUT_INTERLEAVED) || n > MAX_ELEMS / m) {
@@ -350,6 +410,9 @@ tri_plan_t tri_plan(int64_t n, int64_t m, tri_dtype dtype, tri_layout layout) {
     if (st != TRI_OK) { g_last = st; return nullptr; }
     tri_plan_s* p = new tri_plan_s();
     p->n = n; p->m = m; p->dtype = dtype; p->layout = layout; p->device = dev; p->sms = sms;
+    int optin = 0;
+    cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+    p->smem_optin = (size_t)optin;
     p->variant = choose_variant(n, m, dtype, layout, sms);
     p->k = choose_k_for(p->variant, n, m, dtype, layout, sms);
     plan_geometry(p);
@@ -373,11 +436,11 @@ int64_t tri_plan_scratch_bytes(tri_plan_t p) { return p ? (int64_t)p->scratch_by
 int tri_plan_launches(tri_plan_t p) {
     if (!p) return -1;
     if (p->variant == TRI_VARIANT_SPLIT) return p->k > 0 ? 2 : 1;
-    return 1;
+    return 1;  // ONCHIP, FUSED
 }
 
 tri_status tri_plan_set_k(tri_plan_t p, int k) {
-    if (!p || k < 0 || k > kmax_for(p->variant, p->n)) return TRI_ERR_INVALID_ARG;
+    if (!p || k < kmin_for(p->variant) || k > kmax_for(p->variant, p->n)) return TRI_ERR_INVALID_ARG;
     const int old = p->k;
     p->k = k;
     plan_geometry(p);
@@ -390,7 +453,8 @@ tri_status tri_plan_set_variant(tri_plan_t p, tri_variant v) {
     if (!p) return TRI_ERR_INVALID_ARG;
     if (v == TRI_VARIANT_AUTO) v = choose_variant(p->n, p->m, p->dtype, p->layout, p->sms);
     if (v == TRI_VARIANT_ONCHIP && p->n > onchip_rows_budget(p->dtype)) return TRI_ERR_INVALID_ARG;
-    if (v != TRI_VARIANT_ONCHIP && v != TRI_VARIANT_SPLIT) return TRI_ERR_INVALID_ARG;
+    if (v == TRI_VARIANT_FUSED && !fused_ok(p->n, p->m, p->layout)) return TRI_ERR_INVALID_ARG;
+    if (v != TRI_VARIANT_ONCHIP && v != TRI_VARIANT_SPLIT && v != TRI_VARIANT_FUSED) return TRI_ERR_INVALID_ARG;
     const tri_variant ov = p->variant;
     const int ok = p->k;
     p->variant = v;
@@ -407,11 +471,11 @@ void tri_plan_describe(tri_plan_t p, char* buf, int len) {
     static const char* vn[] = {"auto", "onchip", "split", "fused"};
     snprintf(buf, len,
              "n=%lld m=%lld dtype=%s layout=%s variant=%s k=%d G=%d P=%d rpt=%d L=%lld C=%lld region=%lld nreg=%lld "
-             "scratch=%zu sms=%d",
+             "fu_grid=%d fu_son=%d fu_nc=%lld scratch=%zu sms=%d",
              (long long)p->n, (long long)p->m, p->dtype == TRI_F64 ? "f64" : "f32",
              p->layout == TRI_LAYOUT_CONTIGUOUS ? "contiguous" : "interleaved", vn[p->variant], p->k, p->G, p->P,
-             p->rpt, (long long)p->L, (long long)p->C, (long long)p->region, (long long)p->nreg, p->scratch_bytes,
-             p->sms);
+             p->rpt, (long long)p->L, (long long)p->C, (long long)p->region, (long long)p->nreg, p->fu_grid, p->fu_son,
+             (long long)p->fu_nc, p->scratch_bytes, p->sms);
 }
 
 tri_status tri_solve(tri_plan_t p, const void* a, const void* b, const void* c, const void* d, void* x,
@@ -426,6 +490,8 @@ tri_status tri_solve(tri_plan_t p, const void* a, const void* b, const void* c, 
     if (p->variant == TRI_VARIANT_ONCHIP) {
         e = p->dtype == TRI_F64 ? launch_onchip<double>(p, a, b, c, d, x, nullptr, nullptr, nullptr, 0, s)
                                 : launch_onchip<float>(p, a, b, c, d, x, nullptr, nullptr, nullptr, 0, s);
+    } else if (p->variant == TRI_VARIANT_FUSED) {
+        e = p->dtype == TRI_F64 ? launch_fused<double>(p, a, b, c, d, x, s) : launch_fused<float>(p, a, b, c, d, x, s);
     } else {
         e = p->dtype == TRI_F64 ? launch_split<double>(p, a, b, c, d, x, s) : launch_split<float>(p, a, b, c, d, x, s);
     }
@@ -444,6 +510,9 @@ tri_status tri_debug_pcr(tri_plan_t p, const void* a, const void* b, const void*
     if (p->variant == TRI_VARIANT_ONCHIP) {
         e = p->dtype == TRI_F64 ? launch_onchip<double>(p, a, b, c, d, nullptr, ao, co, do_, 1, s)
                                 : launch_onchip<float>(p, a, b, c, d, nullptr, ao, co, do_, 1, s);
+    } else if (p->variant == TRI_VARIANT_FUSED) {
+        e = p->dtype == TRI_F64 ? launch_fused<double>(p, a, b, c, d, nullptr, s, ao, co, do_)
+                                : launch_fused<float>(p, a, b, c, d, nullptr, s, ao, co, do_);
     } else {
         if (p->k == 0) return TRI_ERR_INVALID_ARG;  // no PCR stage to show
         e = p->dtype == TRI_F64 ? launch_tiled<double>(p, a, b, c, d, ao, co, do_, 1, s)

@@ -234,3 +234,64 @@ def test_solve_host(cuda_ok):
     out = torch.empty(n * m, dtype=torch.float64).pin_memory()
     plan.solve_host(*pin, out)
     check_parity(n, m, arrs, out.numpy(), "f64", 0)
+
+
+# ------------------------------------------------------------------ FUSED variant
+FUSED = tri.VARIANT_FUSED
+
+
+@pytest.mark.parametrize("dtype", ["f64", "f32"])
+@pytest.mark.parametrize("n,m", [(512, 3), (2048, 5), (16384, 7), (4099, 2), (4100, 3), (100000, 2), (1001, 300),
+                                 (16392, 150)])
+def test_fused_parity(cuda_ok, dtype, n, m):
+    arrs = gen(n, m, dtype, 0)
+    x, plan = gpu_solve(n, m, arrs, dtype, 0, variant=FUSED)
+    assert plan.k == 3
+    check_parity(n, m, arrs, x, dtype, 0)
+
+
+@pytest.mark.parametrize("family,eps", [("weak", 1e-2), ("weak", 1e-3), ("integer", 0.0), ("poisson", 0.0)])
+def test_fused_families(cuda_ok, family, eps):
+    n, m = 16384, 6
+    arrs = gen(n, m, "f64", 0, family, eps=eps)
+    x, _ = gpu_solve(n, m, arrs, "f64", 0, variant=FUSED)
+    if family == "poisson":
+        # Poisson is ill-conditioned (kappa ~ n^2/2): forward error vs oracle bounded by kappa*u
+        xo = oracle.solve_batch(n, m, *arrs)
+        assert np.max(np.abs(x - xo)) / np.max(np.abs(xo)) <= 2 * (n + 1) ** 2 / 2 * 2.2e-16
+    else:
+        check_parity(n, m, arrs, x, "f64", 0)
+
+
+@pytest.mark.parametrize("n,m", [(4099, 2), (16384, 3)])
+def test_fused_pcr_stage(cuda_ok, n, m):
+    arrs = gen(n, m, "f64", 0, "weak", eps=1e-2)
+    plan = tri.Plan(n, m, tri.F64, 0)
+    plan.variant = FUSED
+    A, C, D = (t.cpu().numpy() for t in plan.debug_pcr(*to_dev(*arrs)))
+    for q in range(m):
+        sl = slice(q * n, (q + 1) * n)
+        ao, bo, co, do = oracle.pcr_k(*(t[sl] for t in arrs), plan.k)
+        for got, ref in ((A[sl], ao / bo), (C[sl], co / bo), (D[sl], do / bo)):
+            assert np.max(np.abs(got - ref)) <= 1e-12 * max(1.0, np.max(np.abs(ref)))
+
+
+def test_fused_edges_and_scaling(cuda_ok):
+    import torch
+    n, m = 9000, 5
+    a, b, c, d = gen(n, m, "f64", 0, "weak", eps=1e-2)
+    plan = tri.Plan(n, m, tri.F64, 0)
+    plan.variant = FUSED
+    da, db, dc, dd = to_dev(a, b, c, d)
+    x1 = plan.solve(da, db, dc, dd).clone()
+    a2, c2 = da.clone(), dc.clone()
+    a2.view(m, n)[:, 0] = float("nan")
+    c2.view(m, n)[:, -1] = float("nan")
+    assert torch.equal(plan.solve(a2, db, c2, dd), x1)
+    p = 2.0 ** np.random.default_rng(1).integers(-20, 20, n * m)
+    x2 = plan.solve(*to_dev(a * p, b * p, c * p, d * p))
+    assert torch.equal(x2, x1)
+    x3 = plan.solve(da, db, dc, dd * 4.0)
+    assert torch.equal(x3, x1 * 4.0)
+    with pytest.raises(tri.TriError):
+        plan.k = 2  # the fused kernel is built for k = 3
