@@ -65,6 +65,10 @@ bool fused_ok(int64_t n, int64_t m, tri_layout layout) {
 
 tri_variant choose_variant(int64_t n, int64_t m, tri_dtype t, tri_layout layout, int sms) {
     if (n <= onchip_rows_budget(t)) return TRI_VARIANT_ONCHIP;
+    // paper rule: with more systems than the machine's parallelism go
+    // straight to p-Thomas (k = 0); between one system per SM and that point
+    // the fused streaming kernel supplies the chains.
+    if (m >= 64 * (int64_t)sms) return TRI_VARIANT_SPLIT;
     if (fused_ok(n, m, layout) && m >= sms) return TRI_VARIANT_FUSED;
     return TRI_VARIANT_SPLIT;
 }
