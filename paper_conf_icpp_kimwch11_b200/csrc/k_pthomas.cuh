@@ -133,7 +133,7 @@ struct PT2Cfg {
     static constexpr int EPC = 16 / sizeof(T);    // elements per 16-byte chunk
     static constexpr int SROW = R + EPC;          // padded per-system stride (80 bytes)
 };
-constexpr int PT2_S = 5;  // pipeline stages
+constexpr int PT2_S = 6;  // pipeline stages
 constexpr int PT2_UB = 16;  // backward-sweep prefetch depth (rows)
 
 template <typename T, int CH>
@@ -154,23 +154,38 @@ __global__ void __launch_bounds__(CH) k_pthomas_contig(PThomasArgs<T> p) {
     const int64_t ntile = (n + R - 1) / R;
     auto src = [&](int arr) { return arr == 0 ? p.a : arr == 1 ? p.b : arr == 2 ? p.c : p.d; };
 
+    // this thread's share of a tile's 16-byte chunks: 4 arrays x CPS (system, chunk)
+    // pairs, fixed for the whole sweep (only the row offset t*R changes)
+    constexpr int CPS = R / EPC;
+    int64_t gofs[CPS];
+    int soff[CPS];
+    bool gval[CPS];
+#pragma unroll
+    for (int jj = 0; jj < CPS; ++jj) {
+        const int rem = tid + jj * CH;
+        const int g = rem / CPS, ck = rem % CPS;
+        gval[jj] = g < G;
+        gofs[jj] = (q0 + (g < G ? g : 0)) * n + ck * EPC;
+        soff[jj] = g * SROW + ck * EPC;
+    }
     auto issue = [&](int64_t t) {
         T* st = sm + (int)(t % PT2_S) * STAGE;
+        const int64_t r0 = t * R;
         if (VEC16) {
-            constexpr int CPS = R / EPC;  // 16-byte chunks per system segment
-#pragma unroll 4
-            for (int e = tid; e < 4 * CH * CPS; e += CH) {
-                const int arr = e / (CH * CPS);
-                const int rem = e - arr * CH * CPS;
-                const int g = rem / CPS, ck = rem - (rem / CPS) * CPS;
-                const int64_t i = t * R + ck * EPC;
-                int bytes = 0;
-                const T* gp = src(arr);
-                if (g < G && i < n) {
-                    bytes = (int)imin64(EPC, n - i) * (int)sizeof(T);
-                    gp = src(arr) + (q0 + g) * n + i;
+            const bool full_tile = r0 + R <= n;
+#pragma unroll
+            for (int arr = 0; arr < 4; ++arr) {
+                const T* base = src(arr);
+#pragma unroll
+                for (int jj = 0; jj < CPS; ++jj) {
+                    int bytes = 16;
+                    if (!full_tile || !gval[jj]) {
+                        const int64_t i = r0 + (soff[jj] % SROW);
+                        bytes = (gval[jj] && i < n) ? (int)imin64(EPC, n - i) * (int)sizeof(T) : 0;
+                    }
+                    cp_async_16(st + arr * CH * SROW + soff[jj], bytes ? (const void*)(base + gofs[jj] + r0)
+                                                                        : (const void*)base, bytes);
                 }
-                cp_async_16(st + (arr * CH + g) * SROW + ck * EPC, gp, bytes);
             }
         } else {
 #pragma unroll 4
@@ -229,31 +244,68 @@ __global__ void __launch_bounds__(CH) k_pthomas_contig(PThomasArgs<T> p) {
             }
         }
     }
+    // backward sweep (Eq 4), tiles of RB positions walked from the end; the c', d'
+    // rows of this CTA's CH chains are staged by cp.async into the (now idle)
+    // ring, PT2_S - 1 tiles ahead, so the scratch reads keep HBM busy.
     cp_async_wait<0>();
-    if (!active) return;
-    // backward sweep (Eq 4) with a PT2_UB-row register prefetch; x stored directly
+    __syncthreads();
+    constexpr int RB = 16;                 // positions per backward tile
+    constexpr int BST = 2 * RB * CH;       // elements per backward stage
+    static_assert(BST <= STAGE, "backward stage must fit a forward stage");
+    const int64_t nb = n - 1;              // positions n-2 .. 0 (x_{n-1} = d'_{n-1})
+    const int64_t nbt = (nb + RB - 1) / RB;
+    auto issue_b = [&](int64_t bt) {       // tile bt covers positions [lo, hi)
+        if (bt < nbt) {
+            T* st = sm + (int)(bt % PT2_S) * STAGE;
+            const int64_t hi = nb - bt * RB, lo = imax64(hi - RB, 0);
+            constexpr int CPR = CH * (int)sizeof(T) / 16;  // 16-byte chunks per position row
+#pragma unroll
+            for (int e = tid; e < 2 * RB * CPR; e += CH) {
+                const int arr = e / (RB * CPR);
+                const int rem = e - arr * RB * CPR;
+                const int u = rem / CPR, ck = rem % CPR;
+                const int64_t j = hi - 1 - u;
+                const int gl = ck * (16 / (int)sizeof(T));
+                const bool ok = j >= lo && q0 + gl < p.m;
+                const T* base = arr == 0 ? p.cps : p.dps;
+                cp_async_16(st + (arr * RB + u) * CH + gl, ok ? (const void*)(base + j * p.C + q0 + gl)
+                                                              : (const void*)base, ok ? 16 : 0);
+            }
+        }
+        cp_async_commit();
+    };
+    const bool vecb = ((p.C * (int64_t)sizeof(T)) % 16 == 0) && ((q0 * (int64_t)sizeof(T)) % 16 == 0) &&
+                      (p.m - q0) >= CH;
     T* xq = p.x + ch * n;
     T xv = dp;
-    xq[n - 1] = xv;
-    int64_t j = n - 2;
-    for (; j >= PT2_UB - 1; j -= PT2_UB) {
-        T cs[PT2_UB], ds[PT2_UB];
+    if (active) xq[n - 1] = xv;
+    if (vecb) {
 #pragma unroll
-        for (int u = 0; u < PT2_UB; ++u) {
-            const int64_t idx = (j - u) * p.C + ch;
-            cs[u] = p.cps[idx];
-            ds[u] = p.dps[idx];
-        }
+        for (int s2 = 0; s2 < PT2_S - 1; ++s2) issue_b(s2);
+        for (int64_t bt = 0; bt < nbt; ++bt) {
+            cp_async_wait<PT2_S - 2>();
+            __syncthreads();
+            issue_b(bt + PT2_S - 1);
+            const T* st = sm + (int)(bt % PT2_S) * STAGE;
+            const int64_t hi = nb - bt * RB, lo = imax64(hi - RB, 0);
+            if (active) {
 #pragma unroll
-        for (int u = 0; u < PT2_UB; ++u) {
-            xv = fma(-cs[u], xv, ds[u]);
-            xq[j - u] = xv;
+                for (int u = 0; u < RB; ++u) {
+                    const int64_t j = hi - 1 - u;
+                    if (j >= lo) {
+                        xv = fma(-st[u * CH + tid], xv, st[(RB + u) * CH + tid]);
+                        xq[j] = xv;
+                    }
+                }
+            }
         }
-    }
-    for (; j >= 0; --j) {
-        const int64_t idx = j * p.C + ch;
-        xv = fma(-p.cps[idx], xv, p.dps[idx]);
-        xq[j] = xv;
+        cp_async_wait<0>();
+    } else if (active) {
+        for (int64_t j = n - 2; j >= 0; --j) {
+            const int64_t idx = j * p.C + ch;
+            xv = fma(-p.cps[idx], xv, p.dps[idx]);
+            xq[j] = xv;
+        }
     }
 }
 
