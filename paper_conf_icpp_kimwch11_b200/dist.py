@@ -1,0 +1,75 @@
+"""Multi-GPU driver for batches of independent systems.
+
+The m systems are split into contiguous ranges, one per rank (tri_shard_range);
+each rank solves its shard on its own GPU with no collective inside the solve
+(the systems are independent: Eq 1 per system).  Collectives
+appear only at the edges:
+  * gather_x:  rank 0 collects the solution (NCCL over NVLink on the GPU box,
+               gloo in the CPU tests);
+  * max_over_ranks: the timing convention (job time = slowest rank).
+A rank holds its shard in the same layout as the full batch with m_r columns
+(CONTIGUOUS: [ql*n + i]; INTERLEAVED: [i*m_r + ql]).
+"""
+import torch
+import torch.distributed as dist
+
+from . import CONTIGUOUS, INTERLEAVED, shard_range as _abi_shard_range
+
+
+def shard_range(m, world, rank):
+    """(q0, m_r): rank r owns systems [q0, q0 + m_r) (tri_shard_range)."""
+    return _abi_shard_range(int(m), int(world), int(rank))
+
+
+def max_over_ranks(value, group=None, device=None):
+    """Maximum of a python float over all ranks (all-reduce MAX)."""
+    if not dist.is_available() or not dist.is_initialized():
+        return float(value)
+    t = torch.tensor([float(value)], dtype=torch.float64, device=device)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX, group=group)
+    return float(t.item())
+
+
+def gather_x(x_local, n, m, layout=CONTIGUOUS, group=None, dst=0):
+    """Assemble the full solution (n*m) on rank `dst` from every rank's shard.
+    Returns the full tensor on dst, None elsewhere.  Shards are padded to
+    ceil(m/G) systems for the collective and unpadded on the root."""
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    per = -(-m // world)
+    q0, mr = shard_range(m, world, rank)
+    pad = torch.zeros(n * per, dtype=x_local.dtype, device=x_local.device)
+    if layout == CONTIGUOUS:
+        pad[: n * mr] = x_local
+    else:
+        pad.view(n, per)[:, :mr] = x_local.view(n, mr)
+    bufs = [torch.empty_like(pad) for _ in range(world)] if rank == dst else None
+    dist.gather(pad, gather_list=bufs, dst=dst, group=group)
+    if rank != dst:
+        return None
+    full = torch.empty(n * m, dtype=x_local.dtype, device=x_local.device)
+    for r in range(world):
+        rq0, rmr = shard_range(m, world, r)
+        if rmr == 0:
+            continue
+        if layout == CONTIGUOUS:
+            full[rq0 * n:(rq0 + rmr) * n] = bufs[r][: n * rmr]
+        else:
+            full.view(n, m)[:, rq0:rq0 + rmr] = bufs[r].view(n, per)[:, :rmr]
+    return full
+
+
+def solve_sharded(n, m, make_inputs, solve_fn, layout=CONTIGUOUS, gather=True, group=None):
+    """Solve this rank's shard.  make_inputs(q0, m_r) -> (a, b, c, d) for the
+    global systems [q0, q0+m_r) (generated locally: shards stay resident, no
+    scatter); solve_fn(a, b, c, d, m_r) -> x.  Returns (x_local, x_full or None)."""
+    world = dist.get_world_size(group) if dist.is_initialized() else 1
+    rank = dist.get_rank(group) if dist.is_initialized() else 0
+    q0, mr = shard_range(m, world, rank)
+    if mr > 0:
+        a, b, c, d = make_inputs(q0, mr)
+        x = solve_fn(a, b, c, d, mr)
+    else:
+        x = torch.empty(0, dtype=torch.float64)
+    full = gather_x(x, n, m, layout, group) if (gather and world > 1) else (x if gather else None)
+    return x, full
