@@ -11,7 +11,7 @@ import ctypes
 import os
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, "libtri.so")
+LIB_PATH = os.environ.get("TRI_LIB_PATH", os.path.join(HERE, "libtri.so"))  # override: experiments only
 
 F32, F64 = 0, 1
 CONTIGUOUS, INTERLEAVED = 0, 1

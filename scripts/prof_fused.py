@@ -16,7 +16,7 @@ plan = tri.Plan(n, m, tri.F64, 0)
 plan.variant = tri.VARIANT_FUSED
 x = torch.empty_like(b)
 plan.solve(a, b, c, d, out=x)
-cnt = torch.zeros(12, dtype=torch.int64, device="cuda")
+cnt = torch.zeros(16, dtype=torch.int64, device="cuda")
 tri.lib().tri_debug_set_profile(cnt.data_ptr())
 s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
 s.record()
@@ -27,8 +27,8 @@ tri.lib().tri_debug_set_profile(None)
 ms = s.elapsed_time(e)
 v = cnt.cpu().tolist()
 ncta = min(m, 148)
-names = ["TC wait full", "TC total", "TR wait TB", "TR store", "PCR wait empty (5 warps)", "PCR total (5 warps)",
-         "TB total", "TB wait TR", "TR total", "TC wait sempty", "TR wait sfull"]
+names = ["TC wait full", "TC total", "TR wait TB", "TR store", "PCR wait empty (all warps)", "PCR total (all warps)",
+         "TB total", "TB wait TR", "TR total", "TC wait sempty", "TR wait sfull", "PCR wait loads (all warps)", "TB on-chip segments", "TB spilled segments"]
 print(f"time {ms:.3f} ms, {ms * 1.965e6:.0f} cycles @1.965GHz; per CTA:")
 for nm, val in zip(names, v):
     print(f"  {nm:28s} {val / ncta:14.0f}")

@@ -246,7 +246,7 @@ FUSED = tri.VARIANT_FUSED
 def test_fused_parity(cuda_ok, dtype, n, m):
     arrs = gen(n, m, dtype, 0)
     x, plan = gpu_solve(n, m, arrs, dtype, 0, variant=FUSED)
-    assert plan.k == 3
+    assert plan.k == 4
     check_parity(n, m, arrs, x, dtype, 0)
 
 
@@ -294,4 +294,4 @@ def test_fused_edges_and_scaling(cuda_ok):
     x3 = plan.solve(da, db, dc, dd * 4.0)
     assert torch.equal(x3, x1 * 4.0)
     with pytest.raises(tri.TriError):
-        plan.k = 2  # the fused kernel is built for k = 3
+        plan.k = 2  # the fused kernel is built for one k
