@@ -64,7 +64,9 @@ typedef enum {
     TRI_VARIANT_AUTO = 0,   /* only as an argument of tri_plan_set_variant */
     TRI_VARIANT_ONCHIP = 1, /* whole system(s) in one CTA's smem: PCR + Thomas (Fig 11a/c) */
     TRI_VARIANT_SPLIT = 2,  /* tiled-PCR pass (sliding window, Figs 8-10) -> scratch, then p-Thomas */
-    TRI_VARIANT_FUSED = 3   /* streaming tiled PCR feeding p-Thomas in one kernel (Sec. III.C) */
+    TRI_VARIANT_FUSED = 3,  /* streaming tiled PCR feeding p-Thomas in one kernel (Sec. III.C) */
+    TRI_VARIANT_WARP = 4    /* 32 <= n <= 1024: one warp per system, k = 5 shuffle PCR steps + in-register
+                               p-Thomas on the 32 subsystems (Sec. III) */
 } tri_variant;
 
 typedef struct tri_plan_s* tri_plan_t;
@@ -78,9 +80,18 @@ TRI_API tri_plan_t tri_plan(int64_t n, int64_t m, tri_dtype dtype, tri_layout la
 /* Thread-local status of the last tri_plan call on this thread. */
 TRI_API tri_status tri_last_status(void);
 
-/* Solve: read a, b, c, d (device, read-only), write x (device).  Asynchronous
- * on `stream`.  At most one tri_solve per plan may be in flight (the plan's
- * scratch is reused); use one plan per concurrent stream. */
+/* Solve A x = d for the plan's m systems (Eq 1).  a, b, c, d: device
+ * pointers (read-only) to n*m elements of the plan's dtype in the plan's layout
+ * (CONTIGUOUS: system q row i at q*n + i; INTERLEAVED: at i*m + q); a of row 0
+ * and c of row n-1 are ignored (never read into arithmetic).  x: device output,
+ * same shape.  All five must be 16-byte aligned (TRI_ERR_ALIGNMENT), non-NULL
+ * (TRI_ERR_INVALID_ARG), on the plan's device (TRI_ERR_DEVICE; verified when
+ * the pointer set differs from the previous call's) and x must not overlap an
+ * input (TRI_ERR_ALIAS).  On error nothing is launched.  Asynchronous on
+ * `stream` (a cudaStream_t; NULL = legacy default stream); launch failures
+ * return TRI_ERR_CUDA.  At most one tri_solve per plan may be in flight (the
+ * plan's scratch is reused); use one plan per concurrent stream.  The caller
+ * owns every buffer; the plan owns its scratch. */
 TRI_API tri_status tri_solve(tri_plan_t plan, const void* a, const void* b, const void* c, const void* d,
                      void* x, void* stream);
 
@@ -98,13 +109,11 @@ TRI_API tri_status tri_solve_host(tri_plan_t plan, const void* a, const void* b,
 TRI_API tri_status tri_debug_pcr(tri_plan_t plan, const void* a, const void* b, const void* c,
                          const void* d, void* ao, void* co, void* do_, void* stream);
 
-/* Diagnostics: when dev_counters (device memory, 9 x uint64, zeroed by the
+/* Diagnostics: when dev_counters (device memory, 16 x uint64, zeroed by the
  * caller) is non-NULL, the fused kernel accumulates per-role clock64() cycle
- * counters into it: [0] forward warp waiting for PCR rows, [1] forward warp
- * total, [2] forward warp waiting for free storage, [3] forward warp storing,
- * [4] PCR warps waiting for handoff slots, [5] PCR warps total, [6] back
- * substitution warp total, [7] back substitution waiting for forward sweeps.
- * Process-wide; NULL disables (default). */
+ * counters into it (layout: scripts/prof_fused.py).  The environment variable
+ * TRI_FUSED_DBG_MODE, read here, disables parts of the fused kernel for cost
+ * attribution (results are then wrong).  Process-wide; NULL disables. */
 TRI_API void tri_debug_set_profile(void* dev_counters);
 
 /* Release the plan and its scratch.  NULL-safe.  Must not race a solve. */

@@ -309,4 +309,187 @@ __global__ void __launch_bounds__(CH) k_pthomas_contig(PThomasArgs<T> p) {
     }
 }
 
+
+// ---------------------------------------------------------------------------
+// MODE 0 / MODE 1 with few, long chains (k_pthomas_ring): a CTA of CW threads
+// owns CW adjacent chains; an 8-stage cp.async ring stages RP positions x CW
+// chains of every input array (RP * CW = 256, 6-8 KB per stage), so each SM
+// keeps ~50 KB of loads in flight even with one 8-thread CTA, and the grid
+// spreads a few thousand chains over all SMs.  The forward sweep is the
+// continuant form of Eqs 2-3 (X18): the serial dependency per
+// position is one FMA, the reciprocal of theta_i is off the chain.
+//   theta_i = theta_{i-1} - A_i C_{i-1} theta_{i-2},  delta_i = D_i theta_{i-1} - A_i delta_{i-1}
+//   c'_i = C_i theta_{i-1} / theta_i,                 d'_i = delta_i / theta_i
+// theta, delta are rescaled by exact powers of two when |theta| leaves
+// [2^-S, 2^S] (ratios, hence c', d', unchanged).  The back substitution (Eq 4)
+// streams c', d' back through the same ring in reverse.
+constexpr int PTR_NS = 8;      // ring stages
+constexpr int PTR_ROWS = 256;  // RP * CW per stage
+
+template <typename T>
+struct PTRScale;
+template <>
+struct PTRScale<double> {
+    static constexpr double lo = 0x1p-200, hi = 0x1p200, up = 0x1p200, down = 0x1p-200;
+};
+template <>
+struct PTRScale<float> {
+    static constexpr float lo = 0x1p-40f, hi = 0x1p40f, up = 0x1p40f, down = 0x1p-40f;
+};
+
+template <typename T, int CW>
+__host__ __device__ constexpr int ptr_smem_bytes(bool raw) {
+    return PTR_NS * (raw ? 4 : 3) * PTR_ROWS * (int)sizeof(T);
+}
+
+template <typename T, int CW, int MODE, bool VEC>
+__global__ void __launch_bounds__(CW) k_pthomas_ring(PThomasArgs<T> p) {
+    static_assert(MODE == 0 || MODE == 1, "ring p-Thomas takes chain-interleaved input");
+    constexpr int RP = PTR_ROWS / CW;            // positions per stage
+    constexpr int NA = MODE == 1 ? 4 : 3;        // input arrays
+    constexpr int EPC = 16 / (int)sizeof(T);     // elements per 16-byte chunk
+    constexpr int STAGE = NA * PTR_ROWS;         // elements per stage
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    T* sm = reinterpret_cast<T*>(smem_raw);
+    const int tid = threadIdx.x;
+    const int64_t ch0 = (int64_t)blockIdx.x * CW;
+    const int64_t ch = ch0 + tid;
+    const int64_t C = p.C, L = p.L;
+    const bool active = ch < C;
+    const int64_t nst = (L + RP - 1) / RP;
+
+    // stage t holds positions [t RP, t RP + RP) of arrays src(0..NA-1), layout [arr][u][CW]
+    auto issue = [&](int64_t t, int na, auto src) {
+        if (t < nst) {
+            T* st = sm + (int)(t % PTR_NS) * STAGE;
+            const int64_t p0 = t * RP;
+            if (VEC) {
+                constexpr int CPR = CW / EPC;      // chunks per (array, position) row
+                for (int e = tid; e < na * RP * CPR; e += CW) {
+                    const int arr = e / (RP * CPR);
+                    const int rem = e - arr * RP * CPR;
+                    const int u = rem / CPR, h = rem - u * CPR;
+                    const int64_t j = p0 + u, c0 = ch0 + h * EPC;
+                    const int64_t ok = (j < L && c0 < C) ? imin64(EPC, C - c0) : 0;
+                    const T* g = src(arr);
+                    cp_async_16(st + (arr * RP + u) * CW + h * EPC, ok ? (const void*)(g + j * C + c0) : (const void*)g,
+                                (int)ok * (int)sizeof(T));
+                }
+            } else {
+                for (int e = tid; e < na * RP * CW; e += CW) {
+                    const int arr = e / (RP * CW);
+                    const int rem = e - arr * RP * CW;
+                    const int u = rem / CW, h = rem - u * CW;
+                    const int64_t j = p0 + u, c = ch0 + h;
+                    const bool ok = j < L && c < C;
+                    const T* g = src(arr);
+                    if (sizeof(T) == 8) cp_async_8(st + (arr * RP + u) * CW + h, ok ? (const void*)(g + j * C + c) : (const void*)g, ok ? 8 : 0);
+                    else cp_async_4(st + (arr * RP + u) * CW + h, ok ? (const void*)(g + j * C + c) : (const void*)g, ok ? 4 : 0);
+                }
+            }
+        }
+        cp_async_commit();
+    };
+    auto fsrc = [&](int arr) -> const T* {
+        if (MODE == 1) return arr == 0 ? p.a : arr == 1 ? p.b : arr == 2 ? p.c : p.d;
+        return arr == 0 ? p.iA : arr == 1 ? p.iC : p.iD;
+    };
+#pragma unroll 1
+    for (int s = 0; s < PTR_NS - 1; ++s) issue(s, NA, fsrc);
+
+    T th1 = T(1), th2 = T(0), de1 = T(0), Cm = T(0);  // theta_{i-1}, theta_{i-2}, delta_{i-1}, C_{i-1}
+#pragma unroll 1
+    for (int64_t t = 0; t < nst; ++t) {
+        cp_async_wait<PTR_NS - 2>();
+        __syncthreads();
+        issue(t + PTR_NS - 1, NA, fsrc);
+        const T* st = sm + (int)(t % PTR_NS) * STAGE + tid;
+        const int64_t p0 = t * RP;
+        if (active) {
+#pragma unroll 4
+            for (int u = 0; u < RP; ++u) {
+                const int64_t j = p0 + u;
+                if (j >= L) break;
+                T A, Cc, D;
+                if (MODE == 1) {
+                    const T r = rcp(st[(1 * RP + u) * CW]);
+                    A = j > 0 ? st[u * CW] * r : T(0);
+                    Cc = j < L - 1 ? st[(2 * RP + u) * CW] * r : T(0);
+                    D = st[(3 * RP + u) * CW] * r;
+                } else {
+                    A = st[u * CW]; Cc = st[(RP + u) * CW]; D = st[(2 * RP + u) * CW];
+                }
+                const T th = fma(-(A * Cm), th2, th1);
+                const T de = fma(-A, de1, D * th1);
+                const T r = rcp(th);
+                const int64_t idx = j * C + ch;
+                p.cps[idx] = Cc * th1 * r;
+                p.dps[idx] = de * r;
+                th2 = th1; th1 = th; de1 = de; Cm = Cc;
+                const T ath = fabs(th1);
+                if (ath < PTRScale<T>::lo || ath > PTRScale<T>::hi) {
+                    const T f = ath < PTRScale<T>::lo ? PTRScale<T>::up : PTRScale<T>::down;
+                    th1 *= f; th2 *= f; de1 *= f;
+                }
+            }
+        }
+    }
+    // back substitution (Eq 4): stage t' holds positions [hi - RP, hi), hi = L - t' RP
+    cp_async_wait<0>();
+    __syncthreads();
+    __threadfence_block();
+    auto bsrc = [&](int arr) -> const T* { return arr == 0 ? p.cps : p.dps; };
+    auto issue_b = [&](int64_t t) {
+        if (t < nst) {
+            T* st = sm + (int)(t % PTR_NS) * STAGE;
+            const int64_t hi = L - t * RP;
+            if (VEC) {
+                constexpr int CPR = CW / EPC;
+                for (int e = tid; e < 2 * RP * CPR; e += CW) {
+                    const int arr = e / (RP * CPR);
+                    const int rem = e - arr * RP * CPR;
+                    const int u = rem / CPR, h = rem - u * CPR;
+                    const int64_t j = hi - 1 - u, c0 = ch0 + h * EPC;
+                    const int64_t ok = (j >= 0 && c0 < C) ? imin64(EPC, C - c0) : 0;
+                    const T* g = bsrc(arr);
+                    cp_async_16(st + (arr * RP + u) * CW + h * EPC, ok ? (const void*)(g + j * C + c0) : (const void*)g,
+                                (int)ok * (int)sizeof(T));
+                }
+            } else {
+                for (int e = tid; e < 2 * RP * CW; e += CW) {
+                    const int arr = e / (RP * CW);
+                    const int rem = e - arr * RP * CW;
+                    const int u = rem / CW, h = rem - u * CW;
+                    const int64_t j = hi - 1 - u, c = ch0 + h;
+                    const bool ok = j >= 0 && c < C;
+                    const T* g = bsrc(arr);
+                    if (sizeof(T) == 8) cp_async_8(st + (arr * RP + u) * CW + h, ok ? (const void*)(g + j * C + c) : (const void*)g, ok ? 8 : 0);
+                    else cp_async_4(st + (arr * RP + u) * CW + h, ok ? (const void*)(g + j * C + c) : (const void*)g, ok ? 4 : 0);
+                }
+            }
+        }
+        cp_async_commit();
+    };
+#pragma unroll 1
+    for (int s = 0; s < PTR_NS - 1; ++s) issue_b(s);
+    T xv = T(0);
+#pragma unroll 1
+    for (int64_t t = 0; t < nst; ++t) {
+        cp_async_wait<PTR_NS - 2>();
+        __syncthreads();
+        issue_b(t + PTR_NS - 1);
+        const T* st = sm + (int)(t % PTR_NS) * STAGE + tid;
+        const int64_t hi = L - t * RP;
+        if (active) {
+#pragma unroll 4
+            for (int u = 0; u < RP; ++u) {
+                const int64_t j = hi - 1 - u;
+                if (j < 0) break;
+                xv = fma(-st[u * CW], xv, st[(RP + u) * CW]);
+                pt_store_x<T, MODE>(p, ch, j, xv);
+            }
+        }
+    }
+}
+
 }  // namespace tri

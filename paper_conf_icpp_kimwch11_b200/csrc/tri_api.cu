@@ -17,6 +17,7 @@
 #include "k_tiled_pcr.cuh"
 #include "k_pthomas.cuh"
 #include "k_fused.cuh"
+#include "k_warp.cuh"
 
 using namespace tri;
 
@@ -63,7 +64,15 @@ bool fused_ok(int64_t n, int64_t m, tri_layout layout) {
     return (layout == TRI_LAYOUT_CONTIGUOUS || m == 1) && n >= 2 * FU_W;
 }
 
+// WARP: 32 <= n <= 32 x WARP_RMAX rows, one system per warp (registers only).
+constexpr int64_t WARP_RMAX = 32;
+bool warp_ok(int64_t n) { return n >= 32 && n <= 32 * WARP_RMAX; }
+
 tri_variant choose_variant(int64_t n, int64_t m, tri_dtype t, tri_layout layout, int sms) {
+    // one warp per system once the batch covers every SM; below that a whole
+    // CTA per system (ONCHIP) shortens the latency chain (measured: n = 1024,
+    // m = 1: ONCHIP 10 us vs WARP 19 us; m = 1024: WARP 31 us vs ONCHIP 76 us)
+    if (warp_ok(n) && m >= sms) return TRI_VARIANT_WARP;
     if (n <= onchip_rows_budget(t)) return TRI_VARIANT_ONCHIP;
     // paper rule: with more systems than the machine's parallelism go
     // straight to p-Thomas (k = 0); between one system per SM and that point
@@ -84,6 +93,7 @@ int choose_k_for(tri_variant v, int64_t n, int64_t m, tri_dtype t, tri_layout la
         return std::min(k, kmax_n);
     }
     if (v == TRI_VARIANT_FUSED) return FU_K;
+    if (v == TRI_VARIANT_WARP) return WARP_K;
     const int64_t P = (int64_t)sms * 64;
     int k = m >= P ? 0 : ceil_log2(cdiv(P, m));
     return std::min(std::min(k, kmax_n), SPLIT_KMAX);
@@ -92,9 +102,10 @@ int choose_k_for(tri_variant v, int64_t n, int64_t m, tri_dtype t, tri_layout la
 int kmax_for(tri_variant v, int64_t n) {
     const int kn = floor_log2(n);
     if (v == TRI_VARIANT_FUSED) return FU_K;
+    if (v == TRI_VARIANT_WARP) return WARP_K;
     return v == TRI_VARIANT_SPLIT ? std::min(kn, SPLIT_KMAX) : kn;
 }
-int kmin_for(tri_variant v) { return v == TRI_VARIANT_FUSED ? FU_K : 0; }
+int kmin_for(tri_variant v) { return v == TRI_VARIANT_FUSED ? FU_K : v == TRI_VARIANT_WARP ? WARP_K : 0; }
 
 }  // namespace
 
@@ -116,6 +127,7 @@ struct tri_plan_s {
     size_t scratch_bytes;
     void* stage;              // tri_solve_host staging (5 arrays), lazily allocated
     size_t stage_bytes;
+    const void* seen[8];      // pointers whose device residency was last verified
 };
 
 namespace {
@@ -123,6 +135,13 @@ namespace {
 // ---- per-plan geometry -----------------------------------------------------
 void plan_geometry(tri_plan_s* p) {
     const int64_t n = p->n, m = p->m;
+    if (p->variant == TRI_VARIANT_WARP) {
+        int R = 1;
+        while (32 * (int64_t)R < n) R *= 2;
+        p->rpt = R;
+        p->G = 0; p->P = 0; p->n_pad = 32 * (int64_t)R; p->L = R; p->C = m * 32; p->region = 0; p->nreg = 0;
+        return;
+    }
     if (p->variant == TRI_VARIANT_ONCHIP) {
         p->G = onchip_G(n, m, p->dtype, p->sms);
         // pad the per-system smem stride so the p-Thomas walk (lanes = chains,
@@ -237,6 +256,29 @@ cudaError_t launch_onchip(const tri_plan_s* p, const void* a, const void* b, con
 }
 
 template <typename T>
+cudaError_t launch_warp(const tri_plan_s* p, const void* a, const void* b, const void* c, const void* d, void* x,
+                        void* ao, void* co, void* do_, int mode, cudaStream_t st) {
+    WarpArgs<T> A;
+    A.a = (const T*)a; A.b = (const T*)b; A.c = (const T*)c; A.d = (const T*)d;
+    A.x = (T*)x; A.ao = (T*)ao; A.co = (T*)co; A.do_ = (T*)do_;
+    A.n = p->n; A.m = p->m; A.layout = p->layout; A.mode = mode;
+    const bool il = p->layout == TRI_LAYOUT_INTERLEAVED && p->m > 1;
+    const int wpb = il ? WARP_WPB_IL : WARP_WPB;
+    const unsigned grid = (unsigned)cdiv(p->m, wpb);
+#define TRI_WARP_CASE(R)                                                                  \
+    case R:                                                                               \
+        if (il) k_warp<T, R, true><<<grid, wpb * 32, 0, st>>>(A);                         \
+        else k_warp<T, R, false><<<grid, wpb * 32, 0, st>>>(A);                           \
+        break;
+    switch (p->rpt) {
+        TRI_WARP_CASE(1) TRI_WARP_CASE(2) TRI_WARP_CASE(4) TRI_WARP_CASE(8) TRI_WARP_CASE(16) TRI_WARP_CASE(32)
+        default: return cudaErrorInvalidValue;
+    }
+#undef TRI_WARP_CASE
+    return cudaGetLastError();
+}
+
+template <typename T>
 cudaError_t launch_tiled(const tri_plan_s* p, const void* a, const void* b, const void* c, const void* d,
                          void* oA, void* oC, void* oD, int mode, cudaStream_t st) {
     TiledArgs<T> A;
@@ -314,12 +356,15 @@ cudaError_t launch_split(const tri_plan_s* p, const void* a, const void* b, cons
     return cudaGetLastError();
 }
 
-tri_status check_ptrs(const tri_plan_s* p, const void* const* in, int nin, const void* const* out, int nout) {
+tri_status check_ptrs(tri_plan_s* p, const void* const* in, int nin, const void* const* out, int nout) {
     const size_t bytes = (size_t)p->n * (size_t)p->m * esize(p->dtype);
+    bool same = nin + nout <= 8;
+    for (int i = 0; i < nin + nout && same; ++i) same = p->seen[i] == (i < nin ? in[i] : out[i - nin]);
     for (int i = 0; i < nin + nout; ++i) {
         const void* q = i < nin ? in[i] : out[i - nin];
         if (!q) return TRI_ERR_INVALID_ARG;
         if (((uintptr_t)q & 15) != 0) return TRI_ERR_ALIGNMENT;
+        if (same) continue;  // residency verified on the previous call with these pointers
         cudaPointerAttributes at;
         if (cudaPointerGetAttributes(&at, q) != cudaSuccess) { cudaGetLastError(); return TRI_ERR_DEVICE; }
         if ((at.type != cudaMemoryTypeDevice && at.type != cudaMemoryTypeManaged) || at.device != p->device)
@@ -335,6 +380,9 @@ tri_status check_ptrs(const tri_plan_s* p, const void* const* in, int nin, const
             const uintptr_t y0 = (uintptr_t)out[o2], y1 = y0 + bytes;
             if (x0 < y1 && y0 < x1) return TRI_ERR_ALIAS;
         }
+    }
+    if (!same && nin + nout <= 8) {
+        for (int i = 0; i < 8; ++i) p->seen[i] = i < nin + nout ? (i < nin ? in[i] : out[i - nin]) : nullptr;
     }
     return TRI_OK;
 }
@@ -458,7 +506,9 @@ tri_status tri_plan_set_variant(tri_plan_t p, tri_variant v) {
     if (v == TRI_VARIANT_AUTO) v = choose_variant(p->n, p->m, p->dtype, p->layout, p->sms);
     if (v == TRI_VARIANT_ONCHIP && p->n > onchip_rows_budget(p->dtype)) return TRI_ERR_INVALID_ARG;
     if (v == TRI_VARIANT_FUSED && !fused_ok(p->n, p->m, p->layout)) return TRI_ERR_INVALID_ARG;
-    if (v != TRI_VARIANT_ONCHIP && v != TRI_VARIANT_SPLIT && v != TRI_VARIANT_FUSED) return TRI_ERR_INVALID_ARG;
+    if (v == TRI_VARIANT_WARP && !warp_ok(p->n)) return TRI_ERR_INVALID_ARG;
+    if (v != TRI_VARIANT_ONCHIP && v != TRI_VARIANT_SPLIT && v != TRI_VARIANT_FUSED && v != TRI_VARIANT_WARP)
+        return TRI_ERR_INVALID_ARG;
     const tri_variant ov = p->variant;
     const int ok = p->k;
     p->variant = v;
@@ -472,7 +522,7 @@ tri_status tri_plan_set_variant(tri_plan_t p, tri_variant v) {
 void tri_plan_describe(tri_plan_t p, char* buf, int len) {
     if (!buf || len <= 0) return;
     if (!p) { snprintf(buf, len, "null plan"); return; }
-    static const char* vn[] = {"auto", "onchip", "split", "fused"};
+    static const char* vn[] = {"auto", "onchip", "split", "fused", "warp"};
     snprintf(buf, len,
              "n=%lld m=%lld dtype=%s layout=%s variant=%s k=%d G=%d P=%d rpt=%d L=%lld C=%lld region=%lld nreg=%lld "
              "fu_grid=%d fu_son=%d fu_nc=%lld scratch=%zu sms=%d",
@@ -491,7 +541,10 @@ tri_status tri_solve(tri_plan_t p, const void* a, const void* b, const void* c, 
     if (st != TRI_OK) return st;
     cudaStream_t s = (cudaStream_t)stream;
     cudaError_t e;
-    if (p->variant == TRI_VARIANT_ONCHIP) {
+    if (p->variant == TRI_VARIANT_WARP) {
+        e = p->dtype == TRI_F64 ? launch_warp<double>(p, a, b, c, d, x, nullptr, nullptr, nullptr, 0, s)
+                                : launch_warp<float>(p, a, b, c, d, x, nullptr, nullptr, nullptr, 0, s);
+    } else if (p->variant == TRI_VARIANT_ONCHIP) {
         e = p->dtype == TRI_F64 ? launch_onchip<double>(p, a, b, c, d, x, nullptr, nullptr, nullptr, 0, s)
                                 : launch_onchip<float>(p, a, b, c, d, x, nullptr, nullptr, nullptr, 0, s);
     } else if (p->variant == TRI_VARIANT_FUSED) {
@@ -511,7 +564,10 @@ tri_status tri_debug_pcr(tri_plan_t p, const void* a, const void* b, const void*
     if (st != TRI_OK) return st;
     cudaStream_t s = (cudaStream_t)stream;
     cudaError_t e;
-    if (p->variant == TRI_VARIANT_ONCHIP) {
+    if (p->variant == TRI_VARIANT_WARP) {
+        e = p->dtype == TRI_F64 ? launch_warp<double>(p, a, b, c, d, nullptr, ao, co, do_, 1, s)
+                                : launch_warp<float>(p, a, b, c, d, nullptr, ao, co, do_, 1, s);
+    } else if (p->variant == TRI_VARIANT_ONCHIP) {
         e = p->dtype == TRI_F64 ? launch_onchip<double>(p, a, b, c, d, nullptr, ao, co, do_, 1, s)
                                 : launch_onchip<float>(p, a, b, c, d, nullptr, ao, co, do_, 1, s);
     } else if (p->variant == TRI_VARIANT_FUSED) {

@@ -34,3 +34,20 @@ e.record()
 torch.cuda.synchronize()
 ms = s.elapsed_time(e)
 print(f"time {ms:.3f} ms  {n * m / ms / 1e3:.1f} Munk/s  {5 * n * m * b.element_size() / ms / 1e6:.1f} GB/s(5 arrays)")
+if os.environ.get("PROF_GRAPH", "1") == "1":
+    # device-only time: the solve captured in a CUDA graph, replayed back to back
+    stream = torch.cuda.Stream()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=stream):
+        plan.solve(a, b, c, d, out=x, stream=stream)
+    reps = max(3, min(200, int(2e9 / max(1, n * m * b.element_size() * 5))))
+    g.replay()
+    torch.cuda.synchronize()
+    s.record()
+    for _ in range(reps):
+        g.replay()
+    e.record()
+    torch.cuda.synchronize()
+    ms = s.elapsed_time(e) / reps
+    print(f"graph {ms * 1e3:.1f} us  {n * m / ms / 1e3:.1f} Munk/s  "
+          f"{5 * n * m * b.element_size() / ms / 1e6:.1f} GB/s(5 arrays)  reps={reps}")

@@ -85,7 +85,7 @@ def test_heuristic_k_valid_and_nonincreasing_in_m(L, dtype, layout, n):
     for m in [1, 2, 16, 32, 100, 512, 1024, 4096, 16384, 1 << 20]:
         k = tri.choose_k(n, m, dtype, layout, 148)
         v = tri.choose_variant(n, m, dtype, layout, 148)
-        assert v in (tri.VARIANT_ONCHIP, tri.VARIANT_SPLIT, tri.VARIANT_FUSED)
+        assert v in (tri.VARIANT_ONCHIP, tri.VARIANT_SPLIT, tri.VARIANT_FUSED, tri.VARIANT_WARP)
         assert 0 <= k <= max(0, n.bit_length() - 1)
         if prev is not None:
             assert k <= prev[0], (n, m, k, prev)

@@ -12,7 +12,7 @@ from tests._helpers import check_parity, gen, gpu_solve, to_dev
 pytestmark = pytest.mark.gpu
 
 tri = pytest.importorskip("paper_conf_icpp_kimwch11_b200")
-ONCHIP, SPLIT = tri.VARIANT_ONCHIP, tri.VARIANT_SPLIT
+ONCHIP, SPLIT, WARP = tri.VARIANT_ONCHIP, tri.VARIANT_SPLIT, tri.VARIANT_WARP
 
 
 # ------------------------------------------------------------------ auto plan
@@ -80,6 +80,7 @@ def test_split_on_small_systems(cuda_ok):
 
 # ------------------------------------------------------------------ PCR stage (row A2)
 @pytest.mark.parametrize("variant,n,m,k", [(ONCHIP, 1024, 3, 3), (ONCHIP, 500, 2, 5), (SPLIT, 9000, 2, 4),
+                                           (WARP, 1000, 3, 5), (WARP, 33, 2, 5), (WARP, 256, 4, 5),
                                            (SPLIT, 20001, 1, 8), (SPLIT, 5000, 3, 1)])
 def test_pcr_stage_matches_oracle(cuda_ok, variant, n, m, k):
     """The reduced system after k PCR steps (Eqs 5-6) vs the oracle's plain PCR,
@@ -106,7 +107,8 @@ def test_pcr_stage_matches_oracle(cuda_ok, variant, n, m, k):
 
 
 # ------------------------------------------------------------------ edge cases / API
-@pytest.mark.parametrize("variant,n,m", [(ONCHIP, 1024, 4), (SPLIT, 9000, 2), (SPLIT, 3000, 130)])
+@pytest.mark.parametrize("variant,n,m", [(ONCHIP, 1024, 4), (SPLIT, 9000, 2), (SPLIT, 3000, 130), (WARP, 1000, 5),
+                                         (WARP, 64, 9)])
 @pytest.mark.parametrize("layout", [0, 1])
 def test_ignored_entries_nan(cuda_ok, variant, n, m, layout):
     """a[q][0] and c[q][n-1] lie outside A (Eq 1, reading X1): NaN there must
@@ -295,3 +297,58 @@ def test_fused_edges_and_scaling(cuda_ok):
     assert torch.equal(x3, x1 * 4.0)
     with pytest.raises(tri.TriError):
         plan.k = 2  # the fused kernel is built for one k
+
+
+# ------------------------------------------------------------------ WARP variant
+@pytest.mark.parametrize("dtype", ["f64", "f32"])
+@pytest.mark.parametrize("layout", [0, 1])
+@pytest.mark.parametrize("n,m", [(32, 5), (33, 4), (63, 7), (64, 1), (100, 9), (128, 33), (200, 3), (256, 130),
+                                 (511, 2), (512, 5), (700, 3), (1023, 4), (1024, 7)])
+def test_warp_parity(cuda_ok, dtype, layout, n, m):
+    """One warp per system (forced; auto picks WARP only when m >= #SMs), every
+    register-slot count R = 1..32 and ragged n."""
+    arrs = gen(n, m, dtype, layout, "weak", eps=1e-2)
+    x, plan = gpu_solve(n, m, arrs, dtype, layout, variant=WARP)
+    assert plan.variant == WARP and plan.k == 5
+    check_parity(n, m, arrs, x, dtype, layout)
+
+
+@pytest.mark.parametrize("family,eps", [("dd", 0.0), ("weak", 1e-3), ("integer", 0.0)])
+def test_warp_families(cuda_ok, family, eps):
+    n, m = 1000, 20
+    arrs = gen(n, m, "f64", 0, family, eps=eps)
+    x, plan = gpu_solve(n, m, arrs, "f64", 0, variant=WARP)
+    check_parity(n, m, arrs, x, "f64", 0)
+
+
+def test_warp_large_batch_sampled(cuda_ok):
+    """c4-shaped batch (n = 256, fp32, m = 2^18): sampled systems vs the oracle."""
+    n, m = 256, 1 << 18
+    arrs = gen(n, m, "f32", 0)
+    x, plan = gpu_solve(n, m, arrs, "f32", 0)
+    assert plan.variant == WARP
+    rng = np.random.default_rng(5)
+    for q in rng.choice(m, 64, replace=False).tolist() + [0, m - 1]:
+        sl = slice(q * n, (q + 1) * n)
+        sub = [t[sl] for t in arrs]
+        check_parity(n, 1, sub, x[sl], "f32", 0)
+
+
+@pytest.mark.parametrize("variant,n,m", [(WARP, 1000, 4), (ONCHIP, 2000, 3), (SPLIT, 5000, 2)])
+def test_poisson_closed_form(cuda_ok, variant, n, m):
+    """The [-1, 2, -1] Poisson system (only weakly dominant, cond ~ n^2, so the
+    elementwise dd tolerance does not apply): normwise error against the
+    manufactured exact solution within cond * eps, and the residual gate."""
+    import trigen
+    a, b, c, d, xs = trigen.generate(n, m, "f64", 0, "poisson", want_xstar=True)
+    x, plan = gpu_solve(n, m, (a, b, c, d), "f64", 0, variant=variant)
+    assert plan.variant == variant
+    cond = (n + 1) ** 2 / 2.0  # ||A||_inf ||A^-1||_inf bound for the 1-D Laplacian
+    for q in range(m):
+        sl = slice(q * n, (q + 1) * n)
+        err = np.max(np.abs(x[sl] - xs[sl])) / np.max(np.abs(xs[sl]))
+        assert err <= 64 * cond * np.finfo(np.float64).eps, err
+    # ||Ax - d|| / ||d|| is ~cond * eps here, so gate the normwise backward error
+    # ||Ax - d|| / (||A|| ||x|| + ||d||) instead
+    r = oracle.residual_batch(n, m, a, b, c, d, x, layout=0)
+    assert r[:, 1].max() <= 1e-14
