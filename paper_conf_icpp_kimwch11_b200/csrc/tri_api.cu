@@ -4,6 +4,7 @@
 //
 // Build: nvcc -gencode arch=compute_100a,code=sm_100a -shared (see _build.py).
 #include <cuda_runtime.h>
+#include <cudaTypedefs.h>
 
 #include <algorithm>
 #include <cstdint>
@@ -18,6 +19,7 @@
 #include "k_pthomas.cuh"
 #include "k_fused.cuh"
 #include "k_warp.cuh"
+#include "k_pthomas_tma.cuh"
 
 using namespace tri;
 
@@ -315,6 +317,59 @@ cudaError_t launch_fused(const tri_plan_s* p, const void* a, const void* b, cons
     return cudaGetLastError();
 }
 
+// ---- TMA tensor maps (cuTensorMapEncodeTiled through the runtime's driver
+// entry point: no link-time dependency on libcuda)
+PFN_cuTensorMapEncodeTiled_v12000 tma_encoder() {
+    static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+    static bool tried = false;
+    if (!tried) {
+        tried = true;
+        void* f = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = (PFN_cuTensorMapEncodeTiled_v12000)f;
+        else
+            cudaGetLastError();
+    }
+    return fn;
+}
+
+template <typename T>
+bool tma_map_2d(CUtensorMap* tm, const void* base, uint64_t d0, uint64_t d1, uint32_t b0, uint32_t b1, bool swz) {
+    auto enc = tma_encoder();
+    if (!enc) return false;
+    cuuint64_t dims[2] = {d0, d1};
+    cuuint64_t strides[1] = {d0 * sizeof(T)};
+    cuuint32_t box[2] = {b0, b1};
+    cuuint32_t es[2] = {1, 1};
+    return enc(tm, sizeof(T) == 8 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT64 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2,
+               const_cast<void*>(base), dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+               swz ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+// k = 0, CONTIGUOUS: the TMA kernel when both row strides (n and m elements)
+// are 16-byte multiples; returns cudaErrorNotSupported to request the fallback.
+template <typename T>
+cudaError_t launch_contig_tma(const tri_plan_s* p, const PThomasArgs<T>& A, cudaStream_t st) {
+    constexpr int R = PTTCfg<T>::R;
+    if ((p->n * (int64_t)sizeof(T)) % 16 || (p->m * (int64_t)sizeof(T)) % 16) return cudaErrorNotSupported;
+    if (p->n > INT32_MAX || p->m > INT32_MAX) return cudaErrorNotSupported;
+    PTTMaps tm;
+    const uint64_t n = (uint64_t)p->n, m = (uint64_t)p->m;
+    bool ok = tma_map_2d<T>(&tm.a, A.a, n, m, R, PTT_CH, true) && tma_map_2d<T>(&tm.b, A.b, n, m, R, PTT_CH, true) &&
+              tma_map_2d<T>(&tm.c, A.c, n, m, R, PTT_CH, true) && tma_map_2d<T>(&tm.d, A.d, n, m, R, PTT_CH, true) &&
+              tma_map_2d<T>(&tm.x, A.x, n, m, R, PTT_CH, true) &&
+              tma_map_2d<T>(&tm.cp, A.cps, m, n, PTT_CH, R, false) && tma_map_2d<T>(&tm.dp, A.dps, m, n, PTT_CH, R, false);
+    if (!ok) return cudaErrorNotSupported;
+    constexpr int smem = ptt_smem_bytes<T>();
+    cudaError_t e = cudaFuncSetAttribute(k_pthomas_tma<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e != cudaSuccess) return e;
+    k_pthomas_tma<T><<<(unsigned)cdiv(p->m, PTT_CH), PTT_CH, smem, st>>>(tm, A);
+    return cudaGetLastError();
+}
+
 template <typename T, int CH>
 cudaError_t launch_contig(const tri_plan_s* p, const PThomasArgs<T>& A, bool vec, cudaStream_t st) {
     constexpr int smem = pt2_smem_bytes<T, CH>();
@@ -323,6 +378,34 @@ cudaError_t launch_contig(const tri_plan_s* p, const PThomasArgs<T>& A, bool vec
     if (e != cudaSuccess) return e;
     kern<<<(unsigned)cdiv(p->m, CH), CH, smem, st>>>(A);
     return cudaGetLastError();
+}
+
+// p-Thomas over chain-interleaved input (MODE 0 scratch, MODE 1 user
+// INTERLEAVED).  Few chains (< 8 warps' worth per SM): the ring-staged kernel
+// with CW chains per CTA, CW the largest of 32/16/8 that still gives every SM
+// a CTA; many chains: one thread per chain with a register prefetch window.
+template <typename T, int CW, int MODE>
+cudaError_t launch_ring(const tri_plan_s* p, const PThomasArgs<T>& A, bool vec, cudaStream_t st) {
+    const int smem = ptr_smem_bytes<T, CW>(MODE == 1);
+    auto kern = vec ? k_pthomas_ring<T, CW, MODE, true> : k_pthomas_ring<T, CW, MODE, false>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e != cudaSuccess) return e;
+    kern<<<(unsigned)cdiv(p->C, CW), CW, smem, st>>>(A);
+    return cudaGetLastError();
+}
+
+template <typename T, int MODE>
+cudaError_t launch_pthomas_il(const tri_plan_s* p, const PThomasArgs<T>& A, cudaStream_t st) {
+    const int64_t C = p->C, sms = p->sms;
+    if (C >= 32 * 8 * sms) {
+        k_pthomas<T, MODE><<<(unsigned)cdiv(C, 128), 128, 0, st>>>(A);
+        return cudaGetLastError();
+    }
+    const T* in0 = MODE == 1 ? A.a : A.iA;
+    const bool vec = ((C * (int64_t)sizeof(T)) % 16) == 0 && ((uintptr_t)in0 % 16) == 0;
+    if (C >= 32 * sms) return launch_ring<T, 32, MODE>(p, A, vec, st);
+    if (C >= 16 * sms) return launch_ring<T, 16, MODE>(p, A, vec, st);
+    return launch_ring<T, 8, MODE>(p, A, vec, st);
 }
 
 template <typename T>
@@ -340,13 +423,17 @@ cudaError_t launch_split(const tri_plan_s* p, const void* a, const void* b, cons
         if (e != cudaSuccess) return e;
         A.iA = rA; A.iC = rC; A.iD = rD;
         A.cps = base + 3 * ce; A.dps = base + 4 * ce;
-        k_pthomas<T, 0><<<(unsigned)cdiv(p->C, 128), 128, 0, st>>>(A);
+        return launch_pthomas_il<T, 0>(p, A, st);
     } else {
         A.iA = A.iC = A.iD = nullptr;
         A.cps = base; A.dps = base + ce;
         if (p->layout == TRI_LAYOUT_INTERLEAVED) {
-            k_pthomas<T, 1><<<(unsigned)cdiv(p->C, 128), 128, 0, st>>>(A);
+            return launch_pthomas_il<T, 1>(p, A, st);
         } else {
+            if (!getenv("TRI_NO_TMA")) {
+                const cudaError_t et = launch_contig_tma<T>(p, A, st);
+                if (et != cudaErrorNotSupported) return et;
+            }
             const bool vec = ((p->n * (int64_t)sizeof(T)) % 16) == 0 && ((uintptr_t)a % 16) == 0;
             // 16 systems per CTA when the batch is thin (finer balance over the SMs)
             const bool thin = cdiv(p->m, 32) < 6 * (int64_t)p->sms;

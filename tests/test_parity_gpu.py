@@ -352,3 +352,25 @@ def test_poisson_closed_form(cuda_ok, variant, n, m):
     # ||Ax - d|| / (||A|| ||x|| + ||d||) instead
     r = oracle.residual_batch(n, m, a, b, c, d, x, layout=0)
     assert r[:, 1].max() <= 1e-14
+
+
+# ------------------------------------------------------------------ k = 0 contiguous, TMA path
+@pytest.mark.parametrize("dtype,n,m", [("f64", 2, 32), ("f64", 16, 32), ("f64", 1000, 70), ("f64", 20000, 64),
+                                       ("f64", 4096, 130), ("f32", 1000, 68), ("f32", 32, 4), ("f32", 5000, 100)])
+def test_split_k0_tma(cuda_ok, dtype, n, m):
+    """k = 0 on the contiguous layout through the TMA kernel (row strides are
+    16-byte multiples): ragged last tile (n % R != 0), ragged last warp (m % 32
+    != 0), one-tile systems; bitwise equal to the cp.async kernel (same
+    arithmetic in the same order)."""
+    import os
+    import torch
+    arrs = gen(n, m, dtype, 0, "weak", eps=1e-2)
+    x, plan = gpu_solve(n, m, arrs, dtype, 0, k=0, variant=SPLIT)
+    check_parity(n, m, arrs, x, dtype, 0)
+    os.environ["TRI_NO_TMA"] = "1"
+    try:
+        x2 = plan.solve(*to_dev(*arrs)).cpu().numpy()
+    finally:
+        del os.environ["TRI_NO_TMA"]
+    assert np.array_equal(x, x2)
+    torch.cuda.synchronize()
