@@ -57,6 +57,7 @@ def parse():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-check", action="store_true")
     ap.add_argument("--no-graph", action="store_true", help="time direct solve calls instead of graph replays")
+    ap.add_argument("--no-collectives", action="store_true", help="N > 1: skip the scatter/gather measurement")
     return ap.parse_args()
 
 
@@ -124,6 +125,50 @@ def dist_env():
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
     return world, rank, local
+
+
+def method_arrays(plan, tri):
+    """Arrays of n*m*s bytes the plan's method moves per solve:
+    compulsory 5 + every materialised PCR pass + spilled Thomas intermediates."""
+    v = plan.variant
+    if v in (tri.VARIANT_WARP, tri.VARIANT_ONCHIP):
+        return 5
+    if v == tri.VARIANT_FUSED:
+        return 5  # c', d' of the first L - S_on positions go to per-CTA scratch that stays in L2
+    if plan.k == 0:
+        return 9  # read a, b, c, d; write + read c', d'; write x
+    # pass 1: read 4 + write 3; [pass 2: read 3 + write 3]; p-Thomas: read 3, c', d' 2 + 2, write x
+    return 15 if plan.launches == 2 else 21
+
+
+def time_collectives(n, m, s, world, rank, dev, tdt):
+    """NCCL edge collectives of SURVEY 8(e): rank 0 scatters a, b, c, d shards
+    and gathers x.  Returns (scatter ms, gather ms, bytes crossing NVLink), max
+    over ranks (CUDA events)."""
+    import torch
+    import torch.distributed as dist
+    per = -(-m // world)
+    recv = torch.empty(n * per, dtype=tdt, device=dev)
+    send = [torch.empty(n * per, dtype=tdt, device=dev) for _ in range(world)] if rank == 0 else None
+    res = []
+    for what in ("scatter", "gather"):
+        for it in range(2):  # one warm-up round
+            dist.barrier()
+            torch.cuda.synchronize()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            for _ in range(4 if what == "scatter" else 1):
+                if what == "scatter":
+                    dist.scatter(recv, scatter_list=send, src=0)
+                else:
+                    dist.gather(recv, gather_list=send, dst=0)
+            e1.record()
+            torch.cuda.synchronize()
+        t = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        res.append(float(t.item()))
+    moved = (world - 1) * n * per * s
+    return res[0], res[1], 4 * moved, moved
 
 
 def cpu_oracle_time(n, mr, arrs, layout, budget_s=20.0):
@@ -315,6 +360,20 @@ def main():
                "how": "tri_solve_host: pinned host a,b,c,d -> device, solve, x -> pinned host, per step"}
         del xh
 
+    # ---- edge collectives (N > 1): scatter of the input shards, gather of x
+    coll = None
+    if world > 1 and not args.no_collectives:
+        try:
+            t_sc, t_ga, b_sc, b_ga = time_collectives(n, m_all, s, world, rank, dev, tdt)
+        except Exception as exc:  # never let the edge measurement cost the solve numbers
+            t_sc = None
+            coll = {"error": repr(exc)[:200]}
+    if coll is None and world > 1 and not args.no_collectives and t_sc is not None:
+        coll = {"scatter_ms": t_sc, "gather_ms": t_ga, "scatter_bytes": b_sc, "gather_bytes": b_ga,
+                "scatter_gbs": b_sc / (t_sc * 1e-3) / 1e9, "gather_gbs": b_ga / (t_ga * 1e-3) / 1e9,
+                "how": "NCCL dist.scatter (4 arrays) / dist.gather (x) from/to rank 0, CUDA events, max over ranks; "
+                       "not part of the timed solve (shards are resident)"}
+
     # ---- CPU oracle baseline (rank 0 at N=1 only)
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu:
@@ -326,6 +385,8 @@ def main():
     peak, peak_src = measured_peaks()
     algo_bytes = 5 * n_unknowns * s          # compulsory 5 arrays per unknown
     achieved = algo_bytes / (t_step * 1e-3) / 1e9
+    marr = method_arrays(plan, tri)
+    method_bytes = marr * n_unknowns * s
     traffic = None
     tf = os.path.join(ROOT, "profiles", f"traffic_{args.config}.json")
     if os.path.exists(tf):
@@ -346,11 +407,15 @@ def main():
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                      "traffic": traffic, "peak_source": peak_src,
                      "algorithmic_bytes_per_launch": algo_bytes,
+                     "method_arrays": marr, "method_bytes_per_launch": method_bytes,
+                     "method_frac": method_bytes / (t_step * 1e-3) / 1e9 / peak,
+                     "excess_traffic": (traffic / method_bytes) if traffic else None,
                      "kernel": "whole solve (%d launch%s)" % (plan.launches, "" if plan.launches == 1 else "es")},
         "clocks": clk.summary(),
         "e2e": e2e,
         "gpu_launches": args.steps * plan.launches,
         "cpu_baseline": cpu,
+        "collectives": coll,
         "parity": parity,
         "step_ms_min": min(step_ms), "step_ms_median": statistics.median(step_ms),
     }

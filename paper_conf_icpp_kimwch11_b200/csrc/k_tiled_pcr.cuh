@@ -58,20 +58,31 @@ __global__ void __launch_bounds__(TPCR_T) k_tiled_pcr(TiledArgs<T> p) {
     for (int e = tid; e < p.ring_total; e += TPCR_T) { rA[e] = T(0); rC[e] = T(0); rD[e] = T(0); }
     __syncthreads();
 
+    // level-0 rows of the next sub-tile are loaded into registers while the
+    // current sub-tile's levels run (hides the HBM latency behind the ring work)
+    T pa = T(0), pb = T(1), pc = T(0), pd = T(0);
+    auto fetch = [&](int64_t s0) {
+        const int64_t i = s0 + tid;
+        pa = T(0); pb = T(1); pc = T(0); pd = T(0);
+        if (i >= 0 && i < n) {
+            const int64_t gi = elem_index(q, i, n, p.m, p.layout);
+            pa = i > 0 ? ldg_stream(p.a + gi) : T(0);
+            pc = i < n - 1 ? ldg_stream(p.c + gi) : T(0);
+            pb = ldg_stream(p.b + gi);
+            pd = ldg_stream(p.d + gi);
+        }
+    };
+    fetch(start);
     for (int64_t s0 = start; s0 - fk < r1; s0 += TPCR_T) {
-        // level 0: load + normalise one row per thread
+        // level 0: normalise this thread's (prefetched) row; rows outside the
+        // system are identity rows (b = 1, a = c = d = 0)
         {
             const int64_t i = s0 + tid;
-            NRow<T> r = identity_row<T>();
-            if (i >= 0 && i < n) {
-                const int64_t gi = elem_index(q, i, n, p.m, p.layout);
-                T av = i > 0 ? ldg_stream(p.a + gi) : T(0);
-                T cv = i < n - 1 ? ldg_stream(p.c + gi) : T(0);
-                r = normalise(av, ldg_stream(p.b + gi), cv, ldg_stream(p.d + gi));
-            }
+            const NRow<T> r = normalise(pa, pb, pc, pd);
             const int s = p.ring_off[0] + (int)(i & p.ring_mask[0]);
             rA[s] = r.A; rC[s] = r.C; rD[s] = r.D;
         }
+        fetch(s0 + TPCR_T);
         __syncthreads();
         int64_t F = s0 + TPCR_T;  // level-j frontier (exclusive)
         for (int j = 0; j < p.k; ++j) {
@@ -94,6 +105,105 @@ __global__ void __launch_bounds__(TPCR_T) k_tiled_pcr(TiledArgs<T> p) {
                 } else if (i < n) {
                     const int64_t gi = elem_index(q, i, n, p.m, p.layout);
                     p.oA[gi] = nr.A; p.oC[gi] = nr.C; p.oD[gi] = nr.D;
+                }
+            }
+            __syncthreads();
+        }
+    }
+}
+
+
+// ---------------------------------------------------------------------------
+// Second tiled-PCR pass (deep k, two passes): the chain-interleaved output of
+// a k1-step pass is itself a batch of C1 = m 2^k1 independent systems in the
+// INTERLEAVED layout (position pos of chain ch at [pos * C1 + ch]).  This pass
+// applies k2 more steps (strides 2^k1 .. 2^(k1+k2-1) of the original system =
+// strides 1 .. 2^(k2-1) in each chain's positions) with the same buffered
+// sliding window, over TPCR_IL_CB adjacent chains per CTA so every position row
+// is one 256-byte segment.  Its output is the layout a single k1 + k2 pass would
+// store: chain ch2 = q 2^k + (r1 + 2^k1 (pos mod 2^k2)), position pos >> k2.
+constexpr int TPCR_IL_CB = 32;                     // chains per CTA
+constexpr int TPCR_IL_TP = TPCR_T / TPCR_IL_CB;    // positions per sub-tile
+
+template <typename T>
+struct TiledILArgs {
+    const T *iA, *iC, *iD;  // pass-1 output, [pos * C1 + ch], normalised rows
+    T *oA, *oC, *oD;        // mode 0: chain-interleaved [pos2 * C + ch2]; mode 1: user layout
+    int64_t n, m, L1, C1, C, region, nreg, nblk;
+    int layout, k1, k2, mode;
+    int ring_off[8];        // position offset of level j's ring
+    int ring_mask[8];
+    int ring_total;         // positions across all rings
+};
+
+template <typename T>
+__global__ void __launch_bounds__(TPCR_T) k_tiled_pcr_il(TiledILArgs<T> p) {
+    constexpr int CB = TPCR_IL_CB, TP = TPCR_IL_TP;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    T* rA = reinterpret_cast<T*>(smem_raw);
+    T* rC = rA + p.ring_total * CB;
+    T* rD = rC + p.ring_total * CB;
+
+    const int tid = threadIdx.x;
+    const int c = tid % CB, u = tid / CB;
+    const int64_t blk = blockIdx.x % p.nblk, reg = blockIdx.x / p.nblk;
+    const int64_t ch = blk * CB + c;
+    const bool chok = ch < p.C1;
+    const int64_t r0 = reg * p.region;
+    const int64_t r1 = imin64(r0 + p.region, p.L1);
+    const int64_t fk = halo_f(p.k2);
+    const int64_t start = r0 - fk;
+    const int k = p.k1 + p.k2;
+    const int64_t S1 = int64_t(1) << p.k1;
+    const int64_t q = ch >> p.k1, rr1 = ch & (S1 - 1);
+
+    for (int e = tid; e < p.ring_total * CB; e += TPCR_T) { rA[e] = T(0); rC[e] = T(0); rD[e] = T(0); }
+    __syncthreads();
+
+    NRow<T> nxt;  // next sub-tile's level-0 row, loaded during this sub-tile's levels
+    auto fetch = [&](int64_t s0) {
+        const int64_t pos = s0 + u;
+        nxt = identity_row<T>();
+        if (pos >= 0 && pos < p.L1 && chok) {
+            const int64_t gi = pos * p.C1 + ch;
+            nxt = NRow<T>{ldg_stream(p.iA + gi), ldg_stream(p.iC + gi), ldg_stream(p.iD + gi)};
+        }
+    };
+    fetch(start);
+    for (int64_t s0 = start; s0 - fk < r1; s0 += TP) {
+        {
+            const int64_t pos = s0 + u;
+            const int sl = (p.ring_off[0] + (int)(pos & p.ring_mask[0])) * CB + c;
+            rA[sl] = nxt.A; rC[sl] = nxt.C; rD[sl] = nxt.D;
+        }
+        fetch(s0 + TP);
+        __syncthreads();
+        int64_t F = s0 + TP;
+        for (int j = 0; j < p.k2; ++j) {
+            const int sg = 1 << j;
+            F -= sg;
+            const int64_t pos = F - TP + u;
+            const int off = p.ring_off[j], msk = p.ring_mask[j];
+            const int so = (off + (int)(pos & msk)) * CB + c;
+            const int sm = (off + (int)((pos - sg) & msk)) * CB + c;
+            const int sp = (off + (int)((pos + sg) & msk)) * CB + c;
+            const NRow<T> nr = pcr_combine(NRow<T>{rA[sm], rC[sm], rD[sm]}, NRow<T>{rA[so], rC[so], rD[so]},
+                                           NRow<T>{rA[sp], rC[sp], rD[sp]});
+            if (j + 1 < p.k2) {
+                const int sd = (p.ring_off[j + 1] + (int)(pos & p.ring_mask[j + 1])) * CB + c;
+                rA[sd] = nr.A; rC[sd] = nr.C; rD[sd] = nr.D;
+            } else if (pos >= r0 && pos < r1 && chok) {
+                const int64_t r = rr1 + ((pos & ((int64_t(1) << p.k2) - 1)) << p.k1);  // residue mod 2^k
+                const int64_t pos2 = pos >> p.k2;
+                if (p.mode == 0) {
+                    const int64_t idx = pos2 * p.C + (q << k) + r;
+                    p.oA[idx] = nr.A; p.oC[idx] = nr.C; p.oD[idx] = nr.D;
+                } else {
+                    const int64_t i = (pos2 << k) + r;
+                    if (i < p.n) {
+                        const int64_t gi = elem_index(q, i, p.n, p.m, p.layout);
+                        p.oA[gi] = nr.A; p.oC[gi] = nr.C; p.oD[gi] = nr.D;
+                    }
                 }
             }
             __syncthreads();

@@ -30,7 +30,9 @@ void* g_fused_prof = nullptr;  // tri_debug_set_profile: device counters for the
 int g_fused_dbg_mode = 0;     // TRI_FUSED_DBG_MODE (diagnostics only)
 
 constexpr int ONCHIP_THREADS = 512;
-constexpr int SPLIT_KMAX = 10;  // deepest k one sliding-window pass holds in smem (T = 256)
+constexpr int SPLIT_K1MAX = 10;  // deepest k one sliding-window pass holds in smem (T = 256)
+constexpr int SPLIT_K2MAX = 5;   // steps of the second (interleaved-batch) pass
+constexpr int SPLIT_KMAX = SPLIT_K1MAX + SPLIT_K2MAX;
 constexpr int64_t MAX_ELEMS = int64_t(1) << 40;
 
 int floor_log2(int64_t v) {
@@ -120,7 +122,10 @@ struct tri_plan_s {
     tri_variant variant;
     int G, P, rpt;            // ONCHIP geometry
     int64_t n_pad, L, C;      // SPLIT: chain length, chains
-    int64_t region, nreg;     // SPLIT: tiled-PCR regions per system
+    int64_t region, nreg;     // SPLIT: tiled-PCR regions per system (pass 1)
+    int k1;                   // SPLIT: steps of pass 1 (k - k1 in pass 2)
+    int64_t L1, C1;           // SPLIT: pass-1 positions per chain, chains
+    int64_t region2, nreg2, nblk2;  // SPLIT pass 2: positions per region, regions, chain blocks
     int fu_grid, fu_son;      // FUSED: persistent CTAs, on-chip positions per chain
     bool fu_vec;              // FUSED: staged 8-row-aligned path
     int64_t fu_nc;            // FUSED: windows per system
@@ -163,16 +168,31 @@ void plan_geometry(tri_plan_s* p) {
         p->L = cdiv(n, S);
         p->n_pad = p->L * S;
         p->C = m * S;
+        p->k1 = std::min(p->k, SPLIT_K1MAX);
+        const int S1 = 1 << p->k1;
+        p->L1 = cdiv(n, S1);
+        p->C1 = m * S1;
+        p->region2 = p->nreg2 = p->nblk2 = 0;
         if (p->k > 0) {
             const int64_t target = 3 * (int64_t)p->sms;
+            const int64_t n_pad1 = p->L1 * S1;
             int64_t nreg = std::max<int64_t>(1, cdiv(target, m));
-            // regions no shorter than 4 f(k) + T so halos stay a small fraction
-            const int64_t minreg = 4 * halo_f(p->k) + TPCR_T;
-            nreg = std::max<int64_t>(1, std::min<int64_t>(nreg, p->n_pad / minreg));
-            p->region = cdiv(p->n_pad, nreg);
-            p->nreg = cdiv(p->n_pad, p->region);
+            // regions no shorter than 4 f(k1) + T so halos stay a small fraction
+            const int64_t minreg = 4 * halo_f(p->k1) + TPCR_T;
+            nreg = std::max<int64_t>(1, std::min<int64_t>(nreg, n_pad1 / minreg));
+            p->region = cdiv(n_pad1, nreg);
+            p->nreg = cdiv(n_pad1, p->region);
         } else {
             p->region = 0; p->nreg = 0;
+        }
+        if (p->k > p->k1) {  // pass 2 over the C1 chains, TPCR_IL_CB per CTA
+            const int k2 = p->k - p->k1;
+            p->nblk2 = cdiv(p->C1, TPCR_IL_CB);
+            int64_t nreg2 = std::max<int64_t>(1, cdiv(3 * (int64_t)p->sms, p->nblk2));
+            const int64_t minreg2 = 4 * halo_f(k2) + TPCR_IL_TP;
+            nreg2 = std::max<int64_t>(1, std::min<int64_t>(nreg2, p->L1 / minreg2));
+            p->region2 = cdiv(p->L1, nreg2);
+            p->nreg2 = cdiv(p->L1, p->region2);
         }
         p->G = 0; p->P = 0; p->rpt = 0;
     }
@@ -198,8 +218,10 @@ size_t scratch_need(const tri_plan_s* p) {
     if (p->variant != TRI_VARIANT_SPLIT) return 0;
     const size_t s = esize(p->dtype);
     const size_t chain_elems = (size_t)p->C * (size_t)p->L;
-    // k > 0: normalised reduced rows (3 arrays) + c', d' (2 arrays); k = 0: c', d'
-    return (p->k > 0 ? 5 : 2) * chain_elems * s;
+    // k > 0: normalised reduced rows (3 arrays) + c', d' (2 arrays); k = 0: c', d';
+    // two passes: + the pass-1 rows (3 arrays of C1 x L1)
+    const size_t pass1 = p->k > p->k1 ? 3 * (size_t)p->C1 * (size_t)p->L1 : 0;
+    return ((p->k > 0 ? 5 : 2) * chain_elems + pass1) * s;
 }
 
 tri_status ensure_scratch(tri_plan_s* p) {
@@ -216,10 +238,10 @@ tri_status ensure_scratch(tri_plan_s* p) {
     return TRI_OK;
 }
 
-int tiled_smem_layout(int k, int* off, int* mask) {
+int tiled_smem_layout(int k, int* off, int* mask, int tile = TPCR_T) {
     int total = 0;
     for (int j = 0; j < k; ++j) {
-        int need = TPCR_T + 2 * (1 << j);
+        int need = tile + 2 * (1 << j);
         int rs = 1;
         while (rs < need) rs *= 2;
         off[j] = total;
@@ -286,14 +308,31 @@ cudaError_t launch_tiled(const tri_plan_s* p, const void* a, const void* b, cons
     TiledArgs<T> A;
     A.a = (const T*)a; A.b = (const T*)b; A.c = (const T*)c; A.d = (const T*)d;
     A.oA = (T*)oA; A.oC = (T*)oC; A.oD = (T*)oD;
-    A.n = p->n; A.m = p->m; A.n_pad = p->n_pad; A.region = p->region; A.nreg = p->nreg; A.C = p->C;
-    A.layout = p->layout; A.k = p->k; A.mode = mode;
-    A.ring_total = tiled_smem_layout(p->k, A.ring_off, A.ring_mask);
+    A.n = p->n; A.m = p->m; A.n_pad = p->L1 << p->k1; A.region = p->region; A.nreg = p->nreg; A.C = p->C1;
+    A.layout = p->layout; A.k = p->k1; A.mode = mode;
+    A.ring_total = tiled_smem_layout(p->k1, A.ring_off, A.ring_mask);
     const size_t smem = (size_t)3 * A.ring_total * sizeof(T);
     cudaError_t e = cudaFuncSetAttribute(k_tiled_pcr<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     const int64_t grid = p->m * p->nreg;
     k_tiled_pcr<T><<<(unsigned)grid, TPCR_T, smem, st>>>(A);
+    return cudaGetLastError();
+}
+
+template <typename T>
+cudaError_t launch_tiled_il(const tri_plan_s* p, const void* iA, const void* iC, const void* iD, void* oA, void* oC,
+                            void* oD, int mode, cudaStream_t st) {
+    TiledILArgs<T> A;
+    A.iA = (const T*)iA; A.iC = (const T*)iC; A.iD = (const T*)iD;
+    A.oA = (T*)oA; A.oC = (T*)oC; A.oD = (T*)oD;
+    A.n = p->n; A.m = p->m; A.L1 = p->L1; A.C1 = p->C1; A.C = p->C;
+    A.region = p->region2; A.nreg = p->nreg2; A.nblk = p->nblk2;
+    A.layout = p->layout; A.k1 = p->k1; A.k2 = p->k - p->k1; A.mode = mode;
+    A.ring_total = tiled_smem_layout(A.k2, A.ring_off, A.ring_mask, TPCR_IL_TP);
+    const size_t smem = (size_t)3 * A.ring_total * TPCR_IL_CB * sizeof(T);
+    cudaError_t e = cudaFuncSetAttribute(k_tiled_pcr_il<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    k_tiled_pcr_il<T><<<(unsigned)(p->nblk2 * p->nreg2), TPCR_T, smem, st>>>(A);
     return cudaGetLastError();
 }
 
@@ -419,7 +458,16 @@ cudaError_t launch_split(const tri_plan_s* p, const void* a, const void* b, cons
     A.n = p->n; A.m = p->m; A.C = p->C; A.L = p->L; A.layout = p->layout; A.k = p->k;
     if (p->k > 0) {
         T *rA = base, *rC = base + ce, *rD = base + 2 * ce;
-        cudaError_t e = launch_tiled<T>(p, a, b, c, d, rA, rC, rD, 0, st);
+        cudaError_t e;
+        if (p->k > p->k1) {  // two passes: pass-1 rows after the 5 chain arrays
+            const size_t ce1 = (size_t)p->C1 * (size_t)p->L1;
+            T *pA = base + 5 * ce, *pC = pA + ce1, *pD = pA + 2 * ce1;
+            e = launch_tiled<T>(p, a, b, c, d, pA, pC, pD, 0, st);
+            if (e != cudaSuccess) return e;
+            e = launch_tiled_il<T>(p, pA, pC, pD, rA, rC, rD, 0, st);
+        } else {
+            e = launch_tiled<T>(p, a, b, c, d, rA, rC, rD, 0, st);
+        }
         if (e != cudaSuccess) return e;
         A.iA = rA; A.iC = rC; A.iD = rD;
         A.cps = base + 3 * ce; A.dps = base + 4 * ce;
@@ -574,7 +622,7 @@ int64_t tri_plan_scratch_bytes(tri_plan_t p) { return p ? (int64_t)p->scratch_by
 
 int tri_plan_launches(tri_plan_t p) {
     if (!p) return -1;
-    if (p->variant == TRI_VARIANT_SPLIT) return p->k > 0 ? 2 : 1;
+    if (p->variant == TRI_VARIANT_SPLIT) return p->k == 0 ? 1 : p->k > p->k1 ? 3 : 2;
     return 1;  // ONCHIP, FUSED
 }
 
@@ -662,8 +710,20 @@ tri_status tri_debug_pcr(tri_plan_t p, const void* a, const void* b, const void*
                                 : launch_fused<float>(p, a, b, c, d, nullptr, s, ao, co, do_);
     } else {
         if (p->k == 0) return TRI_ERR_INVALID_ARG;  // no PCR stage to show
-        e = p->dtype == TRI_F64 ? launch_tiled<double>(p, a, b, c, d, ao, co, do_, 1, s)
-                                : launch_tiled<float>(p, a, b, c, d, ao, co, do_, 1, s);
+        if (p->k > p->k1) {
+            const size_t ce = (size_t)p->C * (size_t)p->L, ce1 = (size_t)p->C1 * (size_t)p->L1;
+            char* pA = (char*)p->scratch + 5 * ce * esize(p->dtype);
+            char* pC = pA + ce1 * esize(p->dtype);
+            char* pD = pC + ce1 * esize(p->dtype);
+            e = p->dtype == TRI_F64 ? launch_tiled<double>(p, a, b, c, d, pA, pC, pD, 0, s)
+                                    : launch_tiled<float>(p, a, b, c, d, pA, pC, pD, 0, s);
+            if (e == cudaSuccess)
+                e = p->dtype == TRI_F64 ? launch_tiled_il<double>(p, pA, pC, pD, ao, co, do_, 1, s)
+                                        : launch_tiled_il<float>(p, pA, pC, pD, ao, co, do_, 1, s);
+        } else {
+            e = p->dtype == TRI_F64 ? launch_tiled<double>(p, a, b, c, d, ao, co, do_, 1, s)
+                                    : launch_tiled<float>(p, a, b, c, d, ao, co, do_, 1, s);
+        }
     }
     return e == cudaSuccess ? TRI_OK : TRI_ERR_CUDA;
 }

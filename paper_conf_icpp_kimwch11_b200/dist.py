@@ -4,6 +4,7 @@ The m systems are split into contiguous ranges, one per rank (tri_shard_range);
 each rank solves its shard on its own GPU with no collective inside the solve
 (the systems are independent: Eq 1 per system).  Collectives
 appear only at the edges:
+  * scatter_inputs: rank 0 hands each rank its a, b, c, d shard;
   * gather_x:  rank 0 collects the solution (NCCL over NVLink on the GPU box,
                gloo in the CPU tests);
   * max_over_ranks: the timing convention (job time = slowest rank).
@@ -57,6 +58,40 @@ def gather_x(x_local, n, m, layout=CONTIGUOUS, group=None, dst=0):
         else:
             full.view(n, m)[:, rq0:rq0 + rmr] = bufs[r].view(n, per)[:, :rmr]
     return full
+
+
+def scatter_inputs(n, m, full=None, layout=CONTIGUOUS, group=None, src=0, dtype=None, device=None):
+    """Distribute a, b, c, d from rank `src` (dist.scatter of the
+    input shards).  `full` (on src only): the 4 full n*m tensors.  Every rank
+    receives its systems [q0, q0+m_r) in the same layout with m_r columns.
+    Shards are padded to ceil(m/G) systems for the collective."""
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    per = -(-m // world)
+    q0, mr = shard_range(m, world, rank)
+    if rank == src:
+        dtype, device = full[0].dtype, full[0].device
+    out = []
+    for arr in range(4):
+        recv = torch.zeros(n * per, dtype=dtype, device=device)
+        send = None
+        if rank == src:
+            send = []
+            for r in range(world):
+                rq0, rmr = shard_range(m, world, r)
+                buf = torch.zeros(n * per, dtype=dtype, device=device)
+                if rmr:
+                    if layout == CONTIGUOUS:
+                        buf[: n * rmr] = full[arr][rq0 * n:(rq0 + rmr) * n]
+                    else:
+                        buf.view(n, per)[:, :rmr] = full[arr].view(n, m)[:, rq0:rq0 + rmr]
+                send.append(buf)
+        dist.scatter(recv, scatter_list=send, src=src, group=group)
+        if layout == CONTIGUOUS:
+            out.append(recv[: n * mr].clone())
+        else:
+            out.append(recv.view(n, per)[:, :mr].contiguous().view(-1))
+    return out
 
 
 def solve_sharded(n, m, make_inputs, solve_fn, layout=CONTIGUOUS, gather=True, group=None):

@@ -69,3 +69,50 @@ def test_sharded_solve_matches_single_process(layout, n, m, dtype):
     full = res[0][4]
     assert full is not None and np.array_equal(full, ref)
     assert res[1][4] is None
+
+
+def _worker_scatter(rank, world, port, n, m, layout, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import oracle
+        import trigen
+        from paper_conf_icpp_kimwch11_b200 import dist as tdist
+        full = None
+        if rank == 0:
+            full = [torch.from_numpy(t) for t in trigen.generate(n, m, "f64", layout, "dd")]
+        a, b, c, d = tdist.scatter_inputs(n, m, full, layout=layout, dtype=torch.float64,
+                                          device=torch.device("cpu"))
+        q0, mr = tdist.shard_range(m, world, rank)
+        # the received shard is exactly the generator's shard (shard-invariant inputs)
+        ref = trigen.generate(n, mr, "f64", layout, "dd", q0=q0) if mr else [np.zeros(0)] * 4
+        same = all(np.array_equal(t.numpy(), r) for t, r in zip((a, b, c, d), ref))
+        x = torch.from_numpy(oracle.solve_batch(n, mr, *(t.numpy() for t in (a, b, c, d)), layout=layout,
+                                                nthreads=1)) if mr else torch.zeros(0, dtype=torch.float64)
+        full_x = tdist.gather_x(x, n, m, layout)
+        q.put((rank, same, None if full_x is None else full_x.numpy()))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("layout", [0, 1])
+@pytest.mark.parametrize("n,m", [(17, 5), (8, 2)])
+def test_scatter_solve_gather_roundtrip(layout, n, m):
+    """Rank 0 scatters the inputs, every rank solves its shard,
+    rank 0 gathers x: equal to the single-process solve."""
+    import oracle
+    import trigen
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = 31500 + (os.getpid() % 2000)
+    procs = [ctx.Process(target=_worker_scatter, args=(r, 2, port, n, m, layout, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    res = sorted([q.get(timeout=120) for _ in range(2)], key=lambda r: r[0])
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    assert all(r[1] for r in res)
+    a, b, c, d = trigen.generate(n, m, "f64", layout, "dd")
+    assert np.array_equal(res[0][2], oracle.solve_batch(n, m, a, b, c, d, layout=layout, nthreads=1))

@@ -64,8 +64,9 @@ def test_split_every_k(cuda_ok, dtype, layout, n, m):
     arrs = gen(n, m, dtype, layout, "weak", eps=1e-2)
     xo = oracle.solve_batch(n, m, *arrs, layout=layout)
     plan = None
-    for k in range(0, min(int(np.log2(n)), 10) + 1):
+    for k in range(0, min(int(np.log2(n)), 15) + 1):  # k > 10: two tiled-PCR passes
         x, plan = gpu_solve(n, m, arrs, dtype, layout, k=k, variant=SPLIT, plan=plan)
+        assert plan.launches == (1 if k == 0 else 2 if k <= 10 else 3)
         check_parity(n, m, arrs, x, dtype, layout, x_oracle=xo)
 
 
@@ -81,6 +82,7 @@ def test_split_on_small_systems(cuda_ok):
 # ------------------------------------------------------------------ PCR stage (row A2)
 @pytest.mark.parametrize("variant,n,m,k", [(ONCHIP, 1024, 3, 3), (ONCHIP, 500, 2, 5), (SPLIT, 9000, 2, 4),
                                            (WARP, 1000, 3, 5), (WARP, 33, 2, 5), (WARP, 256, 4, 5),
+                                           (SPLIT, 70001, 1, 13), (SPLIT, 20001, 2, 12), (SPLIT, 40000, 3, 15),
                                            (SPLIT, 20001, 1, 8), (SPLIT, 5000, 3, 1)])
 def test_pcr_stage_matches_oracle(cuda_ok, variant, n, m, k):
     """The reduced system after k PCR steps (Eqs 5-6) vs the oracle's plain PCR,
