@@ -9,8 +9,8 @@
 // of the same system run in parallel CTAs with f(k)-row halos loaded on both
 // sides (Fig 11b, "overlapping tiles in the boundary of regions").
 //
-// B200 form: one ring buffer per level in shared memory (power-of-two size >=
-// T + 2 sigma_j, modular indexing instead of the paper's buffer shifts);
+// B200 form: one ring buffer per level in shared memory (exactly T + 2 sigma_j
+// rows, modular slots instead of the paper's buffer shifts);
 // rows normalised to unit diagonal (3 values per row; X17); the last
 // level writes its rows straight into the p-Thomas input layout (the interleave
 // transform fused into the last store):
@@ -30,32 +30,53 @@ struct TiledArgs {
     T *oA, *oC, *oD;   // mode 0: chain-interleaved scratch; mode 1: user layout
     int64_t n, m, n_pad, region, nreg, C;
     int layout, k, mode;
-    int ring_off[16];  // row offset of level j's ring inside the smem arrays
-    int ring_mask[16];
-    int ring_total;    // rows across all rings
 };
 
 __host__ __device__ inline int64_t halo_f(int k) { return (int64_t(1) << k) - 1; }  // Eq 8
 
-template <typename T>
-__global__ void __launch_bounds__(TPCR_T) k_tiled_pcr(TiledArgs<T> p) {
+// Ring j holds exactly the T + 2^(j+1) rows level j can touch within one
+// iteration (reads i +- 2^j of this sub-tile, the level below already wrote the
+// next T rows): exact sizes instead of powers of two keep two CTAs per SM at
+// k = 10 (110.5 KB fp64).  Ring slots are tracked incrementally per thread
+// (32-bit, one conditional wrap per step) instead of computed from row indices.
+template <int K>
+struct TPCRRing {
+    static constexpr int size(int j) { return TPCR_T + (2 << j); }
+    static constexpr int off(int j) { return j == 0 ? 0 : off(j - 1) + size(j - 1); }
+    static constexpr int total() { return off(K); }
+};
+
+template <typename T, int K>
+__global__ void __launch_bounds__(TPCR_T, 2) k_tiled_pcr(TiledArgs<T> p) {
+    using RG = TPCRRing<K>;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     T* rA = reinterpret_cast<T*>(smem_raw);
-    T* rC = rA + p.ring_total;
-    T* rD = rC + p.ring_total;
+    T* rC = rA + RG::total();
+    T* rD = rC + RG::total();
 
     const int tid = threadIdx.x;
     const int64_t q = blockIdx.x / p.nreg;
     const int64_t reg = blockIdx.x - q * p.nreg;
     const int64_t r0 = reg * p.region;
     const int64_t r1 = imin64(r0 + p.region, p.n_pad);
-    const int64_t fk = halo_f(p.k);
+    constexpr int64_t fk = (int64_t(1) << K) - 1;  // Eq 8
     const int64_t start = r0 - fk;  // halo: level-0 rows [r0-f(k), r1+f(k)) feed outputs [r0, r1)
     const int64_t n = p.n;
-    const int S = 1 << p.k;
+    constexpr int S = 1 << K;
 
-    // rings start as identity rows (they are only read outside the valid cone)
-    for (int e = tid; e < p.ring_total; e += TPCR_T) { rA[e] = T(0); rC[e] = T(0); rD[e] = T(0); }
+    for (int e = tid; e < RG::total(); e += TPCR_T) { rA[e] = T(0); rC[e] = T(0); rD[e] = T(0); }
+    // slots: w0 = ring-0 slot of row s0 + tid; rs[j] = ring-j slot of the row level j
+    // combines, i_j = s0 - (2^(j+1) - 1) + tid; ws[j] = ring-(j+1) slot of i_j.
+    // Slot of row i in ring j = (i - base) mod size(j), base <= every row touched.
+    const int64_t base = start - (int64_t(2) << K);
+    int w0 = (int)((start + tid - base) % RG::size(0));
+    int rs[K], ws[K];
+#pragma unroll
+    for (int j = 0; j < K; ++j) {
+        const int64_t ij = start - ((int64_t(2) << j) - 1) + tid;
+        rs[j] = (int)((ij - base) % RG::size(j));
+        ws[j] = j + 1 < K ? (int)((ij - base) % RG::size(j + 1)) : 0;
+    }
     __syncthreads();
 
     // level-0 rows of the next sub-tile are loaded into registers while the
@@ -74,44 +95,47 @@ __global__ void __launch_bounds__(TPCR_T) k_tiled_pcr(TiledArgs<T> p) {
     };
     fetch(start);
     for (int64_t s0 = start; s0 - fk < r1; s0 += TPCR_T) {
-        // level 0: normalise this thread's (prefetched) row; rows outside the
-        // system are identity rows (b = 1, a = c = d = 0)
-        {
-            const int64_t i = s0 + tid;
+        {   // level 0: normalise this thread's prefetched row (identity outside the system)
             const NRow<T> r = normalise(pa, pb, pc, pd);
-            const int s = p.ring_off[0] + (int)(i & p.ring_mask[0]);
-            rA[s] = r.A; rC[s] = r.C; rD[s] = r.D;
+            rA[w0] = r.A; rC[w0] = r.C; rD[w0] = r.D;
         }
         fetch(s0 + TPCR_T);
         __syncthreads();
-        int64_t F = s0 + TPCR_T;  // level-j frontier (exclusive)
-        for (int j = 0; j < p.k; ++j) {
-            const int sg = 1 << j;
-            F -= sg;
-            const int64_t i = F - TPCR_T + tid;
-            const int off = p.ring_off[j], msk = p.ring_mask[j];
-            const int so = off + (int)(i & msk), sm = off + (int)((i - sg) & msk), sp = off + (int)((i + sg) & msk);
-            NRow<T> o{rA[so], rC[so], rD[so]};
-            NRow<T> mm{rA[sm], rC[sm], rD[sm]};
-            NRow<T> pp{rA[sp], rC[sp], rD[sp]};
-            NRow<T> nr = pcr_combine(mm, o, pp);
-            if (j + 1 < p.k) {
-                const int sd = p.ring_off[j + 1] + (int)(i & p.ring_mask[j + 1]);
+#pragma unroll
+        for (int j = 0; j < K; ++j) {
+            const int Z = RG::size(j), O = RG::off(j), sg = 1 << j;
+            int sm = rs[j] - sg; sm += sm < 0 ? Z : 0;
+            int sp = rs[j] + sg; sp -= sp >= Z ? Z : 0;
+            const int so = O + rs[j];
+            sm += O; sp += O;
+            const NRow<T> nr = pcr_combine(NRow<T>{rA[sm], rC[sm], rD[sm]}, NRow<T>{rA[so], rC[so], rD[so]},
+                                           NRow<T>{rA[sp], rC[sp], rD[sp]});
+            if (j + 1 < K) {
+                const int sd = RG::off(j + 1) + ws[j];
                 rA[sd] = nr.A; rC[sd] = nr.C; rD[sd] = nr.D;
-            } else if (i >= r0 && i < r1) {
-                if (p.mode == 0) {
-                    const int64_t idx = (i >> p.k) * p.C + q * S + (i & (S - 1));
-                    p.oA[idx] = nr.A; p.oC[idx] = nr.C; p.oD[idx] = nr.D;
-                } else if (i < n) {
-                    const int64_t gi = elem_index(q, i, n, p.m, p.layout);
-                    p.oA[gi] = nr.A; p.oC[gi] = nr.C; p.oD[gi] = nr.D;
+            } else {
+                const int64_t i = s0 - ((int64_t(2) << j) - 1) + tid;
+                if (i >= r0 && i < r1) {
+                    if (p.mode == 0) {
+                        const int64_t idx = (i >> K) * p.C + q * S + (i & (S - 1));
+                        p.oA[idx] = nr.A; p.oC[idx] = nr.C; p.oD[idx] = nr.D;
+                    } else if (i < n) {
+                        const int64_t gi = elem_index(q, i, n, p.m, p.layout);
+                        p.oA[gi] = nr.A; p.oC[gi] = nr.C; p.oD[gi] = nr.D;
+                    }
                 }
             }
             __syncthreads();
         }
+        // every row index advances by T: advance the slots
+        w0 += TPCR_T; w0 -= w0 >= RG::size(0) ? RG::size(0) : 0;
+#pragma unroll
+        for (int j = 0; j < K; ++j) {
+            rs[j] += TPCR_T; rs[j] -= rs[j] >= RG::size(j) ? RG::size(j) : 0;
+            if (j + 1 < K) { ws[j] += TPCR_T; ws[j] -= ws[j] >= RG::size(j + 1) ? RG::size(j + 1) : 0; }
+        }
     }
 }
-
 
 // ---------------------------------------------------------------------------
 // Second tiled-PCR pass (deep k, two passes): the chain-interleaved output of
@@ -122,8 +146,9 @@ __global__ void __launch_bounds__(TPCR_T) k_tiled_pcr(TiledArgs<T> p) {
 // sliding window, over TPCR_IL_CB adjacent chains per CTA so every position row
 // is one 256-byte segment.  Its output is the layout a single k1 + k2 pass would
 // store: chain ch2 = q 2^k + (r1 + 2^k1 (pos mod 2^k2)), position pos >> k2.
-constexpr int TPCR_IL_CB = 32;                     // chains per CTA
-constexpr int TPCR_IL_TP = TPCR_T / TPCR_IL_CB;    // positions per sub-tile
+constexpr int TPCR_IL_CB = 32;                          // chains per CTA
+constexpr int TPCR_IL_RPT = 2;                          // positions per thread per sub-tile
+constexpr int TPCR_IL_TP = TPCR_IL_RPT * TPCR_T / TPCR_IL_CB;  // positions per sub-tile
 
 template <typename T>
 struct TiledILArgs {
@@ -138,14 +163,14 @@ struct TiledILArgs {
 
 template <typename T>
 __global__ void __launch_bounds__(TPCR_T) k_tiled_pcr_il(TiledILArgs<T> p) {
-    constexpr int CB = TPCR_IL_CB, TP = TPCR_IL_TP;
+    constexpr int CB = TPCR_IL_CB, TP = TPCR_IL_TP, RPT = TPCR_IL_RPT, UP = TPCR_T / CB;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     T* rA = reinterpret_cast<T*>(smem_raw);
     T* rC = rA + p.ring_total * CB;
     T* rD = rC + p.ring_total * CB;
 
     const int tid = threadIdx.x;
-    const int c = tid % CB, u = tid / CB;
+    const int c = tid % CB, u0 = tid / CB;  // this thread: chain c, positions u0 + UP * h
     const int64_t blk = blockIdx.x % p.nblk, reg = blockIdx.x / p.nblk;
     const int64_t ch = blk * CB + c;
     const bool chok = ch < p.C1;
@@ -160,21 +185,25 @@ __global__ void __launch_bounds__(TPCR_T) k_tiled_pcr_il(TiledILArgs<T> p) {
     for (int e = tid; e < p.ring_total * CB; e += TPCR_T) { rA[e] = T(0); rC[e] = T(0); rD[e] = T(0); }
     __syncthreads();
 
-    NRow<T> nxt;  // next sub-tile's level-0 row, loaded during this sub-tile's levels
+    NRow<T> nxt[RPT];  // next sub-tile's level-0 rows, loaded during this sub-tile's levels
     auto fetch = [&](int64_t s0) {
-        const int64_t pos = s0 + u;
-        nxt = identity_row<T>();
-        if (pos >= 0 && pos < p.L1 && chok) {
-            const int64_t gi = pos * p.C1 + ch;
-            nxt = NRow<T>{ldg_stream(p.iA + gi), ldg_stream(p.iC + gi), ldg_stream(p.iD + gi)};
+#pragma unroll
+        for (int h = 0; h < RPT; ++h) {
+            const int64_t pos = s0 + u0 + UP * h;
+            nxt[h] = identity_row<T>();
+            if (pos >= 0 && pos < p.L1 && chok) {
+                const int64_t gi = pos * p.C1 + ch;
+                nxt[h] = NRow<T>{ldg_stream(p.iA + gi), ldg_stream(p.iC + gi), ldg_stream(p.iD + gi)};
+            }
         }
     };
     fetch(start);
     for (int64_t s0 = start; s0 - fk < r1; s0 += TP) {
-        {
-            const int64_t pos = s0 + u;
+#pragma unroll
+        for (int h = 0; h < RPT; ++h) {
+            const int64_t pos = s0 + u0 + UP * h;
             const int sl = (p.ring_off[0] + (int)(pos & p.ring_mask[0])) * CB + c;
-            rA[sl] = nxt.A; rC[sl] = nxt.C; rD[sl] = nxt.D;
+            rA[sl] = nxt[h].A; rC[sl] = nxt[h].C; rD[sl] = nxt[h].D;
         }
         fetch(s0 + TP);
         __syncthreads();
@@ -182,27 +211,35 @@ __global__ void __launch_bounds__(TPCR_T) k_tiled_pcr_il(TiledILArgs<T> p) {
         for (int j = 0; j < p.k2; ++j) {
             const int sg = 1 << j;
             F -= sg;
-            const int64_t pos = F - TP + u;
             const int off = p.ring_off[j], msk = p.ring_mask[j];
-            const int so = (off + (int)(pos & msk)) * CB + c;
-            const int sm = (off + (int)((pos - sg) & msk)) * CB + c;
-            const int sp = (off + (int)((pos + sg) & msk)) * CB + c;
-            const NRow<T> nr = pcr_combine(NRow<T>{rA[sm], rC[sm], rD[sm]}, NRow<T>{rA[so], rC[so], rD[so]},
-                                           NRow<T>{rA[sp], rC[sp], rD[sp]});
-            if (j + 1 < p.k2) {
-                const int sd = (p.ring_off[j + 1] + (int)(pos & p.ring_mask[j + 1])) * CB + c;
-                rA[sd] = nr.A; rC[sd] = nr.C; rD[sd] = nr.D;
-            } else if (pos >= r0 && pos < r1 && chok) {
-                const int64_t r = rr1 + ((pos & ((int64_t(1) << p.k2) - 1)) << p.k1);  // residue mod 2^k
-                const int64_t pos2 = pos >> p.k2;
-                if (p.mode == 0) {
-                    const int64_t idx = pos2 * p.C + (q << k) + r;
-                    p.oA[idx] = nr.A; p.oC[idx] = nr.C; p.oD[idx] = nr.D;
-                } else {
-                    const int64_t i = (pos2 << k) + r;
-                    if (i < p.n) {
-                        const int64_t gi = elem_index(q, i, p.n, p.m, p.layout);
-                        p.oA[gi] = nr.A; p.oC[gi] = nr.C; p.oD[gi] = nr.D;
+            NRow<T> nr[RPT];
+#pragma unroll
+            for (int h = 0; h < RPT; ++h) {
+                const int64_t pos = F - TP + u0 + UP * h;
+                const int so = (off + (int)(pos & msk)) * CB + c;
+                const int sm = (off + (int)((pos - sg) & msk)) * CB + c;
+                const int sp = (off + (int)((pos + sg) & msk)) * CB + c;
+                nr[h] = pcr_combine(NRow<T>{rA[sm], rC[sm], rD[sm]}, NRow<T>{rA[so], rC[so], rD[so]},
+                                    NRow<T>{rA[sp], rC[sp], rD[sp]});
+            }
+#pragma unroll
+            for (int h = 0; h < RPT; ++h) {
+                const int64_t pos = F - TP + u0 + UP * h;
+                if (j + 1 < p.k2) {
+                    const int sd = (p.ring_off[j + 1] + (int)(pos & p.ring_mask[j + 1])) * CB + c;
+                    rA[sd] = nr[h].A; rC[sd] = nr[h].C; rD[sd] = nr[h].D;
+                } else if (pos >= r0 && pos < r1 && chok) {
+                    const int64_t r = rr1 + ((pos & ((int64_t(1) << p.k2) - 1)) << p.k1);  // residue mod 2^k
+                    const int64_t pos2 = pos >> p.k2;
+                    if (p.mode == 0) {
+                        const int64_t idx = pos2 * p.C + (q << k) + r;
+                        p.oA[idx] = nr[h].A; p.oC[idx] = nr[h].C; p.oD[idx] = nr[h].D;
+                    } else {
+                        const int64_t i = (pos2 << k) + r;
+                        if (i < p.n) {
+                            const int64_t gi = elem_index(q, i, p.n, p.m, p.layout);
+                            p.oA[gi] = nr[h].A; p.oC[gi] = nr[h].C; p.oD[gi] = nr[h].D;
+                        }
                     }
                 }
             }

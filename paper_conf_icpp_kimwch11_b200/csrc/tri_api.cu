@@ -28,6 +28,13 @@ namespace {
 thread_local tri_status g_last = TRI_OK;
 void* g_fused_prof = nullptr;  // tri_debug_set_profile: device counters for the fused kernel
 int g_fused_dbg_mode = 0;     // TRI_FUSED_DBG_MODE (diagnostics only)
+// waves of regions per tiled-PCR pass (TRI_TILED_WAVES1/2 override, for tuning)
+int env_int(const char* name, int dflt) {
+    const char* e = getenv(name);
+    return e ? std::max(1, atoi(e)) : dflt;
+}
+int g_tiled_waves1 = env_int("TRI_TILED_WAVES1", 1);
+int g_tiled_waves2 = env_int("TRI_TILED_WAVES2", 3);  // measured best at c3 (1 / 3 waves)
 
 constexpr int ONCHIP_THREADS = 512;
 constexpr int SPLIT_K1MAX = 10;  // deepest k one sliding-window pass holds in smem (T = 256)
@@ -139,6 +146,52 @@ struct tri_plan_s {
 
 namespace {
 
+// resident CTAs per SM of the tiled-PCR passes (one full wave of regions)
+template <typename T, int K>
+int tiled_occ_k() {
+    const int smem = 3 * TPCRRing<K>::total() * (int)sizeof(T);
+    if (cudaFuncSetAttribute(k_tiled_pcr<T, K>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess) {
+        cudaGetLastError();
+        return 1;
+    }
+    int occ = 1;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_tiled_pcr<T, K>, TPCR_T, smem) != cudaSuccess) {
+        cudaGetLastError();
+        occ = 1;
+    }
+    return std::max(1, occ);
+}
+template <typename T>
+int tiled_occ(int k1) {
+    switch (k1) {
+        case 1: return tiled_occ_k<T, 1>();
+        case 2: return tiled_occ_k<T, 2>();
+        case 3: return tiled_occ_k<T, 3>();
+        case 4: return tiled_occ_k<T, 4>();
+        case 5: return tiled_occ_k<T, 5>();
+        case 6: return tiled_occ_k<T, 6>();
+        case 7: return tiled_occ_k<T, 7>();
+        case 8: return tiled_occ_k<T, 8>();
+        case 9: return tiled_occ_k<T, 9>();
+        default: return tiled_occ_k<T, 10>();
+    }
+}
+int tiled_il_smem(int k2, size_t es);
+template <typename T>
+int tiled_il_occ(int k2) {
+    const int smem = tiled_il_smem(k2, sizeof(T));
+    if (cudaFuncSetAttribute(k_tiled_pcr_il<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess) {
+        cudaGetLastError();
+        return 1;
+    }
+    int occ = 1;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_tiled_pcr_il<T>, TPCR_T, smem) != cudaSuccess) {
+        cudaGetLastError();
+        occ = 1;
+    }
+    return std::max(1, occ);
+}
+
 // ---- per-plan geometry -----------------------------------------------------
 void plan_geometry(tri_plan_s* p) {
     const int64_t n = p->n, m = p->m;
@@ -174,7 +227,8 @@ void plan_geometry(tri_plan_s* p) {
         p->C1 = m * S1;
         p->region2 = p->nreg2 = p->nblk2 = 0;
         if (p->k > 0) {
-            const int64_t target = 3 * (int64_t)p->sms;
+            const int occ = p->dtype == TRI_F64 ? tiled_occ<double>(p->k1) : tiled_occ<float>(p->k1);
+            const int64_t target = (int64_t)occ * p->sms * g_tiled_waves1;
             const int64_t n_pad1 = p->L1 * S1;
             int64_t nreg = std::max<int64_t>(1, cdiv(target, m));
             // regions no shorter than 4 f(k1) + T so halos stay a small fraction
@@ -188,7 +242,8 @@ void plan_geometry(tri_plan_s* p) {
         if (p->k > p->k1) {  // pass 2 over the C1 chains, TPCR_IL_CB per CTA
             const int k2 = p->k - p->k1;
             p->nblk2 = cdiv(p->C1, TPCR_IL_CB);
-            int64_t nreg2 = std::max<int64_t>(1, cdiv(3 * (int64_t)p->sms, p->nblk2));
+            const int occ2 = p->dtype == TRI_F64 ? tiled_il_occ<double>(k2) : tiled_il_occ<float>(k2);
+            int64_t nreg2 = std::max<int64_t>(1, cdiv((int64_t)occ2 * p->sms * g_tiled_waves2, p->nblk2));
             const int64_t minreg2 = 4 * halo_f(k2) + TPCR_IL_TP;
             nreg2 = std::max<int64_t>(1, std::min<int64_t>(nreg2, p->L1 / minreg2));
             p->region2 = cdiv(p->L1, nreg2);
@@ -302,6 +357,15 @@ cudaError_t launch_warp(const tri_plan_s* p, const void* a, const void* b, const
     return cudaGetLastError();
 }
 
+template <typename T, int K>
+cudaError_t launch_tiled_k(const TiledArgs<T>& A, int64_t grid, cudaStream_t st) {
+    const size_t smem = (size_t)3 * TPCRRing<K>::total() * sizeof(T);
+    cudaError_t e = cudaFuncSetAttribute(k_tiled_pcr<T, K>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    k_tiled_pcr<T, K><<<(unsigned)grid, TPCR_T, smem, st>>>(A);
+    return cudaGetLastError();
+}
+
 template <typename T>
 cudaError_t launch_tiled(const tri_plan_s* p, const void* a, const void* b, const void* c, const void* d,
                          void* oA, void* oC, void* oD, int mode, cudaStream_t st) {
@@ -310,13 +374,25 @@ cudaError_t launch_tiled(const tri_plan_s* p, const void* a, const void* b, cons
     A.oA = (T*)oA; A.oC = (T*)oC; A.oD = (T*)oD;
     A.n = p->n; A.m = p->m; A.n_pad = p->L1 << p->k1; A.region = p->region; A.nreg = p->nreg; A.C = p->C1;
     A.layout = p->layout; A.k = p->k1; A.mode = mode;
-    A.ring_total = tiled_smem_layout(p->k1, A.ring_off, A.ring_mask);
-    const size_t smem = (size_t)3 * A.ring_total * sizeof(T);
-    cudaError_t e = cudaFuncSetAttribute(k_tiled_pcr<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return e;
     const int64_t grid = p->m * p->nreg;
-    k_tiled_pcr<T><<<(unsigned)grid, TPCR_T, smem, st>>>(A);
-    return cudaGetLastError();
+    switch (p->k1) {
+        case 1: return launch_tiled_k<T, 1>(A, grid, st);
+        case 2: return launch_tiled_k<T, 2>(A, grid, st);
+        case 3: return launch_tiled_k<T, 3>(A, grid, st);
+        case 4: return launch_tiled_k<T, 4>(A, grid, st);
+        case 5: return launch_tiled_k<T, 5>(A, grid, st);
+        case 6: return launch_tiled_k<T, 6>(A, grid, st);
+        case 7: return launch_tiled_k<T, 7>(A, grid, st);
+        case 8: return launch_tiled_k<T, 8>(A, grid, st);
+        case 9: return launch_tiled_k<T, 9>(A, grid, st);
+        case 10: return launch_tiled_k<T, 10>(A, grid, st);
+        default: return cudaErrorInvalidValue;
+    }
+}
+
+int tiled_il_smem(int k2, size_t es) {
+    int off[8], mask[8];
+    return 3 * tiled_smem_layout(k2, off, mask, TPCR_IL_TP) * TPCR_IL_CB * (int)es;
 }
 
 template <typename T>
