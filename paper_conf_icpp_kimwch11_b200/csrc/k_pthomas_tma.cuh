@@ -211,3 +211,148 @@ __global__ void __launch_bounds__(PTT_CH) k_pthomas_tma(const __grid_constant__ 
 }
 
 }  // namespace tri
+
+namespace tri {
+
+// ---------------------------------------------------------------------------
+// p-Thomas over chain-interleaved data [pos * C + ch] (MODE 0: normalised rows
+// from tiled PCR; MODE 1: raw rows of the INTERLEAVED user layout, k = 0), one
+// warp = 32 adjacent chains.  Tiles of 32 chains x R positions (256 B x R for
+// fp64) arrive by cp.async.bulk.tensor.2d into a PTT_NS-stage ring; c', d' go to
+// scratch [pos * C + ch] and come back the same way for Eq 4; x leaves by TMA
+// tensor store when the user layout is a 2D [L][C] view (INTERLEAVED, or m = 1
+// with n a multiple of 2^k), else by per-thread stores.
+template <typename T>
+struct PTICfg {
+    static constexpr int R = 16;                 // positions per tile
+    static constexpr int TILE = PTT_CH * R;      // elements per array tile
+};
+
+struct PTIMaps {
+    CUtensorMap a, b, c, d;  // inputs (MODE 0 uses a, b, c for iA, iC, iD), dims {C, L}, box {32, R}
+    CUtensorMap x;           // output view {C, L} (only when x_tma)
+    CUtensorMap cp, dp;      // scratch, dims {C, L}
+};
+
+template <typename T, int MODE>
+__global__ void __launch_bounds__(PTT_CH) k_pthomas_il_tma(const __grid_constant__ PTIMaps tm, PThomasArgs<T> p,
+                                                         int x_tma) {
+    constexpr int R = PTICfg<T>::R, TILE = PTICfg<T>::TILE;
+    constexpr int NA = MODE == 1 ? 4 : 3;
+    constexpr int FSTAGE = NA * TILE, BSTAGE = 2 * TILE;
+    extern __shared__ unsigned char smem_raw[];
+    T* sm = reinterpret_cast<T*>((reinterpret_cast<uintptr_t>(smem_raw) + 127) & ~uintptr_t(127));
+    __shared__ uint64_t fbar[PTT_NS], bbar[PTT_NB];
+    const int t = threadIdx.x;
+    const int c0 = blockIdx.x * PTT_CH;
+    const int64_t ch = c0 + t;
+    const bool active = ch < p.C;
+    const int64_t L = p.L, C = p.C;
+    const int ntile = (int)((L + R - 1) / R);
+    if (t == 0) {
+        for (int s = 0; s < PTT_NS; ++s) ptt_bar_init(&fbar[s]);
+        for (int s = 0; s < PTT_NB; ++s) ptt_bar_init(&bbar[s]);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncwarp();
+    auto issue_f = [&](int tt) {
+        if (t == 0 && tt < ntile) {
+            const int s = tt % PTT_NS;
+            T* st = sm + s * FSTAGE;
+            fence_proxy_async_smem();
+            ptt_expect(&fbar[s], FSTAGE * (unsigned)sizeof(T));
+            ptt_load(st, &tm.a, c0, tt * R, &fbar[s]);
+            ptt_load(st + TILE, &tm.b, c0, tt * R, &fbar[s]);
+            ptt_load(st + 2 * TILE, &tm.c, c0, tt * R, &fbar[s]);
+            if (MODE == 1) ptt_load(st + 3 * TILE, &tm.d, c0, tt * R, &fbar[s]);
+        }
+    };
+    for (int s = 0; s < PTT_NS; ++s) issue_f(s);
+
+    T cp = T(0), dp = T(0);
+    for (int tt = 0; tt < ntile; ++tt) {
+        const int s = tt % PTT_NS;
+        ptt_wait(&fbar[s], (unsigned)((tt / PTT_NS) & 1));
+        const T* st = sm + s * FSTAGE + t;
+        T v[NA][R];
+#pragma unroll
+        for (int arr = 0; arr < NA; ++arr)
+#pragma unroll
+            for (int u = 0; u < R; ++u) v[arr][u] = st[arr * TILE + u * PTT_CH];
+        __syncwarp();
+        issue_f(tt + PTT_NS);
+        const int64_t j0 = (int64_t)tt * R;
+        T* cps = p.cps + j0 * C + ch;
+        T* dps = p.dps + j0 * C + ch;
+#pragma unroll
+        for (int u = 0; u < R; ++u) {
+            const int64_t j = j0 + u;
+            if (j < L) {
+                if (MODE == 1) {
+                    thomas_fwd(Row4<T>{j > 0 ? v[0][u] : T(0), v[1][u], j < L - 1 ? v[2][u] : T(0), v[3][u]}, cp, dp);
+                } else {
+                    thomas_fwd(NRow<T>{v[0][u], v[1][u], v[2][u]}, cp, dp);
+                }
+                if (active) { cps[u * C] = cp; dps[u * C] = dp; }
+            }
+        }
+    }
+
+    __threadfence_block();
+    asm volatile("fence.proxy.async.global;" ::: "memory");
+    __syncwarp();
+    T* xt = sm + PTT_NB * BSTAGE;  // 2 x TILE, [R][32]
+    auto issue_b = [&](int b) {
+        if (t == 0 && b < ntile) {
+            const int s = b % PTT_NB;
+            const int tt = ntile - 1 - b;
+            T* st = sm + s * BSTAGE;
+            fence_proxy_async_smem();
+            ptt_expect(&bbar[s], BSTAGE * (unsigned)sizeof(T));
+            ptt_load(st, &tm.cp, c0, tt * R, &bbar[s]);
+            ptt_load(st + TILE, &tm.dp, c0, tt * R, &bbar[s]);
+        }
+    };
+    for (int s = 0; s < PTT_NB; ++s) issue_b(s);
+    T xv = T(0);
+    for (int b = 0; b < ntile; ++b) {
+        const int s = b % PTT_NB;
+        const int tt = ntile - 1 - b;
+        ptt_wait(&bbar[s], (unsigned)((b / PTT_NB) & 1));
+        const T* st = sm + s * BSTAGE + t;
+        T cs[R], ds[R];
+#pragma unroll
+        for (int u = 0; u < R; ++u) { cs[u] = st[u * PTT_CH]; ds[u] = st[TILE + u * PTT_CH]; }
+        if (x_tma && t == 0) bulk_wait_read<1>();
+        __syncwarp();
+        issue_b(b + PTT_NB);
+        T* xb = xt + (b & 1) * TILE;
+        const int64_t j0 = (int64_t)tt * R;
+#pragma unroll
+        for (int u = R - 1; u >= 0; --u) {
+            const int64_t j = j0 + u;
+            if (j < L) xv = fma(-cs[u], xv, ds[u]);
+            if (x_tma) {
+                xb[u * PTT_CH + t] = xv;
+            } else if (j < L && active) {
+                pt_store_x<T, MODE>(p, ch, j, xv);
+            }
+        }
+        if (x_tma) {
+            fence_proxy_async_smem();
+            __syncwarp();
+            if (t == 0) {
+                ptt_store(&tm.x, c0, tt * R, xb);
+                bulk_commit();
+            }
+        }
+    }
+    if (x_tma && t == 0) bulk_wait<0>();
+}
+
+template <typename T, int MODE>
+__host__ __device__ constexpr int pti_smem_bytes() {
+    return PTT_NS * (MODE == 1 ? 4 : 3) * PTICfg<T>::TILE * (int)sizeof(T) + 128;
+}
+
+}  // namespace tri

@@ -509,9 +509,39 @@ cudaError_t launch_ring(const tri_plan_s* p, const PThomasArgs<T>& A, bool vec, 
     return cudaGetLastError();
 }
 
+// chain-interleaved p-Thomas through TMA (C >= 32 x SMs); cudaErrorNotSupported
+// asks for the fallback kernels
+template <typename T, int MODE>
+cudaError_t launch_pthomas_il_tma(const tri_plan_s* p, const PThomasArgs<T>& A, cudaStream_t st) {
+    constexpr int R = PTICfg<T>::R;
+    const int64_t C = p->C, L = p->L;
+    if ((C * (int64_t)sizeof(T)) % 16 || C > INT32_MAX || L > INT32_MAX) return cudaErrorNotSupported;
+    PTIMaps tm;
+    const void* in[4] = {MODE == 1 ? (const void*)A.a : (const void*)A.iA, MODE == 1 ? (const void*)A.b : (const void*)A.iC,
+                         MODE == 1 ? (const void*)A.c : (const void*)A.iD, MODE == 1 ? (const void*)A.d : (const void*)A.iD};
+    bool ok = true;
+    for (int i = 0; i < 4 && ok; ++i) ok = tma_map_2d<T>(&tm.a + i, in[i], C, L, PTT_CH, R, false);
+    ok = ok && tma_map_2d<T>(&tm.cp, A.cps, C, L, PTT_CH, R, false) && tma_map_2d<T>(&tm.dp, A.dps, C, L, PTT_CH, R, false);
+    // x as a [L][C] view: INTERLEAVED user layout (MODE 1), or one system whose
+    // rows pos * 2^k + r are exactly [pos * C + r] (m = 1, n = L * 2^k)
+    const bool x_view = MODE == 1 || (p->m == 1 && p->n == L * C);
+    int x_tma = 0;
+    if (ok && x_view) x_tma = tma_map_2d<T>(&tm.x, A.x, C, L, PTT_CH, R, false) ? 1 : 0;
+    if (!ok) return cudaErrorNotSupported;
+    constexpr int smem = pti_smem_bytes<T, MODE>();
+    cudaError_t e = cudaFuncSetAttribute(k_pthomas_il_tma<T, MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e != cudaSuccess) return e;
+    k_pthomas_il_tma<T, MODE><<<(unsigned)cdiv(C, PTT_CH), PTT_CH, smem, st>>>(tm, A, x_tma);
+    return cudaGetLastError();
+}
+
 template <typename T, int MODE>
 cudaError_t launch_pthomas_il(const tri_plan_s* p, const PThomasArgs<T>& A, cudaStream_t st) {
     const int64_t C = p->C, sms = p->sms;
+    if (C >= 32 * sms && !getenv("TRI_NO_TMA")) {
+        const cudaError_t et = launch_pthomas_il_tma<T, MODE>(p, A, st);
+        if (et != cudaErrorNotSupported) return et;
+    }
     if (C >= 32 * 8 * sms) {
         k_pthomas<T, MODE><<<(unsigned)cdiv(C, 128), 128, 0, st>>>(A);
         return cudaGetLastError();

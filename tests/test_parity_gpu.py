@@ -376,3 +376,24 @@ def test_split_k0_tma(cuda_ok, dtype, n, m):
         del os.environ["TRI_NO_TMA"]
     assert np.array_equal(x, x2)
     torch.cuda.synchronize()
+
+
+@pytest.mark.parametrize("dtype,n,m,layout,k", [("f64", 300, 5000, 1, 0), ("f64", 77, 4738, 1, 0),
+                                               ("f32", 200, 4800, 1, 0), ("f64", 1 << 16, 1, 0, 13),
+                                               ("f64", 70001, 1, 0, 13), ("f64", 3000, 3, 1, 11)])
+def test_chain_interleaved_tma(cuda_ok, dtype, n, m, layout, k):
+    """p-Thomas over chain-interleaved data through TMA (C = m 2^k >= 32 x SMs):
+    raw interleaved input at k = 0 (MODE 1) and tiled-PCR output (MODE 0), x by
+    TMA store where x is a 2D view; the fallback (ring kernel, continuant
+    forward sweep X18: different rounding) is checked against the oracle too."""
+    import os
+    arrs = gen(n, m, dtype, layout, "weak", eps=1e-2)
+    x, plan = gpu_solve(n, m, arrs, dtype, layout, k=k, variant=SPLIT)
+    xo = oracle.solve_batch(n, m, *arrs, layout=layout)
+    check_parity(n, m, arrs, x, dtype, layout, x_oracle=xo)
+    os.environ["TRI_NO_TMA"] = "1"
+    try:
+        x2 = plan.solve(*to_dev(*arrs)).cpu().numpy()
+    finally:
+        del os.environ["TRI_NO_TMA"]
+    check_parity(n, m, arrs, x2, dtype, layout, x_oracle=xo)
