@@ -41,9 +41,10 @@ __host__ __device__ inline int64_t halo_f(int k) { return (int64_t(1) << k) - 1;
 // (32-bit, one conditional wrap per step) instead of computed from row indices.
 template <int K>
 struct TPCRRing {
-    static constexpr int size(int j) { return TPCR_T + (2 << j); }
-    static constexpr int off(int j) { return j == 0 ? 0 : off(j - 1) + size(j - 1); }
-    static constexpr int total() { return off(K); }
+    // closed forms (no recursion: these must fold to immediates in the unrolled level loop)
+    __host__ __device__ static constexpr int size(int j) { return TPCR_T + (2 << j); }
+    __host__ __device__ static constexpr int off(int j) { return j * TPCR_T + (2 << j) - 2; }  // sum of sizes below j
+    __host__ __device__ static constexpr int total() { return off(K); }
 };
 
 template <typename T, int K>
