@@ -156,19 +156,25 @@ struct TiledILArgs {
     const T *iA, *iC, *iD;  // pass-1 output, [pos * C1 + ch], normalised rows
     T *oA, *oC, *oD;        // mode 0: chain-interleaved [pos2 * C + ch2]; mode 1: user layout
     int64_t n, m, L1, C1, C, region, nreg, nblk;
-    int layout, k1, k2, mode;
-    int ring_off[8];        // position offset of level j's ring
-    int ring_mask[8];
-    int ring_total;         // positions across all rings
+    int layout, k1, mode;
 };
 
-template <typename T>
+// ring j (positions): exactly TP + 2^(j+1), closed-form offsets (see TPCRRing)
+template <int K2>
+struct TPCRILRing {
+    __host__ __device__ static constexpr int size(int j) { return TPCR_IL_TP + (2 << j); }
+    __host__ __device__ static constexpr int off(int j) { return j * TPCR_IL_TP + (2 << j) - 2; }
+    __host__ __device__ static constexpr int total() { return off(K2); }
+};
+
+template <typename T, int K2>
 __global__ void __launch_bounds__(TPCR_T) k_tiled_pcr_il(TiledILArgs<T> p) {
     constexpr int CB = TPCR_IL_CB, TP = TPCR_IL_TP, RPT = TPCR_IL_RPT, UP = TPCR_T / CB;
+    using RG = TPCRILRing<K2>;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     T* rA = reinterpret_cast<T*>(smem_raw);
-    T* rC = rA + p.ring_total * CB;
-    T* rD = rC + p.ring_total * CB;
+    T* rC = rA + RG::total() * CB;
+    T* rD = rC + RG::total() * CB;
 
     const int tid = threadIdx.x;
     const int c = tid % CB, u0 = tid / CB;  // this thread: chain c, positions u0 + UP * h
@@ -177,13 +183,28 @@ __global__ void __launch_bounds__(TPCR_T) k_tiled_pcr_il(TiledILArgs<T> p) {
     const bool chok = ch < p.C1;
     const int64_t r0 = reg * p.region;
     const int64_t r1 = imin64(r0 + p.region, p.L1);
-    const int64_t fk = halo_f(p.k2);
+    constexpr int64_t fk = (int64_t(1) << K2) - 1;  // Eq 8 on the chain positions
     const int64_t start = r0 - fk;
-    const int k = p.k1 + p.k2;
+    const int k = p.k1 + K2;
     const int64_t S1 = int64_t(1) << p.k1;
     const int64_t q = ch >> p.k1, rr1 = ch & (S1 - 1);
 
-    for (int e = tid; e < p.ring_total * CB; e += TPCR_T) { rA[e] = T(0); rC[e] = T(0); rD[e] = T(0); }
+    for (int e = tid; e < RG::total() * CB; e += TPCR_T) { rA[e] = T(0); rC[e] = T(0); rD[e] = T(0); }
+    // slots (positions) of this thread's rows, advanced by TP per iteration:
+    // w0[h] in ring 0 for pos = s0 + u0 + UP h; rs[j][h] in ring j and ws[j][h]
+    // in ring j+1 for the row level j combines, pos_j = s0 - (2^(j+1) - 1) + u0 + UP h
+    const int64_t base = start - (int64_t(2) << K2);
+    int w0[RPT], rs[K2][RPT], ws[K2][RPT];
+#pragma unroll
+    for (int h = 0; h < RPT; ++h) {
+        w0[h] = (int)((start + u0 + UP * h - base) % RG::size(0));
+#pragma unroll
+        for (int j = 0; j < K2; ++j) {
+            const int64_t pj = start - ((int64_t(2) << j) - 1) + u0 + UP * h;
+            rs[j][h] = (int)((pj - base) % RG::size(j));
+            ws[j][h] = j + 1 < K2 ? (int)((pj - base) % RG::size(j + 1)) : 0;
+        }
+    }
     __syncthreads();
 
     NRow<T> nxt[RPT];  // next sub-tile's level-0 rows, loaded during this sub-tile's levels
@@ -202,49 +223,58 @@ __global__ void __launch_bounds__(TPCR_T) k_tiled_pcr_il(TiledILArgs<T> p) {
     for (int64_t s0 = start; s0 - fk < r1; s0 += TP) {
 #pragma unroll
         for (int h = 0; h < RPT; ++h) {
-            const int64_t pos = s0 + u0 + UP * h;
-            const int sl = (p.ring_off[0] + (int)(pos & p.ring_mask[0])) * CB + c;
+            const int sl = w0[h] * CB + c;
             rA[sl] = nxt[h].A; rC[sl] = nxt[h].C; rD[sl] = nxt[h].D;
         }
         fetch(s0 + TP);
         __syncthreads();
-        int64_t F = s0 + TP;
-        for (int j = 0; j < p.k2; ++j) {
-            const int sg = 1 << j;
-            F -= sg;
-            const int off = p.ring_off[j], msk = p.ring_mask[j];
+#pragma unroll
+        for (int j = 0; j < K2; ++j) {
+            const int Z = RG::size(j), O = RG::off(j), sg = 1 << j;
             NRow<T> nr[RPT];
 #pragma unroll
             for (int h = 0; h < RPT; ++h) {
-                const int64_t pos = F - TP + u0 + UP * h;
-                const int so = (off + (int)(pos & msk)) * CB + c;
-                const int sm = (off + (int)((pos - sg) & msk)) * CB + c;
-                const int sp = (off + (int)((pos + sg) & msk)) * CB + c;
+                int sm = rs[j][h] - sg; sm += sm < 0 ? Z : 0;
+                int sp = rs[j][h] + sg; sp -= sp >= Z ? Z : 0;
+                const int so = (O + rs[j][h]) * CB + c;
+                sm = (O + sm) * CB + c;
+                sp = (O + sp) * CB + c;
                 nr[h] = pcr_combine(NRow<T>{rA[sm], rC[sm], rD[sm]}, NRow<T>{rA[so], rC[so], rD[so]},
                                     NRow<T>{rA[sp], rC[sp], rD[sp]});
             }
 #pragma unroll
             for (int h = 0; h < RPT; ++h) {
-                const int64_t pos = F - TP + u0 + UP * h;
-                if (j + 1 < p.k2) {
-                    const int sd = (p.ring_off[j + 1] + (int)(pos & p.ring_mask[j + 1])) * CB + c;
+                if (j + 1 < K2) {
+                    const int sd = (RG::off(j + 1) + ws[j][h]) * CB + c;
                     rA[sd] = nr[h].A; rC[sd] = nr[h].C; rD[sd] = nr[h].D;
-                } else if (pos >= r0 && pos < r1 && chok) {
-                    const int64_t r = rr1 + ((pos & ((int64_t(1) << p.k2) - 1)) << p.k1);  // residue mod 2^k
-                    const int64_t pos2 = pos >> p.k2;
-                    if (p.mode == 0) {
-                        const int64_t idx = pos2 * p.C + (q << k) + r;
-                        p.oA[idx] = nr[h].A; p.oC[idx] = nr[h].C; p.oD[idx] = nr[h].D;
-                    } else {
-                        const int64_t i = (pos2 << k) + r;
-                        if (i < p.n) {
-                            const int64_t gi = elem_index(q, i, p.n, p.m, p.layout);
-                            p.oA[gi] = nr[h].A; p.oC[gi] = nr[h].C; p.oD[gi] = nr[h].D;
+                } else {
+                    const int64_t pos = s0 - ((int64_t(2) << j) - 1) + u0 + UP * h;
+                    if (pos >= r0 && pos < r1 && chok) {
+                        const int64_t r = rr1 + ((pos & ((int64_t(1) << K2) - 1)) << p.k1);  // residue mod 2^k
+                        const int64_t pos2 = pos >> K2;
+                        if (p.mode == 0) {
+                            const int64_t idx = pos2 * p.C + (q << k) + r;
+                            p.oA[idx] = nr[h].A; p.oC[idx] = nr[h].C; p.oD[idx] = nr[h].D;
+                        } else {
+                            const int64_t i = (pos2 << k) + r;
+                            if (i < p.n) {
+                                const int64_t gi = elem_index(q, i, p.n, p.m, p.layout);
+                                p.oA[gi] = nr[h].A; p.oC[gi] = nr[h].C; p.oD[gi] = nr[h].D;
+                            }
                         }
                     }
                 }
             }
             __syncthreads();
+        }
+#pragma unroll
+        for (int h = 0; h < RPT; ++h) {
+            w0[h] += TP; w0[h] -= w0[h] >= RG::size(0) ? RG::size(0) : 0;
+#pragma unroll
+            for (int j = 0; j < K2; ++j) {
+                rs[j][h] += TP; rs[j][h] -= rs[j][h] >= RG::size(j) ? RG::size(j) : 0;
+                if (j + 1 < K2) { ws[j][h] += TP; ws[j][h] -= ws[j][h] >= RG::size(j + 1) ? RG::size(j + 1) : 0; }
+            }
         }
     }
 }

@@ -34,6 +34,7 @@ int env_int(const char* name, int dflt) {
     return e ? std::max(1, atoi(e)) : dflt;
 }
 int g_tiled_waves1 = env_int("TRI_TILED_WAVES1", 1);
+int g_split_k1max = std::min(10, env_int("TRI_SPLIT_K1MAX", 10));  // steps kept in pass 1 (tuning)
 int g_tiled_waves2 = env_int("TRI_TILED_WAVES2", 3);  // measured best at c3 (1 / 3 waves)
 
 constexpr int ONCHIP_THREADS = 512;
@@ -176,20 +177,29 @@ int tiled_occ(int k1) {
         default: return tiled_occ_k<T, 10>();
     }
 }
-int tiled_il_smem(int k2, size_t es);
-template <typename T>
-int tiled_il_occ(int k2) {
-    const int smem = tiled_il_smem(k2, sizeof(T));
-    if (cudaFuncSetAttribute(k_tiled_pcr_il<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess) {
+template <typename T, int K2>
+int tiled_il_occ_k() {
+    const int smem = 3 * TPCRILRing<K2>::total() * TPCR_IL_CB * (int)sizeof(T);
+    if (cudaFuncSetAttribute(k_tiled_pcr_il<T, K2>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess) {
         cudaGetLastError();
         return 1;
     }
     int occ = 1;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_tiled_pcr_il<T>, TPCR_T, smem) != cudaSuccess) {
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_tiled_pcr_il<T, K2>, TPCR_T, smem) != cudaSuccess) {
         cudaGetLastError();
         occ = 1;
     }
     return std::max(1, occ);
+}
+template <typename T>
+int tiled_il_occ(int k2) {
+    switch (k2) {
+        case 1: return tiled_il_occ_k<T, 1>();
+        case 2: return tiled_il_occ_k<T, 2>();
+        case 3: return tiled_il_occ_k<T, 3>();
+        case 4: return tiled_il_occ_k<T, 4>();
+        default: return tiled_il_occ_k<T, 5>();
+    }
 }
 
 // ---- per-plan geometry -----------------------------------------------------
@@ -221,7 +231,8 @@ void plan_geometry(tri_plan_s* p) {
         p->L = cdiv(n, S);
         p->n_pad = p->L * S;
         p->C = m * S;
-        p->k1 = std::min(p->k, SPLIT_K1MAX);
+        p->k1 = std::min(p->k, g_split_k1max);
+        if (p->k - p->k1 > SPLIT_K2MAX) p->k1 = p->k - SPLIT_K2MAX;
         const int S1 = 1 << p->k1;
         p->L1 = cdiv(n, S1);
         p->C1 = m * S1;
@@ -293,18 +304,6 @@ tri_status ensure_scratch(tri_plan_s* p) {
     return TRI_OK;
 }
 
-int tiled_smem_layout(int k, int* off, int* mask, int tile = TPCR_T) {
-    int total = 0;
-    for (int j = 0; j < k; ++j) {
-        int need = tile + 2 * (1 << j);
-        int rs = 1;
-        while (rs < need) rs *= 2;
-        off[j] = total;
-        mask[j] = rs - 1;
-        total += rs;
-    }
-    return total;
-}
 
 // ---- launches ---------------------------------------------------------------
 template <typename T, int RPT>
@@ -390,9 +389,13 @@ cudaError_t launch_tiled(const tri_plan_s* p, const void* a, const void* b, cons
     }
 }
 
-int tiled_il_smem(int k2, size_t es) {
-    int off[8], mask[8];
-    return 3 * tiled_smem_layout(k2, off, mask, TPCR_IL_TP) * TPCR_IL_CB * (int)es;
+template <typename T, int K2>
+cudaError_t launch_tiled_il_k(const TiledILArgs<T>& A, int64_t grid, cudaStream_t st) {
+    const size_t smem = (size_t)3 * TPCRILRing<K2>::total() * TPCR_IL_CB * sizeof(T);
+    cudaError_t e = cudaFuncSetAttribute(k_tiled_pcr_il<T, K2>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    k_tiled_pcr_il<T, K2><<<(unsigned)grid, TPCR_T, smem, st>>>(A);
+    return cudaGetLastError();
 }
 
 template <typename T>
@@ -403,13 +406,16 @@ cudaError_t launch_tiled_il(const tri_plan_s* p, const void* iA, const void* iC,
     A.oA = (T*)oA; A.oC = (T*)oC; A.oD = (T*)oD;
     A.n = p->n; A.m = p->m; A.L1 = p->L1; A.C1 = p->C1; A.C = p->C;
     A.region = p->region2; A.nreg = p->nreg2; A.nblk = p->nblk2;
-    A.layout = p->layout; A.k1 = p->k1; A.k2 = p->k - p->k1; A.mode = mode;
-    A.ring_total = tiled_smem_layout(A.k2, A.ring_off, A.ring_mask, TPCR_IL_TP);
-    const size_t smem = (size_t)3 * A.ring_total * TPCR_IL_CB * sizeof(T);
-    cudaError_t e = cudaFuncSetAttribute(k_tiled_pcr_il<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return e;
-    k_tiled_pcr_il<T><<<(unsigned)(p->nblk2 * p->nreg2), TPCR_T, smem, st>>>(A);
-    return cudaGetLastError();
+    A.layout = p->layout; A.k1 = p->k1; A.mode = mode;
+    const int64_t grid = p->nblk2 * p->nreg2;
+    switch (p->k - p->k1) {
+        case 1: return launch_tiled_il_k<T, 1>(A, grid, st);
+        case 2: return launch_tiled_il_k<T, 2>(A, grid, st);
+        case 3: return launch_tiled_il_k<T, 3>(A, grid, st);
+        case 4: return launch_tiled_il_k<T, 4>(A, grid, st);
+        case 5: return launch_tiled_il_k<T, 5>(A, grid, st);
+        default: return cudaErrorInvalidValue;
+    }
 }
 
 template <typename T>
