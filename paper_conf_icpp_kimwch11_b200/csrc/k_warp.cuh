@@ -22,6 +22,9 @@ namespace tri {
 
 constexpr int WARP_K = 5;       // PCR steps = log2(32)
 constexpr int WARP_WPB = 4;     // warps (systems) per CTA
+#ifndef WARP_NO_PREFETCH
+#define WARP_NO_PREFETCH 0
+#endif
 
 template <typename T>
 struct WarpArgs {
@@ -70,6 +73,51 @@ __device__ __forceinline__ void warp_pcr_step(T (&A)[R], T (&C)[R], T (&D)[R], i
 // goes back the same way.
 constexpr int WARP_WPB_IL = 8;
 
+// measured (B200): fp32 R = 8 (c4) 1.83 -> 1.49 ms with the prefetch; fp64 R = 4
+// 1.36 -> 1.60 ms (the doubled registers cost more occupancy than the overlap
+// gains), larger R spill
+template <typename T, int R>
+__host__ __device__ constexpr bool warp_persistent() {
+    return sizeof(T) == 4 && R <= 8 && !WARP_NO_PREFETCH;
+}
+
+// PCR stage + p-Thomas on one system held in registers, then x (or, in PCR
+// debug mode, the reduced rows) to [base + i * stride]
+template <typename T, int R>
+__device__ __forceinline__ void warp_solve_and_store(const WarpArgs<T>& p, T (&A)[R], T (&C)[R], T (&D)[R], int lane,
+                                                     int64_t base, int64_t stride) {
+    const int64_t n = p.n;
+    warp_pcr_step<T, R, 1>(A, C, D, lane);
+    warp_pcr_step<T, R, 2>(A, C, D, lane);
+    warp_pcr_step<T, R, 4>(A, C, D, lane);
+    warp_pcr_step<T, R, 8>(A, C, D, lane);
+    warp_pcr_step<T, R, 16>(A, C, D, lane);
+    if (p.mode == 1) {
+#pragma unroll
+        for (int t = 0; t < R; ++t) {
+            const int64_t i = (int64_t)t * 32 + lane;
+            if (i < n) {
+                const int64_t e = base + i * stride;
+                p.ao[e] = A[t]; p.co[e] = C[t]; p.do_[e] = D[t];
+            }
+        }
+        return;
+    }
+    T cp = T(0), dp = T(0);
+#pragma unroll
+    for (int t = 0; t < R; ++t) {
+        thomas_fwd(NRow<T>{A[t], C[t], D[t]}, cp, dp);
+        C[t] = cp; D[t] = dp;
+    }
+    T xv = T(0);
+#pragma unroll
+    for (int t = R - 1; t >= 0; --t) {
+        xv = fma(-C[t], xv, D[t]);
+        const int64_t i = (int64_t)t * 32 + lane;
+        if (i < n) p.x[base + i * stride] = xv;
+    }
+}
+
 template <typename T, int R, bool IL>
 __global__ void __launch_bounds__((IL ? WARP_WPB_IL : WARP_WPB) * 32) k_warp(WarpArgs<T> p) {
     constexpr int WPB = IL ? WARP_WPB_IL : WARP_WPB;
@@ -84,21 +132,37 @@ __global__ void __launch_bounds__((IL ? WARP_WPB_IL : WARP_WPB) * 32) k_warp(War
     if constexpr (!IL) {
         // load + normalise (reading X17); a_0 and c_{n-1} are ignored (never
         // read into arithmetic), rows >= n are zero rows
+        T ra[R], rb[R], rc[R], rd[R];
+        auto load = [&](int64_t bq) {
 #pragma unroll
-        for (int t = 0; t < R; ++t) {
-            const int64_t i = (int64_t)t * 32 + lane;
-            if (i < n) {
-                const int64_t e = base + i;
-                const T av = ldg_stream(p.a + e), bv = ldg_stream(p.b + e);
-                const T cv = ldg_stream(p.c + e), dv = ldg_stream(p.d + e);
-                const T r = rcp(bv);
-                A[t] = i > 0 ? av * r : T(0);
-                C[t] = i < n - 1 ? cv * r : T(0);
-                D[t] = dv * r;
-            } else {
-                A[t] = T(0); C[t] = T(0); D[t] = T(0);
+            for (int t = 0; t < R; ++t) {
+                const int64_t i = (int64_t)t * 32 + lane;
+                const bool in = i < n;
+                const int64_t e = bq + i;
+                ra[t] = in ? ldg_stream(p.a + e) : T(0);
+                rb[t] = in ? ldg_stream(p.b + e) : T(1);
+                rc[t] = in ? ldg_stream(p.c + e) : T(0);
+                rd[t] = in ? ldg_stream(p.d + e) : T(0);
             }
+        };
+        load(base);
+        // persistent warps (small R): the next system's rows are in flight while
+        // this one is reduced and solved; large R: one system per warp (the
+        // doubled register footprint would spill)
+        const int64_t qstride = warp_persistent<T, R>() ? (int64_t)gridDim.x * WPB : p.m;
+        for (int64_t qq = q; qq < p.m; qq += qstride) {
+#pragma unroll
+            for (int t = 0; t < R; ++t) {
+                const int64_t i = (int64_t)t * 32 + lane;
+                const T r = rcp(rb[t]);
+                A[t] = i > 0 && i < n ? ra[t] * r : T(0);
+                C[t] = i < n - 1 ? rc[t] * r : T(0);
+                D[t] = rd[t] * r;
+            }
+            if (warp_persistent<T, R>() && qq + qstride < p.m) load((qq + qstride) * n);
+            warp_solve_and_store<T, R>(p, A, C, D, lane, qq * n, 1);
         }
+        return;
     } else {
         __shared__ T tile[4][WPB][33];
         const int th = threadIdx.x;
@@ -163,14 +227,7 @@ __global__ void __launch_bounds__((IL ? WARP_WPB_IL : WARP_WPB) * 32) k_warp(War
         C[t] = cp; D[t] = dp;
     }
     T xv = T(0);
-    if constexpr (!IL) {
-#pragma unroll
-        for (int t = R - 1; t >= 0; --t) {
-            xv = fma(-C[t], xv, D[t]);
-            const int64_t i = (int64_t)t * 32 + lane;
-            if (i < n) p.x[base + i] = xv;
-        }
-    } else {
+    {
         __shared__ T xt[WPB][33];
         const int th = threadIdx.x;
         const int tq = th % WPB, tr = th / WPB;

@@ -342,11 +342,22 @@ cudaError_t launch_warp(const tri_plan_s* p, const void* a, const void* b, const
     A.n = p->n; A.m = p->m; A.layout = p->layout; A.mode = mode;
     const bool il = p->layout == TRI_LAYOUT_INTERLEAVED && p->m > 1;
     const int wpb = il ? WARP_WPB_IL : WARP_WPB;
-    const unsigned grid = (unsigned)cdiv(p->m, wpb);
+    const int64_t need = cdiv(p->m, wpb);
+    // contiguous: persistent warps (one resident wave), each walking systems
+    // q, q + grid*WPB, ... with the next system's loads in flight
+    auto contig_grid = [&](auto kern) {
+        int occ = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, wpb * 32, 0) != cudaSuccess || occ < 1) {
+            cudaGetLastError();
+            occ = 1;
+        }
+        return (unsigned)std::min<int64_t>(need, (int64_t)occ * p->sms);
+    };
 #define TRI_WARP_CASE(R)                                                                  \
     case R:                                                                               \
-        if (il) k_warp<T, R, true><<<grid, wpb * 32, 0, st>>>(A);                         \
-        else k_warp<T, R, false><<<grid, wpb * 32, 0, st>>>(A);                           \
+        if (il) k_warp<T, R, true><<<(unsigned)need, wpb * 32, 0, st>>>(A);               \
+        else k_warp<T, R, false><<<warp_persistent<T, R>() ? contig_grid(k_warp<T, R, false>) : (unsigned)need, \
+                                   wpb * 32, 0, st>>>(A);                                 \
         break;
     switch (p->rpt) {
         TRI_WARP_CASE(1) TRI_WARP_CASE(2) TRI_WARP_CASE(4) TRI_WARP_CASE(8) TRI_WARP_CASE(16) TRI_WARP_CASE(32)
