@@ -70,8 +70,7 @@ int onchip_G(int64_t n, int64_t m, tri_dtype t, int sms) {
     return (int)G;
 }
 
-// FUSED needs the contiguous layout (or m = 1) and enough systems to give
-// every SM its own (one system per CTA at a time).
+// FUSED needs the contiguous layout (or m = 1) and systems of >= 2 windows.
 bool fused_ok(int64_t n, int64_t m, tri_layout layout) {
     return (layout == TRI_LAYOUT_CONTIGUOUS || m == 1) && n >= 2 * FU_W;
 }
@@ -80,23 +79,32 @@ bool fused_ok(int64_t n, int64_t m, tri_layout layout) {
 constexpr int64_t WARP_RMAX = 32;
 bool warp_ok(int64_t n) { return n >= 32 && n <= 32 * WARP_RMAX; }
 
+// Variant choice, calibrated once on B200 (the paper tunes P once) from
+// scripts/sweep_k.py (profiles/r01_sweep_k_*.jsonl): every (variant, k) timed
+// over the paper's shape grid (fixed n with m swept, fixed m with n swept).
+//   * m >= 48 x SMs: straight to p-Thomas (paper rule M > P) -- the TMA
+//     k = 0 kernel moves 9 arrays at ~86 % of the copy bandwidth and beats every
+//     PCR variant there (n = 256..16384; e.g. n = 2048, m = 16384: 438 us vs
+//     1266 us ONCHIP; n = 16384: FUSED wins at m = 4096, k = 0 from m = 8192);
+//   * contiguous, n >= 1024 and (n <= 2048 or m >= 128): FUSED (n = 1024..16384,
+//     m = 1..2048: 1.0-1.65x faster than ONCHIP/WARP/SPLIT);
+//   * 32 <= n <= 1024 with many systems: WARP (contiguous from m = 1024, where
+//     it overtakes ONCHIP; interleaved from one system per SM);
+//   * whole systems that fit a CTA's smem: ONCHIP;
+//   * otherwise (few large systems): SPLIT with k from choose_k_for.
 tri_variant choose_variant(int64_t n, int64_t m, tri_dtype t, tri_layout layout, int sms) {
-    // one warp per system once the batch covers every SM; below that a whole
-    // CTA per system (ONCHIP) shortens the latency chain (measured: n = 1024,
-    // m = 1: ONCHIP 10 us vs WARP 19 us; m = 1024: WARP 31 us vs ONCHIP 76 us)
-    if (warp_ok(n) && m >= sms) return TRI_VARIANT_WARP;
+    if (m >= 48 * (int64_t)sms) return TRI_VARIANT_SPLIT;
+    const bool contig = layout == TRI_LAYOUT_CONTIGUOUS;
+    if (contig && fused_ok(n, m, layout) && n >= 1024 && (n <= 2048 || m >= 128)) return TRI_VARIANT_FUSED;
+    if (warp_ok(n) && m >= (contig ? 1024 : (int64_t)sms)) return TRI_VARIANT_WARP;
     if (n <= onchip_rows_budget(t)) return TRI_VARIANT_ONCHIP;
-    // paper rule: with more systems than the machine's parallelism go
-    // straight to p-Thomas (k = 0); between one system per SM and that point
-    // the fused streaming kernel supplies the chains.
-    if (m >= 64 * (int64_t)sms) return TRI_VARIANT_SPLIT;
-    if (fused_ok(n, m, layout) && m >= sms) return TRI_VARIANT_FUSED;
     return TRI_VARIANT_SPLIT;
 }
 
-// Paper rule: M > P => k = 0; M <= P => the largest k with 2^k M <= P,
-// P the machine's effective parallelism.  B200: P_eff = SMs x chains per SM
-// needed to cover the Thomas recurrence latency.
+// Transition point.  Paper rule: M > P => k = 0; otherwise the largest k
+// with 2^k M <= P; B200 P = 64 chains per SM.  Measured refinement: below P the
+// extra PCR steps stop paying once the subsystems are ~32 rows long (n = 8192,
+// m = 1: k = 8 in 25 us vs k = 13 in 76 us), so k <= floor(log2 n) - 5.
 int choose_k_for(tri_variant v, int64_t n, int64_t m, tri_dtype t, tri_layout layout, int sms) {
     const int kmax_n = floor_log2(n);
     if (v == TRI_VARIANT_ONCHIP) {
@@ -107,7 +115,9 @@ int choose_k_for(tri_variant v, int64_t n, int64_t m, tri_dtype t, tri_layout la
     if (v == TRI_VARIANT_FUSED) return FU_K;
     if (v == TRI_VARIANT_WARP) return WARP_K;
     const int64_t P = (int64_t)sms * 64;
+    if (m >= 48 * (int64_t)sms) return 0;
     int k = m >= P ? 0 : ceil_log2(cdiv(P, m));
+    k = std::min(k, std::max(0, kmax_n - 5));
     return std::min(std::min(k, kmax_n), SPLIT_KMAX);
 }
 

@@ -324,10 +324,11 @@ def test_warp_families(cuda_ok, family, eps):
 
 
 def test_warp_large_batch_sampled(cuda_ok):
-    """c4-shaped batch (n = 256, fp32, m = 2^18): sampled systems vs the oracle."""
+    """Large batch through WARP (n = 256, fp32, m = 2^18; persistent warps with
+    next-system prefetch): sampled systems vs the oracle."""
     n, m = 256, 1 << 18
     arrs = gen(n, m, "f32", 0)
-    x, plan = gpu_solve(n, m, arrs, "f32", 0)
+    x, plan = gpu_solve(n, m, arrs, "f32", 0, variant=WARP)
     assert plan.variant == WARP
     rng = np.random.default_rng(5)
     for q in rng.choice(m, 64, replace=False).tolist() + [0, m - 1]:
@@ -397,3 +398,19 @@ def test_chain_interleaved_tma(cuda_ok, dtype, n, m, layout, k):
     finally:
         del os.environ["TRI_NO_TMA"]
     check_parity(n, m, arrs, x2, dtype, layout, x_oracle=xo)
+
+
+@pytest.mark.parametrize("layout", [0, 1])
+def test_c4_auto_plan_sampled(cuda_ok, layout):
+    """BASELINE config c4 at full size (n = 256, m = 2^20, fp32) through the auto
+    plan (M > P: k = 0, TMA-streamed p-Thomas): sampled systems vs the oracle."""
+    import trigen
+    n, m = 256, 1 << 20
+    arrs = gen(n, m, "f32", layout, seed=trigen.SEED_BASE + 4)
+    x, plan = gpu_solve(n, m, arrs, "f32", layout)
+    assert plan.variant == SPLIT and plan.k == 0
+    rng = np.random.default_rng(4)
+    for q in rng.choice(m, 48, replace=False).tolist() + [0, m - 1]:
+        sub = trigen.generate(n, 1, "f32", 0, "dd", seed=trigen.SEED_BASE + 4, q0=q)
+        xs = x.reshape(m, n)[q] if layout == 0 else x.reshape(n, m)[:, q]
+        check_parity(n, 1, sub, xs, "f32", 0)
