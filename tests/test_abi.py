@@ -107,3 +107,19 @@ def test_shard_range_partitions(L, m, G):
         assert mr >= 0
         covered += list(range(q0, q0 + mr))
     assert covered == list(range(m))
+
+
+@pytest.mark.parametrize("cfg,n,m,dtype,layout,variant,k", [
+    ("c1", 1024, 1, "F64", 0, "VARIANT_FUSED", 4),
+    ("c2", 1024, 1024, "F64", 1, "VARIANT_WARP", 5),
+    ("c3", 1 << 24, 1, "F64", 0, "VARIANT_SPLIT", 14),
+    ("c4", 256, 1 << 20, "F32", 0, "VARIANT_SPLIT", 0),
+    ("c5", 16384, 16384, "F64", 0, "VARIANT_SPLIT", 0),
+    ("c5/8", 16384, 2048, "F64", 0, "VARIANT_FUSED", 4),   # one of 8 ranks (strong scaling)
+])
+def test_planner_picks_for_baseline_configs(L, cfg, n, m, dtype, layout, variant, k):
+    """The planner's (variant, k) on a 148-SM B200 for BASELINE.json's configs,
+    as calibrated by scripts/sweep_k.py (profiles/r01_sweep_k_*.jsonl)."""
+    dt = getattr(tri, dtype)
+    assert tri.choose_variant(n, m, dt, layout, 148) == getattr(tri, variant), cfg
+    assert tri.choose_k(n, m, dt, layout, 148) == k, cfg
