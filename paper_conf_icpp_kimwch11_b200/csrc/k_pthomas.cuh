@@ -29,6 +29,7 @@ struct PThomasArgs {
     T *cps, *dps;             // scratch: c', d' interleaved [j*C + ch]
     int64_t n, m, C, L;       // C chains, L positions per chain
     int layout, k;
+    int discard;              // TMA kernels: L2-discard consumed c', d' lines (rows 128-B aligned)
 };
 
 constexpr int PT_U = 4;  // rows prefetched ahead in modes 0/1

@@ -33,11 +33,16 @@ struct PTTCfg {
     static constexpr int TILE = PTT_CH * R;            // elements per array tile
     static constexpr int FSTAGE = 4 * TILE;            // forward stage: a, b, c, d
     static constexpr int BSTAGE = 2 * TILE;            // backward stage: c', d'
+    // forward ring stages: fp64 3 (16 KB each); fp32 2 (n = 256-class systems are
+    // 8 tiles long: more resident CTAs beat a deeper ring; c4 measured)
+    static constexpr int NS = sizeof(T) == 8 ? 3 : 2;
+    static constexpr int NB = 3;                       // backward stages (+ 2 x tiles fit the forward ring)
+    static_assert(NB * BSTAGE + 2 * TILE <= NS * FSTAGE, "backward ring must fit the forward ring");
 };
 
 template <typename T>
 __host__ __device__ constexpr int ptt_smem_bytes() {
-    return PTT_NS * PTTCfg<T>::FSTAGE * (int)sizeof(T) + 1024;  // + alignment slack (128B swizzle)
+    return PTTCfg<T>::NS * PTTCfg<T>::FSTAGE * (int)sizeof(T) + 1024;  // + alignment slack (128B swizzle)
 }
 
 __device__ __forceinline__ void ptt_bar_init(uint64_t* bar) {
@@ -74,6 +79,13 @@ __device__ __forceinline__ void ptt_store(const CUtensorMap* tm, int x0, int x1,
                  : "memory");
 }
 
+// Drop a consumed scratch line from L2 without writing it back (the c', d'
+// intermediates are dead once the back substitution has read them: without
+// this, every dirty line still costs a DRAM write when L2 evicts it).
+__device__ __forceinline__ void l2_discard(const void* p) {
+    asm volatile("discard.global.L2 [%0], 128;" ::"l"(p) : "memory");
+}
+
 // Offset (elements) of row u of system s inside a 128B-swizzled [32][R] tile:
 // 16-byte chunk j of 128-byte row s lives at chunk j ^ (s & 7).
 template <typename T>
@@ -92,24 +104,25 @@ template <typename T>
 __global__ void __launch_bounds__(PTT_CH) k_pthomas_tma(const __grid_constant__ PTTMaps tm, PThomasArgs<T> p) {
     constexpr int R = PTTCfg<T>::R, EPC = PTTCfg<T>::EPC, TILE = PTTCfg<T>::TILE;
     constexpr int FSTAGE = PTTCfg<T>::FSTAGE, BSTAGE = PTTCfg<T>::BSTAGE;
+    constexpr int NS_ = PTTCfg<T>::NS, NB_ = PTTCfg<T>::NB;
     extern __shared__ unsigned char smem_raw[];
     T* sm = reinterpret_cast<T*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-    __shared__ uint64_t fbar[PTT_NS], bbar[PTT_NB];
+    __shared__ uint64_t fbar[NS_], bbar[NB_];
     const int t = threadIdx.x;
     const int q0 = blockIdx.x * PTT_CH;
     const bool active = q0 + t < p.m;
     const int64_t n = p.n, M = p.m;
     const int ntile = (int)((n + R - 1) / R);
     if (t == 0) {
-        for (int s = 0; s < PTT_NS; ++s) ptt_bar_init(&fbar[s]);
-        for (int s = 0; s < PTT_NB; ++s) ptt_bar_init(&bbar[s]);
+        for (int s = 0; s < NS_; ++s) ptt_bar_init(&fbar[s]);
+        for (int s = 0; s < NB_; ++s) ptt_bar_init(&bbar[s]);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncwarp();
 
     auto issue_f = [&](int tt) {
         if (t == 0 && tt < ntile) {
-            const int s = tt % PTT_NS;
+            const int s = tt % NS_;
             T* st = sm + s * FSTAGE;
             fence_proxy_async_smem();
             ptt_expect(&fbar[s], FSTAGE * (unsigned)sizeof(T));
@@ -119,13 +132,13 @@ __global__ void __launch_bounds__(PTT_CH) k_pthomas_tma(const __grid_constant__ 
             ptt_load(st + 3 * TILE, &tm.d, tt * R, q0, &fbar[s]);
         }
     };
-    for (int s = 0; s < PTT_NS; ++s) issue_f(s);
+    for (int s = 0; s < NS_; ++s) issue_f(s);
 
     // ---- forward sweep (Eqs 2-3)
     T cp = T(0), dp = T(0);
     for (int tt = 0; tt < ntile; ++tt) {
-        const int s = tt % PTT_NS;
-        ptt_wait(&fbar[s], (unsigned)((tt / PTT_NS) & 1));
+        const int s = tt % NS_;
+        ptt_wait(&fbar[s], (unsigned)((tt / NS_) & 1));
         const T* st = sm + s * FSTAGE;
         T v[4][R];
 #pragma unroll
@@ -138,7 +151,7 @@ __global__ void __launch_bounds__(PTT_CH) k_pthomas_tma(const __grid_constant__ 
                 for (int e = 0; e < EPC; ++e) v[arr][ck * EPC + e] = wt[e];
             }
         __syncwarp();
-        issue_f(tt + PTT_NS);  // slot s consumed (values are in registers)
+        issue_f(tt + NS_);  // slot s consumed (values are in registers)
         const int64_t j0 = (int64_t)tt * R;
         T* cps = p.cps + j0 * M + q0 + t;
         T* dps = p.dps + j0 * M + q0 + t;
@@ -167,10 +180,10 @@ __global__ void __launch_bounds__(PTT_CH) k_pthomas_tma(const __grid_constant__ 
     __threadfence_block();
     asm volatile("fence.proxy.async.global;" ::: "memory");
     __syncwarp();
-    T* xt = sm + PTT_NB * BSTAGE;  // 2 x TILE, swizzled [32][R]
+    T* xt = sm + NB_ * BSTAGE;  // 2 x TILE, swizzled [32][R]
     auto issue_b = [&](int b) {
         if (t == 0 && b < ntile) {
-            const int s = b % PTT_NB;
+            const int s = b % NB_;
             const int tt = ntile - 1 - b;
             T* st = sm + s * BSTAGE;
             fence_proxy_async_smem();
@@ -179,20 +192,28 @@ __global__ void __launch_bounds__(PTT_CH) k_pthomas_tma(const __grid_constant__ 
             ptt_load(st + TILE, &tm.dp, q0, tt * R, &bbar[s]);
         }
     };
-    for (int s = 0; s < PTT_NB; ++s) issue_b(s);
+    for (int s = 0; s < NB_; ++s) issue_b(s);
     T xv = T(0);
     for (int b = 0; b < ntile; ++b) {
-        const int s = b % PTT_NB;
+        const int s = b % NB_;
         const int tt = ntile - 1 - b;
-        ptt_wait(&bbar[s], (unsigned)((b / PTT_NB) & 1));
+        ptt_wait(&bbar[s], (unsigned)((b / NB_) & 1));
         const T* st = sm + s * BSTAGE;   // [R positions][32 systems] per array
         T cs[R], ds[R];
 #pragma unroll
         for (int u = 0; u < R; ++u) { cs[u] = st[u * PTT_CH + t]; ds[u] = st[TILE + u * PTT_CH + t]; }
+        if (p.discard && t < R && (int64_t)tt * R + t < n) {  // lane u drops row u's lines (32 systems)
+            const int64_t off = ((int64_t)tt * R + t) * M + q0;
+#pragma unroll
+            for (int h = 0; h < PTT_CH * (int)sizeof(T) / 128; ++h) {
+                l2_discard(p.cps + off + h * (128 / (int)sizeof(T)));
+                l2_discard(p.dps + off + h * (128 / (int)sizeof(T)));
+            }
+        }
         // the x tile written two tiles ago must have been read out by its TMA store
         if (t == 0) bulk_wait_read<1>();
         __syncwarp();
-        issue_b(b + PTT_NB);
+        issue_b(b + NB_);
         T* xb = xt + (b & 1) * TILE;
         const int64_t j0 = (int64_t)tt * R;
 #pragma unroll

@@ -589,6 +589,9 @@ cudaError_t launch_split(const tri_plan_s* p, const void* a, const void* b, cons
     A.a = (const T*)a; A.b = (const T*)b; A.c = (const T*)c; A.d = (const T*)d;
     A.x = (T*)x;
     A.n = p->n; A.m = p->m; A.C = p->C; A.L = p->L; A.layout = p->layout; A.k = p->k;
+    // 32 chains x s bytes per scratch row segment start on 128-byte lines when
+    // the row pitch C s is a multiple of 128 (and the scratch base is 256-aligned)
+    A.discard = ((p->C * (int64_t)sizeof(T)) % 128 == 0 && !getenv("TRI_NO_DISCARD")) ? 1 : 0;
     if (p->k > 0) {
         T *rA = base, *rC = base + ce, *rD = base + 2 * ce;
         cudaError_t e;
