@@ -65,8 +65,12 @@ typedef enum {
     TRI_VARIANT_ONCHIP = 1, /* whole system(s) in one CTA's smem: PCR + Thomas (Fig 11a/c) */
     TRI_VARIANT_SPLIT = 2,  /* tiled-PCR pass (sliding window, Figs 8-10) -> scratch, then p-Thomas */
     TRI_VARIANT_FUSED = 3,  /* streaming tiled PCR feeding p-Thomas in one kernel (Sec. III.C) */
-    TRI_VARIANT_WARP = 4    /* 32 <= n <= 1024: one warp per system, k = 5 shuffle PCR steps + in-register
+    TRI_VARIANT_WARP = 4,   /* 32 <= n <= 1024: one warp per system, k = 5 shuffle PCR steps + in-register
                                p-Thomas on the 32 subsystems (Sec. III) */
+    TRI_VARIANT_STREAM = 5  /* CONTIGUOUS fp64, n % 8 == 0, n >= 512: tiled PCR (k = 3, TMA-staged 256-row
+                               windows with 8-row halos, Eq 8 / Fig 7) streamed into p-Thomas in one
+                               persistent kernel; c', d' stay in shared memory / L2, so HBM moves only
+                               the compulsory 5 arrays (Sec. III.C) */
 } tri_variant;
 
 typedef struct tri_plan_s* tri_plan_t;

@@ -10,19 +10,17 @@ __host__ __device__ __forceinline__ int64_t imin64(int64_t a, int64_t b) { retur
 __host__ __device__ __forceinline__ int64_t imax64(int64_t a, int64_t b) { return a > b ? a : b; }
 
 // Reciprocal used for every division of the method (Eqs 2-6).  fp64: MUFU seed
-// (rcp.approx) refined by two Newton steps on the FMA pipe (~1 ulp); fp32: the
-// MUFU result itself (<= 1 ulp, far inside the 1e-4 fp32 tolerance; one MUFU
-// instead of MUFU + 2 FFMA per division).  Pure mantissa arithmetic, so scaling the
+// (rcp.approx, relative error e0 < 2^-22) refined by one cubic Newton step on the
+// FMA pipe, r (1 + e + e^2) with e = 1 - x r: error O(e0^3) below fp64 rounding,
+// ~1 ulp, three dependent FMAs; fp32: the MUFU result itself (<= 1 ulp, far
+// inside the 1e-4 fp32 tolerance).  Pure mantissa arithmetic, so scaling the
 // argument by 2^p scales the result by 2^-p exactly (metamorphic tests rely on
 // it).  Inputs are pivots of diagonally dominant systems: never 0/denormal.
 __device__ __forceinline__ double rcp(double x) {
     double r;
     asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(r) : "d"(x));
-    double e = fma(-x, r, 1.0);
-    r = fma(r, e, r);
-    e = fma(-x, r, 1.0);
-    r = fma(r, e, r);
-    return r;
+    const double e = fma(-x, r, 1.0);
+    return fma(r, fma(e, e, e), r);
 }
 __device__ __forceinline__ float rcp(float x) {
     float r;

@@ -18,6 +18,7 @@
 #include "k_tiled_pcr.cuh"
 #include "k_pthomas.cuh"
 #include "k_fused.cuh"
+#include "k_stream.cuh"
 #include "k_warp.cuh"
 #include "k_pthomas_tma.cuh"
 
@@ -79,6 +80,14 @@ bool fused_ok(int64_t n, int64_t m, tri_layout layout) {
 constexpr int64_t WARP_RMAX = 32;
 bool warp_ok(int64_t n) { return n >= 32 && n <= 32 * WARP_RMAX; }
 
+// STREAM: fp64, contiguous (or one system), n a multiple of 8 (the TMA tensor
+// view [rows/8][8]), 8 .. 1024 windows of 240 rows (slot barriers, k_stream.cuh);
+// tensor rows fit int32.
+bool stream_ok(int64_t n, int64_t m, tri_dtype t, tri_layout layout) {
+    return t == TRI_F64 && (layout == TRI_LAYOUT_CONTIGUOUS || m == 1) && n % 8 == 0 && n >= 2 * SK_W &&
+           cdiv(n, SK_V) >= 8 && cdiv(n, SK_V) <= SK_NCMAX && (n / 8) * m < ((int64_t)1 << 31);
+}
+
 // Variant choice, calibrated once on B200 (the paper tunes P once) from
 // scripts/sweep_k.py (profiles/r01_sweep_k_*.jsonl): every (variant, k) timed
 // over the paper's shape grid (fixed n with m swept, fixed m with n swept).
@@ -113,6 +122,7 @@ int choose_k_for(tri_variant v, int64_t n, int64_t m, tri_dtype t, tri_layout la
         return std::min(k, kmax_n);
     }
     if (v == TRI_VARIANT_FUSED) return FU_K;
+    if (v == TRI_VARIANT_STREAM) return SK_K;
     if (v == TRI_VARIANT_WARP) return WARP_K;
     const int64_t P = (int64_t)sms * 64;
     if (m >= 48 * (int64_t)sms) return 0;
@@ -124,10 +134,13 @@ int choose_k_for(tri_variant v, int64_t n, int64_t m, tri_dtype t, tri_layout la
 int kmax_for(tri_variant v, int64_t n) {
     const int kn = floor_log2(n);
     if (v == TRI_VARIANT_FUSED) return FU_K;
+    if (v == TRI_VARIANT_STREAM) return SK_K;
     if (v == TRI_VARIANT_WARP) return WARP_K;
     return v == TRI_VARIANT_SPLIT ? std::min(kn, SPLIT_KMAX) : kn;
 }
-int kmin_for(tri_variant v) { return v == TRI_VARIANT_FUSED ? FU_K : v == TRI_VARIANT_WARP ? WARP_K : 0; }
+int kmin_for(tri_variant v) {
+    return v == TRI_VARIANT_FUSED ? FU_K : v == TRI_VARIANT_STREAM ? SK_K : v == TRI_VARIANT_WARP ? WARP_K : 0;
+}
 
 }  // namespace
 
@@ -147,6 +160,7 @@ struct tri_plan_s {
     int fu_grid, fu_son;      // FUSED: persistent CTAs, on-chip positions per chain
     bool fu_vec;              // FUSED: staged 8-row-aligned path
     int64_t fu_nc;            // FUSED: windows per system
+    int sk_grid, sk_nc, sk_son;  // STREAM: persistent CTAs, windows per system, resident storage slots
     size_t smem_optin;
     void* scratch;
     size_t scratch_bytes;
@@ -272,6 +286,15 @@ void plan_geometry(tri_plan_s* p) {
         }
         p->G = 0; p->P = 0; p->rpt = 0;
     }
+    if (p->variant == TRI_VARIANT_STREAM) {
+        p->L = cdiv(n, SK_S);
+        p->n_pad = p->L * SK_S;
+        p->C = m * SK_S;
+        p->sk_nc = (int)cdiv(n, SK_V);
+        p->sk_grid = (int)std::min<int64_t>(m, p->sms);
+        const int64_t avail = ((int64_t)p->smem_optin - SKLayout<double>::off_store - 1024) / SKLayout<double>::slot_bytes;
+        p->sk_son = (int)std::max<int64_t>(0, std::min<int64_t>(p->sk_nc, avail));
+    }
     if (p->variant == TRI_VARIANT_FUSED) {
         const size_t s = esize(p->dtype);
         p->L = cdiv(n, FU_S);
@@ -289,6 +312,8 @@ void plan_geometry(tri_plan_s* p) {
 }
 
 size_t scratch_need(const tri_plan_s* p) {
+    if (p->variant == TRI_VARIANT_STREAM)
+        return (size_t)p->sk_grid * (size_t)std::max(0, p->sk_nc - p->sk_son) * SK_SLOT * esize(p->dtype);
     if (p->variant == TRI_VARIANT_FUSED)
         return (size_t)p->fu_grid * 2 * (size_t)std::max<int64_t>(0, p->L - p->fu_son) * FU_S * 2 * esize(p->dtype);
     if (p->variant != TRI_VARIANT_SPLIT) return 0;
@@ -489,6 +514,41 @@ bool tma_map_2d(CUtensorMap* tm, const void* base, uint64_t d0, uint64_t d1, uin
                const_cast<void*>(base), dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
                swz ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+// ---- STREAM launch: tensor maps [n m / 8][8] (64-byte rows, 64B swizzle, box 8 x 32)
+bool tma_map_rows8(CUtensorMap* tm, const void* base, uint64_t rows8) {
+    auto enc = tma_encoder();
+    if (!enc) return false;
+    cuuint64_t dims[2] = {8, rows8};
+    cuuint64_t strides[1] = {8 * sizeof(double)};
+    cuuint32_t box[2] = {8, 32};
+    cuuint32_t es[2] = {1, 1};
+    return enc(tm, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 2, const_cast<void*>(base), dims, strides, box, es,
+               CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+cudaError_t launch_stream(const tri_plan_s* p, const void* a, const void* b, const void* c, const void* d, void* x,
+                          cudaStream_t st, void* ao = nullptr, void* co = nullptr, void* do_ = nullptr) {
+    StreamMaps tm;
+    const uint64_t rows8 = (uint64_t)(p->n / 8) * (uint64_t)p->m;
+    if (!tma_map_rows8(&tm.a, a, rows8) || !tma_map_rows8(&tm.b, b, rows8) || !tma_map_rows8(&tm.c, c, rows8) ||
+        !tma_map_rows8(&tm.d, d, rows8))
+        return cudaErrorNotSupported;
+    StreamArgs<double> A;
+    A.x = (double*)x;
+    A.spill = (double*)p->scratch;
+    A.n = p->n; A.m = p->m; A.NC = p->sk_nc; A.S_on = p->sk_son;
+    A.dA = (double*)ao; A.dC = (double*)co; A.dD = (double*)do_;
+    A.prof = (unsigned long long*)g_fused_prof;
+    A.dbg = g_fused_dbg_mode;
+    const size_t smem = (size_t)SKLayout<double>::off_store + (size_t)p->sk_son * SKLayout<double>::slot_bytes + 1024;
+    auto kern = A.prof ? k_stream<double, true> : k_stream<double, false>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    kern<<<p->sk_grid, SK_THREADS, smem, st>>>(tm, A);
+    return cudaGetLastError();
 }
 
 // k = 0, CONTIGUOUS: the TMA kernel when both row strides (n and m elements)
@@ -778,7 +838,9 @@ tri_status tri_plan_set_variant(tri_plan_t p, tri_variant v) {
     if (v == TRI_VARIANT_ONCHIP && p->n > onchip_rows_budget(p->dtype)) return TRI_ERR_INVALID_ARG;
     if (v == TRI_VARIANT_FUSED && !fused_ok(p->n, p->m, p->layout)) return TRI_ERR_INVALID_ARG;
     if (v == TRI_VARIANT_WARP && !warp_ok(p->n)) return TRI_ERR_INVALID_ARG;
-    if (v != TRI_VARIANT_ONCHIP && v != TRI_VARIANT_SPLIT && v != TRI_VARIANT_FUSED && v != TRI_VARIANT_WARP)
+    if (v == TRI_VARIANT_STREAM && !stream_ok(p->n, p->m, p->dtype, p->layout)) return TRI_ERR_INVALID_ARG;
+    if (v != TRI_VARIANT_ONCHIP && v != TRI_VARIANT_SPLIT && v != TRI_VARIANT_FUSED && v != TRI_VARIANT_WARP &&
+        v != TRI_VARIANT_STREAM)
         return TRI_ERR_INVALID_ARG;
     const tri_variant ov = p->variant;
     const int ok = p->k;
@@ -793,14 +855,14 @@ tri_status tri_plan_set_variant(tri_plan_t p, tri_variant v) {
 void tri_plan_describe(tri_plan_t p, char* buf, int len) {
     if (!buf || len <= 0) return;
     if (!p) { snprintf(buf, len, "null plan"); return; }
-    static const char* vn[] = {"auto", "onchip", "split", "fused", "warp"};
+    static const char* vn[] = {"auto", "onchip", "split", "fused", "warp", "stream"};
     snprintf(buf, len,
              "n=%lld m=%lld dtype=%s layout=%s variant=%s k=%d G=%d P=%d rpt=%d L=%lld C=%lld region=%lld nreg=%lld "
-             "fu_grid=%d fu_son=%d fu_nc=%lld scratch=%zu sms=%d",
+             "fu_grid=%d fu_son=%d fu_nc=%lld sk_grid=%d sk_nc=%d sk_son=%d scratch=%zu sms=%d",
              (long long)p->n, (long long)p->m, p->dtype == TRI_F64 ? "f64" : "f32",
              p->layout == TRI_LAYOUT_CONTIGUOUS ? "contiguous" : "interleaved", vn[p->variant], p->k, p->G, p->P,
              p->rpt, (long long)p->L, (long long)p->C, (long long)p->region, (long long)p->nreg, p->fu_grid, p->fu_son,
-             (long long)p->fu_nc, p->scratch_bytes, p->sms);
+             (long long)p->fu_nc, p->sk_grid, p->sk_nc, p->sk_son, p->scratch_bytes, p->sms);
 }
 
 tri_status tri_solve(tri_plan_t p, const void* a, const void* b, const void* c, const void* d, void* x,
@@ -818,6 +880,8 @@ tri_status tri_solve(tri_plan_t p, const void* a, const void* b, const void* c, 
     } else if (p->variant == TRI_VARIANT_ONCHIP) {
         e = p->dtype == TRI_F64 ? launch_onchip<double>(p, a, b, c, d, x, nullptr, nullptr, nullptr, 0, s)
                                 : launch_onchip<float>(p, a, b, c, d, x, nullptr, nullptr, nullptr, 0, s);
+    } else if (p->variant == TRI_VARIANT_STREAM) {
+        e = launch_stream(p, a, b, c, d, x, s);
     } else if (p->variant == TRI_VARIANT_FUSED) {
         e = p->dtype == TRI_F64 ? launch_fused<double>(p, a, b, c, d, x, s) : launch_fused<float>(p, a, b, c, d, x, s);
     } else {
@@ -841,6 +905,8 @@ tri_status tri_debug_pcr(tri_plan_t p, const void* a, const void* b, const void*
     } else if (p->variant == TRI_VARIANT_ONCHIP) {
         e = p->dtype == TRI_F64 ? launch_onchip<double>(p, a, b, c, d, nullptr, ao, co, do_, 1, s)
                                 : launch_onchip<float>(p, a, b, c, d, nullptr, ao, co, do_, 1, s);
+    } else if (p->variant == TRI_VARIANT_STREAM) {
+        e = launch_stream(p, a, b, c, d, nullptr, s, ao, co, do_);
     } else if (p->variant == TRI_VARIANT_FUSED) {
         e = p->dtype == TRI_F64 ? launch_fused<double>(p, a, b, c, d, nullptr, s, ao, co, do_)
                                 : launch_fused<float>(p, a, b, c, d, nullptr, s, ao, co, do_);

@@ -301,6 +301,98 @@ def test_fused_edges_and_scaling(cuda_ok):
         plan.k = 2  # the fused kernel is built for one k
 
 
+# ------------------------------------------------------------------ STREAM variant
+STREAM = tri.VARIANT_STREAM
+
+
+@pytest.mark.parametrize("n,m", [(1928, 3), (1936, 2), (2048, 5), (16384, 7), (4104, 2), (16392, 150), (2400, 300),
+                                 (6000, 149), (16384, 300), (100000, 2), (245760, 2)])
+def test_stream_parity(cuda_ok, n, m):
+    """Spans: NC from 9 (all slots resident) to 1024 (most slots spilled), a
+    ragged last window (1928, 4104, 16392), one and several systems per CTA
+    (both slot parities), m > #SMs (uneven systems per CTA)."""
+    arrs = gen(n, m, "f64", 0)
+    x, plan = gpu_solve(n, m, arrs, "f64", 0, variant=STREAM)
+    assert plan.variant == STREAM and plan.k == 3
+    check_parity(n, m, arrs, x, "f64", 0)
+
+
+@pytest.mark.parametrize("family,eps", [("weak", 1e-2), ("weak", 1e-3), ("integer", 0.0), ("poisson", 0.0)])
+def test_stream_families(cuda_ok, family, eps):
+    n, m = 16384, 6
+    arrs = gen(n, m, "f64", 0, family, eps=eps)
+    x, _ = gpu_solve(n, m, arrs, "f64", 0, variant=STREAM)
+    if family == "poisson":
+        # Poisson is ill-conditioned (kappa ~ n^2/2): forward error vs oracle bounded by kappa*u
+        xo = oracle.solve_batch(n, m, *arrs)
+        assert np.max(np.abs(x - xo)) / np.max(np.abs(xo)) <= 2 * (n + 1) ** 2 / 2 * 2.2e-16
+    else:
+        check_parity(n, m, arrs, x, "f64", 0)
+
+
+@pytest.mark.parametrize("n,m", [(1936, 2), (16384, 3)])
+def test_stream_pcr_stage(cuda_ok, n, m):
+    """Row A2 for the STREAM kernel: its 3-step reduced system (normalised) vs
+    the oracle's plain PCR (Eqs 5-6)."""
+    arrs = gen(n, m, "f64", 0, "weak", eps=1e-2)
+    plan = tri.Plan(n, m, tri.F64, 0)
+    plan.variant = STREAM
+    A, C, D = (t.cpu().numpy() for t in plan.debug_pcr(*to_dev(*arrs)))
+    for q in range(m):
+        sl = slice(q * n, (q + 1) * n)
+        ao, bo, co, do = oracle.pcr_k(*(t[sl] for t in arrs), plan.k)
+        for got, ref in ((A[sl], ao / bo), (C[sl], co / bo), (D[sl], do / bo)):
+            assert np.max(np.abs(got - ref)) <= 1e-12 * max(1.0, np.max(np.abs(ref)))
+
+
+def test_stream_edges_and_scaling(cuda_ok):
+    """X1 (NaN in a_0 / c_{n-1} ignored, bitwise), metamorphic row and rhs
+    scaling by powers of two (bitwise), determinism across runs, and the
+    variant's fixed k."""
+    import torch
+    n, m = 9000, 5
+    a, b, c, d = gen(n, m, "f64", 0, "weak", eps=1e-2)
+    plan = tri.Plan(n, m, tri.F64, 0)
+    plan.variant = STREAM
+    da, db, dc, dd = to_dev(a, b, c, d)
+    x1 = plan.solve(da, db, dc, dd).clone()
+    assert torch.equal(plan.solve(da, db, dc, dd), x1)
+    a2, c2 = da.clone(), dc.clone()
+    a2.view(m, n)[:, 0] = float("nan")
+    c2.view(m, n)[:, -1] = float("nan")
+    assert torch.equal(plan.solve(a2, db, c2, dd), x1)
+    p = 2.0 ** np.random.default_rng(1).integers(-20, 20, n * m)
+    x2 = plan.solve(*to_dev(a * p, b * p, c * p, d * p))
+    assert torch.equal(x2, x1)
+    x3 = plan.solve(da, db, dc, dd * 4.0)
+    assert torch.equal(x3, x1 * 4.0)
+    with pytest.raises(tri.TriError):
+        plan.k = 2  # the stream kernel is built for one k
+
+
+def test_stream_rejects_unsupported(cuda_ok):
+    for (n, m, dt, layout) in [(1004, 3, tri.F64, 0), (16384, 3, tri.F32, 0), (16384, 3, tri.F64, 1), (256, 3, tri.F64, 0),
+                               (1672, 3, tri.F64, 0), (245768, 2, tri.F64, 0)]:
+        plan = tri.Plan(n, m, dt, layout)
+        with pytest.raises(tri.TriError):
+            plan.variant = STREAM
+
+
+def test_stream_full_size_sampled(cuda_ok):
+    """BASELINE c5 shape (m = n = 16384) in the launch configuration bench.py
+    times: whole sampled systems (first/last of a CTA's sweep, both slot
+    parities, the last system) vs the oracle element by element."""
+    n, m = 16384, 16384
+    arrs = gen(n, m, "f64", 0)
+    plan = tri.Plan(n, m, tri.F64, 0)
+    plan.variant = STREAM
+    x = plan.solve(*to_dev(*arrs)).cpu().numpy()
+    for q in (0, 1, 147, 148, 149, 8191, 16235, 16383):
+        sl = slice(q * n, (q + 1) * n)
+        sub = [t[sl] for t in arrs]
+        check_parity(n, 1, sub, x[sl], "f64", 0)
+
+
 # ------------------------------------------------------------------ WARP variant
 @pytest.mark.parametrize("dtype", ["f64", "f32"])
 @pytest.mark.parametrize("layout", [0, 1])
