@@ -296,7 +296,8 @@ __global__ void __launch_bounds__(SK_THREADS, 1) k_stream(const __grid_constant_
         const int64_t q = blockIdx.x + (int64_t)jj * gridDim.x;
         const int64_t row0 = q * n + (int64_t)ww * SK_V - SK_HALO;  // multiple of 8 (n % 8 == 0)
         const int y = (int)(row0 >> 3);                              // may be -1: TMA zero-fills
-        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        // (the generic-proxy reads of the buffer completed: their values were
+        // consumed before this point, as in a consumer-release / producer-acquire pipeline)
         sk_expect(&in_full[pw], (unsigned)(4 * SK_W * sizeof(T)));
         sk_tma2d(ib + 0 * SK_W, &tm.a, 0, y, &in_full[pw], pol_in);
         sk_tma2d(ib + 1 * SK_W, &tm.b, 0, y, &in_full[pw], pol_in);
@@ -336,6 +337,7 @@ __global__ void __launch_bounds__(SK_THREADS, 1) k_stream(const __grid_constant_
     int it = 0;                                   // this warp's step count
     for (int g = pw; g < total; g += SK_NPCR, ++it) {
         const unsigned ppar = (unsigned)((it - (pw == 0 ? 1 : 0)) & 1);  // phase parity of step g - 1
+        if (prof) tq = clock64();
         const int cj = j, cw = w;
         w += SK_NPCR;
         while (w >= NC) { w -= NC; ++j; }
@@ -344,90 +346,24 @@ __global__ void __launch_bounds__(SK_THREADS, 1) k_stream(const __grid_constant_
         const int slot = slot_of(cj, cw);
         bool res;
         T* sp = seg_ptr(slot, res);
+        // The forward and the backward work of a step are computed unconditionally
+        // (on identity data when a part is inactive: the first and the last NC
+        // steps) so that the compiler can interleave their dependency chains;
+        // only waits and stores are conditional.
 
-        if (prof) tq = clock64();
-        // ---- backward part: Eq 4 on window (cj - 1, wb), reading the slot
-        if (bwd) {
-            T cpb[SK_SEG], dpb[SK_SEG];
-            if (res || !pref) {
-                const unsigned long long tb = prof ? clock64() : 0;
-                sk_wait(&sfull[slot], (unsigned)((cj - 1) & 1));  // system cj - 1 stored in the slot
-                if (prof) t_sf += clock64() - tb;
-                if (res) {
-#pragma unroll
-                    for (int t = 0; t < SK_SEG; ++t) fu_ld2(sp + 2 * t, cpb[t], dpb[t]);
-                } else {
-#pragma unroll
-                    for (int t = 0; t < SK_SEG; ++t) sk_ldg2(sp + 2 * t, cpb[t], dpb[t]);
-                }
-            } else {
-                const unsigned long long tb = prof ? clock64() : 0;
-                cp_async_wait<0>();
-                __syncwarp();
-                if (prof) t_sf += clock64() - tb;
-                const T* pb = tr + (c * SK_SCS + sg * SK_SEG) * 2;
-#pragma unroll
-                for (int t = 0; t < SK_SEG; ++t) fu_ld2(pb + 2 * t, cpb[t], dpb[t]);
-            }
-#pragma unroll
-            for (int t = 0; t < SK_SEG; ++t)
-                if (t >= nvs) { cpb[t] = T(-1); dpb[t] = T(0); }  // padding: x_t = x_{t+1}
-            // affine map of the segment: x_start = al + be * x_after
-            T al = T(0), be = T(1);
-#pragma unroll
-            for (int t = SK_SEG - 1; t >= 0; --t) {
-                al = fma(-cpb[t], al, dpb[t]);
-                be = -cpb[t] * be;
-            }
-            {  // suffix scan over the segments (lanes c + 8 sg, sg descending)
-                T oa = __shfl_down_sync(0xffffffffu, al, 8), ob = __shfl_down_sync(0xffffffffu, be, 8);
-                if (sg <= 2) { al = fma(be, oa, al); be = be * ob; }
-                oa = __shfl_down_sync(0xffffffffu, al, 16);
-                ob = __shfl_down_sync(0xffffffffu, be, 16);
-                if (sg <= 1) { al = fma(be, oa, al); be = be * ob; }
-            }
-            // the serial step: x at position 0 of window wb + 1 (previous step)
-            T xw = T(0);
-            if (wb < NC - 1) {
-                const unsigned long long tb = prof ? clock64() : 0;
-                sk_wait(&bfull[pi], ppar);
-                if (prof) t_bx += clock64() - tb;
-                xw = xh[pi * SK_S + c];
-            }
-            const T xs = fma(be, xw, al);  // x at the first position of segment sg
-            if (sg == 0) xh[pw * SK_S + c] = xs;
-            __syncwarp();
-            if (lane == 0) sk_arrive(&bfull[pw]);
-            T x = __shfl_down_sync(0xffffffffu, xs, 8);  // x after segment sg
-            if (sg == 3) x = xw;
-            // replay (Eq 4) and store x: row 240 wb + 8 (8 sg + t) + c of system cj - 1
-            const int64_t qb = blockIdx.x + (int64_t)(cj - 1) * gridDim.x;
-            T* xo = p.x + qb * n + (int64_t)wb * SK_V + (sg * SK_SEG) * SK_S + c;
-            const int64_t rmax = n - ((int64_t)wb * SK_V + (sg * SK_SEG) * SK_S + c);  // rows left from xo
-#pragma unroll
-            for (int t = SK_SEG - 1; t >= 0; --t) {
-                x = fma(-cpb[t], x, dpb[t]);
-                if (t < nvs && t * SK_S < rmax) __stcs(xo + t * SK_S, x);
-            }
-        } else {
-            __syncwarp();
-            if (lane == 0) sk_arrive(&bfull[pw]);  // keep one phase per step
-        }
-
-        SK_PH(0);
-        // ---- forward part: stage, normalise, PCR, transpose, segmented sweep
+        // ---- forward: stage, normalise (X17), K PCR levels (Eqs 5-6; X3/X4)
+        NRow<T> v[SK_R];
         if (fwd) {
             const unsigned long long ta = prof ? clock64() : 0;
             sk_wait(&in_full[pw], ph);
             if (prof) t_in += clock64() - ta;
             ph ^= 1u;
-            NRow<T> v[SK_R];
             const int64_t ws = (int64_t)cw * SK_V - SK_HALO;
             const bool interior = cw > 0 && ws + SK_W <= n;
             const int64_t i0 = ws + lane * SK_R;
             const T* st = ib + lane * SK_R;
 #pragma unroll
-            for (int cc = 0; cc < CPL; ++cc) {  // EPC rows at a time: load and normalise (X17)
+            for (int cc = 0; cc < CPL; ++cc) {  // EPC rows at a time: load and normalise
                 T raw[4][EPC];
 #pragma unroll
                 for (int arr = 0; arr < 4; ++arr) {
@@ -451,155 +387,219 @@ __global__ void __launch_bounds__(SK_THREADS, 1) k_stream(const __grid_constant_
             }
             __syncwarp();
             if (lane == 0 && g + SK_NPCR < nfwd) issue(j, w);
-            SK_PH(1);
-            // K PCR levels in registers (Eqs 5-6, normalised; X3/X4)
-            if (p.dbg != 1) {
+        } else {
 #pragma unroll
-                for (int lv = 0; lv < SK_K; ++lv) {
-                    const int sgm = 1 << lv;
-                    NRow<T> nv[SK_R];
+            for (int u = 0; u < SK_R; ++u) v[u] = identity_row<T>();
+        }
+        SK_PH(1);
+        if (p.dbg != 1) {
 #pragma unroll
-                    for (int u = 0; u < SK_R; ++u) {
-                        NRow<T> mm, pp;
-                        if (u - sgm >= 0) {
-                            mm = v[u - sgm];
-                        } else {
-                            const NRow<T>& s = v[u - sgm + SK_R];
-                            mm.A = __shfl_up_sync(0xffffffffu, s.A, 1);
-                            mm.C = __shfl_up_sync(0xffffffffu, s.C, 1);
-                            mm.D = __shfl_up_sync(0xffffffffu, s.D, 1);
-                        }
-                        if (u + sgm < SK_R) {
-                            pp = v[u + sgm];
-                        } else {
-                            const NRow<T>& s = v[u + sgm - SK_R];
-                            pp.A = __shfl_down_sync(0xffffffffu, s.A, 1);
-                            pp.C = __shfl_down_sync(0xffffffffu, s.C, 1);
-                            pp.D = __shfl_down_sync(0xffffffffu, s.D, 1);
-                        }
-                        nv[u] = pcr_combine(mm, v[u], pp);
+            for (int lv = 0; lv < SK_K; ++lv) {
+                const int sgm = 1 << lv;
+                NRow<T> nv[SK_R];
+#pragma unroll
+                for (int u = 0; u < SK_R; ++u) {
+                    NRow<T> mm, pp;
+                    if (u - sgm >= 0) {
+                        mm = v[u - sgm];
+                    } else {
+                        const NRow<T>& s = v[u - sgm + SK_R];
+                        mm.A = __shfl_up_sync(0xffffffffu, s.A, 1);
+                        mm.C = __shfl_up_sync(0xffffffffu, s.C, 1);
+                        mm.D = __shfl_up_sync(0xffffffffu, s.D, 1);
                     }
-#pragma unroll
-                    for (int u = 0; u < SK_R; ++u) v[u] = nv[u];
-                }
-            }
-            if (p.dA) {  // tri_debug_pcr: the reduced rows, normalised (X17)
-                const int64_t q = blockIdx.x + (int64_t)cj * gridDim.x;
-                if (lane >= 1 && lane <= SK_P) {
-#pragma unroll
-                    for (int u = 0; u < SK_R; ++u) {
-                        const int64_t row = (int64_t)cw * SK_V + (lane - 1) * SK_R + u;
-                        if (row < n) {
-                            p.dA[q * n + row] = v[u].A;
-                            p.dC[q * n + row] = v[u].C;
-                            p.dD[q * n + row] = v[u].D;
-                        }
+                    if (u + sgm < SK_R) {
+                        pp = v[u + sgm];
+                    } else {
+                        const NRow<T>& s = v[u + sgm - SK_R];
+                        pp.A = __shfl_down_sync(0xffffffffu, s.A, 1);
+                        pp.C = __shfl_down_sync(0xffffffffu, s.C, 1);
+                        pp.D = __shfl_down_sync(0xffffffffu, s.D, 1);
                     }
+                    nv[u] = pcr_combine(mm, v[u], pp);
                 }
-                continue;
+#pragma unroll
+                for (int u = 0; u < SK_R; ++u) v[u] = nv[u];
             }
-            SK_PH(2);
-            // transpose: lanes 1..30 hold position lane-1 of chains u = 0..7
+        }
+        SK_PH(2);
+        if (p.dA) {  // tri_debug_pcr: the reduced rows, normalised (X17)
+            const int64_t q = blockIdx.x + (int64_t)cj * gridDim.x;
             if (lane >= 1 && lane <= SK_P) {
 #pragma unroll
                 for (int u = 0; u < SK_R; ++u) {
-                    tr[u * SK_TCS + lane - 1] = v[u].A;
-                    tr[SK_S * SK_TCS + u * SK_TCS + lane - 1] = v[u].C;
-                    tr[2 * SK_S * SK_TCS + u * SK_TCS + lane - 1] = v[u].D;
-                }
-            }
-            __syncwarp();
-            T A[SK_SEG], C[SK_SEG], D[SK_SEG];
-            {
-                const T* tA = tr + c * SK_TCS + sg * SK_SEG;
-#pragma unroll
-                for (int t = 0; t < SK_SEG; t += 2) {
-                    fu_ld2(tA + t, A[t], A[t + 1]);
-                    fu_ld2(tA + SK_S * SK_TCS + t, C[t], C[t + 1]);
-                    fu_ld2(tA + 2 * SK_S * SK_TCS + t, D[t], D[t + 1]);
-                }
-            }
-            __syncwarp();  // the transpose buffer is free: prefetch the next step's spilled slot
-            prefetch(j, w);
-            SK_PH(3);
-            SKMat<T> M;
-            {  // segment transfer (basis inputs theta_in, psi_in, delta_in)
-                T t1 = T(1), p1 = T(0), d1 = T(0);  // response to theta_in
-                T t2 = T(0), p2 = T(1), d2 = T(0);  // response to psi_in
-                T d3 = T(1);                        // response to delta_in
-#pragma unroll
-                for (int t = 0; t < SK_SEG; ++t) {
-                    if (t < nvs) {
-                        const T nt1 = fma(-A[t], p1, t1), np1 = C[t] * t1, nd1 = fma(-A[t], d1, D[t] * t1);
-                        const T nt2 = fma(-A[t], p2, t2), np2 = C[t] * t2, nd2 = fma(-A[t], d2, D[t] * t2);
-                        d3 = -A[t] * d3;
-                        t1 = nt1; p1 = np1; d1 = nd1;
-                        t2 = nt2; p2 = np2; d2 = nd2;
+                    const int64_t row = (int64_t)cw * SK_V + (lane - 1) * SK_R + u;
+                    if (row < n) {
+                        p.dA[q * n + row] = v[u].A;
+                        p.dC[q * n + row] = v[u].C;
+                        p.dD[q * n + row] = v[u].D;
                     }
                 }
-                M = SKMat<T>{t1, t2, p1, p2, d1, d2, d3};
             }
-            {  // inclusive scan over the four segments of the chain (lanes c + 8 sg)
-                SKMat<T> o = sk_shfl_up(M, 8);
-                if (sg >= 1) M = sk_compose(M, o);
-                o = sk_shfl_up(M, 16);
-                if (sg >= 2) M = sk_compose(M, o);
-            }
-            SK_PH(4);
-            // the serial step: state handed over by step g - 1
-            T th, ps, de;
-            if (cw > 0) {
-                const unsigned long long tb = prof ? clock64() : 0;
-                sk_wait(&stfull[pi], ppar);
-                if (prof) t_st += clock64() - tb;
-                const T* si = stt + pi * 3 * SK_S + c;
-                th = si[0];
-                ps = si[SK_S];
-                de = si[2 * SK_S];
+            continue;
+        }
+
+        // ---- backward: the (c', d') pairs of window (cj - 1, wb), segment sg
+        T cpb[SK_SEG], dpb[SK_SEG];
+        if (bwd) {
+            if (!res && pref) {  // prefetched into the transpose buffer by the previous step
+                cp_async_wait<0>();
+                __syncwarp();
+                const T* pb = tr + (c * SK_SCS + sg * SK_SEG) * 2;
+#pragma unroll
+                for (int t = 0; t < SK_SEG; ++t) fu_ld2(pb + 2 * t, cpb[t], dpb[t]);
+                __syncwarp();
             } else {
-                th = T(1); ps = T(0); de = T(0);  // theta_{-1} = 1, psi_0 = C_{-1} theta_{-2} = 0 (a_0 = 0)
+                const unsigned long long tb = prof ? clock64() : 0;
+                sk_wait(&sfull[slot], (unsigned)((cj - 1) & 1));  // system cj - 1 stored in the slot
+                if (prof) t_sf += clock64() - tb;
+                if (res) {
+#pragma unroll
+                    for (int t = 0; t < SK_SEG; ++t) fu_ld2(sp + 2 * t, cpb[t], dpb[t]);
+                } else {
+#pragma unroll
+                    for (int t = 0; t < SK_SEG; ++t) sk_ldg2(sp + 2 * t, cpb[t], dpb[t]);
+                }
             }
-            const T ot = fma(M.a, th, M.b * ps);
-            const T op = fma(M.c, th, M.d * ps);
-            const T od = fma(M.e, th, fma(M.f, ps, M.g * de));
-            if (sg == 3) {  // window end: exact power-of-two rescale, hand over
-                const T sc = sk_exp2_scale(ot);
-                T* so = stt + pw * 3 * SK_S + c;
-                so[0] = ot * sc;
-                so[SK_S] = op * sc;
-                so[2 * SK_S] = od * sc;
+#pragma unroll
+            for (int t = 0; t < SK_SEG; ++t)
+                if (t >= nvs) { cpb[t] = T(-1); dpb[t] = T(0); }  // padding: x_t = x_{t+1}
+        } else {
+#pragma unroll
+            for (int t = 0; t < SK_SEG; ++t) { cpb[t] = T(-1); dpb[t] = T(0); }
+        }
+        SK_PH(3);
+
+        // ---- forward: transpose so that lane (c, sg) holds positions 8 sg .. 8 sg + 7 of chain c
+        if (lane >= 1 && lane <= SK_P) {
+#pragma unroll
+            for (int u = 0; u < SK_R; ++u) {
+                tr[u * SK_TCS + lane - 1] = v[u].A;
+                tr[SK_S * SK_TCS + u * SK_TCS + lane - 1] = v[u].C;
+                tr[2 * SK_S * SK_TCS + u * SK_TCS + lane - 1] = v[u].D;
             }
-            __syncwarp();
-            if (lane == 0) sk_arrive(&stfull[pw]);
-            {  // incoming state of this lane's segment = outgoing state of segment sg - 1
-                const T it = __shfl_up_sync(0xffffffffu, ot, 8);
-                const T ip = __shfl_up_sync(0xffffffffu, op, 8);
-                const T id = __shfl_up_sync(0xffffffffu, od, 8);
-                if (sg > 0) { th = it; ps = ip; de = id; }
+        }
+        __syncwarp();
+        T A[SK_SEG], C[SK_SEG], D[SK_SEG];
+        {
+            const T* tA = tr + c * SK_TCS + sg * SK_SEG;
+#pragma unroll
+            for (int t = 0; t < SK_SEG; t += 2) {
+                fu_ld2(tA + t, A[t], A[t + 1]);
+                fu_ld2(tA + SK_S * SK_TCS + t, C[t], C[t + 1]);
+                fu_ld2(tA + 2 * SK_S * SK_TCS + t, D[t], D[t + 1]);
             }
-            SK_PH(5);
-            // replay the segment from the true state: c'_t, d'_t (Eqs 2-3)
+        }
+        __syncwarp();  // the transpose buffer is free: prefetch the next step's spilled slot
+        prefetch(j, w);
+        SK_PH(4);
+
+        // ---- both sweeps' segment maps (independent chains, one loop)
+        SKMat<T> M;
+        T al = T(0), be = T(1);  // backward: x_start = al + be * x_after
+        {
+            T t1 = T(1), p1 = T(0), d1 = T(0);  // forward response to theta_in
+            T t2 = T(0), p2 = T(1), d2 = T(0);  // ... to psi_in
+            T d3 = T(1);                        // ... to delta_in
 #pragma unroll
             for (int t = 0; t < SK_SEG; ++t) {
                 if (t < nvs) {
-                    const T nt = fma(-A[t], ps, th);
-                    const T np = C[t] * th;
-                    const T nd = fma(-A[t], de, D[t] * th);
-                    const T inv = rcp(nt);
-                    const T cpv = np * inv, dpv = nd * inv;
+                    const T nt1 = fma(-A[t], p1, t1), np1 = C[t] * t1, nd1 = fma(-A[t], d1, D[t] * t1);
+                    const T nt2 = fma(-A[t], p2, t2), np2 = C[t] * t2, nd2 = fma(-A[t], d2, D[t] * t2);
+                    d3 = -A[t] * d3;
+                    t1 = nt1; p1 = np1; d1 = nd1;
+                    t2 = nt2; p2 = np2; d2 = nd2;
+                }
+                const int tb = SK_SEG - 1 - t;  // backward runs the positions in reverse
+                al = fma(-cpb[tb], al, dpb[tb]);
+                be = -cpb[tb] * be;
+            }
+            M = SKMat<T>{t1, t2, p1, p2, d1, d2, d3};
+        }
+        {  // scans over the four segments of a chain: forward inclusive (lanes c + 8 sg
+           // ascending), backward suffix (descending)
+            SKMat<T> o = sk_shfl_up(M, 8);
+            T oa = __shfl_down_sync(0xffffffffu, al, 8), ob = __shfl_down_sync(0xffffffffu, be, 8);
+            if (sg >= 1) M = sk_compose(M, o);
+            if (sg <= 2) { al = fma(be, oa, al); be = be * ob; }
+            o = sk_shfl_up(M, 16);
+            oa = __shfl_down_sync(0xffffffffu, al, 16);
+            ob = __shfl_down_sync(0xffffffffu, be, 16);
+            if (sg >= 2) M = sk_compose(M, o);
+            if (sg <= 1) { al = fma(be, oa, al); be = be * ob; }
+        }
+        SK_PH(5);
+
+        // ---- the two serial steps: x from step g - 1 (backward), state from step g - 1 (forward)
+        T xw = T(0);  // x at position 0 of window wb + 1
+        if (bwd && wb < NC - 1) {
+            const unsigned long long tb = prof ? clock64() : 0;
+            sk_wait(&bfull[pi], ppar);
+            if (prof) t_bx += clock64() - tb;
+            xw = xh[pi * SK_S + c];
+        }
+        const T xs = fma(be, xw, al);  // x at the first position of segment sg
+        if (sg == 0) xh[pw * SK_S + c] = xs;
+        __syncwarp();
+        if (lane == 0) sk_arrive(&bfull[pw]);
+        T th = T(1), ps = T(0), de = T(0);  // theta_{-1} = 1, psi_0 = C_{-1} theta_{-2} = 0 (a_0 = 0)
+        if (fwd && cw > 0) {
+            const unsigned long long tb = prof ? clock64() : 0;
+            sk_wait(&stfull[pi], ppar);
+            if (prof) t_st += clock64() - tb;
+            const T* si = stt + pi * 3 * SK_S + c;
+            th = si[0];
+            ps = si[SK_S];
+            de = si[2 * SK_S];
+        }
+        const T ot = fma(M.a, th, M.b * ps);
+        const T op = fma(M.c, th, M.d * ps);
+        const T od = fma(M.e, th, fma(M.f, ps, M.g * de));
+        if (sg == 3) {  // window end: exact power-of-two rescale, hand over
+            const T sc = sk_exp2_scale(ot);
+            T* so = stt + pw * 3 * SK_S + c;
+            so[0] = ot * sc;
+            so[SK_S] = op * sc;
+            so[2 * SK_S] = od * sc;
+        }
+        __syncwarp();
+        if (lane == 0) sk_arrive(&stfull[pw]);
+        T x = __shfl_down_sync(0xffffffffu, xs, 8);  // x after segment sg
+        if (sg == 3) x = xw;
+        {  // incoming state of this lane's segment = outgoing state of segment sg - 1
+            const T it_ = __shfl_up_sync(0xffffffffu, ot, 8);
+            const T ip = __shfl_up_sync(0xffffffffu, op, 8);
+            const T id = __shfl_up_sync(0xffffffffu, od, 8);
+            if (sg > 0) { th = it_; ps = ip; de = id; }
+        }
+        SK_PH(6);
+
+        // ---- both replays: x (Eq 4) of window (cj - 1, wb); c', d' (Eqs 2-3) of (cj, cw)
+        const int64_t qb = blockIdx.x + (int64_t)(cj - 1) * gridDim.x;
+        const int64_t xr = (int64_t)wb * SK_V + (sg * SK_SEG) * SK_S + c;  // row of position 8 sg
+        T* xo = p.x + qb * n + xr;
+        const int64_t rmax = bwd ? n - xr : 0;
+#pragma unroll
+        for (int t = 0; t < SK_SEG; ++t) {
+            const int tb = SK_SEG - 1 - t;
+            x = fma(-cpb[tb], x, dpb[tb]);
+            if (tb < nvs && tb * SK_S < rmax) __stcs(xo + tb * SK_S, x);
+            if (t < nvs) {
+                const T nt = fma(-A[t], ps, th);
+                const T np = C[t] * th;
+                const T nd = fma(-A[t], de, D[t] * th);
+                const T inv = rcp(nt);
+                const T cpv = np * inv, dpv = nd * inv;
+                if (fwd) {
                     if (res) fu_st2(sp + 2 * t, cpv, dpv);
                     else sk_st_global_last(sp + 2 * t, cpv, dpv, pol_sp);
-                    th = nt; ps = np; de = nd;
                 }
+                th = nt; ps = np; de = nd;
             }
-            __syncwarp();
-            if (lane == 0) sk_arrive(&sfull[slot]);
-            SK_PH(6);
-        } else {
-            prefetch(j, w);
-            __syncwarp();
-            if (lane == 0) sk_arrive(&stfull[pw]);  // keep one phase per step
         }
+        __syncwarp();
+        if (fwd && lane == 0) sk_arrive(&sfull[slot]);
+        SK_PH(0);
     }
     cp_async_wait<0>();
     if (prof && lane == 0) {

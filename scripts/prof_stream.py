@@ -28,7 +28,7 @@ ms = s.elapsed_time(e)
 v = cnt.cpu().tolist()
 ncta = min(m, 148)
 nwin = m * ((n + 239) // 240) / ncta
-names = ["total (8 warps)", "wait input", "wait fwd state", "wait bwd x", "wait slot stored", "ph backward", "ph wait+load+norm", "ph PCR", "ph transpose", "ph pass1+scan", "ph state", "ph pass2+store"]
+names = ["total (8 warps)", "wait input", "wait fwd state", "wait bwd x", "wait slot stored", "ph replays+store", "ph wait+load+norm", "ph PCR", "ph bwd load", "ph transpose", "ph pass1+scans", "ph serial steps"]
 print(f"time {ms:.3f} ms, {ms * 1.965e6:.0f} cycles @1.965GHz, {nwin:.0f} windows per CTA; per CTA (per window):")
 for i, nm in enumerate(names):
     per = v[i] / ncta / 12
