@@ -133,8 +133,8 @@ def method_arrays(plan, tri):
     v = plan.variant
     if v in (tri.VARIANT_WARP, tri.VARIANT_ONCHIP):
         return 5
-    if v == tri.VARIANT_FUSED:
-        return 5  # c', d' of the first L - S_on positions go to per-CTA scratch that stays in L2
+    if v in (tri.VARIANT_FUSED, tri.VARIANT_STREAM):
+        return 5  # c', d' stay in smem or in per-CTA scratch that stays in L2 (ncu: 5.0 arrays of DRAM traffic)
     if plan.k == 0:
         return 9  # read a, b, c, d; write + read c', d'; write x
     # pass 1: read 4 + write 3; [pass 2: read 3 + write 3]; p-Thomas: read 3, c', d' 2 + 2, write x

@@ -102,6 +102,12 @@ bool stream_ok(int64_t n, int64_t m, tri_dtype t, tri_layout layout) {
 //   * whole systems that fit a CTA's smem: ONCHIP;
 //   * otherwise (few large systems): SPLIT with k from choose_k_for.
 tri_variant choose_variant(int64_t n, int64_t m, tri_dtype t, tri_layout layout, int sms) {
+    // STREAM (profiles/r01_sweep_stream_f64.jsonl): fastest of all variants for
+    // fp64 contiguous batches with n % 8 == 0 from 8 windows up, except a few
+    // (< 64) very long systems, where SPLIT's deep k keeps more SMs busy
+    // (n = 65536, m = 37: 136 us vs 166 us); e.g. n = m = 16384: 2.92 ms vs
+    // 3.41 ms (k = 0 TMA), n = 2048, m = 2368: 63 us vs 111 us (FUSED).
+    if (layout == TRI_LAYOUT_CONTIGUOUS && stream_ok(n, m, t, layout) && (m >= 64 || n <= 8192)) return TRI_VARIANT_STREAM;
     if (m >= 48 * (int64_t)sms) return TRI_VARIANT_SPLIT;
     const bool contig = layout == TRI_LAYOUT_CONTIGUOUS;
     if (contig && fused_ok(n, m, layout) && n >= 1024 && (n <= 2048 || m >= 128)) return TRI_VARIANT_FUSED;

@@ -1,7 +1,7 @@
 mkdir -p gpurun_out
-set -x
-nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm --format=csv
+nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm --format=csv > gpurun_out/smi.txt
 timeout 1200 python -m pytest tests -x -q -m gpu > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?" >> gpurun_out/pytest_gpu.log
 timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke.log 2>&1; echo "smoke rc=$?" >> gpurun_out/smoke.log
-for c in c1 c2 c3 c4 c5; do timeout 600 python bench.py --config $c > gpurun_out/bench_$c.json 2> gpurun_out/bench_$c.err; done
-timeout 300 python bench.py --impl reference --steps 2 --warmup 1 > gpurun_out/bench_ref.json 2>&1
+for c in c5 c1 c2 c3 c4; do timeout 600 python bench.py --config $c > gpurun_out/bench_$c.json 2> gpurun_out/bench_$c.err; done
+timeout 600 python scripts/launch_times.py python bench.py --config c5 --steps 2 --warmup 1 --no-e2e --no-cpu --no-check > gpurun_out/launches_c5.txt 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_stream -c 1 -o gpurun_out/c5_stream_full python scripts/prof_one.py 16384 16384 f64 0 0 - 1 > gpurun_out/ncu_c5.log 2>&1
