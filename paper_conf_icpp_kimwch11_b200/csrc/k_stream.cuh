@@ -53,7 +53,11 @@ constexpr int SK_HALO = 8;           // >= f(3) = 7 (Eq 8), one lane of rows
 constexpr int SK_V = SK_W - 2 * SK_HALO;  // valid rows per window (240)
 constexpr int SK_P = SK_V / SK_S;    // positions per chain per window (30)
 constexpr int SK_SEG = 8;            // positions per lane segment (4 segments: 8, 8, 8, 6)
-constexpr int SK_NPCR = 12;          // warps
+#ifndef SK_NPCR_DEF
+#define SK_NPCR_DEF 12
+#endif
+constexpr int SK_NPCR = SK_NPCR_DEF;  // warps
+static_assert(SK_NPCR <= 15, "chain handover uses named barriers 1 .. NPCR");
 constexpr int SK_THREADS = 32 * SK_NPCR;
 constexpr int SK_NCMAX = 1024;       // windows per system (one mbarrier per storage slot)
 constexpr int SK_TCS = 34;           // transpose buffer: chain stride (elements; bank-spread)
@@ -247,8 +251,7 @@ __global__ void __launch_bounds__(SK_THREADS, 1) k_stream(const __grid_constant_
     // dynamic smem is only guaranteed 16-byte aligned: align the carve-up to 1 KB
     unsigned char* sbase = sk_smem_raw + ((1024 - ((unsigned)__cvta_generic_to_shared(sk_smem_raw) & 1023)) & 1023);
     uint64_t* in_full = reinterpret_cast<uint64_t*>(sbase + L::off_bar);  // [NPCR] TMA -> warp
-    uint64_t* stfull = in_full + SK_NPCR;                                  // [NPCR] forward state of step g
-    uint64_t* bfull = stfull + SK_NPCR;                                    // [NPCR] backward x of step g
+    uint64_t* bfull = in_full + 2 * SK_NPCR;                               // (layout only)
     // sfull[slot]: one phase per system written into the slot.  A reader waits
     // for phase j-1 only after the write of system j-2 completed: that write was
     // in step (j-2) NC + w', >= 2 NC > NPCR + 1 steps back, and its warp has
@@ -263,8 +266,6 @@ __global__ void __launch_bounds__(SK_THREADS, 1) k_stream(const __grid_constant_
     if (threadIdx.x == 0) {
         for (int i = 0; i < SK_NPCR; ++i) {
             sk_bar_init(&in_full[i], 1);
-            sk_bar_init(&stfull[i], 1);
-            sk_bar_init(&bfull[i], 1);
         }
         for (int i = 0; i < NC; ++i) sk_bar_init(&sfull[i], 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -336,7 +337,6 @@ __global__ void __launch_bounds__(SK_THREADS, 1) k_stream(const __grid_constant_
     const int pi = (pw + SK_NPCR - 1) % SK_NPCR;  // warp of step g - 1
     int it = 0;                                   // this warp's step count
     for (int g = pw; g < total; g += SK_NPCR, ++it) {
-        const unsigned ppar = (unsigned)((it - (pw == 0 ? 1 : 0)) & 1);  // phase parity of step g - 1
         if (prof) tq = clock64();
         const int cj = j, cw = w;
         w += SK_NPCR;
@@ -530,31 +530,29 @@ __global__ void __launch_bounds__(SK_THREADS, 1) k_stream(const __grid_constant_
         }
         SK_PH(5);
 
-        // ---- the two serial steps: x from step g - 1 (backward), state from step g - 1 (forward)
-        T xw = T(0);  // x at position 0 of window wb + 1
-        if (bwd && wb < NC - 1) {
+        // ---- the two serial steps: x (backward) and the state (forward) of step g - 1,
+        // handed over through the hardware named barrier 1 + pi (warp pi -> warp pw,
+        // 64 threads): a waiting warp is descheduled, nothing polls.  Warp pw arrives
+        // on barrier 1 + pw again only after the successor's sync for this step
+        // (its next arrival depends, through the chain, on the successor's step g + 1).
+        if (g > 0) {
             const unsigned long long tb = prof ? clock64() : 0;
-            sk_wait(&bfull[pi], ppar);
-            if (prof) t_bx += clock64() - tb;
-            xw = xh[pi * SK_S + c];
+            asm volatile("bar.sync %0, 64;" ::"r"(1 + pi) : "memory");
+            if (prof) t_st += clock64() - tb;
         }
-        const T xs = fma(be, xw, al);  // x at the first position of segment sg
-        if (sg == 0) xh[pw * SK_S + c] = xs;
-        __syncwarp();
-        if (lane == 0) sk_arrive(&bfull[pw]);
+        const T xw = (bwd && wb < NC - 1) ? xh[pi * SK_S + c] : T(0);  // x at position 0 of window wb + 1
         T th = T(1), ps = T(0), de = T(0);  // theta_{-1} = 1, psi_0 = C_{-1} theta_{-2} = 0 (a_0 = 0)
         if (fwd && cw > 0) {
-            const unsigned long long tb = prof ? clock64() : 0;
-            sk_wait(&stfull[pi], ppar);
-            if (prof) t_st += clock64() - tb;
             const T* si = stt + pi * 3 * SK_S + c;
             th = si[0];
             ps = si[SK_S];
             de = si[2 * SK_S];
         }
+        const T xs = fma(be, xw, al);  // x at the first position of segment sg
         const T ot = fma(M.a, th, M.b * ps);
         const T op = fma(M.c, th, M.d * ps);
         const T od = fma(M.e, th, fma(M.f, ps, M.g * de));
+        if (sg == 0) xh[pw * SK_S + c] = xs;
         if (sg == 3) {  // window end: exact power-of-two rescale, hand over
             const T sc = sk_exp2_scale(ot);
             T* so = stt + pw * 3 * SK_S + c;
@@ -562,8 +560,10 @@ __global__ void __launch_bounds__(SK_THREADS, 1) k_stream(const __grid_constant_
             so[SK_S] = op * sc;
             so[2 * SK_S] = od * sc;
         }
-        __syncwarp();
-        if (lane == 0) sk_arrive(&stfull[pw]);
+        if (g + 1 < total) {
+            __threadfence_block();
+            asm volatile("bar.arrive %0, 64;" ::"r"(1 + pw) : "memory");
+        }
         T x = __shfl_down_sync(0xffffffffu, xs, 8);  // x after segment sg
         if (sg == 3) x = xw;
         {  // incoming state of this lane's segment = outgoing state of segment sg - 1
