@@ -70,7 +70,12 @@ typedef enum {
     TRI_VARIANT_STREAM = 5  /* CONTIGUOUS fp64, n % 8 == 0, n >= 512: tiled PCR (k = 3, TMA-staged 256-row
                                windows with 8-row halos, Eq 8 / Fig 7) streamed into p-Thomas in one
                                persistent kernel; c', d' stay in shared memory / L2, so HBM moves only
-                               the compulsory 5 arrays (Sec. III.C) */
+                               the compulsory 5 arrays (Sec. III.C) */,
+    TRI_VARIANT_SCAN = 6    /* CONTIGUOUS (or m = 1), n % 8 == 0: p-Thomas at k = 0 (M > P) with the
+                               forward sweep (Eqs 2-3) and back substitution (Eq 4) of each system spread
+                               over the 32 lanes of a warp as segment maps combined by a shuffle scan
+                               (X21); 256-row windows chained across warps, c', d' kept in
+                               shared memory / L2: HBM moves only the compulsory 5 arrays */
 } tri_variant;
 
 typedef struct tri_plan_s* tri_plan_t;

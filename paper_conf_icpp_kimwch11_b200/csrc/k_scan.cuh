@@ -1,0 +1,530 @@
+// k_scan.cuh -- TRI_VARIANT_SCAN: p-Thomas at transition point k = 0 (the
+// paper's rule for M > P) for batches of systems in the CONTIGUOUS layout
+// (n % 8 == 0), with the Thomas intermediates kept on chip / in L2, so that HBM
+// moves only the compulsory 5 arrays (read a, b, c, d once; write x once).
+//
+// Paper: Thomas, Eqs 2-4 (reading X2); p-Thomas Sec. III.B
+// (P:645-653); transition point k = 0 for M > P (Sec. III.D).
+//
+// A system is cut into windows of W = 256 rows; lane l of a warp holds rows
+// 8l .. 8l+7 of a window in registers (TMA 2D tile, tensor view [rows/8][8]).
+// The forward sweep is written as the continuant recurrence on the raw rows
+// (X21), with state (theta_{t-1}, psi_t = c_{t-1} theta_{t-2},
+// delta_{t-1}):
+//     theta_t = b_t theta_{t-1} - a_t psi_t,   psi_{t+1} = c_t theta_{t-1},
+//     delta_t = d_t theta_{t-1} - a_t delta_{t-1},
+//     c'_t = psi_{t+1} / theta_t,   d'_t = delta_t / theta_t,
+// algebraically Eqs 2-3 (theta_t / theta_{t-1} is Thomas's pivot
+// b_t - a_t c'_{t-1}).  Each row is a 3x3 linear map of the state, so a lane
+// builds its 8-row segment map, a 5-step shuffle scan composes the 32 segment
+// maps of a window, the window's incoming state is handed over from the warp
+// that ran the previous window (the only serial step: one matrix-vector
+// product), and every lane replays its rows from its true incoming state.  The
+// back substitution (Eq 4, x_t = d'_t - c'_t x_{t+1}) is an affine map per
+// segment, scanned the same way (suffix order), with x handed between windows.
+//
+// Persistent CTAs (one per SM), NW identical warps; step g = j NC + w (system
+// j of this CTA, window w) runs on warp g % NW and does the forward work of
+// window (j, w) and the back substitution of window (j - 1, NC - 1 - w); the
+// latter reads exactly the storage slot the former then rewrites (slot of
+// window w: w for even j, NC - 1 - w for odd j), so one system's worth of
+// (c', d') slots recycles with no extra synchronisation.  The first and last
+// S_on / 2 slots live in shared memory, the middle ones in a per-CTA L2-resident
+// spill region.  Systems of one window (n <= 256) need no chain: each warp solves
+// whole systems on its own (forward and backward in registers).
+#pragma once
+#include "k_stream.cuh"  // sk_* TMA / mbarrier / policy helpers, SKMat
+
+namespace tri {
+
+constexpr int SC_R = 8;            // rows per lane
+constexpr int SC_W = 32 * SC_R;    // rows per window (256)
+#ifndef SC_NW_DEF
+#define SC_NW_DEF 12
+#endif
+constexpr int SC_NW = SC_NW_DEF;   // warps per CTA
+static_assert(SC_NW <= 15, "chain handover uses named barriers 1 .. NW");
+constexpr int SC_THREADS = 32 * SC_NW;
+constexpr int SC_NCMAX = 4096;     // windows per system (per-slot counters live in smem)
+
+template <typename T>
+struct ScanArgs {
+    T* x;
+    T* spill;      // per CTA: (NC - S_on) slots of sc_slot_elems<T>() elements
+    int64_t n, m;
+    int NC;        // windows per system
+    int S_on;      // storage slots resident in shared memory
+    unsigned long long* prof;  // diagnostics (scripts/prof_scan.py): per-phase cycle counters, or null
+    int dbg;       // diagnostics: 1 = no chain handover (wrong results; timing only)
+};
+
+template <typename T>
+__host__ __device__ constexpr int sc_slot_elems() { return 32 * SC_R * 2; }  // (c', d') per row
+
+template <typename T>
+struct SCLayout {
+    static constexpr int in_bytes = 4 * SC_W * (int)sizeof(T);           // one window, 4 arrays
+    static constexpr int in_stride = (in_bytes + 1023) / 1024 * 1024;     // swizzle atoms aligned
+    static constexpr int off_in = 0;
+    static constexpr int off_st = off_in + SC_NW * in_stride;             // [NW][theta|psi|delta]
+    static constexpr int off_xh = off_st + SC_NW * 4 * (int)sizeof(T);    // [NW] x handover
+    static constexpr int off_bar = (off_xh + SC_NW * (int)sizeof(T) + 7) / 8 * 8;  // [NW] in_full
+    static constexpr int off_cnt = off_bar + SC_NW * 8;                   // [NC] slot counters
+    static constexpr int slot_bytes = sc_slot_elems<T>() * (int)sizeof(T);
+    static __host__ __device__ constexpr int off_store(int NC) { return (off_cnt + 4 * NC + 1023) / 1024 * 1024; }
+    static __host__ __device__ constexpr int smem_bytes(int NC, int S_on) {
+        return off_store(NC) + S_on * slot_bytes + 1024;  // + alignment slack
+    }
+};
+
+// 16-byte chunk `ch` of lane `lane` in a storage slot, holding (c', d') of row
+// ch [fp64] or rows (2 ch, 2 ch + 1) [fp32] of the lane: chunk-major, so one
+// warp access covers 512 contiguous bytes (conflict-free in shared memory,
+// full sectors in L2).
+template <typename T>
+__device__ __forceinline__ int sc_chunk(int lane, int ch) {
+    return ch * 32 + lane;
+}
+
+// exact power-of-two scale 2^-e bringing max(|u|, |v|) into [1, 2) (projective
+// rescale of a map or state: ratios c', d' are unchanged)
+template <typename T>
+__device__ __forceinline__ T sc_scale2(T u, T v) {
+    return sk_exp2_scale(fmax(fabs(u), fabs(v)));
+}
+
+template <typename T>
+__device__ __forceinline__ void sc_ld_rows(const T* ib, int lane, T (&ra)[SC_R], T (&rb)[SC_R], T (&rc)[SC_R],
+                                           T (&rd)[SC_R]) {
+    constexpr int EPC = 16 / (int)sizeof(T);   // elements per 16-byte chunk
+    constexpr int CPL = SC_R / EPC;            // chunks per lane-row
+    const int swz = sizeof(T) == 8 ? ((lane >> 1) & 3) : ((lane >> 2) & 1);  // TMA 64B / 32B swizzle
+    const T* st = ib + lane * SC_R;
+#pragma unroll
+    for (int cc = 0; cc < CPL; ++cc) {
+        const int o = (cc ^ swz) * EPC;
+        const int4 va = *reinterpret_cast<const int4*>(st + 0 * SC_W + o);
+        const int4 vb = *reinterpret_cast<const int4*>(st + 1 * SC_W + o);
+        const int4 vc = *reinterpret_cast<const int4*>(st + 2 * SC_W + o);
+        const int4 vd = *reinterpret_cast<const int4*>(st + 3 * SC_W + o);
+#pragma unroll
+        for (int e = 0; e < EPC; ++e) {
+            ra[cc * EPC + e] = reinterpret_cast<const T*>(&va)[e];
+            rb[cc * EPC + e] = reinterpret_cast<const T*>(&vb)[e];
+            rc[cc * EPC + e] = reinterpret_cast<const T*>(&vc)[e];
+            rd[cc * EPC + e] = reinterpret_cast<const T*>(&vd)[e];
+        }
+    }
+}
+
+// rows outside [0, n) are identity rows; a_0 and c_{n-1} lie outside A (X1, X4)
+template <typename T>
+__device__ __forceinline__ void sc_fix_rows(int64_t i0, int64_t n, T (&ra)[SC_R], T (&rb)[SC_R], T (&rc)[SC_R],
+                                            T (&rd)[SC_R]) {
+#pragma unroll
+    for (int u = 0; u < SC_R; ++u) {
+        const int64_t i = i0 + u;
+        if (i == 0) ra[u] = T(0);
+        if (i == n - 1) rc[u] = T(0);
+        if (i >= n) { ra[u] = T(0); rb[u] = T(1); rc[u] = T(0); rd[u] = T(0); }
+    }
+}
+
+// segment map of the lane's rows (forward state transfer, X21),
+// rescaled by an exact power of two
+template <typename T>
+__device__ __forceinline__ SKMat<T> sc_fwd_map(const T (&ra)[SC_R], const T (&rb)[SC_R], const T (&rc)[SC_R],
+                                               const T (&rd)[SC_R]) {
+    // row 0 applied to the identity
+    T t1 = rb[0], p1 = rc[0], d1 = rd[0];      // response to theta_in
+    T t2 = -ra[0], p2 = T(0), d2 = T(0);       // ... to psi_in
+    T d3 = -ra[0];                             // ... to delta_in
+#pragma unroll
+    for (int u = 1; u < SC_R; ++u) {
+        const T nt1 = fma(rb[u], t1, -ra[u] * p1), np1 = rc[u] * t1, nd1 = fma(rd[u], t1, -ra[u] * d1);
+        const T nt2 = fma(rb[u], t2, -ra[u] * p2), np2 = rc[u] * t2, nd2 = fma(rd[u], t2, -ra[u] * d2);
+        d3 = -ra[u] * d3;
+        t1 = nt1; p1 = np1; d1 = nd1;
+        t2 = nt2; p2 = np2; d2 = nd2;
+    }
+    const T s = sc_scale2(t1, t2);
+    return SKMat<T>{t1 * s, t2 * s, p1 * s, p2 * s, d1 * s, d2 * s, d3 * s};
+}
+
+// both scans in one pass (their shuffles and arithmetic interleave): forward
+// inclusive over the lanes, backward suffix
+template <typename T>
+__device__ __forceinline__ void sc_scans(SKMat<T>& M, T& al, T& be, int lane) {
+#pragma unroll
+    for (int dd = 1; dd < 32; dd <<= 1) {
+        const SKMat<T> o = sk_shfl_up(M, dd);
+        T oa = __shfl_down_sync(0xffffffffu, al, dd), ob = __shfl_down_sync(0xffffffffu, be, dd);
+        if (lane + dd >= 32) { oa = T(0); ob = T(1); }
+        al = fma(be, oa, al);
+        be = be * ob;
+        if (lane >= dd) M = sk_compose(M, o);
+    }
+}
+
+// inclusive scan of the segment maps over the lanes (lane order = row order)
+template <typename T>
+__device__ __forceinline__ void sc_fwd_scan(SKMat<T>& M, int lane) {
+#pragma unroll
+    for (int dd = 1; dd < 32; dd <<= 1) {
+        const SKMat<T> o = sk_shfl_up(M, dd);
+        if (lane >= dd) M = sk_compose(M, o);
+    }
+}
+
+// back-substitution map of the lane's rows: x_first = al + be * x_after
+template <typename T>
+__device__ __forceinline__ void sc_bwd_map(const T (&cp)[SC_R], const T (&dp)[SC_R], T& al, T& be) {
+    al = dp[SC_R - 1];
+    be = -cp[SC_R - 1];
+#pragma unroll
+    for (int t = SC_R - 2; t >= 0; --t) {
+        al = fma(-cp[t], al, dp[t]);
+        be = -cp[t] * be;
+    }
+}
+// suffix scan over the lanes: lane l maps x after lane 31 to x at its first row
+template <typename T>
+__device__ __forceinline__ void sc_bwd_scan(T& al, T& be, int lane) {
+#pragma unroll
+    for (int dd = 1; dd < 32; dd <<= 1) {
+        const T oa = __shfl_down_sync(0xffffffffu, al, dd), ob = __shfl_down_sync(0xffffffffu, be, dd);
+        if (lane + dd < 32) { al = fma(be, oa, al); be = be * ob; }
+    }
+}
+
+// forward replay from the lane's incoming state: c', d' of its rows
+template <typename T>
+__device__ __forceinline__ void sc_fwd_replay(const T (&ra)[SC_R], const T (&rb)[SC_R], const T (&rc)[SC_R],
+                                              const T (&rd)[SC_R], T th, T ps, T de, T (&cp)[SC_R], T (&dp)[SC_R]) {
+#pragma unroll
+    for (int u = 0; u < SC_R; ++u) {
+        const T nt = fma(rb[u], th, -ra[u] * ps);
+        const T np = rc[u] * th;
+        const T nd = fma(rd[u], th, -ra[u] * de);
+        const T inv = rcp(nt);
+        cp[u] = np * inv;
+        dp[u] = nd * inv;
+        th = nt; ps = np; de = nd;
+    }
+}
+
+// storage-slot access: shared memory (resident slots) or the per-CTA global
+// spill region (L2, evict_last), with explicit state spaces (no generic ops)
+__device__ __forceinline__ void sc_sts2(unsigned a, double x, double y) {
+    asm volatile("st.shared.v2.f64 [%0], {%1, %2};" ::"r"(a), "d"(x), "d"(y) : "memory");
+}
+__device__ __forceinline__ void sc_lds2(unsigned a, double& x, double& y) {
+    asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(x), "=d"(y) : "r"(a) : "memory");
+}
+__device__ __forceinline__ void sc_sts4(unsigned a, float x, float y, float z, float w) {
+    asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};" ::"r"(a), "f"(x), "f"(y), "f"(z), "f"(w) : "memory");
+}
+__device__ __forceinline__ void sc_lds4(unsigned a, float& x, float& y, float& z, float& w) {
+    asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(x), "=f"(y), "=f"(z), "=f"(w) : "r"(a) : "memory");
+}
+__device__ __forceinline__ void sc_stg4_last(float* p, float x, float y, float z, float w, uint64_t pol) {
+    asm volatile("st.global.L2::cache_hint.v4.f32 [%0], {%1, %2, %3, %4}, %5;" ::"l"(p), "f"(x), "f"(y), "f"(z),
+                 "f"(w), "l"(pol)
+                 : "memory");
+}
+
+template <typename T>
+__device__ __forceinline__ void sc_store_slot_s(unsigned base, int lane, const T (&cp)[SC_R], const T (&dp)[SC_R]) {
+    if constexpr (sizeof(T) == 8) {
+#pragma unroll
+        for (int t = 0; t < SC_R; ++t) sc_sts2(base + 16u * sc_chunk<T>(lane, t), cp[t], dp[t]);
+    } else {
+#pragma unroll
+        for (int t = 0; t < SC_R / 2; ++t)
+            sc_sts4(base + 16u * sc_chunk<T>(lane, t), cp[2 * t], dp[2 * t], cp[2 * t + 1], dp[2 * t + 1]);
+    }
+}
+template <typename T>
+__device__ __forceinline__ void sc_store_slot_g(T* base, int lane, const T (&cp)[SC_R], const T (&dp)[SC_R],
+                                                uint64_t pol) {
+    if constexpr (sizeof(T) == 8) {
+#pragma unroll
+        for (int t = 0; t < SC_R; ++t) sk_st_global_last(base + 2 * sc_chunk<T>(lane, t), cp[t], dp[t], pol);
+    } else {
+#pragma unroll
+        for (int t = 0; t < SC_R / 2; ++t)
+            sc_stg4_last(base + 4 * sc_chunk<T>(lane, t), cp[2 * t], dp[2 * t], cp[2 * t + 1], dp[2 * t + 1], pol);
+    }
+}
+template <typename T>
+__device__ __forceinline__ void sc_load_slot_s(unsigned base, int lane, T (&cp)[SC_R], T (&dp)[SC_R]) {
+    if constexpr (sizeof(T) == 8) {
+#pragma unroll
+        for (int t = 0; t < SC_R; ++t) sc_lds2(base + 16u * sc_chunk<T>(lane, t), cp[t], dp[t]);
+    } else {
+#pragma unroll
+        for (int t = 0; t < SC_R / 2; ++t)
+            sc_lds4(base + 16u * sc_chunk<T>(lane, t), cp[2 * t], dp[2 * t], cp[2 * t + 1], dp[2 * t + 1]);
+    }
+}
+template <typename T>
+__device__ __forceinline__ void sc_load_slot_g(const T* base, int lane, T (&cp)[SC_R], T (&dp)[SC_R]) {
+    if constexpr (sizeof(T) == 8) {
+#pragma unroll
+        for (int t = 0; t < SC_R; ++t) {
+            const double2 v = __ldcg(reinterpret_cast<const double2*>(base + 2 * sc_chunk<T>(lane, t)));
+            cp[t] = v.x;
+            dp[t] = v.y;
+        }
+    } else {
+#pragma unroll
+        for (int t = 0; t < SC_R / 2; ++t) {
+            const float4 v = __ldcg(reinterpret_cast<const float4*>(base + 4 * sc_chunk<T>(lane, t)));
+            cp[2 * t] = v.x; dp[2 * t] = v.y; cp[2 * t + 1] = v.z; dp[2 * t + 1] = v.w;
+        }
+    }
+}
+
+// x of the lane's rows (first row global index xi) -> global, streaming stores
+template <typename T>
+__device__ __forceinline__ void sc_store_x(T* xo, int64_t rmax, const T (&xv)[SC_R]) {
+    if (rmax >= SC_R) {
+        if constexpr (sizeof(T) == 8) {
+#pragma unroll
+            for (int t = 0; t < SC_R; t += 4)
+                asm volatile("st.global.cs.v4.f64 [%0], {%1, %2, %3, %4};" ::"l"(xo + t), "d"(xv[t]), "d"(xv[t + 1]),
+                             "d"(xv[t + 2]), "d"(xv[t + 3])
+                             : "memory");
+        } else {
+#pragma unroll
+            for (int t = 0; t < SC_R; t += 4)
+                __stcs(reinterpret_cast<float4*>(xo + t), make_float4(xv[t], xv[t + 1], xv[t + 2], xv[t + 3]));
+        }
+    } else {
+#pragma unroll
+        for (int t = 0; t < SC_R; ++t)
+            if (t < rmax) __stcs(xo + t, xv[t]);
+    }
+}
+
+template <typename T, bool PROF>
+__global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ StreamMaps tm, ScanArgs<T> p) {
+    using L = SCLayout<T>;
+    extern __shared__ __align__(16) unsigned char sc_smem_raw[];
+    unsigned char* sbase = sc_smem_raw + ((1024 - ((unsigned)__cvta_generic_to_shared(sc_smem_raw) & 1023)) & 1023);
+    uint64_t* in_full = reinterpret_cast<uint64_t*>(sbase + L::off_bar);  // [NW] TMA -> warp
+    int* cnt = reinterpret_cast<int*>(sbase + L::off_cnt);                // [NC] systems stored per slot
+    T* stt = reinterpret_cast<T*>(sbase + L::off_st);
+    T* xh = reinterpret_cast<T*>(sbase + L::off_xh);
+    const int NC = p.NC;
+    const unsigned store_s = (unsigned)__cvta_generic_to_shared(sbase + L::off_store(NC));
+
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (threadIdx.x == 0) {
+        for (int i = 0; i < SC_NW; ++i) sk_bar_init(&in_full[i], 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    }
+    for (int i = threadIdx.x; i < NC; i += blockDim.x) cnt[i] = 0;
+    __syncthreads();
+
+    const int64_t n = p.n;
+    const int nsys = (int)((p.m - blockIdx.x + gridDim.x - 1) / gridDim.x);
+    const int pw = warp;
+    T* ib = reinterpret_cast<T*>(sbase + L::off_in + pw * L::in_stride);
+    const uint64_t pol_in = sk_policy_evict_first();
+    const uint64_t pol_sp = sk_policy_evict_last();
+    auto issue = [&](int jj, int ww) {
+        const int64_t q = blockIdx.x + (int64_t)jj * gridDim.x;
+        const int y = (int)((q * n + (int64_t)ww * SC_W) >> 3);  // n % 8 == 0
+        sk_expect(&in_full[pw], (unsigned)(4 * SC_W * sizeof(T)));
+        sk_tma2d(ib + 0 * SC_W, &tm.a, 0, y, &in_full[pw], pol_in);
+        sk_tma2d(ib + 1 * SC_W, &tm.b, 0, y, &in_full[pw], pol_in);
+        sk_tma2d(ib + 2 * SC_W, &tm.c, 0, y, &in_full[pw], pol_in);
+        sk_tma2d(ib + 3 * SC_W, &tm.d, 0, y, &in_full[pw], pol_in);
+    };
+    unsigned ph = 0;
+
+    if (NC == 1) {
+        // ---- systems of one window: each warp solves whole systems, no chain
+        if (lane == 0 && pw < nsys) issue(pw, 0);
+        for (int j = pw; j < nsys; j += SC_NW) {
+            const int64_t q = blockIdx.x + (int64_t)j * gridDim.x;
+            T ra[SC_R], rb[SC_R], rc[SC_R], rd[SC_R];
+            sk_wait(&in_full[pw], ph);
+            ph ^= 1u;
+            sc_ld_rows(ib, lane, ra, rb, rc, rd);
+            __syncwarp();
+            if (lane == 0 && j + SC_NW < nsys) issue(j + SC_NW, 0);
+            sc_fix_rows<T>((int64_t)lane * SC_R, n, ra, rb, rc, rd);
+            SKMat<T> M = sc_fwd_map(ra, rb, rc, rd);
+            sc_fwd_scan(M, lane);
+            // incoming state of the lane = outgoing state of lane - 1 (window starts at (1, 0, 0))
+            T th = __shfl_up_sync(0xffffffffu, M.a, 1), ps = __shfl_up_sync(0xffffffffu, M.c, 1),
+              de = __shfl_up_sync(0xffffffffu, M.e, 1);
+            if (lane == 0) { th = T(1); ps = T(0); de = T(0); }
+            T cp[SC_R], dp[SC_R];
+            sc_fwd_replay(ra, rb, rc, rd, th, ps, de, cp, dp);
+            T al, be;
+            sc_bwd_map(cp, dp, al, be);
+            sc_bwd_scan(al, be, lane);
+            // x after the lane's rows = x at the first row of lane + 1 (al of lane + 1: x after lane 31 is 0)
+            T x = __shfl_down_sync(0xffffffffu, al, 1);
+            if (lane == 31) x = T(0);
+            T xv[SC_R];
+#pragma unroll
+            for (int t = SC_R - 1; t >= 0; --t) {
+                x = fma(-cp[t], x, dp[t]);
+                xv[t] = x;
+            }
+            sc_store_x(p.x + q * n + lane * SC_R, n - (int64_t)lane * SC_R, xv);
+        }
+        return;
+    }
+
+    const int nfwd = nsys * NC;             // forward steps
+    const int total = (nsys + 1) * NC;      // + the back substitution of the last system
+    const int nspill = NC - p.S_on;
+    T* spill_cta = p.spill + (int64_t)blockIdx.x * (int64_t)(nspill > 0 ? nspill : 0) * sc_slot_elems<T>();
+    int j = 0, w = pw;
+    while (w >= NC) { w -= NC; ++j; }
+    if (lane == 0 && pw < nfwd) issue(j, w);
+    auto slot_of = [&](int jj, int ww) { return (jj & 1) ? NC - 1 - ww : ww; };
+    const int pi = (pw + SC_NW - 1) % SC_NW;  // warp of step g - 1
+    unsigned long long pc[8] = {0, 0, 0, 0, 0, 0, 0, 0}, t0 = PROF ? clock64() : 0, tp = t0;
+#define SC_T(k) do { if (PROF) { const unsigned long long tn_ = clock64(); pc[k] += tn_ - tp; tp = tn_; } } while (0)
+    for (int g = pw; g < total; g += SC_NW) {
+        const int cj = j, cw = w;
+        w += SC_NW;
+        while (w >= NC) { w -= NC; ++j; }
+        const bool fwd = cj < nsys, bwd = cj >= 1;
+        const int wb = NC - 1 - cw;  // backward window (system cj - 1)
+        const int slot = slot_of(cj, cw);
+        const int64_t i0d = (int64_t)cw * SC_W + lane * SC_R;
+        int sidx;
+        const bool res = sk_resident(slot, NC, p.S_on, sidx);
+        const unsigned sp_s = store_s + (unsigned)(sidx * L::slot_bytes);
+        T* sp_g = spill_cta + (size_t)sidx * sc_slot_elems<T>();
+
+        if (p.dbg == 2) {  // diagnostics: the memory pipeline alone (inputs in, x out; no math)
+            if (fwd) {
+                sk_wait(&in_full[pw], ph);
+                ph ^= 1u;
+                __syncwarp();
+                if (lane == 0 && g + SC_NW < nfwd) issue(j, w);
+                T xv[SC_R];
+#pragma unroll
+                for (int t = 0; t < SC_R; ++t) xv[t] = T(0);
+                const int64_t q = blockIdx.x + (int64_t)cj * gridDim.x;
+                sc_store_x(p.x + q * n + i0d, n - i0d, xv);
+            }
+            continue;
+        }
+        // ---- backward: (c', d') of window (cj - 1, wb) from the slot (held in registers)
+        T cpb[SC_R], dpb[SC_R];
+        if (bwd) {
+            SC_T(5);
+            sk_wait_ge(&cnt[slot], cj);  // system cj - 1 stored in the slot
+            SC_T(4);
+            if (res) sc_load_slot_s(sp_s, lane, cpb, dpb);
+            else sc_load_slot_g(sp_g, lane, cpb, dpb);
+        } else {
+#pragma unroll
+            for (int t = 0; t < SC_R; ++t) { cpb[t] = T(0); dpb[t] = T(0); }
+        }
+
+        // ---- forward: segment map of window (cj, cw) (identity rows when inactive);
+        // the rows are read again from the staging buffer for the replay
+        const int64_t i0 = (int64_t)cw * SC_W + lane * SC_R;
+        const bool edge = cw == 0 || (int64_t)(cw + 1) * SC_W > n;
+        SKMat<T> M;
+        if (fwd) {
+            SC_T(5);
+            sk_wait(&in_full[pw], ph);
+            SC_T(1);
+            ph ^= 1u;
+            T ra[SC_R], rb[SC_R], rc[SC_R], rd[SC_R];
+            sc_ld_rows(ib, lane, ra, rb, rc, rd);
+            if (edge) sc_fix_rows<T>(i0, n, ra, rb, rc, rd);
+            M = sc_fwd_map(ra, rb, rc, rd);
+        } else {
+            M = SKMat<T>{T(1), T(0), T(0), T(1), T(0), T(0), T(1)};
+        }
+        T al, be;
+        sc_bwd_map(cpb, dpb, al, be);
+        sc_scans(M, al, be, lane);
+
+        // ---- the serial steps: the forward state and x of step g - 1, handed over
+        // through the hardware named barrier 1 + pi (warp pi -> warp pw, 64 threads)
+        SC_T(5);
+        if (g > 0 && p.dbg != 1) asm volatile("bar.sync %0, 64;" ::"r"(1 + pi) : "memory");
+        SC_T(2);
+        const T xw = (bwd && wb < NC - 1) ? xh[pi] : T(0);  // x at the first row of window wb + 1
+        T th = T(1), ps = T(0), de = T(0);                  // theta_{-1} = 1, psi_0 = 0, delta_{-1} = 0
+        if (fwd && cw > 0) {
+            th = stt[pi * 4 + 0];
+            ps = stt[pi * 4 + 1];
+            de = stt[pi * 4 + 2];
+        }
+        const T xs = fma(be, xw, al);  // x at the lane's first row
+        const T ot = fma(M.a, th, M.b * ps);
+        const T op = fma(M.c, th, M.d * ps);
+        const T od = fma(M.e, th, fma(M.f, ps, M.g * de));
+        if (lane == 0) xh[pw] = xs;
+        if (lane == 31) {  // window end: exact power-of-two rescale, hand over
+            const T sc = sk_exp2_scale(ot);
+            stt[pw * 4 + 0] = ot * sc;
+            stt[pw * 4 + 1] = op * sc;
+            stt[pw * 4 + 2] = od * sc;
+        }
+        if (g + 1 < total && p.dbg != 1) {
+            __threadfence_block();
+            asm volatile("bar.arrive %0, 64;" ::"r"(1 + pw) : "memory");
+        }
+        SC_T(3);
+        T x = __shfl_down_sync(0xffffffffu, xs, 1);  // x after the lane's rows
+        if (lane == 31) x = xw;
+        {
+            const T it_ = __shfl_up_sync(0xffffffffu, ot, 1);
+            const T ip = __shfl_up_sync(0xffffffffu, op, 1);
+            const T id = __shfl_up_sync(0xffffffffu, od, 1);
+            if (lane > 0) { th = it_; ps = ip; de = id; }
+        }
+
+        // ---- forward replay: c', d' (Eqs 2-3) of window (cj, cw) into the slot,
+        // then the next input window of this warp
+        if (fwd) {
+            T ra[SC_R], rb[SC_R], rc[SC_R], rd[SC_R];
+            sc_ld_rows(ib, lane, ra, rb, rc, rd);
+            if (edge) sc_fix_rows<T>(i0, n, ra, rb, rc, rd);
+            __syncwarp();
+            if (lane == 0 && g + SC_NW < nfwd) issue(j, w);
+            T cpf[SC_R], dpf[SC_R];
+            sc_fwd_replay(ra, rb, rc, rd, th, ps, de, cpf, dpf);
+            if (res) sc_store_slot_s(sp_s, lane, cpf, dpf);
+            else sc_store_slot_g(sp_g, lane, cpf, dpf, pol_sp);
+            __syncwarp();
+            if (lane == 0) sk_st_release(&cnt[slot], cj + 1);
+        }
+        // ---- backward replay: x (Eq 4) of window (cj - 1, wb)
+        if (bwd) {
+            T xv[SC_R];
+#pragma unroll
+            for (int t = SC_R - 1; t >= 0; --t) {
+                x = fma(-cpb[t], x, dpb[t]);
+                xv[t] = x;
+            }
+            const int64_t qb = blockIdx.x + (int64_t)(cj - 1) * gridDim.x;
+            const int64_t xr = (int64_t)wb * SC_W + lane * SC_R;
+            sc_store_x(p.x + qb * n + xr, n - xr, xv);
+        }
+        SC_T(6);
+    }
+    if (PROF && lane == 0) {
+        pc[0] = clock64() - t0;
+        for (int k = 0; k < 8; ++k) atomicAdd(&p.prof[k], pc[k]);
+    }
+#undef SC_T
+}
+
+}  // namespace tri

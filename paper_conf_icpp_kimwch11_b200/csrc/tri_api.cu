@@ -19,6 +19,7 @@
 #include "k_pthomas.cuh"
 #include "k_fused.cuh"
 #include "k_stream.cuh"
+#include "k_scan.cuh"
 #include "k_warp.cuh"
 #include "k_pthomas_tma.cuh"
 
@@ -88,6 +89,14 @@ bool stream_ok(int64_t n, int64_t m, tri_dtype t, tri_layout layout) {
            cdiv(n, SK_V) >= 8 && cdiv(n, SK_V) <= SK_NCMAX && (n / 8) * m < ((int64_t)1 << 31);
 }
 
+// SCAN: contiguous (or one system), n a multiple of 8 (the TMA tensor view
+// [rows/8][8]), at most SC_NCMAX windows of 256 rows; tensor rows fit int32.
+bool scan_ok(int64_t n, int64_t m, tri_dtype t, tri_layout layout) {
+    (void)t;
+    return (layout == TRI_LAYOUT_CONTIGUOUS || m == 1) && n % 8 == 0 && cdiv(n, SC_W) <= SC_NCMAX &&
+           (n / 8) * m < ((int64_t)1 << 31);
+}
+
 // Variant choice, calibrated once on B200 (the paper tunes P once) from
 // scripts/sweep_k.py (profiles/r01_sweep_k_*.jsonl): every (variant, k) timed
 // over the paper's shape grid (fixed n with m swept, fixed m with n swept).
@@ -130,6 +139,7 @@ int choose_k_for(tri_variant v, int64_t n, int64_t m, tri_dtype t, tri_layout la
     if (v == TRI_VARIANT_FUSED) return FU_K;
     if (v == TRI_VARIANT_STREAM) return SK_K;
     if (v == TRI_VARIANT_WARP) return WARP_K;
+    if (v == TRI_VARIANT_SCAN) return 0;
     const int64_t P = (int64_t)sms * 64;
     if (m >= 48 * (int64_t)sms) return 0;
     int k = m >= P ? 0 : ceil_log2(cdiv(P, m));
@@ -142,6 +152,7 @@ int kmax_for(tri_variant v, int64_t n) {
     if (v == TRI_VARIANT_FUSED) return FU_K;
     if (v == TRI_VARIANT_STREAM) return SK_K;
     if (v == TRI_VARIANT_WARP) return WARP_K;
+    if (v == TRI_VARIANT_SCAN) return 0;
     return v == TRI_VARIANT_SPLIT ? std::min(kn, SPLIT_KMAX) : kn;
 }
 int kmin_for(tri_variant v) {
@@ -301,6 +312,16 @@ void plan_geometry(tri_plan_s* p) {
         const int64_t avail = ((int64_t)p->smem_optin - SKLayout<double>::off_store - 1024) / SKLayout<double>::slot_bytes;
         p->sk_son = (int)std::max<int64_t>(0, std::min<int64_t>(p->sk_nc, avail));
     }
+    if (p->variant == TRI_VARIANT_SCAN) {
+        p->L = n; p->n_pad = n; p->C = m;
+        p->sk_nc = (int)cdiv(n, SC_W);
+        p->sk_grid = (int)std::min<int64_t>(m, p->sms);
+        const int fixed = p->dtype == TRI_F64 ? SCLayout<double>::smem_bytes(p->sk_nc, 0)
+                                              : SCLayout<float>::smem_bytes(p->sk_nc, 0);
+        const int slot = p->dtype == TRI_F64 ? SCLayout<double>::slot_bytes : SCLayout<float>::slot_bytes;
+        const int64_t avail = ((int64_t)p->smem_optin - fixed) / slot;
+        p->sk_son = p->sk_nc == 1 ? 0 : (int)std::max<int64_t>(0, std::min<int64_t>(p->sk_nc, avail));
+    }
     if (p->variant == TRI_VARIANT_FUSED) {
         const size_t s = esize(p->dtype);
         p->L = cdiv(n, FU_S);
@@ -318,6 +339,10 @@ void plan_geometry(tri_plan_s* p) {
 }
 
 size_t scratch_need(const tri_plan_s* p) {
+    if (p->variant == TRI_VARIANT_SCAN)
+        return p->sk_nc == 1 ? 0
+                             : (size_t)p->sk_grid * (size_t)std::max(0, p->sk_nc - p->sk_son) *
+                                   (size_t)sc_slot_elems<double>() * esize(p->dtype);
     if (p->variant == TRI_VARIANT_STREAM)
         return (size_t)p->sk_grid * (size_t)std::max(0, p->sk_nc - p->sk_son) * SK_SLOT * esize(p->dtype);
     if (p->variant == TRI_VARIANT_FUSED)
@@ -554,6 +579,42 @@ cudaError_t launch_stream(const tri_plan_s* p, const void* a, const void* b, con
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     kern<<<p->sk_grid, SK_THREADS, smem, st>>>(tm, A);
+    return cudaGetLastError();
+}
+
+// ---- SCAN launch: tensor maps [n m / 8][8] (fp64: 64-byte rows, 64B swizzle;
+// fp32: 32-byte rows, 32B swizzle), box 8 x 32 = one 256-row window per array
+bool tma_map_rows8_f32(CUtensorMap* tm, const void* base, uint64_t rows8) {
+    auto enc = tma_encoder();
+    if (!enc) return false;
+    cuuint64_t dims[2] = {8, rows8};
+    cuuint64_t strides[1] = {8 * sizeof(float)};
+    cuuint32_t box[2] = {8, 32};
+    cuuint32_t es[2] = {1, 1};
+    return enc(tm, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<void*>(base), dims, strides, box, es,
+               CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_32B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+template <typename T>
+cudaError_t launch_scan(const tri_plan_s* p, const void* a, const void* b, const void* c, const void* d, void* x,
+                        cudaStream_t st) {
+    StreamMaps tm;
+    const uint64_t rows8 = (uint64_t)(p->n / 8) * (uint64_t)p->m;
+    auto mk = sizeof(T) == 8 ? tma_map_rows8 : tma_map_rows8_f32;
+    if (!mk(&tm.a, a, rows8) || !mk(&tm.b, b, rows8) || !mk(&tm.c, c, rows8) || !mk(&tm.d, d, rows8))
+        return cudaErrorNotSupported;
+    ScanArgs<T> A;
+    A.x = (T*)x;
+    A.spill = (T*)p->scratch;
+    A.n = p->n; A.m = p->m; A.NC = p->sk_nc; A.S_on = p->sk_son;
+    A.prof = (unsigned long long*)g_fused_prof;
+    A.dbg = g_fused_dbg_mode;
+    const size_t smem = (size_t)SCLayout<T>::smem_bytes(p->sk_nc, p->sk_son);
+    auto kern = A.prof ? k_scan<T, true> : k_scan<T, false>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    kern<<<p->sk_grid, SC_THREADS, smem, st>>>(tm, A);
     return cudaGetLastError();
 }
 
@@ -845,8 +906,9 @@ tri_status tri_plan_set_variant(tri_plan_t p, tri_variant v) {
     if (v == TRI_VARIANT_FUSED && !fused_ok(p->n, p->m, p->layout)) return TRI_ERR_INVALID_ARG;
     if (v == TRI_VARIANT_WARP && !warp_ok(p->n)) return TRI_ERR_INVALID_ARG;
     if (v == TRI_VARIANT_STREAM && !stream_ok(p->n, p->m, p->dtype, p->layout)) return TRI_ERR_INVALID_ARG;
+    if (v == TRI_VARIANT_SCAN && !scan_ok(p->n, p->m, p->dtype, p->layout)) return TRI_ERR_INVALID_ARG;
     if (v != TRI_VARIANT_ONCHIP && v != TRI_VARIANT_SPLIT && v != TRI_VARIANT_FUSED && v != TRI_VARIANT_WARP &&
-        v != TRI_VARIANT_STREAM)
+        v != TRI_VARIANT_STREAM && v != TRI_VARIANT_SCAN)
         return TRI_ERR_INVALID_ARG;
     const tri_variant ov = p->variant;
     const int ok = p->k;
@@ -861,7 +923,7 @@ tri_status tri_plan_set_variant(tri_plan_t p, tri_variant v) {
 void tri_plan_describe(tri_plan_t p, char* buf, int len) {
     if (!buf || len <= 0) return;
     if (!p) { snprintf(buf, len, "null plan"); return; }
-    static const char* vn[] = {"auto", "onchip", "split", "fused", "warp", "stream"};
+    static const char* vn[] = {"auto", "onchip", "split", "fused", "warp", "stream", "scan"};
     snprintf(buf, len,
              "n=%lld m=%lld dtype=%s layout=%s variant=%s k=%d G=%d P=%d rpt=%d L=%lld C=%lld region=%lld nreg=%lld "
              "fu_grid=%d fu_son=%d fu_nc=%lld sk_grid=%d sk_nc=%d sk_son=%d scratch=%zu sms=%d",
@@ -888,6 +950,8 @@ tri_status tri_solve(tri_plan_t p, const void* a, const void* b, const void* c, 
                                 : launch_onchip<float>(p, a, b, c, d, x, nullptr, nullptr, nullptr, 0, s);
     } else if (p->variant == TRI_VARIANT_STREAM) {
         e = launch_stream(p, a, b, c, d, x, s);
+    } else if (p->variant == TRI_VARIANT_SCAN) {
+        e = p->dtype == TRI_F64 ? launch_scan<double>(p, a, b, c, d, x, s) : launch_scan<float>(p, a, b, c, d, x, s);
     } else if (p->variant == TRI_VARIANT_FUSED) {
         e = p->dtype == TRI_F64 ? launch_fused<double>(p, a, b, c, d, x, s) : launch_fused<float>(p, a, b, c, d, x, s);
     } else {
@@ -913,6 +977,8 @@ tri_status tri_debug_pcr(tri_plan_t p, const void* a, const void* b, const void*
                                 : launch_onchip<float>(p, a, b, c, d, nullptr, ao, co, do_, 1, s);
     } else if (p->variant == TRI_VARIANT_STREAM) {
         e = launch_stream(p, a, b, c, d, nullptr, s, ao, co, do_);
+    } else if (p->variant == TRI_VARIANT_SCAN) {
+        return TRI_ERR_INVALID_ARG;  // k = 0: no PCR stage to show
     } else if (p->variant == TRI_VARIANT_FUSED) {
         e = p->dtype == TRI_F64 ? launch_fused<double>(p, a, b, c, d, nullptr, s, ao, co, do_)
                                 : launch_fused<float>(p, a, b, c, d, nullptr, s, ao, co, do_);

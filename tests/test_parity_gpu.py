@@ -393,6 +393,86 @@ def test_stream_full_size_sampled(cuda_ok):
         check_parity(n, 1, sub, x[sl], "f64", 0)
 
 
+# ------------------------------------------------------------------ SCAN variant
+SCAN = tri.VARIANT_SCAN
+
+
+@pytest.mark.parametrize("dtype", ["f64", "f32"])
+@pytest.mark.parametrize("n,m", [(8, 5), (248, 300), (256, 1000), (264, 3), (512, 7), (1936, 2), (2048, 5),
+                                 (4104, 2), (16384, 7), (16392, 150), (2400, 300), (6000, 149), (100000, 2),
+                                 (245760, 2), (1 << 20, 1)])
+def test_scan_parity(cuda_ok, dtype, n, m):
+    """Spans: one-window systems (n <= 256: no chain), NC = 2 with an 8-row last
+    window, NC up to 4096 (most slots spilled), ragged last windows, one and
+    several systems per CTA (both slot parities), m > #SMs."""
+    arrs = gen(n, m, dtype, 0)
+    x, plan = gpu_solve(n, m, arrs, dtype, 0, variant=SCAN)
+    assert plan.variant == SCAN and plan.k == 0
+    check_parity(n, m, arrs, x, dtype, 0)
+
+
+@pytest.mark.parametrize("family,eps", [("weak", 1e-2), ("weak", 1e-3), ("integer", 0.0), ("poisson", 0.0)])
+@pytest.mark.parametrize("n,m", [(16384, 6), (256, 40)])
+def test_scan_families(cuda_ok, family, eps, n, m):
+    arrs = gen(n, m, "f64", 0, family, eps=eps)
+    x, _ = gpu_solve(n, m, arrs, "f64", 0, variant=SCAN)
+    if family == "poisson":
+        xo = oracle.solve_batch(n, m, *arrs)
+        assert np.max(np.abs(x - xo)) / np.max(np.abs(xo)) <= 2 * (n + 1) ** 2 / 2 * 2.2e-16
+    else:
+        check_parity(n, m, arrs, x, "f64", 0)
+
+
+@pytest.mark.parametrize("n,m", [(9000, 5), (200, 7)])
+def test_scan_edges_and_scaling(cuda_ok, n, m):
+    """X1 (NaN in a_0 / c_{n-1} ignored, bitwise), metamorphic row and rhs
+    scaling by powers of two (bitwise: the continuant state and the segment maps
+    rescale exactly), determinism across runs, and the variant's fixed k = 0."""
+    import torch
+    a, b, c, d = gen(n, m, "f64", 0, "weak", eps=1e-2)
+    plan = tri.Plan(n, m, tri.F64, 0)
+    plan.variant = SCAN
+    da, db, dc, dd = to_dev(a, b, c, d)
+    x1 = plan.solve(da, db, dc, dd).clone()
+    assert torch.equal(plan.solve(da, db, dc, dd), x1)
+    a2, c2 = da.clone(), dc.clone()
+    a2.view(m, n)[:, 0] = float("nan")
+    c2.view(m, n)[:, -1] = float("nan")
+    assert torch.equal(plan.solve(a2, db, c2, dd), x1)
+    p = 2.0 ** np.random.default_rng(1).integers(-20, 20, n * m)
+    x2 = plan.solve(*to_dev(a * p, b * p, c * p, d * p))
+    assert torch.equal(x2, x1)
+    x3 = plan.solve(da, db, dc, dd * 4.0)
+    assert torch.equal(x3, x1 * 4.0)
+    with pytest.raises(tri.TriError):
+        plan.k = 1  # the scan kernel is p-Thomas at k = 0
+    with pytest.raises(tri.TriError):
+        plan.debug_pcr(da, db, dc, dd)  # no PCR stage
+
+
+def test_scan_rejects_unsupported(cuda_ok):
+    for (n, m, dt, layout) in [(1004, 3, tri.F64, 0), (16384, 3, tri.F64, 1), (7, 3, tri.F32, 0),
+                               ((1 << 20) + 8, 1, tri.F64, 0)]:
+        plan = tri.Plan(n, m, dt, layout)
+        with pytest.raises(tri.TriError):
+            plan.variant = SCAN
+
+
+@pytest.mark.parametrize("dtype,n,m", [("f64", 16384, 16384), ("f32", 256, 1 << 20)])
+def test_scan_full_size_sampled(cuda_ok, dtype, n, m):
+    """BASELINE c5 / c4 shapes in the launch configuration bench.py times: whole
+    sampled systems (first/last of a CTA's sweep, both slot parities, the last
+    system) vs the oracle element by element."""
+    arrs = gen(n, m, dtype, 0)
+    plan = tri.Plan(n, m, tri.F64 if dtype == "f64" else tri.F32, 0)
+    plan.variant = SCAN
+    x = plan.solve(*to_dev(*arrs)).cpu().numpy()
+    for q in (0, 1, 147, 148, 149, 8191, m - 149, m - 1):
+        sl = slice(q * n, (q + 1) * n)
+        sub = [t[sl] for t in arrs]
+        check_parity(n, 1, sub, x[sl], dtype, 0)
+
+
 # ------------------------------------------------------------------ WARP variant
 @pytest.mark.parametrize("dtype", ["f64", "f32"])
 @pytest.mark.parametrize("layout", [0, 1])
