@@ -25,12 +25,12 @@
 //
 // Persistent CTAs (one per SM), NW identical warps; step g = j NC + w (system
 // j of this CTA, window w) runs on warp g % NW and does the forward work of
-// window (j, w) and the back substitution of window (j - 1, NC - 1 - w); the
-// latter reads exactly the storage slot the former then rewrites (slot of
-// window w: w for even j, NC - 1 - w for odd j), so one system's worth of
-// (c', d') slots recycles with no extra synchronisation.  The first and last
-// S_on / 2 slots live in shared memory, the middle ones in a per-CTA L2-resident
-// spill region.  Systems of one window (n <= 256) need no chain: each warp solves
+// window (j, w) and the back substitution of the window NC + delta steps
+// behind it in backward order (windows of a system in reverse); the latter
+// reads a storage slot the former then rewrites, so NC + delta slots of
+// (c', d') recycle with no extra synchronisation, and a window is read back at
+// least delta + 1 steps after it was stored.  The first S_on slots live in
+// shared memory, the others in a per-CTA L2-resident spill region.  Systems of one window (n <= 256) need no chain: each warp solves
 // whole systems on its own (forward and backward in registers).
 #pragma once
 #include "k_stream.cuh"  // sk_* TMA / mbarrier / policy helpers, SKMat
@@ -50,9 +50,10 @@ constexpr int SC_NCMAX = 4096;     // windows per system (per-slot counters live
 template <typename T>
 struct ScanArgs {
     T* x;
-    T* spill;      // per CTA: (NC - S_on) slots of sc_slot_elems<T>() elements
+    T* spill;      // per CTA: (NC + delta - S_on) slots of sc_slot_elems<T>() elements
     int64_t n, m;
     int NC;        // windows per system
+    int delta;     // extra lag (steps) of the back substitution behind the forward sweep
     int S_on;      // storage slots resident in shared memory
     unsigned long long* prof;  // diagnostics (scripts/prof_scan.py): per-phase cycle counters, or null
     int dbg;       // diagnostics: 1 = no chain handover (wrong results; timing only)
@@ -69,11 +70,16 @@ struct SCLayout {
     static constexpr int off_st = off_in + SC_NW * in_stride;             // [NW][theta|psi|delta]
     static constexpr int off_xh = off_st + SC_NW * 4 * (int)sizeof(T);    // [NW] x handover
     static constexpr int off_bar = (off_xh + SC_NW * (int)sizeof(T) + 7) / 8 * 8;  // [NW] in_full
-    static constexpr int off_cnt = off_bar + SC_NW * 8;                   // [NC] slot counters
+    static constexpr int off_cnt = off_bar + SC_NW * 8;                   // [NC] windows-stored counters
+    // [K][NC] u16: slot of window (j, w) at row j % K, K = 3 + (delta - 1) / NC
+    // systems in flight between a window's store and its read-back (<= 3 NC + delta entries)
+    static __host__ __device__ constexpr int off_tab(int NC) { return off_cnt + 4 * NC; }
     static constexpr int slot_bytes = sc_slot_elems<T>() * (int)sizeof(T);
-    static __host__ __device__ constexpr int off_store(int NC) { return (off_cnt + 4 * NC + 1023) / 1024 * 1024; }
-    static __host__ __device__ constexpr int smem_bytes(int NC, int S_on) {
-        return off_store(NC) + S_on * slot_bytes + 1024;  // + alignment slack
+    static __host__ __device__ constexpr int off_store(int NC, int D) {
+        return (off_tab(NC) + 2 * (3 * NC + D) + 1023) / 1024 * 1024;
+    }
+    static __host__ __device__ constexpr int smem_bytes(int NC, int D, int S_on) {
+        return off_store(NC, D) + S_on * slot_bytes + 1024;  // + alignment slack
     }
 };
 
@@ -313,11 +319,12 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
     extern __shared__ __align__(16) unsigned char sc_smem_raw[];
     unsigned char* sbase = sc_smem_raw + ((1024 - ((unsigned)__cvta_generic_to_shared(sc_smem_raw) & 1023)) & 1023);
     uint64_t* in_full = reinterpret_cast<uint64_t*>(sbase + L::off_bar);  // [NW] TMA -> warp
-    int* cnt = reinterpret_cast<int*>(sbase + L::off_cnt);                // [NC] systems stored per slot
+    int* cnt = reinterpret_cast<int*>(sbase + L::off_cnt);    // [NC] systems whose window w is stored
+    unsigned short* tab = reinterpret_cast<unsigned short*>(sbase + L::off_tab(p.NC));  // [K][NC] slot of (j, w)
     T* stt = reinterpret_cast<T*>(sbase + L::off_st);
     T* xh = reinterpret_cast<T*>(sbase + L::off_xh);
     const int NC = p.NC;
-    const unsigned store_s = (unsigned)__cvta_generic_to_shared(sbase + L::off_store(NC));
+    const unsigned store_s = (unsigned)__cvta_generic_to_shared(sbase + L::off_store(NC, p.delta));
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     if (threadIdx.x == 0) {
@@ -382,14 +389,22 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
         return;
     }
 
+    // Step g runs the forward sweep of window g (system g / NC, window g % NC) and
+    // the back substitution of backward index b = g - NC - delta (system b / NC,
+    // window NC - 1 - b % NC): a window is read back >= delta + 1 steps after it
+    // was stored.  The backward part reads a slot, the forward part of the same
+    // step then reuses it (tab[j % 3][w] records where window (j, w) went); the
+    // first NC + delta forward steps take fresh slots.
+    const int D = p.delta;
+    const int NS = NC + D;                  // storage slots
+    const int K = 3 + (D - 1) / NC;         // rows of tab
     const int nfwd = nsys * NC;             // forward steps
-    const int total = (nsys + 1) * NC;      // + the back substitution of the last system
-    const int nspill = NC - p.S_on;
+    const int total = nfwd + NC + D;        // + the back substitution of the last system
+    const int nspill = NS - p.S_on;
     T* spill_cta = p.spill + (int64_t)blockIdx.x * (int64_t)(nspill > 0 ? nspill : 0) * sc_slot_elems<T>();
     int j = 0, w = pw;
     while (w >= NC) { w -= NC; ++j; }
     if (lane == 0 && pw < nfwd) issue(j, w);
-    auto slot_of = [&](int jj, int ww) { return (jj & 1) ? NC - 1 - ww : ww; };
     const int pi = (pw + SC_NW - 1) % SC_NW;  // warp of step g - 1
     unsigned long long pc[8] = {0, 0, 0, 0, 0, 0, 0, 0}, t0 = PROF ? clock64() : 0, tp = t0;
 #define SC_T(k) do { if (PROF) { const unsigned long long tn_ = clock64(); pc[k] += tn_ - tp; tp = tn_; } } while (0)
@@ -397,14 +412,21 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
         const int cj = j, cw = w;
         w += SC_NW;
         while (w >= NC) { w -= NC; ++j; }
-        const bool fwd = cj < nsys, bwd = cj >= 1;
-        const int wb = NC - 1 - cw;  // backward window (system cj - 1)
-        const int slot = slot_of(cj, cw);
+        const int bb = g - NC - D;
+        const bool fwd = cj < nsys, bwd = bb >= 0;
+        const int bj = bwd ? bb / NC : 0;
+        const int wb = NC - 1 - (bb - bj * NC);  // backward window (system bj)
         const int64_t i0d = (int64_t)cw * SC_W + lane * SC_R;
-        int sidx;
-        const bool res = sk_resident(slot, NC, p.S_on, sidx);
-        const unsigned sp_s = store_s + (unsigned)(sidx * L::slot_bytes);
-        T* sp_g = spill_cta + (size_t)sidx * sc_slot_elems<T>();
+        int slot = g;                            // fresh slot (g < NS when !bwd)
+        if (bwd && p.dbg != 2) {
+            SC_T(5);
+            sk_wait_ge(&cnt[wb], bj + 1);  // window (bj, wb) stored
+            SC_T(4);
+            slot = tab[(bj % K) * NC + wb];
+        }
+        const bool res = slot < p.S_on;
+        const unsigned sp_s = store_s + (unsigned)(slot * L::slot_bytes);
+        T* sp_g = spill_cta + (size_t)(res ? 0 : slot - p.S_on) * sc_slot_elems<T>();
 
         if (p.dbg == 2) {  // diagnostics: the memory pipeline alone (inputs in, x out; no math)
             if (fwd) {
@@ -420,12 +442,9 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
             }
             continue;
         }
-        // ---- backward: (c', d') of window (cj - 1, wb) from the slot (held in registers)
+        // ---- backward: (c', d') of window (bj, wb) from the slot (held in registers)
         T cpb[SC_R], dpb[SC_R];
         if (bwd) {
-            SC_T(5);
-            sk_wait_ge(&cnt[slot], cj);  // system cj - 1 stored in the slot
-            SC_T(4);
             if (res) sc_load_slot_s(sp_s, lane, cpb, dpb);
             else sc_load_slot_g(sp_g, lane, cpb, dpb);
         } else {
@@ -477,10 +496,8 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
             stt[pw * 4 + 1] = op * sc;
             stt[pw * 4 + 2] = od * sc;
         }
-        if (g + 1 < total && p.dbg != 1) {
-            __threadfence_block();
+        if (g + 1 < total && p.dbg != 1)  // arrive -> sync: release / acquire (PTX memory model)
             asm volatile("bar.arrive %0, 64;" ::"r"(1 + pw) : "memory");
-        }
         SC_T(3);
         T x = __shfl_down_sync(0xffffffffu, xs, 1);  // x after the lane's rows
         if (lane == 31) x = xw;
@@ -504,9 +521,12 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
             if (res) sc_store_slot_s(sp_s, lane, cpf, dpf);
             else sc_store_slot_g(sp_g, lane, cpf, dpf, pol_sp);
             __syncwarp();
-            if (lane == 0) sk_st_release(&cnt[slot], cj + 1);
+            if (lane == 0) {
+                tab[(cj % K) * NC + cw] = (unsigned short)slot;
+                sk_st_release(&cnt[cw], cj + 1);
+            }
         }
-        // ---- backward replay: x (Eq 4) of window (cj - 1, wb)
+        // ---- backward replay: x (Eq 4) of window (bj, wb)
         if (bwd) {
             T xv[SC_R];
 #pragma unroll
@@ -514,7 +534,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
                 x = fma(-cpb[t], x, dpb[t]);
                 xv[t] = x;
             }
-            const int64_t qb = blockIdx.x + (int64_t)(cj - 1) * gridDim.x;
+            const int64_t qb = blockIdx.x + (int64_t)bj * gridDim.x;
             const int64_t xr = (int64_t)wb * SC_W + lane * SC_R;
             sc_store_x(p.x + qb * n + xr, n - xr, xv);
         }

@@ -38,6 +38,7 @@ int env_int(const char* name, int dflt) {
 int g_tiled_waves1 = env_int("TRI_TILED_WAVES1", 1);
 int g_split_k1max = std::min(10, env_int("TRI_SPLIT_K1MAX", 10));  // steps kept in pass 1 (tuning)
 int g_tiled_waves2 = env_int("TRI_TILED_WAVES2", 3);  // measured best at c3 (1 / 3 waves)
+int g_scan_delta = env_int("TRI_SCAN_DELTA", 8);      // SCAN: back-substitution lag in steps (tuning)
 
 constexpr int ONCHIP_THREADS = 512;
 constexpr int SPLIT_K1MAX = 10;  // deepest k one sliding-window pass holds in smem (T = 256)
@@ -177,7 +178,8 @@ struct tri_plan_s {
     int fu_grid, fu_son;      // FUSED: persistent CTAs, on-chip positions per chain
     bool fu_vec;              // FUSED: staged 8-row-aligned path
     int64_t fu_nc;            // FUSED: windows per system
-    int sk_grid, sk_nc, sk_son;  // STREAM: persistent CTAs, windows per system, resident storage slots
+    int sk_grid, sk_nc, sk_son;  // STREAM / SCAN: persistent CTAs, windows per system, resident storage slots
+    int sk_delta;                // SCAN: back-substitution lag (steps)
     size_t smem_optin;
     void* scratch;
     size_t scratch_bytes;
@@ -316,11 +318,12 @@ void plan_geometry(tri_plan_s* p) {
         p->L = n; p->n_pad = n; p->C = m;
         p->sk_nc = (int)cdiv(n, SC_W);
         p->sk_grid = (int)std::min<int64_t>(m, p->sms);
-        const int fixed = p->dtype == TRI_F64 ? SCLayout<double>::smem_bytes(p->sk_nc, 0)
-                                              : SCLayout<float>::smem_bytes(p->sk_nc, 0);
+        p->sk_delta = g_scan_delta;
+        const int fixed = p->dtype == TRI_F64 ? SCLayout<double>::smem_bytes(p->sk_nc, p->sk_delta, 0)
+                                              : SCLayout<float>::smem_bytes(p->sk_nc, p->sk_delta, 0);
         const int slot = p->dtype == TRI_F64 ? SCLayout<double>::slot_bytes : SCLayout<float>::slot_bytes;
         const int64_t avail = ((int64_t)p->smem_optin - fixed) / slot;
-        p->sk_son = p->sk_nc == 1 ? 0 : (int)std::max<int64_t>(0, std::min<int64_t>(p->sk_nc, avail));
+        p->sk_son = p->sk_nc == 1 ? 0 : (int)std::max<int64_t>(0, std::min<int64_t>(p->sk_nc + p->sk_delta, avail));
     }
     if (p->variant == TRI_VARIANT_FUSED) {
         const size_t s = esize(p->dtype);
@@ -341,7 +344,7 @@ void plan_geometry(tri_plan_s* p) {
 size_t scratch_need(const tri_plan_s* p) {
     if (p->variant == TRI_VARIANT_SCAN)
         return p->sk_nc == 1 ? 0
-                             : (size_t)p->sk_grid * (size_t)std::max(0, p->sk_nc - p->sk_son) *
+                             : (size_t)p->sk_grid * (size_t)std::max(0, p->sk_nc + p->sk_delta - p->sk_son) *
                                    (size_t)sc_slot_elems<double>() * esize(p->dtype);
     if (p->variant == TRI_VARIANT_STREAM)
         return (size_t)p->sk_grid * (size_t)std::max(0, p->sk_nc - p->sk_son) * SK_SLOT * esize(p->dtype);
@@ -607,10 +610,10 @@ cudaError_t launch_scan(const tri_plan_s* p, const void* a, const void* b, const
     ScanArgs<T> A;
     A.x = (T*)x;
     A.spill = (T*)p->scratch;
-    A.n = p->n; A.m = p->m; A.NC = p->sk_nc; A.S_on = p->sk_son;
+    A.n = p->n; A.m = p->m; A.NC = p->sk_nc; A.S_on = p->sk_son; A.delta = p->sk_delta;
     A.prof = (unsigned long long*)g_fused_prof;
     A.dbg = g_fused_dbg_mode;
-    const size_t smem = (size_t)SCLayout<T>::smem_bytes(p->sk_nc, p->sk_son);
+    const size_t smem = (size_t)SCLayout<T>::smem_bytes(p->sk_nc, p->sk_delta, p->sk_son);
     auto kern = A.prof ? k_scan<T, true> : k_scan<T, false>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
