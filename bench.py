@@ -133,7 +133,7 @@ def method_arrays(plan, tri):
     v = plan.variant
     if v in (tri.VARIANT_WARP, tri.VARIANT_ONCHIP):
         return 5
-    if v in (tri.VARIANT_FUSED, tri.VARIANT_STREAM):
+    if v in (tri.VARIANT_FUSED, tri.VARIANT_STREAM, tri.VARIANT_SCAN):
         return 5  # c', d' stay in smem or in per-CTA scratch that stays in L2 (ncu: 5.0 arrays of DRAM traffic)
     if plan.k == 0:
         return 9  # read a, b, c, d; write + read c', d'; write x

@@ -112,6 +112,14 @@ bool scan_ok(int64_t n, int64_t m, tri_dtype t, tri_layout layout) {
 //   * whole systems that fit a CTA's smem: ONCHIP;
 //   * otherwise (few large systems): SPLIT with k from choose_k_for.
 tri_variant choose_variant(int64_t n, int64_t m, tri_dtype t, tri_layout layout, int sms) {
+    // SCAN (profiles/r01_sweep_scan_*.jsonl): fastest of all variants on every
+    // contiguous shape with n % 8 == 0 of the grid n = 256 .. 2^20 x m = 1 .. 2^20
+    // (fp64 and fp32), except a few (< 128) systems of more than 64 windows, where
+    // SPLIT's deep k keeps more SMs busy (n = 65536, m = 16: 86 us vs 100 us);
+    // e.g. n = m = 16384 fp64: 1.84 ms vs 2.92 ms (STREAM), n = 256, m = 2^20 fp32:
+    // 1.01 ms vs 1.12 ms (SPLIT k = 0).  k = 0 throughout: the paper's M > P rule.
+    if (layout == TRI_LAYOUT_CONTIGUOUS && scan_ok(n, m, t, layout) && (cdiv(n, SC_W) <= 64 || m >= 128))
+        return TRI_VARIANT_SCAN;
     // STREAM (profiles/r01_sweep_stream_f64.jsonl): fastest of all variants for
     // fp64 contiguous batches with n % 8 == 0 from 8 windows up, except a few
     // (< 64) very long systems, where SPLIT's deep k keeps more SMs busy

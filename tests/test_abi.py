@@ -85,7 +85,8 @@ def test_heuristic_k_valid_and_nonincreasing_in_m(L, dtype, layout, n):
     for m in [1, 2, 16, 32, 100, 512, 1024, 4096, 16384, 1 << 20]:
         k = tri.choose_k(n, m, dtype, layout, 148)
         v = tri.choose_variant(n, m, dtype, layout, 148)
-        assert v in (tri.VARIANT_ONCHIP, tri.VARIANT_SPLIT, tri.VARIANT_FUSED, tri.VARIANT_WARP, tri.VARIANT_STREAM)
+        assert v in (tri.VARIANT_ONCHIP, tri.VARIANT_SPLIT, tri.VARIANT_FUSED, tri.VARIANT_WARP, tri.VARIANT_STREAM,
+                     tri.VARIANT_SCAN)
         assert 0 <= k <= max(0, n.bit_length() - 1)
         if prev is not None:
             assert k <= prev[0], (n, m, k, prev)
@@ -94,13 +95,12 @@ def test_heuristic_k_valid_and_nonincreasing_in_m(L, dtype, layout, n):
 
 def test_heuristic_paper_rule_extremes(L):
     """P:699: with M > P (plenty of systems) go straight to p-Thomas (k = 0);
-    a single huge system gets deep PCR.  Exception measured on B200: fp64
-    contiguous batches run the STREAM kernel at its built-in k = 3, whose
-    intermediates never reach HBM (planner table)."""
+    a single huge system gets deep PCR.  On B200 contiguous batches run p-Thomas
+    as the SCAN kernel (k = 0, intermediates on chip: DESIGN.md planner table)."""
     assert tri.choose_k(16384, 16384, tri.F64, tri.INTERLEAVED, 148) == 0
     assert tri.choose_k(16384, 16384, tri.F32, tri.CONTIGUOUS, 148) == 0
-    assert tri.choose_variant(16384, 16384, tri.F64, tri.CONTIGUOUS, 148) == tri.VARIANT_STREAM
-    assert tri.choose_k(16384, 16384, tri.F64, tri.CONTIGUOUS, 148) == 3
+    assert tri.choose_variant(16384, 16384, tri.F64, tri.CONTIGUOUS, 148) == tri.VARIANT_SCAN
+    assert tri.choose_k(16384, 16384, tri.F64, tri.CONTIGUOUS, 148) == 0
     assert tri.choose_k(1 << 24, 1, tri.F64, tri.CONTIGUOUS, 148) >= 8
 
 
@@ -115,20 +115,20 @@ def test_shard_range_partitions(L, m, G):
 
 
 @pytest.mark.parametrize("cfg,n,m,dtype,layout,variant,k", [
-    ("c1", 1024, 1, "F64", 0, "VARIANT_FUSED", 4),
+    ("c1", 1024, 1, "F64", 0, "VARIANT_SCAN", 0),
     ("c2", 1024, 1024, "F64", 1, "VARIANT_WARP", 5),
     ("c3", 1 << 24, 1, "F64", 0, "VARIANT_SPLIT", 14),
-    ("c4", 256, 1 << 20, "F32", 0, "VARIANT_SPLIT", 0),
-    ("c5", 16384, 16384, "F64", 0, "VARIANT_STREAM", 3),
-    ("c5/2", 16384, 8192, "F64", 0, "VARIANT_STREAM", 3),  # one of 2 ranks (strong scaling)
-    ("c5/8", 16384, 2048, "F64", 0, "VARIANT_STREAM", 3),  # one of 8 ranks
+    ("c4", 256, 1 << 20, "F32", 0, "VARIANT_SCAN", 0),
+    ("c5", 16384, 16384, "F64", 0, "VARIANT_SCAN", 0),
+    ("c5/2", 16384, 8192, "F64", 0, "VARIANT_SCAN", 0),  # one of 2 ranks (strong scaling)
+    ("c5/8", 16384, 2048, "F64", 0, "VARIANT_SCAN", 0),  # one of 8 ranks
     ("c5-il", 16384, 16384, "F64", 1, "VARIANT_SPLIT", 0),  # interleaved layout: k = 0 TMA p-Thomas
     ("few-long", 65536, 37, "F64", 0, "VARIANT_SPLIT", 8),  # < 64 long systems: deep-k SPLIT
 ])
 def test_planner_picks_for_baseline_configs(L, cfg, n, m, dtype, layout, variant, k):
     """The planner's (variant, k) on a 148-SM B200 for BASELINE.json's configs,
-    as calibrated by scripts/sweep_k.py and scripts/sweep_stream.py
-    (profiles/r01_sweep_k_*.jsonl, profiles/r01_sweep_stream_f64.jsonl)."""
+    as calibrated by scripts/sweep_k.py, scripts/sweep_stream.py and
+    scripts/sweep_scan.py (profiles/r01_sweep_*.jsonl)."""
     dt = getattr(tri, dtype)
     assert tri.choose_variant(n, m, dt, layout, 148) == getattr(tri, variant), cfg
     assert tri.choose_k(n, m, dt, layout, 148) == k, cfg
