@@ -392,7 +392,8 @@ def main():
     if os.path.exists(tf):
         with open(tf) as fh:
             tj = json.load(fh)
-        if tj.get("n") == n and tj.get("m") == mr and tj.get("k") == plan.k:
+        if tj.get("n") == n and tj.get("m") == mr and tj.get("k") == plan.k and \
+                tj.get("variant", plan.variant) == plan.variant:
             traffic = tj.get("dram_bytes_per_launch")
     out = {
         "metric": METRIC, "value": value, "unit": "Munknowns/s", "n_gpus": world, "steps": args.steps,
