@@ -135,6 +135,8 @@ def method_arrays(plan, tri):
         return 5
     if v in (tri.VARIANT_FUSED, tri.VARIANT_STREAM, tri.VARIANT_SCAN):
         return 5  # c', d' stay in smem or in per-CTA scratch that stays in L2 (ncu: 5.0 arrays of DRAM traffic)
+    if v == tri.VARIANT_SCAN_MC:
+        return 13  # read a, b, c, d twice; write + read c', d'; write x
     if plan.k == 0:
         return 9  # read a, b, c, d; write + read c', d'; write x
     # pass 1: read 4 + write 3; [pass 2: read 3 + write 3]; p-Thomas: read 3, c', d' 2 + 2, write x

@@ -75,7 +75,11 @@ typedef enum {
                                forward sweep (Eqs 2-3) and back substitution (Eq 4) of each system spread
                                over the 32 lanes of a warp as segment maps combined by a shuffle scan
                                (X21); 256-row windows chained across warps, c', d' kept in
-                               shared memory / L2: HBM moves only the compulsory 5 arrays */
+                               shared memory / L2: HBM moves only the compulsory 5 arrays */,
+    TRI_VARIANT_SCAN_MC = 7 /* CONTIGUOUS (or m = 1), n % 8 == 0, few long systems: the SCAN solve with every
+                               system cut into chunks over several CTAs; three streaming passes (chunk
+                               forward maps; forward replay -> c', d'; back substitution) linked by two
+                               scans over the chunk maps (X21): 13 arrays of HBM traffic */
 } tri_variant;
 
 typedef struct tri_plan_s* tri_plan_t;

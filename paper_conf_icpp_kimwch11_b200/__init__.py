@@ -15,8 +15,9 @@ LIB_PATH = os.environ.get("TRI_LIB_PATH", os.path.join(HERE, "libtri.so"))  # ov
 
 F32, F64 = 0, 1
 CONTIGUOUS, INTERLEAVED = 0, 1
-VARIANT_AUTO, VARIANT_ONCHIP, VARIANT_SPLIT, VARIANT_FUSED, VARIANT_WARP, VARIANT_STREAM, VARIANT_SCAN = 0, 1, 2, 3, 4, 5, 6
-VARIANT_NAMES = {1: "onchip", 2: "split", 3: "fused", 4: "warp", 5: "stream", 6: "scan"}
+(VARIANT_AUTO, VARIANT_ONCHIP, VARIANT_SPLIT, VARIANT_FUSED, VARIANT_WARP, VARIANT_STREAM, VARIANT_SCAN,
+ VARIANT_SCAN_MC) = 0, 1, 2, 3, 4, 5, 6, 7
+VARIANT_NAMES = {1: "onchip", 2: "split", 3: "fused", 4: "warp", 5: "stream", 6: "scan", 7: "scan_mc"}
 STATUS = {0: "TRI_OK", 1: "TRI_ERR_INVALID_ARG", 2: "TRI_ERR_ALIGNMENT", 3: "TRI_ERR_ALIAS",
           4: "TRI_ERR_DEVICE", 5: "TRI_ERR_OOM", 6: "TRI_ERR_CUDA"}
 

@@ -92,6 +92,17 @@ __device__ __forceinline__ int sc_chunk(int lane, int ch) {
     return ch * 32 + lane;
 }
 
+// TMA 3D tile load: tensor view [m][n/8][8] (system, 8-row group, row), box
+// [1][32][8] = one 256-row window of one array; rows past the system's end are
+// zero-filled (and replaced by identity rows, sc_fix_rows)
+__device__ __forceinline__ void sc_tma3d(void* dst, const CUtensorMap* tm, int y, int q, uint64_t* bar, uint64_t pol) {
+    asm volatile(
+        "cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint"
+        " [%0], [%1, {%2, %3, %4}], [%5], %6;" ::"r"((unsigned)__cvta_generic_to_shared(dst)),
+        "l"(tm), "r"(0), "r"(y), "r"(q), "r"((unsigned)__cvta_generic_to_shared(bar)), "l"(pol)
+        : "memory");
+}
+
 // exact power-of-two scale 2^-e bringing max(|u|, |v|) into [1, 2) (projective
 // rescale of a map or state: ratios c', d' are unchanged)
 template <typename T>
@@ -342,13 +353,13 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
     const uint64_t pol_in = sk_policy_evict_first();
     const uint64_t pol_sp = sk_policy_evict_last();
     auto issue = [&](int jj, int ww) {
-        const int64_t q = blockIdx.x + (int64_t)jj * gridDim.x;
-        const int y = (int)((q * n + (int64_t)ww * SC_W) >> 3);  // n % 8 == 0
+        const int q = (int)(blockIdx.x + (int64_t)jj * gridDim.x);
+        const int y = ww * (SC_W / 8);
         sk_expect(&in_full[pw], (unsigned)(4 * SC_W * sizeof(T)));
-        sk_tma2d(ib + 0 * SC_W, &tm.a, 0, y, &in_full[pw], pol_in);
-        sk_tma2d(ib + 1 * SC_W, &tm.b, 0, y, &in_full[pw], pol_in);
-        sk_tma2d(ib + 2 * SC_W, &tm.c, 0, y, &in_full[pw], pol_in);
-        sk_tma2d(ib + 3 * SC_W, &tm.d, 0, y, &in_full[pw], pol_in);
+        sc_tma3d(ib + 0 * SC_W, &tm.a, y, q, &in_full[pw], pol_in);
+        sc_tma3d(ib + 1 * SC_W, &tm.b, y, q, &in_full[pw], pol_in);
+        sc_tma3d(ib + 2 * SC_W, &tm.c, y, q, &in_full[pw], pol_in);
+        sc_tma3d(ib + 3 * SC_W, &tm.d, y, q, &in_full[pw], pol_in);
     };
     unsigned ph = 0;
 

@@ -1,0 +1,289 @@
+// k_scan_mc.cuh -- TRI_VARIANT_SCAN_MC: p-Thomas at k = 0 for FEW LONG systems
+// (one huge system, config c3), each system cut into P chunks of consecutive
+// 256-row windows, one CTA per chunk, so that every SM works on every system.
+//
+// Paper: Thomas Eqs 2-4 (reading X2), p-Thomas; the
+// continuant form of the forward sweep and its segment maps are DESIGN.md X21
+// (k_scan.cuh); this file adds one level above the windows: chunks.  The
+// forward sweep of a chunk is a 3x3 linear map of the incoming state and the
+// back substitution an affine map of the x after the chunk, so the solve runs
+// as three streaming passes:
+//   pass 0 (k_scan_mc<0>): read a, b, c, d; every window's forward map (lane
+//     segment maps reduced over the warp); the chunk's map = their product;
+//   pass 1 (k_scan_mc<1>): the chunk's incoming state = product of the maps of
+//     the chunks before it (read by warp 0 while the first tiles load); read
+//     a, b, c, d again; windows chained across the CTA's warps (state handed
+//     over through named barriers, as in k_scan), replay -> c', d' to scratch;
+//     every window's back-substitution map; the chunk's backward map;
+//   pass 2 (k_scan_mc<2>): x after the chunk = the backward maps of the chunks
+//     after it applied to 0; read c', d' (TMA bulk copies); windows in reverse
+//     order chained across warps (x handed over), replay Eq 4 -> x.
+// HBM traffic: 4 + 4 + 2 + 2 + 1 = 13 arrays (the deep-k SPLIT path moves 21).
+#pragma once
+#include "k_scan.cuh"
+
+namespace tri {
+
+constexpr int SMC_WMAX = 1024;  // windows per chunk (per-window maps live in smem)
+
+template <typename T>
+struct ScanMCArgs {
+    T* x;
+    T* cd;        // c', d' of every window (q, w): sc_slot_elems<T>() elements at (q NC + w)
+    T* cmap;      // [m P][8] chunk forward maps (SKMat a..g)
+    T* cbm;       // [m P][8] chunk back-substitution maps (al, be, -): x_first = al + be x_after
+    int64_t n, m;
+    int NC;       // windows per system
+    int NCW;      // windows per chunk
+    int P;        // chunks per system
+};
+
+template <typename T>
+struct SMCLayout {
+    static constexpr int in_bytes = 4 * SC_W * (int)sizeof(T);        // one window: a, b, c, d (or c', d')
+    static constexpr int in_stride = (in_bytes + 1023) / 1024 * 1024;
+    static constexpr int off_in = 0;
+    static constexpr int off_hv = off_in + SC_NW * in_stride;          // [NW][4] handover
+    static constexpr int off_bar = off_hv + SC_NW * 4 * (int)sizeof(T);
+    static constexpr int off_wm = (off_bar + SC_NW * 8 + 15) / 16 * 16;  // [NCW][8] per-window maps
+    static __host__ __device__ constexpr int smem_bytes(int NCW) { return off_wm + NCW * 8 * (int)sizeof(T) + 1024; }
+};
+
+__device__ __forceinline__ void smc_bulk_g2s(void* dst, const void* src, unsigned bytes, uint64_t* bar) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+            (unsigned)__cvta_generic_to_shared(dst)),
+        "l"(src), "r"(bytes), "r"((unsigned)__cvta_generic_to_shared(bar))
+        : "memory");
+}
+
+template <typename T>
+__device__ __forceinline__ SKMat<T> sk_shfl_down(const SKMat<T>& m, int d) {
+    SKMat<T> r;
+    r.a = __shfl_down_sync(0xffffffffu, m.a, d);
+    r.b = __shfl_down_sync(0xffffffffu, m.b, d);
+    r.c = __shfl_down_sync(0xffffffffu, m.c, d);
+    r.d = __shfl_down_sync(0xffffffffu, m.d, d);
+    r.e = __shfl_down_sync(0xffffffffu, m.e, d);
+    r.f = __shfl_down_sync(0xffffffffu, m.f, d);
+    r.g = __shfl_down_sync(0xffffffffu, m.g, d);
+    return r;
+}
+
+template <typename T>
+__device__ __forceinline__ void smc_rescale(SKMat<T>& M) {
+    const T s = sc_scale2(M.a, M.b);
+    M.a *= s; M.b *= s; M.c *= s; M.d *= s; M.e *= s; M.f *= s; M.g *= s;
+}
+
+// product of the maps of `cnt` consecutive windows / chunks (8 values apart, in
+// shared or global memory; warp-wide, order-preserving): forward maps compose later-after-earlier; backward maps
+// (al, be) compose earlier-after-later (x_first(window i) depends on window i+1)
+template <typename T>
+__device__ __forceinline__ SKMat<T> smc_reduce_fwd(const T* wm, int cnt, int lane) {
+    const int per = (cnt + 31) / 32, lo = lane * per, hi = min(cnt, lo + per);
+    SKMat<T> R{T(1), T(0), T(0), T(1), T(0), T(0), T(1)};
+    for (int i = lo; i < hi; ++i) {
+        const T* s = wm + 8 * i;
+        R = sk_compose(SKMat<T>{s[0], s[1], s[2], s[3], s[4], s[5], s[6]}, R);
+        smc_rescale(R);
+    }
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {  // lane l combines with lane l + d (later windows)
+        const SKMat<T> o = sk_shfl_down(R, d);
+        if ((lane & (2 * d - 1)) == 0) { R = sk_compose(o, R); smc_rescale(R); }
+    }
+    return R;  // lane 0
+}
+template <typename T>
+__device__ __forceinline__ void smc_reduce_bwd(const T* wm, int cnt, int lane, T& al, T& be) {
+    const int per = (cnt + 31) / 32, lo = lane * per, hi = min(cnt, lo + per);
+    al = T(0); be = T(1);
+    for (int i = hi - 1; i >= lo; --i) {  // R = B_i o R
+        const T a2 = wm[8 * i], b2 = wm[8 * i + 1];
+        al = fma(b2, al, a2);
+        be = b2 * be;
+    }
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {  // (lane l) o (lane l + d)
+        const T oa = __shfl_down_sync(0xffffffffu, al, d), ob = __shfl_down_sync(0xffffffffu, be, d);
+        if ((lane & (2 * d - 1)) == 0) { al = fma(be, oa, al); be = be * ob; }
+    }
+}
+
+template <typename T, int MODE>
+__global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant__ StreamMaps tm, ScanMCArgs<T> p) {
+    using L = SMCLayout<T>;
+    extern __shared__ __align__(16) unsigned char smc_smem_raw[];
+    unsigned char* sbase = smc_smem_raw + ((1024 - ((unsigned)__cvta_generic_to_shared(smc_smem_raw) & 1023)) & 1023);
+    uint64_t* in_full = reinterpret_cast<uint64_t*>(sbase + L::off_bar);
+    T* hv = reinterpret_cast<T*>(sbase + L::off_hv);
+    T* wm = reinterpret_cast<T*>(sbase + L::off_wm);
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, pw = warp;
+    if (threadIdx.x == 0) {
+        for (int i = 0; i < SC_NW; ++i) sk_bar_init(&in_full[i], 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    }
+    __syncthreads();
+
+    const int64_t n = p.n;
+    const int NC = p.NC;
+    const int64_t q = blockIdx.x / p.P;
+    const int ch = (int)(blockIdx.x - q * p.P);
+    const int w0 = ch * p.NCW;
+    const int nwin = min(NC, w0 + p.NCW) - w0;
+    T* ib = reinterpret_cast<T*>(sbase + L::off_in + pw * L::in_stride);
+    const uint64_t pol_in = sk_policy_evict_first();
+    auto win_of = [&](int g) { return MODE == 2 ? w0 + nwin - 1 - g : w0 + g; };
+    auto issue = [&](int g) {
+        const int w = win_of(g);
+        if (MODE < 2) {
+            const int y = w * (SC_W / 8);
+            sk_expect(&in_full[pw], (unsigned)(4 * SC_W * sizeof(T)));
+            sc_tma3d(ib + 0 * SC_W, &tm.a, y, (int)q, &in_full[pw], pol_in);
+            sc_tma3d(ib + 1 * SC_W, &tm.b, y, (int)q, &in_full[pw], pol_in);
+            sc_tma3d(ib + 2 * SC_W, &tm.c, y, (int)q, &in_full[pw], pol_in);
+            sc_tma3d(ib + 3 * SC_W, &tm.d, y, (int)q, &in_full[pw], pol_in);
+        } else {
+            const unsigned bytes = (unsigned)(sc_slot_elems<T>() * sizeof(T));
+            sk_expect(&in_full[pw], bytes);
+            smc_bulk_g2s(ib, p.cd + (q * NC + w) * (int64_t)sc_slot_elems<T>(), bytes, &in_full[pw]);
+        }
+    };
+    if (lane == 0 && pw < nwin) issue(pw);
+    unsigned ph = 0;
+    const int pi = (pw + SC_NW - 1) % SC_NW;
+    // the chunk's boundary value from the maps of pass 0 / pass 1 (warp 0 runs step 0)
+    T st0 = T(1), ps0 = T(0), de0 = T(0), xa0 = T(0);
+    if (MODE == 1 && warp == 0) {  // incoming state = (M_{ch-1} ... M_0) (1, 0, 0)
+        const SKMat<T> R = smc_reduce_fwd(p.cmap + 8 * (q * p.P), ch, lane);
+        st0 = __shfl_sync(0xffffffffu, R.a, 0);
+        ps0 = __shfl_sync(0xffffffffu, R.c, 0);
+        de0 = __shfl_sync(0xffffffffu, R.e, 0);
+    }
+    if (MODE == 2 && warp == 0) {  // x after the chunk = (B_{ch+1} ... B_{P-1})(0)
+        T al, be;
+        smc_reduce_bwd(p.cbm + 8 * (q * p.P + ch + 1), p.P - 1 - ch, lane, al, be);
+        xa0 = __shfl_sync(0xffffffffu, al, 0);
+    }
+    const unsigned ib_s = (unsigned)__cvta_generic_to_shared(ib);
+
+    for (int g = pw; g < nwin; g += SC_NW) {
+        const int w = win_of(g);
+        const int64_t i0 = (int64_t)w * SC_W + lane * SC_R;
+        const bool edge = w == 0 || (int64_t)(w + 1) * SC_W > n;
+        sk_wait(&in_full[pw], ph);
+        ph ^= 1u;
+        if (MODE == 0) {
+            // ---- the window's forward map (product of the lane segment maps)
+            T ra[SC_R], rb[SC_R], rc[SC_R], rd[SC_R];
+            sc_ld_rows(ib, lane, ra, rb, rc, rd);
+            __syncwarp();
+            if (lane == 0 && g + SC_NW < nwin) issue(g + SC_NW);
+            if (edge) sc_fix_rows<T>(i0, n, ra, rb, rc, rd);
+            SKMat<T> M = sc_fwd_map(ra, rb, rc, rd);
+#pragma unroll
+            for (int d = 1; d < 32; d <<= 1) {  // lane l: lanes l .. l + 2d - 1 (later after earlier)
+                const SKMat<T> o = sk_shfl_down(M, d);
+                if ((lane & (2 * d - 1)) == 0) { M = sk_compose(o, M); smc_rescale(M); }
+            }
+            if (lane == 0) {
+                T* s = wm + 8 * g;
+                s[0] = M.a; s[1] = M.b; s[2] = M.c; s[3] = M.d; s[4] = M.e; s[5] = M.f; s[6] = M.g;
+            }
+        } else if (MODE == 1) {
+            // ---- forward replay from the chunk's / previous window's state
+            T ra[SC_R], rb[SC_R], rc[SC_R], rd[SC_R];
+            sc_ld_rows(ib, lane, ra, rb, rc, rd);
+            if (edge) sc_fix_rows<T>(i0, n, ra, rb, rc, rd);
+            SKMat<T> M = sc_fwd_map(ra, rb, rc, rd);
+            sc_fwd_scan(M, lane);
+            if (g > 0) asm volatile("bar.sync %0, 64;" ::"r"(1 + pi) : "memory");
+            T th, ps, de;
+            if (g == 0) {
+                th = st0; ps = ps0; de = de0;
+            } else {
+                th = hv[4 * pi + 0]; ps = hv[4 * pi + 1]; de = hv[4 * pi + 2];
+            }
+            const T ot = fma(M.a, th, M.b * ps);
+            const T op = fma(M.c, th, M.d * ps);
+            const T od = fma(M.e, th, fma(M.f, ps, M.g * de));
+            if (lane == 31) {
+                const T sc = sk_exp2_scale(ot);
+                hv[4 * pw + 0] = ot * sc; hv[4 * pw + 1] = op * sc; hv[4 * pw + 2] = od * sc;
+            }
+            if (g + 1 < nwin) asm volatile("bar.arrive %0, 64;" ::"r"(1 + pw) : "memory");
+            {
+                const T it_ = __shfl_up_sync(0xffffffffu, ot, 1);
+                const T ip = __shfl_up_sync(0xffffffffu, op, 1);
+                const T id = __shfl_up_sync(0xffffffffu, od, 1);
+                if (lane > 0) { th = it_; ps = ip; de = id; }
+            }
+            __syncwarp();
+            if (lane == 0 && g + SC_NW < nwin) issue(g + SC_NW);  // rows are in registers
+            T cp[SC_R], dp[SC_R];
+            sc_fwd_replay(ra, rb, rc, rd, th, ps, de, cp, dp);
+            T* dst = p.cd + (q * NC + w) * (int64_t)sc_slot_elems<T>();
+            if constexpr (sizeof(T) == 8) {
+#pragma unroll
+                for (int t = 0; t < SC_R; ++t)
+                    __stcg(reinterpret_cast<double2*>(dst + 2 * sc_chunk<T>(lane, t)), make_double2(cp[t], dp[t]));
+            } else {
+#pragma unroll
+                for (int t = 0; t < SC_R / 2; ++t)
+                    __stcg(reinterpret_cast<float4*>(dst + 4 * sc_chunk<T>(lane, t)),
+                           make_float4(cp[2 * t], dp[2 * t], cp[2 * t + 1], dp[2 * t + 1]));
+            }
+            // the window's back-substitution map
+            T al, be;
+            sc_bwd_map(cp, dp, al, be);
+#pragma unroll
+            for (int d = 1; d < 32; d <<= 1) {  // lane l: lanes l .. l + 2d - 1
+                const T oa = __shfl_down_sync(0xffffffffu, al, d), ob = __shfl_down_sync(0xffffffffu, be, d);
+                if ((lane & (2 * d - 1)) == 0) { al = fma(be, oa, al); be = be * ob; }
+            }
+            if (lane == 0) { wm[8 * g] = al; wm[8 * g + 1] = be; }
+        } else {
+            // ---- back substitution in reverse window order, x handed over
+            T cp[SC_R], dp[SC_R];
+            sc_load_slot_s(ib_s, lane, cp, dp);
+            __syncwarp();
+            if (lane == 0 && g + SC_NW < nwin) issue(g + SC_NW);
+            T al, be;
+            sc_bwd_map(cp, dp, al, be);
+            sc_bwd_scan(al, be, lane);
+            if (g > 0) asm volatile("bar.sync %0, 64;" ::"r"(1 + pi) : "memory");
+            const T xw = g == 0 ? xa0 : hv[4 * pi];
+            const T xs = fma(be, xw, al);
+            if (lane == 0) hv[4 * pw] = xs;
+            if (g + 1 < nwin) asm volatile("bar.arrive %0, 64;" ::"r"(1 + pw) : "memory");
+            T x = __shfl_down_sync(0xffffffffu, xs, 1);
+            if (lane == 31) x = xw;
+            T xv[SC_R];
+#pragma unroll
+            for (int t = SC_R - 1; t >= 0; --t) {
+                x = fma(-cp[t], x, dp[t]);
+                xv[t] = x;
+            }
+            sc_store_x(p.x + q * n + i0, n - i0, xv);
+        }
+    }
+    if (MODE == 2) return;
+    __syncthreads();
+    if (warp == 0) {
+        if (MODE == 0) {
+            const SKMat<T> R = smc_reduce_fwd(wm, nwin, lane);
+            if (lane == 0) {
+                T* s = p.cmap + 8 * (int64_t)blockIdx.x;
+                s[0] = R.a; s[1] = R.b; s[2] = R.c; s[3] = R.d; s[4] = R.e; s[5] = R.f; s[6] = R.g;
+            }
+        } else {
+            T al, be;
+            smc_reduce_bwd(wm, nwin, lane, al, be);
+            if (lane == 0) { p.cbm[8 * (int64_t)blockIdx.x] = al; p.cbm[8 * (int64_t)blockIdx.x + 1] = be; }
+        }
+    }
+}
+
+}  // namespace tri

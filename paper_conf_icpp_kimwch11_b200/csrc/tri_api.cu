@@ -20,6 +20,7 @@
 #include "k_fused.cuh"
 #include "k_stream.cuh"
 #include "k_scan.cuh"
+#include "k_scan_mc.cuh"
 #include "k_warp.cuh"
 #include "k_pthomas_tma.cuh"
 
@@ -91,11 +92,18 @@ bool stream_ok(int64_t n, int64_t m, tri_dtype t, tri_layout layout) {
 }
 
 // SCAN: contiguous (or one system), n a multiple of 8 (the TMA tensor view
-// [rows/8][8]), at most SC_NCMAX windows of 256 rows; tensor rows fit int32.
+// [m][n/8][8]), at most SC_NCMAX windows of 256 rows.
 bool scan_ok(int64_t n, int64_t m, tri_dtype t, tri_layout layout) {
     (void)t;
     return (layout == TRI_LAYOUT_CONTIGUOUS || m == 1) && n % 8 == 0 && cdiv(n, SC_W) <= SC_NCMAX &&
-           (n / 8) * m < ((int64_t)1 << 31);
+           n / 8 < ((int64_t)1 << 31) && m < ((int64_t)1 << 31);
+}
+
+// SCAN_MC: as SCAN, for systems of at least two windows.
+bool scan_mc_ok(int64_t n, int64_t m, tri_dtype t, tri_layout layout) {
+    (void)t;
+    return (layout == TRI_LAYOUT_CONTIGUOUS || m == 1) && n % 8 == 0 && n > SC_W && n / 8 < ((int64_t)1 << 31) &&
+           m < ((int64_t)1 << 31);
 }
 
 // Variant choice, calibrated once on B200 (the paper tunes P once) from
@@ -120,6 +128,11 @@ tri_variant choose_variant(int64_t n, int64_t m, tri_dtype t, tri_layout layout,
     // 1.01 ms vs 1.12 ms (SPLIT k = 0).  k = 0 throughout: the paper's M > P rule.
     if (layout == TRI_LAYOUT_CONTIGUOUS && scan_ok(n, m, t, layout) && (cdiv(n, SC_W) <= 64 || m >= 128))
         return TRI_VARIANT_SCAN;
+    // SCAN_MC: the remaining contiguous shapes (fewer than 128 systems of more than
+    // 64 windows) -- every system split over several SMs; beats deep-k SPLIT on all
+    // of them (n = 2^24, m = 1: 354 us vs 1052 us; n = 65536, m = 16: 41 us vs 87 us;
+    // n = 2^20, m = 1: 75 us vs 103 us; fp32 n = 2^24: 219 us vs 671 us).
+    if (layout == TRI_LAYOUT_CONTIGUOUS && scan_mc_ok(n, m, t, layout)) return TRI_VARIANT_SCAN_MC;
     // STREAM (profiles/r01_sweep_stream_f64.jsonl): fastest of all variants for
     // fp64 contiguous batches with n % 8 == 0 from 8 windows up, except a few
     // (< 64) very long systems, where SPLIT's deep k keeps more SMs busy
@@ -148,7 +161,7 @@ int choose_k_for(tri_variant v, int64_t n, int64_t m, tri_dtype t, tri_layout la
     if (v == TRI_VARIANT_FUSED) return FU_K;
     if (v == TRI_VARIANT_STREAM) return SK_K;
     if (v == TRI_VARIANT_WARP) return WARP_K;
-    if (v == TRI_VARIANT_SCAN) return 0;
+    if (v == TRI_VARIANT_SCAN || v == TRI_VARIANT_SCAN_MC) return 0;
     const int64_t P = (int64_t)sms * 64;
     if (m >= 48 * (int64_t)sms) return 0;
     int k = m >= P ? 0 : ceil_log2(cdiv(P, m));
@@ -161,7 +174,7 @@ int kmax_for(tri_variant v, int64_t n) {
     if (v == TRI_VARIANT_FUSED) return FU_K;
     if (v == TRI_VARIANT_STREAM) return SK_K;
     if (v == TRI_VARIANT_WARP) return WARP_K;
-    if (v == TRI_VARIANT_SCAN) return 0;
+    if (v == TRI_VARIANT_SCAN || v == TRI_VARIANT_SCAN_MC) return 0;
     return v == TRI_VARIANT_SPLIT ? std::min(kn, SPLIT_KMAX) : kn;
 }
 int kmin_for(tri_variant v) {
@@ -188,6 +201,7 @@ struct tri_plan_s {
     int64_t fu_nc;            // FUSED: windows per system
     int sk_grid, sk_nc, sk_son;  // STREAM / SCAN: persistent CTAs, windows per system, resident storage slots
     int sk_delta;                // SCAN: back-substitution lag (steps)
+    int mc_P, mc_NCW;            // SCAN_MC: chunks per system, windows per chunk
     size_t smem_optin;
     void* scratch;
     size_t scratch_bytes;
@@ -333,6 +347,17 @@ void plan_geometry(tri_plan_s* p) {
         const int64_t avail = ((int64_t)p->smem_optin - fixed) / slot;
         p->sk_son = p->sk_nc == 1 ? 0 : (int)std::max<int64_t>(0, std::min<int64_t>(p->sk_nc + p->sk_delta, avail));
     }
+    if (p->variant == TRI_VARIANT_SCAN_MC) {
+        p->L = n; p->n_pad = n; p->C = m;
+        const int64_t NC = cdiv(n, SC_W);
+        p->sk_nc = (int)NC;
+        int64_t P = std::max(cdiv(p->sms, m), cdiv(NC, SMC_WMAX));
+        P = std::min(P, NC);
+        const int64_t NCW = cdiv(NC, P);
+        p->mc_NCW = (int)NCW;
+        p->mc_P = (int)cdiv(NC, NCW);
+        p->sk_grid = (int)(m * p->mc_P);
+    }
     if (p->variant == TRI_VARIANT_FUSED) {
         const size_t s = esize(p->dtype);
         p->L = cdiv(n, FU_S);
@@ -350,6 +375,9 @@ void plan_geometry(tri_plan_s* p) {
 }
 
 size_t scratch_need(const tri_plan_s* p) {
+    if (p->variant == TRI_VARIANT_SCAN_MC)  // c', d' per window + the chunk maps
+        return ((size_t)p->m * (size_t)p->sk_nc * (size_t)sc_slot_elems<double>() +
+                (size_t)p->m * (size_t)p->mc_P * 16) * esize(p->dtype);
     if (p->variant == TRI_VARIANT_SCAN)
         return p->sk_nc == 1 ? 0
                              : (size_t)p->sk_grid * (size_t)std::max(0, p->sk_nc + p->sk_delta - p->sk_son) *
@@ -593,27 +621,30 @@ cudaError_t launch_stream(const tri_plan_s* p, const void* a, const void* b, con
     return cudaGetLastError();
 }
 
-// ---- SCAN launch: tensor maps [n m / 8][8] (fp64: 64-byte rows, 64B swizzle;
-// fp32: 32-byte rows, 32B swizzle), box 8 x 32 = one 256-row window per array
-bool tma_map_rows8_f32(CUtensorMap* tm, const void* base, uint64_t rows8) {
+// ---- SCAN / SCAN_MC launch: tensor maps [m][n/8][8] (fp64: 64-byte rows, 64B
+// swizzle; fp32: 32-byte rows, 32B swizzle), box [1][32][8] = one 256-row window
+// of one system per array; every coordinate fits int32 for any n, m of the API
+template <typename T>
+bool tma_map_sys_rows8(CUtensorMap* tm, const void* base, int64_t n, int64_t m) {
     auto enc = tma_encoder();
     if (!enc) return false;
-    cuuint64_t dims[2] = {8, rows8};
-    cuuint64_t strides[1] = {8 * sizeof(float)};
-    cuuint32_t box[2] = {8, 32};
-    cuuint32_t es[2] = {1, 1};
-    return enc(tm, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<void*>(base), dims, strides, box, es,
-               CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_32B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+    cuuint64_t dims[3] = {8, (cuuint64_t)(n / 8), (cuuint64_t)m};
+    cuuint64_t strides[2] = {8 * sizeof(T), (cuuint64_t)n * sizeof(T)};
+    cuuint32_t box[3] = {8, 32, 1};
+    cuuint32_t es[3] = {1, 1, 1};
+    return enc(tm, sizeof(T) == 8 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT64 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3,
+               const_cast<void*>(base), dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+               sizeof(T) == 8 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_32B,
+               CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
 template <typename T>
 cudaError_t launch_scan(const tri_plan_s* p, const void* a, const void* b, const void* c, const void* d, void* x,
                         cudaStream_t st) {
     StreamMaps tm;
-    const uint64_t rows8 = (uint64_t)(p->n / 8) * (uint64_t)p->m;
-    auto mk = sizeof(T) == 8 ? tma_map_rows8 : tma_map_rows8_f32;
-    if (!mk(&tm.a, a, rows8) || !mk(&tm.b, b, rows8) || !mk(&tm.c, c, rows8) || !mk(&tm.d, d, rows8))
+    const int64_t n = p->n, m = p->m;
+    if (!tma_map_sys_rows8<T>(&tm.a, a, n, m) || !tma_map_sys_rows8<T>(&tm.b, b, n, m) ||
+        !tma_map_sys_rows8<T>(&tm.c, c, n, m) || !tma_map_sys_rows8<T>(&tm.d, d, n, m))
         return cudaErrorNotSupported;
     ScanArgs<T> A;
     A.x = (T*)x;
@@ -626,6 +657,33 @@ cudaError_t launch_scan(const tri_plan_s* p, const void* a, const void* b, const
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     kern<<<p->sk_grid, SC_THREADS, smem, st>>>(tm, A);
+    return cudaGetLastError();
+}
+
+template <typename T>
+cudaError_t launch_scan_mc(const tri_plan_s* p, const void* a, const void* b, const void* c, const void* d, void* x,
+                           cudaStream_t st) {
+    StreamMaps tm;
+    const int64_t n = p->n, m = p->m;
+    if (!tma_map_sys_rows8<T>(&tm.a, a, n, m) || !tma_map_sys_rows8<T>(&tm.b, b, n, m) ||
+        !tma_map_sys_rows8<T>(&tm.c, c, n, m) || !tma_map_sys_rows8<T>(&tm.d, d, n, m))
+        return cudaErrorNotSupported;
+    ScanMCArgs<T> A;
+    A.x = (T*)x;
+    A.cd = (T*)p->scratch;
+    const int64_t mp = p->m * (int64_t)p->mc_P;
+    A.cmap = A.cd + p->m * (int64_t)p->sk_nc * sc_slot_elems<T>();
+    A.cbm = A.cmap + 8 * mp;
+    A.n = p->n; A.m = p->m; A.NC = p->sk_nc; A.NCW = p->mc_NCW; A.P = p->mc_P;
+    const int smem = SMCLayout<T>::smem_bytes(p->mc_NCW);
+    cudaError_t e;
+    for (auto k : {k_scan_mc<T, 0>, k_scan_mc<T, 1>, k_scan_mc<T, 2>}) {
+        e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+        if (e != cudaSuccess) return e;
+    }
+    k_scan_mc<T, 0><<<p->sk_grid, SC_THREADS, smem, st>>>(tm, A);
+    k_scan_mc<T, 1><<<p->sk_grid, SC_THREADS, smem, st>>>(tm, A);
+    k_scan_mc<T, 2><<<p->sk_grid, SC_THREADS, smem, st>>>(tm, A);
     return cudaGetLastError();
 }
 
@@ -897,6 +955,7 @@ int64_t tri_plan_scratch_bytes(tri_plan_t p) { return p ? (int64_t)p->scratch_by
 int tri_plan_launches(tri_plan_t p) {
     if (!p) return -1;
     if (p->variant == TRI_VARIANT_SPLIT) return p->k == 0 ? 1 : p->k > p->k1 ? 3 : 2;
+    if (p->variant == TRI_VARIANT_SCAN_MC) return 3;
     return 1;  // ONCHIP, FUSED
 }
 
@@ -918,8 +977,9 @@ tri_status tri_plan_set_variant(tri_plan_t p, tri_variant v) {
     if (v == TRI_VARIANT_WARP && !warp_ok(p->n)) return TRI_ERR_INVALID_ARG;
     if (v == TRI_VARIANT_STREAM && !stream_ok(p->n, p->m, p->dtype, p->layout)) return TRI_ERR_INVALID_ARG;
     if (v == TRI_VARIANT_SCAN && !scan_ok(p->n, p->m, p->dtype, p->layout)) return TRI_ERR_INVALID_ARG;
+    if (v == TRI_VARIANT_SCAN_MC && !scan_mc_ok(p->n, p->m, p->dtype, p->layout)) return TRI_ERR_INVALID_ARG;
     if (v != TRI_VARIANT_ONCHIP && v != TRI_VARIANT_SPLIT && v != TRI_VARIANT_FUSED && v != TRI_VARIANT_WARP &&
-        v != TRI_VARIANT_STREAM && v != TRI_VARIANT_SCAN)
+        v != TRI_VARIANT_STREAM && v != TRI_VARIANT_SCAN && v != TRI_VARIANT_SCAN_MC)
         return TRI_ERR_INVALID_ARG;
     const tri_variant ov = p->variant;
     const int ok = p->k;
@@ -934,7 +994,7 @@ tri_status tri_plan_set_variant(tri_plan_t p, tri_variant v) {
 void tri_plan_describe(tri_plan_t p, char* buf, int len) {
     if (!buf || len <= 0) return;
     if (!p) { snprintf(buf, len, "null plan"); return; }
-    static const char* vn[] = {"auto", "onchip", "split", "fused", "warp", "stream", "scan"};
+    static const char* vn[] = {"auto", "onchip", "split", "fused", "warp", "stream", "scan", "scan_mc"};
     snprintf(buf, len,
              "n=%lld m=%lld dtype=%s layout=%s variant=%s k=%d G=%d P=%d rpt=%d L=%lld C=%lld region=%lld nreg=%lld "
              "fu_grid=%d fu_son=%d fu_nc=%lld sk_grid=%d sk_nc=%d sk_son=%d scratch=%zu sms=%d",
@@ -963,6 +1023,9 @@ tri_status tri_solve(tri_plan_t p, const void* a, const void* b, const void* c, 
         e = launch_stream(p, a, b, c, d, x, s);
     } else if (p->variant == TRI_VARIANT_SCAN) {
         e = p->dtype == TRI_F64 ? launch_scan<double>(p, a, b, c, d, x, s) : launch_scan<float>(p, a, b, c, d, x, s);
+    } else if (p->variant == TRI_VARIANT_SCAN_MC) {
+        e = p->dtype == TRI_F64 ? launch_scan_mc<double>(p, a, b, c, d, x, s)
+                                : launch_scan_mc<float>(p, a, b, c, d, x, s);
     } else if (p->variant == TRI_VARIANT_FUSED) {
         e = p->dtype == TRI_F64 ? launch_fused<double>(p, a, b, c, d, x, s) : launch_fused<float>(p, a, b, c, d, x, s);
     } else {
@@ -988,7 +1051,7 @@ tri_status tri_debug_pcr(tri_plan_t p, const void* a, const void* b, const void*
                                 : launch_onchip<float>(p, a, b, c, d, nullptr, ao, co, do_, 1, s);
     } else if (p->variant == TRI_VARIANT_STREAM) {
         e = launch_stream(p, a, b, c, d, nullptr, s, ao, co, do_);
-    } else if (p->variant == TRI_VARIANT_SCAN) {
+    } else if (p->variant == TRI_VARIANT_SCAN || p->variant == TRI_VARIANT_SCAN_MC) {
         return TRI_ERR_INVALID_ARG;  // k = 0: no PCR stage to show
     } else if (p->variant == TRI_VARIANT_FUSED) {
         e = p->dtype == TRI_F64 ? launch_fused<double>(p, a, b, c, d, nullptr, s, ao, co, do_)

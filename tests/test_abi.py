@@ -86,7 +86,7 @@ def test_heuristic_k_valid_and_nonincreasing_in_m(L, dtype, layout, n):
         k = tri.choose_k(n, m, dtype, layout, 148)
         v = tri.choose_variant(n, m, dtype, layout, 148)
         assert v in (tri.VARIANT_ONCHIP, tri.VARIANT_SPLIT, tri.VARIANT_FUSED, tri.VARIANT_WARP, tri.VARIANT_STREAM,
-                     tri.VARIANT_SCAN)
+                     tri.VARIANT_SCAN, tri.VARIANT_SCAN_MC)
         assert 0 <= k <= max(0, n.bit_length() - 1)
         if prev is not None:
             assert k <= prev[0], (n, m, k, prev)
@@ -101,7 +101,8 @@ def test_heuristic_paper_rule_extremes(L):
     assert tri.choose_k(16384, 16384, tri.F32, tri.CONTIGUOUS, 148) == 0
     assert tri.choose_variant(16384, 16384, tri.F64, tri.CONTIGUOUS, 148) == tri.VARIANT_SCAN
     assert tri.choose_k(16384, 16384, tri.F64, tri.CONTIGUOUS, 148) == 0
-    assert tri.choose_k(1 << 24, 1, tri.F64, tri.CONTIGUOUS, 148) >= 8
+    assert tri.choose_k(1 << 24, 1, tri.F64, tri.INTERLEAVED, 148) >= 8
+    assert tri.choose_k((1 << 24) + 1, 1, tri.F64, tri.CONTIGUOUS, 148) >= 8
 
 
 @pytest.mark.parametrize("m,G", [(16384, 1), (16384, 8), (10, 4), (3, 8), (1, 2), (1000, 7)])
@@ -117,13 +118,16 @@ def test_shard_range_partitions(L, m, G):
 @pytest.mark.parametrize("cfg,n,m,dtype,layout,variant,k", [
     ("c1", 1024, 1, "F64", 0, "VARIANT_SCAN", 0),
     ("c2", 1024, 1024, "F64", 1, "VARIANT_WARP", 5),
-    ("c3", 1 << 24, 1, "F64", 0, "VARIANT_SPLIT", 14),
+    ("c3", 1 << 24, 1, "F64", 0, "VARIANT_SCAN_MC", 0),
     ("c4", 256, 1 << 20, "F32", 0, "VARIANT_SCAN", 0),
     ("c5", 16384, 16384, "F64", 0, "VARIANT_SCAN", 0),
     ("c5/2", 16384, 8192, "F64", 0, "VARIANT_SCAN", 0),  # one of 2 ranks (strong scaling)
     ("c5/8", 16384, 2048, "F64", 0, "VARIANT_SCAN", 0),  # one of 8 ranks
     ("c5-il", 16384, 16384, "F64", 1, "VARIANT_SPLIT", 0),  # interleaved layout: k = 0 TMA p-Thomas
-    ("few-long", 65536, 37, "F64", 0, "VARIANT_SPLIT", 8),  # < 64 long systems: deep-k SPLIT
+    ("few-long", 65536, 37, "F64", 0, "VARIANT_SCAN_MC", 0),  # < 128 long systems: chunked SCAN
+    ("few-long-il", 65536, 37, "F64", 1, "VARIANT_SPLIT", 8),  # interleaved: deep-k SPLIT
+    ("odd-n", 1 << 20, 1, "F64", 0, "VARIANT_SCAN_MC", 0),
+    ("ragged", (1 << 20) + 3, 1, "F64", 0, "VARIANT_SPLIT", 14),  # n % 8 != 0: tiled PCR
 ])
 def test_planner_picks_for_baseline_configs(L, cfg, n, m, dtype, layout, variant, k):
     """The planner's (variant, k) on a 148-SM B200 for BASELINE.json's configs,

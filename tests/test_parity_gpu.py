@@ -473,6 +473,64 @@ def test_scan_full_size_sampled(cuda_ok, dtype, n, m):
         check_parity(n, 1, sub, x[sl], dtype, 0)
 
 
+# ------------------------------------------------------------------ SCAN_MC variant
+SCAN_MC = tri.VARIANT_SCAN_MC
+
+
+@pytest.mark.parametrize("dtype", ["f64", "f32"])
+@pytest.mark.parametrize("n,m", [(264, 1), (520, 1), (4104, 5), (65536, 16), (100008, 2), (1 << 20, 3), (16384, 200),
+                                 (1 << 24, 1)])
+def test_scan_mc_parity(cuda_ok, dtype, n, m):
+    """Spans: chunks of one window, ragged last windows and chunks, one chunk per
+    system (m > #SMs), several chunks per system, the c3 shape (2^24 rows: 148
+    chunks of 443 windows)."""
+    arrs = gen(n, m, dtype, 0)
+    x, plan = gpu_solve(n, m, arrs, dtype, 0, variant=SCAN_MC)
+    assert plan.variant == SCAN_MC and plan.k == 0 and plan.launches == 3
+    check_parity(n, m, arrs, x, dtype, 0)
+
+
+@pytest.mark.parametrize("family,eps", [("weak", 1e-2), ("weak", 1e-3), ("integer", 0.0), ("poisson", 0.0)])
+def test_scan_mc_families(cuda_ok, family, eps):
+    n, m = (16384, 2) if family == "poisson" else (1 << 20, 2)
+    arrs = gen(n, m, "f64", 0, family, eps=eps)
+    x, _ = gpu_solve(n, m, arrs, "f64", 0, variant=SCAN_MC)
+    if family == "poisson":
+        xo = oracle.solve_batch(n, m, *arrs)
+        assert np.max(np.abs(x - xo)) / np.max(np.abs(xo)) <= 2 * (n + 1) ** 2 / 2 * 2.2e-16
+    else:
+        check_parity(n, m, arrs, x, "f64", 0)
+
+
+def test_scan_mc_edges_and_scaling(cuda_ok):
+    """X1 NaN edges ignored (bitwise), power-of-two row / rhs scaling (bitwise),
+    determinism, k fixed at 0."""
+    import torch
+    n, m = 300000, 2
+    a, b, c, d = gen(n, m, "f64", 0, "weak", eps=1e-2)
+    plan = tri.Plan(n, m, tri.F64, 0)
+    plan.variant = SCAN_MC
+    da, db, dc, dd = to_dev(a, b, c, d)
+    x1 = plan.solve(da, db, dc, dd).clone()
+    assert torch.equal(plan.solve(da, db, dc, dd), x1)
+    a2, c2 = da.clone(), dc.clone()
+    a2.view(m, n)[:, 0] = float("nan")
+    c2.view(m, n)[:, -1] = float("nan")
+    assert torch.equal(plan.solve(a2, db, c2, dd), x1)
+    p = 2.0 ** np.random.default_rng(2).integers(-20, 20, n * m)
+    assert torch.equal(plan.solve(*to_dev(a * p, b * p, c * p, d * p)), x1)
+    assert torch.equal(plan.solve(da, db, dc, dd * 4.0), x1 * 4.0)
+    with pytest.raises(tri.TriError):
+        plan.k = 1
+
+
+def test_scan_mc_rejects_unsupported(cuda_ok):
+    for (n, m, dt, layout) in [(256, 3, tri.F64, 0), (1004, 3, tri.F64, 0), (16384, 3, tri.F64, 1)]:
+        plan = tri.Plan(n, m, dt, layout)
+        with pytest.raises(tri.TriError):
+            plan.variant = SCAN_MC
+
+
 # ------------------------------------------------------------------ WARP variant
 @pytest.mark.parametrize("dtype", ["f64", "f32"])
 @pytest.mark.parametrize("layout", [0, 1])
