@@ -67,9 +67,9 @@ struct SCLayout {
     static constexpr int in_bytes = 4 * SC_W * (int)sizeof(T);           // one window, 4 arrays
     static constexpr int in_stride = (in_bytes + 1023) / 1024 * 1024;     // swizzle atoms aligned
     static constexpr int off_in = 0;
-    static constexpr int off_st = off_in + SC_NW * in_stride;             // [NW][theta|psi|delta]
-    static constexpr int off_xh = off_st + SC_NW * 4 * (int)sizeof(T);    // [NW] x handover
-    static constexpr int off_bar = (off_xh + SC_NW * (int)sizeof(T) + 7) / 8 * 8;  // [NW] in_full
+    static constexpr int off_st = off_in + SC_NW * in_stride;             // [NW][<= 8 systems][theta|psi|delta]
+    static constexpr int off_xh = off_st + SC_NW * 8 * 4 * (int)sizeof(T);    // [NW][<= 8 systems] x handover
+    static constexpr int off_bar = (off_xh + SC_NW * 8 * (int)sizeof(T) + 7) / 8 * 8;  // [NW] in_full
     static constexpr int off_cnt = off_bar + SC_NW * 8;                   // [NC] windows-stored counters
     // [K][NC] u16: slot of window (j, w) at row j % K, K = 3 + (delta - 1) / NC
     // systems in flight between a window's store and its read-back (<= 3 NC + delta entries)
@@ -134,6 +134,21 @@ __device__ __forceinline__ void sc_ld_rows(const T* ib, int lane, T (&ra)[SC_R],
     }
 }
 
+// INTERLEAVED layout, S systems per window: the TMA tile is [WR rows][S systems]
+// (row-major, unswizzled); lane (s, seg) takes rows seg*8 .. seg*8+7 of system s
+template <int S, typename T>
+__device__ __forceinline__ void sc_ld_rows_il(const T* ib, int s, int seg, T (&ra)[SC_R], T (&rb)[SC_R],
+                                              T (&rc)[SC_R], T (&rd)[SC_R]) {
+    const T* st = ib + seg * SC_R * S + s;
+#pragma unroll
+    for (int t = 0; t < SC_R; ++t) {
+        ra[t] = st[0 * SC_W + t * S];
+        rb[t] = st[1 * SC_W + t * S];
+        rc[t] = st[2 * SC_W + t * S];
+        rd[t] = st[3 * SC_W + t * S];
+    }
+}
+
 // rows outside [0, n) are identity rows; a_0 and c_{n-1} lie outside A (X1, X4)
 template <typename T>
 __device__ __forceinline__ void sc_fix_rows(int64_t i0, int64_t n, T (&ra)[SC_R], T (&rb)[SC_R], T (&rc)[SC_R],
@@ -170,10 +185,10 @@ __device__ __forceinline__ SKMat<T> sc_fwd_map(const T (&ra)[SC_R], const T (&rb
 
 // both scans in one pass (their shuffles and arithmetic interleave): forward
 // inclusive over the lanes, backward suffix
-template <typename T>
+template <int S, typename T>
 __device__ __forceinline__ void sc_scans(SKMat<T>& M, T& al, T& be, int lane) {
 #pragma unroll
-    for (int dd = 1; dd < 32; dd <<= 1) {
+    for (int dd = S; dd < 32; dd <<= 1) {
         const SKMat<T> o = sk_shfl_up(M, dd);
         T oa = __shfl_down_sync(0xffffffffu, al, dd), ob = __shfl_down_sync(0xffffffffu, be, dd);
         if (lane + dd >= 32) { oa = T(0); ob = T(1); }
@@ -324,8 +339,14 @@ __device__ __forceinline__ void sc_store_x(T* xo, int64_t rmax, const T (&xv)[SC
     }
 }
 
-template <typename T, bool PROF>
+// S = systems per window: 1 for the CONTIGUOUS layout (a window = 256 rows of one
+// system, 32 lane segments), 2 / 4 / 8 for the INTERLEAVED layout (a window =
+// 256 / S rows of S adjacent systems, lane (s, seg) = (lane % S, lane / S), the
+// scans run over the 32 / S segments of each system: shuffle distances S .. 16).
+template <typename T, int S, bool PROF>
 __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ StreamMaps tm, ScanArgs<T> p) {
+    constexpr int WR = SC_W / S;      // rows per window
+    constexpr int NSEG = 32 / S;      // lane segments per system
     using L = SCLayout<T>;
     extern __shared__ __align__(16) unsigned char sc_smem_raw[];
     unsigned char* sbase = sc_smem_raw + ((1024 - ((unsigned)__cvta_generic_to_shared(sc_smem_raw) & 1023)) & 1023);
@@ -347,23 +368,33 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
     __syncthreads();
 
     const int64_t n = p.n;
-    const int nsys = (int)((p.m - blockIdx.x + gridDim.x - 1) / gridDim.x);
+    const int64_t ngrp = (p.m + S - 1) / S;  // groups of S systems (one "system" of the chain)
+    const int nsys = (int)((ngrp - blockIdx.x + gridDim.x - 1) / gridDim.x);
     const int pw = warp;
+    const int ls = lane % S, seg = lane / S;
     T* ib = reinterpret_cast<T*>(sbase + L::off_in + pw * L::in_stride);
     const uint64_t pol_in = sk_policy_evict_first();
     const uint64_t pol_sp = sk_policy_evict_last();
     auto issue = [&](int jj, int ww) {
         const int q = (int)(blockIdx.x + (int64_t)jj * gridDim.x);
-        const int y = ww * (SC_W / 8);
         sk_expect(&in_full[pw], (unsigned)(4 * SC_W * sizeof(T)));
-        sc_tma3d(ib + 0 * SC_W, &tm.a, y, q, &in_full[pw], pol_in);
-        sc_tma3d(ib + 1 * SC_W, &tm.b, y, q, &in_full[pw], pol_in);
-        sc_tma3d(ib + 2 * SC_W, &tm.c, y, q, &in_full[pw], pol_in);
-        sc_tma3d(ib + 3 * SC_W, &tm.d, y, q, &in_full[pw], pol_in);
+        if constexpr (S == 1) {
+            const int y = ww * (SC_W / 8);
+            sc_tma3d(ib + 0 * SC_W, &tm.a, y, q, &in_full[pw], pol_in);
+            sc_tma3d(ib + 1 * SC_W, &tm.b, y, q, &in_full[pw], pol_in);
+            sc_tma3d(ib + 2 * SC_W, &tm.c, y, q, &in_full[pw], pol_in);
+            sc_tma3d(ib + 3 * SC_W, &tm.d, y, q, &in_full[pw], pol_in);
+        } else {  // tensor [n][m], box [WR][S]
+            const int y = ww * WR, xq = q * S;
+            sk_tma2d(ib + 0 * SC_W, &tm.a, xq, y, &in_full[pw], pol_in);
+            sk_tma2d(ib + 1 * SC_W, &tm.b, xq, y, &in_full[pw], pol_in);
+            sk_tma2d(ib + 2 * SC_W, &tm.c, xq, y, &in_full[pw], pol_in);
+            sk_tma2d(ib + 3 * SC_W, &tm.d, xq, y, &in_full[pw], pol_in);
+        }
     };
     unsigned ph = 0;
 
-    if (NC == 1) {
+    if (S == 1 && NC == 1) {
         // ---- systems of one window: each warp solves whole systems, no chain
         if (lane == 0 && pw < nsys) issue(pw, 0);
         for (int j = pw; j < nsys; j += SC_NW) {
@@ -372,7 +403,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
             sk_wait(&in_full[pw], ph);
             ph ^= 1u;
             sc_ld_rows(ib, lane, ra, rb, rc, rd);
-            __syncwarp();
+            sc_release_buf();  // this warp's reads of the buffer before the TMA refill
             if (lane == 0 && j + SC_NW < nsys) issue(j + SC_NW, 0);
             sc_fix_rows<T>((int64_t)lane * SC_R, n, ra, rb, rc, rd);
             SKMat<T> M = sc_fwd_map(ra, rb, rc, rd);
@@ -427,7 +458,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
         const bool fwd = cj < nsys, bwd = bb >= 0;
         const int bj = bwd ? bb / NC : 0;
         const int wb = NC - 1 - (bb - bj * NC);  // backward window (system bj)
-        const int64_t i0d = (int64_t)cw * SC_W + lane * SC_R;
+        const int64_t i0d = (int64_t)cw * WR + seg * SC_R;
         int slot = g;                            // fresh slot (g < NS when !bwd)
         if (bwd && p.dbg != 2) {
             SC_T(5);
@@ -448,8 +479,10 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
                 T xv[SC_R];
 #pragma unroll
                 for (int t = 0; t < SC_R; ++t) xv[t] = T(0);
-                const int64_t q = blockIdx.x + (int64_t)cj * gridDim.x;
-                sc_store_x(p.x + q * n + i0d, n - i0d, xv);
+                if constexpr (S == 1) {
+                    const int64_t q = blockIdx.x + (int64_t)cj * gridDim.x;
+                    sc_store_x(p.x + q * n + i0d, n - i0d, xv);
+                }
             }
             continue;
         }
@@ -465,8 +498,20 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
 
         // ---- forward: segment map of window (cj, cw) (identity rows when inactive);
         // the rows are read again from the staging buffer for the replay
-        const int64_t i0 = (int64_t)cw * SC_W + lane * SC_R;
-        const bool edge = cw == 0 || (int64_t)(cw + 1) * SC_W > n;
+        const int64_t i0 = (int64_t)cw * WR + seg * SC_R;
+        const int64_t qf = (blockIdx.x + (int64_t)cj * gridDim.x) * S + ls;  // this lane's system
+        const bool edge = cw == 0 || (int64_t)(cw + 1) * WR > n || (S > 1 && qf >= p.m);
+        auto load_rows = [&](T (&ra)[SC_R], T (&rb)[SC_R], T (&rc)[SC_R], T (&rd)[SC_R]) {
+            if constexpr (S == 1) sc_ld_rows(ib, lane, ra, rb, rc, rd);
+            else sc_ld_rows_il<S>(ib, ls, seg, ra, rb, rc, rd);
+        };
+        auto fix_rows = [&](T (&ra)[SC_R], T (&rb)[SC_R], T (&rc)[SC_R], T (&rd)[SC_R]) {
+            sc_fix_rows<T>(i0, n, ra, rb, rc, rd);
+            if (S > 1 && qf >= p.m) {  // padding systems of the last group: identity rows
+#pragma unroll
+                for (int u = 0; u < SC_R; ++u) { ra[u] = T(0); rb[u] = T(1); rc[u] = T(0); rd[u] = T(0); }
+            }
+        };
         SKMat<T> M;
         if (fwd) {
             SC_T(5);
@@ -474,58 +519,58 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
             SC_T(1);
             ph ^= 1u;
             T ra[SC_R], rb[SC_R], rc[SC_R], rd[SC_R];
-            sc_ld_rows(ib, lane, ra, rb, rc, rd);
-            if (edge) sc_fix_rows<T>(i0, n, ra, rb, rc, rd);
+            load_rows(ra, rb, rc, rd);
+            if (edge) fix_rows(ra, rb, rc, rd);
             M = sc_fwd_map(ra, rb, rc, rd);
         } else {
             M = SKMat<T>{T(1), T(0), T(0), T(1), T(0), T(0), T(1)};
         }
         T al, be;
         sc_bwd_map(cpb, dpb, al, be);
-        sc_scans(M, al, be, lane);
+        sc_scans<S>(M, al, be, lane);
 
         // ---- the serial steps: the forward state and x of step g - 1, handed over
         // through the hardware named barrier 1 + pi (warp pi -> warp pw, 64 threads)
         SC_T(5);
         if (g > 0 && p.dbg != 1) asm volatile("bar.sync %0, 64;" ::"r"(1 + pi) : "memory");
         SC_T(2);
-        const T xw = (bwd && wb < NC - 1) ? xh[pi] : T(0);  // x at the first row of window wb + 1
+        const T xw = (bwd && wb < NC - 1) ? xh[pi * S + ls] : T(0);  // x at the first row of window wb + 1
         T th = T(1), ps = T(0), de = T(0);                  // theta_{-1} = 1, psi_0 = 0, delta_{-1} = 0
         if (fwd && cw > 0) {
-            th = stt[pi * 4 + 0];
-            ps = stt[pi * 4 + 1];
-            de = stt[pi * 4 + 2];
+            th = stt[(pi * S + ls) * 4 + 0];
+            ps = stt[(pi * S + ls) * 4 + 1];
+            de = stt[(pi * S + ls) * 4 + 2];
         }
         const T xs = fma(be, xw, al);  // x at the lane's first row
         const T ot = fma(M.a, th, M.b * ps);
         const T op = fma(M.c, th, M.d * ps);
         const T od = fma(M.e, th, fma(M.f, ps, M.g * de));
-        if (lane == 0) xh[pw] = xs;
-        if (lane == 31) {  // window end: exact power-of-two rescale, hand over
+        if (seg == 0) xh[pw * S + ls] = xs;
+        if (seg == NSEG - 1) {  // window end: exact power-of-two rescale, hand over
             const T sc = sk_exp2_scale(ot);
-            stt[pw * 4 + 0] = ot * sc;
-            stt[pw * 4 + 1] = op * sc;
-            stt[pw * 4 + 2] = od * sc;
+            stt[(pw * S + ls) * 4 + 0] = ot * sc;
+            stt[(pw * S + ls) * 4 + 1] = op * sc;
+            stt[(pw * S + ls) * 4 + 2] = od * sc;
         }
         if (g + 1 < total && p.dbg != 1)  // arrive -> sync: release / acquire (PTX memory model)
             asm volatile("bar.arrive %0, 64;" ::"r"(1 + pw) : "memory");
         SC_T(3);
-        T x = __shfl_down_sync(0xffffffffu, xs, 1);  // x after the lane's rows
-        if (lane == 31) x = xw;
+        T x = __shfl_down_sync(0xffffffffu, xs, S);  // x after the lane's rows
+        if (seg == NSEG - 1) x = xw;
         {
-            const T it_ = __shfl_up_sync(0xffffffffu, ot, 1);
-            const T ip = __shfl_up_sync(0xffffffffu, op, 1);
-            const T id = __shfl_up_sync(0xffffffffu, od, 1);
-            if (lane > 0) { th = it_; ps = ip; de = id; }
+            const T it_ = __shfl_up_sync(0xffffffffu, ot, S);
+            const T ip = __shfl_up_sync(0xffffffffu, op, S);
+            const T id = __shfl_up_sync(0xffffffffu, od, S);
+            if (seg > 0) { th = it_; ps = ip; de = id; }
         }
 
         // ---- forward replay: c', d' (Eqs 2-3) of window (cj, cw) into the slot,
         // then the next input window of this warp
         if (fwd) {
             T ra[SC_R], rb[SC_R], rc[SC_R], rd[SC_R];
-            sc_ld_rows(ib, lane, ra, rb, rc, rd);
-            if (edge) sc_fix_rows<T>(i0, n, ra, rb, rc, rd);
-            __syncwarp();
+            load_rows(ra, rb, rc, rd);
+            if (edge) fix_rows(ra, rb, rc, rd);
+            sc_release_buf();  // this warp's reads of the buffer before the TMA refill
             if (lane == 0 && g + SC_NW < nfwd) issue(j, w);
             T cpf[SC_R], dpf[SC_R];
             sc_fwd_replay(ra, rb, rc, rd, th, ps, de, cpf, dpf);
@@ -546,8 +591,17 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
                 xv[t] = x;
             }
             const int64_t qb = blockIdx.x + (int64_t)bj * gridDim.x;
-            const int64_t xr = (int64_t)wb * SC_W + lane * SC_R;
-            sc_store_x(p.x + qb * n + xr, n - xr, xv);
+            const int64_t xr = (int64_t)wb * WR + seg * SC_R;
+            if constexpr (S == 1) {
+                sc_store_x(p.x + qb * n + xr, n - xr, xv);
+            } else {  // INTERLEAVED: x[row * m + q]
+                const int64_t qx = qb * S + ls;
+                if (qx < p.m) {
+#pragma unroll
+                    for (int t = 0; t < SC_R; ++t)
+                        if (xr + t < n) __stcs(p.x + (xr + t) * p.m + qx, xv[t]);
+                }
+            }
         }
         SC_T(6);
     }

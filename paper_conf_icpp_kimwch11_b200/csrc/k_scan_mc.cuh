@@ -179,7 +179,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant
             // ---- the window's forward map (product of the lane segment maps)
             T ra[SC_R], rb[SC_R], rc[SC_R], rd[SC_R];
             sc_ld_rows(ib, lane, ra, rb, rc, rd);
-            __syncwarp();
+            sc_release_buf();  // this warp's reads of the buffer before the TMA refill
             if (lane == 0 && g + SC_NW < nwin) issue(g + SC_NW);
             if (edge) sc_fix_rows<T>(i0, n, ra, rb, rc, rd);
             SKMat<T> M = sc_fwd_map(ra, rb, rc, rd);
@@ -220,7 +220,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant
                 const T id = __shfl_up_sync(0xffffffffu, od, 1);
                 if (lane > 0) { th = it_; ps = ip; de = id; }
             }
-            __syncwarp();
+            sc_release_buf();  // this warp's reads of the buffer before the TMA refill
             if (lane == 0 && g + SC_NW < nwin) issue(g + SC_NW);  // rows are in registers
             T cp[SC_R], dp[SC_R];
             sc_fwd_replay(ra, rb, rc, rd, th, ps, de, cp, dp);
@@ -248,7 +248,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant
             // ---- back substitution in reverse window order, x handed over
             T cp[SC_R], dp[SC_R];
             sc_load_slot_s(ib_s, lane, cp, dp);
-            __syncwarp();
+            sc_release_buf();  // this warp's reads of the buffer before the TMA refill
             if (lane == 0 && g + SC_NW < nwin) issue(g + SC_NW);
             T al, be;
             sc_bwd_map(cp, dp, al, be);

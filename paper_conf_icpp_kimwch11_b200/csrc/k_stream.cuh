@@ -168,6 +168,15 @@ __device__ __forceinline__ void sk_wait_ge(const int* p, int v) {
     while (sk_ld_acquire(p) < v) __nanosleep(64);
 }
 
+// Before a warp refills a staging buffer it has read with generic-proxy loads by
+// TMA (async proxy): every lane fences its reads against the async proxy, then
+// the warp synchronises, then one lane issues the copy (the write-after-read
+// hazard otherwise lets the refill land before slow shared-memory loads).
+__device__ __forceinline__ void sc_release_buf() {
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    __syncwarp();
+}
+
 template <typename T>
 __device__ __forceinline__ T sk_exp2_scale(T v);
 template <>
@@ -385,7 +394,7 @@ __global__ void __launch_bounds__(SK_THREADS, 1) k_stream(const __grid_constant_
                     }
                 }
             }
-            __syncwarp();
+            sc_release_buf();  // this warp's reads of the buffer before the TMA refill
             if (lane == 0 && g + SK_NPCR < nfwd) issue(j, w);
         } else {
 #pragma unroll

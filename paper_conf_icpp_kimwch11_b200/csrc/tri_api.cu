@@ -93,10 +93,25 @@ bool stream_ok(int64_t n, int64_t m, tri_dtype t, tri_layout layout) {
 
 // SCAN: contiguous (or one system), n a multiple of 8 (the TMA tensor view
 // [m][n/8][8]), at most SC_NCMAX windows of 256 rows.
+int g_scan_s_il = env_int("TRI_SCAN_S", 0);  // SCAN, interleaved: systems per window (tuning; 0 = planner)
+// systems per window of the SCAN kernel: 1 (contiguous), 2 / 4 / 8 (interleaved:
+// the TMA box's inner extent S * s must be >= 16 bytes)
+int scan_systems(int64_t n, int64_t m, tri_dtype t, tri_layout layout) {
+    (void)n; (void)m;
+    if (layout == TRI_LAYOUT_CONTIGUOUS) return 1;
+    // 8: a window's row of S systems is 64 B (fp64) / 32 B (fp32), at least one
+    // whole DRAM sector per TMA row (S = 2 fp64 measured 2x slower: half sectors)
+    const int smin = t == TRI_F64 ? 2 : 4;
+    if (g_scan_s_il == 2 || g_scan_s_il == 4 || g_scan_s_il == 8) return std::max(smin, g_scan_s_il);
+    return 8;
+}
 bool scan_ok(int64_t n, int64_t m, tri_dtype t, tri_layout layout) {
-    (void)t;
-    return (layout == TRI_LAYOUT_CONTIGUOUS || m == 1) && n % 8 == 0 && cdiv(n, SC_W) <= SC_NCMAX &&
-           n / 8 < ((int64_t)1 << 31) && m < ((int64_t)1 << 31);
+    if (layout == TRI_LAYOUT_CONTIGUOUS || m == 1)
+        return n % 8 == 0 && cdiv(n, SC_W) <= SC_NCMAX && n / 8 < ((int64_t)1 << 31) && m < ((int64_t)1 << 31);
+    // INTERLEAVED: TMA tensor [n][m], row stride m * s a multiple of 16 bytes
+    const int S = scan_systems(n, m, t, layout);
+    return (m * (int64_t)esize(t)) % 16 == 0 && cdiv(n, SC_W / S) <= SC_NCMAX && n < ((int64_t)1 << 31) &&
+           m < ((int64_t)1 << 31);
 }
 
 // SCAN_MC: as SCAN, for systems of at least two windows.
@@ -133,6 +148,17 @@ tri_variant choose_variant(int64_t n, int64_t m, tri_dtype t, tri_layout layout,
     // of them (n = 2^24, m = 1: 354 us vs 1052 us; n = 65536, m = 16: 41 us vs 87 us;
     // n = 2^20, m = 1: 75 us vs 103 us; fp32 n = 2^24: 219 us vs 671 us).
     if (layout == TRI_LAYOUT_CONTIGUOUS && scan_mc_ok(n, m, t, layout)) return TRI_VARIANT_SCAN_MC;
+    // SCAN on the INTERLEAVED layout (8 adjacent systems per window;
+    // profiles/r01_sweep_scan_il_*.jsonl): fastest from 256 systems of >= 256 rows
+    // up to where the 8-system groups' intermediates stop fitting on chip / in L2
+    // (fp64 n m >= 2^27: SPLIT k = 0 1.07x faster at 8192 x 16384) or, fp32, where
+    // many short systems favour one thread per system (n < 1024, m > 16384);
+    // e.g. c2 1024 x 1024: 18 us vs 28 us (WARP); 4096 x 4096: 170 us vs 879 us.
+    if (layout == TRI_LAYOUT_INTERLEAVED && m >= 256 && n >= 256 && scan_ok(n, m, t, layout)) {
+        const int64_t N = n * m;
+        const bool fits = t == TRI_F64 ? N < ((int64_t)1 << 27) : N < ((int64_t)1 << 28) && (n >= 1024 || m <= 16384);
+        if (fits) return TRI_VARIANT_SCAN;
+    }
     // STREAM (profiles/r01_sweep_stream_f64.jsonl): fastest of all variants for
     // fp64 contiguous batches with n % 8 == 0 from 8 windows up, except a few
     // (< 64) very long systems, where SPLIT's deep k keeps more SMs busy
@@ -201,6 +227,7 @@ struct tri_plan_s {
     int64_t fu_nc;            // FUSED: windows per system
     int sk_grid, sk_nc, sk_son;  // STREAM / SCAN: persistent CTAs, windows per system, resident storage slots
     int sk_delta;                // SCAN: back-substitution lag (steps)
+    int sk_S;                    // SCAN: systems per window (1 contiguous; 2 / 4 / 8 interleaved)
     int mc_P, mc_NCW;            // SCAN_MC: chunks per system, windows per chunk
     size_t smem_optin;
     void* scratch;
@@ -338,14 +365,16 @@ void plan_geometry(tri_plan_s* p) {
     }
     if (p->variant == TRI_VARIANT_SCAN) {
         p->L = n; p->n_pad = n; p->C = m;
-        p->sk_nc = (int)cdiv(n, SC_W);
-        p->sk_grid = (int)std::min<int64_t>(m, p->sms);
+        const bool il = p->layout == TRI_LAYOUT_INTERLEAVED && m > 1;
+        p->sk_S = il ? scan_systems(n, m, p->dtype, p->layout) : 1;
+        p->sk_nc = (int)cdiv(n, SC_W / p->sk_S);
+        p->sk_grid = (int)std::min<int64_t>(cdiv(m, p->sk_S), p->sms);
         p->sk_delta = g_scan_delta;
         const int fixed = p->dtype == TRI_F64 ? SCLayout<double>::smem_bytes(p->sk_nc, p->sk_delta, 0)
                                               : SCLayout<float>::smem_bytes(p->sk_nc, p->sk_delta, 0);
         const int slot = p->dtype == TRI_F64 ? SCLayout<double>::slot_bytes : SCLayout<float>::slot_bytes;
         const int64_t avail = ((int64_t)p->smem_optin - fixed) / slot;
-        p->sk_son = p->sk_nc == 1 ? 0 : (int)std::max<int64_t>(0, std::min<int64_t>(p->sk_nc + p->sk_delta, avail));
+        p->sk_son = (p->sk_nc == 1 && p->sk_S == 1) ? 0 : (int)std::max<int64_t>(0, std::min<int64_t>(p->sk_nc + p->sk_delta, avail));
     }
     if (p->variant == TRI_VARIANT_SCAN_MC) {
         p->L = n; p->n_pad = n; p->C = m;
@@ -379,7 +408,7 @@ size_t scratch_need(const tri_plan_s* p) {
         return ((size_t)p->m * (size_t)p->sk_nc * (size_t)sc_slot_elems<double>() +
                 (size_t)p->m * (size_t)p->mc_P * 16) * esize(p->dtype);
     if (p->variant == TRI_VARIANT_SCAN)
-        return p->sk_nc == 1 ? 0
+        return (p->sk_nc == 1 && p->sk_S == 1) ? 0
                              : (size_t)p->sk_grid * (size_t)std::max(0, p->sk_nc + p->sk_delta - p->sk_son) *
                                    (size_t)sc_slot_elems<double>() * esize(p->dtype);
     if (p->variant == TRI_VARIANT_STREAM)
@@ -638,14 +667,41 @@ bool tma_map_sys_rows8(CUtensorMap* tm, const void* base, int64_t n, int64_t m) 
                CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
+// INTERLEAVED: tensor [n][m] (row stride m elements), box [256 / S rows][S systems]
+template <typename T>
+bool tma_map_il(CUtensorMap* tm, const void* base, int64_t n, int64_t m, int S) {
+    auto enc = tma_encoder();
+    if (!enc) return false;
+    cuuint64_t dims[2] = {(cuuint64_t)m, (cuuint64_t)n};
+    cuuint64_t strides[1] = {(cuuint64_t)m * sizeof(T)};
+    cuuint32_t box[2] = {(cuuint32_t)S, (cuuint32_t)(SC_W / S)};
+    cuuint32_t es[2] = {1, 1};
+    return enc(tm, sizeof(T) == 8 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT64 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2,
+               const_cast<void*>(base), dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+               CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+template <typename T, int S>
+void* scan_kernel(bool prof) {
+    return prof ? (void*)k_scan<T, S, true> : (void*)k_scan<T, S, false>;
+}
+
 template <typename T>
 cudaError_t launch_scan(const tri_plan_s* p, const void* a, const void* b, const void* c, const void* d, void* x,
                         cudaStream_t st) {
     StreamMaps tm;
     const int64_t n = p->n, m = p->m;
-    if (!tma_map_sys_rows8<T>(&tm.a, a, n, m) || !tma_map_sys_rows8<T>(&tm.b, b, n, m) ||
-        !tma_map_sys_rows8<T>(&tm.c, c, n, m) || !tma_map_sys_rows8<T>(&tm.d, d, n, m))
-        return cudaErrorNotSupported;
+    const int S = p->sk_S;
+    if (S == 1) {
+        if (!tma_map_sys_rows8<T>(&tm.a, a, n, m) || !tma_map_sys_rows8<T>(&tm.b, b, n, m) ||
+            !tma_map_sys_rows8<T>(&tm.c, c, n, m) || !tma_map_sys_rows8<T>(&tm.d, d, n, m))
+            return cudaErrorNotSupported;
+    } else {
+        if (!tma_map_il<T>(&tm.a, a, n, m, S) || !tma_map_il<T>(&tm.b, b, n, m, S) ||
+            !tma_map_il<T>(&tm.c, c, n, m, S) || !tma_map_il<T>(&tm.d, d, n, m, S))
+            return cudaErrorNotSupported;
+    }
     ScanArgs<T> A;
     A.x = (T*)x;
     A.spill = (T*)p->scratch;
@@ -653,11 +709,13 @@ cudaError_t launch_scan(const tri_plan_s* p, const void* a, const void* b, const
     A.prof = (unsigned long long*)g_fused_prof;
     A.dbg = g_fused_dbg_mode;
     const size_t smem = (size_t)SCLayout<T>::smem_bytes(p->sk_nc, p->sk_delta, p->sk_son);
-    auto kern = A.prof ? k_scan<T, true> : k_scan<T, false>;
+    const bool pr = A.prof != nullptr;
+    void* kern = S == 1 ? scan_kernel<T, 1>(pr) : S == 2 ? scan_kernel<T, 2>(pr) : S == 4 ? scan_kernel<T, 4>(pr)
+                                                                                 : scan_kernel<T, 8>(pr);
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
-    kern<<<p->sk_grid, SC_THREADS, smem, st>>>(tm, A);
-    return cudaGetLastError();
+    void* args[] = {(void*)&tm, (void*)&A};
+    return cudaLaunchKernel(kern, dim3(p->sk_grid), dim3(SC_THREADS), args, smem, st);
 }
 
 template <typename T>

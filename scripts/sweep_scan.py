@@ -33,24 +33,31 @@ def time_plan(plan, a, b, c, d, x, reps):
 
 
 DT = sys.argv[1] if len(sys.argv) > 1 else "f64"
+LAYOUT = int(sys.argv[2]) if len(sys.argv) > 2 else 0
 TD = tri.F64 if DT == "f64" else tri.F32
 MAXE = (1 << 27) if DT == "f64" else (1 << 28)
 SHAPES = []
-for n in (256, 512, 1024, 2048, 4096, 8192, 16384, 65536, 1 << 20):
-    for m in (1, 16, 148, 592, 2368, 9472, 37888, 151552, 1 << 20):
-        if n * m <= MAXE and n * m >= 4096:
-            SHAPES.append((n, m))
+if LAYOUT == 0:
+    for n in (256, 512, 1024, 2048, 4096, 8192, 16384, 65536, 1 << 20):
+        for m in (1, 16, 148, 592, 2368, 9472, 37888, 151552, 1 << 20):
+            if n * m <= MAXE and n * m >= 4096:
+                SHAPES.append((n, m))
+else:  # interleaved: m a multiple of 8
+    for n in (64, 256, 1024, 2048, 4096, 8192, 16384):
+        for m in (64, 296, 1024, 2368, 4096, 9472, 16384, 37888, 151552, 1 << 20):
+            if n * m <= MAXE and n * m >= 4096:
+                SHAPES.append((n, m))
 VARS = [tri.VARIANT_SCAN, tri.VARIANT_STREAM, tri.VARIANT_SPLIT, tri.VARIANT_FUSED, tri.VARIANT_WARP, tri.VARIANT_ONCHIP]
 for n, m in SHAPES:
-    arrs = trigen.generate(n, m, DT, 0, "dd")
+    arrs = trigen.generate(n, m, DT, LAYOUT, "dd")
     a, b, c, d = (torch.from_numpy(t).cuda() for t in arrs)
     x = torch.empty_like(b)
     reps = max(3, min(200, int(4e9 / max(1, n * m * b.element_size() * 5))))
-    plan = tri.Plan(n, m, TD, 0)
-    rec = {"n": n, "m": m, "dtype": DT, "auto": {"variant": plan.variant, "k": plan.k, "us": time_plan(plan, a, b, c, d, x, reps)}}
+    plan = tri.Plan(n, m, TD, LAYOUT)
+    rec = {"n": n, "m": m, "dtype": DT, "layout": LAYOUT, "auto": {"variant": plan.variant, "k": plan.k, "us": time_plan(plan, a, b, c, d, x, reps)}}
     allv = []
     for v in VARS:
-        p = tri.Plan(n, m, TD, 0)
+        p = tri.Plan(n, m, TD, LAYOUT)
         try:
             p.variant = v
             if v == tri.VARIANT_SPLIT and m >= 148:

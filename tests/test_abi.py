@@ -117,7 +117,7 @@ def test_shard_range_partitions(L, m, G):
 
 @pytest.mark.parametrize("cfg,n,m,dtype,layout,variant,k", [
     ("c1", 1024, 1, "F64", 0, "VARIANT_SCAN", 0),
-    ("c2", 1024, 1024, "F64", 1, "VARIANT_WARP", 5),
+    ("c2", 1024, 1024, "F64", 1, "VARIANT_SCAN", 0),
     ("c3", 1 << 24, 1, "F64", 0, "VARIANT_SCAN_MC", 0),
     ("c4", 256, 1 << 20, "F32", 0, "VARIANT_SCAN", 0),
     ("c5", 16384, 16384, "F64", 0, "VARIANT_SCAN", 0),

@@ -218,6 +218,7 @@ def test_concurrent_plans_two_streams(cuda_ok):
     a, b, c, d = to_dev(*arrs)
     s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
     p1, p2 = tri.Plan(n, m, tri.F64, 0), tri.Plan(n, m, tri.F64, 0)
+    p2.variant = SPLIT
     p2.k = 3
     torch.cuda.synchronize()
     x1, x2 = torch.empty_like(b), torch.empty_like(b)
@@ -452,10 +453,10 @@ def test_scan_edges_and_scaling(cuda_ok, n, m):
 
 def test_scan_rejects_unsupported(cuda_ok):
     for (n, m, dt, layout) in [(1004, 3, tri.F64, 0), (16384, 3, tri.F64, 1), (7, 3, tri.F32, 0),
-                               ((1 << 20) + 8, 1, tri.F64, 0)]:
+                               ((1 << 20) + 8, 1, tri.F64, 0), (100, 6, tri.F32, 1)]:
         plan = tri.Plan(n, m, dt, layout)
         with pytest.raises(tri.TriError):
-            plan.variant = SCAN
+            plan.variant = SCAN  # n % 8; interleaved row stride not a 16-byte multiple; > 4096 windows
 
 
 @pytest.mark.parametrize("dtype,n,m", [("f64", 16384, 16384), ("f32", 256, 1 << 20)])
@@ -471,6 +472,27 @@ def test_scan_full_size_sampled(cuda_ok, dtype, n, m):
         sl = slice(q * n, (q + 1) * n)
         sub = [t[sl] for t in arrs]
         check_parity(n, 1, sub, x[sl], dtype, 0)
+
+
+@pytest.mark.parametrize("dtype", ["f64", "f32"])
+@pytest.mark.parametrize("n,m", [(1, 8), (5, 12), (200, 64), (1024, 1024), (1000, 36), (333, 300), (4099, 148),
+                                 (16384, 40), (70000, 4)])
+def test_scan_interleaved_parity(cuda_ok, dtype, n, m):
+    """SCAN on the INTERLEAVED layout (S adjacent systems per window, scans over
+    32 / S lane segments): ragged rows and ragged last group of systems, one-row
+    systems, c2's shape, NC from 1 to 1094 windows."""
+    arrs = gen(n, m, dtype, 1)
+    x, plan = gpu_solve(n, m, arrs, dtype, 1, variant=SCAN)
+    assert plan.variant == SCAN and plan.k == 0
+    check_parity(n, m, arrs, x, dtype, 1)
+
+
+@pytest.mark.parametrize("family,eps", [("weak", 1e-3), ("integer", 0.0)])
+def test_scan_interleaved_families(cuda_ok, family, eps):
+    n, m = 5000, 64
+    arrs = gen(n, m, "f64", 1, family, eps=eps)
+    x, _ = gpu_solve(n, m, arrs, "f64", 1, variant=SCAN)
+    check_parity(n, m, arrs, x, "f64", 1)
 
 
 # ------------------------------------------------------------------ SCAN_MC variant
