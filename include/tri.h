@@ -109,9 +109,12 @@ TRI_API tri_status tri_solve(tri_plan_t plan, const void* a, const void* b, cons
                      void* x, void* stream);
 
 /* End-to-end solve through HOST buffers: copies a, b, c, d host->device into
- * plan-owned staging, solves, copies x device->host, all on `stream`, then
- * synchronises `stream`.  Host buffers should be pinned for full bandwidth.
- * Returns after x is in host memory. */
+ * plan-owned staging, solves, copies x device->host, then synchronises
+ * `stream`.  CONTIGUOUS batches of m >= 32 run as a pipeline of 16 chunks of
+ * systems (H2D of chunk i+1, solve of chunk i and D2H of chunk i-1 overlap, on
+ * plan-owned streams ordered after the caller's prior work on `stream`); other
+ * shapes copy, solve and copy back on `stream`.  Host buffers should be pinned
+ * for full bandwidth.  Returns after x is in host memory. */
 TRI_API tri_status tri_solve_host(tri_plan_t plan, const void* a, const void* b, const void* c,
                           const void* d, void* x, void* stream);
 

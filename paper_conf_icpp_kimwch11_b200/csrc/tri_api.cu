@@ -234,6 +234,12 @@ struct tri_plan_s {
     size_t scratch_bytes;
     void* stage;              // tri_solve_host staging (5 arrays), lazily allocated
     size_t stage_bytes;
+    // tri_solve_host pipeline (CONTIGUOUS, m >= 2): chunks of systems flow
+    // H2D -> solve -> D2H on three streams; sub-plans for the chunk sizes
+    tri_plan_s* sub[2];
+    int64_t sub_m[2];
+    cudaStream_t hs[3];
+    cudaEvent_t ev[3 * 16 + 1];
     const void* seen[8];      // pointers whose device residency was last verified
 };
 
@@ -1001,6 +1007,11 @@ tri_plan_t tri_plan(int64_t n, int64_t m, tri_dtype dtype, tri_layout layout) {
 
 void tri_destroy(tri_plan_t p) {
     if (!p) return;
+    for (int i = 0; i < 2; ++i) tri_destroy(p->sub[i]);
+    for (int i = 0; i < 3; ++i)
+        if (p->hs[i]) cudaStreamDestroy(p->hs[i]);
+    for (auto& e : p->ev)
+        if (e) cudaEventDestroy(e);
     if (p->scratch) cudaFree(p->scratch);
     if (p->stage) cudaFree(p->stage);
     delete p;
@@ -1134,6 +1145,67 @@ tri_status tri_debug_pcr(tri_plan_t p, const void* a, const void* b, const void*
     return e == cudaSuccess ? TRI_OK : TRI_ERR_CUDA;
 }
 
+}  // extern "C"
+
+namespace {
+
+constexpr int HOST_CHUNKS = 16;
+
+// Pipelined end-to-end solve for a CONTIGUOUS batch: HOST_CHUNKS ranges of
+// systems; chunk i's H2D copies (stream 0), solve (stream 1, sub-plan for the
+// chunk size) and x D2H copy (stream 2) overlap the other chunks' (PCIe is full
+// duplex; each chunk's staging region is its own, so no buffer is reused).
+tri_status solve_host_pipelined(tri_plan_s* p, const void* const hv[4], void* x, char* const dv[5],
+                                cudaStream_t us) {
+    const size_t es = esize(p->dtype);
+    const int64_t n = p->n, m = p->m;
+    const int64_t mc = cdiv(m, HOST_CHUNKS);
+    const int nch = (int)cdiv(m, mc);
+    for (int i = 0; i < 3; ++i)
+        if (!p->hs[i] && cudaStreamCreateWithFlags(&p->hs[i], cudaStreamNonBlocking) != cudaSuccess) return TRI_ERR_CUDA;
+    for (auto& e : p->ev)
+        if (!e && cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) return TRI_ERR_CUDA;
+    const int64_t sizes[2] = {mc, m - (int64_t)(nch - 1) * mc};
+    for (int i = 0; i < 2; ++i) {
+        if (p->sub[i] && p->sub_m[i] == sizes[i]) continue;
+        tri_destroy(p->sub[i]);
+        p->sub[i] = tri_plan(n, sizes[i], p->dtype, p->layout);
+        p->sub_m[i] = sizes[i];
+        if (!p->sub[i]) return tri_last_status();
+    }
+    cudaEvent_t* evH = p->ev;
+    cudaEvent_t* evC = p->ev + HOST_CHUNKS;
+    cudaEvent_t* evD = p->ev + 2 * HOST_CHUNKS;
+    cudaEvent_t evU = p->ev[3 * HOST_CHUNKS];
+    if (cudaEventRecord(evU, us) != cudaSuccess) return TRI_ERR_CUDA;  // after the caller's prior work
+    if (cudaStreamWaitEvent(p->hs[0], evU, 0) != cudaSuccess) return TRI_ERR_CUDA;
+    for (int i = 0; i < nch; ++i) {
+        const int64_t q0 = (int64_t)i * mc, mi = i + 1 < nch ? mc : sizes[1];
+        const size_t off = (size_t)(q0 * n) * es, bytes = (size_t)(mi * n) * es;
+        for (int k = 0; k < 4; ++k)
+            if (cudaMemcpyAsync(dv[k] + off, (const char*)hv[k] + off, bytes, cudaMemcpyHostToDevice, p->hs[0]) !=
+                cudaSuccess)
+                return TRI_ERR_CUDA;
+        cudaEventRecord(evH[i], p->hs[0]);
+        cudaStreamWaitEvent(p->hs[1], evH[i], 0);
+        const tri_status st = tri_solve(p->sub[i + 1 < nch ? 0 : 1], dv[0] + off, dv[1] + off, dv[2] + off,
+                                        dv[3] + off, dv[4] + off, p->hs[1]);
+        if (st != TRI_OK) return st;
+        cudaEventRecord(evC[i], p->hs[1]);
+        cudaStreamWaitEvent(p->hs[2], evC[i], 0);
+        if (cudaMemcpyAsync((char*)x + off, dv[4] + off, bytes, cudaMemcpyDeviceToHost, p->hs[2]) != cudaSuccess)
+            return TRI_ERR_CUDA;
+        cudaEventRecord(evD[i], p->hs[2]);
+    }
+    if (cudaStreamWaitEvent(us, evD[nch - 1], 0) != cudaSuccess) return TRI_ERR_CUDA;
+    if (cudaStreamSynchronize(us) != cudaSuccess) return TRI_ERR_CUDA;
+    return TRI_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
 tri_status tri_solve_host(tri_plan_t p, const void* a, const void* b, const void* c, const void* d, void* x,
                           void* stream) {
     if (!p || !a || !b || !c || !d || !x) return TRI_ERR_INVALID_ARG;
@@ -1151,6 +1223,10 @@ tri_status tri_solve_host(tri_plan_t p, const void* a, const void* b, const void
     void* dv[5] = {base, base + slot, base + 2 * slot, base + 3 * slot, base + 4 * slot};
     const void* hv[4] = {a, b, c, d};
     cudaStream_t s = (cudaStream_t)stream;
+    if (p->layout == TRI_LAYOUT_CONTIGUOUS && p->m >= 2 * HOST_CHUNKS) {
+        char* const dc[5] = {(char*)dv[0], (char*)dv[1], (char*)dv[2], (char*)dv[3], (char*)dv[4]};
+        return solve_host_pipelined(p, hv, x, dc, s);
+    }
     for (int i = 0; i < 4; ++i)
         if (cudaMemcpyAsync(dv[i], hv[i], bytes, cudaMemcpyHostToDevice, s) != cudaSuccess) return TRI_ERR_CUDA;
     tri_status st = tri_solve(p, dv[0], dv[1], dv[2], dv[3], dv[4], stream);

@@ -230,15 +230,21 @@ def test_concurrent_plans_two_streams(cuda_ok):
         assert np.max(np.abs(x.cpu().numpy() - xo) / np.abs(xo)) <= 1e-10
 
 
-def test_solve_host(cuda_ok):
+@pytest.mark.parametrize("dtype,n,m,layout", [("f64", 4096, 16, 0), ("f64", 2048, 1000, 0), ("f32", 256, 5003, 0),
+                                              ("f64", 1024, 1024, 1), ("f64", 16384, 33, 0)])
+def test_solve_host(cuda_ok, dtype, n, m, layout):
+    """tri_solve_host: one staged copy-solve-copy (small m, interleaved) and the
+    pipelined chunked path (contiguous, m >= 32: 16 chunks of systems, ragged last
+    chunk, two sub-plan sizes), reused twice on the same plan."""
     import torch
-    n, m = 4096, 16
-    arrs = gen(n, m, "f64", 0)
-    plan = tri.Plan(n, m, tri.F64, 0)
+    arrs = gen(n, m, dtype, layout)
+    plan = tri.Plan(n, m, tri.F64 if dtype == "f64" else tri.F32, layout)
     pin = [torch.from_numpy(t).pin_memory() for t in arrs]
-    out = torch.empty(n * m, dtype=torch.float64).pin_memory()
-    plan.solve_host(*pin, out)
-    check_parity(n, m, arrs, out.numpy(), "f64", 0)
+    out = torch.empty(n * m, dtype=pin[0].dtype).pin_memory()
+    for _ in range(2):
+        out.zero_()
+        plan.solve_host(*pin, out)
+        check_parity(n, m, arrs, out.numpy(), dtype, layout)
 
 
 # ------------------------------------------------------------------ FUSED variant
