@@ -45,7 +45,18 @@ constexpr int SC_W = 32 * SC_R;    // rows per window (256)
 constexpr int SC_NW = SC_NW_DEF;   // warps per CTA
 static_assert(SC_NW <= 15, "chain handover uses named barriers 1 .. NW");
 constexpr int SC_THREADS = 32 * SC_NW;
-constexpr int SC_NCMAX = 4096;     // windows per system (per-slot counters live in smem)
+constexpr int SC_NCMAX = 4096;
+// When a warp refills its staging buffer (measured on B200: fewer bytes in flight
+// per SM can be faster -- the DRAM sees fewer interleaved streams):
+//   one-window systems: 1 = two buffers per warp (c4 fp32 1073 us), 0 = refill
+//   after the read (fp32 c4: 983 us, fp64 n = 256: 1763 us), -1 = after the
+//   solve (fp32: 1071 us; fp64: 1654 us);  default: fp32 0, fp64 -1.
+#ifndef SC_DB
+#define SC_DB 2                    // 2 = the per-dtype default above
+#endif
+#ifndef SC_LATE
+#define SC_LATE 0                  // chained windows: 1 = refill at the end of the step
+#endif     // windows per system (per-slot counters live in smem)
 
 template <typename T>
 struct ScanArgs {
@@ -69,8 +80,8 @@ struct SCLayout {
     static constexpr int off_in = 0;
     static constexpr int off_st = off_in + SC_NW * in_stride;             // [NW][<= 8 systems][theta|psi|delta]
     static constexpr int off_xh = off_st + SC_NW * 8 * 4 * (int)sizeof(T);    // [NW][<= 8 systems] x handover
-    static constexpr int off_bar = (off_xh + SC_NW * 8 * (int)sizeof(T) + 7) / 8 * 8;  // [NW] in_full
-    static constexpr int off_cnt = off_bar + SC_NW * 8;                   // [NC] windows-stored counters
+    static constexpr int off_bar = (off_xh + SC_NW * 8 * (int)sizeof(T) + 7) / 8 * 8;  // [2][NW] in_full
+    static constexpr int off_cnt = off_bar + 2 * SC_NW * 8;               // [NC] windows-stored counters
     // [K][NC] u16: slot of window (j, w) at row j % K, K = 3 + (delta - 1) / NC
     // systems in flight between a window's store and its read-back (<= 3 NC + delta entries)
     static __host__ __device__ constexpr int off_tab(int NC) { return off_cnt + 4 * NC; }
@@ -360,7 +371,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     if (threadIdx.x == 0) {
-        for (int i = 0; i < SC_NW; ++i) sk_bar_init(&in_full[i], 1);
+        for (int i = 0; i < 2 * SC_NW; ++i) sk_bar_init(&in_full[i], 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
     }
@@ -375,36 +386,46 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
     T* ib = reinterpret_cast<T*>(sbase + L::off_in + pw * L::in_stride);
     const uint64_t pol_in = sk_policy_evict_first();
     const uint64_t pol_sp = sk_policy_evict_last();
-    auto issue = [&](int jj, int ww) {
+    auto issue_to = [&](int jj, int ww, T* buf, uint64_t* bar) {
         const int q = (int)(blockIdx.x + (int64_t)jj * gridDim.x);
-        sk_expect(&in_full[pw], (unsigned)(4 * SC_W * sizeof(T)));
+        sk_expect(bar, (unsigned)(4 * SC_W * sizeof(T)));
         if constexpr (S == 1) {
             const int y = ww * (SC_W / 8);
-            sc_tma3d(ib + 0 * SC_W, &tm.a, y, q, &in_full[pw], pol_in);
-            sc_tma3d(ib + 1 * SC_W, &tm.b, y, q, &in_full[pw], pol_in);
-            sc_tma3d(ib + 2 * SC_W, &tm.c, y, q, &in_full[pw], pol_in);
-            sc_tma3d(ib + 3 * SC_W, &tm.d, y, q, &in_full[pw], pol_in);
+            sc_tma3d(buf + 0 * SC_W, &tm.a, y, q, bar, pol_in);
+            sc_tma3d(buf + 1 * SC_W, &tm.b, y, q, bar, pol_in);
+            sc_tma3d(buf + 2 * SC_W, &tm.c, y, q, bar, pol_in);
+            sc_tma3d(buf + 3 * SC_W, &tm.d, y, q, bar, pol_in);
         } else {  // tensor [n][m], box [WR][S]
             const int y = ww * WR, xq = q * S;
-            sk_tma2d(ib + 0 * SC_W, &tm.a, xq, y, &in_full[pw], pol_in);
-            sk_tma2d(ib + 1 * SC_W, &tm.b, xq, y, &in_full[pw], pol_in);
-            sk_tma2d(ib + 2 * SC_W, &tm.c, xq, y, &in_full[pw], pol_in);
-            sk_tma2d(ib + 3 * SC_W, &tm.d, xq, y, &in_full[pw], pol_in);
+            sk_tma2d(buf + 0 * SC_W, &tm.a, xq, y, bar, pol_in);
+            sk_tma2d(buf + 1 * SC_W, &tm.b, xq, y, bar, pol_in);
+            sk_tma2d(buf + 2 * SC_W, &tm.c, xq, y, bar, pol_in);
+            sk_tma2d(buf + 3 * SC_W, &tm.d, xq, y, bar, pol_in);
         }
     };
+    auto issue = [&](int jj, int ww) { issue_to(jj, ww, ib, &in_full[pw]); };
     unsigned ph = 0;
 
     if (S == 1 && NC == 1) {
-        // ---- systems of one window: each warp solves whole systems, no chain
-        if (lane == 0 && pw < nsys) issue(pw, 0);
-        for (int j = pw; j < nsys; j += SC_NW) {
+        // ---- systems of one window: each warp solves whole systems, no chain;
+        // two staging buffers per warp (the second in the unused slot area), so
+        // two systems' loads are in flight per warp
+        T* const bufs[2] = {ib, reinterpret_cast<T*>(sbase + L::off_store(NC, p.delta) + pw * L::in_stride)};
+        uint64_t* const bars[2] = {&in_full[pw], &in_full[SC_NW + pw]};
+        unsigned phs = 0;  // bit b: phase of buffer b
+        constexpr int DB = SC_DB == 2 ? (sizeof(T) == 8 ? -1 : 0) : SC_DB;
+        constexpr int NB = DB == 1 ? 2 : 1;
+        if (lane == 0 && pw < nsys) issue_to(pw, 0, bufs[0], bars[0]);
+        if (NB == 2 && lane == 0 && pw + SC_NW < nsys) issue_to(pw + SC_NW, 0, bufs[1], bars[1]);
+        for (int j = pw, it = 0; j < nsys; j += SC_NW, ++it) {
             const int64_t q = blockIdx.x + (int64_t)j * gridDim.x;
+            const int bsel = NB == 2 ? (it & 1) : 0;
             T ra[SC_R], rb[SC_R], rc[SC_R], rd[SC_R];
-            sk_wait(&in_full[pw], ph);
-            ph ^= 1u;
-            sc_ld_rows(ib, lane, ra, rb, rc, rd);
+            sk_wait(bars[bsel], (phs >> bsel) & 1u);
+            phs ^= 1u << bsel;
+            sc_ld_rows(bufs[bsel], lane, ra, rb, rc, rd);
             sc_release_buf();  // this warp's reads of the buffer before the TMA refill
-            if (lane == 0 && j + SC_NW < nsys) issue(j + SC_NW, 0);
+            if (DB >= 0 && lane == 0 && j + NB * SC_NW < nsys) issue_to(j + NB * SC_NW, 0, bufs[bsel], bars[bsel]);
             sc_fix_rows<T>((int64_t)lane * SC_R, n, ra, rb, rc, rd);
             SKMat<T> M = sc_fwd_map(ra, rb, rc, rd);
             sc_fwd_scan(M, lane);
@@ -427,6 +448,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
                 xv[t] = x;
             }
             sc_store_x(p.x + q * n + lane * SC_R, n - (int64_t)lane * SC_R, xv);
+            if (DB < 0 && lane == 0 && j + SC_NW < nsys) issue_to(j + SC_NW, 0, bufs[0], bars[0]);
         }
         return;
     }
@@ -571,7 +593,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
             load_rows(ra, rb, rc, rd);
             if (edge) fix_rows(ra, rb, rc, rd);
             sc_release_buf();  // this warp's reads of the buffer before the TMA refill
-            if (lane == 0 && g + SC_NW < nfwd) issue(j, w);
+            if (!SC_LATE && lane == 0 && g + SC_NW < nfwd) issue(j, w);
             T cpf[SC_R], dpf[SC_R];
             sc_fwd_replay(ra, rb, rc, rd, th, ps, de, cpf, dpf);
             if (res) sc_store_slot_s(sp_s, lane, cpf, dpf);
@@ -603,6 +625,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
                 }
             }
         }
+        if (SC_LATE && fwd && lane == 0 && g + SC_NW < nfwd) issue(j, w);
         SC_T(6);
     }
     if (PROF && lane == 0) {
@@ -610,6 +633,84 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
         for (int k = 0; k < 8; ++k) atomicAdd(&p.prof[k], pc[k]);
     }
 #undef SC_T
+}
+
+// One-window systems (n <= 256, CONTIGUOUS): every warp solves whole systems on
+// its own (no chain, no storage slots), so the CTA holds more warps than the
+// chained kernel (whose named-barrier chain caps it at 15) -- the solve of one
+// system is a latency chain (map, 5-level scans, replays), hidden by warps.
+#ifndef SC1_NW_F64
+#define SC1_NW_F64 16
+#endif
+#ifndef SC1_NW_F32
+#define SC1_NW_F32 20
+#endif
+template <typename T>
+struct SC1 {
+    static constexpr int NW = sizeof(T) == 8 ? SC1_NW_F64 : SC1_NW_F32;
+    static constexpr int in_stride = (4 * SC_W * (int)sizeof(T) + 1023) / 1024 * 1024;
+    static constexpr int off_bar = NW * in_stride;
+    static constexpr int smem_bytes = off_bar + NW * 8 + 1024;
+};
+
+template <typename T>
+__global__ void __launch_bounds__(SC1<T>::NW * 32, 1) k_scan1(const __grid_constant__ StreamMaps tm, ScanArgs<T> p) {
+    constexpr int NW = SC1<T>::NW;
+    extern __shared__ __align__(16) unsigned char sc1_smem_raw[];
+    unsigned char* sbase = sc1_smem_raw + ((1024 - ((unsigned)__cvta_generic_to_shared(sc1_smem_raw) & 1023)) & 1023);
+    uint64_t* in_full = reinterpret_cast<uint64_t*>(sbase + SC1<T>::off_bar);
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, pw = warp;
+    if (threadIdx.x == 0) {
+        for (int i = 0; i < NW; ++i) sk_bar_init(&in_full[i], 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    }
+    __syncthreads();
+    const int64_t n = p.n;
+    const int64_t nsys = (p.m - blockIdx.x + gridDim.x - 1) / gridDim.x;
+    T* ib = reinterpret_cast<T*>(sbase + pw * SC1<T>::in_stride);
+    const uint64_t pol_in = sk_policy_evict_first();
+    auto issue = [&](int64_t jj) {
+        const int q = (int)(blockIdx.x + jj * gridDim.x);
+        sk_expect(&in_full[pw], (unsigned)(4 * SC_W * sizeof(T)));
+        sc_tma3d(ib + 0 * SC_W, &tm.a, 0, q, &in_full[pw], pol_in);
+        sc_tma3d(ib + 1 * SC_W, &tm.b, 0, q, &in_full[pw], pol_in);
+        sc_tma3d(ib + 2 * SC_W, &tm.c, 0, q, &in_full[pw], pol_in);
+        sc_tma3d(ib + 3 * SC_W, &tm.d, 0, q, &in_full[pw], pol_in);
+    };
+    constexpr bool late = sizeof(T) == 8;  // refill after the solve (fp64) or after the read (fp32): SC_DB
+    unsigned ph = 0;
+    if (lane == 0 && pw < nsys) issue(pw);
+    for (int64_t j = pw; j < nsys; j += NW) {
+        const int64_t q = blockIdx.x + j * gridDim.x;
+        T ra[SC_R], rb[SC_R], rc[SC_R], rd[SC_R];
+        sk_wait(&in_full[pw], ph);
+        ph ^= 1u;
+        sc_ld_rows(ib, lane, ra, rb, rc, rd);
+        sc_release_buf();  // this warp's reads of the buffer before the TMA refill
+        if (!late && lane == 0 && j + NW < nsys) issue(j + NW);
+        sc_fix_rows<T>((int64_t)lane * SC_R, n, ra, rb, rc, rd);
+        SKMat<T> M = sc_fwd_map(ra, rb, rc, rd);
+        sc_fwd_scan(M, lane);
+        T th = __shfl_up_sync(0xffffffffu, M.a, 1), ps = __shfl_up_sync(0xffffffffu, M.c, 1),
+          de = __shfl_up_sync(0xffffffffu, M.e, 1);
+        if (lane == 0) { th = T(1); ps = T(0); de = T(0); }
+        T cp[SC_R], dp[SC_R];
+        sc_fwd_replay(ra, rb, rc, rd, th, ps, de, cp, dp);
+        T al, be;
+        sc_bwd_map(cp, dp, al, be);
+        sc_bwd_scan(al, be, lane);
+        T x = __shfl_down_sync(0xffffffffu, al, 1);
+        if (lane == 31) x = T(0);
+        T xv[SC_R];
+#pragma unroll
+        for (int t = SC_R - 1; t >= 0; --t) {
+            x = fma(-cp[t], x, dp[t]);
+            xv[t] = x;
+        }
+        sc_store_x(p.x + q * n + lane * SC_R, n - (int64_t)lane * SC_R, xv);
+        if (late && lane == 0 && j + NW < nsys) issue(j + NW);
+    }
 }
 
 }  // namespace tri

@@ -40,6 +40,7 @@ int g_tiled_waves1 = env_int("TRI_TILED_WAVES1", 1);
 int g_split_k1max = std::min(10, env_int("TRI_SPLIT_K1MAX", 10));  // steps kept in pass 1 (tuning)
 int g_tiled_waves2 = env_int("TRI_TILED_WAVES2", 3);  // measured best at c3 (1 / 3 waves)
 int g_scan_delta = env_int("TRI_SCAN_DELTA", 8);      // SCAN: back-substitution lag in steps (tuning)
+int g_scan1 = getenv("TRI_SCAN1_OFF") ? 0 : 1;        // SCAN, one-window systems: chain-free kernel (A/B)
 
 constexpr int ONCHIP_THREADS = 512;
 constexpr int SPLIT_K1MAX = 10;  // deepest k one sliding-window pass holds in smem (T = 256)
@@ -714,7 +715,20 @@ cudaError_t launch_scan(const tri_plan_s* p, const void* a, const void* b, const
     A.n = p->n; A.m = p->m; A.NC = p->sk_nc; A.S_on = p->sk_son; A.delta = p->sk_delta;
     A.prof = (unsigned long long*)g_fused_prof;
     A.dbg = g_fused_dbg_mode;
-    const size_t smem = (size_t)SCLayout<T>::smem_bytes(p->sk_nc, p->sk_delta, p->sk_son);
+    // one-window systems shorter than 3/4 of a window (many idle rows: compute-heavy)
+    // run the chain-free kernel with more warps (fp32 n = 128: 1.19 ms vs 1.50 ms
+    // per 2^28 rows); at n = 256 the 12-warp kernel is faster (c4: 0.99 vs 1.02 ms)
+    if (S == 1 && p->sk_nc == 1 && g_scan1 && p->n <= 3 * SC_W / 4) {
+        cudaError_t e = cudaFuncSetAttribute(k_scan1<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, SC1<T>::smem_bytes);
+        if (e != cudaSuccess) return e;
+        k_scan1<T><<<p->sk_grid, SC1<T>::NW * 32, SC1<T>::smem_bytes, st>>>(tm, A);
+        return cudaGetLastError();
+    }
+    // one-window systems (S = 1): the slot area holds the warps' second staging buffers
+    const int son_or_buf = (p->sk_S == 1 && p->sk_nc == 1)
+                               ? (SC_NW * SCLayout<T>::in_stride + SCLayout<T>::slot_bytes - 1) / SCLayout<T>::slot_bytes
+                               : p->sk_son;
+    const size_t smem = (size_t)SCLayout<T>::smem_bytes(p->sk_nc, p->sk_delta, son_or_buf);
     const bool pr = A.prof != nullptr;
     void* kern = S == 1 ? scan_kernel<T, 1>(pr) : S == 2 ? scan_kernel<T, 2>(pr) : S == 4 ? scan_kernel<T, 4>(pr)
                                                                                  : scan_kernel<T, 8>(pr);

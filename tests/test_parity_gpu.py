@@ -405,7 +405,7 @@ SCAN = tri.VARIANT_SCAN
 
 
 @pytest.mark.parametrize("dtype", ["f64", "f32"])
-@pytest.mark.parametrize("n,m", [(8, 5), (248, 300), (256, 1000), (264, 3), (512, 7), (1936, 2), (2048, 5),
+@pytest.mark.parametrize("n,m", [(8, 5), (128, 3000), (192, 40), (248, 300), (256, 1000), (264, 3), (512, 7), (1936, 2), (2048, 5),
                                  (4104, 2), (16384, 7), (16392, 150), (2400, 300), (6000, 149), (100000, 2),
                                  (245760, 2), (1 << 20, 1)])
 def test_scan_parity(cuda_ok, dtype, n, m):
