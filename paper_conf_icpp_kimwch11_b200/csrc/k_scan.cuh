@@ -173,20 +173,40 @@ __device__ __forceinline__ void sc_fix_rows(int64_t i0, int64_t n, T (&ra)[SC_R]
     }
 }
 
+// fp32 rows are scaled by 2^-e (e = exponent of b; exact, a row operation that
+// leaves c', d' unchanged, reading X21) before they enter the continuant, so the
+// product of 8 rows cannot overflow fp32's range (|b| up to 2^126 instead of
+// ~2^16); fp64 uses the rows as given (8-row products overflow only beyond
+// |b| ~ 2^127, X21).
+template <typename T>
+__device__ __forceinline__ void sc_row(const T (&ra)[SC_R], const T (&rb)[SC_R], const T (&rc)[SC_R],
+                                       const T (&rd)[SC_R], int u, T& a, T& b, T& c, T& d) {
+    if constexpr (sizeof(T) == 4) {
+        const T s = sk_exp2_scale(rb[u]);
+        a = ra[u] * s; b = rb[u] * s; c = rc[u] * s; d = rd[u] * s;
+    } else {
+        a = ra[u]; b = rb[u]; c = rc[u]; d = rd[u];
+    }
+}
+
 // segment map of the lane's rows (forward state transfer, X21),
 // rescaled by an exact power of two
 template <typename T>
 __device__ __forceinline__ SKMat<T> sc_fwd_map(const T (&ra)[SC_R], const T (&rb)[SC_R], const T (&rc)[SC_R],
                                                const T (&rd)[SC_R]) {
+    T a0, b0, c0, d0;
+    sc_row(ra, rb, rc, rd, 0, a0, b0, c0, d0);
     // row 0 applied to the identity
-    T t1 = rb[0], p1 = rc[0], d1 = rd[0];      // response to theta_in
-    T t2 = -ra[0], p2 = T(0), d2 = T(0);       // ... to psi_in
-    T d3 = -ra[0];                             // ... to delta_in
+    T t1 = b0, p1 = c0, d1 = d0;      // response to theta_in
+    T t2 = -a0, p2 = T(0), d2 = T(0);  // ... to psi_in
+    T d3 = -a0;                        // ... to delta_in
 #pragma unroll
     for (int u = 1; u < SC_R; ++u) {
-        const T nt1 = fma(rb[u], t1, -ra[u] * p1), np1 = rc[u] * t1, nd1 = fma(rd[u], t1, -ra[u] * d1);
-        const T nt2 = fma(rb[u], t2, -ra[u] * p2), np2 = rc[u] * t2, nd2 = fma(rd[u], t2, -ra[u] * d2);
-        d3 = -ra[u] * d3;
+        T au, bu, cu, du;
+        sc_row(ra, rb, rc, rd, u, au, bu, cu, du);
+        const T nt1 = fma(bu, t1, -au * p1), np1 = cu * t1, nd1 = fma(du, t1, -au * d1);
+        const T nt2 = fma(bu, t2, -au * p2), np2 = cu * t2, nd2 = fma(du, t2, -au * d2);
+        d3 = -au * d3;
         t1 = nt1; p1 = np1; d1 = nd1;
         t2 = nt2; p2 = np2; d2 = nd2;
     }
@@ -246,9 +266,11 @@ __device__ __forceinline__ void sc_fwd_replay(const T (&ra)[SC_R], const T (&rb)
                                               const T (&rd)[SC_R], T th, T ps, T de, T (&cp)[SC_R], T (&dp)[SC_R]) {
 #pragma unroll
     for (int u = 0; u < SC_R; ++u) {
-        const T nt = fma(rb[u], th, -ra[u] * ps);
-        const T np = rc[u] * th;
-        const T nd = fma(rd[u], th, -ra[u] * de);
+        T au, bu, cu, du;
+        sc_row(ra, rb, rc, rd, u, au, bu, cu, du);
+        const T nt = fma(bu, th, -au * ps);
+        const T np = cu * th;
+        const T nd = fma(du, th, -au * de);
         const T inv = rcp(nt);
         cp[u] = np * inv;
         dp[u] = nd * inv;

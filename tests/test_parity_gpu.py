@@ -501,6 +501,21 @@ def test_scan_interleaved_families(cuda_ok, family, eps):
     check_parity(n, m, arrs, x, "f64", 1)
 
 
+@pytest.mark.parametrize("dtype,emax", [("f32", 40), ("f64", 100)])
+@pytest.mark.parametrize("n,m,layout,variant", [(256, 300, 0, "SCAN"), (4096, 200, 0, "SCAN"),
+                                                 (100000, 2, 0, "SCAN_MC"), (1024, 512, 1, "SCAN")])
+def test_scan_row_scale_range(cuda_ok, dtype, emax, n, m, layout, variant):
+    """Rows scaled by random powers of two up to 2^+-emax (exact: x unchanged;
+    reading X21): the continuant of 8 raw fp32 rows would leave fp32's range
+    beyond |b| ~ 2^16, so fp32 rows are renormalised in the kernel; fp64 keeps
+    the rows as given within the documented range."""
+    a, b, c, d = gen(n, m, "f64", layout)
+    p = 2.0 ** np.random.default_rng(5).integers(-emax, emax + 1, n * m)
+    arrs = [(t * p).astype(np.float32 if dtype == "f32" else np.float64) for t in (a, b, c, d)]
+    x, plan = gpu_solve(n, m, arrs, dtype, layout, variant=getattr(tri, "VARIANT_" + variant))
+    check_parity(n, m, arrs, x, dtype, layout, resid=False)
+
+
 # ------------------------------------------------------------------ SCAN_MC variant
 SCAN_MC = tri.VARIANT_SCAN_MC
 
