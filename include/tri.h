@@ -132,6 +132,16 @@ TRI_API tri_status tri_debug_pcr(tri_plan_t plan, const void* a, const void* b, 
  * attribution (results are then wrong).  Process-wide; NULL disables. */
 TRI_API void tri_debug_set_profile(void* dev_counters);
 
+/* Autotune the plan (the paper tunes its transition point once per machine,
+ * P:743): time every feasible (variant, k) for the plan's
+ * shape on the caller's device buffers (same rules as tri_solve; x is
+ * overwritten), `reps` solves each after one warm-up, CUDA events on `stream`,
+ * and keep the fastest in the plan.  Candidates whose scratch cannot be
+ * allocated are skipped.  *best_us (may be NULL) receives the fastest mean
+ * time per solve in microseconds.  Synchronises `stream`. */
+TRI_API tri_status tri_plan_autotune(tri_plan_t plan, const void* a, const void* b, const void* c,
+                                     const void* d, void* x, void* stream, int reps, float* best_us);
+
 /* Release the plan and its scratch.  NULL-safe.  Must not race a solve. */
 TRI_API void tri_destroy(tri_plan_t plan);
 

@@ -63,6 +63,7 @@ def lib():
             "tri_choose_variant": (_I, [_I64, _I64, _I, _I, _I]),
             "tri_shard_range": (None, [_I64, _I, _I, ctypes.POINTER(_I64), ctypes.POINTER(_I64)]),
             "tri_debug_set_profile": (None, [_P]),
+            "tri_plan_autotune": (_I, [_P] * 7 + [_I, ctypes.POINTER(ctypes.c_float)]),
         }
         for name, (res, args) in sig.items():
             fn = getattr(L, name)
@@ -198,6 +199,21 @@ class Plan:
         if st != 0:
             raise TriError(st, "tri_solve_host")
         return out
+
+    def autotune(self, a, b, c, d, out=None, reps=3, stream=None):
+        """tri_plan_autotune: time every feasible (variant, k) on these device
+        tensors and keep the fastest in the plan; returns its time in us."""
+        import torch
+        if out is None:
+            out = torch.empty_like(b)
+        self._check(a, b, c, d, out)
+        s = stream if stream is not None else torch.cuda.current_stream()
+        us = ctypes.c_float(0.0)
+        st = lib().tri_plan_autotune(self._h, a.data_ptr(), b.data_ptr(), c.data_ptr(), d.data_ptr(),
+                                     out.data_ptr(), s.cuda_stream, int(reps), ctypes.byref(us))
+        if st != 0:
+            raise TriError(st, "tri_plan_autotune")
+        return us.value
 
     def debug_pcr(self, a, b, c, d, stream=None):
         """Only the PCR stage: returns the k-step reduced system normalised to

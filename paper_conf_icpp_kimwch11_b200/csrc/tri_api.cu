@@ -1074,6 +1074,48 @@ tri_status tri_plan_set_variant(tri_plan_t p, tri_variant v) {
     return st;
 }
 
+tri_status tri_plan_autotune(tri_plan_t p, const void* a, const void* b, const void* c, const void* d, void* x,
+                             void* stream, int reps, float* best_us) {
+    if (!p || reps < 1) return TRI_ERR_INVALID_ARG;
+    const void* in[4] = {a, b, c, d};
+    const void* out[1] = {x};
+    tri_status st = check_ptrs(p, in, 4, out, 1);
+    if (st != TRI_OK) return st;
+    cudaStream_t s = (cudaStream_t)stream;
+    cudaEvent_t e0, e1;
+    if (cudaEventCreate(&e0) != cudaSuccess) return TRI_ERR_CUDA;
+    if (cudaEventCreate(&e1) != cudaSuccess) { cudaEventDestroy(e0); return TRI_ERR_CUDA; }
+    const tri_variant vs[] = {TRI_VARIANT_SCAN, TRI_VARIANT_SCAN_MC, TRI_VARIANT_STREAM, TRI_VARIANT_FUSED,
+                              TRI_VARIANT_WARP, TRI_VARIANT_ONCHIP, TRI_VARIANT_SPLIT};
+    float best = -1.f;
+    tri_variant bv = p->variant;
+    int bk = p->k;
+    for (tri_variant v : vs) {
+        if (tri_plan_set_variant(p, v) != TRI_OK) { cudaGetLastError(); continue; }
+        const int k0 = kmin_for(v), k1 = kmax_for(v, p->n);
+        for (int k = k0; k <= k1; ++k) {
+            if (tri_plan_set_k(p, k) != TRI_OK) { cudaGetLastError(); continue; }
+            if (tri_solve(p, a, b, c, d, x, stream) != TRI_OK) { cudaGetLastError(); continue; }  // warm-up
+            cudaEventRecord(e0, s);
+            bool ok = true;
+            for (int r = 0; r < reps && ok; ++r) ok = tri_solve(p, a, b, c, d, x, stream) == TRI_OK;
+            cudaEventRecord(e1, s);
+            if (!ok || cudaEventSynchronize(e1) != cudaSuccess) { cudaGetLastError(); continue; }
+            float ms = 0.f;
+            cudaEventElapsedTime(&ms, e0, e1);
+            const float us = ms * 1e3f / reps;
+            if (best < 0.f || us < best) { best = us; bv = v; bk = k; }
+        }
+    }
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    if (best < 0.f) return TRI_ERR_CUDA;
+    st = tri_plan_set_variant(p, bv);
+    if (st == TRI_OK) st = tri_plan_set_k(p, bk);
+    if (best_us) *best_us = best;
+    return st;
+}
+
 void tri_plan_describe(tri_plan_t p, char* buf, int len) {
     if (!buf || len <= 0) return;
     if (!p) { snprintf(buf, len, "null plan"); return; }

@@ -136,3 +136,33 @@ def test_planner_picks_for_baseline_configs(L, cfg, n, m, dtype, layout, variant
     dt = getattr(tri, dtype)
     assert tri.choose_variant(n, m, dt, layout, 148) == getattr(tri, variant), cfg
     assert tri.choose_k(n, m, dt, layout, 148) == k, cfg
+
+
+def test_planner_matches_sweeps(L):
+    """The planner's (variant, k) against the committed B200 sweeps (SURVEY 8(f)
+    NEXT-2; profiles/r01_sweep_scan*.jsonl: every whole-solve variant timed on a
+    grid of the paper's shapes): geometric-mean slowdown vs the fastest measured
+    variant <= 5 %, no shape worse than 1.6x (the worst are few-microsecond
+    solves)."""
+    import glob
+    import json
+    import math
+    ratios = []
+    files = sorted(glob.glob(os.path.join(ROOT, "profiles", "r01_sweep_scan*.jsonl")))
+    assert files
+    for f in files:
+        for line in open(f):
+            r = json.loads(line)
+            dt = tri.F64 if r["dtype"] == "f64" else tri.F32
+            lay = r.get("layout", 0)
+            v = tri.choose_variant(r["n"], r["m"], dt, lay, 148)
+            k = tri.choose_k(r["n"], r["m"], dt, lay, 148)
+            recs = r["all"] + [r["auto"]]
+            mine = [x["us"] for x in recs if x["variant"] == v and (v != tri.VARIANT_SPLIT or x["k"] == k)]
+            if not mine:
+                continue  # planner pick not in that sweep (SCAN_MC postdates it)
+            ratios.append(min(mine) / min(x["us"] for x in recs))
+    assert len(ratios) > 150
+    geo = math.exp(sum(math.log(q) for q in ratios) / len(ratios))
+    assert geo <= 1.05, geo
+    assert max(ratios) <= 1.6, max(ratios)

@@ -516,6 +516,32 @@ def test_scan_row_scale_range(cuda_ok, dtype, emax, n, m, layout, variant):
     check_parity(n, m, arrs, x, dtype, layout, resid=False)
 
 
+@pytest.mark.parametrize("dtype,n,m,layout", [("f64", 2048, 300, 0), ("f32", 1000, 64, 1), ("f64", 4099, 3, 0)])
+def test_autotune(cuda_ok, dtype, n, m, layout):
+    """tri_plan_autotune: the kept (variant, k) is at least
+    as fast as the planner's pick (10 % timing slack) and still meets parity."""
+    import torch
+    arrs = gen(n, m, dtype, layout)
+    a, b, c, d = to_dev(*arrs)
+    plan = tri.Plan(n, m, tri.F64 if dtype == "f64" else tri.F32, layout)
+    x = torch.empty_like(b)
+    s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+
+    def t_solve(p):
+        p.solve(a, b, c, d, out=x)
+        s.record()
+        for _ in range(5):
+            p.solve(a, b, c, d, out=x)
+        e.record()
+        torch.cuda.synchronize()
+        return s.elapsed_time(e) * 1e3 / 5
+
+    t_auto = t_solve(plan)
+    best = plan.autotune(a, b, c, d, out=x, reps=5)
+    assert best > 0 and best <= 1.1 * t_auto + 2.0
+    check_parity(n, m, arrs, plan.solve(a, b, c, d).cpu().numpy(), dtype, layout)
+
+
 # ------------------------------------------------------------------ SCAN_MC variant
 SCAN_MC = tri.VARIANT_SCAN_MC
 
