@@ -46,7 +46,10 @@ typedef enum { TRI_F32 = 0, TRI_F64 = 1 } tri_dtype;
 
 typedef enum {
     TRI_LAYOUT_CONTIGUOUS = 0,  /* element i of system q at [q*n + i] */
-    TRI_LAYOUT_INTERLEAVED = 1  /* element i of system q at [i*m + q] */
+    TRI_LAYOUT_INTERLEAVED = 1, /* element i of system q at [i*m + q] */
+    TRI_LAYOUT_BATCHED = 2      /* nb batches of ms interleaved systems (only through tri_plan_batched):
+                                   element i of system q = b*ms + s at [(b*n + i)*ms + s]; e.g. the
+                                   y-lines of a row-major grid [nb][n][ms] (ADI) */
 } tri_layout;
 
 typedef enum {
@@ -141,6 +144,17 @@ TRI_API void tri_debug_set_profile(void* dev_counters);
  * time per solve in microseconds.  Synchronises `stream`. */
 TRI_API tri_status tri_plan_autotune(tri_plan_t plan, const void* a, const void* b, const void* c,
                                      const void* d, void* x, void* stream, int reps, float* best_us);
+
+/* Plan for the BATCHED layout: nb batches, each an INTERLEAVED block of ms
+ * systems of size n (m = ms * nb systems).  Lines of a 3D row-major grid
+ * [nz][ny][nx] (ADI): along x is CONTIGUOUS (n = nx, m =
+ * ny nz), along z is INTERLEAVED (n = nz, m = nx ny), along y is this layout
+ * (n = ny, ms = nx, nb = nz).  ms = 1 and nb = 1 reduce to CONTIGUOUS /
+ * INTERLEAVED plans.  Otherwise the plan runs the SCAN kernel (k = 0) and needs
+ * ms * sizeof(dtype) to be a multiple of 16 bytes (TMA row stride) and n <=
+ * 131072 (4096 windows of 32 rows); else NULL with TRI_ERR_INVALID_ARG.  The
+ * solve semantics, pointer rules and ownership are those of tri_solve. */
+TRI_API tri_plan_t tri_plan_batched(int64_t n, int64_t ms, int64_t nb, tri_dtype dtype);
 
 /* Release the plan and its scratch.  NULL-safe.  Must not race a solve. */
 TRI_API void tri_destroy(tri_plan_t plan);

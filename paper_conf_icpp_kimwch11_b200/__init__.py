@@ -14,7 +14,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.environ.get("TRI_LIB_PATH", os.path.join(HERE, "libtri.so"))  # override: experiments only
 
 F32, F64 = 0, 1
-CONTIGUOUS, INTERLEAVED = 0, 1
+CONTIGUOUS, INTERLEAVED, BATCHED = 0, 1, 2
 (VARIANT_AUTO, VARIANT_ONCHIP, VARIANT_SPLIT, VARIANT_FUSED, VARIANT_WARP, VARIANT_STREAM, VARIANT_SCAN,
  VARIANT_SCAN_MC) = 0, 1, 2, 3, 4, 5, 6, 7
 VARIANT_NAMES = {1: "onchip", 2: "split", 3: "fused", 4: "warp", 5: "stream", 6: "scan", 7: "scan_mc"}
@@ -44,6 +44,7 @@ def lib():
         L = ctypes.CDLL(LIB_PATH)
         sig = {
             "tri_plan": (_P, [_I64, _I64, _I, _I]),
+            "tri_plan_batched": (_P, [_I64, _I64, _I64, _I]),
             "tri_last_status": (_I, []),
             "tri_solve": (_I, [_P] * 7),
             "tri_solve_host": (_I, [_P] * 7),
@@ -113,17 +114,26 @@ class Plan:
     Wraps tri_plan / tri_solve (include/tri.h).  The plan is bound to the CUDA
     device current at construction and owns its scratch."""
 
-    def __init__(self, n, m, dtype=F64, layout=CONTIGUOUS):
+    def __init__(self, n, m, dtype=F64, layout=CONTIGUOUS, _batch=None):
         import torch
         self.n, self.m = int(n), int(m)
         self.dtype_code = _dtype_code(dtype)
         self.torch_dtype = torch.float64 if self.dtype_code == F64 else torch.float32
         self.layout = int(layout)
-        h = lib().tri_plan(self.n, self.m, self.dtype_code, self.layout)
+        if _batch is None:
+            h = lib().tri_plan(self.n, self.m, self.dtype_code, self.layout)
+        else:
+            h = lib().tri_plan_batched(self.n, _batch[0], _batch[1], self.dtype_code)
         if not h:
             raise TriError(lib().tri_last_status(), "tri_plan")
         self._h = ctypes.c_void_p(h)
         self.device = torch.cuda.current_device()
+
+    @classmethod
+    def batched(cls, n, ms, nb, dtype=F64):
+        """tri_plan_batched: nb batches of ms interleaved systems of size n (the
+        y-lines of a row-major grid [nb][n][ms]; ADI)."""
+        return cls(n, int(ms) * int(nb), dtype, BATCHED, _batch=(int(ms), int(nb)))
 
     def __del__(self):
         h = getattr(self, "_h", None)

@@ -63,6 +63,7 @@ struct ScanArgs {
     T* x;
     T* spill;      // per CTA: (NC + delta - S_on) slots of sc_slot_elems<T>() elements
     int64_t n, m;
+    int64_t ms;    // S > 1 (INTERLEAVED / BATCHED): systems per batch (INTERLEAVED: m, one batch)
     int NC;        // windows per system
     int delta;     // extra lag (steps) of the back substitution behind the forward sweep
     int S_on;      // storage slots resident in shared memory
@@ -81,13 +82,14 @@ struct SCLayout {
     static constexpr int off_st = off_in + SC_NW * in_stride;             // [NW][<= 8 systems][theta|psi|delta]
     static constexpr int off_xh = off_st + SC_NW * 8 * 4 * (int)sizeof(T);    // [NW][<= 8 systems] x handover
     static constexpr int off_bar = (off_xh + SC_NW * 8 * (int)sizeof(T) + 7) / 8 * 8;  // [2][NW] in_full
-    static constexpr int off_cnt = off_bar + 2 * SC_NW * 8;               // [NC] windows-stored counters
-    // [K][NC] u16: slot of window (j, w) at row j % K, K = 3 + (delta - 1) / NC
-    // systems in flight between a window's store and its read-back (<= 3 NC + delta entries)
-    static __host__ __device__ constexpr int off_tab(int NC) { return off_cnt + 4 * NC; }
+    static constexpr int off_cnt = off_bar + 2 * SC_NW * 8;               // the slot table follows
+    // [K][NC] u32: tag(j) << 16 | slot of window (j, w) at row j % K, K = 3 +
+    // (delta - 1) / NC systems in flight between a window's store and its
+    // read-back (<= 3 NC + delta entries)
+    static __host__ __device__ constexpr int off_tab(int NC) { return off_cnt + 0 * NC; }
     static constexpr int slot_bytes = sc_slot_elems<T>() * (int)sizeof(T);
     static __host__ __device__ constexpr int off_store(int NC, int D) {
-        return (off_tab(NC) + 2 * (3 * NC + D) + 1023) / 1024 * 1024;
+        return (off_tab(NC) + 4 * (3 * NC + D) + 1023) / 1024 * 1024;
     }
     static __host__ __device__ constexpr int smem_bytes(int NC, int D, int S_on) {
         return off_store(NC, D) + S_on * slot_bytes + 1024;  // + alignment slack
@@ -103,14 +105,16 @@ __device__ __forceinline__ int sc_chunk(int lane, int ch) {
     return ch * 32 + lane;
 }
 
-// TMA 3D tile load: tensor view [m][n/8][8] (system, 8-row group, row), box
-// [1][32][8] = one 256-row window of one array; rows past the system's end are
-// zero-filled (and replaced by identity rows, sc_fix_rows)
-__device__ __forceinline__ void sc_tma3d(void* dst, const CUtensorMap* tm, int y, int q, uint64_t* bar, uint64_t pol) {
+// TMA 3D tile load.  CONTIGUOUS: tensor view [m][n/8][8] (system, 8-row group,
+// row), box [1][32][8] = one 256-row window of one array (x0 = 0).  INTERLEAVED /
+// BATCHED: tensor [nb][n][ms], box [1][256/S][S].  Rows (systems) past the end
+// are zero-filled (and replaced by identity rows, sc_fix_rows).
+__device__ __forceinline__ void sc_tma3d(void* dst, const CUtensorMap* tm, int y, int q, uint64_t* bar, uint64_t pol,
+                                         int x0 = 0) {
     asm volatile(
         "cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint"
         " [%0], [%1, {%2, %3, %4}], [%5], %6;" ::"r"((unsigned)__cvta_generic_to_shared(dst)),
-        "l"(tm), "r"(0), "r"(y), "r"(q), "r"((unsigned)__cvta_generic_to_shared(bar)), "l"(pol)
+        "l"(tm), "r"(x0), "r"(y), "r"(q), "r"((unsigned)__cvta_generic_to_shared(bar)), "l"(pol)
         : "memory");
 }
 
@@ -384,8 +388,11 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
     extern __shared__ __align__(16) unsigned char sc_smem_raw[];
     unsigned char* sbase = sc_smem_raw + ((1024 - ((unsigned)__cvta_generic_to_shared(sc_smem_raw) & 1023)) & 1023);
     uint64_t* in_full = reinterpret_cast<uint64_t*>(sbase + L::off_bar);  // [NW] TMA -> warp
-    int* cnt = reinterpret_cast<int*>(sbase + L::off_cnt);    // [NC] systems whose window w is stored
-    unsigned short* tab = reinterpret_cast<unsigned short*>(sbase + L::off_tab(p.NC));  // [K][NC] slot of (j, w)
+    // [K][NC] slot table: entry (j % K, w) = tag(j) << 16 | slot of window (j, w),
+    // tag(j) = j % 65535 + 1, published (release) once the window is stored; a
+    // reader waits for its exact tag, so stores completing out of order (groups
+    // j and j + 1 of short systems run concurrently) cannot be mistaken
+    unsigned* tab = reinterpret_cast<unsigned*>(sbase + L::off_tab(p.NC));
     T* stt = reinterpret_cast<T*>(sbase + L::off_st);
     T* xh = reinterpret_cast<T*>(sbase + L::off_xh);
     const int NC = p.NC;
@@ -397,11 +404,14 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
     }
-    for (int i = threadIdx.x; i < NC; i += blockDim.x) cnt[i] = 0;
+    for (int i = threadIdx.x; i < 3 * NC + p.delta; i += blockDim.x) tab[i] = 0u;
     __syncthreads();
 
     const int64_t n = p.n;
-    const int64_t ngrp = (p.m + S - 1) / S;  // groups of S systems (one "system" of the chain)
+    // groups of S adjacent systems (one "system" of the chain); INTERLEAVED /
+    // BATCHED: gpb groups per batch of ms systems, group q = (batch q / gpb, q % gpb)
+    const int64_t gpb = (p.ms + S - 1) / S;
+    const int64_t ngrp = S == 1 ? p.m : gpb * (p.m / p.ms);
     const int nsys = (int)((ngrp - blockIdx.x + gridDim.x - 1) / gridDim.x);
     const int pw = warp;
     const int ls = lane % S, seg = lane / S;
@@ -417,12 +427,12 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
             sc_tma3d(buf + 1 * SC_W, &tm.b, y, q, bar, pol_in);
             sc_tma3d(buf + 2 * SC_W, &tm.c, y, q, bar, pol_in);
             sc_tma3d(buf + 3 * SC_W, &tm.d, y, q, bar, pol_in);
-        } else {  // tensor [n][m], box [WR][S]
-            const int y = ww * WR, xq = q * S;
-            sk_tma2d(buf + 0 * SC_W, &tm.a, xq, y, bar, pol_in);
-            sk_tma2d(buf + 1 * SC_W, &tm.b, xq, y, bar, pol_in);
-            sk_tma2d(buf + 2 * SC_W, &tm.c, xq, y, bar, pol_in);
-            sk_tma2d(buf + 3 * SC_W, &tm.d, xq, y, bar, pol_in);
+        } else {  // tensor [nb][n][ms], box [1][WR][S]
+            const int bt = (int)(q / gpb), xq = (int)(q - bt * gpb) * S, y = ww * WR;
+            sc_tma3d(buf + 0 * SC_W, &tm.a, y, bt, bar, pol_in, xq);
+            sc_tma3d(buf + 1 * SC_W, &tm.b, y, bt, bar, pol_in, xq);
+            sc_tma3d(buf + 2 * SC_W, &tm.c, y, bt, bar, pol_in, xq);
+            sc_tma3d(buf + 3 * SC_W, &tm.d, y, bt, bar, pol_in, xq);
         }
     };
     auto issue = [&](int jj, int ww) { issue_to(jj, ww, ib, &in_full[pw]); };
@@ -506,9 +516,15 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
         int slot = g;                            // fresh slot (g < NS when !bwd)
         if (bwd && p.dbg != 2) {
             SC_T(5);
-            sk_wait_ge(&cnt[wb], bj + 1);  // window (bj, wb) stored
+            const unsigned tg = (unsigned)(bj % 65535 + 1);
+            const int* e = reinterpret_cast<const int*>(&tab[(bj % K) * NC + wb]);
+            unsigned v = (unsigned)sk_ld_acquire(e);
+            while ((v >> 16) != tg) {  // window (bj, wb) stored
+                __nanosleep(64);
+                v = (unsigned)sk_ld_acquire(e);
+            }
             SC_T(4);
-            slot = tab[(bj % K) * NC + wb];
+            slot = (int)(v & 0xffffu);
         }
         const bool res = slot < p.S_on;
         const unsigned sp_s = store_s + (unsigned)(slot * L::slot_bytes);
@@ -543,15 +559,17 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
         // ---- forward: segment map of window (cj, cw) (identity rows when inactive);
         // the rows are read again from the staging buffer for the replay
         const int64_t i0 = (int64_t)cw * WR + seg * SC_R;
-        const int64_t qf = (blockIdx.x + (int64_t)cj * gridDim.x) * S + ls;  // this lane's system
-        const bool edge = cw == 0 || (int64_t)(cw + 1) * WR > n || (S > 1 && qf >= p.m);
+        // this lane's system within its batch (S > 1): padding lanes past ms are identity rows
+        const int64_t gq = blockIdx.x + (int64_t)cj * gridDim.x;
+        const int64_t qf = S > 1 ? (gq - (gq / gpb) * gpb) * S + ls : 0;
+        const bool edge = cw == 0 || (int64_t)(cw + 1) * WR > n || (S > 1 && qf >= p.ms);
         auto load_rows = [&](T (&ra)[SC_R], T (&rb)[SC_R], T (&rc)[SC_R], T (&rd)[SC_R]) {
             if constexpr (S == 1) sc_ld_rows(ib, lane, ra, rb, rc, rd);
             else sc_ld_rows_il<S>(ib, ls, seg, ra, rb, rc, rd);
         };
         auto fix_rows = [&](T (&ra)[SC_R], T (&rb)[SC_R], T (&rc)[SC_R], T (&rd)[SC_R]) {
             sc_fix_rows<T>(i0, n, ra, rb, rc, rd);
-            if (S > 1 && qf >= p.m) {  // padding systems of the last group: identity rows
+            if (S > 1 && qf >= p.ms) {  // padding systems of the last group: identity rows
 #pragma unroll
                 for (int u = 0; u < SC_R; ++u) { ra[u] = T(0); rb[u] = T(1); rc[u] = T(0); rd[u] = T(0); }
             }
@@ -622,8 +640,8 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
             else sc_store_slot_g(sp_g, lane, cpf, dpf, pol_sp);
             __syncwarp();
             if (lane == 0) {
-                tab[(cj % K) * NC + cw] = (unsigned short)slot;
-                sk_st_release(&cnt[cw], cj + 1);
+                sk_st_release(reinterpret_cast<int*>(&tab[(cj % K) * NC + cw]),
+                              (int)(((unsigned)(cj % 65535 + 1) << 16) | (unsigned)slot));
             }
         }
         // ---- backward replay: x (Eq 4) of window (bj, wb)
@@ -638,12 +656,13 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
             const int64_t xr = (int64_t)wb * WR + seg * SC_R;
             if constexpr (S == 1) {
                 sc_store_x(p.x + qb * n + xr, n - xr, xv);
-            } else {  // INTERLEAVED: x[row * m + q]
-                const int64_t qx = qb * S + ls;
-                if (qx < p.m) {
+            } else {  // INTERLEAVED / BATCHED: x[(batch n + row) ms + s]
+                const int64_t bt = qb / gpb, qx = (qb - bt * gpb) * S + ls;
+                if (qx < p.ms) {
+                    T* xo = p.x + bt * n * p.ms + qx;
 #pragma unroll
                     for (int t = 0; t < SC_R; ++t)
-                        if (xr + t < n) __stcs(p.x + (xr + t) * p.m + qx, xv[t]);
+                        if (xr + t < n) __stcs(xo + (xr + t) * p.ms, xv[t]);
                 }
             }
         }

@@ -99,14 +99,19 @@ int g_scan_s_il = env_int("TRI_SCAN_S", 0);  // SCAN, interleaved: systems per w
 // the TMA box's inner extent S * s must be >= 16 bytes)
 int scan_systems(int64_t n, int64_t m, tri_dtype t, tri_layout layout) {
     (void)n; (void)m;
-    if (layout == TRI_LAYOUT_CONTIGUOUS) return 1;
+    if (layout == TRI_LAYOUT_CONTIGUOUS) return 1;  // (BATCHED: like INTERLEAVED)
     // 8: a window's row of S systems is 64 B (fp64) / 32 B (fp32), at least one
     // whole DRAM sector per TMA row (S = 2 fp64 measured 2x slower: half sectors)
     const int smin = t == TRI_F64 ? 2 : 4;
     if (g_scan_s_il == 2 || g_scan_s_il == 4 || g_scan_s_il == 8) return std::max(smin, g_scan_s_il);
     return 8;
 }
-bool scan_ok(int64_t n, int64_t m, tri_dtype t, tri_layout layout) {
+bool scan_ok(int64_t n, int64_t m, tri_dtype t, tri_layout layout, int64_t ms = -1) {
+    if (layout == TRI_LAYOUT_BATCHED) {
+        const int S = scan_systems(n, m, t, layout);
+        return ms > 0 && (ms * (int64_t)esize(t)) % 16 == 0 && cdiv(n, SC_W / S) <= SC_NCMAX &&
+               n < ((int64_t)1 << 31) && ms < ((int64_t)1 << 31) && m / ms < ((int64_t)1 << 31);
+    }
     if (layout == TRI_LAYOUT_CONTIGUOUS || m == 1)
         return n % 8 == 0 && cdiv(n, SC_W) <= SC_NCMAX && n / 8 < ((int64_t)1 << 31) && m < ((int64_t)1 << 31);
     // INTERLEAVED: TMA tensor [n][m], row stride m * s a multiple of 16 bytes
@@ -136,6 +141,7 @@ bool scan_mc_ok(int64_t n, int64_t m, tri_dtype t, tri_layout layout) {
 //   * whole systems that fit a CTA's smem: ONCHIP;
 //   * otherwise (few large systems): SPLIT with k from choose_k_for.
 tri_variant choose_variant(int64_t n, int64_t m, tri_dtype t, tri_layout layout, int sms) {
+    if (layout == TRI_LAYOUT_BATCHED) return TRI_VARIANT_SCAN;  // the only kernel for this layout
     // SCAN (profiles/r01_sweep_scan_*.jsonl): fastest of all variants on every
     // contiguous shape with n % 8 == 0 of the grid n = 256 .. 2^20 x m = 1 .. 2^20
     // (fp64 and fp32), except a few (< 128) systems of more than 64 windows, where
@@ -229,6 +235,7 @@ struct tri_plan_s {
     int sk_grid, sk_nc, sk_son;  // STREAM / SCAN: persistent CTAs, windows per system, resident storage slots
     int sk_delta;                // SCAN: back-substitution lag (steps)
     int sk_S;                    // SCAN: systems per window (1 contiguous; 2 / 4 / 8 interleaved)
+    int64_t ms;                  // systems per batch (BATCHED; m otherwise)
     int mc_P, mc_NCW;            // SCAN_MC: chunks per system, windows per chunk
     size_t smem_optin;
     void* scratch;
@@ -372,10 +379,12 @@ void plan_geometry(tri_plan_s* p) {
     }
     if (p->variant == TRI_VARIANT_SCAN) {
         p->L = n; p->n_pad = n; p->C = m;
-        const bool il = p->layout == TRI_LAYOUT_INTERLEAVED && m > 1;
+        const bool il = (p->layout == TRI_LAYOUT_INTERLEAVED && m > 1) || p->layout == TRI_LAYOUT_BATCHED;
         p->sk_S = il ? scan_systems(n, m, p->dtype, p->layout) : 1;
         p->sk_nc = (int)cdiv(n, SC_W / p->sk_S);
-        p->sk_grid = (int)std::min<int64_t>(cdiv(m, p->sk_S), p->sms);
+        const int64_t ms = p->layout == TRI_LAYOUT_BATCHED ? p->ms : m;
+        const int64_t groups = p->sk_S == 1 ? m : cdiv(ms, p->sk_S) * (m / ms);
+        p->sk_grid = (int)std::min<int64_t>(groups, p->sms);
         p->sk_delta = g_scan_delta;
         const int fixed = p->dtype == TRI_F64 ? SCLayout<double>::smem_bytes(p->sk_nc, p->sk_delta, 0)
                                               : SCLayout<float>::smem_bytes(p->sk_nc, p->sk_delta, 0);
@@ -674,16 +683,17 @@ bool tma_map_sys_rows8(CUtensorMap* tm, const void* base, int64_t n, int64_t m) 
                CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
-// INTERLEAVED: tensor [n][m] (row stride m elements), box [256 / S rows][S systems]
+// INTERLEAVED / BATCHED: tensor [nb][n][ms] (row stride ms elements, batch stride
+// n ms), box [1][256 / S rows][S systems]
 template <typename T>
-bool tma_map_il(CUtensorMap* tm, const void* base, int64_t n, int64_t m, int S) {
+bool tma_map_il(CUtensorMap* tm, const void* base, int64_t n, int64_t ms, int64_t nb, int S) {
     auto enc = tma_encoder();
     if (!enc) return false;
-    cuuint64_t dims[2] = {(cuuint64_t)m, (cuuint64_t)n};
-    cuuint64_t strides[1] = {(cuuint64_t)m * sizeof(T)};
-    cuuint32_t box[2] = {(cuuint32_t)S, (cuuint32_t)(SC_W / S)};
-    cuuint32_t es[2] = {1, 1};
-    return enc(tm, sizeof(T) == 8 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT64 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2,
+    cuuint64_t dims[3] = {(cuuint64_t)ms, (cuuint64_t)n, (cuuint64_t)nb};
+    cuuint64_t strides[2] = {(cuuint64_t)ms * sizeof(T), (cuuint64_t)(n * ms) * sizeof(T)};
+    cuuint32_t box[3] = {(cuuint32_t)S, (cuuint32_t)(SC_W / S), 1};
+    cuuint32_t es[3] = {1, 1, 1};
+    return enc(tm, sizeof(T) == 8 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT64 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3,
                const_cast<void*>(base), dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
                CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
@@ -705,14 +715,15 @@ cudaError_t launch_scan(const tri_plan_s* p, const void* a, const void* b, const
             !tma_map_sys_rows8<T>(&tm.c, c, n, m) || !tma_map_sys_rows8<T>(&tm.d, d, n, m))
             return cudaErrorNotSupported;
     } else {
-        if (!tma_map_il<T>(&tm.a, a, n, m, S) || !tma_map_il<T>(&tm.b, b, n, m, S) ||
-            !tma_map_il<T>(&tm.c, c, n, m, S) || !tma_map_il<T>(&tm.d, d, n, m, S))
+        const int64_t ms = p->ms, nb = m / p->ms;
+        if (!tma_map_il<T>(&tm.a, a, n, ms, nb, S) || !tma_map_il<T>(&tm.b, b, n, ms, nb, S) ||
+            !tma_map_il<T>(&tm.c, c, n, ms, nb, S) || !tma_map_il<T>(&tm.d, d, n, ms, nb, S))
             return cudaErrorNotSupported;
     }
     ScanArgs<T> A;
     A.x = (T*)x;
     A.spill = (T*)p->scratch;
-    A.n = p->n; A.m = p->m; A.NC = p->sk_nc; A.S_on = p->sk_son; A.delta = p->sk_delta;
+    A.n = p->n; A.m = p->m; A.ms = p->ms; A.NC = p->sk_nc; A.S_on = p->sk_son; A.delta = p->sk_delta;
     A.prof = (unsigned long long*)g_fused_prof;
     A.dbg = g_fused_dbg_mode;
     // one-window systems shorter than 3/4 of a window (many idle rows: compute-heavy)
@@ -1007,11 +1018,42 @@ tri_plan_t tri_plan(int64_t n, int64_t m, tri_dtype dtype, tri_layout layout) {
     if (st != TRI_OK) { g_last = st; return nullptr; }
     tri_plan_s* p = new tri_plan_s();
     p->n = n; p->m = m; p->dtype = dtype; p->layout = layout; p->device = dev; p->sms = sms;
+    p->ms = m;
     int optin = 0;
     cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
     p->smem_optin = (size_t)optin;
     p->variant = choose_variant(n, m, dtype, layout, sms);
     p->k = choose_k_for(p->variant, n, m, dtype, layout, sms);
+    plan_geometry(p);
+    st = ensure_scratch(p);
+    if (st != TRI_OK) { delete p; g_last = st; return nullptr; }
+    g_last = TRI_OK;
+    return p;
+}
+
+tri_plan_t tri_plan_batched(int64_t n, int64_t ms, int64_t nb, tri_dtype dtype) {
+    if (n < 1 || ms < 1 || nb < 1 || (dtype != TRI_F32 && dtype != TRI_F64) || ms > MAX_ELEMS / nb ||
+        n > MAX_ELEMS / (ms * nb)) {
+        g_last = TRI_ERR_INVALID_ARG;
+        return nullptr;
+    }
+    if (ms == 1) return tri_plan(n, nb, dtype, TRI_LAYOUT_CONTIGUOUS);  // [(b n + i)]: contiguous systems
+    if (nb == 1) return tri_plan(n, ms, dtype, TRI_LAYOUT_INTERLEAVED);
+    if (!scan_ok(n, ms * nb, dtype, TRI_LAYOUT_BATCHED, ms)) {
+        g_last = TRI_ERR_INVALID_ARG;
+        return nullptr;
+    }
+    int dev = 0, sms = 0;
+    tri_status st = current_device_ok(&dev, &sms);
+    if (st != TRI_OK) { g_last = st; return nullptr; }
+    tri_plan_s* p = new tri_plan_s();
+    p->n = n; p->m = ms * nb; p->dtype = dtype; p->layout = TRI_LAYOUT_BATCHED; p->device = dev; p->sms = sms;
+    p->ms = ms;
+    int optin = 0;
+    cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+    p->smem_optin = (size_t)optin;
+    p->variant = TRI_VARIANT_SCAN;
+    p->k = 0;
     plan_geometry(p);
     st = ensure_scratch(p);
     if (st != TRI_OK) { delete p; g_last = st; return nullptr; }
@@ -1054,6 +1096,8 @@ tri_status tri_plan_set_k(tri_plan_t p, int k) {
 
 tri_status tri_plan_set_variant(tri_plan_t p, tri_variant v) {
     if (!p) return TRI_ERR_INVALID_ARG;
+    if (p->layout == TRI_LAYOUT_BATCHED)  // one kernel for this layout
+        return (v == TRI_VARIANT_AUTO || v == TRI_VARIANT_SCAN) ? TRI_OK : TRI_ERR_INVALID_ARG;
     if (v == TRI_VARIANT_AUTO) v = choose_variant(p->n, p->m, p->dtype, p->layout, p->sms);
     if (v == TRI_VARIANT_ONCHIP && p->n > onchip_rows_budget(p->dtype)) return TRI_ERR_INVALID_ARG;
     if (v == TRI_VARIANT_FUSED && !fused_ok(p->n, p->m, p->layout)) return TRI_ERR_INVALID_ARG;
@@ -1124,7 +1168,8 @@ void tri_plan_describe(tri_plan_t p, char* buf, int len) {
              "n=%lld m=%lld dtype=%s layout=%s variant=%s k=%d G=%d P=%d rpt=%d L=%lld C=%lld region=%lld nreg=%lld "
              "fu_grid=%d fu_son=%d fu_nc=%lld sk_grid=%d sk_nc=%d sk_son=%d scratch=%zu sms=%d",
              (long long)p->n, (long long)p->m, p->dtype == TRI_F64 ? "f64" : "f32",
-             p->layout == TRI_LAYOUT_CONTIGUOUS ? "contiguous" : "interleaved", vn[p->variant], p->k, p->G, p->P,
+             p->layout == TRI_LAYOUT_CONTIGUOUS ? "contiguous" : p->layout == TRI_LAYOUT_INTERLEAVED ? "interleaved" : "batched",
+             vn[p->variant], p->k, p->G, p->P,
              p->rpt, (long long)p->L, (long long)p->C, (long long)p->region, (long long)p->nreg, p->fu_grid, p->fu_son,
              (long long)p->fu_nc, p->sk_grid, p->sk_nc, p->sk_son, p->scratch_bytes, p->sms);
 }

@@ -542,6 +542,40 @@ def test_autotune(cuda_ok, dtype, n, m, layout):
     check_parity(n, m, arrs, plan.solve(a, b, c, d).cpu().numpy(), dtype, layout)
 
 
+def _grid_lines(n, ms, nb, dtype, family="dd"):
+    """Seeded systems for the y-lines of a grid [nb][n][ms]: generated as nb*ms
+    contiguous systems (system q = b*ms + s), returned both ways."""
+    arrs = gen(n, ms * nb, dtype, 0, family)
+    grid = [np.ascontiguousarray(t.reshape(nb, ms, n).transpose(0, 2, 1)).reshape(-1) for t in arrs]
+    return arrs, grid
+
+
+@pytest.mark.parametrize("dtype,n,ms,nb", [("f64", 100, 64, 7), ("f64", 1000, 18, 5), ("f32", 333, 36, 9),
+                                           ("f64", 16, 8, 300), ("f32", 4096, 12, 3), ("f64", 64, 1, 50),
+                                           ("f64", 77, 50, 1)])
+def test_batched_layout_adi_lines(cuda_ok, dtype, n, ms, nb):
+    """TRI_LAYOUT_BATCHED: the y-lines of a row-major grid
+    [nb][n][ms] solved in place, vs the oracle on the same systems laid out
+    contiguously; ragged groups of 8 systems, ms = 1 / nb = 1 reductions."""
+    import torch
+    arrs, grid = _grid_lines(n, ms, nb, dtype)
+    plan = tri.Plan.batched(n, ms, nb, tri.F64 if dtype == "f64" else tri.F32)
+    xg = plan.solve(*to_dev(*grid)).cpu().numpy()
+    x = np.ascontiguousarray(xg.reshape(nb, n, ms).transpose(0, 2, 1)).reshape(-1)
+    check_parity(n, ms * nb, arrs, x, dtype, 0)
+
+
+def test_batched_layout_rejects(cuda_ok):
+    with pytest.raises(tri.TriError):
+        tri.Plan.batched(100, 3, 4, tri.F64)   # row stride 24 B: not a 16-byte multiple
+    with pytest.raises(tri.TriError):
+        tri.Plan.batched(0, 8, 4, tri.F64)
+    p = tri.Plan.batched(100, 8, 4, tri.F64)
+    with pytest.raises(tri.TriError):
+        p.variant = tri.VARIANT_SPLIT            # SCAN is the only kernel for this layout
+    assert p.variant == tri.VARIANT_SCAN and p.k == 0
+
+
 # ------------------------------------------------------------------ SCAN_MC variant
 SCAN_MC = tri.VARIANT_SCAN_MC
 
