@@ -156,6 +156,27 @@ TRI_API tri_status tri_plan_autotune(tri_plan_t plan, const void* a, const void*
  * solve semantics, pointer rules and ownership are those of tri_solve. */
 TRI_API tri_plan_t tri_plan_batched(int64_t n, int64_t ms, int64_t nb, tri_dtype dtype);
 
+/* One system spread over several devices.
+ * Device r holds rows [r0, r0 + n) of the system -- a contiguous slice, n % 8
+ * == 0, n > 256 -- in a plan made with tri_plan(n, 1, dtype, CONTIGUOUS) and
+ * set to TRI_VARIANT_SCAN_MC.  The slice's forward sweep is a 3x3 map of the
+ * incoming continuant state and its back substitution an affine map of the x
+ * after it (X21), so the devices exchange only 8 values each, twice:
+ *   phase 0: a, b, c, d (device, the slice) -> out = the slice's forward map
+ *            (8 values of dtype, device);
+ *   [all-gather the nslices forward maps, in slice order, into `maps`]
+ *   phase 1: a, b, c, d, maps -> out = the slice's backward map (8 values);
+ *   [all-gather the backward maps into `maps`]
+ *   phase 2: maps -> out = x of the slice (n values, device).
+ * The first row of slice r > 0 keeps its a (coupled to slice r - 1) and the
+ * last row of slice r < nslices - 1 keeps its c.  Asynchronous on `stream`;
+ * phases run in order on one plan; the plan's scratch carries c', d' from
+ * phase 1 to phase 2.  TRI_ERR_INVALID_ARG for a plan that is not SCAN_MC with
+ * m == 1, a bad phase / slice, or a NULL pointer. */
+TRI_API tri_status tri_slice_solve(tri_plan_t plan, int phase, int slice, int nslices, const void* a,
+                                   const void* b, const void* c, const void* d, const void* maps, void* out,
+                                   void* stream);
+
 /* Release the plan and its scratch.  NULL-safe.  Must not race a solve. */
 TRI_API void tri_destroy(tri_plan_t plan);
 

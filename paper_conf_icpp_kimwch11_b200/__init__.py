@@ -65,6 +65,7 @@ def lib():
             "tri_shard_range": (None, [_I64, _I, _I, ctypes.POINTER(_I64), ctypes.POINTER(_I64)]),
             "tri_debug_set_profile": (None, [_P]),
             "tri_plan_autotune": (_I, [_P] * 7 + [_I, ctypes.POINTER(ctypes.c_float)]),
+            "tri_slice_solve": (_I, [_P, _I, _I, _I] + [_P] * 7),
         }
         for name, (res, args) in sig.items():
             fn = getattr(L, name)
@@ -224,6 +225,27 @@ class Plan:
         if st != 0:
             raise TriError(st, "tri_plan_autotune")
         return us.value
+
+    def slice_phase(self, phase, slice_, nslices, a=None, b=None, c=None, d=None, maps=None, out=None,
+                    stream=None):
+        """tri_slice_solve (NEXT-4): one phase of the solve of a system spread
+        over devices; this plan (m = 1, SCAN_MC) holds one slice.  Phases 0 and
+        1 return the slice's 8-value forward / backward map (device tensor),
+        phase 2 writes and returns x of the slice."""
+        import torch
+        if phase < 2:
+            self._check(a, b, c, d)
+        if out is None:
+            out = torch.empty(8 if phase < 2 else self.n, dtype=self.torch_dtype, device="cuda")
+        s = stream if stream is not None else torch.cuda.current_stream()
+
+        def ptr(t):
+            return t.data_ptr() if t is not None else None
+        st = lib().tri_slice_solve(self._h, int(phase), int(slice_), int(nslices), ptr(a), ptr(b), ptr(c), ptr(d),
+                                   ptr(maps), out.data_ptr(), s.cuda_stream)
+        if st != 0:
+            raise TriError(st, f"tri_slice_solve(phase {phase})")
+        return out
 
     def debug_pcr(self, a, b, c, d, stream=None):
         """Only the PCR stage: returns the k-step reduced system normalised to

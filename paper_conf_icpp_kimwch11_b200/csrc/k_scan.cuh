@@ -165,14 +165,16 @@ __device__ __forceinline__ void sc_ld_rows_il(const T* ib, int s, int seg, T (&r
 }
 
 // rows outside [0, n) are identity rows; a_0 and c_{n-1} lie outside A (X1, X4)
+// (keep_a0 / keep_cn: a slice of a larger system -- its first / last row is
+// coupled to the neighbouring slice, SCAN_MC sliced solves, NEXT-4)
 template <typename T>
 __device__ __forceinline__ void sc_fix_rows(int64_t i0, int64_t n, T (&ra)[SC_R], T (&rb)[SC_R], T (&rc)[SC_R],
-                                            T (&rd)[SC_R]) {
+                                            T (&rd)[SC_R], bool keep_a0 = false, bool keep_cn = false) {
 #pragma unroll
     for (int u = 0; u < SC_R; ++u) {
         const int64_t i = i0 + u;
-        if (i == 0) ra[u] = T(0);
-        if (i == n - 1) rc[u] = T(0);
+        if (i == 0 && !keep_a0) ra[u] = T(0);
+        if (i == n - 1 && !keep_cn) rc[u] = T(0);
         if (i >= n) { ra[u] = T(0); rb[u] = T(1); rc[u] = T(0); rd[u] = T(0); }
     }
 }
@@ -300,6 +302,52 @@ __device__ __forceinline__ void sc_stg4_last(float* p, float x, float y, float z
     asm volatile("st.global.L2::cache_hint.v4.f32 [%0], {%1, %2, %3, %4}, %5;" ::"l"(p), "f"(x), "f"(y), "f"(z),
                  "f"(w), "l"(pol)
                  : "memory");
+}
+
+// Slices of a larger system (SCAN_MC sliced solve): rows past the slice's end in
+// its last window must be transparent -- the state passes through unchanged
+// (an identity ROW would reset psi = c theta) and, for the back substitution,
+// c' = -1, d' = 0 (x_t = x_{t+1}).  Only rows u < nvalid of the lane are real.
+template <typename T>
+__device__ __forceinline__ SKMat<T> sc_fwd_map_n(const T (&ra)[SC_R], const T (&rb)[SC_R], const T (&rc)[SC_R],
+                                                 const T (&rd)[SC_R], int nvalid) {
+    T t1 = T(1), p1 = T(0), d1 = T(0), t2 = T(0), p2 = T(1), d2 = T(0), d3 = T(1);
+#pragma unroll
+    for (int u = 0; u < SC_R; ++u) {
+        if (u < nvalid) {
+            T au, bu, cu, du;
+            sc_row(ra, rb, rc, rd, u, au, bu, cu, du);
+            const T nt1 = fma(bu, t1, -au * p1), np1 = cu * t1, nd1 = fma(du, t1, -au * d1);
+            const T nt2 = fma(bu, t2, -au * p2), np2 = cu * t2, nd2 = fma(du, t2, -au * d2);
+            d3 = -au * d3;
+            t1 = nt1; p1 = np1; d1 = nd1;
+            t2 = nt2; p2 = np2; d2 = nd2;
+        }
+    }
+    const T s = sc_scale2(t1, t2);
+    return SKMat<T>{t1 * s, t2 * s, p1 * s, p2 * s, d1 * s, d2 * s, d3 * s};
+}
+template <typename T>
+__device__ __forceinline__ void sc_fwd_replay_n(const T (&ra)[SC_R], const T (&rb)[SC_R], const T (&rc)[SC_R],
+                                                const T (&rd)[SC_R], T th, T ps, T de, T (&cp)[SC_R], T (&dp)[SC_R],
+                                                int nvalid) {
+#pragma unroll
+    for (int u = 0; u < SC_R; ++u) {
+        if (u < nvalid) {
+            T au, bu, cu, du;
+            sc_row(ra, rb, rc, rd, u, au, bu, cu, du);
+            const T nt = fma(bu, th, -au * ps);
+            const T np = cu * th;
+            const T nd = fma(du, th, -au * de);
+            const T inv = rcp(nt);
+            cp[u] = np * inv;
+            dp[u] = nd * inv;
+            th = nt; ps = np; de = nd;
+        } else {
+            cp[u] = T(-1);
+            dp[u] = T(0);
+        }
+    }
 }
 
 template <typename T>

@@ -36,6 +36,14 @@ struct ScanMCArgs {
     int NC;       // windows per system
     int NCW;      // windows per chunk
     int P;        // chunks per system
+    // sliced solve of one system spread over devices (m == 1; NEXT-4): the rows
+    // here are a slice of a larger system; keep_a0 / keep_cn keep the coupling
+    // of its first / last row; s0 = incoming forward state (theta, psi, delta)
+    // of the slice (null: the system's start, (1, 0, 0)); xe = x after the slice
+    // (null: 0, the system's end)
+    int keep_a0, keep_cn;
+    const T* s0;
+    const T* xe;
 };
 
 template <typename T>
@@ -156,16 +164,19 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant
     const int pi = (pw + SC_NW - 1) % SC_NW;
     // the chunk's boundary value from the maps of pass 0 / pass 1 (warp 0 runs step 0)
     T st0 = T(1), ps0 = T(0), de0 = T(0), xa0 = T(0);
-    if (MODE == 1 && warp == 0) {  // incoming state = (M_{ch-1} ... M_0) (1, 0, 0)
+    if (MODE == 1 && warp == 0) {  // incoming state = (M_{ch-1} ... M_0) S0, S0 = (1, 0, 0) or the slice's
         const SKMat<T> R = smc_reduce_fwd(p.cmap + 8 * (q * p.P), ch, lane);
-        st0 = __shfl_sync(0xffffffffu, R.a, 0);
-        ps0 = __shfl_sync(0xffffffffu, R.c, 0);
-        de0 = __shfl_sync(0xffffffffu, R.e, 0);
+        T t0 = T(1), q0 = T(0), e0 = T(0);
+        if (p.s0) { t0 = p.s0[0]; q0 = p.s0[1]; e0 = p.s0[2]; }
+        st0 = __shfl_sync(0xffffffffu, fma(R.a, t0, R.b * q0), 0);
+        ps0 = __shfl_sync(0xffffffffu, fma(R.c, t0, R.d * q0), 0);
+        de0 = __shfl_sync(0xffffffffu, fma(R.e, t0, fma(R.f, q0, R.g * e0)), 0);
     }
-    if (MODE == 2 && warp == 0) {  // x after the chunk = (B_{ch+1} ... B_{P-1})(0)
+    if (MODE == 2 && warp == 0) {  // x after the chunk = (B_{ch+1} ... B_{P-1})(x_end), x_end = 0 or the slice's
         T al, be;
         smc_reduce_bwd(p.cbm + 8 * (q * p.P + ch + 1), p.P - 1 - ch, lane, al, be);
-        xa0 = __shfl_sync(0xffffffffu, al, 0);
+        const T xend = p.xe ? p.xe[0] : T(0);
+        xa0 = __shfl_sync(0xffffffffu, fma(be, xend, al), 0);
     }
     const unsigned ib_s = (unsigned)__cvta_generic_to_shared(ib);
 
@@ -181,8 +192,9 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant
             sc_ld_rows(ib, lane, ra, rb, rc, rd);
             sc_release_buf();  // this warp's reads of the buffer before the TMA refill
             if (lane == 0 && g + SC_NW < nwin) issue(g + SC_NW);
-            if (edge) sc_fix_rows<T>(i0, n, ra, rb, rc, rd);
-            SKMat<T> M = sc_fwd_map(ra, rb, rc, rd);
+            if (edge) sc_fix_rows<T>(i0, n, ra, rb, rc, rd, p.keep_a0, p.keep_cn);
+            const int nvalid = (int)(n - i0 < 0 ? 0 : n - i0 < SC_R ? n - i0 : SC_R);
+            SKMat<T> M = (p.keep_cn && nvalid < SC_R) ? sc_fwd_map_n(ra, rb, rc, rd, nvalid) : sc_fwd_map(ra, rb, rc, rd);
 #pragma unroll
             for (int d = 1; d < 32; d <<= 1) {  // lane l: lanes l .. l + 2d - 1 (later after earlier)
                 const SKMat<T> o = sk_shfl_down(M, d);
@@ -196,8 +208,10 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant
             // ---- forward replay from the chunk's / previous window's state
             T ra[SC_R], rb[SC_R], rc[SC_R], rd[SC_R];
             sc_ld_rows(ib, lane, ra, rb, rc, rd);
-            if (edge) sc_fix_rows<T>(i0, n, ra, rb, rc, rd);
-            SKMat<T> M = sc_fwd_map(ra, rb, rc, rd);
+            if (edge) sc_fix_rows<T>(i0, n, ra, rb, rc, rd, p.keep_a0, p.keep_cn);
+            const int nvalid = (int)(n - i0 < 0 ? 0 : n - i0 < SC_R ? n - i0 : SC_R);
+            const bool tr = p.keep_cn && nvalid < SC_R;  // transparent padding rows (slice of a larger system)
+            SKMat<T> M = tr ? sc_fwd_map_n(ra, rb, rc, rd, nvalid) : sc_fwd_map(ra, rb, rc, rd);
             sc_fwd_scan(M, lane);
             if (g > 0) asm volatile("bar.sync %0, 64;" ::"r"(1 + pi) : "memory");
             T th, ps, de;
@@ -223,7 +237,8 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant
             sc_release_buf();  // this warp's reads of the buffer before the TMA refill
             if (lane == 0 && g + SC_NW < nwin) issue(g + SC_NW);  // rows are in registers
             T cp[SC_R], dp[SC_R];
-            sc_fwd_replay(ra, rb, rc, rd, th, ps, de, cp, dp);
+            if (tr) sc_fwd_replay_n(ra, rb, rc, rd, th, ps, de, cp, dp, nvalid);
+            else sc_fwd_replay(ra, rb, rc, rd, th, ps, de, cp, dp);
             T* dst = p.cd + (q * NC + w) * (int64_t)sc_slot_elems<T>();
             if constexpr (sizeof(T) == 8) {
 #pragma unroll
@@ -283,6 +298,50 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant
             smc_reduce_bwd(wm, nwin, lane, al, be);
             if (lane == 0) { p.cbm[8 * (int64_t)blockIdx.x] = al; p.cbm[8 * (int64_t)blockIdx.x + 1] = be; }
         }
+    }
+}
+
+// ---- sliced solve of one system over devices (NEXT-4): the products of all P
+// chunk maps of this device's slice (warp 0; MODE 0: forward 3x3 map, MODE 1:
+// backward affine map), written as 8 values to `out`
+template <typename T, int MODE>
+__global__ void k_scan_mc_slice_map(ScanMCArgs<T> p, T* out) {
+    const int lane = threadIdx.x & 31;
+    if (MODE == 0) {
+        const SKMat<T> R = smc_reduce_fwd(p.cmap, p.P, lane);
+        if (lane == 0) {
+            out[0] = R.a; out[1] = R.b; out[2] = R.c; out[3] = R.d; out[4] = R.e; out[5] = R.f; out[6] = R.g;
+            out[7] = T(0);
+        }
+    } else {
+        T al, be;
+        smc_reduce_bwd(p.cbm, p.P, lane, al, be);
+        if (lane == 0) { out[0] = al; out[1] = be; for (int i = 2; i < 8; ++i) out[i] = T(0); }
+    }
+}
+
+// the slice boundary values from every device's slice maps (G x 8 values, in
+// slice order; one thread): MODE 0: incoming forward state of slice r =
+// (M_{r-1} ... M_0)(1, 0, 0), rescaled; MODE 1: x after slice r =
+// (B_{r+1} ... B_{G-1})(0)
+template <typename T, int MODE>
+__global__ void k_scan_mc_slice_link(const T* maps, int G, int r, T* out) {
+    if (threadIdx.x != 0) return;
+    if (MODE == 0) {
+        T th = T(1), ps = T(0), de = T(0);
+        for (int s = 0; s < r; ++s) {
+            const T* M = maps + 8 * s;
+            const T ot = fma(M[0], th, M[1] * ps);
+            const T op = fma(M[2], th, M[3] * ps);
+            const T od = fma(M[4], th, fma(M[5], ps, M[6] * de));
+            const T sc = sk_exp2_scale(ot);
+            th = ot * sc; ps = op * sc; de = od * sc;
+        }
+        out[0] = th; out[1] = ps; out[2] = de;
+    } else {
+        T x = T(0);
+        for (int s = G - 1; s > r; --s) x = fma(maps[8 * s + 1], x, maps[8 * s]);
+        out[0] = x;
     }
 }
 

@@ -422,7 +422,7 @@ void plan_geometry(tri_plan_s* p) {
 size_t scratch_need(const tri_plan_s* p) {
     if (p->variant == TRI_VARIANT_SCAN_MC)  // c', d' per window + the chunk maps
         return ((size_t)p->m * (size_t)p->sk_nc * (size_t)sc_slot_elems<double>() +
-                (size_t)p->m * (size_t)p->mc_P * 16) * esize(p->dtype);
+                (size_t)p->m * (size_t)p->mc_P * 16 + 16) * esize(p->dtype);
     if (p->variant == TRI_VARIANT_SCAN)
         return (p->sk_nc == 1 && p->sk_S == 1) ? 0
                              : (size_t)p->sk_grid * (size_t)std::max(0, p->sk_nc + p->sk_delta - p->sk_son) *
@@ -750,29 +750,73 @@ cudaError_t launch_scan(const tri_plan_s* p, const void* a, const void* b, const
 }
 
 template <typename T>
-cudaError_t launch_scan_mc(const tri_plan_s* p, const void* a, const void* b, const void* c, const void* d, void* x,
-                           cudaStream_t st) {
-    StreamMaps tm;
+cudaError_t scan_mc_setup(const tri_plan_s* p, const void* a, const void* b, const void* c, const void* d, void* x,
+                          StreamMaps& tm, ScanMCArgs<T>& A, int& smem) {
     const int64_t n = p->n, m = p->m;
-    if (!tma_map_sys_rows8<T>(&tm.a, a, n, m) || !tma_map_sys_rows8<T>(&tm.b, b, n, m) ||
-        !tma_map_sys_rows8<T>(&tm.c, c, n, m) || !tma_map_sys_rows8<T>(&tm.d, d, n, m))
+    if (a && (!tma_map_sys_rows8<T>(&tm.a, a, n, m) || !tma_map_sys_rows8<T>(&tm.b, b, n, m) ||
+              !tma_map_sys_rows8<T>(&tm.c, c, n, m) || !tma_map_sys_rows8<T>(&tm.d, d, n, m)))
         return cudaErrorNotSupported;
-    ScanMCArgs<T> A;
+    A = ScanMCArgs<T>{};
     A.x = (T*)x;
     A.cd = (T*)p->scratch;
     const int64_t mp = p->m * (int64_t)p->mc_P;
     A.cmap = A.cd + p->m * (int64_t)p->sk_nc * sc_slot_elems<T>();
     A.cbm = A.cmap + 8 * mp;
     A.n = p->n; A.m = p->m; A.NC = p->sk_nc; A.NCW = p->mc_NCW; A.P = p->mc_P;
-    const int smem = SMCLayout<T>::smem_bytes(p->mc_NCW);
-    cudaError_t e;
+    smem = SMCLayout<T>::smem_bytes(p->mc_NCW);
     for (auto k : {k_scan_mc<T, 0>, k_scan_mc<T, 1>, k_scan_mc<T, 2>}) {
-        e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+        cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
         if (e != cudaSuccess) return e;
     }
+    return cudaSuccess;
+}
+// the 16 values after the chunk maps: the slice's incoming state (3) and x after it (1)
+template <typename T>
+T* scan_mc_slice_vals(const tri_plan_s* p) {
+    return (T*)p->scratch + p->m * (int64_t)p->sk_nc * sc_slot_elems<T>() + 16 * p->m * (int64_t)p->mc_P;
+}
+
+template <typename T>
+cudaError_t launch_scan_mc(const tri_plan_s* p, const void* a, const void* b, const void* c, const void* d, void* x,
+                           cudaStream_t st) {
+    StreamMaps tm;
+    ScanMCArgs<T> A;
+    int smem = 0;
+    cudaError_t e = scan_mc_setup<T>(p, a, b, c, d, x, tm, A, smem);
+    if (e != cudaSuccess) return e;
     k_scan_mc<T, 0><<<p->sk_grid, SC_THREADS, smem, st>>>(tm, A);
     k_scan_mc<T, 1><<<p->sk_grid, SC_THREADS, smem, st>>>(tm, A);
     k_scan_mc<T, 2><<<p->sk_grid, SC_THREADS, smem, st>>>(tm, A);
+    return cudaGetLastError();
+}
+
+// sliced solve of one system over devices (NEXT-4): phase 0 = pass 0 + the
+// slice's forward map; 1 = incoming state from every slice's map, pass 1, the
+// slice's backward map; 2 = x after the slice from every backward map, pass 2
+template <typename T>
+cudaError_t launch_scan_mc_slice(const tri_plan_s* p, int phase, int slice, int nslices, const void* a, const void* b,
+                                 const void* c, const void* d, const void* maps, void* out, cudaStream_t st) {
+    StreamMaps tm;
+    ScanMCArgs<T> A;
+    int smem = 0;
+    cudaError_t e = scan_mc_setup<T>(p, phase < 2 ? a : nullptr, b, c, d, phase == 2 ? out : nullptr, tm, A, smem);
+    if (e != cudaSuccess) return e;
+    A.keep_a0 = slice > 0;
+    A.keep_cn = slice < nslices - 1;
+    T* vals = scan_mc_slice_vals<T>(p);
+    if (phase == 0) {
+        k_scan_mc<T, 0><<<p->sk_grid, SC_THREADS, smem, st>>>(tm, A);
+        k_scan_mc_slice_map<T, 0><<<1, 32, 0, st>>>(A, (T*)out);
+    } else if (phase == 1) {
+        k_scan_mc_slice_link<T, 0><<<1, 32, 0, st>>>((const T*)maps, nslices, slice, vals);
+        A.s0 = vals;
+        k_scan_mc<T, 1><<<p->sk_grid, SC_THREADS, smem, st>>>(tm, A);
+        k_scan_mc_slice_map<T, 1><<<1, 32, 0, st>>>(A, (T*)out);
+    } else {
+        k_scan_mc_slice_link<T, 1><<<1, 32, 0, st>>>((const T*)maps, nslices, slice, vals + 4);
+        A.xe = vals + 4;
+        k_scan_mc<T, 2><<<p->sk_grid, SC_THREADS, smem, st>>>(tm, A);
+    }
     return cudaGetLastError();
 }
 
@@ -1116,6 +1160,24 @@ tri_status tri_plan_set_variant(tri_plan_t p, tri_variant v) {
     tri_status st = ensure_scratch(p);
     if (st != TRI_OK) { p->variant = ov; p->k = ok; plan_geometry(p); }
     return st;
+}
+
+tri_status tri_slice_solve(tri_plan_t p, int phase, int slice, int nslices, const void* a, const void* b,
+                           const void* c, const void* d, const void* maps, void* out, void* stream) {
+    if (!p || p->variant != TRI_VARIANT_SCAN_MC || p->m != 1 || nslices < 1 || slice < 0 || slice >= nslices ||
+        phase < 0 || phase > 2 || !out || (phase > 0 && !maps))
+        return TRI_ERR_INVALID_ARG;
+    if (phase < 2) {  // the slice's rows; `out` is an 8-value map
+        const void* in[4] = {a, b, c, d};
+        tri_status st = check_ptrs(p, in, 4, nullptr, 0);
+        if (st != TRI_OK) return st;
+    }
+    if ((uintptr_t)out % 16 || (maps && (uintptr_t)maps % 16)) return TRI_ERR_ALIGNMENT;
+    cudaStream_t s = (cudaStream_t)stream;
+    const cudaError_t e = p->dtype == TRI_F64
+                              ? launch_scan_mc_slice<double>(p, phase, slice, nslices, a, b, c, d, maps, out, s)
+                              : launch_scan_mc_slice<float>(p, phase, slice, nslices, a, b, c, d, maps, out, s);
+    return e == cudaSuccess ? TRI_OK : TRI_ERR_CUDA;
 }
 
 tri_status tri_plan_autotune(tri_plan_t p, const void* a, const void* b, const void* c, const void* d, void* x,

@@ -108,3 +108,35 @@ def solve_sharded(n, m, make_inputs, solve_fn, layout=CONTIGUOUS, gather=True, g
         x = torch.empty(0, dtype=torch.float64)
     full = gather_x(x, n, m, layout, group) if (gather and world > 1) else (x if gather else None)
     return x, full
+
+
+def solve_one_system_sliced(a, b, c, d, group=None, allgather=None):
+    """One system spread over the ranks: every rank holds a
+    contiguous slice of its rows (a, b, c, d: this rank's slice, device tensors,
+    len % 8 == 0, > 256 rows) and gets x of its slice back.  The slices exchange
+    only their 8-value forward and backward maps (two all-gathers, NCCL over
+    NVLink on the GPU box); all arithmetic runs in the SCAN_MC kernels
+    (tri_slice_solve).  `allgather(t) -> [t_0, ..., t_{G-1}]` overrides the
+    collective (tests run several slices on one device)."""
+    from . import Plan, VARIANT_SCAN_MC, F64, F32
+    if allgather is None:
+        world = dist.get_world_size(group)
+        rank = dist.get_rank(group)
+
+        on_host = dist.get_backend(group) == "gloo"  # gloo: the 8-value maps travel through host memory
+
+        def allgather(t):
+            src = t.cpu() if on_host else t
+            out = [torch.empty_like(src) for _ in range(world)]
+            dist.all_gather(out, src, group=group)
+            return [o.to(t.device) for o in out]
+    else:
+        world, rank = allgather.world, allgather.rank
+    n = a.numel()
+    plan = Plan(n, 1, F64 if a.dtype == torch.float64 else F32, 0)
+    plan.variant = VARIANT_SCAN_MC
+    fmap = plan.slice_phase(0, rank, world, a, b, c, d)
+    maps = torch.cat(allgather(fmap))
+    bmap = plan.slice_phase(1, rank, world, a, b, c, d, maps=maps)
+    bmaps = torch.cat(allgather(bmap))
+    return plan.slice_phase(2, rank, world, maps=bmaps)

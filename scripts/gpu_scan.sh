@@ -1,2 +1,2 @@
 mkdir -p gpurun_out
-( for rep in 1 2; do for lib in paper_conf_icpp_kimwch11_b200/libtri.so build_var/libtri_nw10.so build_var/libtri_nw11.so build_var/libtri_nw13.so build_var/libtri_nw14.so; do echo "== $lib"; for args in "16384 16384 f64 0 0" "16777216 1 f64 0 0" "1024 1024 f64 1 0"; do TRI_LIB_PATH=$lib timeout 120 python scripts/prof_one.py $args - 2 | grep graph; done; done; done ) > gpurun_out/scan_times.log 2>&1
+timeout 900 python -m pytest tests/test_dist_sliced_gpu.py -q --timeout 300 > gpurun_out/pytest_scan.log 2>&1; echo "rc=$?" >> gpurun_out/pytest_scan.log

@@ -634,6 +634,59 @@ def test_scan_mc_rejects_unsupported(cuda_ok):
             plan.variant = SCAN_MC
 
 
+def _sliced_solve_one_device(arrs, cuts, dtype):
+    """NEXT-4 on one device: the system's row ranges [cuts[i], cuts[i+1]) as G
+    'devices' (one plan each), phases run in order with the maps gathered by
+    concatenation (what the all-gather of dist.solve_one_system_sliced does)."""
+    import torch
+    G = len(cuts) - 1
+    td = tri.F64 if dtype == "f64" else tri.F32
+    sl = [[torch.from_numpy(t[cuts[r]:cuts[r + 1]].copy()).cuda() for t in arrs] for r in range(G)]
+    plans = []
+    for r in range(G):
+        p = tri.Plan(cuts[r + 1] - cuts[r], 1, td, 0)
+        p.variant = tri.VARIANT_SCAN_MC
+        plans.append(p)
+    maps = torch.cat([plans[r].slice_phase(0, r, G, *sl[r]) for r in range(G)])
+    bmaps = torch.cat([plans[r].slice_phase(1, r, G, *sl[r], maps=maps) for r in range(G)])
+    return torch.cat([plans[r].slice_phase(2, r, G, maps=bmaps) for r in range(G)]).cpu().numpy()
+
+
+@pytest.mark.parametrize("dtype,family,cuts", [
+    ("f64", "dd", [0, 1 << 20]),
+    ("f64", "dd", [0, 300000, 562144, 1000008, 1 << 21]),
+    ("f64", "weak", [0, 65536, 131072, 196608, 262144, 327680, 393216, 458752, 524288]),
+    ("f64", "poisson", [0, 4096, 8192, 12288, 16384]),
+    ("f32", "dd", [0, 70000, 140000, 1000000]),
+])
+def test_one_system_sliced_over_devices(cuda_ok, dtype, family, cuts):
+    """one system split into row slices (ragged, 1 to 8
+    slices), each solved by its own plan with only 8-value maps exchanged
+    (tri_slice_solve); vs the oracle on the whole system."""
+    n = cuts[-1]
+    arrs = gen(n, 1, dtype, 0, family, eps=1e-2)
+    x = _sliced_solve_one_device(arrs, cuts, dtype)
+    if family == "poisson":
+        xo = oracle.solve_batch(n, 1, *arrs)
+        assert np.max(np.abs(x - xo)) / np.max(np.abs(xo)) <= 2 * (n + 1) ** 2 / 2 * 2.2e-16
+    else:
+        check_parity(n, 1, arrs, x, dtype, 0)
+
+
+def test_one_system_sliced_rejects(cuda_ok):
+    import torch
+    p = tri.Plan(4096, 1, tri.F64, 0)
+    p.variant = tri.VARIANT_SCAN  # not SCAN_MC
+    a = torch.ones(4096, dtype=torch.float64, device="cuda")
+    with pytest.raises(tri.TriError):
+        p.slice_phase(0, 0, 2, a, a, a, a)
+    p.variant = tri.VARIANT_SCAN_MC
+    with pytest.raises(tri.TriError):
+        p.slice_phase(0, 2, 2, a, a, a, a)  # slice out of range
+    with pytest.raises(tri.TriError):
+        p.slice_phase(1, 0, 2, a, a, a, a)  # phase 1 needs the gathered maps
+
+
 # ------------------------------------------------------------------ WARP variant
 @pytest.mark.parametrize("dtype", ["f64", "f32"])
 @pytest.mark.parametrize("layout", [0, 1])
