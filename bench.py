@@ -49,8 +49,10 @@ def parse():
     ap.add_argument("--family", default="dd")
     ap.add_argument("--k", type=int, default=None, help="force the transition point k")
     ap.add_argument("--variant", type=int, default=None, help="force variant (1 onchip, 2 split, 3 fused)")
-    ap.add_argument("--scaling", default="strong", choices=["strong", "weak"],
-                    help="strong: the config's m is split over ranks; weak: every rank solves the full m")
+    ap.add_argument("--scaling", default="weak", choices=["strong", "weak"],
+                    help="weak (default; the systems are independent, so every rank solves its own full "
+                         "batch of the config's m systems, no data-path collective); strong: the config's m is "
+                         "split over ranks")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-e2e", action="store_true")

@@ -1,2 +1,2 @@
 mkdir -p gpurun_out
-timeout 900 python -m pytest tests/test_dist_sliced_gpu.py -q --timeout 300 > gpurun_out/pytest_scan.log 2>&1; echo "rc=$?" >> gpurun_out/pytest_scan.log
+( timeout 120 python scripts/prof_scan.py 16384 16384; TRI_FUSED_DBG_MODE=2 timeout 120 python scripts/prof_scan.py 16384 16384; TRI_FUSED_DBG_MODE=1 timeout 120 python scripts/prof_scan.py 16384 16384 ) > gpurun_out/prof_scan.log 2>&1
