@@ -21,6 +21,7 @@
 #include "k_stream.cuh"
 #include "k_scan.cuh"
 #include "k_scan_mc.cuh"
+#include "k_scan_rs.cuh"
 #include "k_warp.cuh"
 #include "k_pthomas_tma.cuh"
 
@@ -41,6 +42,7 @@ int g_split_k1max = std::min(10, env_int("TRI_SPLIT_K1MAX", 10));  // steps kept
 int g_tiled_waves2 = env_int("TRI_TILED_WAVES2", 3);  // measured best at c3 (1 / 3 waves)
 int g_scan_delta = env_int("TRI_SCAN_DELTA", 8);      // SCAN: back-substitution lag in steps (tuning)
 int g_scan1 = getenv("TRI_SCAN1_OFF") ? 0 : 1;        // SCAN, one-window systems: chain-free kernel (A/B)
+int g_scan_rs = getenv("TRI_SCAN_RS") ? atoi(getenv("TRI_SCAN_RS")) : 0;  // SCAN: role-split kernel (A/B)
 
 constexpr int ONCHIP_THREADS = 512;
 constexpr int SPLIT_K1MAX = 10;  // deepest k one sliding-window pass holds in smem (T = 256)
@@ -726,6 +728,21 @@ cudaError_t launch_scan(const tri_plan_s* p, const void* a, const void* b, const
     A.n = p->n; A.m = p->m; A.ms = p->ms; A.NC = p->sk_nc; A.S_on = p->sk_son; A.delta = p->sk_delta;
     A.prof = (unsigned long long*)g_fused_prof;
     A.dbg = g_fused_dbg_mode;
+    if (S == 1 && p->sk_nc >= 2 && g_scan_rs) {  // role-split warps (k_scan_rs.cuh)
+        const int NS = p->sk_nc + p->sk_delta;
+        const int fixed = RSLayout<T>::smem_bytes(p->sk_nc, p->sk_delta, 0);
+        const int son = (int)std::min<int64_t>(NS, std::max<int64_t>(0, ((int64_t)p->smem_optin - fixed) /
+                                                                             RSLayout<T>::slot_bytes));
+        if (son >= p->sk_son) {  // the plan's spill scratch covers NS - son slots
+            ScanArgs<T> B = A;
+            B.S_on = son;
+            const int smem = RSLayout<T>::smem_bytes(p->sk_nc, p->sk_delta, son);
+            cudaError_t e = cudaFuncSetAttribute(k_scan_rs<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+            if (e != cudaSuccess) return e;
+            k_scan_rs<T><<<p->sk_grid, RS_THREADS, smem, st>>>(tm, B);
+            return cudaGetLastError();
+        }
+    }
     // one-window systems shorter than 3/4 of a window (many idle rows: compute-heavy)
     // run the chain-free kernel with more warps (fp32 n = 128: 1.19 ms vs 1.50 ms
     // per 2^28 rows); at n = 256 the 12-warp kernel is faster (c4: 0.99 vs 1.02 ms)
