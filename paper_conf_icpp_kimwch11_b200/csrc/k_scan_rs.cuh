@@ -4,8 +4,10 @@
 // storage slot) and RS_NB backward warps run the back-substitution chain (slot
 // -> affine maps, scan, x handover, replay -> x), each chain through its own
 // named barriers.  A backward warp holds no rows and a forward warp no (c', d'),
-// so each role needs fewer registers and a shorter step than the combined step
-// of k_scan, and more warps fit the register file.
+// so each role needs fewer registers (124 vs 156 at fp64) and a shorter step.
+// MEASURED SLOWER than the paired k_scan (c5 shape: 2.06-2.08 ms for 10+4,
+// 11+4, 9+5 warps vs 1.86 ms), so it is off by default (TRI_SCAN_RS=1 selects
+// it for A/B measurements; tested by the SCAN parity tests under that switch).
 //
 // Slots: forward step f (window f of the CTA's sequence, system f / NC, window
 // f % NC) stores into a slot; backward step b (system b / NC, window NC - 1 -
