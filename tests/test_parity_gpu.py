@@ -801,3 +801,24 @@ def test_c4_auto_plan_sampled(cuda_ok, layout):
         sub = trigen.generate(n, 1, "f32", 0, "dd", seed=trigen.SEED_BASE + 4, q0=q)
         xs = x.reshape(m, n)[q] if layout == 0 else x.reshape(n, m)[:, q]
         check_parity(n, 1, sub, xs, "f32", 0)
+
+
+def test_scan_role_split_variant(cuda_ok):
+    """The role-split SCAN kernel (k_scan_rs.cuh, selected by TRI_SCAN_RS=1 at
+    library load, hence a subprocess): parity on chained contiguous shapes."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    code = (
+        "import sys; sys.path.insert(0, %r)\n"
+        "from tests._helpers import gen, gpu_solve, check_parity\n"
+        "import paper_conf_icpp_kimwch11_b200 as tri\n"
+        "for dt, n, m in [('f64', 2048, 300), ('f64', 16392, 150), ('f32', 4104, 40), ('f64', 512, 1000)]:\n"
+        "    arrs = gen(n, m, dt, 0)\n"
+        "    x, plan = gpu_solve(n, m, arrs, dt, 0, variant=tri.VARIANT_SCAN)\n"
+        "    check_parity(n, m, arrs, x, dt, 0)\n"
+        "print('ok')\n" % root)
+    env = dict(os.environ, TRI_SCAN_RS="1")
+    r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, timeout=300)
+    assert r.returncode == 0 and "ok" in r.stdout, r.stdout[-2000:] + r.stderr[-2000:]
