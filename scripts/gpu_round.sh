@@ -10,3 +10,7 @@ timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_sc
 python scripts/ncu_summary.py gpurun_out/c5_scan_full.ncu-rep gpurun_out/ncu_c5_scan.txt >> gpurun_out/ncu_c5.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_scan -c 1 -f -o gpurun_out/c4_scan_full python scripts/prof_one.py 256 1048576 f32 0 0 - 1 > gpurun_out/ncu_c4.log 2>&1
 python scripts/ncu_summary.py gpurun_out/c4_scan_full.ncu-rep gpurun_out/ncu_c4_scan.txt >> gpurun_out/ncu_c4.log 2>&1
+# the paper's PCR method on the configs where the planner now prefers SCAN / SCAN_MC
+timeout 600 python bench.py --config c3 --variant 2 --no-e2e --no-cpu > gpurun_out/bench_c3_split.json 2> gpurun_out/bench_c3_split.err
+timeout 600 python bench.py --config c5 --variant 5 --no-e2e --no-cpu > gpurun_out/bench_c5_stream.json 2> gpurun_out/bench_c5_stream.err
+timeout 600 python bench.py --config c4 --variant 2 --k 0 --no-e2e --no-cpu > gpurun_out/bench_c4_split.json 2> gpurun_out/bench_c4_split.err
