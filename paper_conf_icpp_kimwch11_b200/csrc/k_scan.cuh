@@ -51,6 +51,9 @@ constexpr int SC_NCMAX = 4096;
 //   one-window systems: 1 = two buffers per warp (c4 fp32 1073 us), 0 = refill
 //   after the read (fp32 c4: 983 us, fp64 n = 256: 1763 us), -1 = after the
 //   solve (fp32: 1071 us; fp64: 1654 us);  default: fp32 0, fp64 -1.
+//   Also measured for fp32 n = 256: the loads alone (diagnostic mode 2) take as
+//   long as the whole solve (0.98 ms: the memory pipeline is the bound), and two
+//   systems per 2 KB TMA box / warp step were slower (1.18 ms).
 #ifndef SC_DB
 #define SC_DB 2                    // 2 = the per-dtype default above
 #endif
@@ -125,7 +128,7 @@ __device__ __forceinline__ T sc_scale2(T u, T v) {
     return sk_exp2_scale(fmax(fabs(u), fabs(v)));
 }
 
-template <typename T>
+template <typename T, int AS = SC_W>  // AS: elements between the four arrays in the staging buffer
 __device__ __forceinline__ void sc_ld_rows(const T* ib, int lane, T (&ra)[SC_R], T (&rb)[SC_R], T (&rc)[SC_R],
                                            T (&rd)[SC_R]) {
     constexpr int EPC = 16 / (int)sizeof(T);   // elements per 16-byte chunk
@@ -135,10 +138,10 @@ __device__ __forceinline__ void sc_ld_rows(const T* ib, int lane, T (&ra)[SC_R],
 #pragma unroll
     for (int cc = 0; cc < CPL; ++cc) {
         const int o = (cc ^ swz) * EPC;
-        const int4 va = *reinterpret_cast<const int4*>(st + 0 * SC_W + o);
-        const int4 vb = *reinterpret_cast<const int4*>(st + 1 * SC_W + o);
-        const int4 vc = *reinterpret_cast<const int4*>(st + 2 * SC_W + o);
-        const int4 vd = *reinterpret_cast<const int4*>(st + 3 * SC_W + o);
+        const int4 va = *reinterpret_cast<const int4*>(st + 0 * AS + o);
+        const int4 vb = *reinterpret_cast<const int4*>(st + 1 * AS + o);
+        const int4 vc = *reinterpret_cast<const int4*>(st + 2 * AS + o);
+        const int4 vd = *reinterpret_cast<const int4*>(st + 3 * AS + o);
 #pragma unroll
         for (int e = 0; e < EPC; ++e) {
             ra[cc * EPC + e] = reinterpret_cast<const T*>(&va)[e];
@@ -506,6 +509,14 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
             sc_ld_rows(bufs[bsel], lane, ra, rb, rc, rd);
             sc_release_buf();  // this warp's reads of the buffer before the TMA refill
             if (DB >= 0 && lane == 0 && j + NB * SC_NW < nsys) issue_to(j + NB * SC_NW, 0, bufs[bsel], bars[bsel]);
+            if (p.dbg == 2) {  // diagnostics: the memory pipeline alone (inputs in, x out; no math)
+                T xz[SC_R];
+#pragma unroll
+                for (int t = 0; t < SC_R; ++t) xz[t] = ra[t] * T(0);
+                sc_store_x(p.x + q * n + lane * SC_R, n - (int64_t)lane * SC_R, xz);
+                if (DB < 0 && lane == 0 && j + SC_NW < nsys) issue_to(j + SC_NW, 0, bufs[0], bars[0]);
+                continue;
+            }
             sc_fix_rows<T>((int64_t)lane * SC_R, n, ra, rb, rc, rd);
             SKMat<T> M = sc_fwd_map(ra, rb, rc, rd);
             sc_fwd_scan(M, lane);

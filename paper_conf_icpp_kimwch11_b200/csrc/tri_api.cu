@@ -672,12 +672,12 @@ cudaError_t launch_stream(const tri_plan_s* p, const void* a, const void* b, con
 // swizzle; fp32: 32-byte rows, 32B swizzle), box [1][32][8] = one 256-row window
 // of one system per array; every coordinate fits int32 for any n, m of the API
 template <typename T>
-bool tma_map_sys_rows8(CUtensorMap* tm, const void* base, int64_t n, int64_t m) {
+bool tma_map_sys_rows8(CUtensorMap* tm, const void* base, int64_t n, int64_t m, int sys_per_box = 1) {
     auto enc = tma_encoder();
     if (!enc) return false;
     cuuint64_t dims[3] = {8, (cuuint64_t)(n / 8), (cuuint64_t)m};
     cuuint64_t strides[2] = {8 * sizeof(T), (cuuint64_t)n * sizeof(T)};
-    cuuint32_t box[3] = {8, 32, 1};
+    cuuint32_t box[3] = {8, 32, (cuuint32_t)sys_per_box};
     cuuint32_t es[3] = {1, 1, 1};
     return enc(tm, sizeof(T) == 8 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT64 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3,
                const_cast<void*>(base), dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
