@@ -67,6 +67,7 @@ struct ScanArgs {
     T* spill;      // per CTA: (NC + delta - S_on) slots of sc_slot_elems<T>() elements
     int64_t n, m;
     int64_t ms;    // S > 1 (INTERLEAVED / BATCHED): systems per batch (INTERLEAVED: m, one batch)
+    int w128;      // CONTIGUOUS: tensor view [m][n/r][r] with 128-byte rows (r = 32 fp32 / 16 fp64), 128B swizzle
     int NC;        // windows per system
     int delta;     // extra lag (steps) of the back substitution behind the forward sweep
     int S_on;      // storage slots resident in shared memory
@@ -165,6 +166,51 @@ __device__ __forceinline__ void sc_ld_rows_il(const T* ib, int s, int seg, T (&r
         rc[t] = st[2 * SC_W + t * S];
         rd[t] = st[3 * SC_W + t * S];
     }
+}
+
+// fp32 window staged as 128-byte TMA rows (tensor view [m][n/32][32], 128B
+// swizzle: 16-byte chunk c of row r at c ^ (r & 7)): lane l holds rows 8l..8l+7
+// = chunks 2(l%4), 2(l%4)+1 of row l/4.  One TMA request per 128 bytes instead of
+// per 32 bytes (the [n/8][8] view).
+__device__ __forceinline__ void sc_ld_rows_w128(const float* ib, int lane, float (&ra)[SC_R], float (&rb)[SC_R],
+                                                float (&rc)[SC_R], float (&rd)[SC_R]) {
+    const int r = lane >> 2, c0 = (lane & 3) * 2;
+#pragma unroll
+    for (int k = 0; k < 2; ++k) {
+        const int o = r * 32 + (((c0 + k) ^ (r & 7)) * 4);
+        const float4 va = *reinterpret_cast<const float4*>(ib + 0 * SC_W + o);
+        const float4 vb = *reinterpret_cast<const float4*>(ib + 1 * SC_W + o);
+        const float4 vc = *reinterpret_cast<const float4*>(ib + 2 * SC_W + o);
+        const float4 vd = *reinterpret_cast<const float4*>(ib + 3 * SC_W + o);
+        ra[4 * k] = va.x; ra[4 * k + 1] = va.y; ra[4 * k + 2] = va.z; ra[4 * k + 3] = va.w;
+        rb[4 * k] = vb.x; rb[4 * k + 1] = vb.y; rb[4 * k + 2] = vb.z; rb[4 * k + 3] = vb.w;
+        rc[4 * k] = vc.x; rc[4 * k + 1] = vc.y; rc[4 * k + 2] = vc.z; rc[4 * k + 3] = vc.w;
+        rd[4 * k] = vd.x; rd[4 * k + 1] = vd.y; rd[4 * k + 2] = vd.z; rd[4 * k + 3] = vd.w;
+    }
+}
+// fp64 in 128-byte rows (tensor view [m][n/16][16]): lane l holds rows 8l..8l+7 =
+// chunks 4(l%2) .. 4(l%2)+3 of row l/2
+__device__ __forceinline__ void sc_ld_rows_w128(const double* ib, int lane, double (&ra)[SC_R], double (&rb)[SC_R],
+                                                double (&rc)[SC_R], double (&rd)[SC_R]) {
+    const int r = lane >> 1, c0 = (lane & 1) * 4;
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+        const int o = r * 16 + (((c0 + k) ^ (r & 7)) * 2);
+        const double2 va = *reinterpret_cast<const double2*>(ib + 0 * SC_W + o);
+        const double2 vb = *reinterpret_cast<const double2*>(ib + 1 * SC_W + o);
+        const double2 vc = *reinterpret_cast<const double2*>(ib + 2 * SC_W + o);
+        const double2 vd = *reinterpret_cast<const double2*>(ib + 3 * SC_W + o);
+        ra[2 * k] = va.x; ra[2 * k + 1] = va.y;
+        rb[2 * k] = vb.x; rb[2 * k + 1] = vb.y;
+        rc[2 * k] = vc.x; rc[2 * k + 1] = vc.y;
+        rd[2 * k] = vd.x; rd[2 * k + 1] = vd.y;
+    }
+}
+template <typename T>
+__device__ __forceinline__ void sc_ld_rows_any(const T* ib, int lane, bool w128, T (&ra)[SC_R], T (&rb)[SC_R],
+                                               T (&rc)[SC_R], T (&rd)[SC_R]) {
+    if (w128) { sc_ld_rows_w128(ib, lane, ra, rb, rc, rd); return; }
+    sc_ld_rows(ib, lane, ra, rb, rc, rd);
 }
 
 // rows outside [0, n) are identity rows; a_0 and c_{n-1} lie outside A (X1, X4)
@@ -473,7 +519,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
         const int q = (int)(blockIdx.x + (int64_t)jj * gridDim.x);
         sk_expect(bar, (unsigned)(4 * SC_W * sizeof(T)));
         if constexpr (S == 1) {
-            const int y = ww * (SC_W / 8);
+            const int y = ww * (p.w128 ? SC_W * (int)sizeof(T) / 128 : SC_W / 8);
             sc_tma3d(buf + 0 * SC_W, &tm.a, y, q, bar, pol_in);
             sc_tma3d(buf + 1 * SC_W, &tm.b, y, q, bar, pol_in);
             sc_tma3d(buf + 2 * SC_W, &tm.c, y, q, bar, pol_in);
@@ -506,7 +552,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
             T ra[SC_R], rb[SC_R], rc[SC_R], rd[SC_R];
             sk_wait(bars[bsel], (phs >> bsel) & 1u);
             phs ^= 1u << bsel;
-            sc_ld_rows(bufs[bsel], lane, ra, rb, rc, rd);
+            sc_ld_rows_any(bufs[bsel], lane, p.w128 != 0, ra, rb, rc, rd);
             sc_release_buf();  // this warp's reads of the buffer before the TMA refill
             if (DB >= 0 && lane == 0 && j + NB * SC_NW < nsys) issue_to(j + NB * SC_NW, 0, bufs[bsel], bars[bsel]);
             if (p.dbg == 2) {  // diagnostics: the memory pipeline alone (inputs in, x out; no math)
@@ -623,7 +669,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
         const int64_t qf = S > 1 ? (gq - (gq / gpb) * gpb) * S + ls : 0;
         const bool edge = cw == 0 || (int64_t)(cw + 1) * WR > n || (S > 1 && qf >= p.ms);
         auto load_rows = [&](T (&ra)[SC_R], T (&rb)[SC_R], T (&rc)[SC_R], T (&rd)[SC_R]) {
-            if constexpr (S == 1) sc_ld_rows(ib, lane, ra, rb, rc, rd);
+            if constexpr (S == 1) sc_ld_rows_any(ib, lane, p.w128 != 0, ra, rb, rc, rd);
             else sc_ld_rows_il<S>(ib, ls, seg, ra, rb, rc, rd);
         };
         auto fix_rows = [&](T (&ra)[SC_R], T (&rb)[SC_R], T (&rc)[SC_R], T (&rd)[SC_R]) {

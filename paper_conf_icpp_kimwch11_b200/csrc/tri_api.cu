@@ -43,6 +43,7 @@ int g_tiled_waves2 = env_int("TRI_TILED_WAVES2", 3);  // measured best at c3 (1 
 int g_scan_delta = env_int("TRI_SCAN_DELTA", 8);      // SCAN: back-substitution lag in steps (tuning)
 int g_scan1 = getenv("TRI_SCAN1_OFF") ? 0 : 1;        // SCAN, one-window systems: chain-free kernel (A/B)
 int g_scan_rs = getenv("TRI_SCAN_RS") ? atoi(getenv("TRI_SCAN_RS")) : 0;  // SCAN: role-split kernel (A/B)
+int g_scan_w128 = getenv("TRI_SCAN_W128") ? atoi(getenv("TRI_SCAN_W128")) : 3;  // 128-byte TMA rows: bit 0 fp32, bit 1 fp64
 
 constexpr int ONCHIP_THREADS = 512;
 constexpr int SPLIT_K1MAX = 10;  // deepest k one sliding-window pass holds in smem (T = 256)
@@ -672,16 +673,18 @@ cudaError_t launch_stream(const tri_plan_s* p, const void* a, const void* b, con
 // swizzle; fp32: 32-byte rows, 32B swizzle), box [1][32][8] = one 256-row window
 // of one system per array; every coordinate fits int32 for any n, m of the API
 template <typename T>
-bool tma_map_sys_rows8(CUtensorMap* tm, const void* base, int64_t n, int64_t m, int sys_per_box = 1) {
+bool tma_map_sys_rows8(CUtensorMap* tm, const void* base, int64_t n, int64_t m, int sys_per_box = 1,
+                       bool w128 = false) {
     auto enc = tma_encoder();
     if (!enc) return false;
-    cuuint64_t dims[3] = {8, (cuuint64_t)(n / 8), (cuuint64_t)m};
-    cuuint64_t strides[2] = {8 * sizeof(T), (cuuint64_t)n * sizeof(T)};
-    cuuint32_t box[3] = {8, 32, (cuuint32_t)sys_per_box};
+    const int rw = w128 ? 128 / (int)sizeof(T) : 8;  // elements per tensor row (w128: 128-byte rows)
+    cuuint64_t dims[3] = {(cuuint64_t)rw, (cuuint64_t)(n / rw), (cuuint64_t)m};
+    cuuint64_t strides[2] = {(cuuint64_t)rw * sizeof(T), (cuuint64_t)n * sizeof(T)};
+    cuuint32_t box[3] = {(cuuint32_t)rw, (cuuint32_t)(SC_W / rw), (cuuint32_t)sys_per_box};
     cuuint32_t es[3] = {1, 1, 1};
     return enc(tm, sizeof(T) == 8 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT64 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3,
                const_cast<void*>(base), dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
-               sizeof(T) == 8 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_32B,
+               w128 ? CU_TENSOR_MAP_SWIZZLE_128B : sizeof(T) == 8 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_32B,
                CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
@@ -712,9 +715,13 @@ cudaError_t launch_scan(const tri_plan_s* p, const void* a, const void* b, const
     StreamMaps tm;
     const int64_t n = p->n, m = p->m;
     const int S = p->sk_S;
+    // 128-byte TMA rows (n % 32 fp32 / n % 16 fp64; the k_scan chain and one-window
+    // paths): one TMA request per 128 bytes (fp32 c4: 0.99 -> 0.84 ms)
+    const bool w128 = S == 1 && n % (128 / (int)sizeof(T)) == 0 && (g_scan_w128 & (sizeof(T) == 4 ? 1 : 2)) &&
+                      !(p->sk_nc == 1 && g_scan1 && p->n <= 3 * SC_W / 4) && !(p->sk_nc >= 2 && g_scan_rs);
     if (S == 1) {
-        if (!tma_map_sys_rows8<T>(&tm.a, a, n, m) || !tma_map_sys_rows8<T>(&tm.b, b, n, m) ||
-            !tma_map_sys_rows8<T>(&tm.c, c, n, m) || !tma_map_sys_rows8<T>(&tm.d, d, n, m))
+        if (!tma_map_sys_rows8<T>(&tm.a, a, n, m, 1, w128) || !tma_map_sys_rows8<T>(&tm.b, b, n, m, 1, w128) ||
+            !tma_map_sys_rows8<T>(&tm.c, c, n, m, 1, w128) || !tma_map_sys_rows8<T>(&tm.d, d, n, m, 1, w128))
             return cudaErrorNotSupported;
     } else {
         const int64_t ms = p->ms, nb = m / p->ms;
@@ -726,6 +733,7 @@ cudaError_t launch_scan(const tri_plan_s* p, const void* a, const void* b, const
     A.x = (T*)x;
     A.spill = (T*)p->scratch;
     A.n = p->n; A.m = p->m; A.ms = p->ms; A.NC = p->sk_nc; A.S_on = p->sk_son; A.delta = p->sk_delta;
+    A.w128 = w128 ? 1 : 0;
     A.prof = (unsigned long long*)g_fused_prof;
     A.dbg = g_fused_dbg_mode;
     if (S == 1 && p->sk_nc >= 2 && g_scan_rs) {  // role-split warps (k_scan_rs.cuh)
