@@ -42,6 +42,7 @@ struct ScanMCArgs {
     // of the slice (null: the system's start, (1, 0, 0)); xe = x after the slice
     // (null: 0, the system's end)
     int keep_a0, keep_cn;
+    int w128;     // tensor view with 128-byte rows (k_scan.cuh)
     const T* s0;
     const T* xe;
 };
@@ -147,7 +148,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant
     auto issue = [&](int g) {
         const int w = win_of(g);
         if (MODE < 2) {
-            const int y = w * (SC_W / 8);
+            const int y = w * (p.w128 ? SC_W * (int)sizeof(T) / 128 : SC_W / 8);
             sk_expect(&in_full[pw], (unsigned)(4 * SC_W * sizeof(T)));
             sc_tma3d(ib + 0 * SC_W, &tm.a, y, (int)q, &in_full[pw], pol_in);
             sc_tma3d(ib + 1 * SC_W, &tm.b, y, (int)q, &in_full[pw], pol_in);
@@ -189,7 +190,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant
         if (MODE == 0) {
             // ---- the window's forward map (product of the lane segment maps)
             T ra[SC_R], rb[SC_R], rc[SC_R], rd[SC_R];
-            sc_ld_rows(ib, lane, ra, rb, rc, rd);
+            sc_ld_rows_any(ib, lane, p.w128 != 0, ra, rb, rc, rd);
             sc_release_buf();  // this warp's reads of the buffer before the TMA refill
             if (lane == 0 && g + SC_NW < nwin) issue(g + SC_NW);
             if (edge) sc_fix_rows<T>(i0, n, ra, rb, rc, rd, p.keep_a0, p.keep_cn);
@@ -207,7 +208,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant
         } else if (MODE == 1) {
             // ---- forward replay from the chunk's / previous window's state
             T ra[SC_R], rb[SC_R], rc[SC_R], rd[SC_R];
-            sc_ld_rows(ib, lane, ra, rb, rc, rd);
+            sc_ld_rows_any(ib, lane, p.w128 != 0, ra, rb, rc, rd);
             if (edge) sc_fix_rows<T>(i0, n, ra, rb, rc, rd, p.keep_a0, p.keep_cn);
             const int nvalid = (int)(n - i0 < 0 ? 0 : n - i0 < SC_R ? n - i0 : SC_R);
             const bool tr = p.keep_cn && nvalid < SC_R;  // transparent padding rows (slice of a larger system)

@@ -778,10 +778,12 @@ template <typename T>
 cudaError_t scan_mc_setup(const tri_plan_s* p, const void* a, const void* b, const void* c, const void* d, void* x,
                           StreamMaps& tm, ScanMCArgs<T>& A, int& smem) {
     const int64_t n = p->n, m = p->m;
-    if (a && (!tma_map_sys_rows8<T>(&tm.a, a, n, m) || !tma_map_sys_rows8<T>(&tm.b, b, n, m) ||
-              !tma_map_sys_rows8<T>(&tm.c, c, n, m) || !tma_map_sys_rows8<T>(&tm.d, d, n, m)))
+    const bool w = n % (128 / (int)sizeof(T)) == 0 && (g_scan_w128 & (sizeof(T) == 4 ? 1 : 2));
+    if (a && (!tma_map_sys_rows8<T>(&tm.a, a, n, m, 1, w) || !tma_map_sys_rows8<T>(&tm.b, b, n, m, 1, w) ||
+              !tma_map_sys_rows8<T>(&tm.c, c, n, m, 1, w) || !tma_map_sys_rows8<T>(&tm.d, d, n, m, 1, w)))
         return cudaErrorNotSupported;
     A = ScanMCArgs<T>{};
+    A.w128 = w ? 1 : 0;
     A.x = (T*)x;
     A.cd = (T*)p->scratch;
     const int64_t mp = p->m * (int64_t)p->mc_P;
