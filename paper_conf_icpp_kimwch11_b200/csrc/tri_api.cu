@@ -106,7 +106,7 @@ int scan_systems(int64_t n, int64_t m, tri_dtype t, tri_layout layout) {
     // 8: a window's row of S systems is 64 B (fp64) / 32 B (fp32), at least one
     // whole DRAM sector per TMA row (S = 2 fp64 measured 2x slower: half sectors)
     const int smin = t == TRI_F64 ? 2 : 4;
-    if (g_scan_s_il == 2 || g_scan_s_il == 4 || g_scan_s_il == 8) return std::max(smin, g_scan_s_il);
+    if (g_scan_s_il == 2 || g_scan_s_il == 4 || g_scan_s_il == 8 || g_scan_s_il == 16) return std::max(smin, g_scan_s_il);
     return 8;
 }
 bool scan_ok(int64_t n, int64_t m, tri_dtype t, tri_layout layout, int64_t ms = -1) {
@@ -767,7 +767,7 @@ cudaError_t launch_scan(const tri_plan_s* p, const void* a, const void* b, const
     const size_t smem = (size_t)SCLayout<T>::smem_bytes(p->sk_nc, p->sk_delta, son_or_buf);
     const bool pr = A.prof != nullptr;
     void* kern = S == 1 ? scan_kernel<T, 1>(pr) : S == 2 ? scan_kernel<T, 2>(pr) : S == 4 ? scan_kernel<T, 4>(pr)
-                                                                                 : scan_kernel<T, 8>(pr);
+                 : S == 8 ? scan_kernel<T, 8>(pr) : scan_kernel<T, 16>(pr);
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     void* args[] = {(void*)&tm, (void*)&A};
