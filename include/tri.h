@@ -9,12 +9,16 @@
  * system into 2^k interleaved independent subsystems, then thread-level
  * parallel Thomas (Eqs 2-4) solves each subsystem with one
  * thread.  The transition point k is chosen at plan time from n, m, the dtype
- * and the SM count; tri_plan_set_k overrides it.
+ * and the SM count; tri_plan_set_k overrides it.  At k = 0 (the
+ * paper's rule for M > P) the planner's SCAN / SCAN_MC variants run
+ * p-Thomas with each system spread over a warp's lanes (the forward sweep and
+ * back substitution as scans of segment maps, reading X21).
  *
  * Conventions common to every call:
  *   - Element (system q, row i), 0 <= q < m, 0 <= i < n, lives at
  *       TRI_LAYOUT_CONTIGUOUS :  [q*n + i]   (system-major)
  *       TRI_LAYOUT_INTERLEAVED:  [i*m + q]   (the paper's interleave)
+ *       TRI_LAYOUT_BATCHED    :  [(b*n + i)*ms + s] for q = b*ms + s (tri_plan_batched)
  *     in each of a, b, c, d, x; every array holds n*m elements of the dtype.
  *   - a[q][0] and c[q][n-1] lie outside A (Eq 1) and are IGNORED (read as 0,
  *     whatever they hold, including NaN) -- DESIGN.md reading X1.

@@ -12,9 +12,10 @@ import paper_conf_icpp_kimwch11_b200 as tri  # noqa: E402
 
 n, m = int(sys.argv[1]), int(sys.argv[2])
 dt = sys.argv[3] if len(sys.argv) > 3 else "f64"
-arrs = trigen.generate(n, m, dt, 0, "dd")
+lay = int(sys.argv[4]) if len(sys.argv) > 4 else 0
+arrs = trigen.generate(n, m, dt, lay, "dd")
 a, b, c, d = (torch.from_numpy(t).cuda() for t in arrs)
-plan = tri.Plan(n, m, tri.F64 if dt == "f64" else tri.F32, 0)
+plan = tri.Plan(n, m, tri.F64 if dt == "f64" else tri.F32, lay)
 plan.variant = tri.VARIANT_SCAN
 x = torch.empty_like(b)
 plan.solve(a, b, c, d, out=x)
@@ -33,9 +34,10 @@ for prof in (False, True):
     print(f"{'profiled' if prof else 'plain'}: {ms:.3f} ms  dbg={os.environ.get('TRI_FUSED_DBG_MODE', '0')}")
 tri.lib().tri_debug_set_profile(None)
 v = cnt.cpu().tolist()
-ncta = min(m, 148)
+S = 8 if lay == 1 else 1
+ncta = min(-(-m // S), 148)
 nw = int(os.environ.get("SC_NW", "12"))
-steps = m * ((n + 255) // 256) / ncta
+steps = -(-m // S) * ((n + 256 // S - 1) // (256 // S)) / ncta
 names = ["total", "wait input", "wait bar.sync", "handover section", "wait slot counter", "pre-handover compute",
          "post-handover (replays, stores)"]
 print(f"{ms * 1.965e6:.0f} cycles @1.965GHz, {steps:.0f} steps per CTA, {ms * 1.965e6 / steps:.0f} cycles/step; "
