@@ -57,6 +57,17 @@ constexpr int SC_NCMAX = 4096;
 #ifndef SC_DB
 #define SC_DB 2                    // 2 = the per-dtype default above
 #endif
+// cache policies (A/B macros): inputs streamed once (evict_first), spilled slots
+// re-read one system later (evict_last), x written once (.cs streaming store)
+#ifndef SC_POL_IN
+#define SC_POL_IN sk_policy_evict_first()
+#endif
+#ifndef SC_POL_SP
+#define SC_POL_SP sk_policy_evict_last()
+#endif
+#ifndef SC_XST
+#define SC_XST "st.global.cs"
+#endif
 #ifndef SC_LATE
 #define SC_LATE 0                  // chained windows: 1 = refill at the end of the step
 #endif     // windows per system (per-slot counters live in smem)
@@ -458,7 +469,7 @@ __device__ __forceinline__ void sc_store_x(T* xo, int64_t rmax, const T (&xv)[SC
         if constexpr (sizeof(T) == 8) {
 #pragma unroll
             for (int t = 0; t < SC_R; t += 4)
-                asm volatile("st.global.cs.v4.f64 [%0], {%1, %2, %3, %4};" ::"l"(xo + t), "d"(xv[t]), "d"(xv[t + 1]),
+                asm volatile(SC_XST ".v4.f64 [%0], {%1, %2, %3, %4};" ::"l"(xo + t), "d"(xv[t]), "d"(xv[t + 1]),
                              "d"(xv[t + 2]), "d"(xv[t + 3])
                              : "memory");
         } else {
@@ -513,8 +524,8 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
     const int pw = warp;
     const int ls = lane % S, seg = lane / S;
     T* ib = reinterpret_cast<T*>(sbase + L::off_in + pw * L::in_stride);
-    const uint64_t pol_in = sk_policy_evict_first();
-    const uint64_t pol_sp = sk_policy_evict_last();
+    const uint64_t pol_in = SC_POL_IN;
+    const uint64_t pol_sp = SC_POL_SP;
     auto issue_to = [&](int jj, int ww, T* buf, uint64_t* bar) {
         const int q = (int)(blockIdx.x + (int64_t)jj * gridDim.x);
         sk_expect(bar, (unsigned)(4 * SC_W * sizeof(T)));
