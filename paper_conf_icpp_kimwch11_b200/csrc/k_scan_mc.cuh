@@ -45,6 +45,10 @@ struct ScanMCArgs {
     int w128;     // tensor view with 128-byte rows (k_scan.cuh)
     const T* s0;
     const T* xe;
+    // look-back path (k_scan_mc_lb): small-chunk records (x after each at [14]);
+    // null otherwise
+    const T* xafter;
+    int NCWs, Ps;
 };
 
 template <typename T>
@@ -173,7 +177,9 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant
         ps0 = __shfl_sync(0xffffffffu, fma(R.c, t0, R.d * q0), 0);
         de0 = __shfl_sync(0xffffffffu, fma(R.e, t0, fma(R.f, q0, R.g * e0)), 0);
     }
-    if (MODE == 2 && warp == 0) {  // x after the chunk = (B_{ch+1} ... B_{P-1})(x_end), x_end = 0 or the slice's
+    if (MODE == 2 && p.xafter) {  // look-back path: x after the small chunk that ends this chunk
+        xa0 = p.xafter[(int64_t)((q * p.Ps + (w0 + nwin + p.NCWs - 1) / p.NCWs - 1)) * 16 + 14];
+    } else if (MODE == 2 && warp == 0) {  // x after the chunk = (B_{ch+1} ... B_{P-1})(x_end), x_end = 0 or the slice's
         T al, be;
         smc_reduce_bwd(p.cbm + 8 * (q * p.P + ch + 1), p.P - 1 - ch, lane, al, be);
         const T xend = p.xe ? p.xe[0] : T(0);
@@ -299,6 +305,304 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant
             smc_reduce_bwd(wm, nwin, lane, al, be);
             if (lane == 0) { p.cbm[8 * (int64_t)blockIdx.x] = al; p.cbm[8 * (int64_t)blockIdx.x + 1] = be; }
         }
+    }
+}
+
+// ---- SCAN_MC with passes 0 and 1 fused by a decoupled look-back over small
+// chunks (TRI_SCAN_MC_LB): HBM traffic 4 + 2 (+ the
+// L2 re-read of each chunk) + 2 + 1 = 9 arrays instead of 13.
+// Persistent CTAs take chunks of NCWs windows in ticket order (an atomic
+// counter, so a CTA only ever waits on chunks that started before it).  Per
+// chunk: phase A = every window's forward map (as pass 0) and the chunk's
+// aggregate map, published with flag 1; warp 0 looks back over the earlier
+// chunks of the system (32 flags per round: the nearest inclusive state and
+// the aggregates after it) and publishes the chunk's inclusive state with flag
+// 2; phase B = pass 1 on the chunk (re-read from L2, prefetched during the
+// look-back).  k_scan_mc_lb_fin then turns the chunks' backward maps into the x
+// after every chunk, which pass 2 (k_scan_mc<2>, big chunks that are unions of
+// small ones) reads instead of reducing chunk maps.
+// Measured (c3, fp64 n = 2^24, B200; profiles/r01_ncu_c3_scanmc_lb.txt): correct
+// and bitwise reproducible, DRAM traffic as designed (586 MB read + 219 MB
+// written by the look-back kernel: the L2 re-read hits), but the kernel runs at
+// 3.3 TB/s -- 36 % of stall samples at __syncthreads while warp 0 reduces the
+// chunk and looks back -- so the solve takes 0.30-0.33 ms against 0.29 ms for
+// the three-pass path (small chunks of 24 / 32 / 48 / 64 / 80 windows: 0.39 /
+// 0.35 / 0.31-0.34 / 0.30-0.32 / 0.32 ms).  Kept off by default
+// (TRI_SCAN_MC_LB=0); the lever is to overlap the look-back of chunk t with
+// phase A of chunk t + 1 (a dedicated look-back warp, two chunks per CTA in L2).
+// record per small chunk (16 values): [0..6] aggregate map, [8..10] inclusive
+// state, [12..13] backward map (al, be), [14] x after the chunk
+constexpr int SMC_REC = 16;
+
+__device__ __forceinline__ unsigned smc_ld_acquire_gpu(const unsigned* p) {
+    unsigned v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void smc_st_release_gpu(unsigned* p, unsigned v) {
+    asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+template <typename T>
+struct ScanMCLB {
+    T* rec;            // [m Ps][SMC_REC]
+    unsigned* flag;    // [m Ps] (zeroed before the launch), then the ticket counter at [m Ps]
+    int NCWs, Ps;      // windows per small chunk, small chunks per system
+};
+
+template <typename T>
+__global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc_lb(const __grid_constant__ StreamMaps tm, ScanMCArgs<T> p,
+                                                               ScanMCLB<T> lb) {
+    using L = SMCLayout<T>;
+    extern __shared__ __align__(16) unsigned char smc_smem_raw[];
+    __shared__ int s_tk[2];
+    __shared__ T s_st[4];
+    unsigned char* sbase = smc_smem_raw + ((1024 - ((unsigned)__cvta_generic_to_shared(smc_smem_raw) & 1023)) & 1023);
+    uint64_t* in_full = reinterpret_cast<uint64_t*>(sbase + L::off_bar);
+    T* hv = reinterpret_cast<T*>(sbase + L::off_hv);
+    T* wm0 = reinterpret_cast<T*>(sbase + L::off_wm);
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, pw = warp;
+    if (threadIdx.x == 0) {
+        for (int i = 0; i < SC_NW; ++i) sk_bar_init(&in_full[i], 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        s_tk[0] = (int)atomicAdd(&lb.flag[p.m * (int64_t)lb.Ps], 1u);
+    }
+    __syncthreads();
+    const int64_t n = p.n;
+    const int NC = p.NC, NCW = lb.NCWs;
+    const int total = (int)(p.m * lb.Ps);
+    T* ib = reinterpret_cast<T*>(sbase + L::off_in + pw * L::in_stride);
+    const unsigned ib_s = (unsigned)__cvta_generic_to_shared(ib);
+    (void)ib_s;
+    const uint64_t pol_a = sk_policy_evict_normal();  // phase A: keep the chunk in L2 for phase B
+    const uint64_t pol_b = sk_policy_evict_first();   // phase B: last use
+    auto issue = [&](int q, int w, uint64_t pol) {
+        const int y = w * (p.w128 ? SC_W * (int)sizeof(T) / 128 : SC_W / 8);
+        sk_expect(&in_full[pw], (unsigned)(4 * SC_W * sizeof(T)));
+        sc_tma3d(ib + 0 * SC_W, &tm.a, y, q, &in_full[pw], pol);
+        sc_tma3d(ib + 1 * SC_W, &tm.b, y, q, &in_full[pw], pol);
+        sc_tma3d(ib + 2 * SC_W, &tm.c, y, q, &in_full[pw], pol);
+        sc_tma3d(ib + 3 * SC_W, &tm.d, y, q, &in_full[pw], pol);
+    };
+    unsigned ph = 0;
+    int par = 0;
+    int t = s_tk[0];
+    const int pi = (pw + SC_NW - 1) % SC_NW;
+    if (t < total && lane == 0) {
+        const int q = t / lb.Ps, ch = t - q * lb.Ps;
+        if (pw < min(NC, ch * NCW + NCW) - ch * NCW) issue(q, ch * NCW + pw, pol_a);
+    }
+    while (t < total) {
+        const int q = t / lb.Ps, ch = t - q * lb.Ps;
+        const int w0 = ch * NCW;
+        const int nwin = min(NC, w0 + NCW) - w0;
+        T* wm = wm0 + par * 8 * NCW;
+        // the next chunk's ticket (read after the barrier that ends phase A)
+        if (warp == 1 && lane == 0) s_tk[par ^ 1] = (int)atomicAdd(&lb.flag[total], 1u);
+        // ---- phase A: window forward maps
+        for (int g = pw; g < nwin; g += SC_NW) {
+            const int w = w0 + g;
+            const int64_t i0 = (int64_t)w * SC_W + lane * SC_R;
+            const bool edge = w == 0 || (int64_t)(w + 1) * SC_W > n;
+            sk_wait(&in_full[pw], ph);
+            ph ^= 1u;
+            T ra[SC_R], rb[SC_R], rc[SC_R], rd[SC_R];
+            sc_ld_rows_any(ib, lane, p.w128 != 0, ra, rb, rc, rd);
+            sc_release_buf();
+            if (lane == 0) {
+                if (g + SC_NW < nwin) issue((int)q, w + SC_NW, pol_a);
+                else issue((int)q, w0 + pw, pol_b);  // phase B's first window, during the look-back
+            }
+            if (edge) sc_fix_rows<T>(i0, n, ra, rb, rc, rd, 0, 0);
+            SKMat<T> M = sc_fwd_map(ra, rb, rc, rd);
+#pragma unroll
+            for (int d = 1; d < 32; d <<= 1) {
+                const SKMat<T> o = sk_shfl_down(M, d);
+                if ((lane & (2 * d - 1)) == 0) { M = sk_compose(o, M); smc_rescale(M); }
+            }
+            if (lane == 0) {
+                T* s = wm + 8 * g;
+                s[0] = M.a; s[1] = M.b; s[2] = M.c; s[3] = M.d; s[4] = M.e; s[5] = M.f; s[6] = M.g;
+            }
+        }
+        __syncthreads();
+        if (warp == 0) {
+            // aggregate of the chunk, published with flag 1
+            const SKMat<T> R = smc_reduce_fwd(wm, nwin, lane);  // lane 0
+            T* rec = lb.rec + (int64_t)t * SMC_REC;
+            unsigned* fl = lb.flag;
+            if (lane == 0 && ch > 0) {
+                __stcg(rec + 0, R.a); __stcg(rec + 1, R.b); __stcg(rec + 2, R.c); __stcg(rec + 3, R.d);
+                __stcg(rec + 4, R.e); __stcg(rec + 5, R.f); __stcg(rec + 6, R.g);
+                smc_st_release_gpu(fl + t, 1u);  // release: the stores above are visible first
+            }
+            // look-back with a FIXED structure (bitwise reproducible): incoming state =
+            // A_{t-1} ... A_{b+1} S_b, b = the chunk of the system at the largest multiple
+            // of 32 below ch (S_b inclusive, published with flag 2), so one round of 32
+            // flags; ch <= 32 starts from the system start when b = 0 ... and b's own
+            // inclusive state is built the same way from its base
+            SKMat<T> acc{T(1), T(0), T(0), T(1), T(0), T(0), T(1)};
+            T th = T(1), ps = T(0), de = T(0);
+            if (ch > 0) {
+                const int tfirst = (int)(q * lb.Ps);
+                const int b = tfirst + ((ch - 1) / 32) * 32;  // base chunk (inclusive state)
+                const int nag = t - 1 - b;                     // aggregates after it, lanes 0 .. nag - 1
+                const int j = t - 1 - lane;
+                const unsigned want = lane < nag ? 1u : (lane == nag ? 2u : 0u);
+                while (true) {
+                    const unsigned v = want ? smc_ld_acquire_gpu(fl + j) : 0u;
+                    if (!__any_sync(0xffffffffu, v < want)) break;
+                    __nanosleep(32);
+                }
+                SKMat<T> A{T(1), T(0), T(0), T(1), T(0), T(0), T(1)};
+                if (lane < nag) {
+                    const T* r = lb.rec + (int64_t)j * SMC_REC;
+                    A = SKMat<T>{__ldcg(r + 0), __ldcg(r + 1), __ldcg(r + 2), __ldcg(r + 3), __ldcg(r + 4),
+                                 __ldcg(r + 5), __ldcg(r + 6)};
+                }
+#pragma unroll
+                for (int d = 1; d < 32; d <<= 1) {  // lane l: A_{j_l} ... A_{j_{l+2d-1}} (lane l latest)
+                    const SKMat<T> o = sk_shfl_down(A, d);
+                    if ((lane & (2 * d - 1)) == 0) { A = sk_compose(A, o); smc_rescale(A); }
+                }
+                acc.a = __shfl_sync(0xffffffffu, A.a, 0); acc.b = __shfl_sync(0xffffffffu, A.b, 0);
+                acc.c = __shfl_sync(0xffffffffu, A.c, 0); acc.d = __shfl_sync(0xffffffffu, A.d, 0);
+                acc.e = __shfl_sync(0xffffffffu, A.e, 0); acc.f = __shfl_sync(0xffffffffu, A.f, 0);
+                acc.g = __shfl_sync(0xffffffffu, A.g, 0);
+                const T* r = lb.rec + (int64_t)b * SMC_REC;
+                th = __ldcg(r + 8); ps = __ldcg(r + 9); de = __ldcg(r + 10);
+            }
+            const T it = fma(acc.a, th, acc.b * ps);
+            const T ip = fma(acc.c, th, acc.d * ps);
+            const T id = fma(acc.e, th, fma(acc.f, ps, acc.g * de));
+            // inclusive state of this chunk, published with flag 2
+            T ot = fma(R.a, it, R.b * ip), op = fma(R.c, it, R.d * ip), od = fma(R.e, it, fma(R.f, ip, R.g * id));
+            if (lane == 0) {
+                const T sc = sk_exp2_scale(ot);
+                ot *= sc; op *= sc; od *= sc;
+                __stcg(rec + 8, ot); __stcg(rec + 9, op); __stcg(rec + 10, od);
+                smc_st_release_gpu(fl + t, 2u);
+                const T si = sk_exp2_scale(it);
+                s_st[0] = it * si; s_st[1] = ip * si; s_st[2] = id * si;
+            }
+        }
+        __syncthreads();
+        const int tn = s_tk[par ^ 1];
+        // ---- phase B: forward replay (pass 1) from the chunk's incoming state
+        for (int g = pw; g < nwin; g += SC_NW) {
+            const int w = w0 + g;
+            const int64_t i0 = (int64_t)w * SC_W + lane * SC_R;
+            const bool edge = w == 0 || (int64_t)(w + 1) * SC_W > n;
+            sk_wait(&in_full[pw], ph);
+            ph ^= 1u;
+            T ra[SC_R], rb[SC_R], rc[SC_R], rd[SC_R];
+            sc_ld_rows_any(ib, lane, p.w128 != 0, ra, rb, rc, rd);
+            if (edge) sc_fix_rows<T>(i0, n, ra, rb, rc, rd, 0, 0);
+            SKMat<T> M = sc_fwd_map(ra, rb, rc, rd);
+            sc_fwd_scan(M, lane);
+            if (g > 0) asm volatile("bar.sync %0, 64;" ::"r"(1 + pi) : "memory");
+            T th, ps, de;
+            if (g == 0) {
+                th = s_st[0]; ps = s_st[1]; de = s_st[2];
+            } else {
+                th = hv[4 * pi + 0]; ps = hv[4 * pi + 1]; de = hv[4 * pi + 2];
+            }
+            const T ot = fma(M.a, th, M.b * ps);
+            const T op = fma(M.c, th, M.d * ps);
+            const T od = fma(M.e, th, fma(M.f, ps, M.g * de));
+            if (lane == 31) {
+                const T sc = sk_exp2_scale(ot);
+                hv[4 * pw + 0] = ot * sc; hv[4 * pw + 1] = op * sc; hv[4 * pw + 2] = od * sc;
+            }
+            if (g + 1 < nwin) asm volatile("bar.arrive %0, 64;" ::"r"(1 + pw) : "memory");
+            {
+                const T it_ = __shfl_up_sync(0xffffffffu, ot, 1);
+                const T ip = __shfl_up_sync(0xffffffffu, op, 1);
+                const T id = __shfl_up_sync(0xffffffffu, od, 1);
+                if (lane > 0) { th = it_; ps = ip; de = id; }
+            }
+            sc_release_buf();
+            if (lane == 0) {
+                if (g + SC_NW < nwin) {
+                    issue((int)q, w + SC_NW, pol_b);
+                } else if (tn < total) {  // the next chunk's first window for this warp
+                    const int qn = tn / lb.Ps, chn = tn - qn * lb.Ps;
+                    if (pw < min(NC, chn * NCW + NCW) - chn * NCW) issue(qn, chn * NCW + pw, pol_a);
+                }
+            }
+            T cp[SC_R], dp[SC_R];
+            sc_fwd_replay(ra, rb, rc, rd, th, ps, de, cp, dp);
+            T* dst = p.cd + (q * NC + w) * (int64_t)sc_slot_elems<T>();
+            if constexpr (sizeof(T) == 8) {
+#pragma unroll
+                for (int u = 0; u < SC_R; ++u)
+                    __stcg(reinterpret_cast<double2*>(dst + 2 * sc_chunk<T>(lane, u)), make_double2(cp[u], dp[u]));
+            } else {
+#pragma unroll
+                for (int u = 0; u < SC_R / 2; ++u)
+                    __stcg(reinterpret_cast<float4*>(dst + 4 * sc_chunk<T>(lane, u)),
+                           make_float4(cp[2 * u], dp[2 * u], cp[2 * u + 1], dp[2 * u + 1]));
+            }
+            T al, be;
+            sc_bwd_map(cp, dp, al, be);
+#pragma unroll
+            for (int d = 1; d < 32; d <<= 1) {
+                const T oa = __shfl_down_sync(0xffffffffu, al, d), ob = __shfl_down_sync(0xffffffffu, be, d);
+                if ((lane & (2 * d - 1)) == 0) { al = fma(be, oa, al); be = be * ob; }
+            }
+            if (lane == 0) { wm[8 * g] = al; wm[8 * g + 1] = be; }
+        }
+        // warps with no window in this chunk still prefetch the next one
+        if (pw >= nwin && lane == 0 && tn < total) {
+            const int qn = tn / lb.Ps, chn = tn - qn * lb.Ps;
+            if (pw < min(NC, chn * NCW + NCW) - chn * NCW) issue(qn, chn * NCW + pw, pol_a);
+        }
+        __syncthreads();
+        if (warp == 0) {
+            T al, be;
+            smc_reduce_bwd(wm, nwin, lane, al, be);
+            if (lane == 0) { lb.rec[(int64_t)t * SMC_REC + 12] = al; lb.rec[(int64_t)t * SMC_REC + 13] = be; }
+        }
+        t = tn;
+        par ^= 1;
+    }
+}
+
+// x after every small chunk from the chunks' backward maps (one CTA per system):
+// x_after(ch) = B_{ch+1}(... B_{Ps-1}(0)); written to rec[14]
+template <typename T>
+__global__ void __launch_bounds__(1024) k_scan_mc_lb_fin(ScanMCLB<T> lb) {
+    __shared__ T sa[32], sb[32];
+    const int64_t q = blockIdx.x;
+    const int Ps = lb.Ps, tid = threadIdx.x, lane = tid & 31, wp = tid >> 5;
+    T* rec = lb.rec + q * Ps * SMC_REC;
+    const int per = (Ps + 1023) / 1024, lo = min(Ps, tid * per), hi = min(Ps, lo + per);
+    T al = T(0), be = T(1);  // this thread's chunks composed: x_first(lo) = al + be x_after(hi - 1)
+    for (int i = hi - 1; i >= lo; --i) {
+        const T a2 = rec[(int64_t)i * SMC_REC + 12], b2 = rec[(int64_t)i * SMC_REC + 13];
+        al = fma(b2, al, a2);
+        be = b2 * be;
+    }
+    // exclusive suffix over threads: the map of all chunks after this thread's range
+    T sal = al, sbe = be;  // inclusive suffix within the warp (lane l: lanes l..31)
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        const T oa = __shfl_down_sync(0xffffffffu, sal, d), ob = __shfl_down_sync(0xffffffffu, sbe, d);
+        if (lane + d < 32) { sal = fma(sbe, oa, sal); sbe = sbe * ob; }
+    }
+    if (lane == 0) { sa[wp] = sal; sb[wp] = sbe; }
+    __syncthreads();
+    // x after warp wp's range: the warps after it applied to 0
+    T xw = T(0);
+    for (int v = 31; v > wp; --v) xw = fma(sb[v], xw, sa[v]);
+    // x after this thread's range: lanes after it in the warp, then xw
+    T ea = __shfl_down_sync(0xffffffffu, sal, 1), eb = __shfl_down_sync(0xffffffffu, sbe, 1);
+    if (lane == 31) { ea = T(0); eb = T(1); }
+    T x = fma(eb, xw, ea);
+    for (int i = hi - 1; i >= lo; --i) {
+        rec[(int64_t)i * SMC_REC + 14] = x;
+        x = fma(rec[(int64_t)i * SMC_REC + 13], x, rec[(int64_t)i * SMC_REC + 12]);
     }
 }
 

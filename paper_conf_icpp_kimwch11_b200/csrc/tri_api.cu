@@ -40,6 +40,8 @@ int env_int(const char* name, int dflt) {
 int g_tiled_waves1 = env_int("TRI_TILED_WAVES1", 1);
 int g_split_k1max = std::min(10, env_int("TRI_SPLIT_K1MAX", 10));  // steps kept in pass 1 (tuning)
 int g_tiled_waves2 = env_int("TRI_TILED_WAVES2", 3);  // measured best at c3 (1 / 3 waves)
+int g_scan_mc_lb = env_int("TRI_SCAN_MC_LB", 0);     // SCAN_MC: passes 0 + 1 fused by a look-back (tuning)
+int g_scan_mc_lbw = env_int("TRI_SCAN_MC_LBW", 24);   // SCAN_MC look-back: windows per small chunk
 int g_scan_delta = env_int("TRI_SCAN_DELTA", 8);      // SCAN: back-substitution lag in steps (tuning)
 int g_scan1 = getenv("TRI_SCAN1_OFF") ? 0 : 1;        // SCAN, one-window systems: chain-free kernel (A/B)
 int g_scan_rs = getenv("TRI_SCAN_RS") ? atoi(getenv("TRI_SCAN_RS")) : 0;  // SCAN: role-split kernel (A/B)
@@ -240,6 +242,7 @@ struct tri_plan_s {
     int sk_S;                    // SCAN: systems per window (1 contiguous; 2 / 4 / 8 interleaved)
     int64_t ms;                  // systems per batch (BATCHED; m otherwise)
     int mc_P, mc_NCW;            // SCAN_MC: chunks per system, windows per chunk
+    int mc_lb, mc_NCWs, mc_Ps;   // SCAN_MC look-back path: on, windows per small chunk, small chunks per system
     size_t smem_optin;
     void* scratch;
     size_t scratch_bytes;
@@ -401,7 +404,15 @@ void plan_geometry(tri_plan_s* p) {
         p->sk_nc = (int)NC;
         int64_t P = std::max(cdiv(p->sms, m), cdiv(NC, SMC_WMAX));
         P = std::min(P, NC);
-        const int64_t NCW = cdiv(NC, P);
+        int64_t NCW = cdiv(NC, P);
+        p->mc_lb = 0; p->mc_NCWs = 0; p->mc_Ps = 0;
+        if (g_scan_mc_lb && g_scan_mc_lbw >= 1 && 2 * g_scan_mc_lbw <= SMC_WMAX) {
+            // pass 2's chunks are unions of the look-back's small chunks
+            p->mc_lb = 1;
+            p->mc_NCWs = g_scan_mc_lbw;
+            p->mc_Ps = (int)cdiv(NC, p->mc_NCWs);
+            NCW = std::min<int64_t>(SMC_WMAX / p->mc_NCWs * p->mc_NCWs, cdiv(NCW, p->mc_NCWs) * p->mc_NCWs);
+        }
         p->mc_NCW = (int)NCW;
         p->mc_P = (int)cdiv(NC, NCW);
         p->sk_grid = (int)(m * p->mc_P);
@@ -423,9 +434,10 @@ void plan_geometry(tri_plan_s* p) {
 }
 
 size_t scratch_need(const tri_plan_s* p) {
-    if (p->variant == TRI_VARIANT_SCAN_MC)  // c', d' per window + the chunk maps
+    if (p->variant == TRI_VARIANT_SCAN_MC)  // c', d' per window + the chunk maps (+ the look-back records and flags)
         return ((size_t)p->m * (size_t)p->sk_nc * (size_t)sc_slot_elems<double>() +
-                (size_t)p->m * (size_t)p->mc_P * 16 + 16) * esize(p->dtype);
+                (size_t)p->m * (size_t)p->mc_P * 16 + 16) * esize(p->dtype) +
+               (p->mc_lb ? (size_t)p->m * (size_t)p->mc_Ps * (SMC_REC * esize(p->dtype) + 4) + 256 : 0);
     if (p->variant == TRI_VARIANT_SCAN)
         return (p->sk_nc == 1 && p->sk_S == 1) ? 0
                              : (size_t)p->sk_grid * (size_t)std::max(0, p->sk_nc + p->sk_delta - p->sk_son) *
@@ -811,6 +823,27 @@ cudaError_t launch_scan_mc(const tri_plan_s* p, const void* a, const void* b, co
     int smem = 0;
     cudaError_t e = scan_mc_setup<T>(p, a, b, c, d, x, tm, A, smem);
     if (e != cudaSuccess) return e;
+    if (p->mc_lb) {
+        ScanMCLB<T> lb;
+        lb.rec = scan_mc_slice_vals<T>(p) + 16;
+        const int64_t nrec = p->m * (int64_t)p->mc_Ps;
+        lb.flag = (unsigned*)(lb.rec + nrec * SMC_REC);
+        lb.NCWs = p->mc_NCWs;
+        lb.Ps = p->mc_Ps;
+        const int smem_lb = SMCLayout<T>::smem_bytes(2 * p->mc_NCWs);
+        e = cudaFuncSetAttribute(k_scan_mc_lb<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_lb);
+        if (e != cudaSuccess) return e;
+        e = cudaMemsetAsync(lb.flag, 0, (size_t)(nrec + 1) * sizeof(unsigned), st);
+        if (e != cudaSuccess) return e;
+        const int grid = (int)std::min<int64_t>(p->sms, nrec);
+        k_scan_mc_lb<T><<<grid, SC_THREADS, smem_lb, st>>>(tm, A, lb);
+        k_scan_mc_lb_fin<T><<<(unsigned)p->m, 1024, 0, st>>>(lb);
+        A.xafter = lb.rec;
+        A.NCWs = p->mc_NCWs;
+        A.Ps = p->mc_Ps;
+        k_scan_mc<T, 2><<<p->sk_grid, SC_THREADS, smem, st>>>(tm, A);
+        return cudaGetLastError();
+    }
     k_scan_mc<T, 0><<<p->sk_grid, SC_THREADS, smem, st>>>(tm, A);
     k_scan_mc<T, 1><<<p->sk_grid, SC_THREADS, smem, st>>>(tm, A);
     k_scan_mc<T, 2><<<p->sk_grid, SC_THREADS, smem, st>>>(tm, A);

@@ -822,3 +822,32 @@ def test_scan_role_split_variant(cuda_ok):
     env = dict(os.environ, TRI_SCAN_RS="1")
     r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, timeout=300)
     assert r.returncode == 0 and "ok" in r.stdout, r.stdout[-2000:] + r.stderr[-2000:]
+
+
+def test_scan_mc_lookback_variant(cuda_ok):
+    """SCAN_MC with passes 0 and 1 fused by a look-back over small chunks
+    (k_scan_mc_lb, selected by TRI_SCAN_MC_LB=1 at library load, hence a
+    subprocess): parity against the oracle on ragged chunk counts, fp64 / fp32,
+    several systems, and bitwise-identical repeated solves (the look-back has a
+    fixed composition order)."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    code = (
+        "import sys; sys.path.insert(0, %r)\n"
+        "import torch\n"
+        "from tests._helpers import gen, gpu_solve, check_parity\n"
+        "import paper_conf_icpp_kimwch11_b200 as tri\n"
+        "for dt, n, m in [('f64', 65536, 1), ('f64', 256 * 1000 + 8, 1), ('f32', 256 * 2100 - 16, 1),\n"
+        "                 ('f64', 256 * 130, 3), ('f64', 256 * 40 * 33, 2), ('f64', 1 << 22, 1)]:\n"
+        "    arrs = gen(n, m, dt, 0)\n"
+        "    x, plan = gpu_solve(n, m, arrs, dt, 0, variant=tri.VARIANT_SCAN_MC)\n"
+        "    check_parity(n, m, arrs, x, dt, 0)\n"
+        "    x2, _ = gpu_solve(n, m, arrs, dt, 0, plan=plan)\n"
+        "    assert torch.equal(torch.as_tensor(x), torch.as_tensor(x2)), (dt, n, m)\n"
+        "print('ok')\n" % root)
+    for w in ("24", "64"):
+        env = dict(os.environ, TRI_SCAN_MC_LB="1", TRI_SCAN_MC_LBW=w)
+        r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, timeout=300)
+        assert r.returncode == 0 and "ok" in r.stdout, r.stdout[-2000:] + r.stderr[-2000:]
