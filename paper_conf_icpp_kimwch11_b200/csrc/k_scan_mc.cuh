@@ -330,6 +330,12 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant
 // 0.35 / 0.31-0.34 / 0.30-0.32 / 0.32 ms).  Kept off by default
 // (TRI_SCAN_MC_LB=0); the lever is to overlap the look-back of chunk t with
 // phase A of chunk t + 1 (a dedicated look-back warp, two chunks per CTA in L2).
+// Tried and measured slower (not kept): a lag-1 pipeline in which warp 0 looks
+// back on chunk t - 1 after phase A of chunk t (so predecessors have had a phase
+// longer to publish): correct, but 0.33-0.41 ms -- barrier stalls rose to 43 %
+// and two chunks per CTA pushed the L2 re-read out (778 MB DRAM read;
+// profiles/r01_ncu_c3_scanmc_lb_lag1.txt): the bubble is warp 0's serial
+// reduce + publish, not waiting on flags.
 // record per small chunk (16 values): [0..6] aggregate map, [8..10] inclusive
 // state, [12..13] backward map (al, be), [14] x after the chunk
 constexpr int SMC_REC = 16;
