@@ -335,7 +335,11 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant
 // longer to publish): correct, but 0.33-0.41 ms -- barrier stalls rose to 43 %
 // and two chunks per CTA pushed the L2 re-read out (778 MB DRAM read;
 // profiles/r01_ncu_c3_scanmc_lb_lag1.txt): the bubble is warp 0's serial
-// reduce + publish, not waiting on flags.
+// reduce + publish, not waiting on flags.  Also measured and not kept: the
+// other warps only ARRIVE at the post-phase-A barrier (warp 0 alone waits) with
+// tickets claimed two chunks ahead: correct, but 2.3-2.7 ms -- a ticket
+// claimed before its CTA can start it stalls every later chunk's look-back on
+// its aggregate, so tickets must stay just-in-time.
 // record per small chunk (16 values): [0..6] aggregate map, [8..10] inclusive
 // state, [12..13] backward map (al, be), [14] x after the chunk
 constexpr int SMC_REC = 16;
