@@ -327,7 +327,10 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant
 // 3.3 TB/s -- 36 % of stall samples at __syncthreads while warp 0 reduces the
 // chunk and looks back -- so the solve takes 0.30-0.33 ms against 0.29 ms for
 // the three-pass path (small chunks of 24 / 32 / 48 / 64 / 80 windows: 0.39 /
-// 0.35 / 0.31-0.34 / 0.30-0.32 / 0.32 ms).  Kept off by default
+// 0.35 / 0.31-0.34 / 0.30-0.32 / 0.32 ms).  Now only warp 0 waits at the end
+// of phase A (the other warps arrive and start phase B; the next ticket, claimed
+// just in time after the look-back, travels with the state hand-over):
+// 0.380 / 0.342 / 0.307 / 0.301 ms at 24 / 32 / 48 / 64 windows.  Kept off by default
 // (TRI_SCAN_MC_LB=0); the lever is to overlap the look-back of chunk t with
 // phase A of chunk t + 1 (a dedicated look-back warp, two chunks per CTA in L2).
 // Tried and measured slower (not kept): a lag-1 pipeline in which warp 0 looks
@@ -407,9 +410,8 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc_lb(const __grid_const
         const int q = t / lb.Ps, ch = t - q * lb.Ps;
         const int w0 = ch * NCW;
         const int nwin = min(NC, w0 + NCW) - w0;
-        T* wm = wm0 + par * 8 * NCW;
-        // the next chunk's ticket (read after the barrier that ends phase A)
-        if (warp == 1 && lane == 0) s_tk[par ^ 1] = (int)atomicAdd(&lb.flag[total], 1u);
+        T* wm = wm0 + par * 8 * NCW;          // forward window maps (phase A)
+        T* wmb = wm0 + (2 + par) * 8 * NCW;   // backward window maps (phase B)
         // ---- phase A: window forward maps
         for (int g = pw; g < nwin; g += SC_NW) {
             const int w = w0 + g;
@@ -436,7 +438,10 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc_lb(const __grid_const
                 s[0] = M.a; s[1] = M.b; s[2] = M.c; s[3] = M.d; s[4] = M.e; s[5] = M.f; s[6] = M.g;
             }
         }
-        __syncthreads();
+        // warp 0 waits for every warp's window maps; the others go straight on to
+        // phase B (their chain waits for warp 0's first window anyway)
+        if (warp == 0) asm volatile("bar.sync 13, %0;" ::"r"(SC_THREADS) : "memory");
+        else asm volatile("bar.arrive 13, %0;" ::"r"(SC_THREADS) : "memory");
         if (warp == 0) {
             // aggregate of the chunk, published with flag 1
             const SKMat<T> R = smc_reduce_fwd(wm, nwin, lane);  // lane 0
@@ -495,10 +500,14 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc_lb(const __grid_const
                 smc_st_release_gpu(fl + t, 2u);
                 const T si = sk_exp2_scale(it);
                 s_st[0] = it * si; s_st[1] = ip * si; s_st[2] = id * si;
+                s_tk[par ^ 1] = (int)atomicAdd(&lb.flag[total], 1u);  // the next chunk, just in time
             }
         }
-        __syncthreads();
-        const int tn = s_tk[par ^ 1];
+        __syncwarp();
+        // the next ticket: warp 0 from shared memory; the others through the chain
+        // (hv[4 w + 3], handed over with the state); warps with no window here after
+        // the end-of-chunk barrier
+        int tn = warp == 0 ? s_tk[par ^ 1] : total;
         // ---- phase B: forward replay (pass 1) from the chunk's incoming state
         for (int g = pw; g < nwin; g += SC_NW) {
             const int w = w0 + g;
@@ -517,6 +526,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc_lb(const __grid_const
                 th = s_st[0]; ps = s_st[1]; de = s_st[2];
             } else {
                 th = hv[4 * pi + 0]; ps = hv[4 * pi + 1]; de = hv[4 * pi + 2];
+                tn = (int)hv[4 * pi + 3];
             }
             const T ot = fma(M.a, th, M.b * ps);
             const T op = fma(M.c, th, M.d * ps);
@@ -524,6 +534,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc_lb(const __grid_const
             if (lane == 31) {
                 const T sc = sk_exp2_scale(ot);
                 hv[4 * pw + 0] = ot * sc; hv[4 * pw + 1] = op * sc; hv[4 * pw + 2] = od * sc;
+                hv[4 * pw + 3] = (T)tn;
             }
             if (g + 1 < nwin) asm volatile("bar.arrive %0, 64;" ::"r"(1 + pw) : "memory");
             {
@@ -561,17 +572,18 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc_lb(const __grid_const
                 const T oa = __shfl_down_sync(0xffffffffu, al, d), ob = __shfl_down_sync(0xffffffffu, be, d);
                 if ((lane & (2 * d - 1)) == 0) { al = fma(be, oa, al); be = be * ob; }
             }
-            if (lane == 0) { wm[8 * g] = al; wm[8 * g + 1] = be; }
+            if (lane == 0) { wmb[8 * g] = al; wmb[8 * g + 1] = be; }
         }
+        __syncthreads();
+        if (pw >= nwin) tn = s_tk[par ^ 1];
         // warps with no window in this chunk still prefetch the next one
         if (pw >= nwin && lane == 0 && tn < total) {
             const int qn = tn / lb.Ps, chn = tn - qn * lb.Ps;
             if (pw < min(NC, chn * NCW + NCW) - chn * NCW) issue(qn, chn * NCW + pw, pol_a);
         }
-        __syncthreads();
         if (warp == 0) {
             T al, be;
-            smc_reduce_bwd(wm, nwin, lane, al, be);
+            smc_reduce_bwd(wmb, nwin, lane, al, be);
             if (lane == 0) { lb.rec[(int64_t)t * SMC_REC + 12] = al; lb.rec[(int64_t)t * SMC_REC + 13] = be; }
         }
         t = tn;

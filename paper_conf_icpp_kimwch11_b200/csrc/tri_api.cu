@@ -830,7 +830,7 @@ cudaError_t launch_scan_mc(const tri_plan_s* p, const void* a, const void* b, co
         lb.flag = (unsigned*)(lb.rec + nrec * SMC_REC);
         lb.NCWs = p->mc_NCWs;
         lb.Ps = p->mc_Ps;
-        const int smem_lb = SMCLayout<T>::smem_bytes(2 * p->mc_NCWs);
+        const int smem_lb = SMCLayout<T>::smem_bytes(4 * p->mc_NCWs);
         e = cudaFuncSetAttribute(k_scan_mc_lb<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_lb);
         if (e != cudaSuccess) return e;
         e = cudaMemsetAsync(lb.flag, 0, (size_t)(nrec + 1) * sizeof(unsigned), st);
