@@ -41,7 +41,7 @@ int g_tiled_waves1 = env_int("TRI_TILED_WAVES1", 1);
 int g_split_k1max = std::min(10, env_int("TRI_SPLIT_K1MAX", 10));  // steps kept in pass 1 (tuning)
 int g_tiled_waves2 = env_int("TRI_TILED_WAVES2", 3);  // measured best at c3 (1 / 3 waves)
 int g_scan_mc_lb = env_int("TRI_SCAN_MC_LB", 0);     // SCAN_MC: passes 0 + 1 fused by a look-back (tuning)
-int g_scan_mc_lbw = env_int("TRI_SCAN_MC_LBW", 24);   // SCAN_MC look-back: windows per small chunk
+int g_scan_mc_lbw = env_int("TRI_SCAN_MC_LBW", 64);   // SCAN_MC look-back: windows per small chunk (64 measured best at c3)
 int g_scan_delta = env_int("TRI_SCAN_DELTA", 8);      // SCAN: back-substitution lag in steps (tuning)
 int g_scan1 = getenv("TRI_SCAN1_OFF") ? 0 : 1;        // SCAN, one-window systems: chain-free kernel (A/B)
 int g_scan_rs = getenv("TRI_SCAN_RS") ? atoi(getenv("TRI_SCAN_RS")) : 0;  // SCAN: role-split kernel (A/B)
