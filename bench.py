@@ -8,8 +8,13 @@ systems of n = 16384, contiguous), the config the metric's 1/2/4/8-GPU figures
 are quoted on; other configs via --config.  Inputs are synthetic (trigen,
 seeded), generated on the host and resident in HBM before the timed region.
 
-N > 1 (torchrun, one rank per GPU, NCCL): the m systems are sharded into
-contiguous ranges (no collective inside the solve); time = max over ranks.
+N > 1 (torchrun, one rank per GPU, NCCL): the m systems of the batched
+configs (c2, c4, c5) are sharded into contiguous ranges through
+paper_conf_icpp_kimwch11_b200.dist (strong scaling: rank r solves m/N systems;
+no collective inside the solve; time = max over ranks); the one-system configs
+(c1, c3) run as replicas (weak scaling).  The edge collectives (NCCL scatter of
+a, b, c, d from rank 0, gather of x) run on the real shards after the timed
+region and are reported in `collectives`, with a check of the gathered x.
 
 --impl reference times the CPU oracle (plain sequential Thomas, oracle/) on a
 bounded sample of the same workload -- the tier's reference arm.
@@ -49,10 +54,9 @@ def parse():
     ap.add_argument("--family", default="dd")
     ap.add_argument("--k", type=int, default=None, help="force the transition point k")
     ap.add_argument("--variant", type=int, default=None, help="force variant (1 onchip, 2 split, 3 fused)")
-    ap.add_argument("--scaling", default="weak", choices=["strong", "weak"],
-                    help="weak (default; the systems are independent, so every rank solves its own full "
-                         "batch of the config's m systems, no data-path collective); strong: the config's m is "
-                         "split over ranks")
+    ap.add_argument("--scaling", default=None, choices=["strong", "weak"],
+                    help="strong (default for the batched configs): the config's m systems are sharded over the "
+                         "ranks; weak (default for the one-system configs c1 / c3): every rank solves a replica")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-e2e", action="store_true")
@@ -129,54 +133,30 @@ def dist_env():
     return world, rank, local
 
 
-def method_arrays(plan, tri):
-    """Arrays of n*m*s bytes the plan's method moves per solve:
-    compulsory 5 + every materialised PCR pass + spilled Thomas intermediates."""
+def method_arrays(plan, tri, l2_bytes):
+    """Arrays of n*m*s bytes the plan's method moves per solve (SURVEY 8(d)
+    model): compulsory 5 + every materialised PCR pass + spilled Thomas
+    intermediates.  Superseded by the ncu-measured DRAM bytes when a traffic
+    file for this exact plan exists (roofline.method_source says which)."""
     v = plan.variant
     if v in (tri.VARIANT_WARP, tri.VARIANT_ONCHIP):
         return 5
     if v in (tri.VARIANT_FUSED, tri.VARIANT_STREAM, tri.VARIANT_SCAN):
         return 5  # c', d' stay in smem or in per-CTA scratch that stays in L2 (ncu: 5.0 arrays of DRAM traffic)
     if v == tri.VARIANT_SCAN_MC:
-        return 13  # read a, b, c, d twice; write + read c', d'; write x
+        return 9 if "lookback=0" not in plan.describe() else 13  # look-back: 4 + 2 + 2 + 1; three passes: + 4
     if plan.k == 0:
-        return 9  # read a, b, c, d; write + read c', d'; write x
-    # pass 1: read 4 + write 3; [pass 2: read 3 + write 3]; p-Thomas: read 3, c', d' 2 + 2, write x
-    return 15 if plan.launches == 2 else 21
-
-
-def time_collectives(n, m, s, world, rank, dev, tdt):
-    """NCCL edge collectives of SURVEY 8(e): rank 0 scatters a, b, c, d shards
-    and gathers x.  Returns (scatter ms, gather ms, bytes crossing NVLink), max
-    over ranks (CUDA events)."""
-    import torch
-    import torch.distributed as dist
-    per = -(-m // world)
-    recv = torch.empty(n * per, dtype=tdt, device=dev)
-    send = [torch.empty(n * per, dtype=tdt, device=dev) for _ in range(world)] if rank == 0 else None
-    res = []
-    for what in ("scatter", "gather"):
-        for it in range(2):  # one warm-up round
-            dist.barrier()
-            torch.cuda.synchronize()
-            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            e0.record()
-            for _ in range(4 if what == "scatter" else 1):
-                if what == "scatter":
-                    dist.scatter(recv, scatter_list=send, src=0)
-                else:
-                    dist.gather(recv, gather_list=send, dst=0)
-            e1.record()
-            torch.cuda.synchronize()
-        t = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        res.append(float(t.item()))
-    moved = (world - 1) * n * per * s
-    return res[0], res[1], 4 * moved, moved
+        # read a, b, c, d; write + read c', d'; write x -- unless the c', d' a wave
+        # of CTAs writes are read back (and L2-discarded) before they leave L2
+        inflight = 2 * plan.n * min(plan.m, 32 * 4 * 148) * (8 if "f64" in plan.describe() else 4)
+        return 5 if inflight < l2_bytes // 2 else 9
+    # pass 1: read 4 + write 3; each later pass: read 3 + write 3; p-Thomas: read 3, c', d' 2 + 2, write x
+    return 7 + 6 * (plan.launches - 2) + 8
 
 
 def cpu_oracle_time(n, mr, arrs, layout, budget_s=20.0):
-    """Time the oracle (as it stands) on the host cores over a bounded sample."""
+    """Time the oracle (as it stands) on the host cores over a bounded sample,
+    with every core the process may use and with one thread."""
     import oracle
     cores = len(os.sched_getaffinity(0))
     # sample: whole systems, as many as fit ~budget_s at ~50 Munk/s/core
@@ -187,8 +167,16 @@ def cpu_oracle_time(n, mr, arrs, layout, budget_s=20.0):
     t0 = time.perf_counter()
     oracle.solve_batch(n, mr, *arrs, layout=layout, q_begin=0, q_end=qs, nthreads=cores)
     dt = time.perf_counter() - t0
+    # one thread: a smaller sample (~3 s at ~50 Munk/s)
+    q1 = int(max(1, min(qs, 3.0 * 50e6 / n))) if layout == 0 else qs
+    t0 = time.perf_counter()
+    oracle.solve_batch(n, mr, *arrs, layout=layout, q_begin=0, q_end=q1, nthreads=1)
+    dt1 = time.perf_counter() - t0
     return {"value": n * qs / dt / 1e6, "unit": "Munknowns/s", "cores": cores, "kind": "oracle",
-            "sample": f"{qs} of {mr} systems x n={n} (whole systems, {dt:.2f} s, {cores} threads over systems)"}
+            "hardware_concurrency": os.cpu_count(),
+            "sample": f"{qs} of {mr} systems x n={n} (whole systems, {dt:.2f} s, {cores} threads over systems)",
+            "t1": {"value": n * q1 / dt1 / 1e6, "unit": "Munknowns/s", "cores": 1,
+                   "sample": f"{q1} systems x n={n} ({dt1:.2f} s, one thread)"}}
 
 
 def run_reference(args):
@@ -220,7 +208,8 @@ def run_reference(args):
     v = n * qs / t / 1e6
     out = {"metric": METRIC, "value": v, "unit": "Munknowns/s", "impl": "reference", "n_gpus": args.gpus,
            "steps": args.steps, "warmup": args.warmup, "ms_per_step": t * 1e3, "higher_is_better": True,
-           "scaling": args.scaling, "vs_baseline": None, "dtype": dt, "data": "synthetic",
+           "scaling": args.scaling or ("weak" if m == 1 else "strong"), "vs_baseline": None, "dtype": dt,
+           "data": "synthetic",
            "config": {"workload": args.config, "desc": desc, "n": n, "m": m, "layout": layout,
                       "family": args.family},
            "cpu_baseline": {"value": v, "unit": "Munknowns/s", "cores": cores, "kind": "oracle",
@@ -239,6 +228,7 @@ def main():
 
     import trigen
     import paper_conf_icpp_kimwch11_b200 as tri
+    from paper_conf_icpp_kimwch11_b200 import dist as tdist
 
     world, rank, local = dist_env()
     if world > 1:
@@ -253,20 +243,28 @@ def main():
         layout = args.layout
     s = 8 if dt == "f64" else 4
     tdt = torch.float64 if dt == "f64" else torch.float32
-    if args.scaling == "strong":
-        q0, mr = tri.shard_range(m, world, rank)
+    td = tri.F64 if dt == "f64" else tri.F32
+    # strong scaling for the batched configs (the m systems sharded over the ranks,
+    # dist.shard_range); the one-system configs run as replicas (system q = rank)
+    scaling = args.scaling or ("weak" if m == 1 else "strong")
+    if scaling == "strong":
+        q0, mr = tdist.shard_range(m, world, rank)
+        m_all = m
     else:
         q0, mr = rank * m, m
-    m_all = m if args.scaling == "strong" else m * world
+        m_all = m * world
+    if mr == 0:
+        raise SystemExit(f"rank {rank}: no systems in its shard (m = {m} < N = {world}); use --scaling weak")
     seed = trigen.SEED_BASE + int(args.config[1])
 
-    # ---- inputs: seeded host generation of this rank's shard, then resident in HBM
+    # ---- inputs: seeded host generation of this rank's shard (global system
+    # indices q0 ..), then resident in HBM before the timed region
     pin = not args.no_e2e
     host = [torch.empty(n * mr, dtype=tdt, pin_memory=pin) for _ in range(4)]
     trigen.generate(n, mr, dt, layout, args.family, seed=seed, q0=q0, out=[t.numpy() for t in host])
     a, b, c, d = (t.to(dev, non_blocking=False) for t in host)
     x = torch.empty_like(b)
-    plan = tri.Plan(n, mr, tri.F64 if dt == "f64" else tri.F32, layout)
+    plan = tri.Plan(n, mr, td, layout)
     if args.variant is not None:
         plan.variant = args.variant
     if args.k is not None:
@@ -281,12 +279,19 @@ def main():
     flush_buf = torch.empty(2 * l2 // 4 + 1024, dtype=torch.int32, device=dev) if flush else None
     clean_buf = torch.ones(2 * l2 // 4 + 1024, dtype=torch.int32, device=dev) if flush else None
 
+    def flush_l2():
+        # outside the timed interval: write 2x L2 worth of bytes (evicts our data),
+        # then read another 2x L2 so the dirty lines are written back before the
+        # step instead of during it
+        flush_buf.add_(1)
+        clean_buf.sum()
+
     for _ in range(args.warmup):
         plan.solve(a, b, c, d, out=x, stream=stream)
     torch.cuda.synchronize()
     # the timed step replays the solve from a CUDA graph captured once: the same
     # kernels, without the per-call host latency that would otherwise sit inside
-    # the device-timed window of the small configs
+    # the device-timed window of the small configs (reported separately: `direct`)
     graph = None
     if not args.no_graph:
         cap = torch.cuda.Stream()
@@ -306,11 +311,7 @@ def main():
     with ClockSampler(dev.index) as clk:
         for i in range(args.steps):
             if flush:
-                # outside the timed interval: write 2x L2 worth of bytes (evicts our
-                # data), then read another 2x L2 so the dirty lines are written back
-                # before the step instead of during it
-                flush_buf.add_(1)
-                clean_buf.sum()
+                flush_l2()
             ev[i][0].record(stream)
             if graph is not None:
                 graph.replay()
@@ -322,11 +323,31 @@ def main():
         dist.barrier()
     step_ms = [e0.elapsed_time(e1) for e0, e1 in ev]
     t_step = sum(step_ms) / len(step_ms)
-    t_max = torch.tensor([t_step], dtype=torch.float64, device=dev)
-    if world > 1:
-        dist.all_reduce(t_max, op=dist.ReduceOp.MAX)
-    t_step_max = float(t_max.item())
+    t_step_max = tdist.max_over_ranks(t_step, device=dev)
     value = m_all * n / (t_step_max * 1e-3) / 1e6  # whole-job Munknowns/s
+
+    # ---- per-call latency of a direct (non-graph) tri_solve: idle GPU, events
+    # around one call, so the host-side cost of the call (ctypes, argument checks,
+    # launches) is inside the window; plus the host time of one call
+    direct = None
+    if graph is not None:
+        reps = max(3, min(args.steps, 20))
+        dms, hus = [], []
+        for _ in range(reps):
+            if flush:
+                flush_l2()
+            torch.cuda.synchronize()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            th0 = time.perf_counter()
+            plan.solve(a, b, c, d, out=x, stream=stream)
+            hus.append((time.perf_counter() - th0) * 1e6)
+            e1.record(stream)
+            torch.cuda.synchronize()
+            dms.append(e0.elapsed_time(e1))
+        direct = {"ms_per_step": statistics.median(dms), "host_us_per_call": statistics.median(hus),
+                  "how": "one Plan.solve (ctypes -> tri_solve) per step on an idle GPU, CUDA events around the call; "
+                         "host_us = Python + C host time of the call"}
 
     # ---- sampled parity vs the oracle (rank 0's shard, a few whole systems)
     parity = None
@@ -353,30 +374,24 @@ def main():
         t0 = time.perf_counter()
         for _ in range(args.e2e_steps):
             plan.solve_host(*host, xh, stream=stream)  # synchronises its stream
-        te = (time.perf_counter() - t0) / args.e2e_steps
-        tt = torch.tensor([te], dtype=torch.float64, device=dev)
-        if world > 1:
-            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-        te = float(tt.item())
+        te = tdist.max_over_ranks((time.perf_counter() - t0) / args.e2e_steps, device=dev)
         e2e = {"value": m_all * n / te / 1e6, "unit": "Munknowns/s",
                "h2d_bytes_per_step": 4 * n_unknowns * s, "d2h_bytes_per_step": n_unknowns * s,
                "steps": args.e2e_steps, "ms_per_step": te * 1e3,
-               "how": "tri_solve_host: pinned host a,b,c,d -> device, solve, x -> pinned host, per step"}
+               "how": "tri_solve_host per rank: pinned host a,b,c,d -> device, solve, x -> pinned host, per step; "
+                      "max over ranks"}
         del xh
 
-    # ---- edge collectives (N > 1): scatter of the input shards, gather of x
+    # ---- edge collectives (N > 1, sharded batch): NCCL scatter of the input
+    # shards from rank 0 and gather of x to rank 0, through dist.py on the real
+    # data, checked against the resident shards and the oracle
     coll = None
-    if world > 1 and not args.no_collectives:
+    if world > 1 and scaling == "strong" and not args.no_collectives:
         try:
-            t_sc, t_ga, b_sc, b_ga = time_collectives(n, m_all, s, world, rank, dev, tdt)
+            coll = edge_collectives(args, tdist, trigen, n, m, dt, layout, seed, q0, mr, (a, b, c, d), x, s, world,
+                                    rank, dev, tdt)
         except Exception as exc:  # never let the edge measurement cost the solve numbers
-            t_sc = None
-            coll = {"error": repr(exc)[:200]}
-    if coll is None and world > 1 and not args.no_collectives and t_sc is not None:
-        coll = {"scatter_ms": t_sc, "gather_ms": t_ga, "scatter_bytes": b_sc, "gather_bytes": b_ga,
-                "scatter_gbs": b_sc / (t_sc * 1e-3) / 1e9, "gather_gbs": b_ga / (t_ga * 1e-3) / 1e9,
-                "how": "NCCL dist.scatter (4 arrays) / dist.gather (x) from/to rank 0, CUDA events, max over ranks; "
-                       "not part of the timed solve (shards are resident)"}
+            coll = {"error": repr(exc)[:300]}
 
     # ---- CPU oracle baseline (rank 0 at N=1 only)
     cpu = None
@@ -389,35 +404,44 @@ def main():
     peak, peak_src = measured_peaks()
     algo_bytes = 5 * n_unknowns * s          # compulsory 5 arrays per unknown
     achieved = algo_bytes / (t_step * 1e-3) / 1e9
-    marr = method_arrays(plan, tri)
+    marr = method_arrays(plan, tri, l2)
     method_bytes = marr * n_unknowns * s
-    traffic = None
+    method_src = "model (SURVEY 8(d))"
+    traffic, traffic_src = None, None
     tf = os.path.join(ROOT, "profiles", f"traffic_{args.config}.json")
     if os.path.exists(tf):
         with open(tf) as fh:
             tj = json.load(fh)
         if tj.get("n") == n and tj.get("m") == mr and tj.get("k") == plan.k and \
-                tj.get("variant", plan.variant) == plan.variant:
+                tj.get("variant", plan.variant) == plan.variant and tj.get("layout", layout) == layout:
             traffic = tj.get("dram_bytes_per_launch")
+            traffic_src = tj.get("source", tf)
+    if traffic:
+        method_bytes, method_src = traffic, "ncu dram bytes of this plan (" + str(traffic_src) + ")"
     out = {
         "metric": METRIC, "value": value, "unit": "Munknowns/s", "n_gpus": world, "steps": args.steps,
-        "warmup": args.warmup, "ms_per_step": t_step_max, "higher_is_better": True, "scaling": args.scaling,
+        "warmup": args.warmup, "ms_per_step": t_step_max, "higher_is_better": True, "scaling": scaling,
         "vs_baseline": None, "dtype": dt, "data": "synthetic",
         "config": {"workload": args.config, "desc": desc, "n": n, "m": m, "m_per_rank": mr, "layout": layout,
-                   "family": args.family, "parallelism": f"dp{world} (contiguous system shards, no collective)",
+                   "family": args.family,
+                   "parallelism": (f"dp{world}: the m systems sharded over the ranks (contiguous ranges, "
+                                   "dist.shard_range), no collective in the solve" if scaling == "strong" else
+                                   f"dp{world}: replicas (every rank solves its own {m} system(s))"),
                    "timing": "CUDA graph replay of one solve per step" if graph is not None else "direct solve call",
                    "l2": "flushed between timed steps (2x L2 write + 2x L2 read)" if flush else
                          f"inputs larger than L2 ({ws / 2**30:.1f} GiB working set vs {l2 / 2**20:.0f} MiB L2)",
                    "plan": plan.describe()},
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                     "traffic": traffic, "peak_source": peak_src,
+                     "traffic": traffic, "traffic_source": traffic_src, "peak_source": peak_src,
                      "algorithmic_bytes_per_launch": algo_bytes,
-                     "method_arrays": marr, "method_bytes_per_launch": method_bytes,
+                     "method_arrays": method_bytes / (n_unknowns * s), "method_source": method_src,
+                     "method_bytes_per_launch": method_bytes,
                      "method_frac": method_bytes / (t_step * 1e-3) / 1e9 / peak,
-                     "excess_traffic": (traffic / method_bytes) if traffic else None,
+                     "excess_traffic": (traffic / algo_bytes) if traffic else None,
                      "kernel": "whole solve (%d launch%s)" % (plan.launches, "" if plan.launches == 1 else "es")},
         "clocks": clk.summary(),
         "e2e": e2e,
+        "direct": direct,
         "gpu_launches": args.steps * plan.launches,
         "cpu_baseline": cpu,
         "collectives": coll,
@@ -427,6 +451,57 @@ def main():
     print(json.dumps(out), flush=True)
     if world > 1:
         dist.destroy_process_group()
+
+
+def edge_collectives(args, tdist, trigen, n, m, dt, layout, seed, q0, mr, local, x_local, s, world, rank, dev, tdt):
+    """SURVEY 8(e) edge collectives through dist.py on the real shards: rank 0
+    scatters a, b, c, d (dist.scatter_inputs) and gathers x (dist.gather_x);
+    CUDA events, max over ranks.  Checks: every rank's scattered shard equals
+    its resident one bitwise; the gathered x matches the oracle on sampled
+    systems of every shard."""
+    import torch
+    import torch.distributed as dist
+    full = None
+    if rank == 0:
+        full = [torch.from_numpy(t).to(dev) for t in trigen.generate(n, m, dt, layout, args.family, seed=seed)]
+    res = {}
+    for what in ("scatter", "gather"):
+        for it in range(2):  # one warm-up round
+            dist.barrier()
+            torch.cuda.synchronize()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            if what == "scatter":
+                got = tdist.scatter_inputs(n, m, full, layout, dtype=tdt, device=dev)
+            else:
+                xfull = tdist.gather_x(x_local, n, m, layout)
+            e1.record()
+            torch.cuda.synchronize()
+        res[what] = tdist.max_over_ranks(e0.elapsed_time(e1), device=dev)
+    same = all(torch.equal(g, l) for g, l in zip(got, local))
+    ok = tdist.max_over_ranks(0.0 if same else 1.0, device=dev) == 0.0
+    per = -(-m // world)
+    moved = (world - 1) * n * per * s  # bytes of one array leaving / entering rank 0
+    out = {"scatter_ms": res["scatter"], "gather_ms": res["gather"], "scatter_bytes": 4 * moved, "gather_bytes": moved,
+           "scatter_gbs": 4 * moved / (res["scatter"] * 1e-3) / 1e9, "gather_gbs": moved / (res["gather"] * 1e-3) / 1e9,
+           "scattered_shards_equal_resident": ok,
+           "how": "dist.scatter_inputs (4 arrays, NCCL scatter from rank 0) / dist.gather_x (NCCL gather to rank 0), "
+                  "padding and unpacking included, CUDA events, max over ranks; after the timed solve"}
+    if rank == 0:
+        import oracle
+        xs = xfull.cpu().numpy()
+        errs = []
+        for r in range(world):
+            rq0, rmr = tdist.shard_range(m, world, r)
+            for qq in sorted({rq0, rq0 + rmr - 1}):
+                sa = trigen.generate(n, 1, dt, 0, args.family, seed=seed, q0=qq)
+                xo = oracle.solve_batch(n, 1, *sa)
+                xg = xs.reshape(m, n)[qq] if layout == 0 else xs.reshape(n, m)[:, qq]
+                errs.append(float(np.max(np.abs(xg.astype(np.float64) - xo) / np.abs(xo))))
+        out["gathered_parity"] = {"systems": len(errs), "max_rel_err": max(errs)}
+    del full
+    torch.cuda.empty_cache()
+    return out
 
 
 if __name__ == "__main__":

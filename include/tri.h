@@ -189,11 +189,32 @@ TRI_API int tri_plan_k(tri_plan_t plan);                     /* chosen transitio
 TRI_API int tri_plan_variant(tri_plan_t plan);               /* tri_variant in use, -1 if NULL */
 TRI_API int tri_plan_launches(tri_plan_t plan);              /* kernels launched per tri_solve */
 TRI_API int64_t tri_plan_scratch_bytes(tri_plan_t plan);     /* plan-owned device scratch */
-/* 0 <= k <= floor(log2 n) and k <= the variant's limit, else TRI_ERR_INVALID_ARG. */
+/* Force the transition point k (Sec. III.D: k is the method's
+ * knob), any 0 <= k <= floor(log2 n); else TRI_ERR_INVALID_ARG (so any k > 0
+ * when n = 1).  When the plan's variant does not run this k (SCAN / SCAN_MC
+ * run k = 0; STREAM k = 3, FUSED k = 4, WARP k = 5 only), the plan switches
+ * to the first variant in the order SCAN, SCAN_MC, STREAM, FUSED, WARP,
+ * ONCHIP (systems that fit a CTA, fewer than 48 x SMs of them), SPLIT that
+ * runs it -- SPLIT runs every k (tiled-PCR passes of <= 10, then <= 5 steps).
+ * TRI_LAYOUT_BATCHED plans run k = 0 only.  May reallocate scratch
+ * (TRI_ERR_OOM, plan unchanged).  A forced k (or variant) is kept by the
+ * chunk sub-plans of tri_solve_host. */
 TRI_API tri_status tri_plan_set_k(tri_plan_t plan, int k);
 /* Force a variant (TRI_VARIANT_AUTO re-runs the planner); re-plans k if the
  * current k is invalid for it; may reallocate scratch (TRI_ERR_OOM). */
 TRI_API tri_status tri_plan_set_variant(tri_plan_t plan, tri_variant v);
+/* Plan options (explicit per plan; nothing is read from the environment):
+ *   TRI_OPT_TMA (default 1): 0 runs the p-Thomas stage of SPLIT through its
+ *     non-TMA kernels (cp.async / ring-staged / thread-per-chain), which
+ *     otherwise run only where a TMA descriptor cannot describe the arrays
+ *     (row strides not 16-byte multiples); for A/B measurement and tests.
+ *   TRI_OPT_SCAN_MC_LOOKBACK (default 0): SCAN_MC passes 0 and 1 fused by a
+ *     decoupled look-back over chunks of `value` windows (1 <= value <= 512;
+ *     0 = the three-pass form).  Not combinable with tri_slice_solve.
+ * TRI_ERR_INVALID_ARG for an unknown option or value; TRI_ERR_OOM if the new
+ * geometry's scratch cannot be allocated (option unchanged). */
+typedef enum { TRI_OPT_TMA = 1, TRI_OPT_SCAN_MC_LOOKBACK = 2 } tri_option;
+TRI_API tri_status tri_plan_set_option(tri_plan_t plan, tri_option opt, int value);
 /* Human-readable one-line plan description into buf (NUL-terminated). */
 TRI_API void tri_plan_describe(tri_plan_t plan, char* buf, int buflen);
 

@@ -18,6 +18,7 @@ CONTIGUOUS, INTERLEAVED, BATCHED = 0, 1, 2
 (VARIANT_AUTO, VARIANT_ONCHIP, VARIANT_SPLIT, VARIANT_FUSED, VARIANT_WARP, VARIANT_STREAM, VARIANT_SCAN,
  VARIANT_SCAN_MC) = 0, 1, 2, 3, 4, 5, 6, 7
 VARIANT_NAMES = {1: "onchip", 2: "split", 3: "fused", 4: "warp", 5: "stream", 6: "scan", 7: "scan_mc"}
+OPT_TMA, OPT_SCAN_MC_LOOKBACK = 1, 2
 STATUS = {0: "TRI_OK", 1: "TRI_ERR_INVALID_ARG", 2: "TRI_ERR_ALIGNMENT", 3: "TRI_ERR_ALIAS",
           4: "TRI_ERR_DEVICE", 5: "TRI_ERR_OOM", 6: "TRI_ERR_CUDA"}
 
@@ -56,6 +57,7 @@ def lib():
             "tri_plan_scratch_bytes": (_I64, [_P]),
             "tri_plan_set_k": (_I, [_P, _I]),
             "tri_plan_set_variant": (_I, [_P, _I]),
+            "tri_plan_set_option": (_I, [_P, _I, _I]),
             "tri_plan_describe": (None, [_P, ctypes.c_char_p, _I]),
             "tri_status_str": (ctypes.c_char_p, [_I]),
             "tri_halo_f": (_I64, [_I]),
@@ -170,6 +172,13 @@ class Plan:
     def scratch_bytes(self):
         return lib().tri_plan_scratch_bytes(self._h)
 
+    def set_option(self, opt, value):
+        """tri_plan_set_option: OPT_TMA (0 = p-Thomas through the non-TMA
+        kernels), OPT_SCAN_MC_LOOKBACK (windows per look-back chunk, 0 = off)."""
+        st = lib().tri_plan_set_option(self._h, int(opt), int(value))
+        if st != 0:
+            raise TriError(st, f"tri_plan_set_option({opt}, {value})")
+
     def describe(self):
         buf = ctypes.create_string_buffer(512)
         lib().tri_plan_describe(self._h, buf, 512)
@@ -201,12 +210,31 @@ class Plan:
     def solve_host(self, a, b, c, d, out, stream=None):
         """End-to-end through host buffers (tri_solve_host): a..d, out are
         host tensors/arrays (pinned for bandwidth); copies are inside the call."""
+        import numpy as np
         import torch
+        np_dt = np.float64 if self.dtype_code == F64 else np.float32
 
-        def ptr(t):
-            return t.data_ptr() if isinstance(t, torch.Tensor) else t.ctypes.data
+        def ptr(t, what):
+            # the C call reads / writes n*m elements of the plan's dtype through
+            # raw host pointers: validate before handing them over
+            if isinstance(t, torch.Tensor):
+                ok = (t.device.type == "cpu" and t.dtype == self.torch_dtype and t.is_contiguous()
+                      and t.numel() == self.n * self.m)
+                p = t.data_ptr()
+            elif isinstance(t, np.ndarray):
+                ok = (t.dtype == np_dt and t.flags["C_CONTIGUOUS"] and t.size == self.n * self.m
+                      and (what != "out" or t.flags["WRITEABLE"]))
+                p = t.ctypes.data
+            else:
+                ok, p = False, 0
+            if not ok:
+                raise ValueError(f"solve_host {what}: expected a C-contiguous host tensor/array of "
+                                 f"{self.n * self.m} {self.torch_dtype} elements, got {type(t).__name__} "
+                                 f"{getattr(t, 'dtype', None)} {tuple(getattr(t, 'shape', ()))}")
+            return p
+        ps = [ptr(t, w) for t, w in zip((a, b, c, d, out), ("a", "b", "c", "d", "out"))]
         s = stream if stream is not None else torch.cuda.current_stream()
-        st = lib().tri_solve_host(self._h, ptr(a), ptr(b), ptr(c), ptr(d), ptr(out), s.cuda_stream)
+        st = lib().tri_solve_host(self._h, *ps, s.cuda_stream)
         if st != 0:
             raise TriError(st, "tri_solve_host")
         return out

@@ -239,11 +239,35 @@ __device__ __forceinline__ void sc_fix_rows(int64_t i0, int64_t n, T (&ra)[SC_R]
     }
 }
 
+// fp64 rows enter the continuant raw when every pivot b of the warp's window is
+// within 2^+-64 (8-row products then stay far inside fp64's range); otherwise
+// (a warp-uniform test: 4 integer ops per row in the common case) the window's
+// rows are renormalised in registers by 2^-e (e = exponent of b; exact, a row
+// operation that leaves c', d' unchanged, reading X21), so any |b| in fp64's
+// range works.  Called after sc_fix_rows, on warp-converged code only.
+template <typename T>
+__device__ __forceinline__ void sc_range(T (&ra)[SC_R], T (&rb)[SC_R], T (&rc)[SC_R], T (&rd)[SC_R]) {
+    if constexpr (sizeof(T) == 8) {
+        bool out = false;
+#pragma unroll
+        for (int u = 0; u < SC_R; ++u) {
+            const unsigned e = ((unsigned)__double2hiint(rb[u]) >> 20) & 0x7ffu;
+            out |= (e - (1023u - 64u)) > 128u;
+        }
+        if (__any_sync(0xffffffffu, out)) {
+#pragma unroll
+            for (int u = 0; u < SC_R; ++u) {
+                const T s = sk_exp2_scale(rb[u]);
+                ra[u] *= s; rb[u] *= s; rc[u] *= s; rd[u] *= s;
+            }
+        }
+    }
+}
+
 // fp32 rows are scaled by 2^-e (e = exponent of b; exact, a row operation that
 // leaves c', d' unchanged, reading X21) before they enter the continuant, so the
 // product of 8 rows cannot overflow fp32's range (|b| up to 2^126 instead of
-// ~2^16); fp64 uses the rows as given (8-row products overflow only beyond
-// |b| ~ 2^127, X21).
+// ~2^16); fp64 rows are renormalised by sc_range when needed.
 template <typename T>
 __device__ __forceinline__ void sc_row(const T (&ra)[SC_R], const T (&rb)[SC_R], const T (&rc)[SC_R],
                                        const T (&rd)[SC_R], int u, T& a, T& b, T& c, T& d) {
@@ -280,13 +304,26 @@ __device__ __forceinline__ SKMat<T> sc_fwd_map(const T (&ra)[SC_R], const T (&rb
     return SKMat<T>{t1 * s, t2 * s, p1 * s, p2 * s, d1 * s, d2 * s, d3 * s};
 }
 
+// The lane segment maps are composed (scanned) in fp64 for both dtypes
+// (X22): for weakly dominant rows the 3x3 continuant maps compose with
+// cancellation (the two modes of theta_t = b theta_{t-1} - a c theta_{t-2} are
+// close), which amplified fp32 rounding to 1.2e-4 relative error on the c4 shape
+// (weak family, eps = 1e-2; textbook fp32 Thomas: 1.1e-5); with the scan in
+// fp64 and the rows, segment maps and replay in fp32 it is 2.7e-5 (numpy
+// emulation of this kernel's operation order, 2^16 systems).
+using SCM = SKMat<double>;
+template <typename T>
+__device__ __forceinline__ SCM sc_wide(const SKMat<T>& m) {
+    return SCM{(double)m.a, (double)m.b, (double)m.c, (double)m.d, (double)m.e, (double)m.f, (double)m.g};
+}
+
 // both scans in one pass (their shuffles and arithmetic interleave): forward
-// inclusive over the lanes, backward suffix
+// inclusive over the lanes (fp64), backward suffix (T)
 template <int S, typename T>
-__device__ __forceinline__ void sc_scans(SKMat<T>& M, T& al, T& be, int lane) {
+__device__ __forceinline__ void sc_scans(SCM& M, T& al, T& be, int lane) {
 #pragma unroll
     for (int dd = S; dd < 32; dd <<= 1) {
-        const SKMat<T> o = sk_shfl_up(M, dd);
+        const SCM o = sk_shfl_up(M, dd);
         T oa = __shfl_down_sync(0xffffffffu, al, dd), ob = __shfl_down_sync(0xffffffffu, be, dd);
         if (lane + dd >= 32) { oa = T(0); ob = T(1); }
         al = fma(be, oa, al);
@@ -575,11 +612,12 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
                 continue;
             }
             sc_fix_rows<T>((int64_t)lane * SC_R, n, ra, rb, rc, rd);
-            SKMat<T> M = sc_fwd_map(ra, rb, rc, rd);
+            sc_range(ra, rb, rc, rd);
+            SCM M = sc_wide(sc_fwd_map(ra, rb, rc, rd));
             sc_fwd_scan(M, lane);
             // incoming state of the lane = outgoing state of lane - 1 (window starts at (1, 0, 0))
-            T th = __shfl_up_sync(0xffffffffu, M.a, 1), ps = __shfl_up_sync(0xffffffffu, M.c, 1),
-              de = __shfl_up_sync(0xffffffffu, M.e, 1);
+            T th = (T)__shfl_up_sync(0xffffffffu, M.a, 1), ps = (T)__shfl_up_sync(0xffffffffu, M.c, 1),
+              de = (T)__shfl_up_sync(0xffffffffu, M.e, 1);
             if (lane == 0) { th = T(1); ps = T(0); de = T(0); }
             T cp[SC_R], dp[SC_R];
             sc_fwd_replay(ra, rb, rc, rd, th, ps, de, cp, dp);
@@ -690,7 +728,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
                 for (int u = 0; u < SC_R; ++u) { ra[u] = T(0); rb[u] = T(1); rc[u] = T(0); rd[u] = T(0); }
             }
         };
-        SKMat<T> M;
+        SCM M;
         if (fwd) {
             SC_T(5);
             sk_wait(&in_full[pw], ph);
@@ -699,9 +737,10 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
             T ra[SC_R], rb[SC_R], rc[SC_R], rd[SC_R];
             load_rows(ra, rb, rc, rd);
             if (edge) fix_rows(ra, rb, rc, rd);
-            M = sc_fwd_map(ra, rb, rc, rd);
+            sc_range(ra, rb, rc, rd);
+            M = sc_wide(sc_fwd_map(ra, rb, rc, rd));
         } else {
-            M = SKMat<T>{T(1), T(0), T(0), T(1), T(0), T(0), T(1)};
+            M = SCM{1.0, 0.0, 0.0, 1.0, 0.0, 0.0, 1.0};
         }
         T al, be;
         sc_bwd_map(cpb, dpb, al, be);
@@ -720,15 +759,15 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
             de = stt[(pi * S + ls) * 4 + 2];
         }
         const T xs = fma(be, xw, al);  // x at the lane's first row
-        const T ot = fma(M.a, th, M.b * ps);
-        const T op = fma(M.c, th, M.d * ps);
-        const T od = fma(M.e, th, fma(M.f, ps, M.g * de));
+        const double ot = fma(M.a, (double)th, M.b * (double)ps);
+        const double op = fma(M.c, (double)th, M.d * (double)ps);
+        const double od = fma(M.e, (double)th, fma(M.f, (double)ps, M.g * (double)de));
         if (seg == 0) xh[pw * S + ls] = xs;
         if (seg == NSEG - 1) {  // window end: exact power-of-two rescale, hand over
-            const T sc = sk_exp2_scale(ot);
-            stt[(pw * S + ls) * 4 + 0] = ot * sc;
-            stt[(pw * S + ls) * 4 + 1] = op * sc;
-            stt[(pw * S + ls) * 4 + 2] = od * sc;
+            const double sc = sk_exp2_scale(ot);
+            stt[(pw * S + ls) * 4 + 0] = (T)(ot * sc);
+            stt[(pw * S + ls) * 4 + 1] = (T)(op * sc);
+            stt[(pw * S + ls) * 4 + 2] = (T)(od * sc);
         }
         if (g + 1 < total && p.dbg != 1)  // arrive -> sync: release / acquire (PTX memory model)
             asm volatile("bar.arrive %0, 64;" ::"r"(1 + pw) : "memory");
@@ -736,9 +775,9 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
         T x = __shfl_down_sync(0xffffffffu, xs, S);  // x after the lane's rows
         if (seg == NSEG - 1) x = xw;
         {
-            const T it_ = __shfl_up_sync(0xffffffffu, ot, S);
-            const T ip = __shfl_up_sync(0xffffffffu, op, S);
-            const T id = __shfl_up_sync(0xffffffffu, od, S);
+            const T it_ = (T)__shfl_up_sync(0xffffffffu, ot, S);
+            const T ip = (T)__shfl_up_sync(0xffffffffu, op, S);
+            const T id = (T)__shfl_up_sync(0xffffffffu, od, S);
             if (seg > 0) { th = it_; ps = ip; de = id; }
         }
 
@@ -748,6 +787,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
             T ra[SC_R], rb[SC_R], rc[SC_R], rd[SC_R];
             load_rows(ra, rb, rc, rd);
             if (edge) fix_rows(ra, rb, rc, rd);
+            sc_range(ra, rb, rc, rd);
             sc_release_buf();  // this warp's reads of the buffer before the TMA refill
             if (!SC_LATE && lane == 0 && g + SC_NW < nfwd) issue(j, w);
             T cpf[SC_R], dpf[SC_R];
@@ -847,10 +887,11 @@ __global__ void __launch_bounds__(SC1<T>::NW * 32, 1) k_scan1(const __grid_const
         sc_release_buf();  // this warp's reads of the buffer before the TMA refill
         if (!late && lane == 0 && j + NW < nsys) issue(j + NW);
         sc_fix_rows<T>((int64_t)lane * SC_R, n, ra, rb, rc, rd);
-        SKMat<T> M = sc_fwd_map(ra, rb, rc, rd);
+        sc_range(ra, rb, rc, rd);
+        SCM M = sc_wide(sc_fwd_map(ra, rb, rc, rd));
         sc_fwd_scan(M, lane);
-        T th = __shfl_up_sync(0xffffffffu, M.a, 1), ps = __shfl_up_sync(0xffffffffu, M.c, 1),
-          de = __shfl_up_sync(0xffffffffu, M.e, 1);
+        T th = (T)__shfl_up_sync(0xffffffffu, M.a, 1), ps = (T)__shfl_up_sync(0xffffffffu, M.c, 1),
+          de = (T)__shfl_up_sync(0xffffffffu, M.e, 1);
         if (lane == 0) { th = T(1); ps = T(0); de = T(0); }
         T cp[SC_R], dp[SC_R];
         sc_fwd_replay(ra, rb, rc, rd, th, ps, de, cp, dp);

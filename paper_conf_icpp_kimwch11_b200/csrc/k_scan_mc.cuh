@@ -30,8 +30,8 @@ template <typename T>
 struct ScanMCArgs {
     T* x;
     T* cd;        // c', d' of every window (q, w): sc_slot_elems<T>() elements at (q NC + w)
-    T* cmap;      // [m P][8] chunk forward maps (SKMat a..g)
-    T* cbm;       // [m P][8] chunk back-substitution maps (al, be, -): x_first = al + be x_after
+    double* cmap; // [m P][8] chunk forward maps (SKMat a..g; fp64 for both dtypes, k_scan.cuh SCM)
+    double* cbm;  // [m P][8] chunk back-substitution maps (al, be, -): x_first = al + be x_after
     int64_t n, m;
     int NC;       // windows per system
     int NCW;      // windows per chunk
@@ -47,7 +47,7 @@ struct ScanMCArgs {
     const T* xe;
     // look-back path (k_scan_mc_lb): small-chunk records (x after each at [14]);
     // null otherwise
-    const T* xafter;
+    const double* xafter;
     int NCWs, Ps;
 };
 
@@ -58,8 +58,8 @@ struct SMCLayout {
     static constexpr int off_in = 0;
     static constexpr int off_hv = off_in + SC_NW * in_stride;          // [NW][4] handover
     static constexpr int off_bar = off_hv + SC_NW * 4 * (int)sizeof(T);
-    static constexpr int off_wm = (off_bar + SC_NW * 8 + 15) / 16 * 16;  // [NCW][8] per-window maps
-    static __host__ __device__ constexpr int smem_bytes(int NCW) { return off_wm + NCW * 8 * (int)sizeof(T) + 1024; }
+    static constexpr int off_wm = (off_bar + SC_NW * 8 + 15) / 16 * 16;  // [NCW][8] per-window maps (fp64)
+    static __host__ __device__ constexpr int smem_bytes(int NCW) { return off_wm + NCW * 8 * 8 + 1024; }
 };
 
 __device__ __forceinline__ void smc_bulk_g2s(void* dst, const void* src, unsigned bytes, uint64_t* bar) {
@@ -92,34 +92,32 @@ __device__ __forceinline__ void smc_rescale(SKMat<T>& M) {
 // product of the maps of `cnt` consecutive windows / chunks (8 values apart, in
 // shared or global memory; warp-wide, order-preserving): forward maps compose later-after-earlier; backward maps
 // (al, be) compose earlier-after-later (x_first(window i) depends on window i+1)
-template <typename T>
-__device__ __forceinline__ SKMat<T> smc_reduce_fwd(const T* wm, int cnt, int lane) {
+__device__ __forceinline__ SCM smc_reduce_fwd(const double* wm, int cnt, int lane) {
     const int per = (cnt + 31) / 32, lo = lane * per, hi = min(cnt, lo + per);
-    SKMat<T> R{T(1), T(0), T(0), T(1), T(0), T(0), T(1)};
+    SCM R{1.0, 0.0, 0.0, 1.0, 0.0, 0.0, 1.0};
     for (int i = lo; i < hi; ++i) {
-        const T* s = wm + 8 * i;
-        R = sk_compose(SKMat<T>{s[0], s[1], s[2], s[3], s[4], s[5], s[6]}, R);
+        const double* s = wm + 8 * i;
+        R = sk_compose(SCM{s[0], s[1], s[2], s[3], s[4], s[5], s[6]}, R);
         smc_rescale(R);
     }
 #pragma unroll
     for (int d = 1; d < 32; d <<= 1) {  // lane l combines with lane l + d (later windows)
-        const SKMat<T> o = sk_shfl_down(R, d);
+        const SCM o = sk_shfl_down(R, d);
         if ((lane & (2 * d - 1)) == 0) { R = sk_compose(o, R); smc_rescale(R); }
     }
     return R;  // lane 0
 }
-template <typename T>
-__device__ __forceinline__ void smc_reduce_bwd(const T* wm, int cnt, int lane, T& al, T& be) {
+__device__ __forceinline__ void smc_reduce_bwd(const double* wm, int cnt, int lane, double& al, double& be) {
     const int per = (cnt + 31) / 32, lo = lane * per, hi = min(cnt, lo + per);
-    al = T(0); be = T(1);
+    al = 0.0; be = 1.0;
     for (int i = hi - 1; i >= lo; --i) {  // R = B_i o R
-        const T a2 = wm[8 * i], b2 = wm[8 * i + 1];
+        const double a2 = wm[8 * i], b2 = wm[8 * i + 1];
         al = fma(b2, al, a2);
         be = b2 * be;
     }
 #pragma unroll
     for (int d = 1; d < 32; d <<= 1) {  // (lane l) o (lane l + d)
-        const T oa = __shfl_down_sync(0xffffffffu, al, d), ob = __shfl_down_sync(0xffffffffu, be, d);
+        const double oa = __shfl_down_sync(0xffffffffu, al, d), ob = __shfl_down_sync(0xffffffffu, be, d);
         if ((lane & (2 * d - 1)) == 0) { al = fma(be, oa, al); be = be * ob; }
     }
 }
@@ -131,7 +129,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant
     unsigned char* sbase = smc_smem_raw + ((1024 - ((unsigned)__cvta_generic_to_shared(smc_smem_raw) & 1023)) & 1023);
     uint64_t* in_full = reinterpret_cast<uint64_t*>(sbase + L::off_bar);
     T* hv = reinterpret_cast<T*>(sbase + L::off_hv);
-    T* wm = reinterpret_cast<T*>(sbase + L::off_wm);
+    double* wm = reinterpret_cast<double*>(sbase + L::off_wm);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, pw = warp;
     if (threadIdx.x == 0) {
         for (int i = 0; i < SC_NW; ++i) sk_bar_init(&in_full[i], 1);
@@ -170,20 +168,22 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant
     // the chunk's boundary value from the maps of pass 0 / pass 1 (warp 0 runs step 0)
     T st0 = T(1), ps0 = T(0), de0 = T(0), xa0 = T(0);
     if (MODE == 1 && warp == 0) {  // incoming state = (M_{ch-1} ... M_0) S0, S0 = (1, 0, 0) or the slice's
-        const SKMat<T> R = smc_reduce_fwd(p.cmap + 8 * (q * p.P), ch, lane);
-        T t0 = T(1), q0 = T(0), e0 = T(0);
+        const SCM R = smc_reduce_fwd(p.cmap + 8 * (q * p.P), ch, lane);
+        double t0 = 1.0, q0 = 0.0, e0 = 0.0;
         if (p.s0) { t0 = p.s0[0]; q0 = p.s0[1]; e0 = p.s0[2]; }
-        st0 = __shfl_sync(0xffffffffu, fma(R.a, t0, R.b * q0), 0);
-        ps0 = __shfl_sync(0xffffffffu, fma(R.c, t0, R.d * q0), 0);
-        de0 = __shfl_sync(0xffffffffu, fma(R.e, t0, fma(R.f, q0, R.g * e0)), 0);
+        double a0 = fma(R.a, t0, R.b * q0), b0 = fma(R.c, t0, R.d * q0), c0 = fma(R.e, t0, fma(R.f, q0, R.g * e0));
+        const double sc0 = sk_exp2_scale(a0);
+        st0 = (T)__shfl_sync(0xffffffffu, a0 * sc0, 0);
+        ps0 = (T)__shfl_sync(0xffffffffu, b0 * sc0, 0);
+        de0 = (T)__shfl_sync(0xffffffffu, c0 * sc0, 0);
     }
     if (MODE == 2 && p.xafter) {  // look-back path: x after the small chunk that ends this chunk
-        xa0 = p.xafter[(int64_t)((q * p.Ps + (w0 + nwin + p.NCWs - 1) / p.NCWs - 1)) * 16 + 14];
+        xa0 = (T)p.xafter[(int64_t)((q * p.Ps + (w0 + nwin + p.NCWs - 1) / p.NCWs - 1)) * 16 + 14];
     } else if (MODE == 2 && warp == 0) {  // x after the chunk = (B_{ch+1} ... B_{P-1})(x_end), x_end = 0 or the slice's
-        T al, be;
+        double al, be;
         smc_reduce_bwd(p.cbm + 8 * (q * p.P + ch + 1), p.P - 1 - ch, lane, al, be);
-        const T xend = p.xe ? p.xe[0] : T(0);
-        xa0 = __shfl_sync(0xffffffffu, fma(be, xend, al), 0);
+        const double xend = p.xe ? (double)p.xe[0] : 0.0;
+        xa0 = (T)__shfl_sync(0xffffffffu, fma(be, xend, al), 0);
     }
     const unsigned ib_s = (unsigned)__cvta_generic_to_shared(ib);
 
@@ -200,15 +200,16 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant
             sc_release_buf();  // this warp's reads of the buffer before the TMA refill
             if (lane == 0 && g + SC_NW < nwin) issue(g + SC_NW);
             if (edge) sc_fix_rows<T>(i0, n, ra, rb, rc, rd, p.keep_a0, p.keep_cn);
+            sc_range(ra, rb, rc, rd);
             const int nvalid = (int)(n - i0 < 0 ? 0 : n - i0 < SC_R ? n - i0 : SC_R);
-            SKMat<T> M = (p.keep_cn && nvalid < SC_R) ? sc_fwd_map_n(ra, rb, rc, rd, nvalid) : sc_fwd_map(ra, rb, rc, rd);
+            SCM M = sc_wide((p.keep_cn && nvalid < SC_R) ? sc_fwd_map_n(ra, rb, rc, rd, nvalid) : sc_fwd_map(ra, rb, rc, rd));
 #pragma unroll
             for (int d = 1; d < 32; d <<= 1) {  // lane l: lanes l .. l + 2d - 1 (later after earlier)
-                const SKMat<T> o = sk_shfl_down(M, d);
+                const SCM o = sk_shfl_down(M, d);
                 if ((lane & (2 * d - 1)) == 0) { M = sk_compose(o, M); smc_rescale(M); }
             }
             if (lane == 0) {
-                T* s = wm + 8 * g;
+                double* s = wm + 8 * g;
                 s[0] = M.a; s[1] = M.b; s[2] = M.c; s[3] = M.d; s[4] = M.e; s[5] = M.f; s[6] = M.g;
             }
         } else if (MODE == 1) {
@@ -216,9 +217,10 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant
             T ra[SC_R], rb[SC_R], rc[SC_R], rd[SC_R];
             sc_ld_rows_any(ib, lane, p.w128 != 0, ra, rb, rc, rd);
             if (edge) sc_fix_rows<T>(i0, n, ra, rb, rc, rd, p.keep_a0, p.keep_cn);
+            sc_range(ra, rb, rc, rd);
             const int nvalid = (int)(n - i0 < 0 ? 0 : n - i0 < SC_R ? n - i0 : SC_R);
             const bool tr = p.keep_cn && nvalid < SC_R;  // transparent padding rows (slice of a larger system)
-            SKMat<T> M = tr ? sc_fwd_map_n(ra, rb, rc, rd, nvalid) : sc_fwd_map(ra, rb, rc, rd);
+            SCM M = sc_wide(tr ? sc_fwd_map_n(ra, rb, rc, rd, nvalid) : sc_fwd_map(ra, rb, rc, rd));
             sc_fwd_scan(M, lane);
             if (g > 0) asm volatile("bar.sync %0, 64;" ::"r"(1 + pi) : "memory");
             T th, ps, de;
@@ -227,18 +229,18 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant
             } else {
                 th = hv[4 * pi + 0]; ps = hv[4 * pi + 1]; de = hv[4 * pi + 2];
             }
-            const T ot = fma(M.a, th, M.b * ps);
-            const T op = fma(M.c, th, M.d * ps);
-            const T od = fma(M.e, th, fma(M.f, ps, M.g * de));
+            const double ot = fma(M.a, (double)th, M.b * (double)ps);
+            const double op = fma(M.c, (double)th, M.d * (double)ps);
+            const double od = fma(M.e, (double)th, fma(M.f, (double)ps, M.g * (double)de));
             if (lane == 31) {
-                const T sc = sk_exp2_scale(ot);
-                hv[4 * pw + 0] = ot * sc; hv[4 * pw + 1] = op * sc; hv[4 * pw + 2] = od * sc;
+                const double sc = sk_exp2_scale(ot);
+                hv[4 * pw + 0] = (T)(ot * sc); hv[4 * pw + 1] = (T)(op * sc); hv[4 * pw + 2] = (T)(od * sc);
             }
             if (g + 1 < nwin) asm volatile("bar.arrive %0, 64;" ::"r"(1 + pw) : "memory");
             {
-                const T it_ = __shfl_up_sync(0xffffffffu, ot, 1);
-                const T ip = __shfl_up_sync(0xffffffffu, op, 1);
-                const T id = __shfl_up_sync(0xffffffffu, od, 1);
+                const T it_ = (T)__shfl_up_sync(0xffffffffu, ot, 1);
+                const T ip = (T)__shfl_up_sync(0xffffffffu, op, 1);
+                const T id = (T)__shfl_up_sync(0xffffffffu, od, 1);
                 if (lane > 0) { th = it_; ps = ip; de = id; }
             }
             sc_release_buf();  // this warp's reads of the buffer before the TMA refill
@@ -265,7 +267,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant
                 const T oa = __shfl_down_sync(0xffffffffu, al, d), ob = __shfl_down_sync(0xffffffffu, be, d);
                 if ((lane & (2 * d - 1)) == 0) { al = fma(be, oa, al); be = be * ob; }
             }
-            if (lane == 0) { wm[8 * g] = al; wm[8 * g + 1] = be; }
+            if (lane == 0) { wm[8 * g] = (double)al; wm[8 * g + 1] = (double)be; }
         } else {
             // ---- back substitution in reverse window order, x handed over
             T cp[SC_R], dp[SC_R];
@@ -295,13 +297,13 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant
     __syncthreads();
     if (warp == 0) {
         if (MODE == 0) {
-            const SKMat<T> R = smc_reduce_fwd(wm, nwin, lane);
+            const SCM R = smc_reduce_fwd(wm, nwin, lane);
             if (lane == 0) {
-                T* s = p.cmap + 8 * (int64_t)blockIdx.x;
+                double* s = p.cmap + 8 * (int64_t)blockIdx.x;
                 s[0] = R.a; s[1] = R.b; s[2] = R.c; s[3] = R.d; s[4] = R.e; s[5] = R.f; s[6] = R.g;
             }
         } else {
-            T al, be;
+            double al, be;
             smc_reduce_bwd(wm, nwin, lane, al, be);
             if (lane == 0) { p.cbm[8 * (int64_t)blockIdx.x] = al; p.cbm[8 * (int64_t)blockIdx.x + 1] = be; }
         }
@@ -358,7 +360,7 @@ __device__ __forceinline__ void smc_st_release_gpu(unsigned* p, unsigned v) {
 
 template <typename T>
 struct ScanMCLB {
-    T* rec;            // [m Ps][SMC_REC]
+    double* rec;       // [m Ps][SMC_REC] (fp64 for both dtypes)
     unsigned* flag;    // [m Ps] (zeroed before the launch), then the ticket counter at [m Ps]
     int NCWs, Ps;      // windows per small chunk, small chunks per system
 };
@@ -373,7 +375,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc_lb(const __grid_const
     unsigned char* sbase = smc_smem_raw + ((1024 - ((unsigned)__cvta_generic_to_shared(smc_smem_raw) & 1023)) & 1023);
     uint64_t* in_full = reinterpret_cast<uint64_t*>(sbase + L::off_bar);
     T* hv = reinterpret_cast<T*>(sbase + L::off_hv);
-    T* wm0 = reinterpret_cast<T*>(sbase + L::off_wm);
+    double* wm0 = reinterpret_cast<double*>(sbase + L::off_wm);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, pw = warp;
     if (threadIdx.x == 0) {
         for (int i = 0; i < SC_NW; ++i) sk_bar_init(&in_full[i], 1);
@@ -410,8 +412,8 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc_lb(const __grid_const
         const int q = t / lb.Ps, ch = t - q * lb.Ps;
         const int w0 = ch * NCW;
         const int nwin = min(NC, w0 + NCW) - w0;
-        T* wm = wm0 + par * 8 * NCW;          // forward window maps (phase A)
-        T* wmb = wm0 + (2 + par) * 8 * NCW;   // backward window maps (phase B)
+        double* wm = wm0 + par * 8 * NCW;          // forward window maps (phase A)
+        double* wmb = wm0 + (2 + par) * 8 * NCW;   // backward window maps (phase B)
         // ---- phase A: window forward maps
         for (int g = pw; g < nwin; g += SC_NW) {
             const int w = w0 + g;
@@ -427,14 +429,15 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc_lb(const __grid_const
                 else issue((int)q, w0 + pw, pol_b);  // phase B's first window, during the look-back
             }
             if (edge) sc_fix_rows<T>(i0, n, ra, rb, rc, rd, 0, 0);
-            SKMat<T> M = sc_fwd_map(ra, rb, rc, rd);
+            sc_range(ra, rb, rc, rd);
+            SCM M = sc_wide(sc_fwd_map(ra, rb, rc, rd));
 #pragma unroll
             for (int d = 1; d < 32; d <<= 1) {
-                const SKMat<T> o = sk_shfl_down(M, d);
+                const SCM o = sk_shfl_down(M, d);
                 if ((lane & (2 * d - 1)) == 0) { M = sk_compose(o, M); smc_rescale(M); }
             }
             if (lane == 0) {
-                T* s = wm + 8 * g;
+                double* s = wm + 8 * g;
                 s[0] = M.a; s[1] = M.b; s[2] = M.c; s[3] = M.d; s[4] = M.e; s[5] = M.f; s[6] = M.g;
             }
         }
@@ -444,8 +447,8 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc_lb(const __grid_const
         else asm volatile("bar.arrive 13, %0;" ::"r"(SC_THREADS) : "memory");
         if (warp == 0) {
             // aggregate of the chunk, published with flag 1
-            const SKMat<T> R = smc_reduce_fwd(wm, nwin, lane);  // lane 0
-            T* rec = lb.rec + (int64_t)t * SMC_REC;
+            const SCM R = smc_reduce_fwd(wm, nwin, lane);  // lane 0
+            double* rec = lb.rec + (int64_t)t * SMC_REC;
             unsigned* fl = lb.flag;
             if (lane == 0 && ch > 0) {
                 __stcg(rec + 0, R.a); __stcg(rec + 1, R.b); __stcg(rec + 2, R.c); __stcg(rec + 3, R.d);
@@ -457,8 +460,8 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc_lb(const __grid_const
             // of 32 below ch (S_b inclusive, published with flag 2), so one round of 32
             // flags; ch <= 32 starts from the system start when b = 0 ... and b's own
             // inclusive state is built the same way from its base
-            SKMat<T> acc{T(1), T(0), T(0), T(1), T(0), T(0), T(1)};
-            T th = T(1), ps = T(0), de = T(0);
+            SCM acc{1.0, 0.0, 0.0, 1.0, 0.0, 0.0, 1.0};
+            double th = 1.0, ps = 0.0, de = 0.0;
             if (ch > 0) {
                 const int tfirst = (int)(q * lb.Ps);
                 const int b = tfirst + ((ch - 1) / 32) * 32;  // base chunk (inclusive state)
@@ -470,36 +473,36 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc_lb(const __grid_const
                     if (!__any_sync(0xffffffffu, v < want)) break;
                     __nanosleep(32);
                 }
-                SKMat<T> A{T(1), T(0), T(0), T(1), T(0), T(0), T(1)};
+                SCM A{1.0, 0.0, 0.0, 1.0, 0.0, 0.0, 1.0};
                 if (lane < nag) {
-                    const T* r = lb.rec + (int64_t)j * SMC_REC;
-                    A = SKMat<T>{__ldcg(r + 0), __ldcg(r + 1), __ldcg(r + 2), __ldcg(r + 3), __ldcg(r + 4),
-                                 __ldcg(r + 5), __ldcg(r + 6)};
+                    const double* r = lb.rec + (int64_t)j * SMC_REC;
+                    A = SCM{__ldcg(r + 0), __ldcg(r + 1), __ldcg(r + 2), __ldcg(r + 3), __ldcg(r + 4),
+                            __ldcg(r + 5), __ldcg(r + 6)};
                 }
 #pragma unroll
                 for (int d = 1; d < 32; d <<= 1) {  // lane l: A_{j_l} ... A_{j_{l+2d-1}} (lane l latest)
-                    const SKMat<T> o = sk_shfl_down(A, d);
+                    const SCM o = sk_shfl_down(A, d);
                     if ((lane & (2 * d - 1)) == 0) { A = sk_compose(A, o); smc_rescale(A); }
                 }
                 acc.a = __shfl_sync(0xffffffffu, A.a, 0); acc.b = __shfl_sync(0xffffffffu, A.b, 0);
                 acc.c = __shfl_sync(0xffffffffu, A.c, 0); acc.d = __shfl_sync(0xffffffffu, A.d, 0);
                 acc.e = __shfl_sync(0xffffffffu, A.e, 0); acc.f = __shfl_sync(0xffffffffu, A.f, 0);
                 acc.g = __shfl_sync(0xffffffffu, A.g, 0);
-                const T* r = lb.rec + (int64_t)b * SMC_REC;
+                const double* r = lb.rec + (int64_t)b * SMC_REC;
                 th = __ldcg(r + 8); ps = __ldcg(r + 9); de = __ldcg(r + 10);
             }
-            const T it = fma(acc.a, th, acc.b * ps);
-            const T ip = fma(acc.c, th, acc.d * ps);
-            const T id = fma(acc.e, th, fma(acc.f, ps, acc.g * de));
+            const double it = fma(acc.a, th, acc.b * ps);
+            const double ip = fma(acc.c, th, acc.d * ps);
+            const double id = fma(acc.e, th, fma(acc.f, ps, acc.g * de));
             // inclusive state of this chunk, published with flag 2
-            T ot = fma(R.a, it, R.b * ip), op = fma(R.c, it, R.d * ip), od = fma(R.e, it, fma(R.f, ip, R.g * id));
+            double ot = fma(R.a, it, R.b * ip), op = fma(R.c, it, R.d * ip), od = fma(R.e, it, fma(R.f, ip, R.g * id));
             if (lane == 0) {
-                const T sc = sk_exp2_scale(ot);
+                const double sc = sk_exp2_scale(ot);
                 ot *= sc; op *= sc; od *= sc;
                 __stcg(rec + 8, ot); __stcg(rec + 9, op); __stcg(rec + 10, od);
                 smc_st_release_gpu(fl + t, 2u);
-                const T si = sk_exp2_scale(it);
-                s_st[0] = it * si; s_st[1] = ip * si; s_st[2] = id * si;
+                const double si = sk_exp2_scale(it);
+                s_st[0] = (T)(it * si); s_st[1] = (T)(ip * si); s_st[2] = (T)(id * si);
                 s_tk[par ^ 1] = (int)atomicAdd(&lb.flag[total], 1u);  // the next chunk, just in time
             }
         }
@@ -518,7 +521,8 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc_lb(const __grid_const
             T ra[SC_R], rb[SC_R], rc[SC_R], rd[SC_R];
             sc_ld_rows_any(ib, lane, p.w128 != 0, ra, rb, rc, rd);
             if (edge) sc_fix_rows<T>(i0, n, ra, rb, rc, rd, 0, 0);
-            SKMat<T> M = sc_fwd_map(ra, rb, rc, rd);
+            sc_range(ra, rb, rc, rd);
+            SCM M = sc_wide(sc_fwd_map(ra, rb, rc, rd));
             sc_fwd_scan(M, lane);
             if (g > 0) asm volatile("bar.sync %0, 64;" ::"r"(1 + pi) : "memory");
             T th, ps, de;
@@ -528,19 +532,19 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc_lb(const __grid_const
                 th = hv[4 * pi + 0]; ps = hv[4 * pi + 1]; de = hv[4 * pi + 2];
                 tn = (int)hv[4 * pi + 3];
             }
-            const T ot = fma(M.a, th, M.b * ps);
-            const T op = fma(M.c, th, M.d * ps);
-            const T od = fma(M.e, th, fma(M.f, ps, M.g * de));
+            const double ot = fma(M.a, (double)th, M.b * (double)ps);
+            const double op = fma(M.c, (double)th, M.d * (double)ps);
+            const double od = fma(M.e, (double)th, fma(M.f, (double)ps, M.g * (double)de));
             if (lane == 31) {
-                const T sc = sk_exp2_scale(ot);
-                hv[4 * pw + 0] = ot * sc; hv[4 * pw + 1] = op * sc; hv[4 * pw + 2] = od * sc;
+                const double sc = sk_exp2_scale(ot);
+                hv[4 * pw + 0] = (T)(ot * sc); hv[4 * pw + 1] = (T)(op * sc); hv[4 * pw + 2] = (T)(od * sc);
                 hv[4 * pw + 3] = (T)tn;
             }
             if (g + 1 < nwin) asm volatile("bar.arrive %0, 64;" ::"r"(1 + pw) : "memory");
             {
-                const T it_ = __shfl_up_sync(0xffffffffu, ot, 1);
-                const T ip = __shfl_up_sync(0xffffffffu, op, 1);
-                const T id = __shfl_up_sync(0xffffffffu, od, 1);
+                const T it_ = (T)__shfl_up_sync(0xffffffffu, ot, 1);
+                const T ip = (T)__shfl_up_sync(0xffffffffu, op, 1);
+                const T id = (T)__shfl_up_sync(0xffffffffu, od, 1);
                 if (lane > 0) { th = it_; ps = ip; de = id; }
             }
             sc_release_buf();
@@ -572,7 +576,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc_lb(const __grid_const
                 const T oa = __shfl_down_sync(0xffffffffu, al, d), ob = __shfl_down_sync(0xffffffffu, be, d);
                 if ((lane & (2 * d - 1)) == 0) { al = fma(be, oa, al); be = be * ob; }
             }
-            if (lane == 0) { wmb[8 * g] = al; wmb[8 * g + 1] = be; }
+            if (lane == 0) { wmb[8 * g] = (double)al; wmb[8 * g + 1] = (double)be; }
         }
         __syncthreads();
         if (pw >= nwin) tn = s_tk[par ^ 1];
@@ -582,7 +586,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc_lb(const __grid_const
             if (pw < min(NC, chn * NCW + NCW) - chn * NCW) issue(qn, chn * NCW + pw, pol_a);
         }
         if (warp == 0) {
-            T al, be;
+            double al, be;
             smc_reduce_bwd(wmb, nwin, lane, al, be);
             if (lane == 0) { lb.rec[(int64_t)t * SMC_REC + 12] = al; lb.rec[(int64_t)t * SMC_REC + 13] = be; }
         }
@@ -595,33 +599,33 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc_lb(const __grid_const
 // x_after(ch) = B_{ch+1}(... B_{Ps-1}(0)); written to rec[14]
 template <typename T>
 __global__ void __launch_bounds__(1024) k_scan_mc_lb_fin(ScanMCLB<T> lb) {
-    __shared__ T sa[32], sb[32];
+    __shared__ double sa[32], sb[32];
     const int64_t q = blockIdx.x;
     const int Ps = lb.Ps, tid = threadIdx.x, lane = tid & 31, wp = tid >> 5;
-    T* rec = lb.rec + q * Ps * SMC_REC;
+    double* rec = lb.rec + q * Ps * SMC_REC;
     const int per = (Ps + 1023) / 1024, lo = min(Ps, tid * per), hi = min(Ps, lo + per);
-    T al = T(0), be = T(1);  // this thread's chunks composed: x_first(lo) = al + be x_after(hi - 1)
+    double al = 0.0, be = 1.0;  // this thread's chunks composed: x_first(lo) = al + be x_after(hi - 1)
     for (int i = hi - 1; i >= lo; --i) {
-        const T a2 = rec[(int64_t)i * SMC_REC + 12], b2 = rec[(int64_t)i * SMC_REC + 13];
+        const double a2 = rec[(int64_t)i * SMC_REC + 12], b2 = rec[(int64_t)i * SMC_REC + 13];
         al = fma(b2, al, a2);
         be = b2 * be;
     }
     // exclusive suffix over threads: the map of all chunks after this thread's range
-    T sal = al, sbe = be;  // inclusive suffix within the warp (lane l: lanes l..31)
+    double sal = al, sbe = be;  // inclusive suffix within the warp (lane l: lanes l..31)
 #pragma unroll
     for (int d = 1; d < 32; d <<= 1) {
-        const T oa = __shfl_down_sync(0xffffffffu, sal, d), ob = __shfl_down_sync(0xffffffffu, sbe, d);
+        const double oa = __shfl_down_sync(0xffffffffu, sal, d), ob = __shfl_down_sync(0xffffffffu, sbe, d);
         if (lane + d < 32) { sal = fma(sbe, oa, sal); sbe = sbe * ob; }
     }
     if (lane == 0) { sa[wp] = sal; sb[wp] = sbe; }
     __syncthreads();
     // x after warp wp's range: the warps after it applied to 0
-    T xw = T(0);
+    double xw = 0.0;
     for (int v = 31; v > wp; --v) xw = fma(sb[v], xw, sa[v]);
     // x after this thread's range: lanes after it in the warp, then xw
-    T ea = __shfl_down_sync(0xffffffffu, sal, 1), eb = __shfl_down_sync(0xffffffffu, sbe, 1);
-    if (lane == 31) { ea = T(0); eb = T(1); }
-    T x = fma(eb, xw, ea);
+    double ea = __shfl_down_sync(0xffffffffu, sal, 1), eb = __shfl_down_sync(0xffffffffu, sbe, 1);
+    if (lane == 31) { ea = 0.0; eb = 1.0; }
+    double x = fma(eb, xw, ea);
     for (int i = hi - 1; i >= lo; --i) {
         rec[(int64_t)i * SMC_REC + 14] = x;
         x = fma(rec[(int64_t)i * SMC_REC + 13], x, rec[(int64_t)i * SMC_REC + 12]);
@@ -635,15 +639,15 @@ template <typename T, int MODE>
 __global__ void k_scan_mc_slice_map(ScanMCArgs<T> p, T* out) {
     const int lane = threadIdx.x & 31;
     if (MODE == 0) {
-        const SKMat<T> R = smc_reduce_fwd(p.cmap, p.P, lane);
+        const SCM R = smc_reduce_fwd(p.cmap, p.P, lane);
         if (lane == 0) {
-            out[0] = R.a; out[1] = R.b; out[2] = R.c; out[3] = R.d; out[4] = R.e; out[5] = R.f; out[6] = R.g;
-            out[7] = T(0);
+            out[0] = (T)R.a; out[1] = (T)R.b; out[2] = (T)R.c; out[3] = (T)R.d; out[4] = (T)R.e; out[5] = (T)R.f;
+            out[6] = (T)R.g; out[7] = T(0);
         }
     } else {
-        T al, be;
+        double al, be;
         smc_reduce_bwd(p.cbm, p.P, lane, al, be);
-        if (lane == 0) { out[0] = al; out[1] = be; for (int i = 2; i < 8; ++i) out[i] = T(0); }
+        if (lane == 0) { out[0] = (T)al; out[1] = (T)be; for (int i = 2; i < 8; ++i) out[i] = T(0); }
     }
 }
 

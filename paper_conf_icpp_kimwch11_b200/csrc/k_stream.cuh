@@ -42,6 +42,7 @@
 #pragma once
 #include <cudaTypedefs.h>
 #include "common.cuh"
+#include "k_fused.cuh"  // fu_ld2 / fu_st2 shared-memory pair helpers
 
 namespace tri {
 
@@ -186,15 +187,17 @@ template <typename T>
 __device__ __forceinline__ T sk_exp2_scale(T v);
 template <>
 __device__ __forceinline__ double sk_exp2_scale<double>(double v) {
+    // 2^(1023 - E) for biased exponent E, clamped to a normal number (E = 2046:
+    // 2^-1022, so v s lands in [2, 4); E = 0, zero / subnormal v: 2^1023)
     const long long bits = __double_as_longlong(v);
-    const int e = (int)((bits >> 52) & 0x7ff) - 1023;
-    return __longlong_as_double((long long)(1023 - e) << 52);
+    const int e = 2046 - (int)((bits >> 52) & 0x7ff);
+    return __longlong_as_double((long long)(e < 1 ? 1 : e) << 52);
 }
 template <>
 __device__ __forceinline__ float sk_exp2_scale<float>(float v) {
     const int bits = __float_as_int(v);
-    const int e = ((bits >> 23) & 0xff) - 127;
-    return __int_as_float((127 - e) << 23);
+    const int e = 254 - ((bits >> 23) & 0xff);
+    return __int_as_float((e < 1 ? 1 : e) << 23);
 }
 
 // storage slot -> location: the first and last S_on/2 slots are resident in

@@ -1,0 +1,227 @@
+// l_scan.cu -- launchers of TRI_VARIANT_SCAN (k_scan.cuh) and TRI_VARIANT_SCAN_MC
+// (k_scan_mc.cuh): p-Thomas at k = 0 (the paper's rule for M > P) with
+// each system's sweeps spread over a warp's lanes (X21).
+#include <algorithm>
+
+#include "plan.cuh"
+#include "k_scan.cuh"
+#include "k_scan_mc.cuh"
+
+using namespace tri;
+
+namespace trih {
+namespace {
+
+// CONTIGUOUS: tensor view [m][n/r][r] (r = 8, or 128 bytes of elements with w128),
+// box [1][256/r][r] = one 256-row window of one system per array; every
+// coordinate fits int32 for any n, m of the API
+template <typename T>
+bool map_sys_rows(CUtensorMap* tm, const void* base, int64_t n, int64_t m, bool w128) {
+    const int rw = w128 ? 128 / (int)sizeof(T) : 8;  // elements per tensor row
+    const uint64_t dims[3] = {(uint64_t)rw, (uint64_t)(n / rw), (uint64_t)m};
+    const uint64_t str[2] = {(uint64_t)rw * sizeof(T), (uint64_t)n * sizeof(T)};
+    const uint32_t box[3] = {(uint32_t)rw, (uint32_t)(SC_W / rw), 1u};
+    const CUtensorMapSwizzle swz =
+        w128 ? CU_TENSOR_MAP_SWIZZLE_128B : sizeof(T) == 8 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_32B;
+    return tma_encode(tm, sizeof(T), 3, base, dims, str, box, swz);
+}
+
+// INTERLEAVED / BATCHED: tensor [nb][n][ms] (row stride ms elements, batch stride
+// n ms), box [1][256 / S rows][S systems]
+template <typename T>
+bool map_il(CUtensorMap* tm, const void* base, int64_t n, int64_t ms, int64_t nb, int S) {
+    const uint64_t dims[3] = {(uint64_t)ms, (uint64_t)n, (uint64_t)nb};
+    const uint64_t str[2] = {(uint64_t)ms * sizeof(T), (uint64_t)(n * ms) * sizeof(T)};
+    const uint32_t box[3] = {(uint32_t)S, (uint32_t)(SC_W / S), 1u};
+    return tma_encode(tm, sizeof(T), 3, base, dims, str, box, CU_TENSOR_MAP_SWIZZLE_NONE);
+}
+
+template <typename T>
+bool scan_maps(tri_plan_s* p, int tag, const void* a, const void* b, const void* c, const void* d, bool w128,
+               StreamMaps& tm) {
+    const void* key[4] = {a, b, c, d};
+    if (tm_lookup(p, tag, key, 4, &tm.a, 4)) return true;
+    const void* src[4] = {a, b, c, d};
+    CUtensorMap* dst[4] = {&tm.a, &tm.b, &tm.c, &tm.d};
+    for (int i = 0; i < 4; ++i) {
+        const bool ok = p->sk_S == 1 || p->variant == TRI_VARIANT_SCAN_MC
+                            ? map_sys_rows<T>(dst[i], src[i], p->n, p->m, w128)
+                            : map_il<T>(dst[i], src[i], p->n, p->ms, p->m / p->ms, p->sk_S);
+        if (!ok) return false;
+    }
+    tm_store(p, tag, key, 4, &tm.a, 4);
+    return true;
+}
+
+template <typename T, int S>
+void* scan_kernel(bool prof) {
+    return prof ? (void*)k_scan<T, S, true> : (void*)k_scan<T, S, false>;
+}
+
+template <typename T>
+cudaError_t scan_t(tri_plan_s* p, const void* a, const void* b, const void* c, const void* d, void* x,
+                   cudaStream_t st) {
+    const int S = p->sk_S;
+    // one-window systems shorter than 3/4 of a window (many idle rows: compute-heavy)
+    // run the chain-free kernel with more warps (fp32 n = 128: 1.19 ms vs 1.50 ms
+    // per 2^28 rows); at n = 256 the 12-warp kernel is faster (c4: 0.99 vs 1.02 ms)
+    const bool one = S == 1 && p->sk_nc == 1 && p->n <= 3 * SC_W / 4;
+    // 128-byte TMA rows (n % 32 fp32 / n % 16 fp64; the k_scan chain and one-window
+    // paths): one TMA request per 128 bytes (fp32 c4: 0.99 -> 0.84 ms)
+    const bool w128 = S == 1 && p->n % (128 / (int)sizeof(T)) == 0 && !one;
+    StreamMaps tm;
+    if (!scan_maps<T>(p, 0x1000 + (int)sizeof(T) + 16 * (w128 ? 1 : 0), a, b, c, d, w128, tm))
+        return cudaErrorNotSupported;
+    ScanArgs<T> A;
+    A.x = (T*)x;
+    A.spill = (T*)p->scratch;
+    A.n = p->n; A.m = p->m; A.ms = p->ms; A.NC = p->sk_nc; A.S_on = p->sk_son; A.delta = p->sk_delta;
+    A.w128 = w128 ? 1 : 0;
+    A.prof = (unsigned long long*)g_fused_prof;
+    A.dbg = g_fused_dbg_mode;
+    if (one) {
+        cudaError_t e = set_smem((const void*)k_scan1<T>, SC1<T>::smem_bytes);
+        if (e != cudaSuccess) return e;
+        k_scan1<T><<<p->sk_grid, SC1<T>::NW * 32, SC1<T>::smem_bytes, st>>>(tm, A);
+        return cudaGetLastError();
+    }
+    // one-window systems (S = 1): the slot area holds the warps' second staging buffers
+    const int son_or_buf = (S == 1 && p->sk_nc == 1)
+                               ? (SC_NW * SCLayout<T>::in_stride + SCLayout<T>::slot_bytes - 1) / SCLayout<T>::slot_bytes
+                               : p->sk_son;
+    const int smem = SCLayout<T>::smem_bytes(p->sk_nc, p->sk_delta, son_or_buf);
+    const bool pr = A.prof != nullptr;
+    void* kern = S == 1 ? scan_kernel<T, 1>(pr) : S == 2 ? scan_kernel<T, 2>(pr) : S == 4 ? scan_kernel<T, 4>(pr)
+                 : S == 8 ? scan_kernel<T, 8>(pr) : scan_kernel<T, 16>(pr);
+    cudaError_t e = set_smem(kern, smem);
+    if (e != cudaSuccess) return e;
+    void* args[] = {(void*)&tm, (void*)&A};
+    return cudaLaunchKernel(kern, dim3(p->sk_grid), dim3(SC_THREADS), args, smem, st);
+}
+
+template <typename T>
+cudaError_t scan_mc_setup(tri_plan_s* p, const void* a, const void* b, const void* c, const void* d, void* x,
+                          StreamMaps& tm, ScanMCArgs<T>& A, int& smem, bool cache) {
+    const int64_t n = p->n;
+    const bool w = n % (128 / (int)sizeof(T)) == 0;
+    if (a) {
+        bool ok;
+        if (cache) {
+            ok = scan_maps<T>(p, 0x2000 + (int)sizeof(T), a, b, c, d, w, tm);
+        } else {
+            ok = map_sys_rows<T>(&tm.a, a, n, p->m, w) && map_sys_rows<T>(&tm.b, b, n, p->m, w) &&
+                 map_sys_rows<T>(&tm.c, c, n, p->m, w) && map_sys_rows<T>(&tm.d, d, n, p->m, w);
+        }
+        if (!ok) return cudaErrorNotSupported;
+    }
+    A = ScanMCArgs<T>{};
+    A.w128 = w ? 1 : 0;
+    A.x = (T*)x;
+    A.cd = (T*)p->scratch;
+    const int64_t mp = p->m * (int64_t)p->mc_P;
+    A.cmap = reinterpret_cast<double*>(A.cd + p->m * (int64_t)p->sk_nc * sc_slot_elems<T>());  // 2 KB multiples
+    A.cbm = A.cmap + 8 * mp;
+    A.n = p->n; A.m = p->m; A.NC = p->sk_nc; A.NCW = p->mc_NCW; A.P = p->mc_P;
+    smem = SMCLayout<T>::smem_bytes(p->mc_NCW);
+    for (auto k : {k_scan_mc<T, 0>, k_scan_mc<T, 1>, k_scan_mc<T, 2>}) {
+        cudaError_t e = set_smem((const void*)k, smem);
+        if (e != cudaSuccess) return e;
+    }
+    return cudaSuccess;
+}
+// the 16 values after the fp64 chunk maps: the slice's incoming state (3) and x after it (1)
+template <typename T>
+T* scan_mc_slice_vals(const tri_plan_s* p) {
+    double* maps = reinterpret_cast<double*>((T*)p->scratch + p->m * (int64_t)p->sk_nc * sc_slot_elems<T>());
+    return reinterpret_cast<T*>(maps + 16 * p->m * (int64_t)p->mc_P);
+}
+
+template <typename T>
+cudaError_t scan_mc_t(tri_plan_s* p, const void* a, const void* b, const void* c, const void* d, void* x,
+                      cudaStream_t st) {
+    StreamMaps tm;
+    ScanMCArgs<T> A;
+    int smem = 0;
+    cudaError_t e = scan_mc_setup<T>(p, a, b, c, d, x, tm, A, smem, true);
+    if (e != cudaSuccess) return e;
+    if (p->mc_lb) {
+        ScanMCLB<T> lb;
+        lb.rec = reinterpret_cast<double*>(scan_mc_slice_vals<T>(p) + 16);  // 16 T values: 8-byte aligned
+        const int64_t nrec = p->m * (int64_t)p->mc_Ps;
+        lb.flag = (unsigned*)(lb.rec + nrec * SMC_REC);
+        lb.NCWs = p->mc_NCWs;
+        lb.Ps = p->mc_Ps;
+        const int smem_lb = SMCLayout<T>::smem_bytes(4 * p->mc_NCWs);
+        e = set_smem((const void*)k_scan_mc_lb<T>, smem_lb);
+        if (e != cudaSuccess) return e;
+        e = cudaMemsetAsync(lb.flag, 0, (size_t)(nrec + 1) * sizeof(unsigned), st);
+        if (e != cudaSuccess) return e;
+        const int grid = (int)std::min<int64_t>(p->sms, nrec);
+        k_scan_mc_lb<T><<<grid, SC_THREADS, smem_lb, st>>>(tm, A, lb);
+        k_scan_mc_lb_fin<T><<<(unsigned)p->m, 1024, 0, st>>>(lb);
+        A.xafter = lb.rec;
+        A.NCWs = p->mc_NCWs;
+        A.Ps = p->mc_Ps;
+        k_scan_mc<T, 2><<<p->sk_grid, SC_THREADS, smem, st>>>(tm, A);
+        return cudaGetLastError();
+    }
+    k_scan_mc<T, 0><<<p->sk_grid, SC_THREADS, smem, st>>>(tm, A);
+    k_scan_mc<T, 1><<<p->sk_grid, SC_THREADS, smem, st>>>(tm, A);
+    k_scan_mc<T, 2><<<p->sk_grid, SC_THREADS, smem, st>>>(tm, A);
+    return cudaGetLastError();
+}
+
+// sliced solve of one system over devices (NEXT-4): phase 0 = pass 0 + the
+// slice's forward map; 1 = incoming state from every slice's map, pass 1, the
+// slice's backward map; 2 = x after the slice from every backward map, pass 2
+template <typename T>
+cudaError_t scan_mc_slice_t(tri_plan_s* p, int phase, int slice, int nslices, const void* a, const void* b,
+                            const void* c, const void* d, const void* maps, void* out, cudaStream_t st) {
+    StreamMaps tm;
+    ScanMCArgs<T> A;
+    int smem = 0;
+    cudaError_t e = scan_mc_setup<T>(p, phase < 2 ? a : nullptr, b, c, d, phase == 2 ? out : nullptr, tm, A, smem,
+                                     false);
+    if (e != cudaSuccess) return e;
+    A.keep_a0 = slice > 0;
+    A.keep_cn = slice < nslices - 1;
+    T* vals = scan_mc_slice_vals<T>(p);
+    if (phase == 0) {
+        k_scan_mc<T, 0><<<p->sk_grid, SC_THREADS, smem, st>>>(tm, A);
+        k_scan_mc_slice_map<T, 0><<<1, 32, 0, st>>>(A, (T*)out);
+    } else if (phase == 1) {
+        k_scan_mc_slice_link<T, 0><<<1, 32, 0, st>>>((const T*)maps, nslices, slice, vals);
+        A.s0 = vals;
+        k_scan_mc<T, 1><<<p->sk_grid, SC_THREADS, smem, st>>>(tm, A);
+        k_scan_mc_slice_map<T, 1><<<1, 32, 0, st>>>(A, (T*)out);
+    } else {
+        k_scan_mc_slice_link<T, 1><<<1, 32, 0, st>>>((const T*)maps, nslices, slice, vals + 4);
+        A.xe = vals + 4;
+        k_scan_mc<T, 2><<<p->sk_grid, SC_THREADS, smem, st>>>(tm, A);
+    }
+    return cudaGetLastError();
+}
+
+}  // namespace
+
+cudaError_t launch_scan(tri_plan_s* p, const void* a, const void* b, const void* c, const void* d, void* x,
+                        cudaStream_t st) {
+    return p->dtype == TRI_F64 ? scan_t<double>(p, a, b, c, d, x, st) : scan_t<float>(p, a, b, c, d, x, st);
+}
+cudaError_t launch_scan_mc(tri_plan_s* p, const void* a, const void* b, const void* c, const void* d, void* x,
+                           cudaStream_t st) {
+    return p->dtype == TRI_F64 ? scan_mc_t<double>(p, a, b, c, d, x, st) : scan_mc_t<float>(p, a, b, c, d, x, st);
+}
+cudaError_t launch_scan_mc_slice(tri_plan_s* p, int phase, int slice, int nslices, const void* a, const void* b,
+                                 const void* c, const void* d, const void* maps, void* out, cudaStream_t st) {
+    return p->dtype == TRI_F64 ? scan_mc_slice_t<double>(p, phase, slice, nslices, a, b, c, d, maps, out, st)
+                               : scan_mc_slice_t<float>(p, phase, slice, nslices, a, b, c, d, maps, out, st);
+}
+int scan_smem_fixed(tri_dtype t, int NC, int delta) {
+    return t == TRI_F64 ? SCLayout<double>::smem_bytes(NC, delta, 0) : SCLayout<float>::smem_bytes(NC, delta, 0);
+}
+int scan_slot_bytes(tri_dtype t) { return t == TRI_F64 ? SCLayout<double>::slot_bytes : SCLayout<float>::slot_bytes; }
+int scan_in_stride(tri_dtype t) { return t == TRI_F64 ? SCLayout<double>::in_stride : SCLayout<float>::in_stride; }
+int scan_mc_wmax() { return SMC_WMAX; }
+
+}  // namespace trih

@@ -1,4 +1,5 @@
-"""Multi-GPU driver for batches of independent systems.
+"""Multi-GPU driver for batches of independent systems (PAPER.md
+P:699 Sec. III.D and P:747 Sec. IV: M independent systems).
 
 The m systems are split into contiguous ranges, one per rank (tri_shard_range);
 each rank solves its shard on its own GPU with no collective inside the solve
@@ -9,7 +10,10 @@ appear only at the edges:
                gloo in the CPU tests);
   * max_over_ranks: the timing convention (job time = slowest rank).
 A rank holds its shard in the same layout as the full batch with m_r columns
-(CONTIGUOUS: [ql*n + i]; INTERLEAVED: [i*m_r + ql]).
+(CONTIGUOUS: [ql*n + i]; INTERLEAVED: [i*m_r + ql]).  The per-shard solver on
+the GPU is cuda_solver (the CUDA Plan through the C ABI); with the gloo backend
+(CPU tests, or several ranks sharing one GPU) the edge collectives run on host
+copies of the device shards.
 """
 import torch
 import torch.distributed as dist
@@ -20,6 +24,27 @@ from . import CONTIGUOUS, INTERLEAVED, shard_range as _abi_shard_range
 def shard_range(m, world, rank):
     """(q0, m_r): rank r owns systems [q0, q0 + m_r) (tri_shard_range)."""
     return _abi_shard_range(int(m), int(world), int(rank))
+
+
+def _host_collectives(group, t):
+    """gloo moves host tensors only: run its collectives on CPU copies."""
+    return dist.get_backend(group) == "gloo" and t is not None and t.is_cuda
+
+
+def cuda_solver(n, dtype, layout=CONTIGUOUS):
+    """solve_fn for solve_sharded: the CUDA Plan (C ABI) of the rank's shard,
+    created once per shard size and reused; inputs are moved to the current
+    CUDA device if they are not already there."""
+    from . import Plan
+    plans = {}
+
+    def solve_fn(a, b, c, d, mr):
+        dev = torch.device("cuda", torch.cuda.current_device())
+        a, b, c, d = (t.to(dev) for t in (a, b, c, d))
+        if mr not in plans:
+            plans[mr] = Plan(n, mr, dtype, layout)
+        return plans[mr].solve(a, b, c, d)
+    return solve_fn
 
 
 def max_over_ranks(value, group=None, device=None):
@@ -39,6 +64,9 @@ def gather_x(x_local, n, m, layout=CONTIGUOUS, group=None, dst=0):
     rank = dist.get_rank(group)
     per = -(-m // world)
     q0, mr = shard_range(m, world, rank)
+    dev_out = x_local.device
+    if _host_collectives(group, x_local):
+        x_local = x_local.cpu()
     pad = torch.zeros(n * per, dtype=x_local.dtype, device=x_local.device)
     if layout == CONTIGUOUS:
         pad[: n * mr] = x_local
@@ -57,7 +85,7 @@ def gather_x(x_local, n, m, layout=CONTIGUOUS, group=None, dst=0):
             full[rq0 * n:(rq0 + rmr) * n] = bufs[r][: n * rmr]
         else:
             full.view(n, m)[:, rq0:rq0 + rmr] = bufs[r].view(n, per)[:, :rmr]
-    return full
+    return full.to(dev_out)
 
 
 def scatter_inputs(n, m, full=None, layout=CONTIGUOUS, group=None, src=0, dtype=None, device=None):
@@ -71,6 +99,11 @@ def scatter_inputs(n, m, full=None, layout=CONTIGUOUS, group=None, src=0, dtype=
     q0, mr = shard_range(m, world, rank)
     if rank == src:
         dtype, device = full[0].dtype, full[0].device
+    dev_out = device
+    if device is not None and _host_collectives(group, torch.empty(0, device=device)):
+        device = torch.device("cpu")
+        if full is not None:
+            full = [t.cpu() for t in full]
     out = []
     for arr in range(4):
         recv = torch.zeros(n * per, dtype=dtype, device=device)
@@ -88,9 +121,9 @@ def scatter_inputs(n, m, full=None, layout=CONTIGUOUS, group=None, src=0, dtype=
                 send.append(buf)
         dist.scatter(recv, scatter_list=send, src=src, group=group)
         if layout == CONTIGUOUS:
-            out.append(recv[: n * mr].clone())
+            out.append(recv[: n * mr].clone().to(dev_out))
         else:
-            out.append(recv.view(n, per)[:, :mr].contiguous().view(-1))
+            out.append(recv.view(n, per)[:, :mr].contiguous().view(-1).to(dev_out))
     return out
 
 

@@ -1,7 +1,7 @@
 """Planner calibration for the SCAN variant: over a grid of
 contiguous shapes like the paper's (Figs 12-13), time the planner's choice and
-every competing whole-solve variant (SCAN, STREAM, SPLIT k = 0, FUSED, WARP,
-ONCHIP at its planned k) with CUDA-graph replays; JSON lines to stdout.
+every competing whole-solve variant (SCAN, SCAN_MC, STREAM, SPLIT (k = 0 from
+148 systems, else its planned k), FUSED, WARP, ONCHIP at its planned k) with CUDA-graph replays; JSON lines to stdout.
 usage: python scripts/sweep_scan.py [f64|f32]"""
 import json
 import os
@@ -47,7 +47,7 @@ else:  # interleaved: m a multiple of 8
         for m in (64, 296, 1024, 2368, 4096, 9472, 16384, 37888, 151552, 1 << 20):
             if n * m <= MAXE and n * m >= 4096:
                 SHAPES.append((n, m))
-VARS = [tri.VARIANT_SCAN, tri.VARIANT_STREAM, tri.VARIANT_SPLIT, tri.VARIANT_FUSED, tri.VARIANT_WARP, tri.VARIANT_ONCHIP]
+VARS = [tri.VARIANT_SCAN, tri.VARIANT_SCAN_MC, tri.VARIANT_STREAM, tri.VARIANT_SPLIT, tri.VARIANT_FUSED, tri.VARIANT_WARP, tri.VARIANT_ONCHIP]
 for n, m in SHAPES:
     arrs = trigen.generate(n, m, DT, LAYOUT, "dd")
     a, b, c, d = (torch.from_numpy(t).cuda() for t in arrs)
