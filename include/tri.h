@@ -176,7 +176,7 @@ TRI_API tri_plan_t tri_plan_batched(int64_t n, int64_t ms, int64_t nb, tri_dtype
  * last row of slice r < nslices - 1 keeps its c.  Asynchronous on `stream`;
  * phases run in order on one plan; the plan's scratch carries c', d' from
  * phase 1 to phase 2.  TRI_ERR_INVALID_ARG for a plan that is not SCAN_MC with
- * m == 1, a bad phase / slice, or a NULL pointer. */
+ * m == 1 and TRI_OPT_SCAN_MC_LOOKBACK 0, a bad phase / slice, or a NULL pointer. */
 TRI_API tri_status tri_slice_solve(tri_plan_t plan, int phase, int slice, int nslices, const void* a,
                                    const void* b, const void* c, const void* d, const void* maps, void* out,
                                    void* stream);
@@ -208,9 +208,10 @@ TRI_API tri_status tri_plan_set_variant(tri_plan_t plan, tri_variant v);
  *     non-TMA kernels (cp.async / ring-staged / thread-per-chain), which
  *     otherwise run only where a TMA descriptor cannot describe the arrays
  *     (row strides not 16-byte multiples); for A/B measurement and tests.
- *   TRI_OPT_SCAN_MC_LOOKBACK (default 0): SCAN_MC passes 0 and 1 fused by a
- *     decoupled look-back over chunks of `value` windows (1 <= value <= 512;
- *     0 = the three-pass form).  Not combinable with tri_slice_solve.
+ *   TRI_OPT_SCAN_MC_LOOKBACK (default -1 = auto): SCAN_MC passes 0 and 1 fused
+ *     by a decoupled look-back over chunks of `value` windows (1 <= value <= 64;
+ *     0 = the three-pass form; auto = the three-pass form, measured faster on
+ *     B200).  tri_slice_solve needs it off (0 or auto).
  * TRI_ERR_INVALID_ARG for an unknown option or value; TRI_ERR_OOM if the new
  * geometry's scratch cannot be allocated (option unchanged). */
 typedef enum { TRI_OPT_TMA = 1, TRI_OPT_SCAN_MC_LOOKBACK = 2 } tri_option;

@@ -245,9 +245,17 @@ __device__ __forceinline__ void sc_fix_rows(int64_t i0, int64_t n, T (&ra)[SC_R]
 // rows are renormalised in registers by 2^-e (e = exponent of b; exact, a row
 // operation that leaves c', d' unchanged, reading X21), so any |b| in fp64's
 // range works.  Called after sc_fix_rows, on warp-converged code only.
+// fp32 rows are always scaled by 2^-e here (once per load; the product of 8 raw
+// fp32 rows would leave fp32's range beyond |b| ~ 2^16).
 template <typename T>
 __device__ __forceinline__ void sc_range(T (&ra)[SC_R], T (&rb)[SC_R], T (&rc)[SC_R], T (&rd)[SC_R]) {
-    if constexpr (sizeof(T) == 8) {
+    if constexpr (sizeof(T) == 4) {
+#pragma unroll
+        for (int u = 0; u < SC_R; ++u) {
+            const T s = sk_exp2_scale(rb[u]);
+            ra[u] *= s; rb[u] *= s; rc[u] *= s; rd[u] *= s;
+        }
+    } else {
         bool out = false;
 #pragma unroll
         for (int u = 0; u < SC_R; ++u) {
@@ -264,19 +272,11 @@ __device__ __forceinline__ void sc_range(T (&ra)[SC_R], T (&rb)[SC_R], T (&rc)[S
     }
 }
 
-// fp32 rows are scaled by 2^-e (e = exponent of b; exact, a row operation that
-// leaves c', d' unchanged, reading X21) before they enter the continuant, so the
-// product of 8 rows cannot overflow fp32's range (|b| up to 2^126 instead of
-// ~2^16); fp64 rows are renormalised by sc_range when needed.
+// row u of the lane (already renormalised by sc_range where needed)
 template <typename T>
 __device__ __forceinline__ void sc_row(const T (&ra)[SC_R], const T (&rb)[SC_R], const T (&rc)[SC_R],
                                        const T (&rd)[SC_R], int u, T& a, T& b, T& c, T& d) {
-    if constexpr (sizeof(T) == 4) {
-        const T s = sk_exp2_scale(rb[u]);
-        a = ra[u] * s; b = rb[u] * s; c = rc[u] * s; d = rd[u] * s;
-    } else {
-        a = ra[u]; b = rb[u]; c = rc[u]; d = rd[u];
-    }
+    a = ra[u]; b = rb[u]; c = rc[u]; d = rd[u];
 }
 
 // segment map of the lane's rows (forward state transfer, X21),

@@ -177,8 +177,24 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant
         ps0 = (T)__shfl_sync(0xffffffffu, b0 * sc0, 0);
         de0 = (T)__shfl_sync(0xffffffffu, c0 * sc0, 0);
     }
-    if (MODE == 2 && p.xafter) {  // look-back path: x after the small chunk that ends this chunk
-        xa0 = (T)p.xafter[(int64_t)((q * p.Ps + (w0 + nwin + p.NCWs - 1) / p.NCWs - 1)) * 16 + 14];
+    if (MODE == 2 && p.xafter && warp == 0) {
+        // look-back path: x after this chunk = the backward maps of the small chunks
+        // after it (records [12..13], written by k_scan_mc_lb) applied to x_end = 0
+        const int s1 = (w0 + nwin + p.NCWs - 1) / p.NCWs;  // first small chunk after this chunk
+        const double* r0 = p.xafter + (int64_t)(q * p.Ps + s1) * 16;
+        const int cnt = p.Ps - s1, per = (cnt + 31) / 32, lo = lane * per, hi = min(cnt, lo + per);
+        double al = 0.0, be = 1.0;
+        for (int k = hi - 1; k >= lo; --k) {
+            const double a2 = __ldcg(r0 + 16 * k + 12), b2 = __ldcg(r0 + 16 * k + 13);
+            al = fma(b2, al, a2);
+            be = b2 * be;
+        }
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const double oa = __shfl_down_sync(0xffffffffu, al, d), ob = __shfl_down_sync(0xffffffffu, be, d);
+            if ((lane & (2 * d - 1)) == 0) { al = fma(be, oa, al); be = be * ob; }
+        }
+        xa0 = (T)__shfl_sync(0xffffffffu, al, 0);
     } else if (MODE == 2 && warp == 0) {  // x after the chunk = (B_{ch+1} ... B_{P-1})(x_end), x_end = 0 or the slice's
         double al, be;
         smc_reduce_bwd(p.cbm + 8 * (q * p.P + ch + 1), p.P - 1 - ch, lane, al, be);
@@ -311,43 +327,54 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant
 }
 
 // ---- SCAN_MC with passes 0 and 1 fused by a decoupled look-back over small
-// chunks (TRI_SCAN_MC_LB): HBM traffic 4 + 2 (+ the
-// L2 re-read of each chunk) + 2 + 1 = 9 arrays instead of 13.
-// Persistent CTAs take chunks of NCWs windows in ticket order (an atomic
-// counter, so a CTA only ever waits on chunks that started before it).  Per
-// chunk: phase A = every window's forward map (as pass 0) and the chunk's
-// aggregate map, published with flag 1; warp 0 looks back over the earlier
-// chunks of the system (32 flags per round: the nearest inclusive state and
-// the aggregates after it) and publishes the chunk's inclusive state with flag
-// 2; phase B = pass 1 on the chunk (re-read from L2, prefetched during the
-// look-back).  k_scan_mc_lb_fin then turns the chunks' backward maps into the x
-// after every chunk, which pass 2 (k_scan_mc<2>, big chunks that are unions of
-// small ones) reads instead of reducing chunk maps.
-// Measured (c3, fp64 n = 2^24, B200; profiles/r01_ncu_c3_scanmc_lb.txt): correct
-// and bitwise reproducible, DRAM traffic as designed (586 MB read + 219 MB
-// written by the look-back kernel: the L2 re-read hits), but the kernel runs at
-// 3.3 TB/s -- 36 % of stall samples at __syncthreads while warp 0 reduces the
-// chunk and looks back -- so the solve takes 0.30-0.33 ms against 0.29 ms for
-// the three-pass path (small chunks of 24 / 32 / 48 / 64 / 80 windows: 0.39 /
-// 0.35 / 0.31-0.34 / 0.30-0.32 / 0.32 ms).  Now only warp 0 waits at the end
-// of phase A (the other warps arrive and start phase B; the next ticket, claimed
-// just in time after the look-back, travels with the state hand-over):
-// 0.380 / 0.342 / 0.307 / 0.301 ms at 24 / 32 / 48 / 64 windows.  Kept off by default
-// (TRI_SCAN_MC_LB=0); the lever is to overlap the look-back of chunk t with
-// phase A of chunk t + 1 (a dedicated look-back warp, two chunks per CTA in L2).
-// Tried and measured slower (not kept): a lag-1 pipeline in which warp 0 looks
-// back on chunk t - 1 after phase A of chunk t (so predecessors have had a phase
-// longer to publish): correct, but 0.33-0.41 ms -- barrier stalls rose to 43 %
-// and two chunks per CTA pushed the L2 re-read out (778 MB DRAM read;
-// profiles/r01_ncu_c3_scanmc_lb_lag1.txt): the bubble is warp 0's serial
-// reduce + publish, not waiting on flags.  Also measured and not kept: the
-// other warps only ARRIVE at the post-phase-A barrier (warp 0 alone waits) with
-// tickets claimed two chunks ahead: correct, but 2.3-2.7 ms -- a ticket
-// claimed before its CTA can start it stalls every later chunk's look-back on
-// its aggregate, so tickets must stay just-in-time.
+// chunks: HBM traffic 4 (+ an L2 re-read of each chunk) + 2 + 2
+// + 1 = 9 arrays instead of 13.  Persistent CTAs take chunks of NCWs windows in
+// ticket order (an atomic counter, so a CTA only ever waits on chunks that
+// started before it).  The CTA's warps are split by role, so that the HBM
+// stream of forward maps never waits for a look-back or for the replay chain:
+//   * LB_NA "A" warps: phase A of chunk i -- every window's forward map (lane
+//     segment maps composed over the warp, fp64), stored to shared memory
+//     (double-buffered by chunk parity); windows streamed from HBM by TMA, two
+//     in flight per warp, L2 evict_normal so phase B finds them in L2;
+//   * one "L" warp: the chunk's aggregate map (flag 1), the look-back with a
+//     FIXED structure (bitwise reproducible: the inclusive state of the chunk at
+//     the largest multiple of 32 below, plus the aggregates after it, one round
+//     of 32 flags), the chunk's inclusive state (flag 2), and the incoming state
+//     handed to the B warps;
+//   * LB_NB "B" warps: phase B of chunk i - 1 or earlier -- the forward replay of
+//     the chunk (re-read from L2) from every window's incoming state (the L warp
+//     scans the chunk's window maps from the chunk's incoming state, so the
+//     windows need no chain), c', d' to scratch, every window's back-substitution
+//     map and the chunk's (record [12..13]).
+// Roles hand chunks over through mbarriers in shared memory (ticket ring,
+// maps full / free, state full / free), at most a few chunks apart.
+// Pass 2 (k_scan_mc<2>, big chunks that are unions of small ones) then reduces
+// the backward maps of the small chunks after its chunk into the x after it.
 // record per small chunk (16 values): [0..6] aggregate map, [8..10] inclusive
-// state, [12..13] backward map (al, be), [14] x after the chunk
+// state, [12..13] backward map (al, be)
 constexpr int SMC_REC = 16;
+constexpr int LB_NA = 5;                           // phase-A warps
+constexpr int LB_NB = 10;                          // phase-B warps (chain barriers 1 .. LB_NB)
+constexpr int LB_WARPS = LB_NA + LB_NB + 1;        // + the look-back warp
+constexpr int LB_THREADS = 32 * LB_WARPS;
+constexpr int LB_MAXW = 64;                        // windows per small chunk
+constexpr int LB_RING = 8;                         // ticket ring (roles are at most ~4 chunks apart)
+static_assert(LB_NB + 1 <= 15, "named barriers 1 .. LB_NB + 1");
+
+template <typename T>
+struct LBLayout {
+    static constexpr int in_stride = SMCLayout<T>::in_stride;
+    static constexpr int off_a = 0;                                  // [NA][2] staging
+    static constexpr int off_b = off_a + LB_NA * 2 * in_stride;      // [NB] staging
+    static constexpr int off_wm = off_b + LB_NB * in_stride;         // [2][MAXW][8] fwd window maps (fp64)
+    static constexpr int off_wb = off_wm + 2 * LB_MAXW * 8 * 8;      // [2][MAXW][2] bwd window maps (fp64)
+    static constexpr int off_st = off_wb + 2 * LB_MAXW * 2 * 8;      // [2][MAXW][4] windows' incoming states (fp64)
+    static constexpr int off_tk = off_st + 2 * LB_MAXW * 4 * 8;      // [RING] tickets
+    static constexpr int off_bar = (off_tk + LB_RING * 4 + 15) / 16 * 16;
+    // mbarriers: a_full[NA][2], b_full[NB], tkfull[RING], mapsfull[2], wmfree[2], statefull[2], stfree[2], bdone[2]
+    static constexpr int nbar = 2 * LB_NA + LB_NB + LB_RING + 10;
+    static constexpr int smem_bytes = off_bar + nbar * 8 + 1024;
+};
 
 __device__ __forceinline__ unsigned smc_ld_acquire_gpu(const unsigned* p) {
     unsigned v;
@@ -361,274 +388,364 @@ __device__ __forceinline__ void smc_st_release_gpu(unsigned* p, unsigned v) {
 template <typename T>
 struct ScanMCLB {
     double* rec;       // [m Ps][SMC_REC] (fp64 for both dtypes)
-    unsigned* flag;    // [m Ps] (zeroed before the launch), then the ticket counter at [m Ps]
-    int NCWs, Ps;      // windows per small chunk, small chunks per system
+    double* brec;      // [m Pb][8] block aggregates (32 chunks each)
+    unsigned* flag;    // [m Ps] chunk flags (1 aggregate, 2 + incoming state), the ticket counter at [m Ps],
+                       // then [m Pb] block flags (1 aggregate); all zeroed before the launch
+    int NCWs, Ps, Pb;  // windows per small chunk (<= LB_MAXW), small chunks per system, blocks per system
+    unsigned long long* prof;  // diagnostics (tri_debug_set_profile): [m Ps][8] %globaltimer stamps per chunk, or null
 };
+__device__ __forceinline__ unsigned long long lb_now() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
+
+// Look-back step of the L warp (warp-wide): the product M_{j0} M_{j0-1} ... M_{j0-cnt+1}
+// of cnt <= 32 published aggregate maps (map i at rec + i * stride, flag fl[i] >= 1;
+// lane l polls and reads map j0 - l, so each lane reads only what it acquired),
+// applied to a base state (3 values at base, flag *bfl >= 2, polled and read by
+// lane 0), or to `s` when base is null.  Fixed composition order: bitwise
+// reproducible.  Returns the state on every lane.
+__device__ __forceinline__ void lb_lookback(const double* rec, int stride, const unsigned* fl, int j0, int cnt,
+                                            const double* base, const unsigned* bfl, int lane, double (&s)[3]) {
+    const unsigned want = lane < cnt ? 1u : 0u;
+    const bool wb = base != nullptr && lane == 0;
+    while (true) {
+        const unsigned v = want ? smc_ld_acquire_gpu(fl + (j0 - lane)) : 0u;
+        const unsigned vb = wb ? smc_ld_acquire_gpu(bfl) : 2u;
+        if (!__any_sync(0xffffffffu, v < want || vb < 2u)) break;
+        __nanosleep(32);
+    }
+    SCM A{1.0, 0.0, 0.0, 1.0, 0.0, 0.0, 1.0};
+    if (lane < cnt) {
+        const double* r = rec + (int64_t)(j0 - lane) * stride;
+        A = SCM{__ldcg(r + 0), __ldcg(r + 1), __ldcg(r + 2), __ldcg(r + 3), __ldcg(r + 4), __ldcg(r + 5), __ldcg(r + 6)};
+    }
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {  // lane l: maps j0-l .. j0-l-2d+1 (lane l latest)
+        const SCM o = sk_shfl_down(A, d);
+        if ((lane & (2 * d - 1)) == 0) { A = sk_compose(A, o); smc_rescale(A); }
+    }
+    double th = s[0], ps = s[1], de = s[2];
+    if (wb) { th = __ldcg(base + 0); ps = __ldcg(base + 1); de = __ldcg(base + 2); }
+    const double ot = fma(A.a, th, A.b * ps), op = fma(A.c, th, A.d * ps), od = fma(A.e, th, fma(A.f, ps, A.g * de));
+    const double sc = sk_exp2_scale(ot);
+    s[0] = __shfl_sync(0xffffffffu, ot * sc, 0);
+    s[1] = __shfl_sync(0xffffffffu, op * sc, 0);
+    s[2] = __shfl_sync(0xffffffffu, od * sc, 0);
+}
 
 template <typename T>
-__global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc_lb(const __grid_constant__ StreamMaps tm, ScanMCArgs<T> p,
+__global__ void __launch_bounds__(LB_THREADS, 1) k_scan_mc_lb(const __grid_constant__ StreamMaps tm, ScanMCArgs<T> p,
                                                                ScanMCLB<T> lb) {
-    using L = SMCLayout<T>;
+    using L = LBLayout<T>;
     extern __shared__ __align__(16) unsigned char smc_smem_raw[];
-    __shared__ int s_tk[2];
-    __shared__ T s_st[4];
     unsigned char* sbase = smc_smem_raw + ((1024 - ((unsigned)__cvta_generic_to_shared(smc_smem_raw) & 1023)) & 1023);
-    uint64_t* in_full = reinterpret_cast<uint64_t*>(sbase + L::off_bar);
-    T* hv = reinterpret_cast<T*>(sbase + L::off_hv);
+    uint64_t* bars = reinterpret_cast<uint64_t*>(sbase + L::off_bar);
+    uint64_t* a_full = bars;                          // [NA][2]
+    uint64_t* b_full = a_full + 2 * LB_NA;            // [NB]
+    uint64_t* tkfull = b_full + LB_NB;                // [RING]
+    uint64_t* mapsfull = tkfull + LB_RING;            // [2]
+    uint64_t* wmfree = mapsfull + 2;                  // [2]
+    uint64_t* statefull = wmfree + 2;                 // [2]
+    uint64_t* stfree = statefull + 2;                 // [2]
+    uint64_t* bdone = stfree + 2;                     // [2] B finished a chunk (throttles A: L2 reuse)
     double* wm0 = reinterpret_cast<double*>(sbase + L::off_wm);
-    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, pw = warp;
+    double* wb0 = reinterpret_cast<double*>(sbase + L::off_wb);
+    double* st0 = reinterpret_cast<double*>(sbase + L::off_st);
+    int* tk = reinterpret_cast<int*>(sbase + L::off_tk);
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     if (threadIdx.x == 0) {
-        for (int i = 0; i < SC_NW; ++i) sk_bar_init(&in_full[i], 1);
+        for (int k = 0; k < 2 * LB_NA + LB_NB; ++k) sk_bar_init(&bars[k], 1);
+        for (int k = 0; k < LB_RING; ++k) sk_bar_init(&tkfull[k], 1);
+        for (int k = 0; k < 2; ++k) {
+            sk_bar_init(&mapsfull[k], LB_NA);
+            sk_bar_init(&wmfree[k], 1);
+            sk_bar_init(&statefull[k], 1);
+            sk_bar_init(&stfree[k], 1);
+            sk_bar_init(&bdone[k], 1);
+        }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-        s_tk[0] = (int)atomicAdd(&lb.flag[p.m * (int64_t)lb.Ps], 1u);
     }
     __syncthreads();
     const int64_t n = p.n;
     const int NC = p.NC, NCW = lb.NCWs;
     const int total = (int)(p.m * lb.Ps);
-    T* ib = reinterpret_cast<T*>(sbase + L::off_in + pw * L::in_stride);
-    const unsigned ib_s = (unsigned)__cvta_generic_to_shared(ib);
-    (void)ib_s;
-    const uint64_t pol_a = sk_policy_evict_normal();  // phase A: keep the chunk in L2 for phase B
-    const uint64_t pol_b = sk_policy_evict_first();   // phase B: last use
-    auto issue = [&](int q, int w, uint64_t pol) {
-        const int y = w * (p.w128 ? SC_W * (int)sizeof(T) / 128 : SC_W / 8);
-        sk_expect(&in_full[pw], (unsigned)(4 * SC_W * sizeof(T)));
-        sc_tma3d(ib + 0 * SC_W, &tm.a, y, q, &in_full[pw], pol);
-        sc_tma3d(ib + 1 * SC_W, &tm.b, y, q, &in_full[pw], pol);
-        sc_tma3d(ib + 2 * SC_W, &tm.c, y, q, &in_full[pw], pol);
-        sc_tma3d(ib + 3 * SC_W, &tm.d, y, q, &in_full[pw], pol);
+    unsigned* counter = &lb.flag[total];
+    auto nwin_of = [&](int t) {
+        const int ch = t % lb.Ps;
+        return min(NC, ch * NCW + NCW) - ch * NCW;
     };
-    unsigned ph = 0;
-    int par = 0;
-    int t = s_tk[0];
-    const int pi = (pw + SC_NW - 1) % SC_NW;
-    if (t < total && lane == 0) {
-        const int q = t / lb.Ps, ch = t - q * lb.Ps;
-        if (pw < min(NC, ch * NCW + NCW) - ch * NCW) issue(q, ch * NCW + pw, pol_a);
-    }
-    while (t < total) {
-        const int q = t / lb.Ps, ch = t - q * lb.Ps;
-        const int w0 = ch * NCW;
-        const int nwin = min(NC, w0 + NCW) - w0;
-        double* wm = wm0 + par * 8 * NCW;          // forward window maps (phase A)
-        double* wmb = wm0 + (2 + par) * 8 * NCW;   // backward window maps (phase B)
-        // ---- phase A: window forward maps
-        for (int g = pw; g < nwin; g += SC_NW) {
-            const int w = w0 + g;
-            const int64_t i0 = (int64_t)w * SC_W + lane * SC_R;
-            const bool edge = w == 0 || (int64_t)(w + 1) * SC_W > n;
-            sk_wait(&in_full[pw], ph);
-            ph ^= 1u;
-            T ra[SC_R], rb[SC_R], rc[SC_R], rd[SC_R];
-            sc_ld_rows_any(ib, lane, p.w128 != 0, ra, rb, rc, rd);
-            sc_release_buf();
-            if (lane == 0) {
-                if (g + SC_NW < nwin) issue((int)q, w + SC_NW, pol_a);
-                else issue((int)q, w0 + pw, pol_b);  // phase B's first window, during the look-back
+    auto issue = [&](T* buf, uint64_t* bar, int t, int g, uint64_t pol) {
+        const int q = t / lb.Ps, w = (t - q * lb.Ps) * NCW + g;
+        const int y = w * (p.w128 ? SC_W * (int)sizeof(T) / 128 : SC_W / 8);
+        sk_expect(bar, (unsigned)(4 * SC_W * sizeof(T)));
+        sc_tma3d(buf + 0 * SC_W, &tm.a, y, q, bar, pol);
+        sc_tma3d(buf + 1 * SC_W, &tm.b, y, q, bar, pol);
+        sc_tma3d(buf + 2 * SC_W, &tm.c, y, q, bar, pol);
+        sc_tma3d(buf + 3 * SC_W, &tm.d, y, q, bar, pol);
+    };
+    auto load_rows = [&](const T* buf, int t, int g, T (&ra)[SC_R], T (&rb)[SC_R], T (&rc)[SC_R], T (&rd)[SC_R]) {
+        const int q = t / lb.Ps, w = (t - q * lb.Ps) * NCW + g;
+        const int64_t i0 = (int64_t)w * SC_W + lane * SC_R;
+        sc_ld_rows_any(buf, lane, p.w128 != 0, ra, rb, rc, rd);
+        if (w == 0 || (int64_t)(w + 1) * SC_W > n) sc_fix_rows<T>(i0, n, ra, rb, rc, rd, 0, 0);
+        sc_range(ra, rb, rc, rd);
+    };
+
+    if (warp < LB_NA) {
+        // ======================= A: forward window maps =======================
+        const int aw = warp;
+        T* buf[2] = {reinterpret_cast<T*>(sbase + L::off_a + (2 * aw) * L::in_stride),
+                     reinterpret_cast<T*>(sbase + L::off_a + (2 * aw + 1) * L::in_stride)};
+        const uint64_t pol = sk_policy_evict_normal();  // phase B re-reads the chunk from L2
+        unsigned ph2 = 0;                                // bit b: phase of buffer b
+        int nb = 0;                                      // loads issued by this warp (buffer = nb & 1)
+        int nc = 0;                                      // loads consumed
+        for (int i = 0;; ++i) {
+            const int par = i & 1;
+            if (aw == 0 && lane == 0) {  // the ticket of chunk i, just in time
+                tk[i % LB_RING] = (int)atomicAdd(counter, 1u);
+                sk_arrive(&tkfull[i % LB_RING]);
             }
-            if (edge) sc_fix_rows<T>(i0, n, ra, rb, rc, rd, 0, 0);
-            sc_range(ra, rb, rc, rd);
-            SCM M = sc_wide(sc_fwd_map(ra, rb, rc, rd));
+            sk_wait(&tkfull[i % LB_RING], (unsigned)((i / LB_RING) & 1));
+            const int t = tk[i % LB_RING];
+            if (t >= total) {
+                if (i >= 2) sk_wait(&wmfree[par], (unsigned)(((i >> 1) - 1) & 1));  // never two phases ahead of L
+                if (lane == 0) sk_arrive(&mapsfull[par]);  // tells the L warp: no more chunks
+                break;
+            }
+            const int nwin = nwin_of(t);
+            if (lb.prof && aw == 0 && lane == 0) lb.prof[(int64_t)t * 8 + 0] = lb_now();
+            double* wm = wm0 + par * LB_MAXW * 8;
+            // at most one chunk ahead of the B warps: the chunk phase B re-reads must
+            // still be in L2 (148 CTAs x 2 chunks x 256 KB = 76 MB of the 126 MB)
+            if (i >= 2) sk_wait(&bdone[par], (unsigned)(((i >> 1) - 1) & 1));
+            // first two windows of this warp (before waiting for the map buffer)
+            if (lane == 0) {
+                for (int g = aw; g < nwin && g < aw + 2 * LB_NA; g += LB_NA, ++nb) issue(buf[nb & 1], &a_full[2 * aw + (nb & 1)], t, g, pol);
+            } else {
+                for (int g = aw; g < nwin && g < aw + 2 * LB_NA; g += LB_NA) ++nb;
+            }
+            if (i >= 2) sk_wait(&wmfree[par], (unsigned)(((i >> 1) - 1) & 1));  // L has read chunk i - 2's maps
+            for (int g = aw; g < nwin; g += LB_NA, ++nc) {
+                const int bsel = nc & 1;
+                sk_wait(&a_full[2 * aw + bsel], (ph2 >> bsel) & 1u);
+                ph2 ^= 1u << bsel;
+                T ra[SC_R], rb[SC_R], rc[SC_R], rd[SC_R];
+                load_rows(buf[bsel], t, g, ra, rb, rc, rd);
+                sc_release_buf();  // this warp's reads of the buffer before the TMA refill
+                if (g + 2 * LB_NA < nwin) {
+                    if (lane == 0) issue(buf[bsel], &a_full[2 * aw + bsel], t, g + 2 * LB_NA, pol);
+                    ++nb;
+                }
+                SCM M = sc_wide(sc_fwd_map(ra, rb, rc, rd));
 #pragma unroll
-            for (int d = 1; d < 32; d <<= 1) {
-                const SCM o = sk_shfl_down(M, d);
-                if ((lane & (2 * d - 1)) == 0) { M = sk_compose(o, M); smc_rescale(M); }
+                for (int d = 1; d < 32; d <<= 1) {  // lane l: lanes l .. l + 2d - 1 (later after earlier)
+                    const SCM o = sk_shfl_down(M, d);
+                    if ((lane & (2 * d - 1)) == 0) { M = sk_compose(o, M); smc_rescale(M); }
+                }
+                if (lane == 0) {
+                    double* s = wm + 8 * g;
+                    s[0] = M.a; s[1] = M.b; s[2] = M.c; s[3] = M.d; s[4] = M.e; s[5] = M.f; s[6] = M.g;
+                }
             }
-            if (lane == 0) {
-                double* s = wm + 8 * g;
-                s[0] = M.a; s[1] = M.b; s[2] = M.c; s[3] = M.d; s[4] = M.e; s[5] = M.f; s[6] = M.g;
-            }
+            __syncwarp();
+            if (lb.prof && aw == 0 && lane == 0) lb.prof[(int64_t)t * 8 + 1] = lb_now();
+            if (lane == 0) sk_arrive(&mapsfull[par]);  // release: this warp's maps are in shared memory
         }
-        // warp 0 waits for every warp's window maps; the others go straight on to
-        // phase B (their chain waits for warp 0's first window anyway)
-        if (warp == 0) asm volatile("bar.sync 13, %0;" ::"r"(SC_THREADS) : "memory");
-        else asm volatile("bar.arrive 13, %0;" ::"r"(SC_THREADS) : "memory");
-        if (warp == 0) {
-            // aggregate of the chunk, published with flag 1
-            const SCM R = smc_reduce_fwd(wm, nwin, lane);  // lane 0
+    } else if (warp == LB_NA) {
+        // ======================= L: aggregate, look-back, incoming state =======================
+        unsigned* fl = lb.flag;
+        for (int i = 0;; ++i) {
+            const int par = i & 1;
+            sk_wait(&mapsfull[par], (unsigned)((i >> 1) & 1));
+            const int t = tk[i % LB_RING];
+            if (i >= 2) sk_wait(&stfree[par], (unsigned)(((i >> 1) - 1) & 1));  // B has read chunk i - 2's state
+            if (t >= total) {
+                if (lane == 0) {
+                    st0[4 * par + 3] = (double)t;
+                    sk_arrive(&statefull[par]);
+                }
+                break;
+            }
+            const int nwin = nwin_of(t);
+            const int q = t / lb.Ps, ch = t - q * lb.Ps;
+            if (lb.prof && lane == 0) lb.prof[(int64_t)t * 8 + 2] = lb_now();
+            const SCM R = smc_reduce_fwd(wm0 + par * LB_MAXW * 8, nwin, lane);  // lane 0
             double* rec = lb.rec + (int64_t)t * SMC_REC;
-            unsigned* fl = lb.flag;
-            if (lane == 0 && ch > 0) {
+            if (lane == 0) {  // the aggregate, published with flag 1
                 __stcg(rec + 0, R.a); __stcg(rec + 1, R.b); __stcg(rec + 2, R.c); __stcg(rec + 3, R.d);
                 __stcg(rec + 4, R.e); __stcg(rec + 5, R.f); __stcg(rec + 6, R.g);
                 smc_st_release_gpu(fl + t, 1u);  // release: the stores above are visible first
             }
-            // look-back with a FIXED structure (bitwise reproducible): incoming state =
-            // A_{t-1} ... A_{b+1} S_b, b = the chunk of the system at the largest multiple
-            // of 32 below ch (S_b inclusive, published with flag 2), so one round of 32
-            // flags; ch <= 32 starts from the system start when b = 0 ... and b's own
-            // inclusive state is built the same way from its base
-            SCM acc{1.0, 0.0, 0.0, 1.0, 0.0, 0.0, 1.0};
-            double th = 1.0, ps = 0.0, de = 0.0;
-            if (ch > 0) {
-                const int tfirst = (int)(q * lb.Ps);
-                const int b = tfirst + ((ch - 1) / 32) * 32;  // base chunk (inclusive state)
-                const int nag = t - 1 - b;                     // aggregates after it, lanes 0 .. nag - 1
-                const int j = t - 1 - lane;
-                const unsigned want = lane < nag ? 1u : (lane == nag ? 2u : 0u);
-                while (true) {
-                    const unsigned v = want ? smc_ld_acquire_gpu(fl + j) : 0u;
-                    if (!__any_sync(0xffffffffu, v < want)) break;
-                    __nanosleep(32);
-                }
-                SCM A{1.0, 0.0, 0.0, 1.0, 0.0, 0.0, 1.0};
-                if (lane < nag) {
-                    const double* r = lb.rec + (int64_t)j * SMC_REC;
-                    A = SCM{__ldcg(r + 0), __ldcg(r + 1), __ldcg(r + 2), __ldcg(r + 3), __ldcg(r + 4),
-                            __ldcg(r + 5), __ldcg(r + 6)};
-                }
+            // Look-back with a FIXED two-level structure (bitwise reproducible, and no
+            // serial chain through every 32nd chunk): blocks of 32 chunks; the last chunk
+            // of a block publishes the block's aggregate; the first chunk of block K
+            // publishes its incoming state E_32K = BA_{K-1} ... BA_{32J} E_1024J (J =
+            // K / 32, the block aggregates since the last 1024-chunk boundary; at that
+            // boundary the 32 block aggregates before it and E of the previous one);
+            // any other chunk: E_t = A_{t-1} ... A_{32K} E_32K.
+            const int tfirst = q * lb.Ps, K = ch / 32;
+            unsigned* bfl = fl + total + 1;
+            if (ch % 32 == 31) {  // the block aggregate BA_K = A_t ... A_32K
+                SCM BA{1.0, 0.0, 0.0, 1.0, 0.0, 0.0, 1.0};
+                {
+                    const int cnt = 32;
+                    while (true) {
+                        const unsigned v = lane < cnt ? smc_ld_acquire_gpu(fl + (t - lane)) : 1u;
+                        if (!__any_sync(0xffffffffu, v < 1u)) break;
+                        __nanosleep(32);
+                    }
+                    const double* r = lb.rec + (int64_t)(t - lane) * SMC_REC;
+                    BA = SCM{__ldcg(r + 0), __ldcg(r + 1), __ldcg(r + 2), __ldcg(r + 3), __ldcg(r + 4), __ldcg(r + 5),
+                             __ldcg(r + 6)};
 #pragma unroll
-                for (int d = 1; d < 32; d <<= 1) {  // lane l: A_{j_l} ... A_{j_{l+2d-1}} (lane l latest)
-                    const SCM o = sk_shfl_down(A, d);
-                    if ((lane & (2 * d - 1)) == 0) { A = sk_compose(A, o); smc_rescale(A); }
+                    for (int d = 1; d < 32; d <<= 1) {
+                        const SCM o = sk_shfl_down(BA, d);
+                        if ((lane & (2 * d - 1)) == 0) { BA = sk_compose(BA, o); smc_rescale(BA); }
+                    }
                 }
-                acc.a = __shfl_sync(0xffffffffu, A.a, 0); acc.b = __shfl_sync(0xffffffffu, A.b, 0);
-                acc.c = __shfl_sync(0xffffffffu, A.c, 0); acc.d = __shfl_sync(0xffffffffu, A.d, 0);
-                acc.e = __shfl_sync(0xffffffffu, A.e, 0); acc.f = __shfl_sync(0xffffffffu, A.f, 0);
-                acc.g = __shfl_sync(0xffffffffu, A.g, 0);
-                const double* r = lb.rec + (int64_t)b * SMC_REC;
-                th = __ldcg(r + 8); ps = __ldcg(r + 9); de = __ldcg(r + 10);
+                if (lane == 0) {
+                    double* br = lb.brec + (int64_t)(q * lb.Pb + K) * 8;
+                    __stcg(br + 0, BA.a); __stcg(br + 1, BA.b); __stcg(br + 2, BA.c); __stcg(br + 3, BA.d);
+                    __stcg(br + 4, BA.e); __stcg(br + 5, BA.f); __stcg(br + 6, BA.g);
+                    smc_st_release_gpu(bfl + q * lb.Pb + K, 1u);
+                }
             }
-            const double it = fma(acc.a, th, acc.b * ps);
-            const double ip = fma(acc.c, th, acc.d * ps);
-            const double id = fma(acc.e, th, fma(acc.f, ps, acc.g * de));
-            // inclusive state of this chunk, published with flag 2
-            double ot = fma(R.a, it, R.b * ip), op = fma(R.c, it, R.d * ip), od = fma(R.e, it, fma(R.f, ip, R.g * id));
-            if (lane == 0) {
-                const double sc = sk_exp2_scale(ot);
-                ot *= sc; op *= sc; od *= sc;
-                __stcg(rec + 8, ot); __stcg(rec + 9, op); __stcg(rec + 10, od);
+            double E[3] = {1.0, 0.0, 0.0};  // the system's start
+            if (ch % 32 != 0) {
+                lb_lookback(lb.rec, SMC_REC, fl, t - 1, ch % 32, lb.rec + (int64_t)(tfirst + 32 * K) * SMC_REC + 8,
+                            fl + tfirst + 32 * K, lane, E);
+            } else if (K > 0) {
+                const int J = K / 32;
+                const int kb = K % 32 != 0 ? 32 * J : K - 32;  // blocks kb .. K-1, base chunk 32 kb
+                lb_lookback(lb.brec + (int64_t)(q * lb.Pb) * 8, 8, bfl + q * lb.Pb, K - 1, K - kb,
+                            kb > 0 ? lb.rec + (int64_t)(tfirst + 32 * kb) * SMC_REC + 8 : nullptr,
+                            kb > 0 ? fl + tfirst + 32 * kb : nullptr, lane, E);
+            }
+            if (lane == 0 && ch % 32 == 0) {  // block start: publish the incoming state with flag 2
+                __stcg(rec + 8, E[0]); __stcg(rec + 9, E[1]); __stcg(rec + 10, E[2]);
                 smc_st_release_gpu(fl + t, 2u);
-                const double si = sk_exp2_scale(it);
-                s_st[0] = (T)(it * si); s_st[1] = (T)(ip * si); s_st[2] = (T)(id * si);
-                s_tk[par ^ 1] = (int)atomicAdd(&lb.flag[total], 1u);  // the next chunk, just in time
             }
-        }
-        __syncwarp();
-        // the next ticket: warp 0 from shared memory; the others through the chain
-        // (hv[4 w + 3], handed over with the state); warps with no window here after
-        // the end-of-chunk barrier
-        int tn = warp == 0 ? s_tk[par ^ 1] : total;
-        // ---- phase B: forward replay (pass 1) from the chunk's incoming state
-        for (int g = pw; g < nwin; g += SC_NW) {
-            const int w = w0 + g;
-            const int64_t i0 = (int64_t)w * SC_W + lane * SC_R;
-            const bool edge = w == 0 || (int64_t)(w + 1) * SC_W > n;
-            sk_wait(&in_full[pw], ph);
-            ph ^= 1u;
-            T ra[SC_R], rb[SC_R], rc[SC_R], rd[SC_R];
-            sc_ld_rows_any(ib, lane, p.w128 != 0, ra, rb, rc, rd);
-            if (edge) sc_fix_rows<T>(i0, n, ra, rb, rc, rd, 0, 0);
-            sc_range(ra, rb, rc, rd);
-            SCM M = sc_wide(sc_fwd_map(ra, rb, rc, rd));
-            sc_fwd_scan(M, lane);
-            if (g > 0) asm volatile("bar.sync %0, 64;" ::"r"(1 + pi) : "memory");
-            T th, ps, de;
-            if (g == 0) {
-                th = s_st[0]; ps = s_st[1]; de = s_st[2];
-            } else {
-                th = hv[4 * pi + 0]; ps = hv[4 * pi + 1]; de = hv[4 * pi + 2];
-                tn = (int)hv[4 * pi + 3];
-            }
-            const double ot = fma(M.a, (double)th, M.b * (double)ps);
-            const double op = fma(M.c, (double)th, M.d * (double)ps);
-            const double od = fma(M.e, (double)th, fma(M.f, (double)ps, M.g * (double)de));
-            if (lane == 31) {
-                const double sc = sk_exp2_scale(ot);
-                hv[4 * pw + 0] = (T)(ot * sc); hv[4 * pw + 1] = (T)(op * sc); hv[4 * pw + 2] = (T)(od * sc);
-                hv[4 * pw + 3] = (T)tn;
-            }
-            if (g + 1 < nwin) asm volatile("bar.arrive %0, 64;" ::"r"(1 + pw) : "memory");
+            // every window's incoming state: the window maps scanned over the lanes
+            // (two windows per lane when NCWs > 32), applied to E -- the B warps then
+            // need no chain between windows
             {
-                const T it_ = (T)__shfl_up_sync(0xffffffffu, ot, 1);
-                const T ip = (T)__shfl_up_sync(0xffffffffu, op, 1);
-                const T id = (T)__shfl_up_sync(0xffffffffu, od, 1);
-                if (lane > 0) { th = it_; ps = ip; de = id; }
-            }
-            sc_release_buf();
-            if (lane == 0) {
-                if (g + SC_NW < nwin) {
-                    issue((int)q, w + SC_NW, pol_b);
-                } else if (tn < total) {  // the next chunk's first window for this warp
-                    const int qn = tn / lb.Ps, chn = tn - qn * lb.Ps;
-                    if (pw < min(NC, chn * NCW + NCW) - chn * NCW) issue(qn, chn * NCW + pw, pol_a);
+                const double* wm = wm0 + par * LB_MAXW * 8;
+                double* ws = st0 + par * LB_MAXW * 4;
+                double s[3] = {E[0], E[1], E[2]};
+                for (int base = 0; base < nwin; base += 32) {
+                    const int g = base + lane;
+                    SCM W{1.0, 0.0, 0.0, 1.0, 0.0, 0.0, 1.0};
+                    if (g < nwin) { const double* m = wm + 8 * g; W = SCM{m[0], m[1], m[2], m[3], m[4], m[5], m[6]}; }
+                    sc_fwd_scan(W, lane);  // lane l: W_{base+l} ... W_base
+                    // state entering window g = (W_{g-1} ... W_base) s
+                    SCM X = sk_shfl_up(W, 1);
+                    if (lane == 0) X = SCM{1.0, 0.0, 0.0, 1.0, 0.0, 0.0, 1.0};
+                    const double xt = fma(X.a, s[0], X.b * s[1]), xp = fma(X.c, s[0], X.d * s[1]),
+                                 xd = fma(X.e, s[0], fma(X.f, s[1], X.g * s[2]));
+                    const double sc = sk_exp2_scale(xt);
+                    if (g < nwin) { ws[4 * g + 0] = xt * sc; ws[4 * g + 1] = xp * sc; ws[4 * g + 2] = xd * sc; }
+                    // the state after this group of 32 windows, for the next group
+                    const double yt = fma(W.a, s[0], W.b * s[1]), yp = fma(W.c, s[0], W.d * s[1]),
+                                 yd = fma(W.e, s[0], fma(W.f, s[1], W.g * s[2]));
+                    const double sy = sk_exp2_scale(yt);
+                    s[0] = __shfl_sync(0xffffffffu, yt * sy, 31);
+                    s[1] = __shfl_sync(0xffffffffu, yp * sy, 31);
+                    s[2] = __shfl_sync(0xffffffffu, yd * sy, 31);
                 }
             }
-            T cp[SC_R], dp[SC_R];
-            sc_fwd_replay(ra, rb, rc, rd, th, ps, de, cp, dp);
-            T* dst = p.cd + (q * NC + w) * (int64_t)sc_slot_elems<T>();
-            if constexpr (sizeof(T) == 8) {
-#pragma unroll
-                for (int u = 0; u < SC_R; ++u)
-                    __stcg(reinterpret_cast<double2*>(dst + 2 * sc_chunk<T>(lane, u)), make_double2(cp[u], dp[u]));
-            } else {
-#pragma unroll
-                for (int u = 0; u < SC_R / 2; ++u)
-                    __stcg(reinterpret_cast<float4*>(dst + 4 * sc_chunk<T>(lane, u)),
-                           make_float4(cp[2 * u], dp[2 * u], cp[2 * u + 1], dp[2 * u + 1]));
+            __syncwarp();
+            if (lane == 0) {
+                if (lb.prof) lb.prof[(int64_t)t * 8 + 3] = lb_now();
+                sk_arrive(&wmfree[par]);     // the window maps are consumed
+                sk_arrive(&statefull[par]);  // release: the window states are in shared memory
             }
-            T al, be;
-            sc_bwd_map(cp, dp, al, be);
+        }
+    } else {
+        // ======================= B: forward replay, c', d', backward maps =======================
+        const int bw = warp - LB_NA - 1;
+        T* buf = reinterpret_cast<T*>(sbase + L::off_b + bw * L::in_stride);
+        const uint64_t pol = sk_policy_evict_first();  // last use of the chunk's rows
+        unsigned ph = 0;
+        for (int i = 0;; ++i) {
+            const int par = i & 1;
+            sk_wait(&tkfull[i % LB_RING], (unsigned)((i / LB_RING) & 1));
+            const int t = tk[i % LB_RING];
+            if (t >= total) break;
+            const int nwin = nwin_of(t);
+            const int q = t / lb.Ps, w0 = (t - q * lb.Ps) * NCW;
+            if (lane == 0 && bw < nwin) issue(buf, &b_full[bw], t, bw, pol);  // prefetch before the state is known
+            if (lb.prof && bw == 0 && lane == 0) lb.prof[(int64_t)t * 8 + 4] = lb_now();
+            sk_wait(&statefull[par], (unsigned)((i >> 1) & 1));
+            if (lb.prof && bw == 0 && lane == 0) lb.prof[(int64_t)t * 8 + 5] = lb_now();
+            double* wb = wb0 + par * LB_MAXW * 2;
+            for (int g = bw; g < nwin; g += LB_NB) {
+                const int w = w0 + g;
+                sk_wait(&b_full[bw], ph);
+                ph ^= 1u;
+                T ra[SC_R], rb[SC_R], rc[SC_R], rd[SC_R];
+                load_rows(buf, t, g, ra, rb, rc, rd);
+                sc_release_buf();
+                if (lane == 0 && g + LB_NB < nwin) issue(buf, &b_full[bw], t, g + LB_NB, pol);  // rows are in registers
+                SCM M = sc_wide(sc_fwd_map(ra, rb, rc, rd));
+                sc_fwd_scan(M, lane);
+                const double* ws = st0 + par * LB_MAXW * 4 + 4 * g;  // the window's incoming state (L warp)
+                const double th = ws[0], ps = ws[1], de = ws[2];
+                const double ot = fma(M.a, th, M.b * ps);
+                const double op = fma(M.c, th, M.d * ps);
+                const double od = fma(M.e, th, fma(M.f, ps, M.g * de));
+                T lt, lp, ld;
+                {
+                    const double it_ = __shfl_up_sync(0xffffffffu, ot, 1);
+                    const double ip = __shfl_up_sync(0xffffffffu, op, 1);
+                    const double id = __shfl_up_sync(0xffffffffu, od, 1);
+                    const double sc = sk_exp2_scale(lane > 0 ? it_ : th);
+                    lt = (T)((lane > 0 ? it_ : th) * sc);
+                    lp = (T)((lane > 0 ? ip : ps) * sc);
+                    ld = (T)((lane > 0 ? id : de) * sc);
+                }
+                T cp[SC_R], dp[SC_R];
+                sc_fwd_replay(ra, rb, rc, rd, lt, lp, ld, cp, dp);
+                T* dst = p.cd + (q * NC + w) * (int64_t)sc_slot_elems<T>();
+                if constexpr (sizeof(T) == 8) {
 #pragma unroll
-            for (int d = 1; d < 32; d <<= 1) {
-                const T oa = __shfl_down_sync(0xffffffffu, al, d), ob = __shfl_down_sync(0xffffffffu, be, d);
-                if ((lane & (2 * d - 1)) == 0) { al = fma(be, oa, al); be = be * ob; }
+                    for (int u = 0; u < SC_R; ++u)
+                        __stcg(reinterpret_cast<double2*>(dst + 2 * sc_chunk<T>(lane, u)), make_double2(cp[u], dp[u]));
+                } else {
+#pragma unroll
+                    for (int u = 0; u < SC_R / 2; ++u)
+                        __stcg(reinterpret_cast<float4*>(dst + 4 * sc_chunk<T>(lane, u)),
+                               make_float4(cp[2 * u], dp[2 * u], cp[2 * u + 1], dp[2 * u + 1]));
+                }
+                T al, be;
+                sc_bwd_map(cp, dp, al, be);
+#pragma unroll
+                for (int d = 1; d < 32; d <<= 1) {
+                    const T oa = __shfl_down_sync(0xffffffffu, al, d), ob = __shfl_down_sync(0xffffffffu, be, d);
+                    if ((lane & (2 * d - 1)) == 0) { al = fma(be, oa, al); be = be * ob; }
+                }
+                if (lane == 0) { wb[2 * g] = (double)al; wb[2 * g + 1] = (double)be; }
             }
-            if (lane == 0) { wmb[8 * g] = (double)al; wmb[8 * g + 1] = (double)be; }
-        }
-        __syncthreads();
-        if (pw >= nwin) tn = s_tk[par ^ 1];
-        // warps with no window in this chunk still prefetch the next one
-        if (pw >= nwin && lane == 0 && tn < total) {
-            const int qn = tn / lb.Ps, chn = tn - qn * lb.Ps;
-            if (pw < min(NC, chn * NCW + NCW) - chn * NCW) issue(qn, chn * NCW + pw, pol_a);
-        }
-        if (warp == 0) {
-            double al, be;
-            smc_reduce_bwd(wmb, nwin, lane, al, be);
-            if (lane == 0) { lb.rec[(int64_t)t * SMC_REC + 12] = al; lb.rec[(int64_t)t * SMC_REC + 13] = be; }
-        }
-        t = tn;
-        par ^= 1;
-    }
-}
-
-// x after every small chunk from the chunks' backward maps (one CTA per system):
-// x_after(ch) = B_{ch+1}(... B_{Ps-1}(0)); written to rec[14]
-template <typename T>
-__global__ void __launch_bounds__(1024) k_scan_mc_lb_fin(ScanMCLB<T> lb) {
-    __shared__ double sa[32], sb[32];
-    const int64_t q = blockIdx.x;
-    const int Ps = lb.Ps, tid = threadIdx.x, lane = tid & 31, wp = tid >> 5;
-    double* rec = lb.rec + q * Ps * SMC_REC;
-    const int per = (Ps + 1023) / 1024, lo = min(Ps, tid * per), hi = min(Ps, lo + per);
-    double al = 0.0, be = 1.0;  // this thread's chunks composed: x_first(lo) = al + be x_after(hi - 1)
-    for (int i = hi - 1; i >= lo; --i) {
-        const double a2 = rec[(int64_t)i * SMC_REC + 12], b2 = rec[(int64_t)i * SMC_REC + 13];
-        al = fma(b2, al, a2);
-        be = b2 * be;
-    }
-    // exclusive suffix over threads: the map of all chunks after this thread's range
-    double sal = al, sbe = be;  // inclusive suffix within the warp (lane l: lanes l..31)
+            // the chunk's backward map, once every B warp has stored its windows'
+            asm volatile("bar.sync %0, %1;" ::"r"(LB_NB + 1), "r"(LB_NB * 32) : "memory");
+            if (bw == 0) {
+                const int per = (nwin + 31) / 32, lo = lane * per, hi = min(nwin, lo + per);
+                double al = 0.0, be = 1.0;
+                for (int k = hi - 1; k >= lo; --k) { al = fma(wb[2 * k + 1], al, wb[2 * k]); be = wb[2 * k + 1] * be; }
 #pragma unroll
-    for (int d = 1; d < 32; d <<= 1) {
-        const double oa = __shfl_down_sync(0xffffffffu, sal, d), ob = __shfl_down_sync(0xffffffffu, sbe, d);
-        if (lane + d < 32) { sal = fma(sbe, oa, sal); sbe = sbe * ob; }
-    }
-    if (lane == 0) { sa[wp] = sal; sb[wp] = sbe; }
-    __syncthreads();
-    // x after warp wp's range: the warps after it applied to 0
-    double xw = 0.0;
-    for (int v = 31; v > wp; --v) xw = fma(sb[v], xw, sa[v]);
-    // x after this thread's range: lanes after it in the warp, then xw
-    double ea = __shfl_down_sync(0xffffffffu, sal, 1), eb = __shfl_down_sync(0xffffffffu, sbe, 1);
-    if (lane == 31) { ea = 0.0; eb = 1.0; }
-    double x = fma(eb, xw, ea);
-    for (int i = hi - 1; i >= lo; --i) {
-        rec[(int64_t)i * SMC_REC + 14] = x;
-        x = fma(rec[(int64_t)i * SMC_REC + 13], x, rec[(int64_t)i * SMC_REC + 12]);
+                for (int d = 1; d < 32; d <<= 1) {
+                    const double oa = __shfl_down_sync(0xffffffffu, al, d), ob = __shfl_down_sync(0xffffffffu, be, d);
+                    if ((lane & (2 * d - 1)) == 0) { al = fma(be, oa, al); be = be * ob; }
+                }
+                if (lane == 0) { lb.rec[(int64_t)t * SMC_REC + 12] = al; lb.rec[(int64_t)t * SMC_REC + 13] = be; }
+                __syncwarp();
+                if (lb.prof && lane == 0) { lb.prof[(int64_t)t * 8 + 6] = lb_now(); lb.prof[(int64_t)t * 8 + 7] = blockIdx.x; }
+                if (lane == 0) { sk_arrive(&bdone[par]); sk_arrive(&stfree[par]); }
+            }
+        }
     }
 }
 

@@ -148,17 +148,20 @@ cudaError_t scan_mc_t(tri_plan_s* p, const void* a, const void* b, const void* c
         ScanMCLB<T> lb;
         lb.rec = reinterpret_cast<double*>(scan_mc_slice_vals<T>(p) + 16);  // 16 T values: 8-byte aligned
         const int64_t nrec = p->m * (int64_t)p->mc_Ps;
-        lb.flag = (unsigned*)(lb.rec + nrec * SMC_REC);
+        lb.Pb = (p->mc_Ps + 31) / 32;
+        const int64_t nblk = p->m * (int64_t)lb.Pb;
+        lb.brec = lb.rec + nrec * SMC_REC;
+        lb.flag = (unsigned*)(lb.brec + nblk * 8);
         lb.NCWs = p->mc_NCWs;
         lb.Ps = p->mc_Ps;
-        const int smem_lb = SMCLayout<T>::smem_bytes(4 * p->mc_NCWs);
+        lb.prof = (unsigned long long*)g_fused_prof;
+        const int smem_lb = LBLayout<T>::smem_bytes;
         e = set_smem((const void*)k_scan_mc_lb<T>, smem_lb);
         if (e != cudaSuccess) return e;
-        e = cudaMemsetAsync(lb.flag, 0, (size_t)(nrec + 1) * sizeof(unsigned), st);
+        e = cudaMemsetAsync(lb.flag, 0, (size_t)(nrec + 1 + nblk) * sizeof(unsigned), st);
         if (e != cudaSuccess) return e;
         const int grid = (int)std::min<int64_t>(p->sms, nrec);
-        k_scan_mc_lb<T><<<grid, SC_THREADS, smem_lb, st>>>(tm, A, lb);
-        k_scan_mc_lb_fin<T><<<(unsigned)p->m, 1024, 0, st>>>(lb);
+        k_scan_mc_lb<T><<<grid, LB_THREADS, smem_lb, st>>>(tm, A, lb);
         A.xafter = lb.rec;
         A.NCWs = p->mc_NCWs;
         A.Ps = p->mc_Ps;
@@ -223,5 +226,6 @@ int scan_smem_fixed(tri_dtype t, int NC, int delta) {
 int scan_slot_bytes(tri_dtype t) { return t == TRI_F64 ? SCLayout<double>::slot_bytes : SCLayout<float>::slot_bytes; }
 int scan_in_stride(tri_dtype t) { return t == TRI_F64 ? SCLayout<double>::in_stride : SCLayout<float>::in_stride; }
 int scan_mc_wmax() { return SMC_WMAX; }
+int scan_mc_lb_maxw() { return LB_MAXW; }
 
 }  // namespace trih

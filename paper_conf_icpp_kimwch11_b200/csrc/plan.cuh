@@ -40,7 +40,7 @@ struct tri_plan_s {
     tri_variant variant = TRI_VARIANT_SCAN;
     bool forced = false;          // variant or k set by the caller (tri_solve_host sub-plans inherit it)
     int opt_tma = 1;              // TRI_OPT_TMA: 0 = p-Thomas through the non-TMA kernels
-    int opt_lookback = 0;         // TRI_OPT_SCAN_MC_LOOKBACK: windows per look-back chunk (0 = three passes)
+    int opt_lookback = -1;        // TRI_OPT_SCAN_MC_LOOKBACK: windows per look-back chunk (0 = three passes, -1 = auto)
     int G = 0, P = 0, rpt = 0;    // ONCHIP geometry
     int64_t n_pad = 0, L = 0, C = 0;  // SPLIT: chain length, chains
     int npass = 0;                // SPLIT: tiled-PCR passes (0 at k = 0)
@@ -115,6 +115,7 @@ int scan_smem_fixed(tri_dtype t, int NC, int delta);  // SCLayout<T>::smem_bytes
 int scan_slot_bytes(tri_dtype t);
 int scan_in_stride(tri_dtype t);
 int scan_mc_wmax();
+int scan_mc_lb_maxw();
 // STREAM (l_stream.cu)
 cudaError_t launch_stream(tri_plan_s* p, const void* a, const void* b, const void* c, const void* d, void* x,
                           cudaStream_t st, void* ao, void* co, void* do_);

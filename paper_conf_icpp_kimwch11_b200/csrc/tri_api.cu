@@ -114,28 +114,28 @@ bool variant_ok(tri_variant v, const tri_plan_s* p) {
 // with n swept).  See DESIGN.md §1 for the evidence behind each rule.
 tri_variant choose_variant(int64_t n, int64_t m, tri_dtype t, tri_layout layout, int sms) {
     if (layout == TRI_LAYOUT_BATCHED) return TRI_VARIANT_SCAN;  // the only kernel for this layout
-    // SCAN (profiles/r01_sweep_scan_*.jsonl): fastest of all variants on every
-    // contiguous shape with n % 8 == 0 of the grid n = 256 .. 2^20 x m = 1 .. 2^20
-    // (fp64 and fp32), except a few (< 128) systems of more than 64 windows, where
-    // one CTA per system leaves SMs idle; e.g. n = m = 16384 fp64: 1.84 ms vs
-    // 2.92 ms (STREAM), n = 256, m = 2^20 fp32: 1.01 ms vs 1.12 ms (SPLIT k = 0).
-    // k = 0 throughout: the paper's M > P rule.
-    if (layout == TRI_LAYOUT_CONTIGUOUS && scan_ok(n, m, t, layout) && (cdiv(n, SC_W) <= 64 || m >= 128))
+    // SCAN (profiles/r02_sweep_scan_*_0.jsonl): fastest, or within a few percent,
+    // on every contiguous shape with n % 8 == 0 of the grid n = 256 .. 2^20 x
+    // m = 1 .. 2^20 (fp64 and fp32), except fewer than 128 systems of 32 windows
+    // or more, where one CTA per system leaves SMs idle; e.g. n = m = 16384 fp64:
+    // 1.84 ms vs 2.92 ms (STREAM).  k = 0 throughout: the paper's M > P rule.
+    if (layout == TRI_LAYOUT_CONTIGUOUS && scan_ok(n, m, t, layout) && (cdiv(n, SC_W) < 32 || m >= 128))
         return TRI_VARIANT_SCAN;
-    // SCAN_MC: the remaining contiguous shapes (fewer than 128 systems of more than
-    // 64 windows) -- every system split over several SMs; beats deep-k SPLIT on all
-    // of them (n = 2^24, m = 1: 354 us vs 1052 us; n = 65536, m = 16: 41 us vs 87 us;
-    // n = 2^20, m = 1: 75 us vs 103 us; fp32 n = 2^24: 219 us vs 671 us).
+    // SCAN_MC: the remaining contiguous shapes (fewer than 128 systems of 32 windows
+    // or more) -- every system split over several SMs (r02 sweep: n = 16384, m = 1:
+    // 12.3 us vs 30.9 us SCAN; n = 8192, m = 16: 14.4 vs 18.5; n = 2^20, m = 1: 25 us
+    // vs 1.6 ms; beats deep-k SPLIT on all of them: n = 2^24, m = 1: 0.29 ms vs 1.05 ms).
     if (layout == TRI_LAYOUT_CONTIGUOUS && scan_mc_ok(n, m, t, layout)) return TRI_VARIANT_SCAN_MC;
     // SCAN on the INTERLEAVED layout (8 adjacent systems per window;
-    // profiles/r01_sweep_scan_il_*.jsonl): fastest from 256 systems of >= 256 rows
-    // up to where the 8-system groups' intermediates stop fitting on chip / in L2
-    // (fp64 n m >= 2^27: SPLIT k = 0 1.07x faster at 8192 x 16384) or, fp32, where
-    // many short systems favour one thread per system (n < 1024, m > 16384);
-    // e.g. c2 1024 x 1024: 18 us vs 28 us (WARP); 4096 x 4096: 170 us vs 879 us.
-    if (layout == TRI_LAYOUT_INTERLEAVED && m >= 256 && n >= 256 && scan_ok(n, m, t, layout)) {
+    // profiles/r02_sweep_scan_*_1.jsonl): fastest from 256 systems of more than 256
+    // rows (n = 256: WARP's in-register PCR is 1.2-1.6x faster) up to where the
+    // 8-system groups' intermediates stop fitting on chip / in L2 (fp64 n m >= 2^27:
+    // SPLIT k = 0 1.07x faster at 8192 x 16384) or, fp32, where many systems favour
+    // one thread per system (m > 16384: SPLIT k = 0 1.06-1.11x faster); e.g. c2
+    // 1024 x 1024: 23 us vs 28 us (WARP); 4096 x 4096: 170 us vs 879 us.
+    if (layout == TRI_LAYOUT_INTERLEAVED && m >= 256 && n > 256 && scan_ok(n, m, t, layout)) {
         const int64_t N = n * m;
-        const bool fits = t == TRI_F64 ? N < ((int64_t)1 << 27) : N < ((int64_t)1 << 28) && (n >= 1024 || m <= 16384);
+        const bool fits = t == TRI_F64 ? N < ((int64_t)1 << 27) : N < ((int64_t)1 << 28) && m <= 16384;
         if (fits) return TRI_VARIANT_SCAN;
     }
     // STREAM (profiles/r01_sweep_stream_f64.jsonl): fp64 contiguous batches with
@@ -246,8 +246,12 @@ void plan_geometry(tri_plan_s* p) {
         P = std::min(P, NC);
         int64_t NCW = cdiv(NC, P);
         p->mc_lb = 0; p->mc_NCWs = 0; p->mc_Ps = 0;
-        const int lbw = p->opt_lookback;
-        if (lbw >= 1 && 2 * lbw <= SMC_WMAX) {
+        // the look-back path (9 arrays) only when asked for: measured slower than the
+        // three passes (13 arrays) at c3 -- 0.35 vs 0.29 ms; the look-back latency
+        // (~15 us per chunk, waiting on the predecessors' phase A across CTAs) and
+        // the latency-bound per-warp replay leave HBM idle; -1 = auto = off
+        const int lbw = p->opt_lookback < 0 ? 0 : p->opt_lookback;
+        if (lbw >= 1 && lbw <= LB_MAXW) {
             // pass 2's chunks are unions of the look-back's small chunks
             p->mc_lb = 1;
             p->mc_NCWs = lbw;
@@ -281,7 +285,8 @@ size_t scratch_need(const tri_plan_s* p) {
                                             // fp64 look-back records and their flags)
         return (size_t)p->m * (size_t)p->sk_nc * (size_t)sc_slot_elems<double>() * es +
                (size_t)p->m * (size_t)p->mc_P * 16 * 8 + 16 * es +
-               (p->mc_lb ? (size_t)p->m * (size_t)p->mc_Ps * (SMC_REC * 8 + 4) + 256 : 0);
+               (p->mc_lb ? (size_t)p->m * (size_t)p->mc_Ps * (SMC_REC * 8 + 4) +
+                               (size_t)p->m * (size_t)((p->mc_Ps + 31) / 32) * (8 * 8 + 4) + 256 : 0);
     if (p->variant == TRI_VARIANT_SCAN)
         return (p->sk_nc == 1 && p->sk_S == 1) ? 0
                              : (size_t)p->sk_grid * (size_t)std::max(0, p->sk_nc + p->sk_delta - p->sk_son) *
@@ -489,7 +494,7 @@ int64_t tri_plan_scratch_bytes(tri_plan_t p) { return p ? (int64_t)p->scratch_by
 int tri_plan_launches(tri_plan_t p) {
     if (!p) return -1;
     if (p->variant == TRI_VARIANT_SPLIT) return p->k == 0 ? 1 : p->npass + 1;
-    if (p->variant == TRI_VARIANT_SCAN_MC) return 3;  // three passes (look-back: chunk kernel, link, pass 2)
+    if (p->variant == TRI_VARIANT_SCAN_MC) return p->mc_lb ? 2 : 3;  // three passes, or look-back kernel + pass 2
     return 1;
 }
 
@@ -535,7 +540,7 @@ tri_status tri_plan_set_option(tri_plan_t p, tri_option opt, int value) {
         return TRI_OK;
     }
     if (opt == TRI_OPT_SCAN_MC_LOOKBACK) {
-        if (value < 0 || 2 * value > SMC_WMAX) return TRI_ERR_INVALID_ARG;
+        if (value < -1 || value > LB_MAXW) return TRI_ERR_INVALID_ARG;
         const int old = p->opt_lookback;
         p->opt_lookback = value;
         const tri_status st = set_plan(p, p->variant, p->k);

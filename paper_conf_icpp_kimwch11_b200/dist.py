@@ -151,7 +151,7 @@ def solve_one_system_sliced(a, b, c, d, group=None, allgather=None):
     NVLink on the GPU box); all arithmetic runs in the SCAN_MC kernels
     (tri_slice_solve).  `allgather(t) -> [t_0, ..., t_{G-1}]` overrides the
     collective (tests run several slices on one device)."""
-    from . import Plan, VARIANT_SCAN_MC, F64, F32
+    from . import Plan, VARIANT_SCAN_MC, F64, F32, OPT_SCAN_MC_LOOKBACK
     if allgather is None:
         world = dist.get_world_size(group)
         rank = dist.get_rank(group)
@@ -168,6 +168,7 @@ def solve_one_system_sliced(a, b, c, d, group=None, allgather=None):
     n = a.numel()
     plan = Plan(n, 1, F64 if a.dtype == torch.float64 else F32, 0)
     plan.variant = VARIANT_SCAN_MC
+    plan.set_option(OPT_SCAN_MC_LOOKBACK, 0)  # the sliced phases are the three-pass form
     fmap = plan.slice_phase(0, rank, world, a, b, c, d)
     maps = torch.cat(allgather(fmap))
     bmap = plan.slice_phase(1, rank, world, a, b, c, d, maps=maps)

@@ -598,7 +598,7 @@ def test_scan_mc_parity(cuda_ok, dtype, n, m):
     chunks of 443 windows)."""
     arrs = gen(n, m, dtype, 0)
     x, plan = gpu_solve(n, m, arrs, dtype, 0, variant=SCAN_MC)
-    assert plan.variant == SCAN_MC and plan.k == 0 and plan.launches == 3
+    assert plan.variant == SCAN_MC and plan.k == 0 and plan.launches in (2, 3)
     check_parity(n, m, arrs, x, dtype, 0)
 
 
@@ -806,7 +806,7 @@ def test_c4_auto_plan_sampled(cuda_ok, layout):
         check_parity(n, 1, sub, xs, "f32", 0)
 
 
-@pytest.mark.parametrize("w", [24, 64])
+@pytest.mark.parametrize("w", [24, 32, 64, 0])
 def test_scan_mc_lookback_variant(cuda_ok, w):
     """SCAN_MC with passes 0 and 1 fused by a look-back over small chunks
     (k_scan_mc_lb, tri_plan_set_option(TRI_OPT_SCAN_MC_LOOKBACK, w)): parity
@@ -815,7 +815,8 @@ def test_scan_mc_lookback_variant(cuda_ok, w):
     order)."""
     import torch
     for dt, n, m in [('f64', 65536, 1), ('f64', 256 * 1000 + 8, 1), ('f32', 256 * 2100 - 16, 1),
-                     ('f64', 256 * 130, 3), ('f64', 256 * 40 * 33, 2), ('f64', 1 << 22, 1)]:
+                     ('f64', 256 * 130, 3), ('f64', 256 * 40 * 33, 2), ('f64', 1 << 22, 1), ('f64', 1 << 24, 1),
+                     ('f32', 1 << 24, 1), ('f64', (1 << 22) + 8, 5)]:
         arrs = gen(n, m, dt, 0)
         plan = tri.Plan(n, m, tri.F64 if dt == "f64" else tri.F32, 0)
         plan.variant = tri.VARIANT_SCAN_MC
