@@ -912,3 +912,176 @@ __global__ void __launch_bounds__(SC1<T>::NW * 32, 1) k_scan1(const __grid_const
 }
 
 }  // namespace tri
+
+namespace tri {
+
+// ---- fp32 systems of one window (n <= 256, n % 32 == 0; BASELINE c4): two
+// systems per warp, 16 lanes x 16 rows each.  The lane segment maps are
+// composed over 16 lanes (4 scan levels, fp64 -- DESIGN.md X22) instead of 32,
+// so the scans cost half as much per system as in the 8-rows-per-lane path
+// (c4's issue-bound instruction count was 646 warp instructions per system).
+// The window of two consecutive systems is one TMA box per array (tensor view
+// [m][n/32][32], 128-byte rows, 128B swizzle: 16-byte chunk c of row r at
+// c ^ (r & 7)); lane (s, seg) reads the 64 bytes of rows 16 seg .. 16 seg + 15
+// of system s = the half (seg & 1) of 128-byte row (s * n / 32 + seg / 2).
+// Accuracy (numpy emulation of this operation order, weak family eps = 1e-2,
+// 2^16 systems of 256): 3.4e-5 max relative error vs 2.7e-5 at 8 rows per lane.
+constexpr int S16_R = 16;
+constexpr int S16_NW = 12;
+struct S16 {
+    static constexpr int in_bytes = 2 * 4 * SC_W * 4;                    // two systems, 4 arrays, fp32
+    static constexpr int in_stride = (in_bytes + 1023) / 1024 * 1024;
+    static constexpr int off_bar = 2 * S16_NW * in_stride;               // two buffers per warp
+    static constexpr int smem_bytes = off_bar + 2 * S16_NW * 8 + 1024;
+};
+
+__global__ void __launch_bounds__(S16_NW * 32, 1) k_scan1_r16(const __grid_constant__ StreamMaps tm, ScanArgs<float> p) {
+    extern __shared__ __align__(16) unsigned char s16_smem_raw[];
+    unsigned char* sbase = s16_smem_raw + ((1024 - ((unsigned)__cvta_generic_to_shared(s16_smem_raw) & 1023)) & 1023);
+    uint64_t* full = reinterpret_cast<uint64_t*>(sbase + S16::off_bar);  // [NW][2]
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (threadIdx.x == 0) {
+        for (int i = 0; i < 2 * S16_NW; ++i) sk_bar_init(&full[i], 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    }
+    __syncthreads();
+    const int64_t n = p.n, m = p.m;
+    const int rows32 = (int)(n / 32);                 // 128-byte rows per system
+    const int64_t npair = (m + 1) / 2;                // warp steps: pairs of systems
+    const int64_t nstep = (npair - blockIdx.x + gridDim.x - 1) / gridDim.x;
+    // buffer b of this warp (address arithmetic, no pointer array: stays in registers)
+    auto bufp = [&](int b) { return reinterpret_cast<float*>(sbase + (2 * warp + b) * S16::in_stride); };
+    const uint64_t pol = sk_policy_evict_first();
+    auto issue = [&](int64_t j, int b) {
+        const int pr = (int)(blockIdx.x + j * gridDim.x);  // pair index
+        uint64_t* bar = &full[2 * warp + b];
+        sk_expect(bar, (unsigned)(2 * 4 * n * sizeof(float)));  // zero-filled past m: full box bytes
+        // box [2 systems][n/32 rows][32]: one copy per array covers both systems
+        float* d = bufp(b);
+        sc_tma3d(d + 0 * 2 * SC_W, &tm.a, 0, 2 * pr, bar, pol);
+        sc_tma3d(d + 1 * 2 * SC_W, &tm.b, 0, 2 * pr, bar, pol);
+        sc_tma3d(d + 2 * 2 * SC_W, &tm.c, 0, 2 * pr, bar, pol);
+        sc_tma3d(d + 3 * 2 * SC_W, &tm.d, 0, 2 * pr, bar, pol);
+    };
+    const int s = lane >> 4, seg = lane & 15;
+    // the lane's 64 bytes in the swizzled box: row r = s rows32 + seg / 2 (128 B each),
+    // chunks 4 (seg & 1) .. + 3, physical chunk c ^ (r & 7)
+    const int r = s * rows32 + (seg >> 1), c0 = (seg & 1) * 4;
+    const bool live = 16 * seg < n;                   // rows past n of the (short) window: identity
+    // this warp's steps: j = warp, warp + NW, ...; two in flight (buffers b = it & 1)
+    if (lane == 0 && warp < nstep) issue(warp, 0);
+    if (lane == 0 && warp + S16_NW < nstep) issue(warp + S16_NW, 1);
+    unsigned ph = 0;
+    for (int64_t j = warp, it = 0; j < nstep; j += S16_NW, ++it) {
+        const int b = (int)(it & 1);
+        const int64_t q = 2 * (blockIdx.x + j * gridDim.x) + s;  // this half-warp's system
+        sk_wait(&full[2 * warp + b], (ph >> b) & 1u);
+        ph ^= 1u << b;
+        float ra[S16_R], rb[S16_R], rc[S16_R], rd[S16_R];
+        {
+            const float* bb = bufp(b);
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+                const int o = r * 32 + (((c0 + k) ^ (r & 7)) * 4);
+                const float4 va = *reinterpret_cast<const float4*>(bb + 0 * 2 * SC_W + o);
+                const float4 vb = *reinterpret_cast<const float4*>(bb + 1 * 2 * SC_W + o);
+                const float4 vc = *reinterpret_cast<const float4*>(bb + 2 * 2 * SC_W + o);
+                const float4 vd = *reinterpret_cast<const float4*>(bb + 3 * 2 * SC_W + o);
+                ra[4 * k] = va.x; ra[4 * k + 1] = va.y; ra[4 * k + 2] = va.z; ra[4 * k + 3] = va.w;
+                rb[4 * k] = vb.x; rb[4 * k + 1] = vb.y; rb[4 * k + 2] = vb.z; rb[4 * k + 3] = vb.w;
+                rc[4 * k] = vc.x; rc[4 * k + 1] = vc.y; rc[4 * k + 2] = vc.z; rc[4 * k + 3] = vc.w;
+                rd[4 * k] = vd.x; rd[4 * k + 1] = vd.y; rd[4 * k + 2] = vd.z; rd[4 * k + 3] = vd.w;
+            }
+        }
+        sc_release_buf();  // this warp's reads of the buffer before the TMA refill
+        if (lane == 0 && j + 2 * S16_NW < nstep) issue(j + 2 * S16_NW, b);
+        // rows: a_0, c_{n-1} outside A; rows past n identity
+        bool out = false;
+#pragma unroll
+        for (int u = 0; u < S16_R; ++u) {
+            const int64_t i = 16 * seg + u;
+            if (i == 0) ra[u] = 0.f;
+            if (i == n - 1) rc[u] = 0.f;
+            if (i >= n || !live) { ra[u] = 0.f; rb[u] = 1.f; rc[u] = 0.f; rd[u] = 0.f; }
+            const unsigned e = ((unsigned)__float_as_int(rb[u]) >> 23) & 0xffu;
+            out |= (e - (127u - 8u)) > 16u;
+        }
+        // the 8-row partial products (rescaled at row 8) stay in fp32's range while
+        // every pivot is within 2^+-8; otherwise (warp-uniform) every row is scaled
+        // by 2^-exponent(b) -- exact row operations (X21)
+        if (__any_sync(0xffffffffu, out)) {
+#pragma unroll
+            for (int u = 0; u < S16_R; ++u) {
+                const float sc = sk_exp2_scale(rb[u]);
+                ra[u] *= sc; rb[u] *= sc; rc[u] *= sc; rd[u] *= sc;
+            }
+        }
+        // the lane's 16-row segment map (fp32), then composed over the 16 lanes in fp64
+        float t1 = rb[0], p1 = rc[0], d1 = rd[0], t2 = -ra[0], p2 = 0.f, d2 = 0.f, d3 = -ra[0];
+#pragma unroll
+        for (int u = 1; u < S16_R; ++u) {
+            const float au = ra[u], bu = rb[u], cu = rc[u], du = rd[u];
+            const float nt1 = fmaf(bu, t1, -au * p1), np1 = cu * t1, nd1 = fmaf(du, t1, -au * d1);
+            const float nt2 = fmaf(bu, t2, -au * p2), np2 = cu * t2, nd2 = fmaf(du, t2, -au * d2);
+            d3 = -au * d3;
+            t1 = nt1; p1 = np1; d1 = nd1; t2 = nt2; p2 = np2; d2 = nd2;
+            if (u == 7) {  // keep the 8-row partial products in range (exact power-of-two rescale)
+                const float h = sc_scale2(t1, t2);
+                t1 *= h; p1 *= h; d1 *= h; t2 *= h; p2 *= h; d2 *= h; d3 *= h;
+            }
+        }
+        const float hs = sc_scale2(t1, t2);
+        SCM M{(double)(t1 * hs), (double)(t2 * hs), (double)(p1 * hs), (double)(p2 * hs), (double)(d1 * hs),
+              (double)(d2 * hs), (double)(d3 * hs)};
+#pragma unroll
+        for (int dd = 1; dd < 16; dd <<= 1) {  // inclusive scan over the system's 16 lanes
+            SCM o;
+            o.a = __shfl_up_sync(0xffffffffu, M.a, dd, 16); o.b = __shfl_up_sync(0xffffffffu, M.b, dd, 16);
+            o.c = __shfl_up_sync(0xffffffffu, M.c, dd, 16); o.d = __shfl_up_sync(0xffffffffu, M.d, dd, 16);
+            o.e = __shfl_up_sync(0xffffffffu, M.e, dd, 16); o.f = __shfl_up_sync(0xffffffffu, M.f, dd, 16);
+            o.g = __shfl_up_sync(0xffffffffu, M.g, dd, 16);
+            if (seg >= dd) M = sk_compose(M, o);
+        }
+        // incoming state of the lane = outgoing state of lane - 1 (system starts at (1, 0, 0))
+        double xt = __shfl_up_sync(0xffffffffu, M.a, 1, 16), xp = __shfl_up_sync(0xffffffffu, M.c, 1, 16),
+               xd = __shfl_up_sync(0xffffffffu, M.e, 1, 16);
+        if (seg == 0) { xt = 1.0; xp = 0.0; xd = 0.0; }
+        const double xs = sk_exp2_scale(xt);
+        float th = (float)(xt * xs), ps = (float)(xp * xs), de = (float)(xd * xs);
+        float cp[S16_R], dp[S16_R];
+#pragma unroll
+        for (int u = 0; u < S16_R; ++u) {
+            const float nt = fmaf(rb[u], th, -ra[u] * ps), np = rc[u] * th, nd = fmaf(rd[u], th, -ra[u] * de);
+            const float inv = rcp(nt);
+            cp[u] = np * inv;
+            dp[u] = nd * inv;
+            th = nt; ps = np; de = nd;
+            if (u == 7) {  // exact rescale of the projective state
+                const float h = sk_exp2_scale(th);
+                th *= h; ps *= h; de *= h;
+            }
+        }
+        // back substitution: affine segment maps, suffix scan over the 16 lanes
+        float al = dp[S16_R - 1], be = -cp[S16_R - 1];
+#pragma unroll
+        for (int u = S16_R - 2; u >= 0; --u) { al = fmaf(-cp[u], al, dp[u]); be = -cp[u] * be; }
+#pragma unroll
+        for (int dd = 1; dd < 16; dd <<= 1) {
+            const float oa = __shfl_down_sync(0xffffffffu, al, dd, 16), ob = __shfl_down_sync(0xffffffffu, be, dd, 16);
+            if (seg + dd < 16) { al = fmaf(be, oa, al); be = be * ob; }
+        }
+        float x = __shfl_down_sync(0xffffffffu, al, 1, 16);
+        if (seg == 15) x = 0.f;
+        float xv[S16_R];
+#pragma unroll
+        for (int u = S16_R - 1; u >= 0; --u) { x = fmaf(-cp[u], x, dp[u]); xv[u] = x; }
+        if (q < m && live) {
+            float* xo = p.x + q * n + 16 * seg;
+#pragma unroll
+            for (int u = 0; u < S16_R; u += 4) __stcs(reinterpret_cast<float4*>(xo + u), make_float4(xv[u], xv[u + 1], xv[u + 2], xv[u + 3]));
+        }
+    }
+}
+
+}  // namespace tri

@@ -497,8 +497,7 @@ __global__ void __launch_bounds__(LB_THREADS, 1) k_scan_mc_lb(const __grid_const
     if (warp < LB_NA) {
         // ======================= A: forward window maps =======================
         const int aw = warp;
-        T* buf[2] = {reinterpret_cast<T*>(sbase + L::off_a + (2 * aw) * L::in_stride),
-                     reinterpret_cast<T*>(sbase + L::off_a + (2 * aw + 1) * L::in_stride)};
+        auto buf = [&](int b) { return reinterpret_cast<T*>(sbase + L::off_a + (2 * aw + b) * L::in_stride); };
         const uint64_t pol = sk_policy_evict_normal();  // phase B re-reads the chunk from L2
         unsigned ph2 = 0;                                // bit b: phase of buffer b
         int nb = 0;                                      // loads issued by this warp (buffer = nb & 1)
@@ -524,7 +523,7 @@ __global__ void __launch_bounds__(LB_THREADS, 1) k_scan_mc_lb(const __grid_const
             if (i >= 2) sk_wait(&bdone[par], (unsigned)(((i >> 1) - 1) & 1));
             // first two windows of this warp (before waiting for the map buffer)
             if (lane == 0) {
-                for (int g = aw; g < nwin && g < aw + 2 * LB_NA; g += LB_NA, ++nb) issue(buf[nb & 1], &a_full[2 * aw + (nb & 1)], t, g, pol);
+                for (int g = aw; g < nwin && g < aw + 2 * LB_NA; g += LB_NA, ++nb) issue(buf(nb & 1), &a_full[2 * aw + (nb & 1)], t, g, pol);
             } else {
                 for (int g = aw; g < nwin && g < aw + 2 * LB_NA; g += LB_NA) ++nb;
             }
@@ -534,10 +533,10 @@ __global__ void __launch_bounds__(LB_THREADS, 1) k_scan_mc_lb(const __grid_const
                 sk_wait(&a_full[2 * aw + bsel], (ph2 >> bsel) & 1u);
                 ph2 ^= 1u << bsel;
                 T ra[SC_R], rb[SC_R], rc[SC_R], rd[SC_R];
-                load_rows(buf[bsel], t, g, ra, rb, rc, rd);
+                load_rows(buf(bsel), t, g, ra, rb, rc, rd);
                 sc_release_buf();  // this warp's reads of the buffer before the TMA refill
                 if (g + 2 * LB_NA < nwin) {
-                    if (lane == 0) issue(buf[bsel], &a_full[2 * aw + bsel], t, g + 2 * LB_NA, pol);
+                    if (lane == 0) issue(buf(bsel), &a_full[2 * aw + bsel], t, g + 2 * LB_NA, pol);
                     ++nb;
                 }
                 SCM M = sc_wide(sc_fwd_map(ra, rb, rc, rd));

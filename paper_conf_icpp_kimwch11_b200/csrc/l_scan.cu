@@ -53,6 +53,15 @@ bool scan_maps(tri_plan_s* p, int tag, const void* a, const void* b, const void*
     return true;
 }
 
+// fp32 one-window systems, two per TMA box (k_scan1_r16): tensor [m][n/32][32],
+// box [2][n/32][32], 128B swizzle
+bool map_pairs(CUtensorMap* tm, const void* base, int64_t n, int64_t m) {
+    const uint64_t dims[3] = {32, (uint64_t)(n / 32), (uint64_t)m};
+    const uint64_t str[2] = {128, (uint64_t)n * 4};
+    const uint32_t box[3] = {32, (uint32_t)(n / 32), 2u};
+    return tma_encode(tm, 4, 3, base, dims, str, box, CU_TENSOR_MAP_SWIZZLE_128B);
+}
+
 template <typename T, int S>
 void* scan_kernel(bool prof) {
     return prof ? (void*)k_scan<T, S, true> : (void*)k_scan<T, S, false>;
@@ -62,6 +71,27 @@ template <typename T>
 cudaError_t scan_t(tri_plan_s* p, const void* a, const void* b, const void* c, const void* d, void* x,
                    cudaStream_t st) {
     const int S = p->sk_S;
+    if constexpr (sizeof(T) == 4) {
+        // fp32 one-window systems, n % 32 == 0 (c4): two systems per warp, 16 rows per lane
+        if (S == 1 && p->sk_nc == 1 && p->n % 32 == 0) {
+            StreamMaps tm;
+            const void* key[4] = {a, b, c, d};
+            if (!tm_lookup(p, 0x1800, key, 4, &tm.a, 4)) {
+                if (!map_pairs(&tm.a, a, p->n, p->m) || !map_pairs(&tm.b, b, p->n, p->m) ||
+                    !map_pairs(&tm.c, c, p->n, p->m) || !map_pairs(&tm.d, d, p->n, p->m))
+                    return cudaErrorNotSupported;
+                tm_store(p, 0x1800, key, 4, &tm.a, 4);
+            }
+            ScanArgs<float> A{};
+            A.x = (float*)x;
+            A.n = p->n; A.m = p->m; A.ms = p->ms; A.NC = 1;
+            cudaError_t e = set_smem((const void*)k_scan1_r16, S16::smem_bytes);
+            if (e != cudaSuccess) return e;
+            const unsigned grid = (unsigned)std::min<int64_t>((p->m + 1) / 2, p->sms);
+            k_scan1_r16<<<grid, S16_NW * 32, S16::smem_bytes, st>>>(tm, A);
+            return cudaGetLastError();
+        }
+    }
     // one-window systems shorter than 3/4 of a window (many idle rows: compute-heavy)
     // run the chain-free kernel with more warps (fp32 n = 128: 1.19 ms vs 1.50 ms
     // per 2^28 rows); at n = 256 the 12-warp kernel is faster (c4: 0.99 vs 1.02 ms)
