@@ -51,9 +51,12 @@ typedef enum { TRI_F32 = 0, TRI_F64 = 1 } tri_dtype;
 typedef enum {
     TRI_LAYOUT_CONTIGUOUS = 0,  /* element i of system q at [q*n + i] */
     TRI_LAYOUT_INTERLEAVED = 1, /* element i of system q at [i*m + q] */
-    TRI_LAYOUT_BATCHED = 2      /* nb batches of ms interleaved systems (only through tri_plan_batched):
+    TRI_LAYOUT_BATCHED = 2,     /* nb batches of ms interleaved systems (only through tri_plan_batched):
                                    element i of system q = b*ms + s at [(b*n + i)*ms + s]; e.g. the
                                    y-lines of a row-major grid [nb][n][ms] (ADI) */
+    TRI_LAYOUT_STRIDED = 3      /* caller's strides (only through tri_plan_strided): element i of system
+                                   q = b*ms + s at [i*es + s*ss + b*bs] (elements); lines of pitched and
+                                   sub-grid views of 3D arrays along any axis */
 } tri_layout;
 
 typedef enum {
@@ -159,6 +162,30 @@ TRI_API tri_status tri_plan_autotune(tri_plan_t plan, const void* a, const void*
  * 131072 (4096 windows of 32 rows); else NULL with TRI_ERR_INVALID_ARG.  The
  * solve semantics, pointer rules and ownership are those of tri_solve. */
 TRI_API tri_plan_t tri_plan_batched(int64_t n, int64_t ms, int64_t nb, tri_dtype dtype);
+
+/* Plan for arbitrary element / system / batch strides (ADI
+ * line solves on pitched and sub-grid views of a 3D array).  m = ms * nb
+ * systems of size n; element i of system q = b*ms + s (0 <= s < ms, 0 <= b < nb)
+ * is at element offset i*es + s*ss + b*bs from each array's base pointer (a, b,
+ * c, d and x alike; the base may point into a larger array).  All strides >= 1
+ * and the caller guarantees distinct elements (no two (q, i) at one offset).
+ * For lines of a row-major array [nz][ny][nx] with row pitch py and plane pitch
+ * pz (elements): x-lines (n, ms, nb, es, ss, bs) = (nx, ny, nz, 1, py, pz);
+ * y-lines (ny, nx, nz, py, 1, pz); z-lines (nz, nx, ny, pz, 1, py).
+ * Runs the SCAN kernel (k = 0) directly on the caller's arrays when a TMA
+ * tensor map can describe them -- es == 1 (n % 8 == 0) or ss == 1 (ms > 1), the
+ * other strides 16-byte multiples; otherwise (odd pitches) a gather kernel packs
+ * a, b, c, d into plan-owned dense arrays, an inner plan solves them and x is
+ * scattered back (2 extra passes over the data); a TMA-path plan switches to the
+ * packed path at the first solve whose view origins are not 16-byte aligned.
+ * Pointers: element-aligned device pointers; x must not overlap the inputs'
+ * footprint (TRI_ERR_ALIAS).
+ * tri_solve_host, tri_debug_pcr and tri_plan_autotune return
+ * TRI_ERR_INVALID_ARG for these plans; tri_plan_set_k runs k = 0 on the TMA path
+ * and any k on the packed one.  NULL with TRI_ERR_INVALID_ARG for bad sizes or
+ * strides < 1. */
+TRI_API tri_plan_t tri_plan_strided(int64_t n, int64_t ms, int64_t nb, tri_dtype dtype, int64_t es, int64_t ss,
+                                    int64_t bs);
 
 /* One system spread over several devices.
  * Device r holds rows [r0, r0 + n) of the system -- a contiguous slice, n % 8

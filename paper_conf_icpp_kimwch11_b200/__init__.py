@@ -14,7 +14,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.environ.get("TRI_LIB_PATH", os.path.join(HERE, "libtri.so"))  # override: experiments only
 
 F32, F64 = 0, 1
-CONTIGUOUS, INTERLEAVED, BATCHED = 0, 1, 2
+CONTIGUOUS, INTERLEAVED, BATCHED, STRIDED = 0, 1, 2, 3
 (VARIANT_AUTO, VARIANT_ONCHIP, VARIANT_SPLIT, VARIANT_FUSED, VARIANT_WARP, VARIANT_STREAM, VARIANT_SCAN,
  VARIANT_SCAN_MC) = 0, 1, 2, 3, 4, 5, 6, 7
 VARIANT_NAMES = {1: "onchip", 2: "split", 3: "fused", 4: "warp", 5: "stream", 6: "scan", 7: "scan_mc"}
@@ -46,6 +46,7 @@ def lib():
         sig = {
             "tri_plan": (_P, [_I64, _I64, _I, _I]),
             "tri_plan_batched": (_P, [_I64, _I64, _I64, _I]),
+            "tri_plan_strided": (_P, [_I64, _I64, _I64, _I, _I64, _I64, _I64]),
             "tri_last_status": (_I, []),
             "tri_solve": (_I, [_P] * 7),
             "tri_solve_host": (_I, [_P] * 7),
@@ -117,13 +118,17 @@ class Plan:
     Wraps tri_plan / tri_solve (include/tri.h).  The plan is bound to the CUDA
     device current at construction and owns its scratch."""
 
-    def __init__(self, n, m, dtype=F64, layout=CONTIGUOUS, _batch=None):
+    def __init__(self, n, m, dtype=F64, layout=CONTIGUOUS, _batch=None, _strides=None):
         import torch
         self.n, self.m = int(n), int(m)
         self.dtype_code = _dtype_code(dtype)
         self.torch_dtype = torch.float64 if self.dtype_code == F64 else torch.float32
         self.layout = int(layout)
-        if _batch is None:
+        self.strides = _strides
+        if _strides is not None:
+            ms, nb, es, ss, bs = _strides
+            h = lib().tri_plan_strided(self.n, ms, nb, self.dtype_code, es, ss, bs)
+        elif _batch is None:
             h = lib().tri_plan(self.n, self.m, self.dtype_code, self.layout)
         else:
             h = lib().tri_plan_batched(self.n, _batch[0], _batch[1], self.dtype_code)
@@ -137,6 +142,23 @@ class Plan:
         """tri_plan_batched: nb batches of ms interleaved systems of size n (the
         y-lines of a row-major grid [nb][n][ms]; ADI)."""
         return cls(n, int(ms) * int(nb), dtype, BATCHED, _batch=(int(ms), int(nb)))
+
+    @classmethod
+    def strided(cls, n, ms, nb, es, ss, bs, dtype=F64):
+        """tri_plan_strided: m = ms*nb systems of size n, element i of system
+        q = b*ms + s at offset i*es + s*ss + b*bs of every array (lines of pitched /
+        sub-grid views of a 3D array along any axis).  Solve
+        with tensors whose data_ptr() is the view's origin (e.g. a sliced view
+        of the parent array)."""
+        strides = tuple(int(v) for v in (ms, nb, es, ss, bs))
+        return cls(n, strides[0] * strides[1], dtype, STRIDED, _strides=strides)
+
+    def footprint(self):
+        """Elements from an array's base to its last element + 1."""
+        if self.strides is None:
+            return self.n * self.m
+        ms, nb, es, ss, bs = self.strides
+        return (self.n - 1) * es + (ms - 1) * ss + (nb - 1) * bs + 1
 
     def __del__(self):
         h = getattr(self, "_h", None)
@@ -185,6 +207,14 @@ class Plan:
         return buf.value.decode()
 
     def _check(self, *ts):
+        if self.strides is not None:  # views into larger arrays: the storage must hold the footprint
+            need = self.footprint()
+            for t in ts:
+                avail = t.untyped_storage().nbytes() // t.element_size() - t.storage_offset()
+                if not t.is_cuda or t.dtype != self.torch_dtype or avail < need:
+                    raise ValueError(f"expected a CUDA {self.torch_dtype} view with >= {need} elements of storage "
+                                     f"from its origin, got {t.dtype} on {t.device} ({avail} elements)")
+            return
         for t in ts:
             if not t.is_cuda or t.dtype != self.torch_dtype or t.numel() != self.n * self.m \
                     or not t.is_contiguous():
@@ -194,6 +224,8 @@ class Plan:
     def solve(self, a, b, c, d, out=None, stream=None):
         import torch
         if out is None:
+            if self.strides is not None:
+                raise ValueError("strided plans need out= (a view with the plan's strides)")
             out = torch.empty_like(b)
         self._check(a, b, c, d, out)
         s = stream if stream is not None else torch.cuda.current_stream()

@@ -15,7 +15,8 @@ CSRC = os.path.join(HERE, "csrc")
 INCLUDE = os.path.join(ROOT, "include")
 LIB = os.path.join(HERE, "libtri.so")
 OBJ = os.path.join(HERE, "build_obj")
-SOURCES = ["tri_api.cu", "host_util.cu", "l_scan.cu", "l_split.cu", "l_stream.cu", "l_fused.cu", "l_small.cu"]
+SOURCES = ["tri_api.cu", "host_util.cu", "l_scan.cu", "l_split.cu", "l_stream.cu", "l_fused.cu", "l_small.cu",
+           "l_strided.cu"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-fvisibility=hidden",

@@ -77,7 +77,13 @@ struct ScanArgs {
     T* x;
     T* spill;      // per CTA: (NC + delta - S_on) slots of sc_slot_elems<T>() elements
     int64_t n, m;
-    int64_t ms;    // S > 1 (INTERLEAVED / BATCHED): systems per batch (INTERLEAVED: m, one batch)
+    int64_t ms;    // systems per batch (CONTIGUOUS / INTERLEAVED: m, one batch)
+    // x addressing (elements; the inputs use the same strides through the tensor maps):
+    // S == 1: system s of batch b starts at s xsys + b xbat, rows consecutive;
+    // S > 1: row i of system s of batch b at b xbat + i xel + s
+    int64_t xsys, xbat, xel;
+    int nb;        // batches (1: no division of the system index)
+    int x32;       // fp64, S == 1: every system's x row is 32-byte aligned (256-bit stores)
     int w128;      // CONTIGUOUS: tensor view [m][n/r][r] with 128-byte rows (r = 32 fp32 / 16 fp64), 128B swizzle
     int NC;        // windows per system
     int delta;     // extra lag (steps) of the back substitution behind the forward sweep
@@ -118,6 +124,17 @@ struct SCLayout {
 template <typename T>
 __device__ __forceinline__ int sc_chunk(int lane, int ch) {
     return ch * 32 + lane;
+}
+
+// TMA 4D tile load: CONTIGUOUS (and STRIDED with unit element stride) tensor view
+// [nb][ms][n/r][r] (batch, system, row group, row), box [1][1][256/r][r].
+__device__ __forceinline__ void sc_tma4d(void* dst, const CUtensorMap* tm, int y, int s, int b, uint64_t* bar,
+                                         uint64_t pol) {
+    asm volatile(
+        "cp.async.bulk.tensor.4d.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint"
+        " [%0], [%1, {%2, %3, %4, %5}], [%6], %7;" ::"r"((unsigned)__cvta_generic_to_shared(dst)),
+        "l"(tm), "r"(0), "r"(y), "r"(s), "r"(b), "r"((unsigned)__cvta_generic_to_shared(bar)), "l"(pol)
+        : "memory");
 }
 
 // TMA 3D tile load.  CONTIGUOUS: tensor view [m][n/8][8] (system, 8-row group,
@@ -501,14 +518,19 @@ __device__ __forceinline__ void sc_load_slot_g(const T* base, int lane, T (&cp)[
 
 // x of the lane's rows (first row global index xi) -> global, streaming stores
 template <typename T>
-__device__ __forceinline__ void sc_store_x(T* xo, int64_t rmax, const T (&xv)[SC_R]) {
+__device__ __forceinline__ void sc_store_x(T* xo, int64_t rmax, const T (&xv)[SC_R], bool x32 = true) {
     if (rmax >= SC_R) {
         if constexpr (sizeof(T) == 8) {
+            if (x32) {  // 32-byte stores (one warp store = 512 contiguous bytes) need 32-byte aligned rows
 #pragma unroll
-            for (int t = 0; t < SC_R; t += 4)
-                asm volatile(SC_XST ".v4.f64 [%0], {%1, %2, %3, %4};" ::"l"(xo + t), "d"(xv[t]), "d"(xv[t + 1]),
-                             "d"(xv[t + 2]), "d"(xv[t + 3])
-                             : "memory");
+                for (int t = 0; t < SC_R; t += 4)
+                    asm volatile(SC_XST ".v4.f64 [%0], {%1, %2, %3, %4};" ::"l"(xo + t), "d"(xv[t]), "d"(xv[t + 1]),
+                                 "d"(xv[t + 2]), "d"(xv[t + 3])
+                                 : "memory");
+            } else {
+#pragma unroll
+                for (int t = 0; t < SC_R; t += 2) __stcs(reinterpret_cast<double2*>(xo + t), make_double2(xv[t], xv[t + 1]));
+            }
         } else {
 #pragma unroll
             for (int t = 0; t < SC_R; t += 4)
@@ -568,10 +590,18 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
         sk_expect(bar, (unsigned)(4 * SC_W * sizeof(T)));
         if constexpr (S == 1) {
             const int y = ww * (p.w128 ? SC_W * (int)sizeof(T) / 128 : SC_W / 8);
-            sc_tma3d(buf + 0 * SC_W, &tm.a, y, q, bar, pol_in);
-            sc_tma3d(buf + 1 * SC_W, &tm.b, y, q, bar, pol_in);
-            sc_tma3d(buf + 2 * SC_W, &tm.c, y, q, bar, pol_in);
-            sc_tma3d(buf + 3 * SC_W, &tm.d, y, q, bar, pol_in);
+            if (p.nb == 1) {  // one batch: 3D view [ms][n/r][r]
+                sc_tma3d(buf + 0 * SC_W, &tm.a, y, q, bar, pol_in);
+                sc_tma3d(buf + 1 * SC_W, &tm.b, y, q, bar, pol_in);
+                sc_tma3d(buf + 2 * SC_W, &tm.c, y, q, bar, pol_in);
+                sc_tma3d(buf + 3 * SC_W, &tm.d, y, q, bar, pol_in);
+            } else {          // STRIDED batches: 4D view [nb][ms][n/r][r]
+                const int bt = q / (int)p.ms, sq = q - bt * (int)p.ms;  // q < 2^31 (planner)
+                sc_tma4d(buf + 0 * SC_W, &tm.a, y, sq, bt, bar, pol_in);
+                sc_tma4d(buf + 1 * SC_W, &tm.b, y, sq, bt, bar, pol_in);
+                sc_tma4d(buf + 2 * SC_W, &tm.c, y, sq, bt, bar, pol_in);
+                sc_tma4d(buf + 3 * SC_W, &tm.d, y, sq, bt, bar, pol_in);
+            }
         } else {  // tensor [nb][n][ms], box [1][WR][S]
             const int bt = (int)(q / gpb), xq = (int)(q - bt * gpb) * S, y = ww * WR;
             sc_tma3d(buf + 0 * SC_W, &tm.a, y, bt, bar, pol_in, xq);
@@ -581,6 +611,12 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
         }
     };
     auto issue = [&](int jj, int ww) { issue_to(jj, ww, ib, &in_full[pw]); };
+    // S == 1: first element of system q (batch q / ms, system q % ms)
+    auto xbase = [&](int64_t q) {
+        if (p.nb == 1) return p.x + q * p.xsys;
+        const int bt = (int)q / (int)p.ms;  // q < 2^31 (planner)
+        return p.x + (q - (int64_t)bt * p.ms) * p.xsys + bt * p.xbat;
+    };
     unsigned ph = 0;
 
     if (S == 1 && NC == 1) {
@@ -607,7 +643,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
                 T xz[SC_R];
 #pragma unroll
                 for (int t = 0; t < SC_R; ++t) xz[t] = ra[t] * T(0);
-                sc_store_x(p.x + q * n + lane * SC_R, n - (int64_t)lane * SC_R, xz);
+                sc_store_x(xbase(q) + lane * SC_R, n - (int64_t)lane * SC_R, xz, p.x32 != 0);
                 if (DB < 0 && lane == 0 && j + SC_NW < nsys) issue_to(j + SC_NW, 0, bufs[0], bars[0]);
                 continue;
             }
@@ -633,7 +669,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
                 x = fma(-cp[t], x, dp[t]);
                 xv[t] = x;
             }
-            sc_store_x(p.x + q * n + lane * SC_R, n - (int64_t)lane * SC_R, xv);
+            sc_store_x(xbase(q) + lane * SC_R, n - (int64_t)lane * SC_R, xv, p.x32 != 0);
             if (DB < 0 && lane == 0 && j + SC_NW < nsys) issue_to(j + SC_NW, 0, bufs[0], bars[0]);
         }
         return;
@@ -695,7 +731,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
                 for (int t = 0; t < SC_R; ++t) xv[t] = T(0);
                 if constexpr (S == 1) {
                     const int64_t q = blockIdx.x + (int64_t)cj * gridDim.x;
-                    sc_store_x(p.x + q * n + i0d, n - i0d, xv);
+                    sc_store_x(xbase(q) + i0d, n - i0d, xv, p.x32 != 0);
                 }
             }
             continue;
@@ -811,14 +847,14 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
             const int64_t qb = blockIdx.x + (int64_t)bj * gridDim.x;
             const int64_t xr = (int64_t)wb * WR + seg * SC_R;
             if constexpr (S == 1) {
-                sc_store_x(p.x + qb * n + xr, n - xr, xv);
+                sc_store_x(xbase(qb) + xr, n - xr, xv, p.x32 != 0);
             } else {  // INTERLEAVED / BATCHED: x[(batch n + row) ms + s]
                 const int64_t bt = qb / gpb, qx = (qb - bt * gpb) * S + ls;
                 if (qx < p.ms) {
-                    T* xo = p.x + bt * n * p.ms + qx;
+                    T* xo = p.x + bt * p.xbat + qx;
 #pragma unroll
                     for (int t = 0; t < SC_R; ++t)
-                        if (xr + t < n) __stcs(xo + (xr + t) * p.ms, xv[t]);
+                        if (xr + t < n) __stcs(xo + (xr + t) * p.xel, xv[t]);
                 }
             }
         }
@@ -906,7 +942,7 @@ __global__ void __launch_bounds__(SC1<T>::NW * 32, 1) k_scan1(const __grid_const
             x = fma(-cp[t], x, dp[t]);
             xv[t] = x;
         }
-        sc_store_x(p.x + q * n + lane * SC_R, n - (int64_t)lane * SC_R, xv);
+        sc_store_x(p.x + q * n + lane * SC_R, n - (int64_t)lane * SC_R, xv, p.x32 != 0);
         if (late && lane == 0 && j + NW < nsys) issue(j + NW);
     }
 }
@@ -935,7 +971,8 @@ struct S16 {
     static constexpr int smem_bytes = off_bar + 2 * S16_NW * 8 + 1024;
 };
 
-__global__ void __launch_bounds__(S16_NW * 32, 1) k_scan1_r16(const __grid_constant__ StreamMaps tm, ScanArgs<float> p) {
+template <typename T = float>  // fp32 only (a template: defined once across the translation units)
+__global__ void __launch_bounds__(S16_NW * 32, 1) k_scan1_r16(const __grid_constant__ StreamMaps tm, ScanArgs<T> p) {
     extern __shared__ __align__(16) unsigned char s16_smem_raw[];
     unsigned char* sbase = s16_smem_raw + ((1024 - ((unsigned)__cvta_generic_to_shared(s16_smem_raw) & 1023)) & 1023);
     uint64_t* full = reinterpret_cast<uint64_t*>(sbase + S16::off_bar);  // [NW][2]

@@ -43,6 +43,7 @@ struct ScanMCArgs {
     // (null: 0, the system's end)
     int keep_a0, keep_cn;
     int w128;     // tensor view with 128-byte rows (k_scan.cuh)
+    int x32;      // fp64: x rows 32-byte aligned (256-bit stores)
     const T* s0;
     const T* xe;
     // look-back path (k_scan_mc_lb): small-chunk records (x after each at [14]);
@@ -306,7 +307,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant
                 x = fma(-cp[t], x, dp[t]);
                 xv[t] = x;
             }
-            sc_store_x(p.x + q * n + i0, n - i0, xv);
+            sc_store_x(p.x + q * n + i0, n - i0, xv, p.x32 != 0);
         }
     }
     if (MODE == 2) return;

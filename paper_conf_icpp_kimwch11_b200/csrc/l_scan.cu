@@ -26,12 +26,37 @@ bool map_sys_rows(CUtensorMap* tm, const void* base, int64_t n, int64_t m, bool 
     return tma_encode(tm, sizeof(T), 3, base, dims, str, box, swz);
 }
 
-// INTERLEAVED / BATCHED: tensor [nb][n][ms] (row stride ms elements, batch stride
-// n ms), box [1][256 / S rows][S systems]
+// SCAN, unit element stride (CONTIGUOUS, STRIDED x-lines): tensor view
+// [nb][ms][n/r][r] with the plan's system / batch strides, box [1][1][256/r][r]
 template <typename T>
-bool map_il(CUtensorMap* tm, const void* base, int64_t n, int64_t ms, int64_t nb, int S) {
+bool map_sys_rows4(CUtensorMap* tm, const void* base, const tri_plan_s* p, bool w128) {
+    const int rw = w128 ? 128 / (int)sizeof(T) : 8;
+    const uint64_t dims[4] = {(uint64_t)rw, (uint64_t)(p->n / rw), (uint64_t)p->ms, (uint64_t)p->nb};
+    const uint64_t str[3] = {(uint64_t)rw * sizeof(T), (uint64_t)p->ss * sizeof(T), (uint64_t)p->bs * sizeof(T)};
+    const uint32_t box[4] = {(uint32_t)rw, (uint32_t)(SC_W / rw), 1u, 1u};
+    const CUtensorMapSwizzle swz =
+        w128 ? CU_TENSOR_MAP_SWIZZLE_128B : sizeof(T) == 8 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_32B;
+    return tma_encode(tm, sizeof(T), 4, base, dims, str, box, swz);
+}
+
+// ... one batch: 3D view [ms][n/r][r] with the plan's system stride
+template <typename T>
+bool map_sys_rows3(CUtensorMap* tm, const void* base, const tri_plan_s* p, bool w128) {
+    const int rw = w128 ? 128 / (int)sizeof(T) : 8;
+    const uint64_t dims[3] = {(uint64_t)rw, (uint64_t)(p->n / rw), (uint64_t)p->ms};
+    const uint64_t str[2] = {(uint64_t)rw * sizeof(T), (uint64_t)p->ss * sizeof(T)};
+    const uint32_t box[3] = {(uint32_t)rw, (uint32_t)(SC_W / rw), 1u};
+    const CUtensorMapSwizzle swz =
+        w128 ? CU_TENSOR_MAP_SWIZZLE_128B : sizeof(T) == 8 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_32B;
+    return tma_encode(tm, sizeof(T), 3, base, dims, str, box, swz);
+}
+
+// SCAN, unit system stride (INTERLEAVED / BATCHED / STRIDED y- and z-lines):
+// tensor [nb][n][ms] (row stride es, batch stride bs elements), box [1][256 / S rows][S systems]
+template <typename T>
+bool map_il(CUtensorMap* tm, const void* base, int64_t n, int64_t ms, int64_t nb, int S, int64_t es, int64_t bs) {
     const uint64_t dims[3] = {(uint64_t)ms, (uint64_t)n, (uint64_t)nb};
-    const uint64_t str[2] = {(uint64_t)ms * sizeof(T), (uint64_t)(n * ms) * sizeof(T)};
+    const uint64_t str[2] = {(uint64_t)es * sizeof(T), (uint64_t)bs * sizeof(T)};
     const uint32_t box[3] = {(uint32_t)S, (uint32_t)(SC_W / S), 1u};
     return tma_encode(tm, sizeof(T), 3, base, dims, str, box, CU_TENSOR_MAP_SWIZZLE_NONE);
 }
@@ -44,9 +69,10 @@ bool scan_maps(tri_plan_s* p, int tag, const void* a, const void* b, const void*
     const void* src[4] = {a, b, c, d};
     CUtensorMap* dst[4] = {&tm.a, &tm.b, &tm.c, &tm.d};
     for (int i = 0; i < 4; ++i) {
-        const bool ok = p->sk_S == 1 || p->variant == TRI_VARIANT_SCAN_MC
-                            ? map_sys_rows<T>(dst[i], src[i], p->n, p->m, w128)
-                            : map_il<T>(dst[i], src[i], p->n, p->ms, p->m / p->ms, p->sk_S);
+        const bool ok = p->variant == TRI_VARIANT_SCAN_MC ? map_sys_rows<T>(dst[i], src[i], p->n, p->m, w128)
+                        : p->sk_S == 1 ? (p->nb == 1 ? map_sys_rows3<T>(dst[i], src[i], p, w128)
+                                                     : map_sys_rows4<T>(dst[i], src[i], p, w128))
+                                       : map_il<T>(dst[i], src[i], p->n, p->ms, p->nb, p->sk_S, p->es, p->bs);
         if (!ok) return false;
     }
     tm_store(p, tag, key, 4, &tm.a, 4);
@@ -71,9 +97,10 @@ template <typename T>
 cudaError_t scan_t(tri_plan_s* p, const void* a, const void* b, const void* c, const void* d, void* x,
                    cudaStream_t st) {
     const int S = p->sk_S;
+    const bool contig = p->layout == TRI_LAYOUT_CONTIGUOUS;  // the one-window kernels assume system stride n
     if constexpr (sizeof(T) == 4) {
         // fp32 one-window systems, n % 32 == 0 (c4): two systems per warp, 16 rows per lane
-        if (S == 1 && p->sk_nc == 1 && p->n % 32 == 0) {
+        if (contig && S == 1 && p->sk_nc == 1 && p->n % 32 == 0) {
             StreamMaps tm;
             const void* key[4] = {a, b, c, d};
             if (!tm_lookup(p, 0x1800, key, 4, &tm.a, 4)) {
@@ -85,27 +112,39 @@ cudaError_t scan_t(tri_plan_s* p, const void* a, const void* b, const void* c, c
             ScanArgs<float> A{};
             A.x = (float*)x;
             A.n = p->n; A.m = p->m; A.ms = p->ms; A.NC = 1;
-            cudaError_t e = set_smem((const void*)k_scan1_r16, S16::smem_bytes);
+            cudaError_t e = set_smem((const void*)k_scan1_r16<float>, S16::smem_bytes);
             if (e != cudaSuccess) return e;
             const unsigned grid = (unsigned)std::min<int64_t>((p->m + 1) / 2, p->sms);
-            k_scan1_r16<<<grid, S16_NW * 32, S16::smem_bytes, st>>>(tm, A);
+            k_scan1_r16<float><<<grid, S16_NW * 32, S16::smem_bytes, st>>>(tm, A);
             return cudaGetLastError();
         }
     }
     // one-window systems shorter than 3/4 of a window (many idle rows: compute-heavy)
     // run the chain-free kernel with more warps (fp32 n = 128: 1.19 ms vs 1.50 ms
     // per 2^28 rows); at n = 256 the 12-warp kernel is faster (c4: 0.99 vs 1.02 ms)
-    const bool one = S == 1 && p->sk_nc == 1 && p->n <= 3 * SC_W / 4;
+    const bool one = contig && S == 1 && p->sk_nc == 1 && p->n <= 3 * SC_W / 4;
     // 128-byte TMA rows (n % 32 fp32 / n % 16 fp64; the k_scan chain and one-window
     // paths): one TMA request per 128 bytes (fp32 c4: 0.99 -> 0.84 ms)
     const bool w128 = S == 1 && p->n % (128 / (int)sizeof(T)) == 0 && !one;
     StreamMaps tm;
-    if (!scan_maps<T>(p, 0x1000 + (int)sizeof(T) + 16 * (w128 ? 1 : 0), a, b, c, d, w128, tm))
+    if (one) {  // k_scan1: 3D view [m][n/8][8]
+        const void* key[4] = {a, b, c, d};
+        if (!tm_lookup(p, 0x1400 + (int)sizeof(T), key, 4, &tm.a, 4)) {
+            if (!map_sys_rows<T>(&tm.a, a, p->n, p->m, false) || !map_sys_rows<T>(&tm.b, b, p->n, p->m, false) ||
+                !map_sys_rows<T>(&tm.c, c, p->n, p->m, false) || !map_sys_rows<T>(&tm.d, d, p->n, p->m, false))
+                return cudaErrorNotSupported;
+            tm_store(p, 0x1400 + (int)sizeof(T), key, 4, &tm.a, 4);
+        }
+    } else if (!scan_maps<T>(p, 0x1000 + (int)sizeof(T) + 16 * (w128 ? 1 : 0), a, b, c, d, w128, tm)) {
         return cudaErrorNotSupported;
+    }
     ScanArgs<T> A;
     A.x = (T*)x;
     A.spill = (T*)p->scratch;
     A.n = p->n; A.m = p->m; A.ms = p->ms; A.NC = p->sk_nc; A.S_on = p->sk_son; A.delta = p->sk_delta;
+    A.xsys = p->ss; A.xbat = p->bs; A.xel = p->es; A.nb = (int)p->nb;
+    A.x32 = ((uintptr_t)x % 32 == 0 && (p->ss * (int64_t)sizeof(T)) % 32 == 0 &&
+             (p->nb == 1 || (p->bs * (int64_t)sizeof(T)) % 32 == 0)) ? 1 : 0;
     A.w128 = w128 ? 1 : 0;
     A.prof = (unsigned long long*)g_fused_prof;
     A.dbg = g_fused_dbg_mode;
@@ -147,6 +186,7 @@ cudaError_t scan_mc_setup(tri_plan_s* p, const void* a, const void* b, const voi
     A = ScanMCArgs<T>{};
     A.w128 = w ? 1 : 0;
     A.x = (T*)x;
+    A.x32 = ((uintptr_t)x % 32 == 0 && (n * (int64_t)sizeof(T)) % 32 == 0) ? 1 : 0;
     A.cd = (T*)p->scratch;
     const int64_t mp = p->m * (int64_t)p->mc_P;
     A.cmap = reinterpret_cast<double*>(A.cd + p->m * (int64_t)p->sk_nc * sc_slot_elems<T>());  // 2 KB multiples

@@ -53,7 +53,14 @@ struct tri_plan_s {
     int sk_grid = 0, sk_nc = 0, sk_son = 0;  // STREAM / SCAN: persistent CTAs, windows per system, resident slots
     int sk_delta = 8;             // SCAN: back-substitution lag (steps)
     int sk_S = 1;                 // SCAN: systems per window (1 contiguous; 8 interleaved)
-    int64_t ms = 0;               // systems per batch (BATCHED; m otherwise)
+    int64_t ms = 0;               // systems per batch (BATCHED / STRIDED; m otherwise)
+    // element (system q = b ms + s, row i) at offset i es + s ss + b bs (elements) of
+    // every array, for every layout: CONTIGUOUS (1, n, n m), INTERLEAVED (m, 1, n m),
+    // BATCHED (ms, 1, n ms), STRIDED (caller's)
+    int64_t es = 1, ss = 0, bs = 0, nb = 1;
+    tri_plan_s* inner = nullptr;  // STRIDED, strides no TMA map can describe: packed CONTIGUOUS / INTERLEAVED plan
+    void* packbuf = nullptr;      // ... and its 5 packed arrays
+    size_t packbuf_bytes = 0;
     int mc_P = 0, mc_NCW = 0;     // SCAN_MC: chunks per system, windows per chunk
     int mc_lb = 0, mc_NCWs = 0, mc_Ps = 0;  // SCAN_MC look-back path: on, windows per small chunk, small chunks
     size_t smem_optin = 0;
@@ -134,6 +141,10 @@ cudaError_t launch_split(tri_plan_s* p, const void* a, const void* b, const void
 cudaError_t launch_split_pcr(tri_plan_s* p, const void* a, const void* b, const void* c, const void* d, void* ao,
                              void* co, void* do_, cudaStream_t st);  // tri_debug_pcr: the PCR passes only
 void split_geometry(tri_plan_s* p);
+// STRIDED fallback (l_strided.cu): gather a, b, c, d into the inner plan's layout,
+// scatter its x back (one thread per element)
+cudaError_t launch_pack(const tri_plan_s* p, const void* const src[4], void* const dst[4], cudaStream_t st);
+cudaError_t launch_unpack(const tri_plan_s* p, const void* src, void* dst, cudaStream_t st);
 size_t split_scratch(const tri_plan_s* p);
 
 extern void* g_fused_prof;    // tri_debug_set_profile: device counters (diagnostics)

@@ -95,7 +95,24 @@ bool scan_mc_ok(int64_t n, int64_t m, tri_dtype t, tri_layout layout) {
            m < ((int64_t)1 << 31);
 }
 
+// STRIDED plans: the SCAN kernel through TMA maps when the caller's strides allow
+// it -- unit element stride (x-lines: 4D view [nb][ms][n/8][8], n % 8 == 0) or unit
+// system stride (y / z-lines: 3D view [nb][n][ms], 8 systems per window) -- with
+// every other stride a 16-byte multiple; else the packed fallback (l_strided.cu)
+bool strided_fast(int64_t n, int64_t ms, int64_t nb, tri_dtype t, int64_t es, int64_t ss, int64_t bs) {
+    const int64_t sz = (int64_t)esize(t);
+    const bool bok = nb == 1 || (bs * sz) % 16 == 0;
+    if (es == 1 && n % 8 == 0 && (ms == 1 || (ss * sz) % 16 == 0) && bok && cdiv(n, SC_W) <= SC_NCMAX &&
+        n / 8 < ((int64_t)1 << 31) && ms < ((int64_t)1 << 31) && nb < ((int64_t)1 << 31))
+        return true;
+    if (ss == 1 && ms > 1 && (es * sz) % 16 == 0 && bok && cdiv(n, SC_W / 8) <= SC_NCMAX && n < ((int64_t)1 << 31) &&
+        ms < ((int64_t)1 << 31) && nb < ((int64_t)1 << 31))
+        return true;
+    return false;
+}
+
 bool variant_ok(tri_variant v, const tri_plan_s* p) {
+    if (p->layout == TRI_LAYOUT_STRIDED) return v == TRI_VARIANT_SCAN && !p->inner;
     switch (v) {
         case TRI_VARIANT_ONCHIP: return onchip_ok(p->n, p->dtype, p->layout);
         case TRI_VARIANT_SPLIT: return p->layout != TRI_LAYOUT_BATCHED;
@@ -226,9 +243,9 @@ void plan_geometry(tri_plan_s* p) {
     }
     if (p->variant == TRI_VARIANT_SCAN) {
         p->L = n; p->n_pad = n; p->C = m;
-        p->sk_S = scan_systems(p->layout, m);
+        p->sk_S = p->layout == TRI_LAYOUT_STRIDED ? (p->es == 1 ? 1 : 8) : scan_systems(p->layout, m);
         p->sk_nc = (int)cdiv(n, SC_W / p->sk_S);
-        const int64_t ms = p->layout == TRI_LAYOUT_BATCHED ? p->ms : m;
+        const int64_t ms = p->ms;
         const int64_t groups = p->sk_S == 1 ? m : cdiv(ms, p->sk_S) * (m / ms);
         p->sk_grid = (int)std::min<int64_t>(groups, p->sms);
         p->sk_delta = SCAN_DELTA;
@@ -333,14 +350,21 @@ tri_status set_plan(tri_plan_s* p, tri_variant v, int k) {
     return st;
 }
 
+// STRIDED packed fallback: gather into the dense layout whose order follows the
+// source's unit stride (rows -> CONTIGUOUS, systems -> INTERLEAVED), solve with an
+// inner plan, scatter x (l_strided.cu)
+tri_status make_packed(tri_plan_s* p);
+
 tri_status check_ptrs(tri_plan_s* p, const void* const* in, int nin, const void* const* out, int nout) {
-    const size_t bytes = (size_t)p->n * (size_t)p->m * esize(p->dtype);
+    // footprint of an array: its last element's offset + 1 (n m for the dense layouts)
+    const size_t bytes = (size_t)((p->n - 1) * p->es + (p->ms - 1) * p->ss + (p->nb - 1) * p->bs + 1) * esize(p->dtype);
     bool same = nin + nout <= 8;
     for (int i = 0; i < nin + nout && same; ++i) same = p->seen[i] == (i < nin ? in[i] : out[i - nin]);
     for (int i = 0; i < nin + nout; ++i) {
         const void* q = i < nin ? in[i] : out[i - nin];
         if (!q) return TRI_ERR_INVALID_ARG;
-        if (((uintptr_t)q & 15) != 0) return TRI_ERR_ALIGNMENT;
+        // STRIDED views may start anywhere (element-aligned); tri_solve picks the path
+        if (((uintptr_t)q & (p->layout == TRI_LAYOUT_STRIDED ? esize(p->dtype) - 1 : 15)) != 0) return TRI_ERR_ALIGNMENT;
         if (same) continue;  // residency verified on the previous call with these pointers
         cudaPointerAttributes at;
         if (cudaPointerGetAttributes(&at, q) != cudaSuccess) { cudaGetLastError(); return TRI_ERR_DEVICE; }
@@ -376,12 +400,31 @@ tri_status current_device_ok(int* dev, int* sms) {
     return TRI_OK;
 }
 
+tri_plan_s* new_plan(int64_t n, int64_t m, int64_t ms, tri_dtype dtype, tri_layout layout, tri_status* st);
+
+tri_status make_packed(tri_plan_s* p) {
+    const tri_layout il = (p->ss == 1 && p->es != 1) ? TRI_LAYOUT_INTERLEAVED : TRI_LAYOUT_CONTIGUOUS;
+    tri_status st;
+    p->inner = new_plan(p->n, p->m, p->m, p->dtype, il, &st);
+    if (!p->inner) return st;
+    p->variant = p->inner->variant;
+    p->k = p->inner->k;
+    const size_t bytes = 5 * ((size_t)p->n * (size_t)p->m * esize(p->dtype) / 256 * 256 + 256);
+    if (cudaMalloc(&p->packbuf, bytes) != cudaSuccess) { cudaGetLastError(); return TRI_ERR_OOM; }
+    p->packbuf_bytes = bytes;
+    return TRI_OK;
+}
+
 tri_plan_s* new_plan(int64_t n, int64_t m, int64_t ms, tri_dtype dtype, tri_layout layout, tri_status* st) {
     int dev = 0, sms = 0;
     *st = current_device_ok(&dev, &sms);
     if (*st != TRI_OK) return nullptr;
     tri_plan_s* p = new tri_plan_s();
     p->n = n; p->m = m; p->ms = ms; p->dtype = dtype; p->layout = layout; p->device = dev; p->sms = sms;
+    p->nb = m / ms;
+    if (layout == TRI_LAYOUT_CONTIGUOUS) { p->es = 1; p->ss = n; p->bs = n * m; }
+    else if (layout == TRI_LAYOUT_INTERLEAVED) { p->es = m; p->ss = 1; p->bs = n * m; }
+    else { p->es = ms; p->ss = 1; p->bs = n * ms; }  // BATCHED
     int optin = 0;
     cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
     p->smem_optin = (size_t)optin;
@@ -475,8 +518,42 @@ tri_plan_t tri_plan_batched(int64_t n, int64_t ms, int64_t nb, tri_dtype dtype) 
     return p;
 }
 
+tri_plan_t tri_plan_strided(int64_t n, int64_t ms, int64_t nb, tri_dtype dtype, int64_t es, int64_t ss,
+                            int64_t bs) {
+    if (n < 1 || ms < 1 || nb < 1 || (dtype != TRI_F32 && dtype != TRI_F64) || ms > MAX_ELEMS / nb ||
+        n > MAX_ELEMS / (ms * nb) || es < 1 || ss < 1 || bs < 1) {
+        g_last = TRI_ERR_INVALID_ARG;
+        return nullptr;
+    }
+    // distinct elements: a row / system / batch step must move past the other two
+    // dimensions' extents in at least the order the caller nests them -- the
+    // footprint check is the caller's; here only positive strides are required
+    int dev = 0, sms = 0;
+    tri_status st = current_device_ok(&dev, &sms);
+    if (st != TRI_OK) { g_last = st; return nullptr; }
+    tri_plan_s* p = new tri_plan_s();
+    p->n = n; p->m = ms * nb; p->ms = ms; p->nb = nb; p->dtype = dtype; p->layout = TRI_LAYOUT_STRIDED;
+    p->device = dev; p->sms = sms; p->es = es; p->ss = ss; p->bs = bs;
+    int optin = 0;
+    cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+    p->smem_optin = (size_t)optin;
+    if (strided_fast(n, ms, nb, dtype, es, ss, bs)) {
+        p->variant = TRI_VARIANT_SCAN;
+        p->k = 0;
+        plan_geometry(p);
+        st = ensure_scratch(p);
+    } else {
+        st = make_packed(p);
+    }
+    if (st != TRI_OK) { tri_destroy(p); g_last = st; return nullptr; }
+    g_last = TRI_OK;
+    return p;
+}
+
 void tri_destroy(tri_plan_t p) {
     if (!p) return;
+    tri_destroy(p->inner);
+    if (p->packbuf) cudaFree(p->packbuf);
     for (int i = 0; i < 2; ++i) tri_destroy(p->sub[i]);
     for (int i = 0; i < 3; ++i)
         if (p->hs[i]) cudaStreamDestroy(p->hs[i]);
@@ -493,6 +570,7 @@ int64_t tri_plan_scratch_bytes(tri_plan_t p) { return p ? (int64_t)p->scratch_by
 
 int tri_plan_launches(tri_plan_t p) {
     if (!p) return -1;
+    if (p->inner) return tri_plan_launches(p->inner) + 2;  // gather, inner solve, scatter
     if (p->variant == TRI_VARIANT_SPLIT) return p->k == 0 ? 1 : p->npass + 1;
     if (p->variant == TRI_VARIANT_SCAN_MC) return p->mc_lb ? 2 : 3;  // three passes, or look-back kernel + pass 2
     return 1;
@@ -500,6 +578,12 @@ int tri_plan_launches(tri_plan_t p) {
 
 tri_status tri_plan_set_k(tri_plan_t p, int k) {
     if (!p || k < 0 || k > floor_log2(p->n)) return TRI_ERR_INVALID_ARG;
+    if (p->layout == TRI_LAYOUT_STRIDED) {  // the packed fallback's inner plan runs any k
+        if (!p->inner) return k == 0 ? TRI_OK : TRI_ERR_INVALID_ARG;
+        const tri_status st = tri_plan_set_k(p->inner, k);
+        if (st == TRI_OK) { p->k = p->inner->k; p->variant = p->inner->variant; }
+        return st;
+    }
     tri_variant v = p->variant;
     if (k < kmin_for(v) || k > kmax_for(v, p->n)) {
         // the current variant does not run this k: the fastest variant that does
@@ -523,6 +607,12 @@ tri_status tri_plan_set_k(tri_plan_t p, int k) {
 
 tri_status tri_plan_set_variant(tri_plan_t p, tri_variant v) {
     if (!p) return TRI_ERR_INVALID_ARG;
+    if (p->layout == TRI_LAYOUT_STRIDED) {
+        if (!p->inner) return (v == TRI_VARIANT_AUTO || v == TRI_VARIANT_SCAN) ? TRI_OK : TRI_ERR_INVALID_ARG;
+        const tri_status st = tri_plan_set_variant(p->inner, v);
+        if (st == TRI_OK) { p->k = p->inner->k; p->variant = p->inner->variant; }
+        return st;
+    }
     const bool autov = v == TRI_VARIANT_AUTO;
     if (autov) v = choose_variant(p->n, p->m, p->dtype, p->layout, p->sms);
     if (!variant_ok(v, p)) return TRI_ERR_INVALID_ARG;
@@ -533,6 +623,7 @@ tri_status tri_plan_set_variant(tri_plan_t p, tri_variant v) {
 
 tri_status tri_plan_set_option(tri_plan_t p, tri_option opt, int value) {
     if (!p) return TRI_ERR_INVALID_ARG;
+    if (p->layout == TRI_LAYOUT_STRIDED) return p->inner ? tri_plan_set_option(p->inner, opt, value) : TRI_ERR_INVALID_ARG;
     if (opt == TRI_OPT_TMA) {
         if (value != 0 && value != 1) return TRI_ERR_INVALID_ARG;
         p->opt_tma = value;
@@ -567,7 +658,7 @@ tri_status tri_slice_solve(tri_plan_t p, int phase, int slice, int nslices, cons
 
 tri_status tri_plan_autotune(tri_plan_t p, const void* a, const void* b, const void* c, const void* d, void* x,
                              void* stream, int reps, float* best_us) {
-    if (!p || reps < 1) return TRI_ERR_INVALID_ARG;
+    if (!p || reps < 1 || p->layout == TRI_LAYOUT_STRIDED) return TRI_ERR_INVALID_ARG;
     const void* in[4] = {a, b, c, d};
     const void* out[1] = {x};
     tri_status st = check_ptrs(p, in, 4, out, 1);
@@ -623,7 +714,8 @@ void tri_plan_describe(tri_plan_t p, char* buf, int len) {
              "fu_grid=%d fu_son=%d fu_nc=%lld sk_grid=%d sk_nc=%d sk_son=%d mc_P=%d lookback=%d tma=%d scratch=%zu "
              "sms=%d",
              (long long)p->n, (long long)p->m, p->dtype == TRI_F64 ? "f64" : "f32",
-             p->layout == TRI_LAYOUT_CONTIGUOUS ? "contiguous" : p->layout == TRI_LAYOUT_INTERLEAVED ? "interleaved" : "batched",
+             p->layout == TRI_LAYOUT_CONTIGUOUS ? "contiguous" : p->layout == TRI_LAYOUT_INTERLEAVED ? "interleaved"
+             : p->layout == TRI_LAYOUT_BATCHED ? "batched" : (p->inner ? "strided(packed)" : "strided"),
              vn[p->variant], p->k, passes, p->G, p->P, p->rpt, (long long)p->L, (long long)p->C, p->fu_grid,
              p->fu_son, (long long)p->fu_nc, p->sk_grid, p->sk_nc, p->sk_son, p->mc_P, p->mc_lb ? p->mc_NCWs : 0,
              p->opt_tma, p->scratch_bytes, p->sms);
@@ -638,6 +730,24 @@ tri_status tri_solve(tri_plan_t p, const void* a, const void* b, const void* c, 
     if (st != TRI_OK) return st;
     cudaStream_t s = (cudaStream_t)stream;
     cudaError_t e;
+    if (p->layout == TRI_LAYOUT_STRIDED && !p->inner) {
+        // the TMA path needs 16-byte aligned view origins; a view that starts
+        // elsewhere (odd x0 of a sub-grid) switches the plan to the packed path
+        bool al = ((uintptr_t)x & 15) == 0;
+        for (int i = 0; i < 4; ++i) al = al && ((uintptr_t)in[i] & 15) == 0;
+        if (!al && (st = make_packed(p)) != TRI_OK) return st;
+    }
+    if (p->inner) {  // STRIDED, packed fallback: gather, solve the dense copy, scatter x
+        const size_t slot = (size_t)p->n * (size_t)p->m * esize(p->dtype) / 256 * 256 + 256;
+        char* pb = (char*)p->packbuf;
+        void* const dv[4] = {pb, pb + slot, pb + 2 * slot, pb + 3 * slot};
+        e = launch_pack(p, in, dv, s);
+        if (e != cudaSuccess) return TRI_ERR_CUDA;
+        st = tri_solve(p->inner, dv[0], dv[1], dv[2], dv[3], pb + 4 * slot, stream);
+        if (st != TRI_OK) return st;
+        e = launch_unpack(p, pb + 4 * slot, x, s);
+        return e == cudaSuccess ? TRI_OK : TRI_ERR_CUDA;
+    }
     switch (p->variant) {
         case TRI_VARIANT_WARP: e = launch_warp(p, a, b, c, d, x, nullptr, nullptr, nullptr, 0, s); break;
         case TRI_VARIANT_ONCHIP: e = launch_onchip(p, a, b, c, d, x, nullptr, nullptr, nullptr, 0, s); break;
@@ -652,7 +762,7 @@ tri_status tri_solve(tri_plan_t p, const void* a, const void* b, const void* c, 
 
 tri_status tri_debug_pcr(tri_plan_t p, const void* a, const void* b, const void* c, const void* d, void* ao,
                          void* co, void* do_, void* stream) {
-    if (!p) return TRI_ERR_INVALID_ARG;
+    if (!p || p->layout == TRI_LAYOUT_STRIDED) return TRI_ERR_INVALID_ARG;
     const void* in[4] = {a, b, c, d};
     const void* out[3] = {ao, co, do_};
     tri_status st = check_ptrs(p, in, 4, out, 3);
@@ -782,7 +892,7 @@ extern "C" {
 
 tri_status tri_solve_host(tri_plan_t p, const void* a, const void* b, const void* c, const void* d, void* x,
                           void* stream) {
-    if (!p || !a || !b || !c || !d || !x) return TRI_ERR_INVALID_ARG;
+    if (!p || !a || !b || !c || !d || !x || p->layout == TRI_LAYOUT_STRIDED) return TRI_ERR_INVALID_ARG;
     const size_t bytes = (size_t)p->n * (size_t)p->m * esize(p->dtype);
     const bool pipe = p->layout == TRI_LAYOUT_CONTIGUOUS && p->m >= 2 * HOST_CHUNKS;
     const size_t slot = pipe ? host_chunks(p).slot : align256(bytes);
