@@ -28,8 +28,10 @@ CASES = {
              (128, 40, "f32", 0, V.VARIANT_SCAN, None)],     # short one-window systems (k_scan1)
     "scan_il": [(1024, 16, "f64", 1, V.VARIANT_SCAN, None),  # interleaved, S = 8: two 8-system groups
                 (520, 24, "f32", 1, V.VARIANT_SCAN, None)],  # ragged last window
+    "scan_r16": [(256, 40, "f32", 0, V.VARIANT_SCAN, None), (224, 33, "f32", 0, V.VARIANT_SCAN, None)],
     "scan_mc": [(1 << 16, 1, "f64", 0, V.VARIANT_SCAN_MC, None),
                 (40960, 2, "f32", 0, V.VARIANT_SCAN_MC, None)],
+    "scan_mc_lb": [(1 << 16, 1, "f64", 0, V.VARIANT_SCAN_MC, "lb32"), (40960, 2, "f32", 0, V.VARIANT_SCAN_MC, "lb16")],
     "stream": [(4096, 3, "f64", 0, V.VARIANT_STREAM, None)],
     "fused": [(2048, 3, "f64", 0, V.VARIANT_FUSED, None), (2000, 2, "f32", 0, V.VARIANT_FUSED, None)],
     "warp": [(512, 16, "f64", 0, V.VARIANT_WARP, None), (256, 16, "f32", 1, V.VARIANT_WARP, None)],
@@ -45,11 +47,13 @@ def main():
     torch.cuda.set_device(0)
     worst = 0.0
     for f in fams:
-        for (n, m, dt, layout, v, k) in CASES[f]:
+        for (n, m, dt, layout, v, k) in CASES.get(f, []):
             arrs = trigen.generate(n, m, dt, layout, "dd")
             plan = tri.Plan(n, m, tri.F64 if dt == "f64" else tri.F32, layout)
             plan.variant = v
-            if k is not None:
+            if isinstance(k, str):  # "lbW": SCAN_MC look-back with W-window chunks
+                plan.set_option(tri.OPT_SCAN_MC_LOOKBACK, int(k[2:]))
+            elif k is not None:
                 plan.k = k
             a, b, c, d = (torch.from_numpy(t).cuda() for t in arrs)
             x = plan.solve(a, b, c, d)
@@ -60,6 +64,26 @@ def main():
             worst = max(worst, err / tol)
             print(f"{f}: n={n} m={m} {dt} layout={layout} err={err:.2e} [{plan.describe()}]", flush=True)
             assert err <= tol
+    if "strided" in fams:
+        # pitched views of a [5][24][72] array: x-lines (TMA path) and an odd-pitch packed case
+        for (n, ms, nb, es, ss, bs, off) in [(64, 20, 4, 1, 72, 24 * 72, 72 + 8), (20, 60, 4, 72, 1, 24 * 72, 1)]:
+            m = ms * nb
+            arrs = trigen.generate(n, m, "f64", 0, "dd")
+            q = np.arange(m)
+            flat = (off + (q % ms)[:, None] * ss + (q // ms)[:, None] * bs + np.arange(n)[None, :] * es).reshape(-1)
+            par = []
+            for t in arrs:
+                P = np.zeros(5 * 24 * 72, dtype=np.float64)
+                P[flat] = t
+                par.append(torch.from_numpy(P).cuda())
+            xd = torch.zeros_like(par[0])
+            plan = tri.Plan.strided(n, ms, nb, es, ss, bs, tri.F64)
+            plan.solve(*[t[off:] for t in par], out=xd[off:])
+            torch.cuda.synchronize()
+            xo = oracle.solve_batch(n, m, *arrs)
+            err = float(np.max(np.abs(xd.cpu().numpy()[flat] - xo) / np.abs(xo)))
+            print(f"strided: n={n} ms={ms} nb={nb} err={err:.2e} [{plan.describe()}]", flush=True)
+            assert err <= 1e-10
     print(f"sanitize cases ok (worst err / tol = {worst:.2e})")
 
 
