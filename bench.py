@@ -231,12 +231,21 @@ def main():
     from paper_conf_icpp_kimwch11_b200 import dist as tdist
 
     world, rank, local = dist_env()
-    if world > 1:
+    ngpu = torch.cuda.device_count()
+    backend = "nccl"
+    if world > 1 and ngpu >= world:
         torch.cuda.set_device(local)
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    elif world > 1:
+        # fewer GPUs than ranks (a code-path check on a 1-GPU box, not a scaling
+        # measurement): ranks share devices, collectives over gloo; the line says so
+        backend = "gloo"
+        torch.cuda.set_device(local % ngpu)
+        dist.init_process_group("gloo")
     else:
         torch.cuda.set_device(0)
     dev = torch.device("cuda", torch.cuda.current_device())
+    rdev = dev if backend == "nccl" else torch.device("cpu")  # device of the all-reduce scalars
 
     n, m, dt, layout, desc = CONFIGS[args.config]
     if args.layout is not None:
@@ -323,7 +332,7 @@ def main():
         dist.barrier()
     step_ms = [e0.elapsed_time(e1) for e0, e1 in ev]
     t_step = sum(step_ms) / len(step_ms)
-    t_step_max = tdist.max_over_ranks(t_step, device=dev)
+    t_step_max = tdist.max_over_ranks(t_step, device=rdev)
     value = m_all * n / (t_step_max * 1e-3) / 1e6  # whole-job Munknowns/s
 
     # ---- per-call latency of a direct (non-graph) tri_solve: idle GPU, events
@@ -374,7 +383,7 @@ def main():
         t0 = time.perf_counter()
         for _ in range(args.e2e_steps):
             plan.solve_host(*host, xh, stream=stream)  # synchronises its stream
-        te = tdist.max_over_ranks((time.perf_counter() - t0) / args.e2e_steps, device=dev)
+        te = tdist.max_over_ranks((time.perf_counter() - t0) / args.e2e_steps, device=rdev)
         e2e = {"value": m_all * n / te / 1e6, "unit": "Munknowns/s",
                "h2d_bytes_per_step": 4 * n_unknowns * s, "d2h_bytes_per_step": n_unknowns * s,
                "steps": args.e2e_steps, "ms_per_step": te * 1e3,
@@ -389,7 +398,7 @@ def main():
     if world > 1 and scaling == "strong" and not args.no_collectives:
         try:
             coll = edge_collectives(args, tdist, trigen, n, m, dt, layout, seed, q0, mr, (a, b, c, d), x, s, world,
-                                    rank, dev, tdt)
+                                    rank, dev, tdt, rdev)
         except Exception as exc:  # never let the edge measurement cost the solve numbers
             coll = {"error": repr(exc)[:300]}
 
@@ -426,7 +435,9 @@ def main():
                    "family": args.family,
                    "parallelism": (f"dp{world}: the m systems sharded over the ranks (contiguous ranges, "
                                    "dist.shard_range), no collective in the solve" if scaling == "strong" else
-                                   f"dp{world}: replicas (every rank solves its own {m} system(s))"),
+                                   f"dp{world}: replicas (every rank solves its own {m} system(s))") +
+                                  ("" if backend == "nccl" or world == 1 else
+                                   f" [code-path check: {world} ranks on {ngpu} GPU(s), gloo collectives]"),
                    "timing": "CUDA graph replay of one solve per step" if graph is not None else "direct solve call",
                    "l2": "flushed between timed steps (2x L2 write + 2x L2 read)" if flush else
                          f"inputs larger than L2 ({ws / 2**30:.1f} GiB working set vs {l2 / 2**20:.0f} MiB L2)",
@@ -453,7 +464,8 @@ def main():
         dist.destroy_process_group()
 
 
-def edge_collectives(args, tdist, trigen, n, m, dt, layout, seed, q0, mr, local, x_local, s, world, rank, dev, tdt):
+def edge_collectives(args, tdist, trigen, n, m, dt, layout, seed, q0, mr, local, x_local, s, world, rank, dev, tdt,
+                     rdev):
     """SURVEY 8(e) edge collectives through dist.py on the real shards: rank 0
     scatters a, b, c, d (dist.scatter_inputs) and gathers x (dist.gather_x);
     CUDA events, max over ranks.  Checks: every rank's scattered shard equals
@@ -477,9 +489,9 @@ def edge_collectives(args, tdist, trigen, n, m, dt, layout, seed, q0, mr, local,
                 xfull = tdist.gather_x(x_local, n, m, layout)
             e1.record()
             torch.cuda.synchronize()
-        res[what] = tdist.max_over_ranks(e0.elapsed_time(e1), device=dev)
+        res[what] = tdist.max_over_ranks(e0.elapsed_time(e1), device=rdev)
     same = all(torch.equal(g, l) for g, l in zip(got, local))
-    ok = tdist.max_over_ranks(0.0 if same else 1.0, device=dev) == 0.0
+    ok = tdist.max_over_ranks(0.0 if same else 1.0, device=rdev) == 0.0
     per = -(-m // world)
     moved = (world - 1) * n * per * s  # bytes of one array leaving / entering rank 0
     out = {"scatter_ms": res["scatter"], "gather_ms": res["gather"], "scatter_bytes": 4 * moved, "gather_bytes": moved,

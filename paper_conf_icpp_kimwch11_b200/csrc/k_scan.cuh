@@ -707,11 +707,17 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
         if (bwd && p.dbg != 2) {
             SC_T(5);
             const unsigned tg = (unsigned)(bj % 65535 + 1);
-            const int* e = reinterpret_cast<const int*>(&tab[(bj % K) * NC + wb]);
-            unsigned v = (unsigned)sk_ld_acquire(e);
+            // The window was stored at step gs >= g - delta - 1 by warp gs % NW, after
+            // that step's handover; with delta >= 2 NW the named-barrier chain orders it
+            // before this read (gs's store precedes warp gs % NW's arrive at step
+            // gs + NW, which every step >= gs + NW + 1 syncs after, and this step's
+            // warp synced at step g - NW >= gs + NW + 1): a plain load sees the entry.
+            // The tag check stays as a guard (never spins when delta >= 2 NW).
+            const volatile unsigned* e = &tab[(bj % K) * NC + wb];
+            unsigned v = *e;
             while ((v >> 16) != tg) {  // window (bj, wb) stored
                 __nanosleep(64);
-                v = (unsigned)sk_ld_acquire(e);
+                v = *e;
             }
             SC_T(4);
             slot = (int)(v & 0xffffu);
@@ -831,10 +837,8 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
             if (res) sc_store_slot_s(sp_s, lane, cpf, dpf);
             else sc_store_slot_g(sp_g, lane, cpf, dpf, pol_sp);
             __syncwarp();
-            if (lane == 0) {
-                sk_st_release(reinterpret_cast<int*>(&tab[(cj % K) * NC + cw]),
-                              (int)(((unsigned)(cj % 65535 + 1) << 16) | (unsigned)slot));
-            }
+            if (lane == 0)  // read >= 2 NW + 1 steps later, ordered by the barrier chain (see the read)
+                *reinterpret_cast<volatile unsigned*>(&tab[(cj % K) * NC + cw]) = ((unsigned)(cj % 65535 + 1) << 16) | (unsigned)slot;
         }
         // ---- backward replay: x (Eq 4) of window (bj, wb)
         if (bwd) {

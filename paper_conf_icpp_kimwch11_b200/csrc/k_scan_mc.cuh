@@ -147,7 +147,10 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant
     const int nwin = min(NC, w0 + p.NCW) - w0;
     T* ib = reinterpret_cast<T*>(sbase + L::off_in + pw * L::in_stride);
     const uint64_t pol_in = sk_policy_evict_first();
-    auto win_of = [&](int g) { return MODE == 2 ? w0 + nwin - 1 - g : w0 + g; };
+    // pass 0 and pass 2 walk their chunk backwards, pass 1 forwards: each pass
+    // starts where the previous one ended, so the windows still in L2 (the last
+    // ~100 MB a pass touched, at the same end of every chunk) are read first
+    auto win_of = [&](int g) { return MODE != 1 ? w0 + nwin - 1 - g : w0 + g; };
     auto issue = [&](int g) {
         const int w = win_of(g);
         if (MODE < 2) {
@@ -226,7 +229,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant
                 if ((lane & (2 * d - 1)) == 0) { M = sk_compose(o, M); smc_rescale(M); }
             }
             if (lane == 0) {
-                double* s = wm + 8 * g;
+                double* s = wm + 8 * (w - w0);  // by window (pass 0 walks backwards)
                 s[0] = M.a; s[1] = M.b; s[2] = M.c; s[3] = M.d; s[4] = M.e; s[5] = M.f; s[6] = M.g;
             }
         } else if (MODE == 1) {
@@ -460,11 +463,13 @@ __global__ void __launch_bounds__(LB_THREADS, 1) k_scan_mc_lb(const __grid_const
         for (int k = 0; k < 2 * LB_NA + LB_NB; ++k) sk_bar_init(&bars[k], 1);
         for (int k = 0; k < LB_RING; ++k) sk_bar_init(&tkfull[k], 1);
         for (int k = 0; k < 2; ++k) {
-            sk_bar_init(&mapsfull[k], LB_NA);
-            sk_bar_init(&wmfree[k], 1);
-            sk_bar_init(&statefull[k], 1);
-            sk_bar_init(&stfree[k], 1);
-            sk_bar_init(&bdone[k], 1);
+            // every lane of the arriving warp(s) arrives: each releases its own
+            // shared-memory accesses (no reliance on __syncwarp cumulativity)
+            sk_bar_init(&mapsfull[k], LB_NA * 32);
+            sk_bar_init(&wmfree[k], 32);
+            sk_bar_init(&statefull[k], 32);
+            sk_bar_init(&stfree[k], 32);
+            sk_bar_init(&bdone[k], 32);
         }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
@@ -513,7 +518,7 @@ __global__ void __launch_bounds__(LB_THREADS, 1) k_scan_mc_lb(const __grid_const
             const int t = tk[i % LB_RING];
             if (t >= total) {
                 if (i >= 2) sk_wait(&wmfree[par], (unsigned)(((i >> 1) - 1) & 1));  // never two phases ahead of L
-                if (lane == 0) sk_arrive(&mapsfull[par]);  // tells the L warp: no more chunks
+                sk_arrive(&mapsfull[par]);  // tells the L warp: no more chunks
                 break;
             }
             const int nwin = nwin_of(t);
@@ -553,7 +558,7 @@ __global__ void __launch_bounds__(LB_THREADS, 1) k_scan_mc_lb(const __grid_const
             }
             __syncwarp();
             if (lb.prof && aw == 0 && lane == 0) lb.prof[(int64_t)t * 8 + 1] = lb_now();
-            if (lane == 0) sk_arrive(&mapsfull[par]);  // release: this warp's maps are in shared memory
+            sk_arrive(&mapsfull[par]);  // release: this warp's maps are in shared memory
         }
     } else if (warp == LB_NA) {
         // ======================= L: aggregate, look-back, incoming state =======================
@@ -564,10 +569,8 @@ __global__ void __launch_bounds__(LB_THREADS, 1) k_scan_mc_lb(const __grid_const
             const int t = tk[i % LB_RING];
             if (i >= 2) sk_wait(&stfree[par], (unsigned)(((i >> 1) - 1) & 1));  // B has read chunk i - 2's state
             if (t >= total) {
-                if (lane == 0) {
-                    st0[4 * par + 3] = (double)t;
-                    sk_arrive(&statefull[par]);
-                }
+                if (lane == 0) st0[4 * par + 3] = (double)t;
+                sk_arrive(&statefull[par]);
                 break;
             }
             const int nwin = nwin_of(t);
@@ -657,12 +660,9 @@ __global__ void __launch_bounds__(LB_THREADS, 1) k_scan_mc_lb(const __grid_const
                     s[2] = __shfl_sync(0xffffffffu, yd * sy, 31);
                 }
             }
-            __syncwarp();
-            if (lane == 0) {
-                if (lb.prof) lb.prof[(int64_t)t * 8 + 3] = lb_now();
-                sk_arrive(&wmfree[par]);     // the window maps are consumed
-                sk_arrive(&statefull[par]);  // release: the window states are in shared memory
-            }
+            if (lb.prof && lane == 0) lb.prof[(int64_t)t * 8 + 3] = lb_now();
+            sk_arrive(&wmfree[par]);     // the window maps are consumed
+            sk_arrive(&statefull[par]);  // release: the window states are in shared memory
         }
     } else {
         // ======================= B: forward replay, c', d', backward maps =======================
@@ -743,7 +743,8 @@ __global__ void __launch_bounds__(LB_THREADS, 1) k_scan_mc_lb(const __grid_const
                 if (lane == 0) { lb.rec[(int64_t)t * SMC_REC + 12] = al; lb.rec[(int64_t)t * SMC_REC + 13] = be; }
                 __syncwarp();
                 if (lb.prof && lane == 0) { lb.prof[(int64_t)t * 8 + 6] = lb_now(); lb.prof[(int64_t)t * 8 + 7] = blockIdx.x; }
-                if (lane == 0) { sk_arrive(&bdone[par]); sk_arrive(&stfree[par]); }
+                sk_arrive(&bdone[par]);
+                sk_arrive(&stfree[par]);
             }
         }
     }

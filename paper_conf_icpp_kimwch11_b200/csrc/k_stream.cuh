@@ -284,7 +284,7 @@ __global__ void __launch_bounds__(SK_THREADS, 1) k_stream(const __grid_constant_
         for (int i = 0; i < SK_NPCR; ++i) {
             sk_bar_init(&in_full[i], 1);
         }
-        for (int i = 0; i < NC; ++i) sk_bar_init(&sfull[i], 1);
+        for (int i = 0; i < NC; ++i) sk_bar_init(&sfull[i], 32);  // every lane releases its own slot stores
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
     }
@@ -615,7 +615,7 @@ __global__ void __launch_bounds__(SK_THREADS, 1) k_stream(const __grid_constant_
             }
         }
         __syncwarp();
-        if (fwd && lane == 0) sk_arrive(&sfull[slot]);
+        if (fwd) sk_arrive(&sfull[slot]);
         SK_PH(0);
     }
     cp_async_wait<0>();

@@ -28,8 +28,11 @@ namespace {
 thread_local tri_status g_last = TRI_OK;
 
 constexpr int64_t MAX_ELEMS = int64_t(1) << 40;
-constexpr int SCAN_DELTA = 8;  // SCAN: back-substitution lag in steps (0..8 measured equal at c1/c2; 8 keeps a
-                               // window's read-back >= 9 steps after its store)
+// SCAN: back-substitution lag in steps.  A window is read back >= delta + 1 steps
+// after its store; with delta >= 2 x warps the named-barrier chain of the step
+// handover orders every store before its read (k_scan.cuh), so no flag protocol
+// is needed (compute-sanitizer racecheck models barriers, not release/acquire flags)
+constexpr int SCAN_DELTA = 2 * SC_NW;
 
 // ---- pure host planner ------------------------------------------------------
 // Rows of (normalised, 3-array) system data one ONCHIP CTA holds: sized for

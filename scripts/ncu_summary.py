@@ -1,5 +1,5 @@
 """Summarise an ncu report (.ncu-rep) into a short text file for profiles/.
-usage: python scripts/ncu_summary.py REPORT OUT.txt [traffic_json n m k]"""
+usage: python scripts/ncu_summary.py REPORT OUT.txt [traffic_json n m k [variant [layout]]]"""
 import csv
 import io
 import json
@@ -36,9 +36,18 @@ for r in rows[2:]:
 open(out, "w").write("\n".join(lines) + "\n")
 print("\n".join(lines))
 if len(sys.argv) > 3:
-    d = dict(zip(hdr, rows[2]))
-    u = dict(zip(hdr, units))
+    # the solve's DRAM bytes: every launch in the report (profile exactly one solve's launches)
     scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}
-    tb = sum(float(d[k].replace(",", "")) * scale.get(u[k], 1) for k in ("dram__bytes_read.sum", "dram__bytes_write.sum"))
-    json.dump({"source": rep, "kernel": d["Kernel Name"], "dram_bytes_per_launch": tb, "n": int(sys.argv[4]),
-               "m": int(sys.argv[5]), "k": int(sys.argv[6])}, open(sys.argv[3], "w"), indent=1)
+    tb, names = 0.0, []
+    for r in rows[2:]:
+        d = dict(zip(hdr, r))
+        u = dict(zip(hdr, units))
+        tb += sum(float(d[k].replace(",", "")) * scale.get(u[k], 1) for k in ("dram__bytes_read.sum", "dram__bytes_write.sum"))
+        names.append(d["Kernel Name"])
+    rec = {"source": rep, "kernels": names, "dram_bytes_per_launch": tb, "n": int(sys.argv[4]), "m": int(sys.argv[5]),
+           "k": int(sys.argv[6])}
+    if len(sys.argv) > 7:
+        rec["variant"] = int(sys.argv[7])
+    if len(sys.argv) > 8:
+        rec["layout"] = int(sys.argv[8])
+    json.dump(rec, open(sys.argv[3], "w"), indent=1)
