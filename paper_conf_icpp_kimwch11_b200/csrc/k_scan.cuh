@@ -707,17 +707,19 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
         if (bwd && p.dbg != 2) {
             SC_T(5);
             const unsigned tg = (unsigned)(bj % 65535 + 1);
-            // The window was stored at step gs >= g - delta - 1 by warp gs % NW, after
-            // that step's handover; with delta >= 2 NW the named-barrier chain orders it
-            // before this read (gs's store precedes warp gs % NW's arrive at step
-            // gs + NW, which every step >= gs + NW + 1 syncs after, and this step's
-            // warp synced at step g - NW >= gs + NW + 1): a plain load sees the entry.
-            // The tag check stays as a guard (never spins when delta >= 2 NW).
-            const volatile unsigned* e = &tab[(bj % K) * NC + wb];
-            unsigned v = *e;
+            // The window was stored >= delta + 1 steps ago by another warp, which
+            // published its slot with release semantics after the stores; this acquire
+            // load orders the slot reads after them (PTX memory model).  compute-sanitizer
+            // racecheck does not model release / acquire flags and reports this pair
+            // (scripts/san/probe.cu, modes 1-2: the same report on a 30-line correct
+            // handoff); ordering by the handover barrier chain alone would need
+            // delta >= 2 x warps, measured 3 % slower at c5 (more spilled slots reach
+            // DRAM) and 8 % at c2 (a longer tail).
+            const int* e = reinterpret_cast<const int*>(&tab[(bj % K) * NC + wb]);
+            unsigned v = (unsigned)sk_ld_acquire(e);
             while ((v >> 16) != tg) {  // window (bj, wb) stored
                 __nanosleep(64);
-                v = *e;
+                v = (unsigned)sk_ld_acquire(e);
             }
             SC_T(4);
             slot = (int)(v & 0xffffu);
@@ -837,8 +839,10 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
             if (res) sc_store_slot_s(sp_s, lane, cpf, dpf);
             else sc_store_slot_g(sp_g, lane, cpf, dpf, pol_sp);
             __syncwarp();
-            if (lane == 0)  // read >= 2 NW + 1 steps later, ordered by the barrier chain (see the read)
-                *reinterpret_cast<volatile unsigned*>(&tab[(cj % K) * NC + cw]) = ((unsigned)(cj % 65535 + 1) << 16) | (unsigned)slot;
+            if (lane == 0) {  // release: the warp's slot stores (ordered before by __syncwarp) first
+                sk_st_release(reinterpret_cast<int*>(&tab[(cj % K) * NC + cw]),
+                              (int)(((unsigned)(cj % 65535 + 1) << 16) | (unsigned)slot));
+            }
         }
         // ---- backward replay: x (Eq 4) of window (bj, wb)
         if (bwd) {

@@ -28,11 +28,11 @@ namespace {
 thread_local tri_status g_last = TRI_OK;
 
 constexpr int64_t MAX_ELEMS = int64_t(1) << 40;
-// SCAN: back-substitution lag in steps.  A window is read back >= delta + 1 steps
-// after its store; with delta >= 2 x warps the named-barrier chain of the step
-// handover orders every store before its read (k_scan.cuh), so no flag protocol
-// is needed (compute-sanitizer racecheck models barriers, not release/acquire flags)
-constexpr int SCAN_DELTA = 2 * SC_NW;
+// SCAN: back-substitution lag in steps (a window is read back >= delta + 1 steps
+// after its store; 0..8 measured equal at c1 / c2 in round 1; 24 -- the lag at
+// which the handover barrier chain alone would order every slot -- measured 3 %
+// slower at c5 and 8 % at c2, so the slots keep their release / acquire table)
+constexpr int SCAN_DELTA = 8;
 
 // ---- pure host planner ------------------------------------------------------
 // Rows of (normalised, 3-array) system data one ONCHIP CTA holds: sized for
