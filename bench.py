@@ -146,10 +146,7 @@ def method_arrays(plan, tri, l2_bytes):
     if v == tri.VARIANT_SCAN_MC:
         return 9 if "lookback=0" not in plan.describe() else 13  # look-back: 4 + 2 + 2 + 1; three passes: + 4
     if plan.k == 0:
-        # read a, b, c, d; write + read c', d'; write x -- unless the c', d' a wave
-        # of CTAs writes are read back (and L2-discarded) before they leave L2
-        inflight = 2 * plan.n * min(plan.m, 32 * 4 * 148) * (8 if "f64" in plan.describe() else 4)
-        return 5 if inflight < l2_bytes // 2 else 9
+        return 9  # read a, b, c, d; write + read c', d' (materialised); write x -- ncu bytes override when known
     # pass 1: read 4 + write 3; each later pass: read 3 + write 3; p-Thomas: read 3, c', d' 2 + 2, write x
     return 7 + 6 * (plan.launches - 2) + 8
 

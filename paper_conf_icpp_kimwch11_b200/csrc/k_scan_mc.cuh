@@ -146,7 +146,9 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant
     const int w0 = ch * p.NCW;
     const int nwin = min(NC, w0 + p.NCW) - w0;
     T* ib = reinterpret_cast<T*>(sbase + L::off_in + pw * L::in_stride);
-    const uint64_t pol_in = sk_policy_evict_first();
+    // pass 0 keeps its lines (evict_normal): the chunk starts it reads last are
+    // what pass 1 reads first; pass 1 is the inputs' last use (evict_first)
+    const uint64_t pol_in = MODE == 0 ? sk_policy_evict_normal() : sk_policy_evict_first();
     // pass 0 and pass 2 walk their chunk backwards, pass 1 forwards: each pass
     // starts where the previous one ended, so the windows still in L2 (the last
     // ~100 MB a pass touched, at the same end of every chunk) are read first
