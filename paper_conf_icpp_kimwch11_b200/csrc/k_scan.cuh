@@ -265,7 +265,7 @@ __device__ __forceinline__ void sc_fix_rows(int64_t i0, int64_t n, T (&ra)[SC_R]
 // fp32 rows are always scaled by 2^-e here (once per load; the product of 8 raw
 // fp32 rows would leave fp32's range beyond |b| ~ 2^16).
 template <typename T>
-__device__ __forceinline__ void sc_range(T (&ra)[SC_R], T (&rb)[SC_R], T (&rc)[SC_R], T (&rd)[SC_R]) {
+__device__ __forceinline__ void sc_range(T (&ra)[SC_R], T (&rb)[SC_R], T (&rc)[SC_R], T (&rd)[SC_R], int* known = nullptr) {
     if constexpr (sizeof(T) == 4) {
 #pragma unroll
         for (int u = 0; u < SC_R; ++u) {
@@ -273,13 +273,22 @@ __device__ __forceinline__ void sc_range(T (&ra)[SC_R], T (&rb)[SC_R], T (&rc)[S
             ra[u] *= s; rb[u] *= s; rc[u] *= s; rd[u] *= s;
         }
     } else {
-        bool out = false;
+        // `known`: the decision of an earlier load of the same rows (-1: not taken yet)
+        bool scale;
+        if (known && *known >= 0) {
+            scale = *known != 0;
+        } else {
+            unsigned mx = 0u, mn = 0xffffffffu;  // exponent bits of the pivots (high words)
 #pragma unroll
-        for (int u = 0; u < SC_R; ++u) {
-            const unsigned e = ((unsigned)__double2hiint(rb[u]) >> 20) & 0x7ffu;
-            out |= (e - (1023u - 64u)) > 128u;
+            for (int u = 0; u < SC_R; ++u) {
+                const unsigned hb = (unsigned)__double2hiint(rb[u]) & 0x7ff00000u;
+                mx = max(mx, hb);
+                mn = min(mn, hb);
+            }
+            scale = __any_sync(0xffffffffu, mx > ((1023u + 64u) << 20) || mn < ((1023u - 64u) << 20));
+            if (known) *known = scale ? 1 : 0;
         }
-        if (__any_sync(0xffffffffu, out)) {
+        if (scale) {
 #pragma unroll
             for (int u = 0; u < SC_R; ++u) {
                 const T s = sk_exp2_scale(rb[u]);
@@ -773,6 +782,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
             }
         };
         SCM M;
+        int scl = -1;  // fp64 row renormalisation of this window: decided once (sc_range)
         if (fwd) {
             SC_T(5);
             sk_wait(&in_full[pw], ph);
@@ -781,7 +791,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
             T ra[SC_R], rb[SC_R], rc[SC_R], rd[SC_R];
             load_rows(ra, rb, rc, rd);
             if (edge) fix_rows(ra, rb, rc, rd);
-            sc_range(ra, rb, rc, rd);
+            sc_range(ra, rb, rc, rd, &scl);
             M = sc_wide(sc_fwd_map(ra, rb, rc, rd));
         } else {
             M = SCM{1.0, 0.0, 0.0, 1.0, 0.0, 0.0, 1.0};
@@ -831,7 +841,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
             T ra[SC_R], rb[SC_R], rc[SC_R], rd[SC_R];
             load_rows(ra, rb, rc, rd);
             if (edge) fix_rows(ra, rb, rc, rd);
-            sc_range(ra, rb, rc, rd);
+            sc_range(ra, rb, rc, rd, &scl);  // the decision of the map's load of the same rows
             sc_release_buf();  // this warp's reads of the buffer before the TMA refill
             if (!SC_LATE && lane == 0 && g + SC_NW < nfwd) issue(j, w);
             T cpf[SC_R], dpf[SC_R];
