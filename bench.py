@@ -399,6 +399,30 @@ def main():
         except Exception as exc:  # never let the edge measurement cost the solve numbers
             coll = {"error": repr(exc)[:300]}
 
+    # ---- the copy bandwidth of this GPU in this run (re-measure the
+    # denominator in the same session; the roofline keeps MEASURED_PEAKS.json's)
+    copy_gbs = None
+    if rank == 0:
+        try:
+            src = torch.empty(1 << 30, dtype=torch.uint8, device=dev)
+            dst = torch.empty_like(src)
+            for _ in range(2):
+                dst.copy_(src)
+            best = None
+            for _ in range(5):
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record()
+                dst.copy_(src)
+                e1.record()
+                torch.cuda.synchronize()
+                t = e0.elapsed_time(e1)
+                best = t if best is None else min(best, t)
+            copy_gbs = 2 * src.numel() / (best * 1e-3) / 1e9
+            del src, dst
+            torch.cuda.empty_cache()
+        except Exception:  # never let the side measurement cost the line
+            copy_gbs = None
+
     # ---- CPU oracle baseline (rank 0 at N=1 only)
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu:
@@ -441,6 +465,7 @@ def main():
                    "plan": plan.describe()},
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                      "traffic": traffic, "traffic_source": traffic_src, "peak_source": peak_src,
+                     "copy_gbs_same_run": copy_gbs,
                      "algorithmic_bytes_per_launch": algo_bytes,
                      "method_arrays": method_bytes / (n_unknowns * s), "method_source": method_src,
                      "method_bytes_per_launch": method_bytes,

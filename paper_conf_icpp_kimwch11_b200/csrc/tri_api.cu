@@ -104,6 +104,8 @@ bool scan_mc_ok(int64_t n, int64_t m, tri_dtype t, tri_layout layout) {
 // every other stride a 16-byte multiple; else the packed fallback (l_strided.cu)
 bool strided_fast(int64_t n, int64_t ms, int64_t nb, tri_dtype t, int64_t es, int64_t ss, int64_t bs) {
     const int64_t sz = (int64_t)esize(t);
+    const int64_t tma_stride = int64_t(1) << 40;  // a tensor map's byte strides must stay below 2^40
+    if (es * sz >= tma_stride || ss * sz >= tma_stride || bs * sz >= tma_stride) return false;
     const bool bok = nb == 1 || (bs * sz) % 16 == 0;
     if (es == 1 && n % 8 == 0 && (ms == 1 || (ss * sz) % 16 == 0) && bok && cdiv(n, SC_W) <= SC_NCMAX &&
         n / 8 < ((int64_t)1 << 31) && ms < ((int64_t)1 << 31) && nb < ((int64_t)1 << 31))
@@ -523,14 +525,15 @@ tri_plan_t tri_plan_batched(int64_t n, int64_t ms, int64_t nb, tri_dtype dtype) 
 
 tri_plan_t tri_plan_strided(int64_t n, int64_t ms, int64_t nb, tri_dtype dtype, int64_t es, int64_t ss,
                             int64_t bs) {
+    // strides >= 1 and every offset (n-1) es + (ms-1) ss + (nb-1) bs below 2^52 elements
+    // (no int64 overflow anywhere in the index arithmetic); that the (q, i) map to
+    // distinct elements is the caller's contract
+    constexpr int64_t LIM = int64_t(1) << 50;
     if (n < 1 || ms < 1 || nb < 1 || (dtype != TRI_F32 && dtype != TRI_F64) || ms > MAX_ELEMS / nb ||
-        n > MAX_ELEMS / (ms * nb) || es < 1 || ss < 1 || bs < 1) {
+        n > MAX_ELEMS / (ms * nb) || es < 1 || ss < 1 || bs < 1 || es > LIM / n || ss > LIM / ms || bs > LIM / nb) {
         g_last = TRI_ERR_INVALID_ARG;
         return nullptr;
     }
-    // distinct elements: a row / system / batch step must move past the other two
-    // dimensions' extents in at least the order the caller nests them -- the
-    // footprint check is the caller's; here only positive strides are required
     int dev = 0, sms = 0;
     tri_status st = current_device_ok(&dev, &sms);
     if (st != TRI_OK) { g_last = st; return nullptr; }

@@ -70,6 +70,13 @@ def test_plan_without_gpu_fails_cleanly(L):
     assert L.tri_last_status() == 1
     assert not L.tri_plan(16, 4, tri.F64, 9)
     assert L.tri_last_status() == 1
+    assert not L.tri_plan_strided(64, 4, 2, tri.F64, 1, 64, 256)
+    assert L.tri_last_status() == 4  # TRI_ERR_DEVICE (valid arguments, no GPU)
+    for bad in [(64, 4, 2, tri.F64, 0, 64, 256), (64, 4, 2, tri.F64, 1, -1, 256), (0, 4, 2, tri.F64, 1, 64, 256),
+                (64, 4, 2, 5, 1, 64, 256), (64, 4, 2, tri.F64, 1 << 50, 64, 256)]:
+        assert not L.tri_plan_strided(*bad)
+        assert L.tri_last_status() == 1, bad  # TRI_ERR_INVALID_ARG
+    assert L.tri_plan_set_option(None, 1, 0) == 1
     assert L.tri_plan_k(None) == -1
     L.tri_destroy(None)  # NULL-safe
     with pytest.raises(tri.TriError):
