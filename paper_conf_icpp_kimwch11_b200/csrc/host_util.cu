@@ -46,19 +46,26 @@ bool tma_encode(CUtensorMap* tm, size_t es, int rank, const void* base, const ui
 }
 
 bool tm_lookup(tri_plan_s* p, int tag, const void* const* key, int nkey, CUtensorMap* maps, int nmaps) {
-    TmCache& c = p->tmc;
-    if (!c.valid || c.tag != tag || nkey > TM_MAX || nmaps > TM_MAX) return false;
-    for (int i = 0; i < nkey; ++i)
-        if (c.key[i] != key[i]) return false;
-    for (int i = nkey; i < TM_MAX; ++i)
-        if (c.key[i] != nullptr) return false;
-    std::memcpy(maps, c.maps, sizeof(CUtensorMap) * nmaps);
-    return true;
+    if (nkey > TM_MAX || nmaps > TM_MAX) return false;
+    for (const TmEntry& c : p->tmc.e) {
+        if (!c.valid || c.tag != tag) continue;
+        bool same = true;
+        for (int i = 0; i < TM_MAX && same; ++i) same = c.key[i] == (i < nkey ? key[i] : nullptr);
+        if (!same) continue;
+        std::memcpy(maps, c.maps, sizeof(CUtensorMap) * nmaps);
+        return true;
+    }
+    return false;
 }
 
 void tm_store(tri_plan_s* p, int tag, const void* const* key, int nkey, const CUtensorMap* maps, int nmaps) {
-    TmCache& c = p->tmc;
-    if (nkey > TM_MAX || nmaps > TM_MAX) { c.valid = false; return; }
+    if (nkey > TM_MAX || nmaps > TM_MAX) return;
+    // the entry of the same launcher (tag) is replaced; otherwise the round-robin victim
+    int v = -1;
+    for (int i = 0; i < TM_ENT && v < 0; ++i)
+        if (p->tmc.e[i].valid && p->tmc.e[i].tag == tag) v = i;
+    if (v < 0) { v = p->tmc.next; p->tmc.next = (v + 1) % TM_ENT; }
+    TmEntry& c = p->tmc.e[v];
     for (int i = 0; i < TM_MAX; ++i) c.key[i] = i < nkey ? key[i] : nullptr;
     std::memcpy(c.maps, maps, sizeof(CUtensorMap) * nmaps);
     c.tag = tag;

@@ -4,16 +4,23 @@
 // system chain-interleaved (the interleave transform fused into the last store,
 // P:647), then p-Thomas with one thread per subsystem (Sec. III.B).
 //
-// Any 0 <= k <= floor(log2 n): pass 1 applies up to 10 steps on
-// the user layout; every further pass applies up to 5 more steps to the
-// chain-interleaved batch the previous pass wrote (strides 2^K.. of the
-// original system are strides 1.. of each chain), ping-ponging between two
-// scratch buffers; the last pass writes the p-Thomas input.
+// Any 0 <= k <= floor(log2 n).  Pass 1 works on the user layout,
+// every further pass on the chain-interleaved batch the previous pass wrote
+// (strides 2^K.. of the original system are strides 1.. of each chain),
+// ping-ponging between two scratch buffers; the last pass writes the p-Thomas
+// input.  Two kernel families (PassKind):
+//   register tiles (k_pcr_reg.cuh, TMA-fed, the default): pass 1 up to 5 steps
+//     on CONTIGUOUS rows (3 on the user's INTERLEAVED rows), later passes up to 3
+//     steps each, the remaining steps balanced over the fewest passes;
+//   the paper's shared-memory sliding window (k_tiled_pcr.cuh): pass 1 up to 10
+//     steps, later passes up to 5 -- with TRI_OPT_TMA off, the BATCHED layout,
+//     and shapes the TMA maps cannot describe.
 #include <algorithm>
 
 #include "plan.cuh"
 #include "common.cuh"
 #include "k_tiled_pcr.cuh"
+#include "k_pcr_reg.cuh"
 #include "k_pthomas.cuh"
 #include "k_pthomas_tma.cuh"
 
@@ -156,10 +163,96 @@ cudaError_t launch_pass(const tri_plan_s* p, int i, const void* iA, const void* 
     }
 }
 
+// ---- register-tile passes (k_pcr_reg.cuh) --------------------------------------
+template <typename T, int K>
+cudaError_t launch_rows_k(const PRArgs<T>& A, int sms, cudaStream_t st) {
+    int occ = 1;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_pcr_rows<T, K>, 32 * PR_WARPS, 0) != cudaSuccess) {
+        cudaGetLastError();
+        occ = 1;
+    }
+    const int64_t grid = std::max<int64_t>(1, std::min<int64_t>(cdiv(A.ntask, PR_WARPS), (int64_t)std::max(1, occ) * sms));
+    k_pcr_rows<T, K><<<(unsigned)grid, 32 * PR_WARPS, 0, st>>>(A);
+    return cudaGetLastError();
+}
+
+// pass 0 on CONTIGUOUS rows
+template <typename T>
+cudaError_t launch_rows(tri_plan_s* p, const void* a, const void* b, const void* c, const void* d, void* oA, void* oC,
+                        void* oD, int mode, cudaStream_t st) {
+    const int K = p->kp[0];
+    PRArgs<T> A;
+    A.a = (const T*)a; A.b = (const T*)b; A.c = (const T*)c; A.d = (const T*)d;
+    A.oA = (T*)oA; A.oC = (T*)oC; A.oD = (T*)oD;
+    A.n = p->n; A.m = p->m; A.n_pad = p->Lp[0] << K;
+    A.ntile = p->region[0]; A.ntask = p->m * p->region[0];
+    A.C = p->Cp[0]; A.mode = mode;
+    A.vec = (((uintptr_t)a | (uintptr_t)b | (uintptr_t)c | (uintptr_t)d) & 31) == 0;
+    switch (K) {
+        case 1: return launch_rows_k<T, 1>(A, p->sms, st);
+        case 2: return launch_rows_k<T, 2>(A, p->sms, st);
+        case 3: return launch_rows_k<T, 3>(A, p->sms, st);
+        case 4: return launch_rows_k<T, 4>(A, p->sms, st);
+        case 5: return launch_rows_k<T, 5>(A, p->sms, st);
+        default: return cudaErrorInvalidValue;
+    }
+}
+
+template <typename T, bool RAW>
+int chains_ctas(const tri_plan_s* p) {
+    const int occ = std::max(1, (227 * 1024) / PCCfg<T, RAW>::smem_bytes());
+    return occ * p->sms;
+}
+
+template <typename T, int K, bool RAW>
+cudaError_t launch_chains_k(const PCMaps& tm, const PCArgs<T>& A, int grid, cudaStream_t st) {
+    constexpr int smem = PCCfg<T, RAW>::smem_bytes();
+    cudaError_t e = set_smem((const void*)k_pcr_chains<T, K, RAW>, smem);
+    if (e != cudaSuccess) return e;
+    k_pcr_chains<T, K, RAW><<<grid, 32 * PCCfg<T, RAW>::WARPS, smem, st>>>(tm, A);
+    return cudaGetLastError();
+}
+
+// pass i on a chain-interleaved batch (the previous pass's output, or -- RAW, pass
+// 0 -- the user's INTERLEAVED arrays a, b, c, d)
+template <typename T, bool RAW>
+cudaError_t launch_chains(tri_plan_s* p, int i, const void* in0, const void* in1, const void* in2, const void* in3,
+                          void* oA, void* oC, void* oD, int mode, cudaStream_t st) {
+    const int K = p->kp[i];
+    const int64_t C1 = i == 0 ? p->m : p->Cp[i - 1], L1 = i == 0 ? p->n : p->Lp[i - 1];
+    PCMaps tm;
+    const void* key[4] = {in0, in1, in2, in3};
+    const int nk = RAW ? 4 : 3;
+    const int tag = 0x7200 + 16 * i + (int)sizeof(T);
+    if (!tm_lookup(p, tag, key, nk, &tm.a, nk)) {
+        const uint64_t dims[2] = {(uint64_t)C1, (uint64_t)L1}, str[1] = {(uint64_t)C1 * sizeof(T)};
+        const uint32_t box[2] = {32u, (uint32_t)PC_PO};
+        CUtensorMap* dst[4] = {&tm.a, &tm.c, &tm.d, &tm.b};
+        for (int j = 0; j < nk; ++j)
+            if (!tma_encode(dst[j], sizeof(T), 2, key[j], dims, str, box, CU_TENSOR_MAP_SWIZZLE_NONE))
+                return cudaErrorNotSupported;
+        tm_store(p, tag, key, nk, &tm.a, nk);
+    }
+    PCArgs<T> A;
+    A.oA = (T*)oA; A.oC = (T*)oC; A.oD = (T*)oD;
+    A.n = p->n; A.m = p->m; A.L1 = L1; A.C1 = C1; A.C = p->Cp[i];
+    A.Lout = p->Lp[i] << K;
+    A.ntile_reg = p->region[i]; A.nreg = p->nreg[i]; A.nblk = p->nblk[i]; A.ntask = p->nreg[i] * p->nblk[i];
+    A.k1 = i == 0 ? 0 : ksum(p, i - 1); A.mode = mode; A.layout = p->layout;
+    const int grid = (int)std::max<int64_t>(
+        1, std::min<int64_t>(cdiv(A.ntask, PCCfg<T, RAW>::WARPS), chains_ctas<T, RAW>(p)));
+    switch (K) {
+        case 1: return launch_chains_k<T, 1, RAW>(tm, A, grid, st);
+        case 2: return launch_chains_k<T, 2, RAW>(tm, A, grid, st);
+        case 3: return launch_chains_k<T, 3, RAW>(tm, A, grid, st);
+        default: return cudaErrorInvalidValue;
+    }
+}
+
 // all PCR passes; the last one writes (fA, fC, fD) in `mode` (0: chain-
 // interleaved p-Thomas input, 1: the user layout for tri_debug_pcr)
 template <typename T>
-cudaError_t run_passes(const tri_plan_s* p, const void* a, const void* b, const void* c, const void* d, void* fA,
+cudaError_t run_passes(tri_plan_s* p, const void* a, const void* b, const void* c, const void* d, void* fA,
                        void* fC, void* fD, int mode, cudaStream_t st) {
     const size_t ce = (size_t)p->C * (size_t)p->L;
     const size_t ie = (size_t)inter_elems(p);
@@ -173,8 +266,14 @@ cudaError_t run_passes(const tri_plan_s* p, const void* a, const void* b, const 
         void* oC = last ? fC : (void*)(o + ie);
         void* oD = last ? fD : (void*)(o + 2 * ie);
         const int md = last ? mode : 0;
-        cudaError_t e = i == 0 ? launch_pass0<T>(p, a, b, c, d, oA, oC, oD, md, st)
-                               : launch_pass<T>(p, i, in[0], in[1], in[2], oA, oC, oD, md, st);
+        cudaError_t e;
+        switch (p->pk[i]) {
+            case PK_ROWS: e = launch_rows<T>(p, a, b, c, d, oA, oC, oD, md, st); break;
+            case PK_RAW: e = launch_chains<T, true>(p, i, a, c, d, b, oA, oC, oD, md, st); break;
+            case PK_CHAINS: e = launch_chains<T, false>(p, i, in[0], in[1], in[2], nullptr, oA, oC, oD, md, st); break;
+            case PK_RING: e = launch_pass0<T>(p, a, b, c, d, oA, oC, oD, md, st); break;
+            default: e = launch_pass<T>(p, i, in[0], in[1], in[2], oA, oC, oD, md, st); break;
+        }
         if (e != cudaSuccess) return e;
         in[0] = oA; in[1] = oC; in[2] = oD;
     }
@@ -323,6 +422,15 @@ cudaError_t split_t(tri_plan_s* p, const void* a, const void* b, const void* c, 
 
 }  // namespace
 
+// register-tile passes: can the TMA maps describe pass 1's input / a batch of C1 chains?
+bool rows_ok(const tri_plan_s* p) {
+    return p->opt_tma && p->layout == TRI_LAYOUT_CONTIGUOUS;
+}
+bool chains_ok(const tri_plan_s* p, int64_t C1, int64_t L1) {
+    return p->opt_tma && (C1 * (int64_t)esize(p->dtype)) % 16 == 0 && C1 < INT32_MAX &&
+           L1 + 4 * PC_PO + 64 < INT32_MAX;
+}
+
 void split_geometry(tri_plan_s* p) {
     const int64_t n = p->n, m = p->m;
     const int S = 1 << p->k;
@@ -330,27 +438,73 @@ void split_geometry(tri_plan_s* p) {
     p->n_pad = p->L * S;
     p->C = m * S;
     p->npass = 0;
-    for (int i = 0; i < 8; ++i) { p->kp[i] = 0; p->Lp[i] = p->Cp[i] = p->region[i] = p->nreg[i] = p->nblk[i] = 0; }
-    if (p->k == 0) return;
-    // pass 1 up to 10 steps; two passes split as (k - 5, 5) beyond that; deeper k
-    // adds passes of 5 steps
-    int rem = p->k;
-    int k1 = std::min(rem, SPLIT_K1MAX);
-    if (rem > SPLIT_K1MAX && rem <= SPLIT_K1MAX + SPLIT_KNMAX && rem - k1 > SPLIT_KNMAX) k1 = rem - SPLIT_KNMAX;
-    p->kp[p->npass++] = k1;
-    rem -= k1;
-    while (rem > 0) {
-        const int kk = std::min(rem, SPLIT_KNMAX);
-        p->kp[p->npass++] = kk;
-        rem -= kk;
+    for (int i = 0; i < 8; ++i) {
+        p->kp[i] = p->pk[i] = 0;
+        p->Lp[i] = p->Cp[i] = p->region[i] = p->nreg[i] = p->nblk[i] = 0;
     }
+    if (p->k == 0) return;
     const bool f64 = p->dtype == TRI_F64;
+    int rem = p->k;
+    if (rows_ok(p) || (p->layout == TRI_LAYOUT_INTERLEAVED && chains_ok(p, m, n))) {
+        // register tiles: pass 1 up to 5 (rows) / 3 (interleaved) steps, then the
+        // remaining steps over the fewest passes of <= 3, balanced
+        const bool rows = rows_ok(p);
+        const int k1 = std::min(rem, rows ? 5 : 3);
+        p->kp[0] = k1;
+        p->pk[0] = rows ? PK_ROWS : PK_RAW;
+        p->npass = 1;
+        rem -= k1;
+        const int np = (int)cdiv(rem, 3);
+        for (int j = 0; j < np; ++j) {
+            p->kp[p->npass] = rem / np + (j < rem % np ? 1 : 0);
+            p->pk[p->npass] = PK_CHAINS;
+            ++p->npass;
+        }
+    } else {
+        // sliding window: pass 1 up to 10 steps; two passes split as (k - 5, 5)
+        // beyond that; deeper k adds passes of 5 steps
+        int k1 = std::min(rem, SPLIT_K1MAX);
+        if (rem > SPLIT_K1MAX && rem <= SPLIT_K1MAX + SPLIT_KNMAX && rem - k1 > SPLIT_KNMAX) k1 = rem - SPLIT_KNMAX;
+        p->kp[0] = k1;
+        p->pk[0] = PK_RING;
+        p->npass = 1;
+        rem -= k1;
+        while (rem > 0) {
+            const int kk = std::min(rem, SPLIT_KNMAX);
+            p->pk[p->npass] = PK_IL;
+            p->kp[p->npass++] = kk;
+            rem -= kk;
+        }
+    }
     int K = 0;
     for (int i = 0; i < p->npass; ++i) {
         K += p->kp[i];
         p->Lp[i] = cdiv(n, int64_t(1) << K);
         p->Cp[i] = m << K;
-        if (i == 0) {
+        const int64_t C1 = i == 0 ? m : p->Cp[i - 1], L1 = i == 0 ? n : p->Lp[i - 1];
+        if (p->pk[i] == PK_CHAINS && !chains_ok(p, C1, L1)) p->pk[i] = PK_IL;  // K <= 3 <= 5
+        if (p->pk[i] == PK_ROWS) {
+            // tiles of OUT rows cover the L 2^K rows pass 1 writes per system (from
+            // up to 3 (fp64) / 7 (fp32) rows before row 0: 32-byte aligned lane rows)
+            const int h = ((1 << p->kp[0]) - 1 + 7) / 8 * 8;
+            p->region[0] = cdiv((p->Lp[0] << p->kp[0]) + 32 / (int64_t)esize(p->dtype) - 1, PR_ROWS - 2 * h);
+            p->nreg[0] = 1;
+            p->nblk[0] = m;
+        } else if (p->pk[i] == PK_CHAINS || p->pk[i] == PK_RAW) {
+            // tasks = (32-chain block, region of tiles): about two per resident warp,
+            // regions of >= 16 tiles (the two halo tiles stay a small fraction)
+            const int64_t ntile = cdiv(p->Lp[i] << p->kp[i], PC_PO);
+            const bool raw = p->pk[i] == PK_RAW;
+            const int64_t warps = (int64_t)(raw ? (f64 ? chains_ctas<double, true>(p) * PCCfg<double, true>::WARPS
+                                                       : chains_ctas<float, true>(p) * PCCfg<float, true>::WARPS)
+                                                : (f64 ? chains_ctas<double, false>(p) * PCCfg<double, false>::WARPS
+                                                       : chains_ctas<float, false>(p) * PCCfg<float, false>::WARPS));
+            p->nblk[i] = cdiv(C1, 32);
+            int64_t nreg = std::max<int64_t>(1, cdiv(2 * warps, p->nblk[i]));
+            nreg = std::max<int64_t>(1, std::min<int64_t>(nreg, ntile / 16));
+            p->region[i] = cdiv(ntile, nreg);
+            p->nreg[i] = cdiv(ntile, p->region[i]);
+        } else if (i == 0) {
             const int occ = f64 ? tiled_occ<double>(p->kp[0]) : tiled_occ<float>(p->kp[0]);
             const int64_t target = (int64_t)occ * p->sms * TILED_WAVES1;
             const int64_t n_pad1 = p->Lp[0] << p->kp[0];
@@ -363,8 +517,7 @@ void split_geometry(tri_plan_s* p) {
             p->nblk[0] = m;
         } else {  // over the Cp[i-1] chains, TPCR_IL_CB per CTA
             const int k2 = p->kp[i];
-            const int64_t L1 = p->Lp[i - 1];
-            p->nblk[i] = cdiv(p->Cp[i - 1], TPCR_IL_CB);
+            p->nblk[i] = cdiv(C1, TPCR_IL_CB);
             const int occ2 = f64 ? tiled_il_occ<double>(k2) : tiled_il_occ<float>(k2);
             int64_t nreg2 = std::max<int64_t>(1, cdiv((int64_t)occ2 * p->sms * TILED_WAVES2, p->nblk[i]));
             const int64_t minreg2 = 4 * halo_f(k2) + TPCR_IL_TP;

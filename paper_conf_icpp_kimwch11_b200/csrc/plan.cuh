@@ -16,17 +16,25 @@
 namespace trih {
 
 constexpr int HOST_CHUNKS = 16;  // tri_solve_host pipeline depth (chunks of systems)
-constexpr int TM_MAX = 8;        // tensor maps cached per plan
+constexpr int TM_MAX = 8;        // tensor maps per cache entry
+constexpr int TM_ENT = 6;        // cache entries per plan (one per launch of a multi-kernel solve)
 
-// Tensor maps of the last pointer set a launcher saw (tri_solve then does no
+// Tensor maps of the last pointer sets the launchers saw (tri_solve then does no
 // cuTensorMapEncode work when the caller reuses its buffers, as bench.py and a
 // time-stepping ADI code do).  `tag` names the launcher (and its geometry);
-// any plan change (k, variant, option) clears `valid`.
-struct TmCache {
+// any plan change (k, variant, option) clears the cache.
+struct TmEntry {
     bool valid = false;
     int tag = 0;
     const void* key[TM_MAX] = {};
     alignas(64) CUtensorMap maps[TM_MAX];
+};
+struct TmCache {
+    TmEntry e[TM_ENT];
+    int next = 0;  // round-robin victim
+    void clear() {
+        for (auto& x : e) x.valid = false;
+    }
 };
 
 }  // namespace trih
@@ -45,8 +53,11 @@ struct tri_plan_s {
     int64_t n_pad = 0, L = 0, C = 0;  // SPLIT: chain length, chains
     int npass = 0;                // SPLIT: tiled-PCR passes (0 at k = 0)
     int kp[8] = {};               // SPLIT: PCR steps of each pass
+    int pk[8] = {};               // SPLIT: kernel of each pass (trih::PassKind)
     int64_t Lp[8] = {}, Cp[8] = {};   // SPLIT: positions per chain, chains AFTER pass i
-    int64_t region[8] = {}, nreg[8] = {}, nblk[8] = {};  // SPLIT: regions per chain block, chain blocks of pass i
+    // SPLIT: region length (rows / positions; tiles for the register kernels), regions per
+    // system or chain block, chain blocks of pass i
+    int64_t region[8] = {}, nreg[8] = {}, nblk[8] = {};
     int fu_grid = 0, fu_son = 0;  // FUSED: persistent CTAs, on-chip positions per chain
     bool fu_vec = false;          // FUSED: staged 8-row-aligned path
     int64_t fu_nc = 0;            // FUSED: windows per system
@@ -79,6 +90,12 @@ struct tri_plan_s {
 };
 
 namespace trih {
+
+// SPLIT pass kernels: the shared-memory sliding window of the paper (first pass
+// on the user layout, later passes on chain-interleaved batches), or the
+// register-resident tiles (k_pcr_reg.cuh: rows of the CONTIGUOUS layout, chains
+// of a chain-interleaved batch, the user's INTERLEAVED rows)
+enum PassKind { PK_RING = 0, PK_IL = 1, PK_ROWS = 2, PK_CHAINS = 3, PK_RAW = 4 };
 
 inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
 inline size_t esize(tri_dtype t) { return t == TRI_F64 ? 8 : 4; }

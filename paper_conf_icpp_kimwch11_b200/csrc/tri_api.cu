@@ -209,7 +209,7 @@ int kmin_for(tri_variant v) {
 // ---- per-plan geometry -----------------------------------------------------
 void plan_geometry(tri_plan_s* p) {
     const int64_t n = p->n, m = p->m;
-    p->tmc.valid = false;
+    p->tmc.clear();
     if (p->variant == TRI_VARIANT_WARP) {
         int R = 1;
         while (32 * (int64_t)R < n) R *= 2;
@@ -632,9 +632,12 @@ tri_status tri_plan_set_option(tri_plan_t p, tri_option opt, int value) {
     if (p->layout == TRI_LAYOUT_STRIDED) return p->inner ? tri_plan_set_option(p->inner, opt, value) : TRI_ERR_INVALID_ARG;
     if (opt == TRI_OPT_TMA) {
         if (value != 0 && value != 1) return TRI_ERR_INVALID_ARG;
+        const int old = p->opt_tma;
         p->opt_tma = value;
-        p->tmc.valid = false;
-        return TRI_OK;
+        // the SPLIT pass structure (and so its scratch) depends on the TMA kernels
+        const tri_status st = set_plan(p, p->variant, p->k);
+        if (st != TRI_OK) { p->opt_tma = old; plan_geometry(p); }
+        return st;
     }
     if (opt == TRI_OPT_SCAN_MC_LOOKBACK) {
         if (value < -1 || value > LB_MAXW) return TRI_ERR_INVALID_ARG;

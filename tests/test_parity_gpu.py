@@ -57,17 +57,41 @@ def test_onchip_every_k(cuda_ok, dtype, layout, n, m):
         check_parity(n, m, arrs, x, dtype, layout, x_oracle=xo)
 
 
+def split_launches(n, m, k, layout, dtype, tma=True):
+    """tri_plan_launches of a SPLIT plan (l_split.cu split_geometry): p-Thomas plus
+    the tiled-PCR passes -- register tiles (5 steps on CONTIGUOUS rows, 3 on
+    INTERLEAVED rows whose row pitch m s is a 16-byte multiple, then passes of
+    <= 3), else the sliding window (10 steps, then passes of <= 5)."""
+    if k == 0:
+        return 1
+    es = 8 if dtype == "f64" else 4
+    if tma and layout == 0:
+        return 2 + -(-max(0, k - 5) // 3)
+    if tma and layout == 1 and (m * es) % 16 == 0:
+        return 2 + -(-max(0, k - 3) // 3)
+    return 2 + (0 if k <= 10 else -(-(k - 10) // 5))
+
+
 @pytest.mark.parametrize("dtype", ["f64", "f32"])
 @pytest.mark.parametrize("layout", [0, 1])
-@pytest.mark.parametrize("n,m", [(10007, 3), (4099, 1), (70001, 1)])
+@pytest.mark.parametrize("n,m", [(10007, 3), (4099, 1), (70001, 1), (10007, 4), (3001, 40), (1 << 12, 64)])
 def test_split_every_k(cuda_ok, dtype, layout, n, m):
+    """Every k through both tiled-PCR kernel families (register tiles by
+    default, the paper's shared-memory sliding window with TRI_OPT_TMA off):
+    ragged n, m = 1 .. 64, chain blocks with idle lanes (m = 3, 40)."""
     arrs = gen(n, m, dtype, layout, "weak", eps=1e-2)
     xo = oracle.solve_batch(n, m, *arrs, layout=layout)
-    plan = None
-    for k in range(0, min(int(np.log2(n)), 15) + 1):  # k > 10: two tiled-PCR passes
-        x, plan = gpu_solve(n, m, arrs, dtype, layout, k=k, variant=SPLIT, plan=plan)
-        assert plan.launches == (1 if k == 0 else 2 if k <= 10 else 3)
-        check_parity(n, m, arrs, x, dtype, layout, x_oracle=xo)
+    dev = to_dev(*arrs)
+    kmax = min(int(np.log2(n)), 15)
+    for tma in (1, 0):
+        plan = tri.Plan(n, m, tri.F64 if dtype == "f64" else tri.F32, layout)
+        plan.set_option(tri.OPT_TMA, tma)
+        plan.variant = SPLIT
+        for k in range(0, kmax + 1):
+            plan.k = k
+            assert plan.launches == split_launches(n, m, k, layout, dtype, bool(tma)), (k, plan.describe())
+            x = plan.solve(*dev).cpu().numpy()
+            check_parity(n, m, arrs, x, dtype, layout, x_oracle=xo)
 
 
 def test_split_on_small_systems(cuda_ok):
@@ -80,22 +104,27 @@ def test_split_on_small_systems(cuda_ok):
 
 
 # ------------------------------------------------------------------ PCR stage (row A2)
-@pytest.mark.parametrize("variant,n,m,k", [(ONCHIP, 1024, 3, 3), (ONCHIP, 500, 2, 5), (SPLIT, 9000, 2, 4),
-                                           (WARP, 1000, 3, 5), (WARP, 33, 2, 5), (WARP, 256, 4, 5),
-                                           (SPLIT, 70001, 1, 13), (SPLIT, 20001, 2, 12), (SPLIT, 40000, 3, 15),
-                                           (SPLIT, 20001, 1, 8), (SPLIT, 5000, 3, 1)])
-def test_pcr_stage_matches_oracle(cuda_ok, variant, n, m, k):
+@pytest.mark.parametrize("variant,n,m,k,layout,tma", [
+    (ONCHIP, 1024, 3, 3, 0, 1), (ONCHIP, 500, 2, 5, 0, 1), (SPLIT, 9000, 2, 4, 0, 1), (WARP, 1000, 3, 5, 0, 1),
+    (WARP, 33, 2, 5, 0, 1), (WARP, 256, 4, 5, 0, 1), (SPLIT, 70001, 1, 13, 0, 1), (SPLIT, 20001, 2, 12, 0, 1),
+    (SPLIT, 40000, 3, 15, 0, 1), (SPLIT, 20001, 1, 8, 0, 1), (SPLIT, 5000, 3, 1, 0, 1), (SPLIT, 9000, 2, 5, 0, 1),
+    (SPLIT, 3001, 40, 7, 0, 1), (SPLIT, 3001, 4, 6, 1, 1), (SPLIT, 3001, 40, 9, 1, 1), (SPLIT, 4001, 4, 2, 1, 1),
+    (SPLIT, 70001, 1, 13, 0, 0),
+])
+def test_pcr_stage_matches_oracle(cuda_ok, variant, n, m, k, layout, tma):
     """The reduced system after k PCR steps (Eqs 5-6) vs the oracle's plain PCR,
-    normalised to unit diagonal, and satisfied by the oracle solution."""
-    arrs = gen(n, m, "f64", 0, "weak", eps=1e-2)
-    plan = tri.Plan(n, m, tri.F64, 0)
+    normalised to unit diagonal, and satisfied by the oracle solution (both
+    tiled-PCR kernel families, both layouts)."""
+    arrs = gen(n, m, "f64", layout, "weak", eps=1e-2)
+    plan = tri.Plan(n, m, tri.F64, layout)
+    plan.set_option(tri.OPT_TMA, tma)
     plan.variant = variant
     plan.k = k
     A, C, D = (t.cpu().numpy() for t in plan.debug_pcr(*to_dev(*arrs)))
-    xo = oracle.solve_batch(n, m, *arrs)
+    xo = oracle.solve_batch(n, m, *arrs, layout=layout)
     s = 1 << k
     for q in range(m):
-        sl = slice(q * n, (q + 1) * n)
+        sl = slice(q * n, (q + 1) * n) if layout == 0 else slice(q, None, m)
         ao, bo, co, do = oracle.pcr_k(*(t[sl] for t in arrs), k)
         An, Cn, Dn = ao / bo, co / bo, do / bo
         for got, ref in ((A[sl], An), (C[sl], Cn), (D[sl], Dn)):
