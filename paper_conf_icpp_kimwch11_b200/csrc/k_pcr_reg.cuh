@@ -229,6 +229,7 @@ struct PCCfg {
 
 template <typename T>
 struct PCArgs {
+    const T* in[4];        // cp.async path: A, C, D (RAW: a, c, d, b) -- the arrays the maps describe
     T *oA, *oC, *oD;       // mode 0: chain-interleaved [pos2 * C + ch2]; mode 1: user layout
     int64_t n, m;          // original system size, systems
     int64_t L1, C1;        // input positions per chain, input chains
@@ -257,7 +258,11 @@ __device__ __forceinline__ void pc_levels(NRow<T> (&R)[E]) {
     }
 }
 
-template <typename T, int K, bool RAW>
+// TMA: one 2D box per array per tile, lane 0 issues, an mbarrier per ring slot
+// (needs a 16-byte row pitch C1 sizeof(T)); otherwise every lane copies its own
+// chain's elements with cp.async (zero fill outside the batch), one commit group
+// per tile -- each lane reads only what it copied, so no cross-lane handshake.
+template <typename T, int K, bool RAW, bool TMA>
 __global__ void __launch_bounds__(32 * PCCfg<T, RAW>::WARPS, 1) k_pcr_chains(const __grid_constant__ PCMaps tm,
                                                                              PCArgs<T> p) {
     using CF = PCCfg<T, RAW>;
@@ -271,7 +276,7 @@ __global__ void __launch_bounds__(32 * PCCfg<T, RAW>::WARPS, 1) k_pcr_chains(con
     const int64_t TW = (int64_t)gridDim.x * NW;
     const int k = p.k1 + K;
 
-    if (lane == 0) {
+    if (TMA && lane == 0) {
         for (int s = 0; s < PC_NS; ++s) ptt_bar_init(&bar[warp][s]);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
@@ -290,24 +295,52 @@ __global__ void __launch_bounds__(32 * PCCfg<T, RAW>::WARPS, 1) k_pcr_chains(con
             const uint32_t gl = g + (uint32_t)l;
             const int s = (int)(gl % PC_NS);
             T* dst = ring + s * STAGE;
-            const int y0 = (int)((tb - 1 + l) * PO);
-            ptt_expect(&bar[warp][s], (unsigned)(STAGE * sizeof(T)));
-            ptt_load(dst, &tm.a, x0, y0, &bar[warp][s]);
-            ptt_load(dst + TILE, &tm.c, x0, y0, &bar[warp][s]);
-            ptt_load(dst + 2 * TILE, &tm.d, x0, y0, &bar[warp][s]);
-            if constexpr (RAW) ptt_load(dst + 3 * TILE, &tm.b, x0, y0, &bar[warp][s]);
+            const int64_t y0 = (tb - 1 + l) * PO;
+            if constexpr (TMA) {
+                if (lane == 0) {
+                    ptt_expect(&bar[warp][s], (unsigned)(STAGE * sizeof(T)));
+                    ptt_load(dst, &tm.a, x0, (int)y0, &bar[warp][s]);
+                    ptt_load(dst + TILE, &tm.c, x0, (int)y0, &bar[warp][s]);
+                    ptt_load(dst + 2 * TILE, &tm.d, x0, (int)y0, &bar[warp][s]);
+                    if constexpr (RAW) ptt_load(dst + 3 * TILE, &tm.b, x0, (int)y0, &bar[warp][s]);
+                }
+            } else {
+#pragma unroll
+                for (int u = 0; u < PO; ++u) {
+                    const int64_t pos = y0 + u;
+                    const bool ok = chok && pos >= 0 && pos < p.L1;
+                    const int64_t gi = ok ? pos * p.C1 + ch : 0;
+#pragma unroll
+                    for (int j = 0; j < CF::NA; ++j) {
+                        if constexpr (sizeof(T) == 8)
+                            cp_async_8(dst + j * TILE + u * 32 + lane, p.in[j] + gi, ok ? 8 : 0);
+                        else
+                            cp_async_4(dst + j * TILE + u * 32 + lane, p.in[j] + gi, ok ? 4 : 0);
+                    }
+                }
+                cp_async_commit();
+            }
         };
-        auto wait = [&](int l) {
-            const uint32_t gl = g + (uint32_t)l;
-            ptt_wait(&bar[warp][gl % PC_NS], (gl / PC_NS) & 1);
+        // TMA: wait for load l; cp.async: for every group but the `pend` newest
+        auto wait = [&](int l, int pend) {
+            if constexpr (TMA) {
+                const uint32_t gl = g + (uint32_t)l;
+                ptt_wait(&bar[warp][gl % PC_NS], (gl / PC_NS) & 1);
+            } else {
+                if (pend >= 2) cp_async_wait<2>();
+                else if (pend == 1) cp_async_wait<1>();
+                else cp_async_wait<0>();
+            }
         };
-        if (lane == 0)
-            for (int l = 0; l < 3 && l < nt + 2; ++l) issue(l);
-        wait(0);
-        wait(1);
+        for (int l = 0; l < 3; ++l)
+            if (l < nt + 2) issue(l);
+            else if constexpr (!TMA) cp_async_commit();  // empty group: uniform counts
+        wait(0, 2);
+        wait(1, 1);
         for (int jt = 0; jt < nt; ++jt) {
-            if (lane == 0 && jt + 3 < nt + 2) issue(jt + 3);
-            wait(jt + 2);
+            if (jt + 3 < nt + 2) issue(jt + 3);
+            else if constexpr (!TMA) cp_async_commit();
+            wait(jt + 2, 1);
             const T* tp = ring + ((g + jt) % PC_NS) * STAGE + lane;       // tile jt - 1
             const T* tc = ring + ((g + jt + 1) % PC_NS) * STAGE + lane;   // tile jt
             const T* tn = ring + ((g + jt + 2) % PC_NS) * STAGE + lane;   // tile jt + 1

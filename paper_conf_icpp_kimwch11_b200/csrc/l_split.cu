@@ -205,11 +205,12 @@ int chains_ctas(const tri_plan_s* p) {
 }
 
 template <typename T, int K, bool RAW>
-cudaError_t launch_chains_k(const PCMaps& tm, const PCArgs<T>& A, int grid, cudaStream_t st) {
+cudaError_t launch_chains_k(const PCMaps& tm, const PCArgs<T>& A, bool tma, int grid, cudaStream_t st) {
     constexpr int smem = PCCfg<T, RAW>::smem_bytes();
-    cudaError_t e = set_smem((const void*)k_pcr_chains<T, K, RAW>, smem);
+    auto kern = tma ? k_pcr_chains<T, K, RAW, true> : k_pcr_chains<T, K, RAW, false>;
+    cudaError_t e = set_smem((const void*)kern, smem);
     if (e != cudaSuccess) return e;
-    k_pcr_chains<T, K, RAW><<<grid, 32 * PCCfg<T, RAW>::WARPS, smem, st>>>(tm, A);
+    kern<<<grid, 32 * PCCfg<T, RAW>::WARPS, smem, st>>>(tm, A);
     return cudaGetLastError();
 }
 
@@ -224,16 +225,19 @@ cudaError_t launch_chains(tri_plan_s* p, int i, const void* in0, const void* in1
     const void* key[4] = {in0, in1, in2, in3};
     const int nk = RAW ? 4 : 3;
     const int tag = 0x7200 + 16 * i + (int)sizeof(T);
-    if (!tm_lookup(p, tag, key, nk, &tm.a, nk)) {
+    // TMA needs a 16-byte row pitch and 16-byte aligned bases; cp.async otherwise
+    bool tma = (C1 * (int64_t)sizeof(T)) % 16 == 0 && C1 < INT32_MAX && L1 + 4 * PC_PO + 64 < INT32_MAX;
+    for (int j = 0; j < nk; ++j) tma = tma && ((uintptr_t)key[j] % 16) == 0;
+    if (tma && !tm_lookup(p, tag, key, nk, &tm.a, nk)) {
         const uint64_t dims[2] = {(uint64_t)C1, (uint64_t)L1}, str[1] = {(uint64_t)C1 * sizeof(T)};
         const uint32_t box[2] = {32u, (uint32_t)PC_PO};
         CUtensorMap* dst[4] = {&tm.a, &tm.c, &tm.d, &tm.b};
-        for (int j = 0; j < nk; ++j)
-            if (!tma_encode(dst[j], sizeof(T), 2, key[j], dims, str, box, CU_TENSOR_MAP_SWIZZLE_NONE))
-                return cudaErrorNotSupported;
-        tm_store(p, tag, key, nk, &tm.a, nk);
+        for (int j = 0; j < nk && tma; ++j)
+            tma = tma_encode(dst[j], sizeof(T), 2, key[j], dims, str, box, CU_TENSOR_MAP_SWIZZLE_NONE);
+        if (tma) tm_store(p, tag, key, nk, &tm.a, nk);
     }
     PCArgs<T> A;
+    for (int j = 0; j < 4; ++j) A.in[j] = (const T*)key[j];
     A.oA = (T*)oA; A.oC = (T*)oC; A.oD = (T*)oD;
     A.n = p->n; A.m = p->m; A.L1 = L1; A.C1 = C1; A.C = p->Cp[i];
     A.Lout = p->Lp[i] << K;
@@ -242,9 +246,9 @@ cudaError_t launch_chains(tri_plan_s* p, int i, const void* in0, const void* in1
     const int grid = (int)std::max<int64_t>(
         1, std::min<int64_t>(cdiv(A.ntask, PCCfg<T, RAW>::WARPS), chains_ctas<T, RAW>(p)));
     switch (K) {
-        case 1: return launch_chains_k<T, 1, RAW>(tm, A, grid, st);
-        case 2: return launch_chains_k<T, 2, RAW>(tm, A, grid, st);
-        case 3: return launch_chains_k<T, 3, RAW>(tm, A, grid, st);
+        case 1: return launch_chains_k<T, 1, RAW>(tm, A, tma, grid, st);
+        case 2: return launch_chains_k<T, 2, RAW>(tm, A, tma, grid, st);
+        case 3: return launch_chains_k<T, 3, RAW>(tm, A, tma, grid, st);
         default: return cudaErrorInvalidValue;
     }
 }
@@ -426,9 +430,8 @@ cudaError_t split_t(tri_plan_s* p, const void* a, const void* b, const void* c, 
 bool rows_ok(const tri_plan_s* p) {
     return p->opt_tma && p->layout == TRI_LAYOUT_CONTIGUOUS;
 }
-bool chains_ok(const tri_plan_s* p, int64_t C1, int64_t L1) {
-    return p->opt_tma && (C1 * (int64_t)esize(p->dtype)) % 16 == 0 && C1 < INT32_MAX &&
-           L1 + 4 * PC_PO + 64 < INT32_MAX;
+bool chains_ok(const tri_plan_s* p) {
+    return p->opt_tma && p->layout != TRI_LAYOUT_BATCHED;
 }
 
 void split_geometry(tri_plan_s* p) {
@@ -445,7 +448,7 @@ void split_geometry(tri_plan_s* p) {
     if (p->k == 0) return;
     const bool f64 = p->dtype == TRI_F64;
     int rem = p->k;
-    if (rows_ok(p) || (p->layout == TRI_LAYOUT_INTERLEAVED && chains_ok(p, m, n))) {
+    if (rows_ok(p) || (p->layout == TRI_LAYOUT_INTERLEAVED && chains_ok(p))) {
         // register tiles: pass 1 up to 5 (rows) / 3 (interleaved) steps, then the
         // remaining steps over the fewest passes of <= 3, balanced
         const bool rows = rows_ok(p);
@@ -482,7 +485,6 @@ void split_geometry(tri_plan_s* p) {
         p->Lp[i] = cdiv(n, int64_t(1) << K);
         p->Cp[i] = m << K;
         const int64_t C1 = i == 0 ? m : p->Cp[i - 1], L1 = i == 0 ? n : p->Lp[i - 1];
-        if (p->pk[i] == PK_CHAINS && !chains_ok(p, C1, L1)) p->pk[i] = PK_IL;  // K <= 3 <= 5
         if (p->pk[i] == PK_ROWS) {
             // tiles of OUT rows cover the L 2^K rows pass 1 writes per system (from
             // up to 3 (fp64) / 7 (fp32) rows before row 0: 32-byte aligned lane rows)

@@ -60,14 +60,13 @@ def test_onchip_every_k(cuda_ok, dtype, layout, n, m):
 def split_launches(n, m, k, layout, dtype, tma=True):
     """tri_plan_launches of a SPLIT plan (l_split.cu split_geometry): p-Thomas plus
     the tiled-PCR passes -- register tiles (5 steps on CONTIGUOUS rows, 3 on
-    INTERLEAVED rows whose row pitch m s is a 16-byte multiple, then passes of
-    <= 3), else the sliding window (10 steps, then passes of <= 5)."""
+    INTERLEAVED rows, then passes of <= 3), else the sliding window (10 steps,
+    then passes of <= 5)."""
     if k == 0:
         return 1
-    es = 8 if dtype == "f64" else 4
     if tma and layout == 0:
         return 2 + -(-max(0, k - 5) // 3)
-    if tma and layout == 1 and (m * es) % 16 == 0:
+    if tma and layout == 1:
         return 2 + -(-max(0, k - 3) // 3)
     return 2 + (0 if k <= 10 else -(-(k - 10) // 5))
 
@@ -92,6 +91,22 @@ def test_split_every_k(cuda_ok, dtype, layout, n, m):
             assert plan.launches == split_launches(n, m, k, layout, dtype, bool(tma)), (k, plan.describe())
             x = plan.solve(*dev).cpu().numpy()
             check_parity(n, m, arrs, x, dtype, layout, x_oracle=xo)
+
+
+@pytest.mark.parametrize("dtype", ["f64", "f32"])
+@pytest.mark.parametrize("n,m,k", [(3001, 3, 7), (5003, 37, 8), (2001, 5, 10), (999, 1, 9)])
+def test_split_chains_cp_async(cuda_ok, dtype, n, m, k):
+    """INTERLEAVED rows whose pitch m s is not a 16-byte multiple (m = 1, 3, 5,
+    37) go through the cp.async chain kernel instead of TMA boxes in the first
+    pass (later passes: pitch m 2^k1 s)."""
+    arrs = gen(n, m, dtype, 1, "weak", eps=1e-2)
+    xo = oracle.solve_batch(n, m, *arrs, layout=1)
+    plan = tri.Plan(n, m, tri.F64 if dtype == "f64" else tri.F32, 1)
+    plan.variant = SPLIT
+    plan.k = k
+    assert plan.launches == split_launches(n, m, k, 1, dtype)
+    x = plan.solve(*to_dev(*arrs)).cpu().numpy()
+    check_parity(n, m, arrs, x, dtype, 1, x_oracle=xo)
 
 
 def test_split_on_small_systems(cuda_ok):
