@@ -44,6 +44,22 @@ METRIC = "Munknowns/s fp64/fp32 and % of HBM roofline at 1/2/4/8 B200"
 FALLBACK_HBM_GBS = 6650.0  # /opt/skills/guides/B200_PROFILING.md fallback
 
 
+def config_of(args):
+    """(n, m, dtype, layout, desc) of --config, with the --n / --m / --layout overrides
+    (an overridden shape is a side measurement, not a BASELINE config)."""
+    n, m, dt, layout, desc = CONFIGS[args.config]
+    if args.layout is not None:
+        layout = args.layout
+    if args.n is not None or args.m is not None:
+        n, m = args.n or n, args.m or m
+        desc = f"custom shape n={n} m={m} ({dt}, layout {layout}); not a BASELINE config"
+    return n, m, dt, layout, desc
+
+
+def workload_of(args):
+    return args.config if args.n is None and args.m is None else args.config + "-custom"
+
+
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -51,6 +67,8 @@ def parse():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--config", default="c5", choices=sorted(CONFIGS))
     ap.add_argument("--layout", type=int, default=None, help="override layout (0 contiguous, 1 interleaved)")
+    ap.add_argument("--n", type=int, default=None, help="override n (side measurement: workload named custom)")
+    ap.add_argument("--m", type=int, default=None, help="override m (side measurement: workload named custom)")
     ap.add_argument("--family", default="dd")
     ap.add_argument("--k", type=int, default=None, help="force the transition point k")
     ap.add_argument("--variant", type=int, default=None, help="force variant (1 onchip, 2 split, 3 fused)")
@@ -179,9 +197,7 @@ def cpu_oracle_time(n, mr, arrs, layout, budget_s=20.0):
 def run_reference(args):
     """--impl reference: the CPU oracle on the box's host cores."""
     world, rank, _ = dist_env()
-    n, m, dt, layout, desc = CONFIGS[args.config]
-    if args.layout is not None:
-        layout = args.layout
+    n, m, dt, layout, desc = config_of(args)
     if rank != 0:
         return  # rank 0 alone runs and prints it
     import oracle
@@ -207,7 +223,7 @@ def run_reference(args):
            "steps": args.steps, "warmup": args.warmup, "ms_per_step": t * 1e3, "higher_is_better": True,
            "scaling": args.scaling or ("weak" if m == 1 else "strong"), "vs_baseline": None, "dtype": dt,
            "data": "synthetic",
-           "config": {"workload": args.config, "desc": desc, "n": n, "m": m, "layout": layout,
+           "config": {"workload": workload_of(args), "desc": desc, "n": n, "m": m, "layout": layout,
                       "family": args.family},
            "cpu_baseline": {"value": v, "unit": "Munknowns/s", "cores": cores, "kind": "oracle",
                             "sample": f"{qs} of {m} systems x n={n} per step (whole systems)"},
@@ -244,9 +260,7 @@ def main():
     dev = torch.device("cuda", torch.cuda.current_device())
     rdev = dev if backend == "nccl" else torch.device("cpu")  # device of the all-reduce scalars
 
-    n, m, dt, layout, desc = CONFIGS[args.config]
-    if args.layout is not None:
-        layout = args.layout
+    n, m, dt, layout, desc = config_of(args)
     s = 8 if dt == "f64" else 4
     tdt = torch.float64 if dt == "f64" else torch.float32
     td = tri.F64 if dt == "f64" else tri.F32
@@ -452,7 +466,7 @@ def main():
         "metric": METRIC, "value": value, "unit": "Munknowns/s", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": t_step_max, "higher_is_better": True, "scaling": scaling,
         "vs_baseline": None, "dtype": dt, "data": "synthetic",
-        "config": {"workload": args.config, "desc": desc, "n": n, "m": m, "m_per_rank": mr, "layout": layout,
+        "config": {"workload": workload_of(args), "desc": desc, "n": n, "m": m, "m_per_rank": mr, "layout": layout,
                    "family": args.family,
                    "parallelism": (f"dp{world}: the m systems sharded over the ranks (contiguous ranges, "
                                    "dist.shard_range), no collective in the solve" if scaling == "strong" else

@@ -71,20 +71,29 @@ __device__ __forceinline__ void pr_st8(float* p, const float (&v)[8]) {
 }
 
 // ---------------------------------------------------------------------------
-// k_pcr_rows: CONTIGUOUS user layout, K <= 5 steps.  Lane l loads its 8 rows
-// straight from global memory as two 32-byte vectors per array (one sector each:
-// a warp reads 2 KB contiguous per array); the next tile's loads are issued
-// before the current tile's steps (register double buffer).  No shared memory:
-// a TMA-staged version measured L1-bound on 4-way bank conflicts of the
-// lane-blocked reads (profiles/r02_ncu_split_rows_tma.txt).
+// k_pcr_rows: CONTIGUOUS user layout, K <= 5 steps.  Every warp owns whole
+// tiles of 32 RPL consecutive rows of one system (lane l rows RPL l .. RPL l +
+// RPL - 1), loaded as 32-byte vectors straight into registers (one sector each:
+// a warp reads 32 RPL elements contiguous per array); with PF the next tile's
+// loads are issued before the current tile's steps (register double buffer).
+// Measured at c3, SPLIT k = 14 (profiles/r02_ncu_split_rows*.txt,
+// scripts/gpu_ab_rows.sh): RPL = 8 with prefetch 0.828 ms per solve; RPL = 16
+// (3x fewer halo rows, 42 % fewer shuffles per row) 0.855 ms without prefetch
+// and spills with it; RPL = 8 without prefetch 0.852 ms; a TMA-staged version
+// was L1-bound on 4-way bank conflicts of the lane-blocked shared reads; CTA
+// super-tiles with shared-memory boundary exchange between warps (no halo
+// tiles) 0.92 ms -- the predicated boundary stores/loads cost more MIO issue
+// than the halo recompute, and the warps of a CTA run in lockstep.
 constexpr int PR_WARPS = 8;   // independent warps per CTA
-constexpr int PR_ROWS = 256;  // rows per tile (8 per lane)
 
-template <int K>
+// RPL rows per lane: a warp tile is 32 RPL rows; the halo is HL whole lanes at
+// each end (RPL HL >= f(K) rows, Eq 8)
+template <int K, int RPL>
 struct PRGeo {
-    static constexpr int HL = ((1 << K) - 1 + 7) / 8;  // halo lanes per side: 8 HL >= f(K) rows (Eq 8)
-    static constexpr int H = 8 * HL;                   // halo rows per side
-    static constexpr int OUT = PR_ROWS - 2 * H;        // rows a tile writes
+    static constexpr int ROWS = 32 * RPL;
+    static constexpr int HL = ((1 << K) - 1 + RPL - 1) / RPL;
+    static constexpr int H = RPL * HL;
+    static constexpr int OUT = ROWS - 2 * H;  // rows a tile writes
 };
 
 template <typename T>
@@ -99,100 +108,110 @@ struct PRArgs {
 };
 
 // 8 consecutive elements, 32-byte aligned, read once (no L1 allocation)
-__device__ __forceinline__ void pr_ld8(const double* p, double (&v)[8]) {
+__device__ __forceinline__ void pr_ld8(const double* p, double* v) {
     asm("ld.global.nc.L1::no_allocate.v4.f64 {%0, %1, %2, %3}, [%4];"
         : "=d"(v[0]), "=d"(v[1]), "=d"(v[2]), "=d"(v[3]) : "l"(p));
     asm("ld.global.nc.L1::no_allocate.v4.f64 {%0, %1, %2, %3}, [%4];"
         : "=d"(v[4]), "=d"(v[5]), "=d"(v[6]), "=d"(v[7]) : "l"(p + 4));
 }
-__device__ __forceinline__ void pr_ld8(const float* p, float (&v)[8]) {
+__device__ __forceinline__ void pr_ld8(const float* p, float* v) {
     asm("ld.global.nc.L1::no_allocate.v8.f32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];"
         : "=f"(v[0]), "=f"(v[1]), "=f"(v[2]), "=f"(v[3]), "=f"(v[4]), "=f"(v[5]), "=f"(v[6]), "=f"(v[7])
         : "l"(p));
 }
 
-template <typename T, int K>
+template <typename T, int K, int RPL, bool PF>
 __global__ void __launch_bounds__(32 * PR_WARPS, 1) k_pcr_rows(PRArgs<T> p) {
-    using G = PRGeo<K>;
+    using G = PRGeo<K, RPL>;
     constexpr int S = 1 << K;
     constexpr int EPC = 32 / (int)sizeof(T);  // elements per 32-byte vector
     const int lane = threadIdx.x & 31;
     const int64_t TW = (int64_t)gridDim.x * PR_WARPS;
     const int64_t n = p.n, N = n * p.m;
 
-    // tile `tile` of system q covers rows [e0, e0 + 256), e0 = tile OUT - H - dq,
+    // tile `tile` of system q covers rows [e0, e0 + 32 RPL), e0 = tile OUT - H - dq,
     // dq = (q n) mod EPC: the tiles of system q shift back by up to EPC - 1 rows
-    // so that every lane's 8 rows start on a 32-byte boundary.  Rows of the
+    // so that every lane's rows start on a 32-byte boundary.  Rows of the
     // neighbouring systems are replaced by identity rows below; rows outside the
     // arrays are not read.
-    T na[8], nb[8], nc[8], nd[8];
+    T va[RPL], vb[RPL], vc[RPL], vd[RPL];
     auto fetch = [&](int64_t task) {
         const int64_t q = task / p.ntile, tile = task - q * p.ntile;
         const int64_t qn = q * n;
-        const int64_t f0 = qn - (qn & (EPC - 1)) + tile * G::OUT - G::H + 8 * lane;  // flat index of row 0
-        if (p.vec && f0 >= 0 && f0 + 8 <= N) {
-            pr_ld8(p.a + f0, na); pr_ld8(p.b + f0, nb); pr_ld8(p.c + f0, nc); pr_ld8(p.d + f0, nd);
+        const int64_t f0 = qn - (qn & (EPC - 1)) + tile * G::OUT - G::H + RPL * lane;  // flat index of row 0
+        if (p.vec && f0 >= 0 && f0 + RPL <= N) {
+#pragma unroll
+            for (int h = 0; h < RPL; h += 8) {
+                pr_ld8(p.a + f0 + h, va + h); pr_ld8(p.b + f0 + h, vb + h);
+                pr_ld8(p.c + f0 + h, vc + h); pr_ld8(p.d + f0 + h, vd + h);
+            }
         } else {
 #pragma unroll
-            for (int u = 0; u < 8; ++u) {
+            for (int u = 0; u < RPL; ++u) {
                 const bool in = f0 + u >= 0 && f0 + u < N;
-                na[u] = in ? p.a[f0 + u] : T(0); nb[u] = in ? p.b[f0 + u] : T(1);
-                nc[u] = in ? p.c[f0 + u] : T(0); nd[u] = in ? p.d[f0 + u] : T(0);
+                va[u] = in ? p.a[f0 + u] : T(0); vb[u] = in ? p.b[f0 + u] : T(1);
+                vc[u] = in ? p.c[f0 + u] : T(0); vd[u] = in ? p.d[f0 + u] : T(0);
             }
         }
     };
     int64_t task = (int64_t)blockIdx.x * PR_WARPS + (threadIdx.x >> 5);
-    if (task < p.ntask) fetch(task);
+    if (PF && task < p.ntask) fetch(task);
     for (; task < p.ntask; task += TW) {
-        T va[8], vb[8], vc[8], vd[8];
-#pragma unroll
-        for (int u = 0; u < 8; ++u) { va[u] = na[u]; vb[u] = nb[u]; vc[u] = nc[u]; vd[u] = nd[u]; }
-        if (task + TW < p.ntask) fetch(task + TW);
-
+        NRow<T> R[RPL];
         const int64_t q = task / p.ntile, tile = task - q * p.ntile;
-        const int64_t i0 = tile * G::OUT - G::H - ((q * n) & (EPC - 1)) + 8 * lane;  // row of register 0
-        NRow<T> R[8];
+        const int64_t i0 = tile * G::OUT - G::H - ((q * n) & (EPC - 1)) + RPL * lane;  // row of register 0
+        if constexpr (PF) {
+            // normalise this tile's rows, then issue the next tile's loads into the
+            // same registers (they are free again) before the steps
 #pragma unroll
-        for (int u = 0; u < 8; ++u) R[u] = pr_norm(i0 + u, n, va[u], vb[u], vc[u], vd[u]);
+            for (int u = 0; u < RPL; ++u) R[u] = pr_norm(i0 + u, n, va[u], vb[u], vc[u], vd[u]);
+            if (task + TW < p.ntask) fetch(task + TW);
+        } else {
+            fetch(task);
+#pragma unroll
+            for (int u = 0; u < RPL; ++u) R[u] = pr_norm(i0 + u, n, va[u], vb[u], vc[u], vd[u]);
+        }
         // PCR steps at strides 1, 2, .., 2^(K-1) (Eqs 5-6); out-of-tile neighbours of
         // the halo lanes are garbage, which only reaches rows within f(K) of the
         // tile edge -- the halo, never written
 #pragma unroll
         for (int j = 0; j < K; ++j) {
             const int sg = 1 << j;
-            NRow<T> N[8];
-            if (sg < 8) {
+            NRow<T> N[RPL];
+            if (sg < RPL) {
 #pragma unroll
-                for (int u = 0; u < 8; ++u) {
-                    const NRow<T> mr = u - sg >= 0 ? R[(u - sg) & 7] : pr_shfl_up(R[(u - sg + 8) & 7], 1);
-                    const NRow<T> pr = u + sg < 8 ? R[(u + sg) & 7] : pr_shfl_down(R[(u + sg - 8) & 7], 1);
+                for (int u = 0; u < RPL; ++u) {
+                    const NRow<T> mr = u - sg >= 0 ? R[(u - sg + RPL) % RPL] : pr_shfl_up(R[(u - sg + RPL) % RPL], 1);
+                    const NRow<T> pr = u + sg < RPL ? R[(u + sg) % RPL] : pr_shfl_down(R[(u + sg) % RPL], 1);
                     N[u] = pcr_combine(mr, R[u], pr);
                 }
             } else {
 #pragma unroll
-                for (int u = 0; u < 8; ++u)
-                    N[u] = pcr_combine(pr_shfl_up(R[u], sg / 8), R[u], pr_shfl_down(R[u], sg / 8));
+                for (int u = 0; u < RPL; ++u)
+                    N[u] = pcr_combine(pr_shfl_up(R[u], sg / RPL), R[u], pr_shfl_down(R[u], sg / RPL));
             }
 #pragma unroll
-            for (int u = 0; u < 8; ++u) R[u] = N[u];
+            for (int u = 0; u < RPL; ++u) R[u] = N[u];
         }
         if (lane < G::HL || lane >= 32 - G::HL) continue;
         if (p.mode == 0) {
-            if (K >= 3 && (i0 & 7) == 0) {
-                // 8 rows of one position, chains q 2^K + (i0 mod 2^K) .. + 7: 64 contiguous bytes
-                if (i0 < p.n_pad) {
-                    T* dA = p.oA + (i0 >> K) * p.C + q * S + (i0 & (S - 1));
+            if (K >= 3 && (i0 & 7) == 0 && i0 + RPL <= p.n_pad) {
+                // 8 rows of one position, chains q 2^K + (i mod 2^K) .. + 7: 64 contiguous bytes
+#pragma unroll
+                for (int h = 0; h < RPL; h += 8) {
+                    const int64_t i = i0 + h;
+                    T* dA = p.oA + (i >> K) * p.C + q * S + (i & (S - 1));
                     const int64_t off = dA - p.oA;
                     T a8[8], c8[8], d8[8];
 #pragma unroll
-                    for (int u = 0; u < 8; ++u) { a8[u] = R[u].A; c8[u] = R[u].C; d8[u] = R[u].D; }
+                    for (int u = 0; u < 8; ++u) { a8[u] = R[h + u].A; c8[u] = R[h + u].C; d8[u] = R[h + u].D; }
                     pr_st8(dA, a8);
                     pr_st8(p.oC + off, c8);
                     pr_st8(p.oD + off, d8);
                 }
             } else {
 #pragma unroll
-                for (int u = 0; u < 8; ++u) {
+                for (int u = 0; u < RPL; ++u) {
                     const int64_t i = i0 + u;
                     if (i >= 0 && i < p.n_pad) {
                         const int64_t idx = (i >> K) * p.C + q * S + (i & (S - 1));
@@ -202,7 +221,7 @@ __global__ void __launch_bounds__(32 * PR_WARPS, 1) k_pcr_rows(PRArgs<T> p) {
             }
         } else {
 #pragma unroll
-            for (int u = 0; u < 8; ++u) {
+            for (int u = 0; u < RPL; ++u) {
                 const int64_t i = i0 + u;
                 if (i >= 0 && i < n) {
                     const int64_t gi = q * n + i;

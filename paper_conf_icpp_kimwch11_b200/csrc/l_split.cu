@@ -164,15 +164,23 @@ cudaError_t launch_pass(const tri_plan_s* p, int i, const void* iA, const void* 
 }
 
 // ---- register-tile passes (k_pcr_reg.cuh) --------------------------------------
+#ifndef PR_RPL
+#define PR_RPL 8   // rows per lane of k_pcr_rows (A/B builds: -DPR_RPL=16)
+#endif
+#ifndef PR_PF
+#define PR_PF 1    // k_pcr_rows register prefetch of the next tile
+#endif
+
 template <typename T, int K>
 cudaError_t launch_rows_k(const PRArgs<T>& A, int sms, cudaStream_t st) {
+    auto kern = k_pcr_rows<T, K, PR_RPL, PR_PF != 0>;
     int occ = 1;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_pcr_rows<T, K>, 32 * PR_WARPS, 0) != cudaSuccess) {
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, 32 * PR_WARPS, 0) != cudaSuccess) {
         cudaGetLastError();
         occ = 1;
     }
     const int64_t grid = std::max<int64_t>(1, std::min<int64_t>(cdiv(A.ntask, PR_WARPS), (int64_t)std::max(1, occ) * sms));
-    k_pcr_rows<T, K><<<(unsigned)grid, 32 * PR_WARPS, 0, st>>>(A);
+    kern<<<(unsigned)grid, 32 * PR_WARPS, 0, st>>>(A);
     return cudaGetLastError();
 }
 
@@ -488,13 +496,14 @@ void split_geometry(tri_plan_s* p) {
         if (p->pk[i] == PK_ROWS) {
             // tiles of OUT rows cover the L 2^K rows pass 1 writes per system (from
             // up to 3 (fp64) / 7 (fp32) rows before row 0: 32-byte aligned lane rows)
-            const int h = ((1 << p->kp[0]) - 1 + 7) / 8 * 8;
-            p->region[0] = cdiv((p->Lp[0] << p->kp[0]) + 32 / (int64_t)esize(p->dtype) - 1, PR_ROWS - 2 * h);
+            const int h = ((1 << p->kp[0]) - 1 + PR_RPL - 1) / PR_RPL * PR_RPL;
+            p->region[0] = cdiv((p->Lp[0] << p->kp[0]) + 32 / (int64_t)esize(p->dtype) - 1, 32 * PR_RPL - 2 * h);
             p->nreg[0] = 1;
             p->nblk[0] = m;
         } else if (p->pk[i] == PK_CHAINS || p->pk[i] == PK_RAW) {
             // tasks = (32-chain block, region of tiles): about two per resident warp,
-            // regions of >= 16 tiles (the two halo tiles stay a small fraction)
+            // regions of >= 4 tiles (two halo tiles per region: at most a third of the
+            // loads, and only on passes too small to fill the GPU otherwise)
             const int64_t ntile = cdiv(p->Lp[i] << p->kp[i], PC_PO);
             const bool raw = p->pk[i] == PK_RAW;
             const int64_t warps = (int64_t)(raw ? (f64 ? chains_ctas<double, true>(p) * PCCfg<double, true>::WARPS
@@ -503,7 +512,7 @@ void split_geometry(tri_plan_s* p) {
                                                        : chains_ctas<float, false>(p) * PCCfg<float, false>::WARPS));
             p->nblk[i] = cdiv(C1, 32);
             int64_t nreg = std::max<int64_t>(1, cdiv(2 * warps, p->nblk[i]));
-            nreg = std::max<int64_t>(1, std::min<int64_t>(nreg, ntile / 16));
+            nreg = std::max<int64_t>(1, std::min<int64_t>(nreg, ntile / 4));
             p->region[i] = cdiv(ntile, nreg);
             p->nreg[i] = cdiv(ntile, p->region[i]);
         } else if (i == 0) {
