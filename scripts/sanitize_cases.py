@@ -36,8 +36,15 @@ CASES = {
     "fused": [(2048, 3, "f64", 0, V.VARIANT_FUSED, None), (2000, 2, "f32", 0, V.VARIANT_FUSED, None)],
     "warp": [(512, 16, "f64", 0, V.VARIANT_WARP, None), (256, 16, "f32", 1, V.VARIANT_WARP, None)],
     "onchip": [(1000, 3, "f64", 0, V.VARIANT_ONCHIP, None)],
+    # register-tile passes: rows kernel (contiguous, ragged, several systems), chain
+    # passes by TMA and by cp.async (interleaved odd pitch), RAW first pass
     "split": [(4096, 2, "f64", 0, V.VARIANT_SPLIT, 3), (1 << 14, 1, "f64", 0, V.VARIANT_SPLIT, 12),
+              (5003, 3, "f64", 0, V.VARIANT_SPLIT, 9), (3001, 4, "f32", 0, V.VARIANT_SPLIT, 7),
+              (1000, 37, "f64", 1, V.VARIANT_SPLIT, 7), (1024, 40, "f32", 1, V.VARIANT_SPLIT, 5),
               (2048, 64, "f64", 0, V.VARIANT_SPLIT, 0), (1000, 64, "f32", 1, V.VARIANT_SPLIT, 0)],
+    # the paper's shared-memory sliding window (TRI_OPT_TMA off)
+    "split_sw": [(4096, 2, "f64", 0, V.VARIANT_SPLIT, "tma0:3"), (1 << 14, 1, "f64", 0, V.VARIANT_SPLIT, "tma0:12"),
+                 (1000, 37, "f64", 1, V.VARIANT_SPLIT, "tma0:7")],
 }
 
 
@@ -51,7 +58,10 @@ def main():
             arrs = trigen.generate(n, m, dt, layout, "dd")
             plan = tri.Plan(n, m, tri.F64 if dt == "f64" else tri.F32, layout)
             plan.variant = v
-            if isinstance(k, str):  # "lbW": SCAN_MC look-back with W-window chunks
+            if isinstance(k, str) and k.startswith("tma0:"):  # TRI_OPT_TMA off, then k
+                plan.set_option(tri.OPT_TMA, 0)
+                plan.k = int(k[5:])
+            elif isinstance(k, str):  # "lbW": SCAN_MC look-back with W-window chunks
                 plan.set_option(tri.OPT_SCAN_MC_LOOKBACK, int(k[2:]))
             elif k is not None:
                 plan.k = k
