@@ -231,17 +231,25 @@ TRI_API tri_status tri_plan_set_k(tri_plan_t plan, int k);
  * current k is invalid for it; may reallocate scratch (TRI_ERR_OOM). */
 TRI_API tri_status tri_plan_set_variant(tri_plan_t plan, tri_variant v);
 /* Plan options (explicit per plan; nothing is read from the environment):
- *   TRI_OPT_TMA (default 1): 0 runs the p-Thomas stage of SPLIT through its
- *     non-TMA kernels (cp.async / ring-staged / thread-per-chain), which
- *     otherwise run only where a TMA descriptor cannot describe the arrays
- *     (row strides not 16-byte multiples); for A/B measurement and tests.
+ *   TRI_OPT_TMA (default 1): 0 runs SPLIT through its pre-TMA kernels: the
+ *     paper's shared-memory sliding-window tiled PCR (Figs 8-10) instead of the
+ *     register-tile passes, and the non-TMA p-Thomas kernels (cp.async /
+ *     ring-staged / thread-per-chain), which otherwise run only where a TMA
+ *     descriptor cannot describe the arrays; for A/B measurement and tests.
  *   TRI_OPT_SCAN_MC_LOOKBACK (default -1 = auto): SCAN_MC passes 0 and 1 fused
  *     by a decoupled look-back over chunks of `value` windows (1 <= value <= 64;
  *     0 = the three-pass form; auto = the three-pass form, measured faster on
  *     B200).  tri_slice_solve needs it off (0 or auto).
+ *   TRI_OPT_SCAN_CLUSTER (default 0): 1 solves INTERLEAVED SCAN batches of at
+ *     most one 8-system group per SM (m <= 8 x SMs, n >= 512, n <= 16384) with
+ *     one thread-block cluster of 2-8 CTAs per group, the group's windows
+ *     spread over the cluster's warps and the forward state / x handed between
+ *     its CTAs through distributed shared memory (P:687
+ *     Fig 11b).  Off by default: measured slower than the chained kernel at c2
+ *     (27.5 vs 21.0 us).
  * TRI_ERR_INVALID_ARG for an unknown option or value; TRI_ERR_OOM if the new
  * geometry's scratch cannot be allocated (option unchanged). */
-typedef enum { TRI_OPT_TMA = 1, TRI_OPT_SCAN_MC_LOOKBACK = 2 } tri_option;
+typedef enum { TRI_OPT_TMA = 1, TRI_OPT_SCAN_MC_LOOKBACK = 2, TRI_OPT_SCAN_CLUSTER = 3 } tri_option;
 TRI_API tri_status tri_plan_set_option(tri_plan_t plan, tri_option opt, int value);
 /* Human-readable one-line plan description into buf (NUL-terminated). */
 TRI_API void tri_plan_describe(tri_plan_t plan, char* buf, int buflen);

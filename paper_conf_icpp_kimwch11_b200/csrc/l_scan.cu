@@ -6,6 +6,7 @@
 #include "plan.cuh"
 #include "k_scan.cuh"
 #include "k_scan_mc.cuh"
+#include "k_scan_cl.cuh"
 
 using namespace tri;
 
@@ -93,6 +94,63 @@ void* scan_kernel(bool prof) {
     return prof ? (void*)k_scan<T, S, true> : (void*)k_scan<T, S, false>;
 }
 
+// TRI_OPT_SCAN_CLUSTER: INTERLEAVED batches of few 8-system groups (no more groups
+// than SMs: the chained kernel leaves SMs idle and walks every window in sequence)
+// through one cluster of CL CTAs per group (k_scan_cl.cuh), CL the smallest of
+// 2 / 4 / 8 whose CTAs are all resident at once; cudaErrorNotSupported leaves the
+// shape to the chained kernel.  Measured slower at c2 (27.5 vs 21.0 us in ncu):
+// every warp walks its windows three times (maps, replay, back substitution) with
+// one load in flight, at 16 warps per SM (registers).
+template <typename T>
+int scan_cl_choose(const tri_plan_s* p, int& wpw) {
+    const int64_t ngrp = cdiv(p->m, SCL_S), nwin = cdiv(p->n, SCL_WR);
+    if (ngrp > p->sms || nwin < 2 * SCL_NW) return 0;
+    const int smem = SCL_NW * SCLayout<T>::in_stride + 1024;
+    int occ = 0;
+    if (set_smem((const void*)k_scan_cl<T, 2>, smem) != cudaSuccess ||
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_scan_cl<T, 2>, 32 * SCL_NW, smem) != cudaSuccess) {
+        cudaGetLastError();
+        return 0;
+    }
+    for (int cl = 2; cl <= 8; cl *= 2) {
+        wpw = (int)cdiv(nwin, (int64_t)cl * SCL_NW);
+        if (wpw <= SCL_WMAX && ngrp * cl <= (int64_t)occ * p->sms) return cl;
+    }
+    return 0;
+}
+
+template <typename T, int CL>
+cudaError_t scan_cl_launch(const tri_plan_s* p, const StreamMaps& tm, const SCLArgs<T>& A, cudaStream_t st) {
+    const int smem = SCL_NW * SCLayout<T>::in_stride + 1024;
+    cudaError_t e = set_smem((const void*)k_scan_cl<T, CL>, smem);
+    if (e != cudaSuccess) return e;
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)(cdiv(p->m, SCL_S) * CL));
+    cfg.blockDim = dim3(32 * SCL_NW);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = CL;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, k_scan_cl<T, CL>, tm, A);
+}
+
+template <typename T>
+cudaError_t scan_cl_t(tri_plan_s* p, const StreamMaps& tm, void* x, cudaStream_t st) {
+    int wpw = 0;
+    const int cl = scan_cl_choose<T>(p, wpw);
+    if (cl == 0) return cudaErrorNotSupported;
+    SCLArgs<T> A;
+    A.x = (T*)x;
+    A.n = p->n; A.m = p->m; A.wpw = wpw;
+    return cl == 2 ? scan_cl_launch<T, 2>(p, tm, A, st)
+                   : cl == 4 ? scan_cl_launch<T, 4>(p, tm, A, st) : scan_cl_launch<T, 8>(p, tm, A, st);
+}
+
 template <typename T>
 cudaError_t scan_t(tri_plan_s* p, const void* a, const void* b, const void* c, const void* d, void* x,
                    cudaStream_t st) {
@@ -137,6 +195,10 @@ cudaError_t scan_t(tri_plan_s* p, const void* a, const void* b, const void* c, c
         }
     } else if (!scan_maps<T>(p, 0x1000 + (int)sizeof(T) + 16 * (w128 ? 1 : 0), a, b, c, d, w128, tm)) {
         return cudaErrorNotSupported;
+    }
+    if (S == 8 && p->nb == 1 && p->opt_cluster) {
+        const cudaError_t ec = scan_cl_t<T>(p, tm, x, st);
+        if (ec != cudaErrorNotSupported) return ec;
     }
     ScanArgs<T> A;
     A.x = (T*)x;

@@ -49,6 +49,7 @@ struct tri_plan_s {
     bool forced = false;          // variant or k set by the caller (tri_solve_host sub-plans inherit it)
     int opt_tma = 1;              // TRI_OPT_TMA: 0 = p-Thomas through the non-TMA kernels
     int opt_lookback = -1;        // TRI_OPT_SCAN_MC_LOOKBACK: windows per look-back chunk (0 = three passes, -1 = auto)
+    int opt_cluster = 0;          // TRI_OPT_SCAN_CLUSTER: interleaved SCAN through thread-block clusters
     int G = 0, P = 0, rpt = 0;    // ONCHIP geometry
     int64_t n_pad = 0, L = 0, C = 0;  // SPLIT: chain length, chains
     int npass = 0;                // SPLIT: tiled-PCR passes (0 at k = 0)

@@ -639,6 +639,12 @@ tri_status tri_plan_set_option(tri_plan_t p, tri_option opt, int value) {
         if (st != TRI_OK) { p->opt_tma = old; plan_geometry(p); }
         return st;
     }
+    if (opt == TRI_OPT_SCAN_CLUSTER) {
+        if (value != 0 && value != 1) return TRI_ERR_INVALID_ARG;
+        p->opt_cluster = value;
+        p->tmc.clear();
+        return TRI_OK;
+    }
     if (opt == TRI_OPT_SCAN_MC_LOOKBACK) {
         if (value < -1 || value > LB_MAXW) return TRI_ERR_INVALID_ARG;
         const int old = p->opt_lookback;
@@ -820,7 +826,7 @@ HostChunks host_chunks(const tri_plan_s* p) {
 tri_status make_sub(tri_plan_s* p, int i, int64_t mi) {
     if (p->sub[i] && p->sub_m[i] == mi && p->sub[i]->variant == (p->forced ? p->variant : p->sub[i]->variant) &&
         (!p->forced || p->sub[i]->k == p->k) && p->sub[i]->opt_tma == p->opt_tma &&
-        p->sub[i]->opt_lookback == p->opt_lookback)
+        p->sub[i]->opt_lookback == p->opt_lookback && p->sub[i]->opt_cluster == p->opt_cluster)
         return TRI_OK;
     tri_destroy(p->sub[i]);
     p->sub[i] = nullptr;
@@ -829,6 +835,7 @@ tri_status make_sub(tri_plan_s* p, int i, int64_t mi) {
     if (!s) return st;
     s->opt_tma = p->opt_tma;
     s->opt_lookback = p->opt_lookback;
+    s->opt_cluster = p->opt_cluster;
     if (p->forced) {
         if (!variant_ok(p->variant, s)) { tri_destroy(s); return TRI_ERR_INVALID_ARG; }
         st = set_plan(s, p->variant, p->k);

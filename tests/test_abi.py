@@ -77,6 +77,7 @@ def test_plan_without_gpu_fails_cleanly(L):
         assert not L.tri_plan_strided(*bad)
         assert L.tri_last_status() == 1, bad  # TRI_ERR_INVALID_ARG
     assert L.tri_plan_set_option(None, 1, 0) == 1
+    assert L.tri_plan_set_option(None, 3, 1) == 1
     assert L.tri_plan_k(None) == -1
     L.tri_destroy(None)  # NULL-safe
     with pytest.raises(tri.TriError):

@@ -850,6 +850,29 @@ def test_c4_auto_plan_sampled(cuda_ok, layout):
         check_parity(n, 1, sub, xs, "f32", 0)
 
 
+@pytest.mark.parametrize("dtype", ["f64", "f32"])
+@pytest.mark.parametrize("n,m", [(1024, 1024), (1000, 36), (4099, 148), (16384, 40), (600, 64), (1024, 8)])
+def test_scan_cluster_option(cuda_ok, dtype, n, m):
+    """Interleaved SCAN through thread-block clusters (TRI_OPT_SCAN_CLUSTER,
+    k_scan_cl: windows of a group spread over 2-8 CTAs, forward state and x
+    handed over through distributed shared memory): parity on 2-, 4- and 8-CTA
+    clusters, ragged n, padded last groups, fewer windows than warps; the same
+    plan without the option runs the chained kernel; repeated solves are
+    bitwise identical (fixed composition order)."""
+    arrs = gen(n, m, dtype, 1, "weak", eps=1e-2)
+    xo = oracle.solve_batch(n, m, *arrs, layout=1)
+    plan = tri.Plan(n, m, tri.F64 if dtype == "f64" else tri.F32, 1)
+    plan.variant = tri.VARIANT_SCAN
+    plan.set_option(tri.OPT_SCAN_CLUSTER, 1)
+    x, _ = gpu_solve(n, m, arrs, dtype, 1, plan=plan)
+    check_parity(n, m, arrs, x, dtype, 1, x_oracle=xo)
+    x2, _ = gpu_solve(n, m, arrs, dtype, 1, plan=plan)
+    assert np.array_equal(x, x2)
+    plan.set_option(tri.OPT_SCAN_CLUSTER, 0)
+    x3, _ = gpu_solve(n, m, arrs, dtype, 1, plan=plan)
+    check_parity(n, m, arrs, x3, dtype, 1, x_oracle=xo)
+
+
 @pytest.mark.parametrize("w", [24, 32, 64, 0])
 def test_scan_mc_lookback_variant(cuda_ok, w):
     """SCAN_MC with passes 0 and 1 fused by a look-back over small chunks
