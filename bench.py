@@ -20,6 +20,7 @@ region and are reported in `collectives`, with a check of the gathered x.
 bounded sample of the same workload -- the tier's reference arm.
 """
 import argparse
+import glob
 import json
 import os
 import statistics
@@ -452,14 +453,15 @@ def main():
     method_bytes = marr * n_unknowns * s
     method_src = "model (SURVEY 8(d))"
     traffic, traffic_src = None, None
-    tf = os.path.join(ROOT, "profiles", f"traffic_{args.config}.json")
-    if os.path.exists(tf):
+    # profiles/traffic_<config>*.json: one ncu capture per plan (n, m, k, variant, layout)
+    for tf in sorted(glob.glob(os.path.join(ROOT, "profiles", f"traffic_{args.config}*.json"))):
         with open(tf) as fh:
             tj = json.load(fh)
         if tj.get("n") == n and tj.get("m") == mr and tj.get("k") == plan.k and \
                 tj.get("variant", plan.variant) == plan.variant and tj.get("layout", layout) == layout:
             traffic = tj.get("dram_bytes_per_launch")
             traffic_src = tj.get("source", tf)
+            break
     if traffic:
         method_bytes, method_src = traffic, "ncu dram bytes of this plan (" + str(traffic_src) + ")"
     out = {
