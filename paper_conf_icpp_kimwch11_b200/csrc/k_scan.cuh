@@ -90,6 +90,10 @@ struct ScanArgs {
     int S_on;      // storage slots resident in shared memory
     unsigned long long* prof;  // diagnostics (scripts/prof_scan.py): per-phase cycle counters, or null
     int dbg;       // diagnostics: 1 = no chain handover (wrong results; timing only)
+    // S == 1, ragged n (sc_patch_tail): rows >= n_al of each system read from the
+    // arrays directly (system q at q xsys); n_al == n otherwise
+    const T *ga, *gb, *gc, *gd;
+    int64_t n_al;
 };
 
 template <typename T>
@@ -253,6 +257,22 @@ __device__ __forceinline__ void sc_fix_rows(int64_t i0, int64_t n, T (&ra)[SC_R]
         if (i == 0 && !keep_a0) ra[u] = T(0);
         if (i == n - 1 && !keep_cn) rc[u] = T(0);
         if (i >= n) { ra[u] = T(0); rb[u] = T(1); rc[u] = T(0); rd[u] = T(0); }
+    }
+}
+
+// Ragged n (n not a multiple of the tensor view's row group r; one system, or a
+// 16-byte system pitch): the tensor map covers rows < n_al = r floor(n / r) and
+// TMA zero-fills the rest of the last window; its rows [n_al, n) come from global
+// memory here (g*: row 0 of the lane's system), before sc_fix_rows.
+template <typename T>
+__device__ __forceinline__ void sc_patch_tail(int64_t i0, int64_t n_al, int64_t n, const T* ga, const T* gb,
+                                              const T* gc, const T* gd, T (&ra)[SC_R], T (&rb)[SC_R], T (&rc)[SC_R],
+                                              T (&rd)[SC_R]) {
+    if (i0 + SC_R <= n_al || i0 >= n) return;
+#pragma unroll
+    for (int u = 0; u < SC_R; ++u) {
+        const int64_t i = i0 + u;
+        if (i >= n_al && i < n) { ra[u] = ga[i]; rb[u] = gb[i]; rc[u] = gc[i]; rd[u] = gd[i]; }
     }
 }
 
@@ -656,6 +676,10 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
                 if (DB < 0 && lane == 0 && j + SC_NW < nsys) issue_to(j + SC_NW, 0, bufs[0], bars[0]);
                 continue;
             }
+            if (p.n_al < n) {
+                const int64_t o = q * p.xsys;
+                sc_patch_tail<T>((int64_t)lane * SC_R, p.n_al, n, p.ga + o, p.gb + o, p.gc + o, p.gd + o, ra, rb, rc, rd);
+            }
             sc_fix_rows<T>((int64_t)lane * SC_R, n, ra, rb, rc, rd);
             sc_range(ra, rb, rc, rd);
             SCM M = sc_wide(sc_fwd_map(ra, rb, rc, rd));
@@ -775,6 +799,10 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
             else sc_ld_rows_il<S>(ib, ls, seg, ra, rb, rc, rd);
         };
         auto fix_rows = [&](T (&ra)[SC_R], T (&rb)[SC_R], T (&rc)[SC_R], T (&rd)[SC_R]) {
+            if (S == 1 && p.n_al < n) {
+                const int64_t o = gq * p.xsys;
+                sc_patch_tail<T>(i0, p.n_al, n, p.ga + o, p.gb + o, p.gc + o, p.gd + o, ra, rb, rc, rd);
+            }
             sc_fix_rows<T>(i0, n, ra, rb, rc, rd);
             if (S > 1 && qf >= p.ms) {  // padding systems of the last group: identity rows
 #pragma unroll

@@ -50,6 +50,10 @@ struct ScanMCArgs {
     // null otherwise
     const double* xafter;
     int NCWs, Ps;
+    // ragged n (k_scan.cuh sc_patch_tail): rows >= n_al of system q from the arrays
+    // (q n); n_al == n otherwise
+    const T *ga, *gb, *gc, *gd;
+    int64_t n_al;
 };
 
 template <typename T>
@@ -221,7 +225,11 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant
             sc_ld_rows_any(ib, lane, p.w128 != 0, ra, rb, rc, rd);
             sc_release_buf();  // this warp's reads of the buffer before the TMA refill
             if (lane == 0 && g + SC_NW < nwin) issue(g + SC_NW);
-            if (edge) sc_fix_rows<T>(i0, n, ra, rb, rc, rd, p.keep_a0, p.keep_cn);
+            if (edge) {
+                if (p.n_al < n)
+                    sc_patch_tail<T>(i0, p.n_al, n, p.ga + q * n, p.gb + q * n, p.gc + q * n, p.gd + q * n, ra, rb, rc, rd);
+                sc_fix_rows<T>(i0, n, ra, rb, rc, rd, p.keep_a0, p.keep_cn);
+            }
             sc_range(ra, rb, rc, rd);
             const int nvalid = (int)(n - i0 < 0 ? 0 : n - i0 < SC_R ? n - i0 : SC_R);
             SCM M = sc_wide((p.keep_cn && nvalid < SC_R) ? sc_fwd_map_n(ra, rb, rc, rd, nvalid) : sc_fwd_map(ra, rb, rc, rd));
@@ -238,7 +246,11 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant
             // ---- forward replay from the chunk's / previous window's state
             T ra[SC_R], rb[SC_R], rc[SC_R], rd[SC_R];
             sc_ld_rows_any(ib, lane, p.w128 != 0, ra, rb, rc, rd);
-            if (edge) sc_fix_rows<T>(i0, n, ra, rb, rc, rd, p.keep_a0, p.keep_cn);
+            if (edge) {
+                if (p.n_al < n)
+                    sc_patch_tail<T>(i0, p.n_al, n, p.ga + q * n, p.gb + q * n, p.gc + q * n, p.gd + q * n, ra, rb, rc, rd);
+                sc_fix_rows<T>(i0, n, ra, rb, rc, rd, p.keep_a0, p.keep_cn);
+            }
             sc_range(ra, rb, rc, rd);
             const int nvalid = (int)(n - i0 < 0 ? 0 : n - i0 < SC_R ? n - i0 : SC_R);
             const bool tr = p.keep_cn && nvalid < SC_R;  // transparent padding rows (slice of a larger system)
@@ -498,7 +510,11 @@ __global__ void __launch_bounds__(LB_THREADS, 1) k_scan_mc_lb(const __grid_const
         const int q = t / lb.Ps, w = (t - q * lb.Ps) * NCW + g;
         const int64_t i0 = (int64_t)w * SC_W + lane * SC_R;
         sc_ld_rows_any(buf, lane, p.w128 != 0, ra, rb, rc, rd);
-        if (w == 0 || (int64_t)(w + 1) * SC_W > n) sc_fix_rows<T>(i0, n, ra, rb, rc, rd, 0, 0);
+        if (w == 0 || (int64_t)(w + 1) * SC_W > n) {
+            if (p.n_al < n)
+                sc_patch_tail<T>(i0, p.n_al, n, p.ga + q * n, p.gb + q * n, p.gc + q * n, p.gd + q * n, ra, rb, rc, rd);
+            sc_fix_rows<T>(i0, n, ra, rb, rc, rd, 0, 0);
+        }
         sc_range(ra, rb, rc, rd);
     };
 

@@ -19,8 +19,10 @@ namespace {
 template <typename T>
 bool map_sys_rows(CUtensorMap* tm, const void* base, int64_t n, int64_t m, bool w128) {
     const int rw = w128 ? 128 / (int)sizeof(T) : 8;  // elements per tensor row
+    // one system: its stride is never stepped, but must still be a 16-byte multiple
+    const uint64_t sys = m == 1 ? ((uint64_t)n * sizeof(T) + 15) / 16 * 16 : (uint64_t)n * sizeof(T);
     const uint64_t dims[3] = {(uint64_t)rw, (uint64_t)(n / rw), (uint64_t)m};
-    const uint64_t str[2] = {(uint64_t)rw * sizeof(T), (uint64_t)n * sizeof(T)};
+    const uint64_t str[2] = {(uint64_t)rw * sizeof(T), sys};
     const uint32_t box[3] = {(uint32_t)rw, (uint32_t)(SC_W / rw), 1u};
     const CUtensorMapSwizzle swz =
         w128 ? CU_TENSOR_MAP_SWIZZLE_128B : sizeof(T) == 8 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_32B;
@@ -44,8 +46,9 @@ bool map_sys_rows4(CUtensorMap* tm, const void* base, const tri_plan_s* p, bool 
 template <typename T>
 bool map_sys_rows3(CUtensorMap* tm, const void* base, const tri_plan_s* p, bool w128) {
     const int rw = w128 ? 128 / (int)sizeof(T) : 8;
+    const uint64_t sys = p->ms == 1 ? ((uint64_t)p->ss * sizeof(T) + 15) / 16 * 16 : (uint64_t)p->ss * sizeof(T);
     const uint64_t dims[3] = {(uint64_t)rw, (uint64_t)(p->n / rw), (uint64_t)p->ms};
-    const uint64_t str[2] = {(uint64_t)rw * sizeof(T), (uint64_t)p->ss * sizeof(T)};
+    const uint64_t str[2] = {(uint64_t)rw * sizeof(T), sys};
     const uint32_t box[3] = {(uint32_t)rw, (uint32_t)(SC_W / rw), 1u};
     const CUtensorMapSwizzle swz =
         w128 ? CU_TENSOR_MAP_SWIZZLE_128B : sizeof(T) == 8 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_32B;
@@ -208,6 +211,11 @@ cudaError_t scan_t(tri_plan_s* p, const void* a, const void* b, const void* c, c
     A.x32 = ((uintptr_t)x % 32 == 0 && (p->ss * (int64_t)sizeof(T)) % 32 == 0 &&
              (p->nb == 1 || (p->bs * (int64_t)sizeof(T)) % 32 == 0)) ? 1 : 0;
     A.w128 = w128 ? 1 : 0;
+    A.ga = (const T*)a; A.gb = (const T*)b; A.gc = (const T*)c; A.gd = (const T*)d;
+    {
+        const int64_t rw = S > 1 ? 1 : w128 ? 128 / (int64_t)sizeof(T) : 8;
+        A.n_al = p->n / rw * rw;  // ragged n: the rows past the tensor map's last row group (sc_patch_tail)
+    }
     A.prof = (unsigned long long*)g_fused_prof;
     A.dbg = g_fused_dbg_mode;
     if (one) {
@@ -247,6 +255,8 @@ cudaError_t scan_mc_setup(tri_plan_s* p, const void* a, const void* b, const voi
     }
     A = ScanMCArgs<T>{};
     A.w128 = w ? 1 : 0;
+    A.ga = (const T*)a; A.gb = (const T*)b; A.gc = (const T*)c; A.gd = (const T*)d;
+    A.n_al = n / (w ? 128 / (int64_t)sizeof(T) : 8) * (w ? 128 / (int64_t)sizeof(T) : 8);
     A.x = (T*)x;
     A.x32 = ((uintptr_t)x % 32 == 0 && (n * (int64_t)sizeof(T)) % 32 == 0) ? 1 : 0;
     A.cd = (T*)p->scratch;

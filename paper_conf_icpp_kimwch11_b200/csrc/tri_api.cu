@@ -83,8 +83,12 @@ bool scan_ok(int64_t n, int64_t m, tri_dtype t, tri_layout layout, int64_t ms = 
         return ms > 0 && (ms * (int64_t)esize(t)) % 16 == 0 && cdiv(n, SC_W / S) <= SC_NCMAX &&
                n < ((int64_t)1 << 31) && ms < ((int64_t)1 << 31) && m / ms < ((int64_t)1 << 31);
     }
+    // CONTIGUOUS: n % 8 == 0, or ragged n of more than one window whose system
+    // starts stay 16-byte aligned (one system, or n s % 16 == 0): the kernels read
+    // the rows past the tensor map's last 8-row group directly (sc_patch_tail)
     if (layout == TRI_LAYOUT_CONTIGUOUS || m == 1)
-        return n % 8 == 0 && cdiv(n, SC_W) <= SC_NCMAX && n / 8 < ((int64_t)1 << 31) && m < ((int64_t)1 << 31);
+        return (n % 8 == 0 || (n > SC_W && (m == 1 || (n * (int64_t)esize(t)) % 16 == 0))) &&
+               cdiv(n, SC_W) <= SC_NCMAX && n / 8 < ((int64_t)1 << 31) && m < ((int64_t)1 << 31);
     // INTERLEAVED: TMA tensor [n][m], row stride m * s a multiple of 16 bytes
     const int S = scan_systems(layout, m);
     return (m * (int64_t)esize(t)) % 16 == 0 && cdiv(n, SC_W / S) <= SC_NCMAX && n < ((int64_t)1 << 31) &&
@@ -93,9 +97,8 @@ bool scan_ok(int64_t n, int64_t m, tri_dtype t, tri_layout layout, int64_t ms = 
 
 // SCAN_MC: as SCAN, for systems of at least two windows.
 bool scan_mc_ok(int64_t n, int64_t m, tri_dtype t, tri_layout layout) {
-    (void)t;
-    return (layout == TRI_LAYOUT_CONTIGUOUS || m == 1) && n % 8 == 0 && n > SC_W && n / 8 < ((int64_t)1 << 31) &&
-           m < ((int64_t)1 << 31);
+    return (layout == TRI_LAYOUT_CONTIGUOUS || m == 1) && (n % 8 == 0 || m == 1 || (n * (int64_t)esize(t)) % 16 == 0) &&
+           n > SC_W && n / 8 < ((int64_t)1 << 31) && m < ((int64_t)1 << 31);
 }
 
 // STRIDED plans: the SCAN kernel through TMA maps when the caller's strides allow

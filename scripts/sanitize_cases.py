@@ -25,12 +25,15 @@ CASES = {
              (16384, 2, "f64", 0, V.VARIANT_SCAN, None),     # NC = 64 > on-chip slots: spill path
              (1024, 5, "f32", 0, V.VARIANT_SCAN, None),
              (256, 40, "f64", 0, V.VARIANT_SCAN, None),      # one-window systems, several per warp
-             (128, 40, "f32", 0, V.VARIANT_SCAN, None)],     # short one-window systems (k_scan1)
+             (128, 40, "f32", 0, V.VARIANT_SCAN, None),      # short one-window systems (k_scan1)
+             (1002, 3, "f64", 0, V.VARIANT_SCAN, None),      # ragged n, 16-byte pitch: tail rows from global
+             (5003, 1, "f32", 0, V.VARIANT_SCAN, None)],     # ragged n, one system
     "scan_il": [(1024, 16, "f64", 1, V.VARIANT_SCAN, None),  # interleaved, S = 8: two 8-system groups
                 (520, 24, "f32", 1, V.VARIANT_SCAN, None)],  # ragged last window
     "scan_r16": [(256, 40, "f32", 0, V.VARIANT_SCAN, None), (224, 33, "f32", 0, V.VARIANT_SCAN, None)],
     "scan_mc": [(1 << 16, 1, "f64", 0, V.VARIANT_SCAN_MC, None),
-                (40960, 2, "f32", 0, V.VARIANT_SCAN_MC, None)],
+                (40960, 2, "f32", 0, V.VARIANT_SCAN_MC, None),
+                (65537, 1, "f64", 0, V.VARIANT_SCAN_MC, None)],  # ragged n
     "scan_mc_lb": [(1 << 16, 1, "f64", 0, V.VARIANT_SCAN_MC, "lb32"), (40960, 2, "f32", 0, V.VARIANT_SCAN_MC, "lb16")],
     "stream": [(4096, 3, "f64", 0, V.VARIANT_STREAM, None)],
     "fused": [(2048, 3, "f64", 0, V.VARIANT_FUSED, None), (2000, 2, "f32", 0, V.VARIANT_FUSED, None)],

@@ -110,7 +110,9 @@ def test_heuristic_paper_rule_extremes(L):
     assert tri.choose_variant(16384, 16384, tri.F64, tri.CONTIGUOUS, 148) == tri.VARIANT_SCAN
     assert tri.choose_k(16384, 16384, tri.F64, tri.CONTIGUOUS, 148) == 0
     assert tri.choose_k(1 << 24, 1, tri.F64, tri.INTERLEAVED, 148) >= 8
-    assert tri.choose_k((1 << 24) + 1, 1, tri.F64, tri.CONTIGUOUS, 148) >= 8
+    # one huge CONTIGUOUS system, any n: chunked SCAN (SCAN_MC) at k = 0; a ragged
+    # n reads its last rows past the tensor map's 8-row groups directly
+    assert tri.choose_variant((1 << 24) + 1, 1, tri.F64, tri.CONTIGUOUS, 148) == tri.VARIANT_SCAN_MC
 
 
 @pytest.mark.parametrize("m,G", [(16384, 1), (16384, 8), (10, 4), (3, 8), (1, 2), (1000, 7)])
@@ -135,7 +137,9 @@ def test_shard_range_partitions(L, m, G):
     ("few-long", 65536, 37, "F64", 0, "VARIANT_SCAN_MC", 0),  # < 128 long systems: chunked SCAN
     ("few-long-il", 65536, 37, "F64", 1, "VARIANT_SPLIT", 8),  # interleaved: deep-k SPLIT
     ("odd-n", 1 << 20, 1, "F64", 0, "VARIANT_SCAN_MC", 0),
-    ("ragged", (1 << 20) + 3, 1, "F64", 0, "VARIANT_SPLIT", 14),  # n % 8 != 0: tiled PCR
+    ("ragged", (1 << 20) + 3, 1, "F64", 0, "VARIANT_SCAN_MC", 0),  # n % 8 != 0, one system: tail rows read directly
+    ("ragged-batch", 1002, 4096, "F64", 0, "VARIANT_SCAN", 0),  # n % 8 != 0, 16-byte system pitch
+    ("ragged-odd", 1001, 4096, "F64", 0, "VARIANT_WARP", 5),  # unaligned system starts: PCR in a warp + p-Thomas
 ])
 def test_planner_picks_for_baseline_configs(L, cfg, n, m, dtype, layout, variant, k):
     """The planner's (variant, k) on a 148-SM B200 for BASELINE.json's configs,

@@ -502,11 +502,14 @@ def test_scan_edges_and_scaling(cuda_ok, n, m):
 
 
 def test_scan_rejects_unsupported(cuda_ok):
-    for (n, m, dt, layout) in [(1004, 3, tri.F64, 0), (16384, 3, tri.F64, 1), (7, 3, tri.F32, 0),
-                               ((1 << 20) + 8, 1, tri.F64, 0), (100, 6, tri.F32, 1)]:
+    for (n, m, dt, layout) in [(1001, 3, tri.F64, 0), (1002, 3, tri.F32, 0), (250, 3, tri.F64, 0),
+                               (16384, 3, tri.F64, 1), (7, 3, tri.F32, 0), ((1 << 20) + 8, 1, tri.F64, 0),
+                               (100, 6, tri.F32, 1)]:
         plan = tri.Plan(n, m, dt, layout)
         with pytest.raises(tri.TriError):
-            plan.variant = SCAN  # n % 8; interleaved row stride not a 16-byte multiple; > 4096 windows
+            # ragged n with unaligned system starts, or of one window; interleaved row
+            # stride not a 16-byte multiple; > 4096 windows
+            plan.variant = SCAN
 
 
 @pytest.mark.parametrize("family", ["dd", "weak"])
@@ -681,7 +684,7 @@ def test_scan_mc_edges_and_scaling(cuda_ok):
 
 
 def test_scan_mc_rejects_unsupported(cuda_ok):
-    for (n, m, dt, layout) in [(256, 3, tri.F64, 0), (1004, 3, tri.F64, 0), (16384, 3, tri.F64, 1)]:
+    for (n, m, dt, layout) in [(256, 3, tri.F64, 0), (1001, 3, tri.F64, 0), (16384, 3, tri.F64, 1)]:
         plan = tri.Plan(n, m, dt, layout)
         with pytest.raises(tri.TriError):
             plan.variant = SCAN_MC
@@ -711,6 +714,7 @@ def _sliced_solve_one_device(arrs, cuts, dtype):
     ("f64", "weak", [0, 65536, 131072, 196608, 262144, 327680, 393216, 458752, 524288]),
     ("f64", "poisson", [0, 4096, 8192, 12288, 16384]),
     ("f32", "dd", [0, 70000, 140000, 1000000]),
+    ("f64", "dd", [0, 300003, 700001, 1000003]),  # ragged slice lengths (tail rows read directly)
 ])
 def test_one_system_sliced_over_devices(cuda_ok, dtype, family, cuts):
     """one system split into row slices (ragged, 1 to 8
@@ -871,6 +875,29 @@ def test_scan_cluster_option(cuda_ok, dtype, n, m):
     plan.set_option(tri.OPT_SCAN_CLUSTER, 0)
     x3, _ = gpu_solve(n, m, arrs, dtype, 1, plan=plan)
     check_parity(n, m, arrs, x3, dtype, 1, x_oracle=xo)
+
+
+@pytest.mark.parametrize("dtype,n,m,variant", [
+    ("f64", (1 << 20) + 3, 1, "SCAN_MC"), ("f64", 65537, 1, "SCAN_MC"), ("f64", 1000003, 1, "SCAN_MC"),
+    ("f32", (1 << 20) + 5, 1, "SCAN_MC"), ("f64", 300, 1, "SCAN"), ("f64", 5003, 1, "SCAN"),
+    ("f64", 1002, 64, "SCAN"), ("f32", 1004, 100, "SCAN"), ("f64", 514, 300, "SCAN"), ("f32", 4100, 3, "SCAN"),
+    ("f64", 40002, 3, "SCAN_MC")])
+def test_scan_ragged_n(cuda_ok, dtype, n, m, variant):
+    """SCAN / SCAN_MC with n % 8 != 0 (one system, or a 16-byte system pitch):
+    the TMA maps cover the full 8-row groups and the last rows of each system
+    come from global memory (k_scan.cuh sc_patch_tail); every system vs the
+    oracle, weak family, plus the SCAN_MC look-back path on one system."""
+    arrs = gen(n, m, dtype, 0, "weak", eps=1e-2)
+    xo = oracle.solve_batch(n, m, *arrs)
+    plan = tri.Plan(n, m, tri.F64 if dtype == "f64" else tri.F32, 0)
+    plan.variant = getattr(tri, "VARIANT_" + variant)
+    assert plan.variant == getattr(tri, "VARIANT_" + variant)
+    x, _ = gpu_solve(n, m, arrs, dtype, 0, plan=plan)
+    check_parity(n, m, arrs, x, dtype, 0, x_oracle=xo)
+    if variant == "SCAN_MC" and m == 1:
+        plan.set_option(tri.OPT_SCAN_MC_LOOKBACK, 32)
+        x2, _ = gpu_solve(n, m, arrs, dtype, 0, plan=plan)
+        check_parity(n, m, arrs, x2, dtype, 0, x_oracle=xo)
 
 
 @pytest.mark.parametrize("w", [24, 32, 64, 0])
