@@ -7,10 +7,11 @@
 // paper keeps the levels of a sub-tile in shared memory and slides a window
 // (Figs 8-10); on sm_100a that window is bound by shared-memory bandwidth
 // (k_tiled_pcr.cuh: 12 shared-memory accesses per row per level).  Here every
-// warp owns whole tiles: a tile plus its f(k) halo is read once (by TMA through
-// shared memory, or straight into registers), and all k levels run in registers -- in-lane neighbours directly, cross-lane neighbours by warp
-// shuffle -- so shared memory is touched once per row, not once per row per
-// level.  The halo rows are recomputed by the neighbouring tile (redundant
+// warp owns whole tiles: a tile plus its f(k) halo is read once (straight into
+// registers, or by TMA / cp.async through a per-warp shared-memory ring), and
+// all k levels run in registers -- in-lane neighbours directly, cross-lane
+// neighbours by warp shuffle -- so shared memory is touched at most once per
+// row, not once per row per level.  The halo rows are recomputed by the neighbouring tile (redundant
 // arithmetic instead of the paper's cached dependency rows: the ALU and shuffle
 // pipes have headroom, HBM does not).
 //

@@ -40,10 +40,8 @@ constexpr int SCL_WR = SC_W / SCL_S;  // rows per window (32)
 constexpr int SCL_WMAX = 8;           // windows per warp (shared-memory state table)
 
 template <typename T>
-struct SCLArgs {
+struct SCLArgs {  // dynamic shared memory: SCL_NW staging buffers of SCLayout<T>::in_stride bytes + 1 KB slack
     T* x;
-    // dynamic shared memory: SCL_NW staging buffers of SCLayout<T>::in_stride bytes
-    // (+ 1 KB alignment slack)
     int64_t n, m;  // rows, systems (one batch: row i of system q at i m + q)
     int wpw;       // windows per warp
 };
