@@ -214,6 +214,38 @@ def test_power_of_two_row_scaling_bitwise(cuda_ok):
         assert np.array_equal(x2, x0 * 1024.0)
 
 
+@pytest.mark.parametrize("variant,k,n,m,layout", [
+    ("SCAN", None, 4096, 6, 0), ("SCAN", None, 1024, 64, 1), ("SCAN_MC", None, 1 << 16, 1, 0),
+    ("SPLIT", 0, 3000, 40, 0), ("SPLIT", 4, 3000, 40, 0), ("SPLIT", 9, 20001, 3, 0), ("SPLIT", 6, 3000, 40, 1),
+    ("STREAM", None, 4096, 6, 0), ("FUSED", None, 2048, 160, 0), ("WARP", None, 512, 160, 0),
+    ("ONCHIP", 3, 1000, 3, 0)])
+def test_degenerate_systems(cuda_ok, variant, k, n, m, layout):
+    """Special cases with a plain answer, on every variant: a diagonal system
+    (a = c = 0: x = d / b, within 2 ulp -- the path divides through reciprocals
+    and scales by powers of two), d = 0 (x = 0 exactly, no NaN from 0 / 0 or
+    inf * 0), and the identity (x = d bitwise)."""
+    import torch
+    g = torch.Generator().manual_seed(5)
+    N = n * m
+    b = (1.0 + torch.rand(N, generator=g, dtype=torch.float64)).cuda()
+    d = (torch.rand(N, generator=g, dtype=torch.float64) - 0.5).cuda()
+    zero = torch.zeros(N, dtype=torch.float64, device="cuda")
+    plan = tri.Plan(n, m, tri.F64, layout)
+    plan.variant = getattr(tri, "VARIANT_" + variant)
+    if k is not None:
+        plan.k = k
+    x = plan.solve(zero, b, zero, d)
+    ref = d / b
+    assert float(((x - ref).abs() / ref.abs().clamp_min(1e-300)).max()) <= 4.5e-16, plan.describe()
+    a = (torch.rand(N, generator=g, dtype=torch.float64) - 0.5).cuda() * 0.4
+    c = (torch.rand(N, generator=g, dtype=torch.float64) - 0.5).cuda() * 0.4
+    x0 = plan.solve(a, b, c, zero)
+    assert bool((x0 == 0).all()), plan.describe()
+    one = torch.ones(N, dtype=torch.float64, device="cuda")
+    x1 = plan.solve(zero, one, zero, d)
+    assert torch.equal(x1, d), plan.describe()
+
+
 def test_flip(cuda_ok):
     """Reversing the rows and swapping a and c reverses x (within tolerance)."""
     n, m = 5000, 4
