@@ -247,9 +247,22 @@ TRI_API tri_status tri_plan_set_variant(tri_plan_t plan, tri_variant v);
  *     its CTAs through distributed shared memory (P:687
  *     Fig 11b).  Off by default: measured slower than the chained kernel at c2
  *     (27.5 vs 21.0 us).
+ *   TRI_OPT_SCAN_GRID (default -1 = auto = on where it fits): INTERLEAVED
+ *     (and unit-system-stride BATCHED / STRIDED) SCAN batches whose 32-system
+ *     blocks split into Q <= 8 row pieces of 16 warps x <= 16 rows with every
+ *     block's thread-block cluster of Q CTAs resident at once (one wave) run
+ *     k_scan_grid: each lane owns one system's run of rows, the whole batch is
+ *     in flight at once, and the Q CTAs of a block exchange their forward /
+ *     backward aggregate maps through distributed shared memory; 0 = the
+ *     chained 8-system-window kernel; 1 = as auto.
  * TRI_ERR_INVALID_ARG for an unknown option or value; TRI_ERR_OOM if the new
  * geometry's scratch cannot be allocated (option unchanged). */
-typedef enum { TRI_OPT_TMA = 1, TRI_OPT_SCAN_MC_LOOKBACK = 2, TRI_OPT_SCAN_CLUSTER = 3 } tri_option;
+typedef enum {
+    TRI_OPT_TMA = 1,
+    TRI_OPT_SCAN_MC_LOOKBACK = 2,
+    TRI_OPT_SCAN_CLUSTER = 3,
+    TRI_OPT_SCAN_GRID = 4
+} tri_option;
 TRI_API tri_status tri_plan_set_option(tri_plan_t plan, tri_option opt, int value);
 /* Human-readable one-line plan description into buf (NUL-terminated). */
 TRI_API void tri_plan_describe(tri_plan_t plan, char* buf, int buflen);

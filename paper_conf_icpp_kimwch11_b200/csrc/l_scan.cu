@@ -7,6 +7,7 @@
 #include "k_scan.cuh"
 #include "k_scan_mc.cuh"
 #include "k_scan_cl.cuh"
+#include "k_scan_grid.cuh"
 
 using namespace tri;
 
@@ -154,9 +155,82 @@ cudaError_t scan_cl_t(tri_plan_s* p, const StreamMaps& tm, void* x, cudaStream_t
                    : cl == 4 ? scan_cl_launch<T, 4>(p, tm, A, st) : scan_cl_launch<T, 8>(p, tm, A, st);
 }
 
+// k_scan_grid (the planner's sg_Q > 0): tensor [nb][n][ms] (row stride es, batch
+// stride bs), box [1][4 rows][32 systems]; blocks x Q CTAs in clusters of Q (the
+// Q row pieces of a 32-system block exchange their aggregates through DSMEM)
+template <typename T>
+cudaError_t scan_grid_t(tri_plan_s* p, const void* a, const void* b, const void* c, const void* d, void* x,
+                        cudaStream_t st) {
+    StreamMaps tm;
+    const void* key[4] = {a, b, c, d};
+    if (!tm_lookup(p, 0x2800 + (int)sizeof(T), key, 4, &tm.a, 4)) {
+        const void* src[4] = {a, b, c, d};
+        CUtensorMap* dst[4] = {&tm.a, &tm.b, &tm.c, &tm.d};
+        for (int i = 0; i < 4; ++i) {
+            const uint64_t dims[3] = {(uint64_t)p->ms, (uint64_t)p->n, (uint64_t)p->nb};
+            const uint64_t str[2] = {(uint64_t)p->es * sizeof(T), (uint64_t)p->bs * sizeof(T)};
+            const uint32_t box[3] = {32u, (uint32_t)SG_SR, 1u};
+            if (!tma_encode(dst[i], sizeof(T), 3, src[i], dims, str, box, CU_TENSOR_MAP_SWIZZLE_NONE))
+                return cudaErrorNotSupported;
+        }
+        tm_store(p, 0x2800 + (int)sizeof(T), key, 4, &tm.a, 4);
+    }
+    const int ctas = p->sg_Q * p->sg_bpb * (int)p->nb;
+    SGArgs<T> A;
+    A.x = (T*)x;
+    A.n = p->n; A.ms = p->ms; A.xel = p->es; A.xbat = p->bs;
+    A.bpb = p->sg_bpb; A.Q = p->sg_Q;
+    A.prof = (unsigned long long*)g_fused_prof;  // tri_debug_set_profile: [CTAs][16][16] phase timestamps
+    A.dbg = g_fused_dbg_mode;
+    const int nst = p->sg_R / SG_SR;
+    void* kern = nst == 1 ? (void*)k_scan_grid<T, 1> : nst == 2 ? (void*)k_scan_grid<T, 2>
+                 : nst == 3 ? (void*)k_scan_grid<T, 3> : (void*)k_scan_grid<T, 4>;
+    const int smem = SGLayout<T>::smem_bytes;
+    cudaError_t e = set_smem(kern, smem);
+    if (e != cudaSuccess) return e;
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)ctas);
+    cfg.blockDim = dim3(SG_THREADS);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = (unsigned)p->sg_Q;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    void* args[] = {(void*)&tm, (void*)&A};
+    return cudaLaunchKernelExC(&cfg, kern, args);
+}
+
+template <typename T>
+bool scan_grid_fits_t(const tri_plan_s* p, int Q, int R, int64_t nblk) {
+    const int nst = R / SG_SR;
+    const void* kern = nst == 1 ? (const void*)k_scan_grid<T, 1> : nst == 2 ? (const void*)k_scan_grid<T, 2>
+                       : nst == 3 ? (const void*)k_scan_grid<T, 3> : (const void*)k_scan_grid<T, 4>;
+    const int smem = SGLayout<T>::smem_bytes;
+    if (set_smem(kern, smem) != cudaSuccess) { cudaGetLastError(); return false; }
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)(nblk * Q));
+    cfg.blockDim = dim3(SG_THREADS);
+    cfg.dynamicSmemBytes = smem;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = (unsigned)Q;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    int ncl = 0;
+    if (cudaOccupancyMaxActiveClusters(&ncl, kern, &cfg) != cudaSuccess) { cudaGetLastError(); return false; }
+    return (int64_t)ncl >= nblk;
+}
+
 template <typename T>
 cudaError_t scan_t(tri_plan_s* p, const void* a, const void* b, const void* c, const void* d, void* x,
                    cudaStream_t st) {
+    if (p->sg_Q > 0) return scan_grid_t<T>(p, a, b, c, d, x, st);
     const int S = p->sk_S;
     const bool contig = p->layout == TRI_LAYOUT_CONTIGUOUS;  // the one-window kernels assume system stride n
     if constexpr (sizeof(T) == 4) {
@@ -368,6 +442,9 @@ int scan_smem_fixed(tri_dtype t, int NC, int delta) {
 int scan_slot_bytes(tri_dtype t) { return t == TRI_F64 ? SCLayout<double>::slot_bytes : SCLayout<float>::slot_bytes; }
 int scan_in_stride(tri_dtype t) { return t == TRI_F64 ? SCLayout<double>::in_stride : SCLayout<float>::in_stride; }
 int scan_mc_wmax() { return SMC_WMAX; }
+bool scan_grid_fits(const tri_plan_s* p, int Q, int R, int64_t nblk) {
+    return p->dtype == TRI_F64 ? scan_grid_fits_t<double>(p, Q, R, nblk) : scan_grid_fits_t<float>(p, Q, R, nblk);
+}
 int scan_mc_lb_maxw() { return LB_MAXW; }
 
 }  // namespace trih

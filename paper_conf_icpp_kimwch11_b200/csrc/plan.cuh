@@ -50,6 +50,7 @@ struct tri_plan_s {
     int opt_tma = 1;              // TRI_OPT_TMA: 0 = p-Thomas through the non-TMA kernels
     int opt_lookback = -1;        // TRI_OPT_SCAN_MC_LOOKBACK: windows per look-back chunk (0 = three passes, -1 = auto)
     int opt_cluster = 0;          // TRI_OPT_SCAN_CLUSTER: interleaved SCAN through thread-block clusters
+    int opt_grid = -1;            // TRI_OPT_SCAN_GRID: interleaved SCAN split over the grid (k_scan_grid; -1 auto)
     int G = 0, P = 0, rpt = 0;    // ONCHIP geometry
     int64_t n_pad = 0, L = 0, C = 0;  // SPLIT: chain length, chains
     int npass = 0;                // SPLIT: tiled-PCR passes (0 at k = 0)
@@ -65,6 +66,7 @@ struct tri_plan_s {
     int sk_grid = 0, sk_nc = 0, sk_son = 0;  // STREAM / SCAN: persistent CTAs, windows per system, resident slots
     int sk_delta = 8;             // SCAN: back-substitution lag (steps)
     int sk_S = 1;                 // SCAN: systems per window (1 contiguous; 8 interleaved)
+    int sg_Q = 0, sg_R = 0, sg_bpb = 0;  // SCAN, k_scan_grid: CTAs per 32-system block, rows per warp, blocks per batch
     int64_t ms = 0;               // systems per batch (BATCHED / STRIDED; m otherwise)
     // element (system q = b ms + s, row i) at offset i es + s ss + b bs (elements) of
     // every array, for every layout: CONTIGUOUS (1, n, n m), INTERLEAVED (m, 1, n m),
@@ -140,6 +142,8 @@ int scan_smem_fixed(tri_dtype t, int NC, int delta);  // SCLayout<T>::smem_bytes
 int scan_slot_bytes(tri_dtype t);
 int scan_in_stride(tri_dtype t);
 int scan_mc_wmax();
+// k_scan_grid: nblk clusters of Q CTAs (R rows per warp) all resident at once
+bool scan_grid_fits(const tri_plan_s* p, int Q, int R, int64_t nblk);
 int scan_mc_lb_maxw();
 // STREAM (l_stream.cu)
 cudaError_t launch_stream(tri_plan_s* p, const void* a, const void* b, const void* c, const void* d, void* x,

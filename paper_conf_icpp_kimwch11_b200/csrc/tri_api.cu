@@ -16,6 +16,7 @@
 #include "k_fused.cuh"
 #include "k_scan.cuh"
 #include "k_scan_mc.cuh"
+#include "k_scan_grid.cuh"
 #include "k_stream.cuh"
 #include "k_tiled_pcr.cuh"
 #include "k_warp.cuh"
@@ -119,6 +120,13 @@ bool strided_fast(int64_t n, int64_t ms, int64_t nb, tri_dtype t, int64_t es, in
     return false;
 }
 
+// the arithmetic part of k_scan_grid's feasibility (scan_grid_geometry adds the
+// cluster occupancy check on the device)
+bool grid_shape_ok(int64_t n, int64_t m, int sms) {
+    const int64_t nblk = cdiv(m, 32), Q = cdiv(n, (int64_t)SG_NW * SG_RMAX);
+    return m >= 8 && Q <= SG_QMAX && nblk * Q <= sms;
+}
+
 bool variant_ok(tri_variant v, const tri_plan_s* p) {
     if (p->layout == TRI_LAYOUT_STRIDED) return v == TRI_VARIANT_SCAN && !p->inner;
     switch (v) {
@@ -158,6 +166,12 @@ tri_variant choose_variant(int64_t n, int64_t m, tri_dtype t, tri_layout layout,
     // SPLIT k = 0 1.07x faster at 8192 x 16384) or, fp32, where many systems favour
     // one thread per system (m > 16384: SPLIT k = 0 1.06-1.11x faster); e.g. c2
     // 1024 x 1024: 23 us vs 28 us (WARP); 4096 x 4096: 170 us vs 879 us.
+    // ... and from fewer systems where the whole batch fits the grid kernel (k_scan_grid:
+    // 32-system blocks x <= 8 row pieces of <= 256 rows, one CTA per SM; r02
+    // sweep_grid: n = 1024, m = 64: 14.4 us vs 18.4 us ONCHIP; n = 2048, m = 64: 16.4
+    // vs 28.7; n <= 256 stays with WARP / ONCHIP, 1.2-1.5x faster there)
+    if (layout == TRI_LAYOUT_INTERLEAVED && n > 256 && scan_ok(n, m, t, layout) && grid_shape_ok(n, m, sms))
+        return TRI_VARIANT_SCAN;
     if (layout == TRI_LAYOUT_INTERLEAVED && m >= 256 && n > 256 && scan_ok(n, m, t, layout)) {
         const int64_t N = n * m;
         const bool fits = t == TRI_F64 ? N < ((int64_t)1 << 27) : N < ((int64_t)1 << 28) && m <= 16384;
@@ -210,6 +224,27 @@ int kmin_for(tri_variant v) {
 }
 
 // ---- per-plan geometry -----------------------------------------------------
+// SCAN on a unit-system-stride layout (8-system windows) through k_scan_grid when
+// every 32-system block's rows split into Q <= 8 pieces of 16 warps x R rows (one
+// thread-block cluster per block) and all the clusters are resident at once (one
+// wave; cudaOccupancyMaxActiveClusters -- clusters of 8 need 8 free SMs of one
+// GPC): R = 4 .. 16, the smallest that fits (the most SMs stream).  Off with
+// TRI_OPT_SCAN_GRID 0.
+void scan_grid_geometry(tri_plan_s* p) {
+    p->sg_Q = p->sg_R = p->sg_bpb = 0;
+    if (p->sk_S != 8 || p->opt_grid == 0 || p->n >= ((int64_t)1 << 30)) return;
+    const int64_t bpb = cdiv(p->ms, 32), nblk = bpb * p->nb;
+    for (int R = SG_SR; R <= SG_RMAX; R += SG_SR) {
+        const int64_t Q = cdiv(p->n, (int64_t)SG_NW * R);
+        if (Q <= SG_QMAX && nblk * Q <= p->sms && scan_grid_fits(p, (int)Q, R, nblk)) {
+            p->sg_Q = (int)Q;
+            p->sg_R = R;
+            p->sg_bpb = (int)bpb;
+            return;
+        }
+    }
+}
+
 void plan_geometry(tri_plan_s* p) {
     const int64_t n = p->n, m = p->m;
     p->tmc.clear();
@@ -262,6 +297,7 @@ void plan_geometry(tri_plan_s* p) {
         const int slot = p->dtype == TRI_F64 ? SCLayout<double>::slot_bytes : SCLayout<float>::slot_bytes;
         const int64_t avail = ((int64_t)p->smem_optin - (p->dtype == TRI_F64 ? fixed : fixed32)) / slot;
         p->sk_son = (p->sk_nc == 1 && p->sk_S == 1) ? 0 : (int)std::max<int64_t>(0, std::min<int64_t>(p->sk_nc + p->sk_delta, avail));
+        scan_grid_geometry(p);
     }
     if (p->variant == TRI_VARIANT_SCAN_MC) {
         p->L = n; p->n_pad = n; p->C = m;
@@ -312,6 +348,7 @@ size_t scratch_need(const tri_plan_s* p) {
                (size_t)p->m * (size_t)p->mc_P * 16 * 8 + 16 * es +
                (p->mc_lb ? (size_t)p->m * (size_t)p->mc_Ps * (SMC_REC * 8 + 4) +
                                (size_t)p->m * (size_t)((p->mc_Ps + 31) / 32) * (8 * 8 + 4) + 256 : 0);
+    if (p->variant == TRI_VARIANT_SCAN && p->sg_Q > 0) return 0;  // k_scan_grid: no global scratch
     if (p->variant == TRI_VARIANT_SCAN)
         return (p->sk_nc == 1 && p->sk_S == 1) ? 0
                              : (size_t)p->sk_grid * (size_t)std::max(0, p->sk_nc + p->sk_delta - p->sk_son) *
@@ -648,6 +685,14 @@ tri_status tri_plan_set_option(tri_plan_t p, tri_option opt, int value) {
         p->tmc.clear();
         return TRI_OK;
     }
+    if (opt == TRI_OPT_SCAN_GRID) {
+        if (value < -1 || value > 1) return TRI_ERR_INVALID_ARG;
+        const int old = p->opt_grid;
+        p->opt_grid = value;
+        const tri_status st = set_plan(p, p->variant, p->k);
+        if (st != TRI_OK) { p->opt_grid = old; plan_geometry(p); }
+        return st;
+    }
     if (opt == TRI_OPT_SCAN_MC_LOOKBACK) {
         if (value < -1 || value > LB_MAXW) return TRI_ERR_INVALID_ARG;
         const int old = p->opt_lookback;
@@ -730,13 +775,13 @@ void tri_plan_describe(tri_plan_t p, char* buf, int len) {
     snprintf(buf, len,
              "n=%lld m=%lld dtype=%s layout=%s variant=%s k=%d%s G=%d P=%d rpt=%d L=%lld C=%lld "
              "fu_grid=%d fu_son=%d fu_nc=%lld sk_grid=%d sk_nc=%d sk_son=%d mc_P=%d lookback=%d tma=%d scratch=%zu "
-             "sms=%d",
+             "sms=%d grid_Q=%d grid_R=%d",
              (long long)p->n, (long long)p->m, p->dtype == TRI_F64 ? "f64" : "f32",
              p->layout == TRI_LAYOUT_CONTIGUOUS ? "contiguous" : p->layout == TRI_LAYOUT_INTERLEAVED ? "interleaved"
              : p->layout == TRI_LAYOUT_BATCHED ? "batched" : (p->inner ? "strided(packed)" : "strided"),
              vn[p->variant], p->k, passes, p->G, p->P, p->rpt, (long long)p->L, (long long)p->C, p->fu_grid,
              p->fu_son, (long long)p->fu_nc, p->sk_grid, p->sk_nc, p->sk_son, p->mc_P, p->mc_lb ? p->mc_NCWs : 0,
-             p->opt_tma, p->scratch_bytes, p->sms);
+             p->opt_tma, p->scratch_bytes, p->sms, p->sg_Q, p->sg_R);
 }
 
 tri_status tri_solve(tri_plan_t p, const void* a, const void* b, const void* c, const void* d, void* x,
@@ -829,7 +874,8 @@ HostChunks host_chunks(const tri_plan_s* p) {
 tri_status make_sub(tri_plan_s* p, int i, int64_t mi) {
     if (p->sub[i] && p->sub_m[i] == mi && p->sub[i]->variant == (p->forced ? p->variant : p->sub[i]->variant) &&
         (!p->forced || p->sub[i]->k == p->k) && p->sub[i]->opt_tma == p->opt_tma &&
-        p->sub[i]->opt_lookback == p->opt_lookback && p->sub[i]->opt_cluster == p->opt_cluster)
+        p->sub[i]->opt_lookback == p->opt_lookback && p->sub[i]->opt_cluster == p->opt_cluster &&
+        p->sub[i]->opt_grid == p->opt_grid)
         return TRI_OK;
     tri_destroy(p->sub[i]);
     p->sub[i] = nullptr;
@@ -839,6 +885,7 @@ tri_status make_sub(tri_plan_s* p, int i, int64_t mi) {
     s->opt_tma = p->opt_tma;
     s->opt_lookback = p->opt_lookback;
     s->opt_cluster = p->opt_cluster;
+    s->opt_grid = p->opt_grid;
     if (p->forced) {
         if (!variant_ok(p->variant, s)) { tri_destroy(s); return TRI_ERR_INVALID_ARG; }
         st = set_plan(s, p->variant, p->k);

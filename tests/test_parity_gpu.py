@@ -1027,3 +1027,80 @@ def test_fp32_weak_accuracy(cuda_ok, n, m, layout, variant, lookback):
     xo = oracle.solve_batch(n, m, *arrs, layout=layout)
     from tests._helpers import max_rel_err
     assert max_rel_err(x, xo) <= 5e-5
+
+
+# ---------------------------------------------- interleaved SCAN split over the grid
+def _grid_qr(plan):
+    d = dict(kv.split("=") for kv in plan.describe().split() if "=" in kv)
+    return int(d["grid_Q"]), int(d["grid_R"])
+
+
+@pytest.mark.parametrize("dtype", ["f64", "f32"])
+@pytest.mark.parametrize("n,m", [(1024, 1024), (1000, 36), (1, 8), (5, 12), (60, 40), (257, 64), (700, 300),
+                                 (2048, 300), (2000, 32), (96, 4096), (1023, 100), (2048, 64)])
+def test_scan_grid_parity(cuda_ok, dtype, n, m):
+    """Interleaved SCAN through k_scan_grid (TRI_OPT_SCAN_GRID, the auto choice
+    where 32-system blocks x Q row pieces fit one CTA per SM): every element vs
+    the oracle for c2's shape, ragged last blocks (m % 32 != 0), rows past n in
+    the last piece and warp, 1 to 4 TMA stages per warp (R = 4 .. 16), Q = 1 ..
+    8 (thread-block clusters); repeated solves are bitwise identical; the
+    chained kernel (option 0) agrees."""
+    arrs = gen(n, m, dtype, 1, "weak", eps=1e-2)
+    xo = oracle.solve_batch(n, m, *arrs, layout=1)
+    plan = tri.Plan(n, m, tri.F64 if dtype == "f64" else tri.F32, 1)
+    plan.variant = tri.VARIANT_SCAN
+    Q, R = _grid_qr(plan)
+    assert Q > 0 and R in (4, 8, 12, 16)
+    xs = [gpu_solve(n, m, arrs, dtype, 1, plan=plan)[0] for _ in range(3)]
+    check_parity(n, m, arrs, xs[0], dtype, 1, x_oracle=xo)
+    assert np.array_equal(xs[0], xs[1]) and np.array_equal(xs[0], xs[2])
+    plan.set_option(tri.OPT_SCAN_GRID, 0)
+    assert _grid_qr(plan) == (0, 0)
+    x3, _ = gpu_solve(n, m, arrs, dtype, 1, plan=plan)
+    check_parity(n, m, arrs, x3, dtype, 1, x_oracle=xo)
+    plan.set_option(tri.OPT_SCAN_GRID, -1)
+    x4, _ = gpu_solve(n, m, arrs, dtype, 1, plan=plan)
+    assert np.array_equal(xs[0], x4)
+
+
+def test_scan_grid_graph_replay_and_variant_switch(cuda_ok):
+    """k_scan_grid under CUDA-graph replay (bench.py's timing) and after another
+    variant has run on the same plan: every replay matches the oracle."""
+    import torch
+    n, m = 1024, 1024
+    arrs = gen(n, m, "f64", 1)
+    xo = oracle.solve_batch(n, m, *arrs, layout=1)
+    plan = tri.Plan(n, m, tri.F64, 1)
+    assert _grid_qr(plan)[0] > 0
+    a, b, c, d = to_dev(*arrs)
+    x = torch.empty_like(a)
+    plan.solve(a, b, c, d, out=x)
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):
+        with torch.cuda.graph(g, stream=s):
+            plan.solve(a, b, c, d, out=x)
+    for _ in range(5):
+        x.fill_(float("nan"))
+        g.replay()
+        torch.cuda.synchronize()
+        check_parity(n, m, arrs, x.cpu().numpy(), "f64", 1, x_oracle=xo)
+    plan.variant = SPLIT
+    plan.solve(a, b, c, d, out=x)
+    plan.variant = tri.VARIANT_SCAN
+    assert _grid_qr(plan)[0] > 0
+    x.fill_(float("nan"))
+    plan.solve(a, b, c, d, out=x)
+    check_parity(n, m, arrs, x.cpu().numpy(), "f64", 1, x_oracle=xo)
+
+
+@pytest.mark.parametrize("dtype,n,ms,nb", [("f64", 100, 64, 7), ("f32", 333, 36, 9), ("f64", 1000, 18, 5)])
+def test_scan_grid_batched(cuda_ok, dtype, n, ms, nb):
+    """k_scan_grid on BATCHED y-lines [nb][n][ms] (blocks per batch, batch stride)."""
+    arrs, grid = _grid_lines(n, ms, nb, dtype, "weak")
+    plan = tri.Plan.batched(n, ms, nb, tri.F64 if dtype == "f64" else tri.F32)
+    assert _grid_qr(plan)[0] > 0
+    xg = plan.solve(*to_dev(*grid)).cpu().numpy()
+    x = np.ascontiguousarray(xg.reshape(nb, n, ms).transpose(0, 2, 1)).reshape(-1)
+    check_parity(n, ms * nb, arrs, x, dtype, 0)
