@@ -724,22 +724,41 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
     int j = 0, w = pw;
     while (w >= NC) { w -= NC; ++j; }
     if (lane == 0 && pw < nfwd) issue(j, w);
+    // per-step bookkeeping kept incrementally (no integer division in the loop):
+    // forward system j with jk = j % K, jt = j % 65535 + 1 (its tab row and tag);
+    // backward index b = g - NC - D = bj NC + br (0 <= br < NC; bj < 0 while b < 0)
+    int jk = j % K, jt = j % 65535 + 1;
+    int bjv, br;
+    {
+        const int b0 = pw - NC - D;
+        bjv = b0 >= 0 ? b0 / NC : -((-b0 + NC - 1) / NC);
+        br = b0 - bjv * NC;
+    }
+    int bk = ((bjv % K) + K) % K, bt = ((bjv % 65535) + 65535) % 65535 + 1;
     const int pi = (pw + SC_NW - 1) % SC_NW;  // warp of step g - 1
     unsigned long long pc[8] = {0, 0, 0, 0, 0, 0, 0, 0}, t0 = PROF ? clock64() : 0, tp = t0;
 #define SC_T(k) do { if (PROF) { const unsigned long long tn_ = clock64(); pc[k] += tn_ - tp; tp = tn_; } } while (0)
     for (int g = pw; g < total; g += SC_NW) {
-        const int cj = j, cw = w;
+        const int cj = j, cw = w, cjk = jk, cjt = jt;
         w += SC_NW;
-        while (w >= NC) { w -= NC; ++j; }
-        const int bb = g - NC - D;
-        const bool fwd = cj < nsys, bwd = bb >= 0;
-        const int bj = bwd ? bb / NC : 0;
-        const int wb = NC - 1 - (bb - bj * NC);  // backward window (system bj)
+        while (w >= NC) {
+            w -= NC; ++j;
+            jk = jk + 1 == K ? 0 : jk + 1;
+            jt = jt == 65535 ? 1 : jt + 1;
+        }
+        const int bj = bjv, bjk = bk, bjt = bt, wb = NC - 1 - br;  // backward window (system bj)
+        br += SC_NW;
+        while (br >= NC) {
+            br -= NC; ++bjv;
+            bk = bk + 1 == K ? 0 : bk + 1;
+            bt = bt == 65535 ? 1 : bt + 1;
+        }
+        const bool fwd = cj < nsys, bwd = bj >= 0;
         const int64_t i0d = (int64_t)cw * WR + seg * SC_R;
         int slot = g;                            // fresh slot (g < NS when !bwd)
         if (bwd && p.dbg != 2) {
             SC_T(5);
-            const unsigned tg = (unsigned)(bj % 65535 + 1);
+            const unsigned tg = (unsigned)bjt;
             // The window was stored >= delta + 1 steps ago by another warp, which
             // published its slot with release semantics after the stores; this acquire
             // load orders the slot reads after them (PTX memory model).  compute-sanitizer
@@ -748,7 +767,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
             // handoff); ordering by the handover barrier chain alone would need
             // delta >= 2 x warps, measured 3 % slower at c5 (more spilled slots reach
             // DRAM) and 8 % at c2 (a longer tail).
-            const int* e = reinterpret_cast<const int*>(&tab[(bj % K) * NC + wb]);
+            const int* e = reinterpret_cast<const int*>(&tab[bjk * NC + wb]);
             unsigned v = (unsigned)sk_ld_acquire(e);
             while ((v >> 16) != tg) {  // window (bj, wb) stored
                 __nanosleep(64);
@@ -878,8 +897,8 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
             else sc_store_slot_g(sp_g, lane, cpf, dpf, pol_sp);
             __syncwarp();
             if (lane == 0) {  // release: the warp's slot stores (ordered before by __syncwarp) first
-                sk_st_release(reinterpret_cast<int*>(&tab[(cj % K) * NC + cw]),
-                              (int)(((unsigned)(cj % 65535 + 1) << 16) | (unsigned)slot));
+                sk_st_release(reinterpret_cast<int*>(&tab[cjk * NC + cw]),
+                              (int)(((unsigned)cjt << 16) | (unsigned)slot));
             }
         }
         // ---- backward replay: x (Eq 4) of window (bj, wb)

@@ -10,14 +10,16 @@ sys.path.insert(0, ROOT)
 from paper_conf_icpp_kimwch11_b200 import _build as B  # noqa: E402
 
 name, extra = sys.argv[1], sys.argv[2:]
+# TRI_CSRC=dir: build another copy of the sources (e.g. a git revision exported for an A/B)
+CSRC = os.environ.get("TRI_CSRC", B.CSRC)
 out = os.path.join(ROOT, "build_var", name)
 os.makedirs(out, exist_ok=True)
 
 
 def comp(src):
     obj = os.path.join(out, src.replace(".cu", ".o"))
-    subprocess.check_call([B.NVCC, *B.ARCH, *B.FLAGS, *extra, "-I", B.INCLUDE, "-I", B.CSRC, "-c", "-o", obj,
-                           os.path.join(B.CSRC, src)], stderr=subprocess.DEVNULL)
+    subprocess.check_call([B.NVCC, *B.ARCH, *B.FLAGS, *extra, "-I", B.INCLUDE, "-I", CSRC, "-c", "-o", obj,
+                           os.path.join(CSRC, src)], stderr=subprocess.DEVNULL)
     return obj
 
 
