@@ -28,8 +28,12 @@ CASES = {
              (128, 40, "f32", 0, V.VARIANT_SCAN, None),      # short one-window systems (k_scan1)
              (1002, 3, "f64", 0, V.VARIANT_SCAN, None),      # ragged n, 16-byte pitch: tail rows from global
              (5003, 1, "f32", 0, V.VARIANT_SCAN, None)],     # ragged n, one system
-    "scan_il": [(1024, 16, "f64", 1, V.VARIANT_SCAN, None),  # interleaved, S = 8: two 8-system groups
-                (520, 24, "f32", 1, V.VARIANT_SCAN, None)],  # ragged last window
+    "scan_il": [(1024, 16, "f64", 1, V.VARIANT_SCAN, "grid0"),  # interleaved, S = 8: two 8-system groups
+                (520, 24, "f32", 1, V.VARIANT_SCAN, "grid0")],  # ragged last window (chained kernel)
+    # k_scan_grid: clusters of Q CTAs exchanging aggregates through DSMEM; ragged
+    # blocks (m % 32), rows past n, 1 / 3 / 4 stages per warp, Q = 1 .. 8
+    "scan_grid": [(1024, 40, "f64", 1, V.VARIANT_SCAN, None), (700, 36, "f32", 1, V.VARIANT_SCAN, None),
+                  (60, 12, "f64", 1, V.VARIANT_SCAN, None), (2000, 32, "f64", 1, V.VARIANT_SCAN, None)],
     "scan_r16": [(256, 40, "f32", 0, V.VARIANT_SCAN, None), (224, 33, "f32", 0, V.VARIANT_SCAN, None)],
     "scan_mc": [(1 << 16, 1, "f64", 0, V.VARIANT_SCAN_MC, None),
                 (40960, 2, "f32", 0, V.VARIANT_SCAN_MC, None),
@@ -64,6 +68,8 @@ def main():
             if isinstance(k, str) and k.startswith("tma0:"):  # TRI_OPT_TMA off, then k
                 plan.set_option(tri.OPT_TMA, 0)
                 plan.k = int(k[5:])
+            elif k == "grid0":  # interleaved SCAN through the chained kernel
+                plan.set_option(tri.OPT_SCAN_GRID, 0)
             elif isinstance(k, str):  # "lbW": SCAN_MC look-back with W-window chunks
                 plan.set_option(tri.OPT_SCAN_MC_LOOKBACK, int(k[2:]))
             elif k is not None:
