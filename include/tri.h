@@ -255,13 +255,18 @@ TRI_API tri_status tri_plan_set_variant(tri_plan_t plan, tri_variant v);
  *     in flight at once, and the Q CTAs of a block exchange their forward /
  *     backward aggregate maps through distributed shared memory; 0 = the
  *     chained 8-system-window kernel; 1 = as auto.
+ *   TRI_OPT_SCAN_W512 (default -1 = auto = on): fp64 CONTIGUOUS SCAN batches
+ *     with n % 16 == 0 and at least two 512-row windows run k_scan_w512 (16 rows
+ *     per lane, 512-row windows: the per-window scans and handover paid once
+ *     per 512 rows); 0 = the 256-row-window kernel; 1 = as auto.
  * TRI_ERR_INVALID_ARG for an unknown option or value; TRI_ERR_OOM if the new
  * geometry's scratch cannot be allocated (option unchanged). */
 typedef enum {
     TRI_OPT_TMA = 1,
     TRI_OPT_SCAN_MC_LOOKBACK = 2,
     TRI_OPT_SCAN_CLUSTER = 3,
-    TRI_OPT_SCAN_GRID = 4
+    TRI_OPT_SCAN_GRID = 4,
+    TRI_OPT_SCAN_W512 = 5
 } tri_option;
 TRI_API tri_status tri_plan_set_option(tri_plan_t plan, tri_option opt, int value);
 /* Human-readable one-line plan description into buf (NUL-terminated). */

@@ -18,7 +18,7 @@ CONTIGUOUS, INTERLEAVED, BATCHED, STRIDED = 0, 1, 2, 3
 (VARIANT_AUTO, VARIANT_ONCHIP, VARIANT_SPLIT, VARIANT_FUSED, VARIANT_WARP, VARIANT_STREAM, VARIANT_SCAN,
  VARIANT_SCAN_MC) = 0, 1, 2, 3, 4, 5, 6, 7
 VARIANT_NAMES = {1: "onchip", 2: "split", 3: "fused", 4: "warp", 5: "stream", 6: "scan", 7: "scan_mc"}
-OPT_TMA, OPT_SCAN_MC_LOOKBACK, OPT_SCAN_CLUSTER, OPT_SCAN_GRID = 1, 2, 3, 4
+OPT_TMA, OPT_SCAN_MC_LOOKBACK, OPT_SCAN_CLUSTER, OPT_SCAN_GRID, OPT_SCAN_W512 = 1, 2, 3, 4, 5
 STATUS = {0: "TRI_OK", 1: "TRI_ERR_INVALID_ARG", 2: "TRI_ERR_ALIGNMENT", 3: "TRI_ERR_ALIAS",
           4: "TRI_ERR_DEVICE", 5: "TRI_ERR_OOM", 6: "TRI_ERR_CUDA"}
 
@@ -199,7 +199,8 @@ class Plan:
         OPT_SCAN_MC_LOOKBACK (windows per look-back chunk, 0 = off),
         OPT_SCAN_CLUSTER (1 = interleaved SCAN through thread-block clusters),
         OPT_SCAN_GRID (0 = interleaved SCAN through the chained kernel, -1/1 = the
-        grid-split kernel where it fits)."""
+        grid-split kernel where it fits), OPT_SCAN_W512 (0 = fp64 contiguous SCAN
+        with 256-row windows, -1/1 = 512-row windows where n % 16 == 0)."""
         st = lib().tri_plan_set_option(self._h, int(opt), int(value))
         if st != 0:
             raise TriError(st, f"tri_plan_set_option({opt}, {value})")

@@ -8,6 +8,7 @@
 #include "k_scan_mc.cuh"
 #include "k_scan_cl.cuh"
 #include "k_scan_grid.cuh"
+#include "k_scan_w512.cuh"
 
 using namespace tri;
 
@@ -227,10 +228,43 @@ bool scan_grid_fits_t(const tri_plan_s* p, int Q, int R, int64_t nblk) {
     return (int64_t)ncl >= nblk;
 }
 
+// k_scan_w512 (the planner's s5): tensor view [m][n/16][16] (128-byte rows), box
+// [1][32][16] = one 512-row window of one array, 128B swizzle
+cudaError_t scan_w512_t(tri_plan_s* p, const void* a, const void* b, const void* c, const void* d, void* x,
+                        cudaStream_t st) {
+    StreamMaps tm;
+    const void* key[4] = {a, b, c, d};
+    if (!tm_lookup(p, 0x3008, key, 4, &tm.a, 4)) {
+        const void* src[4] = {a, b, c, d};
+        CUtensorMap* dst[4] = {&tm.a, &tm.b, &tm.c, &tm.d};
+        const uint64_t sys = p->m == 1 ? ((uint64_t)p->n * 8 + 15) / 16 * 16 : (uint64_t)p->n * 8;
+        for (int i = 0; i < 4; ++i) {
+            const uint64_t dims[3] = {16, (uint64_t)(p->n / 16), (uint64_t)p->m};
+            const uint64_t str[2] = {128, sys};
+            const uint32_t box[3] = {16, (uint32_t)(S5_W / 16), 1u};
+            if (!tma_encode(dst[i], 8, 3, src[i], dims, str, box, CU_TENSOR_MAP_SWIZZLE_128B))
+                return cudaErrorNotSupported;
+        }
+        tm_store(p, 0x3008, key, 4, &tm.a, 4);
+    }
+    ScanArgs<double> A{};
+    A.x = (double*)x;
+    A.spill = (double*)p->scratch;
+    A.n = p->n; A.m = p->m; A.ms = p->ms; A.NC = p->sk_nc; A.S_on = p->sk_son; A.delta = p->sk_delta;
+    A.xsys = p->ss; A.xbat = p->bs; A.xel = p->es; A.nb = 1;
+    A.x32 = ((uintptr_t)x % 32 == 0 && (p->ss * 8) % 32 == 0) ? 1 : 0;
+    const int smem = S5Layout::smem_bytes(p->sk_nc, p->sk_delta, p->sk_son);
+    cudaError_t e = set_smem((const void*)k_scan_w512<double>, smem);
+    if (e != cudaSuccess) return e;
+    k_scan_w512<double><<<p->sk_grid, S5_THREADS, smem, st>>>(tm, A);
+    return cudaGetLastError();
+}
+
 template <typename T>
 cudaError_t scan_t(tri_plan_s* p, const void* a, const void* b, const void* c, const void* d, void* x,
                    cudaStream_t st) {
     if (p->sg_Q > 0) return scan_grid_t<T>(p, a, b, c, d, x, st);
+    if (p->s5) return scan_w512_t(p, a, b, c, d, x, st);
     const int S = p->sk_S;
     const bool contig = p->layout == TRI_LAYOUT_CONTIGUOUS;  // the one-window kernels assume system stride n
     if constexpr (sizeof(T) == 4) {

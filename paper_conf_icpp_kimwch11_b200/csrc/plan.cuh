@@ -51,6 +51,7 @@ struct tri_plan_s {
     int opt_lookback = -1;        // TRI_OPT_SCAN_MC_LOOKBACK: windows per look-back chunk (0 = three passes, -1 = auto)
     int opt_cluster = 0;          // TRI_OPT_SCAN_CLUSTER: interleaved SCAN through thread-block clusters
     int opt_grid = -1;            // TRI_OPT_SCAN_GRID: interleaved SCAN split over the grid (k_scan_grid; -1 auto)
+    int opt_w512 = -1;            // TRI_OPT_SCAN_W512: fp64 contiguous SCAN with 512-row windows (k_scan_w512; -1 auto)
     int G = 0, P = 0, rpt = 0;    // ONCHIP geometry
     int64_t n_pad = 0, L = 0, C = 0;  // SPLIT: chain length, chains
     int npass = 0;                // SPLIT: tiled-PCR passes (0 at k = 0)
@@ -66,6 +67,7 @@ struct tri_plan_s {
     int sk_grid = 0, sk_nc = 0, sk_son = 0;  // STREAM / SCAN: persistent CTAs, windows per system, resident slots
     int sk_delta = 8;             // SCAN: back-substitution lag (steps)
     int sk_S = 1;                 // SCAN: systems per window (1 contiguous; 8 interleaved)
+    int s5 = 0;                   // SCAN through k_scan_w512 (sk_nc / sk_son then count 512-row windows / 8 KB slots)
     int sg_Q = 0, sg_R = 0, sg_bpb = 0;  // SCAN, k_scan_grid: CTAs per 32-system block, rows per warp, blocks per batch
     int64_t ms = 0;               // systems per batch (BATCHED / STRIDED; m otherwise)
     // element (system q = b ms + s, row i) at offset i es + s ss + b bs (elements) of

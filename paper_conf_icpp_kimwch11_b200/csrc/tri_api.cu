@@ -17,6 +17,7 @@
 #include "k_scan.cuh"
 #include "k_scan_mc.cuh"
 #include "k_scan_grid.cuh"
+#include "k_scan_w512.cuh"
 #include "k_stream.cuh"
 #include "k_tiled_pcr.cuh"
 #include "k_warp.cuh"
@@ -34,6 +35,9 @@ constexpr int64_t MAX_ELEMS = int64_t(1) << 40;
 // which the handover barrier chain alone would order every slot -- measured 3 %
 // slower at c5 and 8 % at c2, so the slots keep their release / acquire table)
 constexpr int SCAN_DELTA = 8;
+#ifndef S5_DELTA
+#define S5_DELTA 8                 // k_scan_w512's lag (A/B macro)
+#endif
 
 // ---- pure host planner ------------------------------------------------------
 // Rows of (normalised, 3-array) system data one ONCHIP CTA holds: sized for
@@ -298,6 +302,18 @@ void plan_geometry(tri_plan_s* p) {
         const int64_t avail = ((int64_t)p->smem_optin - (p->dtype == TRI_F64 ? fixed : fixed32)) / slot;
         p->sk_son = (p->sk_nc == 1 && p->sk_S == 1) ? 0 : (int)std::max<int64_t>(0, std::min<int64_t>(p->sk_nc + p->sk_delta, avail));
         scan_grid_geometry(p);
+        // fp64 contiguous batches of >= 2 windows of 512 rows (n % 16: the 128-byte
+        // tensor rows): k_scan_w512, 16 rows per lane (the per-window scans, handover
+        // and bookkeeping paid once per 512 rows)
+        p->s5 = 0;
+        if (p->opt_w512 != 0 && p->dtype == TRI_F64 && p->layout == TRI_LAYOUT_CONTIGUOUS && p->sk_S == 1 &&
+            p->n % 16 == 0 && cdiv(n, S5_W) >= 2 && cdiv(n, S5_W) <= SC_NCMAX) {
+            p->s5 = 1;
+            p->sk_nc = (int)cdiv(n, S5_W);
+            p->sk_delta = S5_DELTA;
+            const int64_t av5 = ((int64_t)p->smem_optin - S5Layout::smem_bytes(p->sk_nc, p->sk_delta, 0)) / S5Layout::slot_bytes;
+            p->sk_son = (int)std::max<int64_t>(0, std::min<int64_t>(p->sk_nc + p->sk_delta, av5));
+        }
     }
     if (p->variant == TRI_VARIANT_SCAN_MC) {
         p->L = n; p->n_pad = n; p->C = m;
@@ -349,6 +365,8 @@ size_t scratch_need(const tri_plan_s* p) {
                (p->mc_lb ? (size_t)p->m * (size_t)p->mc_Ps * (SMC_REC * 8 + 4) +
                                (size_t)p->m * (size_t)((p->mc_Ps + 31) / 32) * (8 * 8 + 4) + 256 : 0);
     if (p->variant == TRI_VARIANT_SCAN && p->sg_Q > 0) return 0;  // k_scan_grid: no global scratch
+    if (p->variant == TRI_VARIANT_SCAN && p->s5)  // k_scan_w512: spilled 8 KB slots per CTA
+        return (size_t)p->sk_grid * (size_t)std::max(0, p->sk_nc + p->sk_delta - p->sk_son) * S5Layout::slot_bytes;
     if (p->variant == TRI_VARIANT_SCAN)
         return (p->sk_nc == 1 && p->sk_S == 1) ? 0
                              : (size_t)p->sk_grid * (size_t)std::max(0, p->sk_nc + p->sk_delta - p->sk_son) *
@@ -685,6 +703,14 @@ tri_status tri_plan_set_option(tri_plan_t p, tri_option opt, int value) {
         p->tmc.clear();
         return TRI_OK;
     }
+    if (opt == TRI_OPT_SCAN_W512) {
+        if (value < -1 || value > 1) return TRI_ERR_INVALID_ARG;
+        const int old = p->opt_w512;
+        p->opt_w512 = value;
+        const tri_status st = set_plan(p, p->variant, p->k);
+        if (st != TRI_OK) { p->opt_w512 = old; plan_geometry(p); }
+        return st;
+    }
     if (opt == TRI_OPT_SCAN_GRID) {
         if (value < -1 || value > 1) return TRI_ERR_INVALID_ARG;
         const int old = p->opt_grid;
@@ -775,13 +801,13 @@ void tri_plan_describe(tri_plan_t p, char* buf, int len) {
     snprintf(buf, len,
              "n=%lld m=%lld dtype=%s layout=%s variant=%s k=%d%s G=%d P=%d rpt=%d L=%lld C=%lld "
              "fu_grid=%d fu_son=%d fu_nc=%lld sk_grid=%d sk_nc=%d sk_son=%d mc_P=%d lookback=%d tma=%d scratch=%zu "
-             "sms=%d grid_Q=%d grid_R=%d",
+             "sms=%d grid_Q=%d grid_R=%d w512=%d",
              (long long)p->n, (long long)p->m, p->dtype == TRI_F64 ? "f64" : "f32",
              p->layout == TRI_LAYOUT_CONTIGUOUS ? "contiguous" : p->layout == TRI_LAYOUT_INTERLEAVED ? "interleaved"
              : p->layout == TRI_LAYOUT_BATCHED ? "batched" : (p->inner ? "strided(packed)" : "strided"),
              vn[p->variant], p->k, passes, p->G, p->P, p->rpt, (long long)p->L, (long long)p->C, p->fu_grid,
              p->fu_son, (long long)p->fu_nc, p->sk_grid, p->sk_nc, p->sk_son, p->mc_P, p->mc_lb ? p->mc_NCWs : 0,
-             p->opt_tma, p->scratch_bytes, p->sms, p->sg_Q, p->sg_R);
+             p->opt_tma, p->scratch_bytes, p->sms, p->sg_Q, p->sg_R, p->s5);
 }
 
 tri_status tri_solve(tri_plan_t p, const void* a, const void* b, const void* c, const void* d, void* x,
@@ -875,7 +901,7 @@ tri_status make_sub(tri_plan_s* p, int i, int64_t mi) {
     if (p->sub[i] && p->sub_m[i] == mi && p->sub[i]->variant == (p->forced ? p->variant : p->sub[i]->variant) &&
         (!p->forced || p->sub[i]->k == p->k) && p->sub[i]->opt_tma == p->opt_tma &&
         p->sub[i]->opt_lookback == p->opt_lookback && p->sub[i]->opt_cluster == p->opt_cluster &&
-        p->sub[i]->opt_grid == p->opt_grid)
+        p->sub[i]->opt_grid == p->opt_grid && p->sub[i]->opt_w512 == p->opt_w512)
         return TRI_OK;
     tri_destroy(p->sub[i]);
     p->sub[i] = nullptr;
@@ -886,6 +912,7 @@ tri_status make_sub(tri_plan_s* p, int i, int64_t mi) {
     s->opt_lookback = p->opt_lookback;
     s->opt_cluster = p->opt_cluster;
     s->opt_grid = p->opt_grid;
+    s->opt_w512 = p->opt_w512;
     if (p->forced) {
         if (!variant_ok(p->variant, s)) { tri_destroy(s); return TRI_ERR_INVALID_ARG; }
         st = set_plan(s, p->variant, p->k);

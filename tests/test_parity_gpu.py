@@ -1104,3 +1104,28 @@ def test_scan_grid_batched(cuda_ok, dtype, n, ms, nb):
     xg = plan.solve(*to_dev(*grid)).cpu().numpy()
     x = np.ascontiguousarray(xg.reshape(nb, n, ms).transpose(0, 2, 1)).reshape(-1)
     check_parity(n, ms * nb, arrs, x, dtype, 0)
+
+
+# ------------------------------------------ fp64 contiguous SCAN with 512-row windows
+@pytest.mark.parametrize("n,m", [(16384, 40), (1024, 300), (1040, 64), (8192, 5), (4112, 7), (16384, 1),
+                                 (528, 150), (65536, 3)])
+@pytest.mark.parametrize("family", ["dd", "weak"])
+def test_scan_w512_parity(cuda_ok, n, m, family):
+    """k_scan_w512 (TRI_OPT_SCAN_W512, auto for fp64 contiguous n % 16 == 0 with
+    >= 2 windows of 512 rows): every element vs the oracle; 2 .. 128 windows, a
+    ragged last window (n % 512 != 0), one system (several windows per warp
+    step), more systems than CTAs; repeated solves bitwise identical; the
+    256-row-window kernel (option 0) agrees within the tolerance."""
+    arrs = gen(n, m, "f64", 0, family, eps=1e-2)
+    xo = oracle.solve_batch(n, m, *arrs)
+    plan = tri.Plan(n, m, tri.F64, 0)
+    plan.variant = tri.VARIANT_SCAN
+    assert "w512=1" in plan.describe()
+    x, _ = gpu_solve(n, m, arrs, "f64", 0, plan=plan)
+    check_parity(n, m, arrs, x, "f64", 0, x_oracle=xo)
+    x2, _ = gpu_solve(n, m, arrs, "f64", 0, plan=plan)
+    assert np.array_equal(x, x2)
+    plan.set_option(tri.OPT_SCAN_W512, 0)
+    assert "w512=0" in plan.describe()
+    x3, _ = gpu_solve(n, m, arrs, "f64", 0, plan=plan)
+    check_parity(n, m, arrs, x3, "f64", 0, x_oracle=xo)
