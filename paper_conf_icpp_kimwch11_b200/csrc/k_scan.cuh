@@ -370,10 +370,11 @@ __device__ __forceinline__ void sc_scans(SCM& M, T& al, T& be, int lane) {
 #pragma unroll
     for (int dd = S; dd < 32; dd <<= 1) {
         const SCM o = sk_shfl_up(M, dd);
-        T oa = __shfl_down_sync(0xffffffffu, al, dd), ob = __shfl_down_sync(0xffffffffu, be, dd);
-        if (lane + dd >= 32) { oa = T(0); ob = T(1); }
-        al = fma(be, oa, al);
-        be = be * ob;
+        const T oa = __shfl_down_sync(0xffffffffu, al, dd), ob = __shfl_down_sync(0xffffffffu, be, dd);
+        if (lane + dd < 32) {  // predicated in place (no selects)
+            al = fma(be, oa, al);
+            be = be * ob;
+        }
         if (lane >= dd) M = sk_compose(M, o);
     }
 }

@@ -87,11 +87,14 @@ __device__ __forceinline__ void s5_ld_group(const double* ib, int lane, int h, d
     }
 }
 
-// group fix-ups: a_0, c_{n-1} outside A; identity rows past n (edge windows only);
-// then renormalise the group if a live pivot leaves 2^+-64 (warp-uniform)
-__device__ __forceinline__ void s5_fix_group(bool edge, int64_t i0, int64_t n, double (&a)[S5_G], double (&b)[S5_G],
-                                             double (&c)[S5_G], double (&d)[S5_G]) {
-    if (edge) {
+// group fix-ups: a_0, c_{n-1} outside A; identity rows past n (edge windows only).
+// Then the range decision (fp64 raw rows, X21): `scl` bit h set = renormalise
+// group h by 2^-exponent(b) because a live pivot leaves 2^+-64; the map pass
+// takes the decision (warp-uniform), the replay pass reuses it (bit known).
+__device__ __forceinline__ void s5_fix_group(bool edge, int64_t i0, int64_t n, int h, unsigned& scl, bool decide,
+                                             double (&a)[S5_G], double (&b)[S5_G], double (&c)[S5_G],
+                                             double (&d)[S5_G]) {
+    if (__builtin_expect(edge, 0)) {
 #pragma unroll
         for (int u = 0; u < S5_G; ++u) {
             const int64_t i = i0 + u;
@@ -100,13 +103,17 @@ __device__ __forceinline__ void s5_fix_group(bool edge, int64_t i0, int64_t n, d
             if (i >= n) { a[u] = 0.0; b[u] = 1.0; c[u] = 0.0; d[u] = 0.0; }
         }
     }
-    bool out = false;
+    if (decide) {
+        unsigned mx = 0u, mn = 0xffffffffu;
 #pragma unroll
-    for (int u = 0; u < S5_G; ++u) {
-        const unsigned hb = (unsigned)__double2hiint(b[u]) & 0x7ff00000u;
-        out |= hb - ((1023u - 64u) << 20) > (128u << 20);
+        for (int u = 0; u < S5_G; ++u) {
+            const unsigned hb = (unsigned)__double2hiint(b[u]) & 0x7ff00000u;
+            mx = max(mx, hb);
+            mn = min(mn, hb);
+        }
+        if (__any_sync(0xffffffffu, mx > ((1023u + 64u) << 20) || mn < ((1023u - 64u) << 20))) scl |= 1u << h;
     }
-    if (__any_sync(0xffffffffu, out)) {
+    if (scl & (1u << h)) {
 #pragma unroll
         for (int u = 0; u < S5_G; ++u) {
             const double s = sk_exp2_scale(b[u]);
@@ -224,6 +231,7 @@ __global__ void __launch_bounds__(S5_THREADS, 1) k_scan_w512(const __grid_consta
         const int64_t i0 = (int64_t)cw * S5_W + lane * S5_R;
         const bool edge = cw == 0 || (int64_t)(cw + 1) * S5_W > n;
         SCM M{1.0, 0.0, 0.0, 1.0, 0.0, 0.0, 1.0};
+        unsigned scl = 0u;  // per 4-row group: renormalised (decided by the map pass)
         if (fwd) {
             sk_wait(&in_full[pw], ph);
             ph ^= 1u;
@@ -232,7 +240,7 @@ __global__ void __launch_bounds__(S5_THREADS, 1) k_scan_w512(const __grid_consta
             for (int h = 0; h < S5_R / S5_G; ++h) {
                 double ra[S5_G], rb[S5_G], rc[S5_G], rd[S5_G];
                 s5_ld_group(ib, lane, h, ra, rb, rc, rd);
-                s5_fix_group(edge, i0 + h * S5_G, n, ra, rb, rc, rd);
+                s5_fix_group(edge, i0 + h * S5_G, n, h, scl, true, ra, rb, rc, rd);
 #pragma unroll
                 for (int u = 0; u < S5_G; ++u) {
                     const double au = ra[u], bu = rb[u], cu = rc[u], du = rd[u];
@@ -295,7 +303,7 @@ __global__ void __launch_bounds__(S5_THREADS, 1) k_scan_w512(const __grid_consta
             for (int h = 0; h < S5_R / S5_G; ++h) {
                 double ra[S5_G], rb[S5_G], rc[S5_G], rd[S5_G];
                 s5_ld_group(ib, lane, h, ra, rb, rc, rd);
-                s5_fix_group(edge, i0 + h * S5_G, n, ra, rb, rc, rd);
+                s5_fix_group(edge, i0 + h * S5_G, n, h, scl, false, ra, rb, rc, rd);
                 if (h == S5_R / S5_G - 1) {  // the buffer's last read: refill it
                     sc_release_buf();
                     if (lane == 0 && g + S5_NW < nfwd) issue(j, w);
