@@ -254,7 +254,8 @@ TRI_API tri_status tri_plan_set_variant(tri_plan_t plan, tri_variant v);
  *     k_scan_grid: each lane owns one system's run of rows, the whole batch is
  *     in flight at once, and the Q CTAs of a block exchange their forward /
  *     backward aggregate maps through distributed shared memory; 0 = the
- *     chained 8-system-window kernel; 1 = as auto.
+ *     chained 8-system-window kernel; 1 = also batches of several waves
+ *     (Q <= 8; measured slower than the chained kernel beyond one wave).
  *   TRI_OPT_SCAN_W512 (default -1 = auto = on): fp64 CONTIGUOUS SCAN batches
  *     with n % 16 == 0 and at least two 512-row windows run k_scan_w512 (16 rows
  *     per lane, 512-row windows: the per-window scans and handover paid once

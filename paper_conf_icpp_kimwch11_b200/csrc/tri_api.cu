@@ -247,6 +247,18 @@ void scan_grid_geometry(tri_plan_s* p) {
             return;
         }
     }
+    // TRI_OPT_SCAN_GRID 1: also batches of several waves (clusters are independent:
+    // no co-residency needed), with the longest runs per warp (fewest CTAs)
+    if (p->opt_grid == 1) {
+        const int64_t Q = cdiv(p->n, (int64_t)SG_NW * SG_RMAX);
+        if (Q <= SG_QMAX) {
+            int R = SG_SR;
+            while (cdiv(p->n, (int64_t)SG_NW * R) > Q) R += SG_SR;
+            p->sg_Q = (int)Q;
+            p->sg_R = R;
+            p->sg_bpb = (int)bpb;
+        }
+    }
 }
 
 void plan_geometry(tri_plan_s* p) {

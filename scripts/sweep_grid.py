@@ -38,20 +38,25 @@ def time_plan(plan, a, b, c, d, x, reps=15):
     return sorted(ts)[len(ts) // 2]
 
 
-for n in (64, 128, 256, 512, 1024, 2048):
-    for m in (64, 128, 256, 512, 1024, 2048, 4096):
-        plan = tri.Plan(n, m, TD, 1)
-        plan.variant = tri.VARIANT_SCAN
-        d_ = dict(kv.split("=") for kv in plan.describe().split() if "=" in kv)
-        if int(d_["grid_Q"]) == 0:
-            continue
-        arrs = trigen.generate(n, m, DT, 1, "dd")
-        a, b, c, d = (torch.from_numpy(t).cuda() for t in arrs)
-        x = torch.empty_like(b)
-        tg = time_plan(plan, a, b, c, d, x)
-        plan.set_option(tri.OPT_SCAN_GRID, 0)
-        tc = time_plan(plan, a, b, c, d, x)
-        auto = tri.Plan(n, m, TD, 1)
-        ta = time_plan(auto, a, b, c, d, x)
-        print(json.dumps({"n": n, "m": m, "dtype": DT, "Q": int(d_["grid_Q"]), "R": int(d_["grid_R"]), "grid_us": round(tg, 2),
-                          "chained_us": round(tc, 2), "auto_variant": auto.variant, "auto_us": round(ta, 2)}), flush=True)
+def main():
+    for n in (64, 128, 256, 512, 1024, 2048):
+      for m in (64, 128, 256, 512, 1024, 2048, 4096):
+          plan = tri.Plan(n, m, TD, 1)
+          plan.variant = tri.VARIANT_SCAN
+          d_ = dict(kv.split("=") for kv in plan.describe().split() if "=" in kv)
+          if int(d_["grid_Q"]) == 0:
+              continue
+          arrs = trigen.generate(n, m, DT, 1, "dd")
+          a, b, c, d = (torch.from_numpy(t).cuda() for t in arrs)
+          x = torch.empty_like(b)
+          tg = time_plan(plan, a, b, c, d, x)
+          plan.set_option(tri.OPT_SCAN_GRID, 0)
+          tc = time_plan(plan, a, b, c, d, x)
+          auto = tri.Plan(n, m, TD, 1)
+          ta = time_plan(auto, a, b, c, d, x)
+          print(json.dumps({"n": n, "m": m, "dtype": DT, "Q": int(d_["grid_Q"]), "R": int(d_["grid_R"]), "grid_us": round(tg, 2),
+                            "chained_us": round(tc, 2), "auto_variant": auto.variant, "auto_us": round(ta, 2)}), flush=True)
+
+
+if __name__ == "__main__":
+    main()
