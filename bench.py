@@ -495,7 +495,8 @@ def main():
         with open(tf) as fh:
             tj = json.load(fh)
         if tj.get("n") == n and tj.get("m") == mr and tj.get("k") == plan.k and \
-                tj.get("variant", plan.variant) == plan.variant and tj.get("layout", layout) == layout:
+                tj.get("variant", plan.variant) == plan.variant and tj.get("layout", layout) == layout and \
+                all(t in plan.describe().split() for t in tj.get("describe_has", [])):
             traffic = tj.get("dram_bytes_per_launch")
             traffic_src = tj.get("source", tf)
             break
