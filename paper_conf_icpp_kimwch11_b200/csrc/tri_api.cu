@@ -264,6 +264,8 @@ void scan_grid_geometry(tri_plan_s* p) {
 void plan_geometry(tri_plan_s* p) {
     const int64_t n = p->n, m = p->m;
     p->tmc.clear();
+    p->s5 = 0;  // SCAN kernel choices: set again below when the variant is SCAN
+    p->sg_Q = p->sg_R = p->sg_bpb = 0;
     if (p->variant == TRI_VARIANT_WARP) {
         int R = 1;
         while (32 * (int64_t)R < n) R *= 2;

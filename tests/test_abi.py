@@ -181,3 +181,22 @@ included) timed on a
     geo = math.exp(sum(math.log(q) for q in ratios) / len(ratios))
     assert geo <= 1.05, geo
     assert max(ratios) <= 1.6, max(ratios)
+
+
+def test_planner_grid_rule_matches_sweeps(L):
+    """Interleaved SCAN through k_scan_grid (one wave of 32-system blocks x <= 8
+    row pieces): on every swept shape with n > 256 where it fits
+    (profiles/r02_sweep_grid_f64.jsonl, L2 flushed per replay) the planner picks
+    SCAN and the grid kernel is no slower than the chained kernel (within the
+    event timer's 2 us quantum); beyond one wave (r02_sweep_grid_multiwave_*) the
+    chained kernel wins on the larger shapes, which is why the rule stops at one wave."""
+    import json
+    one = [json.loads(x) for x in open(os.path.join(ROOT, "profiles", "r02_sweep_grid_f64.jsonl"))]
+    one = [r for r in one if r["n"] > 256]
+    assert len(one) >= 10
+    for r in one:
+        assert tri.choose_variant(r["n"], r["m"], tri.F64, 1, 148) == tri.VARIANT_SCAN, r
+        assert r["grid_us"] <= r["chained_us"] + 2.1, r
+    multi = [json.loads(x) for x in open(os.path.join(ROOT, "profiles", "r02_sweep_grid_multiwave_f64.jsonl"))]
+    big = [r for r in multi if (r["m"] + 31) // 32 * r["Q"] > 2 * 148]
+    assert big and all(r["grid_us"] > r["chained_us"] for r in big)
