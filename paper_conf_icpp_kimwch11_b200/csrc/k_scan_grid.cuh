@@ -414,12 +414,23 @@ __global__ void __launch_bounds__(SG_THREADS, 1) k_scan_grid(const __grid_consta
     // ---- phase D: back substitution (Eq 4) and the x stores
     if (live_w) {
         double x = fma(X(1, lane, warp), cst[96 + lane], X(0, lane, warp));  // x after the warp's rows
-        T* xo = p.x + (int64_t)bt * p.xbat + sys;
-        const bool full = r0 + R <= n;  // warp-uniform: no row past n
+        const int64_t xel = p.xel;
+        // the warp's last row; walked backwards one row stride at a time
+        T* xp = p.x + (int64_t)bt * p.xbat + sys + (int64_t)(r0 + R - 1) * xel;
+        if (r0 + R <= n) {  // warp-uniform: no row past n
 #pragma unroll
-        for (int t = R - 1; t >= 0; --t) {
-            x = fma(-cp[t], x, dp[t]);
-            if (live_sys && (full || r0 + t < n)) __stcs(xo + (int64_t)(r0 + t) * p.xel, (T)x);
+            for (int t = R - 1; t >= 0; --t) {
+                x = fma(-cp[t], x, dp[t]);
+                if (live_sys) __stcs(xp, (T)x);
+                xp -= xel;
+            }
+        } else {
+#pragma unroll
+            for (int t = R - 1; t >= 0; --t) {
+                x = fma(-cp[t], x, dp[t]);
+                if (live_sys && r0 + t < n) __stcs(xp, (T)x);
+                xp -= xel;
+            }
         }
     }
 
