@@ -42,6 +42,12 @@ struct ScanMCArgs {
     // of the slice (null: the system's start, (1, 0, 0)); xe = x after the slice
     // (null: 0, the system's end)
     int keep_a0, keep_cn;
+    // L2 reuse between the passes: pass 0 loads the last `keep0` windows it reads of
+    // its chunk (the chunk start, which pass 1 reads first) with evict_last; pass 1
+    // stores c', d' of the last `keep1` windows it writes (the chunk end, which pass 2
+    // reads first) with evict_last; 0 = plain policies
+    int keep0, keep1;
+    int discard;  // pass 2 discards each window's (c', d') L2 lines after reading them
     int w128;     // tensor view with 128-byte rows (k_scan.cuh)
     int x32;      // fp64: x rows 32-byte aligned (256-bit stores)
     const T* s0;
@@ -153,6 +159,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant
     // pass 0 keeps its lines (evict_normal): the chunk starts it reads last are
     // what pass 1 reads first; pass 1 is the inputs' last use (evict_first)
     const uint64_t pol_in = MODE == 0 ? sk_policy_evict_normal() : sk_policy_evict_first();
+    const uint64_t pol_keep = sk_policy_evict_last();
     // pass 0 and pass 2 walk their chunk backwards, pass 1 forwards: each pass
     // starts where the previous one ended, so the windows still in L2 (the last
     // ~100 MB a pass touched, at the same end of every chunk) are read first
@@ -161,11 +168,12 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant
         const int w = win_of(g);
         if (MODE < 2) {
             const int y = w * (p.w128 ? SC_W * (int)sizeof(T) / 128 : SC_W / 8);
+            const uint64_t pl = (MODE == 0 && g >= nwin - p.keep0) ? pol_keep : pol_in;
             sk_expect(&in_full[pw], (unsigned)(4 * SC_W * sizeof(T)));
-            sc_tma3d(ib + 0 * SC_W, &tm.a, y, (int)q, &in_full[pw], pol_in);
-            sc_tma3d(ib + 1 * SC_W, &tm.b, y, (int)q, &in_full[pw], pol_in);
-            sc_tma3d(ib + 2 * SC_W, &tm.c, y, (int)q, &in_full[pw], pol_in);
-            sc_tma3d(ib + 3 * SC_W, &tm.d, y, (int)q, &in_full[pw], pol_in);
+            sc_tma3d(ib + 0 * SC_W, &tm.a, y, (int)q, &in_full[pw], pl);
+            sc_tma3d(ib + 1 * SC_W, &tm.b, y, (int)q, &in_full[pw], pl);
+            sc_tma3d(ib + 2 * SC_W, &tm.c, y, (int)q, &in_full[pw], pl);
+            sc_tma3d(ib + 3 * SC_W, &tm.d, y, (int)q, &in_full[pw], pl);
         } else {
             const unsigned bytes = (unsigned)(sc_slot_elems<T>() * sizeof(T));
             sk_expect(&in_full[pw], bytes);
@@ -283,7 +291,17 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant
             if (tr) sc_fwd_replay_n(ra, rb, rc, rd, th, ps, de, cp, dp, nvalid);
             else sc_fwd_replay(ra, rb, rc, rd, th, ps, de, cp, dp);
             T* dst = p.cd + (q * NC + w) * (int64_t)sc_slot_elems<T>();
-            if constexpr (sizeof(T) == 8) {
+            if (g >= nwin - p.keep1) {  // read first by pass 2: keep in L2
+                if constexpr (sizeof(T) == 8) {
+#pragma unroll
+                    for (int t = 0; t < SC_R; ++t) sk_st_global_last(dst + 2 * sc_chunk<T>(lane, t), cp[t], dp[t], pol_keep);
+                } else {
+#pragma unroll
+                    for (int t = 0; t < SC_R / 2; ++t)
+                        sc_stg4_last(dst + 4 * sc_chunk<T>(lane, t), cp[2 * t], dp[2 * t], cp[2 * t + 1], dp[2 * t + 1],
+                                     pol_keep);
+                }
+            } else if constexpr (sizeof(T) == 8) {
 #pragma unroll
                 for (int t = 0; t < SC_R; ++t)
                     __stcg(reinterpret_cast<double2*>(dst + 2 * sc_chunk<T>(lane, t)), make_double2(cp[t], dp[t]));
@@ -306,6 +324,15 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant
             // ---- back substitution in reverse window order, x handed over
             T cp[SC_R], dp[SC_R];
             sc_load_slot_s(ib_s, lane, cp, dp);
+            if (p.discard) {
+                // the scratch copy of (c', d') is dead after this read: drop its L2 lines
+                // without a write-back (pass 1 leaves the chunk ends dirty in L2)
+                constexpr int lines = (int)(sc_slot_elems<T>() * sizeof(T) / 128);
+                if (lane < lines) {
+                    const T* src = p.cd + (q * NC + w) * (int64_t)sc_slot_elems<T>() + lane * (128 / (int)sizeof(T));
+                    asm volatile("discard.global.L2 [%0], 128;" ::"l"(src) : "memory");
+                }
+            }
             sc_release_buf();  // this warp's reads of the buffer before the TMA refill
             if (lane == 0 && g + SC_NW < nwin) issue(g + SC_NW);
             T al, be;

@@ -10,6 +10,13 @@
 #include "k_scan_grid.cuh"
 #include "k_scan_w512.cuh"
 
+#ifndef SMC_DISCARD
+#define SMC_DISCARD 1            // SCAN_MC pass 2: discard the read (c', d') lines (A/B macro)
+#endif
+#ifndef SMC_KEEP_MB
+#define SMC_KEEP_MB 64           // SCAN_MC: L2 megabytes kept between passes (A/B macro)
+#endif
+
 using namespace tri;
 
 namespace trih {
@@ -372,6 +379,17 @@ cudaError_t scan_mc_setup(tri_plan_s* p, const void* a, const void* b, const voi
     A.cmap = reinterpret_cast<double*>(A.cd + p->m * (int64_t)p->sk_nc * sc_slot_elems<T>());  // 2 KB multiples
     A.cbm = A.cmap + 8 * mp;
     A.n = p->n; A.m = p->m; A.NC = p->sk_nc; A.NCW = p->mc_NCW; A.P = p->mc_P;
+    // L2 reuse between the passes (~SMC_KEEP_MB of each pass's last data per pass;
+    // only when the system does not fit L2 anyway)
+    {
+        const int64_t kb = (int64_t)SMC_KEEP_MB << 20;
+        const int64_t in_w = 4 * SC_W * (int64_t)sizeof(T), cd_w = (int64_t)sc_slot_elems<T>() * sizeof(T);
+        const int64_t chunks = p->m * (int64_t)p->mc_P;
+        const bool big = chunks * p->mc_NCW * in_w > 2 * kb;
+        A.keep0 = big ? (int)std::min<int64_t>(p->mc_NCW, kb / (chunks * in_w)) : 0;
+        A.keep1 = big ? (int)std::min<int64_t>(p->mc_NCW, kb / (chunks * cd_w)) : 0;
+        A.discard = SMC_DISCARD;
+    }
     smem = SMCLayout<T>::smem_bytes(p->mc_NCW);
     for (auto k : {k_scan_mc<T, 0>, k_scan_mc<T, 1>, k_scan_mc<T, 2>}) {
         cudaError_t e = set_smem((const void*)k, smem);
