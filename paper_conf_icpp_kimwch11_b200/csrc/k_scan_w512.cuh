@@ -265,6 +265,15 @@ __global__ void __launch_bounds__(S5_THREADS, 1) k_scan_w512(const __grid_consta
             al = fma(-cpb[t], al, dpb[t]);
             be = -cpb[t] * be;
         }
+        if (bwd && !fwd && !res) {
+            // draining steps: this spilled slot is never written again in this solve;
+            // its (c', d') are in registers (used above), so drop its dirty L2 lines
+            // instead of letting them be written back during the next solve
+            __syncwarp();
+#pragma unroll
+            for (int k = 0; k < L::slot_bytes / 128 / 32; ++k)
+                asm volatile("discard.global.L2 [%0], 128;" ::"l"(sp_g + (k * 32 + lane) * 16) : "memory");
+        }
         sc_scans<1>(M, al, be, lane);
 
         // ---- the serial steps: the forward state and x of step g - 1 (named barrier 1 + pi)
