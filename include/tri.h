@@ -145,8 +145,9 @@ TRI_API void tri_debug_set_profile(void* dev_counters);
 /* Autotune the plan (the paper tunes its transition point once per machine,
  * P:743): time every feasible (variant, k) for the plan's
  * shape on the caller's device buffers (same rules as tri_solve; x is
- * overwritten), `reps` solves each after one warm-up, CUDA events on `stream`,
- * and keep the fastest in the plan.  Candidates whose scratch cannot be
+ * overwritten) -- for SCAN also with TRI_OPT_SCAN_GRID / TRI_OPT_SCAN_W512 off
+ * where the planner's geometry uses those kernels -- `reps` solves each after
+ * one warm-up, CUDA events on `stream`, and keep the fastest in the plan.  Candidates whose scratch cannot be
  * allocated are skipped.  *best_us (may be NULL) receives the fastest mean
  * time per solve in microseconds.  Synchronises `stream`. */
 TRI_API tri_status tri_plan_autotune(tri_plan_t plan, const void* a, const void* b, const void* c,

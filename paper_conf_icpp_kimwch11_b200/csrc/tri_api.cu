@@ -775,28 +775,41 @@ tri_status tri_plan_autotune(tri_plan_t p, const void* a, const void* b, const v
     float best = -1.f;
     tri_variant bv = p->variant;
     int bk = p->k;
+    const int og = p->opt_grid, ow = p->opt_w512;
+    int bg = og, bw = ow;
+    auto time_it = [&](tri_variant v, int k) {
+        if (set_plan(p, v, k) != TRI_OK) { cudaGetLastError(); return; }
+        if (tri_solve(p, a, b, c, d, x, stream) != TRI_OK) { cudaGetLastError(); return; }  // warm-up
+        cudaEventRecord(e0, s);
+        bool ok = true;
+        for (int r = 0; r < reps && ok; ++r) ok = tri_solve(p, a, b, c, d, x, stream) == TRI_OK;
+        cudaEventRecord(e1, s);
+        if (!ok || cudaEventSynchronize(e1) != cudaSuccess) { cudaGetLastError(); return; }
+        float ms = 0.f;
+        cudaEventElapsedTime(&ms, e0, e1);
+        const float us = ms * 1e3f / reps;
+        if (best < 0.f || us < best) { best = us; bv = v; bk = k; bg = p->opt_grid; bw = p->opt_w512; }
+    };
     for (tri_variant v : vs) {
         if (!variant_ok(v, p)) continue;
         // SPLIT / ONCHIP run any k; the sweep stops at 15 (deeper k only shortens
         // chains below 2^(log2 n - 15) rows, never faster on the sweep grid)
         const int k0 = kmin_for(v), k1 = std::min(kmax_for(v, p->n), 15);
         for (int k = k0; k <= k1; ++k) {
-            if (set_plan(p, v, k) != TRI_OK) { cudaGetLastError(); continue; }
-            if (tri_solve(p, a, b, c, d, x, stream) != TRI_OK) { cudaGetLastError(); continue; }  // warm-up
-            cudaEventRecord(e0, s);
-            bool ok = true;
-            for (int r = 0; r < reps && ok; ++r) ok = tri_solve(p, a, b, c, d, x, stream) == TRI_OK;
-            cudaEventRecord(e1, s);
-            if (!ok || cudaEventSynchronize(e1) != cudaSuccess) { cudaGetLastError(); continue; }
-            float ms = 0.f;
-            cudaEventElapsedTime(&ms, e0, e1);
-            const float us = ms * 1e3f / reps;
-            if (best < 0.f || us < best) { best = us; bv = v; bk = k; }
+            p->opt_grid = og; p->opt_w512 = ow;
+            time_it(v, k);
+            if (v == TRI_VARIANT_SCAN) {  // SCAN's kernel choices: the cluster / 512-row kernels or not
+                const bool grid = p->sg_Q > 0, w512 = p->s5 != 0;
+                if (grid) { p->opt_grid = 0; time_it(v, k); p->opt_grid = og; }
+                if (w512) { p->opt_w512 = 0; time_it(v, k); p->opt_w512 = ow; }
+            }
         }
     }
     cudaEventDestroy(e0);
     cudaEventDestroy(e1);
     if (best < 0.f) return TRI_ERR_CUDA;
+    p->opt_grid = bg;
+    p->opt_w512 = bw;
     st = set_plan(p, bv, bk);
     if (best_us) *best_us = best;
     return st;
