@@ -15,9 +15,10 @@
 // SM), the handover between warps, the slot table and the TMA issue.  With 16
 // rows per lane a window holds 512 rows, so that work is paid once per 512 rows
 // (ncu at c5: 740 M warp instructions instead of 1104 M).  The rows are streamed
-// from the staging buffer 4 at a time (they do not all fit in registers), the
+// from the staging buffer 8 at a time (they do not all fit in registers; 8-row
+// groups measured 0.8 % faster than 4-row ones), the
 // lane's forward map is rescaled by an exact power of two every 8 rows (raw fp64
-// rows with pivots in 2^+-64, X21), and 4-row groups whose live pivots leave
+// rows with pivots in 2^+-64, X21), and 8-row groups whose live pivots leave
 // 2^+-64 are renormalised by 2^-exponent(b) (warp-uniform test per group;
 // scaling a row by a power of two leaves c', d' unchanged and is exact, so the
 // two passes over a window need not take the same decisions).
@@ -44,7 +45,10 @@ namespace tri {
 
 constexpr int S5_R = 16;             // rows per lane
 constexpr int S5_W = 32 * S5_R;      // rows per window (512)
-constexpr int S5_G = 4;              // rows per streamed group
+#ifndef S5_G_DEF
+#define S5_G_DEF 8
+#endif
+constexpr int S5_G = S5_G_DEF;       // rows per streamed group
 #ifndef S5_NW_DEF
 #define S5_NW_DEF 8
 #endif
@@ -68,14 +72,14 @@ struct S5Layout {
     }
 };
 
-// rows 4 h .. 4 h + 3 of lane `lane` from the window's staging buffer: box row
+// rows G h .. G h + G - 1 of lane `lane` from the window's staging buffer: box row
 // `lane` of each array (128 bytes = 16 fp64), 16-byte chunk c at c ^ (lane & 7)
 __device__ __forceinline__ void s5_ld_group(const double* ib, int lane, int h, double (&a)[S5_G], double (&b)[S5_G],
                                             double (&c)[S5_G], double (&d)[S5_G]) {
     const int sw = lane & 7;
 #pragma unroll
-    for (int k = 0; k < 2; ++k) {
-        const int o = lane * 16 + (((2 * h + k) ^ sw) * 2);
+    for (int k = 0; k < S5_G / 2; ++k) {
+        const int o = lane * 16 + ((((S5_G / 2) * h + k) ^ sw) * 2);
         const double2 va = *reinterpret_cast<const double2*>(ib + 0 * S5_W + o);
         const double2 vb = *reinterpret_cast<const double2*>(ib + 1 * S5_W + o);
         const double2 vc = *reinterpret_cast<const double2*>(ib + 2 * S5_W + o);
@@ -250,7 +254,7 @@ __global__ void __launch_bounds__(S5_THREADS, 1) k_scan_w512(const __grid_consta
                     t1 = nt1; p1 = np1; d1 = nd1;
                     t2 = nt2; p2 = np2; d2 = nd2;
                 }
-                if (h & 1) {  // every 8 rows: exact power-of-two rescale
+                if (((h + 1) * S5_G) % 8 == 0) {  // every 8 rows: exact power-of-two rescale
                     const double s = sc_scale2(t1, t2);
                     t1 *= s; p1 *= s; d1 *= s; t2 *= s; p2 *= s; d2 *= s; d3 *= s;
                 }
@@ -329,7 +333,7 @@ __global__ void __launch_bounds__(S5_THREADS, 1) k_scan_w512(const __grid_consta
                     else sk_st_global_last(sp_g + 2 * (t * 32 + lane), c_, d_, pol_sp);
                     th = nt; ps = np; de = nd;
                 }
-                if (h & 1) {
+                if (((h + 1) * S5_G) % 8 == 0) {
                     const double s = sk_exp2_scale(th);
                     th *= s; ps *= s; de *= s;
                 }
