@@ -1100,16 +1100,26 @@ __global__ void __launch_bounds__(S16_NW * 32, 1) k_scan1_r16(const __grid_const
         sc_release_buf();  // this warp's reads of the buffer before the TMA refill
         if (lane == 0 && j + 2 * S16_NW < nstep) issue(j + 2 * S16_NW, b);
         // rows: a_0, c_{n-1} outside A; rows past n identity
-        bool out = false;
+        if (n == 16 * S16_R) {  // full windows (c4): row 0 and row n - 1 are fixed lane slots
+            if (seg == 0) ra[0] = 0.f;
+            if (seg == 15) rc[S16_R - 1] = 0.f;
+        } else {
+#pragma unroll
+            for (int u = 0; u < S16_R; ++u) {
+                const int i = 16 * seg + u;
+                if (i == 0) ra[u] = 0.f;
+                if (i == n - 1) rc[u] = 0.f;
+                if (i >= n || !live) { ra[u] = 0.f; rb[u] = 1.f; rc[u] = 0.f; rd[u] = 0.f; }
+            }
+        }
+        unsigned emx = 0u, emn = 0xffu;  // exponent range of the pivots
 #pragma unroll
         for (int u = 0; u < S16_R; ++u) {
-            const int64_t i = 16 * seg + u;
-            if (i == 0) ra[u] = 0.f;
-            if (i == n - 1) rc[u] = 0.f;
-            if (i >= n || !live) { ra[u] = 0.f; rb[u] = 1.f; rc[u] = 0.f; rd[u] = 0.f; }
             const unsigned e = ((unsigned)__float_as_int(rb[u]) >> 23) & 0xffu;
-            out |= (e - (127u - 8u)) > 16u;
+            emx = max(emx, e);
+            emn = min(emn, e);
         }
+        const bool out = emx > 127u + 8u || emn < 127u - 8u;
         // the 8-row partial products (rescaled at row 8) stay in fp32's range while
         // every pivot is within 2^+-8; otherwise (warp-uniform) every row is scaled
         // by 2^-exponent(b) -- exact row operations (X21)
