@@ -813,7 +813,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
         // this lane's system within its batch (S > 1): padding lanes past ms are identity rows
         const int64_t gq = blockIdx.x + (int64_t)cj * gridDim.x;
         const int64_t qf = S > 1 ? (gq - (gq / gpb) * gpb) * S + ls : 0;
-        const bool edge = cw == 0 || (int64_t)(cw + 1) * WR > n || (S > 1 && qf >= p.ms);
+        const bool edge = cw == 0 || (int64_t)(cw + 1) * WR >= n || (S > 1 && qf >= p.ms);  // holds row 0 or row n - 1
         auto load_rows = [&](T (&ra)[SC_R], T (&rb)[SC_R], T (&rc)[SC_R], T (&rd)[SC_R]) {
             if constexpr (S == 1) sc_ld_rows_any(ib, lane, p.w128 != 0, ra, rb, rc, rd);
             else sc_ld_rows_il<S>(ib, ls, seg, ra, rb, rc, rd);

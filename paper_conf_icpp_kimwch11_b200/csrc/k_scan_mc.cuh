@@ -224,7 +224,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan_mc(const __grid_constant
     for (int g = pw; g < nwin; g += SC_NW) {
         const int w = win_of(g);
         const int64_t i0 = (int64_t)w * SC_W + lane * SC_R;
-        const bool edge = w == 0 || (int64_t)(w + 1) * SC_W > n;
+        const bool edge = w == 0 || (int64_t)(w + 1) * SC_W >= n;  // holds row 0 or row n - 1
         sk_wait(&in_full[pw], ph);
         ph ^= 1u;
         if (MODE == 0) {
@@ -537,7 +537,7 @@ __global__ void __launch_bounds__(LB_THREADS, 1) k_scan_mc_lb(const __grid_const
         const int q = t / lb.Ps, w = (t - q * lb.Ps) * NCW + g;
         const int64_t i0 = (int64_t)w * SC_W + lane * SC_R;
         sc_ld_rows_any(buf, lane, p.w128 != 0, ra, rb, rc, rd);
-        if (w == 0 || (int64_t)(w + 1) * SC_W > n) {
+        if (w == 0 || (int64_t)(w + 1) * SC_W >= n) {  // holds row 0 or row n - 1
             if (p.n_al < n)
                 sc_patch_tail<T>(i0, p.n_al, n, p.ga + q * n, p.gb + q * n, p.gc + q * n, p.gd + q * n, ra, rb, rc, rd);
             sc_fix_rows<T>(i0, n, ra, rb, rc, rd, 0, 0);

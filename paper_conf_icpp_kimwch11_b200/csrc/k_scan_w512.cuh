@@ -233,7 +233,7 @@ __global__ void __launch_bounds__(S5_THREADS, 1) k_scan_w512(const __grid_consta
 
         // ---- forward: the lane's 16-row map, rows streamed from the staging buffer
         const int64_t i0 = (int64_t)cw * S5_W + lane * S5_R;
-        const bool edge = cw == 0 || (int64_t)(cw + 1) * S5_W > n;
+        const bool edge = cw == 0 || (int64_t)(cw + 1) * S5_W >= n;  // holds row 0 or row n - 1
         SCM M{1.0, 0.0, 0.0, 1.0, 0.0, 0.0, 1.0};
         unsigned scl = 0u;  // per 4-row group: renormalised (decided by the map pass)
         if (fwd) {

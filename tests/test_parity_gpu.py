@@ -1129,3 +1129,41 @@ def test_scan_w512_parity(cuda_ok, n, m, family):
     assert "w512=0" in plan.describe()
     x3, _ = gpu_solve(n, m, arrs, "f64", 0, plan=plan)
     check_parity(n, m, arrs, x3, "f64", 0, x_oracle=xo)
+
+
+@pytest.mark.parametrize("dtype,n,m,layout,variant,opt", [
+    ("f64", 1024, 40, 0, "SCAN", None),             # k_scan_w512, n a multiple of its 512-row window
+    ("f64", 1024, 40, 0, "SCAN", ("W512", 0)),      # k_scan, n a multiple of its 256-row window
+    ("f32", 768, 50, 0, "SCAN", None),              # k_scan fp32
+    ("f32", 256, 64, 0, "SCAN", None),              # k_scan1_r16 (c4's kernel)
+    ("f64", 256, 40, 0, "SCAN", None),              # one-window fp64
+    ("f64", 65536, 1, 0, "SCAN_MC", None),          # SCAN_MC, n a multiple of 256
+    ("f64", 65536, 1, 0, "SCAN_MC", ("LB", 32)),    # look-back SCAN_MC
+    ("f64", 1024, 64, 1, "SCAN", None),             # k_scan_grid
+    ("f64", 2048, 2048, 1, "SCAN", None),           # chained interleaved (beyond one wave)
+    ("f64", 1024, 64, 1, "SCAN", ("CL", 1)),        # thread-block cluster option
+    ("f64", 4800, 3, 0, "STREAM", None),            # STREAM, n a multiple of its 240-row window
+    ("f64", 2048, 150, 0, "FUSED", None),           # FUSED
+    ("f32", 1536, 200, 0, "FUSED", None),
+])
+def test_ignored_entries_nan_scan(cuda_ok, dtype, n, m, layout, variant, opt):
+    """a[q][0] and c[q][n-1] lie outside A (Eq 1, reading X1): NaN there must not
+    change x (bitwise) on the SCAN-family kernels, including systems whose length
+    is a multiple of the kernel's window (the last window must still drop c_{n-1})."""
+    import torch
+    arrs = gen(n, m, dtype, layout)
+    plan = tri.Plan(n, m, tri.F64 if dtype == "f64" else tri.F32, layout)
+    plan.variant = getattr(tri, "VARIANT_" + variant)
+    if opt is not None:
+        plan.set_option({"W512": tri.OPT_SCAN_W512, "LB": tri.OPT_SCAN_MC_LOOKBACK, "CL": tri.OPT_SCAN_CLUSTER}[opt[0]], opt[1])
+    a, b, c, d = to_dev(*arrs)
+    x1 = plan.solve(a, b, c, d).clone()
+    a2, c2 = a.clone(), c.clone()
+    if layout == 0:
+        a2.view(m, n)[:, 0] = float("nan")
+        c2.view(m, n)[:, -1] = float("nan")
+    else:
+        a2.view(n, m)[0, :] = float("nan")
+        c2.view(n, m)[-1, :] = float("nan")
+    x2 = plan.solve(a2, b, c2, d)
+    assert torch.equal(x1, x2), plan.describe()
