@@ -1167,3 +1167,32 @@ def test_ignored_entries_nan_scan(cuda_ok, dtype, n, m, layout, variant, opt):
         c2.view(n, m)[-1, :] = float("nan")
     x2 = plan.solve(a2, b, c2, d)
     assert torch.equal(x1, x2), plan.describe()
+
+
+@pytest.mark.parametrize("dtype,n,m,layout,variant", [
+    ("f64", 1024, 40, 0, "SCAN"), ("f64", 1032, 40, 0, "SCAN"), ("f32", 1024, 40, 0, "SCAN"),
+    ("f32", 256, 64, 0, "SCAN"), ("f64", 65536, 1, 0, "SCAN_MC"), ("f64", 1024, 64, 1, "SCAN"),
+    ("f64", 1024, 2048, 1, "SCAN")])
+def test_scan_kernels_16_byte_offsets(cuda_ok, dtype, n, m, layout, variant):
+    """Arrays that are 16-byte but not 32- / 128-byte aligned (views into larger
+    buffers; the ABI's only alignment rule is 16 bytes): the TMA descriptors take
+    any 16-byte base and the x stores fall back from 256-bit to narrower ones."""
+    import torch
+    arrs = gen(n, m, dtype, layout)
+    xo = oracle.solve_batch(n, m, *arrs, layout=layout)
+    tdt = torch.float64 if dtype == "f64" else torch.float32
+    off = 16 // (8 if dtype == "f64" else 4)
+    views = []
+    for t in arrs:
+        buf = torch.empty(n * m + 64, dtype=tdt, device="cuda")
+        v = buf[off:off + n * m]
+        v.copy_(torch.from_numpy(t))
+        views.append(v)
+    xbuf = torch.full((n * m + 64,), float("nan"), dtype=tdt, device="cuda")
+    x = xbuf[off:off + n * m]
+    assert x.data_ptr() % 32 == 16
+    plan = tri.Plan(n, m, tri.F64 if dtype == "f64" else tri.F32, layout)
+    plan.variant = getattr(tri, "VARIANT_" + variant)
+    plan.solve(*views, out=x)
+    check_parity(n, m, arrs, x.cpu().numpy(), dtype, layout, x_oracle=xo)
+    assert torch.isnan(xbuf[:off]).all() and torch.isnan(xbuf[off + n * m:]).all()
