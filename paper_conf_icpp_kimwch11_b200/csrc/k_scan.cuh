@@ -104,9 +104,9 @@ struct SCLayout {
     static constexpr int in_bytes = 4 * SC_W * (int)sizeof(T);           // one window, 4 arrays
     static constexpr int in_stride = (in_bytes + 1023) / 1024 * 1024;     // swizzle atoms aligned
     static constexpr int off_in = 0;
-    static constexpr int off_st = off_in + SC_NW * in_stride;             // [NW][<= 16 systems][theta|psi|delta]
-    static constexpr int off_xh = off_st + SC_NW * 16 * 4 * (int)sizeof(T);   // [NW][<= 16 systems] x handover
-    static constexpr int off_bar = (off_xh + SC_NW * 16 * (int)sizeof(T) + 7) / 8 * 8;  // [2][NW] in_full
+    static constexpr int off_st = off_in + SC_NW * in_stride;             // [NW][<= 32 systems][theta|psi|delta]
+    static constexpr int off_xh = off_st + SC_NW * 32 * 4 * (int)sizeof(T);   // [NW][<= 32 systems] x handover
+    static constexpr int off_bar = (off_xh + SC_NW * 32 * (int)sizeof(T) + 7) / 8 * 8;  // [2][NW] in_full
     static constexpr int off_cnt = off_bar + 2 * SC_NW * 8;               // the slot table follows
     // [K][NC] u32: tag(j) << 16 | slot of window (j, w) at row j % K, K = 3 +
     // (delta - 1) / NC systems in flight between a window's store and its

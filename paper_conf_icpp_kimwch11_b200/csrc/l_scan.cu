@@ -346,7 +346,7 @@ cudaError_t scan_t(tri_plan_s* p, const void* a, const void* b, const void* c, c
     const int smem = SCLayout<T>::smem_bytes(p->sk_nc, p->sk_delta, son_or_buf);
     const bool pr = A.prof != nullptr;
     void* kern = S == 1 ? scan_kernel<T, 1>(pr) : S == 2 ? scan_kernel<T, 2>(pr) : S == 4 ? scan_kernel<T, 4>(pr)
-                 : S == 8 ? scan_kernel<T, 8>(pr) : scan_kernel<T, 16>(pr);
+                 : S == 8 ? scan_kernel<T, 8>(pr) : S == 16 ? scan_kernel<T, 16>(pr) : scan_kernel<T, 32>(pr);
     cudaError_t e = set_smem(kern, smem);
     if (e != cudaSuccess) return e;
     void* args[] = {(void*)&tm, (void*)&A};

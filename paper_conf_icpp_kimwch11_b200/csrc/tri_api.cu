@@ -35,6 +35,12 @@ constexpr int64_t MAX_ELEMS = int64_t(1) << 40;
 // which the handover barrier chain alone would order every slot -- measured 3 %
 // slower at c5 and 8 % at c2, so the slots keep their release / acquire table)
 constexpr int SCAN_DELTA = 8;
+#ifndef S32_F64_NMAX
+#define S32_F64_NMAX 256           // fp64 interleaved: the longest systems the planner sends to S = 32
+#endif
+#ifndef S32_ENABLE
+#define S32_ENABLE 1               // interleaved SCAN with 32 systems per window (A/B macro)
+#endif
 #ifndef S5_DELTA
 #define S5_DELTA 8                 // k_scan_w512's lag (A/B macro)
 #endif
@@ -124,6 +130,23 @@ bool strided_fast(int64_t n, int64_t ms, int64_t nb, tri_dtype t, int64_t es, in
     return false;
 }
 
+// Interleaved SCAN with one system per lane (32 systems x 8 rows per window,
+// 256-byte TMA rows, no lane scans): a 32-system group's (c', d') slots
+// (cdiv(n, 8) + delta windows) live in the CTA's shared memory, the overflow in an
+// L2-resident spill of <= 24 MB over all CTAs, and there is a group for every SM.
+bool s32_ok(int64_t n, int64_t m, tri_dtype t, int sms) {
+    if (!S32_ENABLE) return false;
+    const int64_t nc32 = cdiv(n, SC_W / 32), groups = cdiv(m, 32);
+    if (nc32 > SC_NCMAX || groups < sms || n >= ((int64_t)1 << 31)) return false;
+    // smem_optin is not known here: the B200's 227 KB per CTA
+    const int64_t optin = 232448, slot = SC_W * 2 * (int64_t)esize(t);
+    const int64_t fixed = t == TRI_F64 ? SCLayout<double>::smem_bytes((int)nc32, SCAN_DELTA, 0)
+                                       : SCLayout<float>::smem_bytes((int)nc32, SCAN_DELTA, 0);
+    const int64_t on_chip = std::max<int64_t>(0, (optin - fixed) / slot);
+    const int64_t spill = std::max<int64_t>(0, nc32 + SCAN_DELTA - on_chip) * slot * std::min<int64_t>(groups, sms);
+    return spill <= ((int64_t)24 << 20);
+}
+
 // the arithmetic part of k_scan_grid's feasibility (scan_grid_geometry adds the
 // cluster occupancy check on the device)
 bool grid_shape_ok(int64_t n, int64_t m, int sms) {
@@ -181,6 +204,13 @@ tri_variant choose_variant(int64_t n, int64_t m, tri_dtype t, tri_layout layout,
         const bool fits = t == TRI_F64 ? N < ((int64_t)1 << 27) : N < ((int64_t)1 << 28) && m <= 16384;
         if (fits) return TRI_VARIANT_SCAN;
     }
+    // ... and many short interleaved systems, one system per lane (s32_ok;
+    // profiles/r02_sweep_s32.jsonl, back-to-back replays): fp64 n <= 128 and fp32
+    // 128 <= n <= 512 beat SPLIT k = 0 / WARP (fp64 n = 128, m = 2^20: 0.86 vs 1.22 ms;
+    // fp32 n = 256, m = 2^20 (c4 interleaved): 1.35 vs 1.51 ms); fp32 n <= 64 does not
+    if (layout == TRI_LAYOUT_INTERLEAVED && scan_ok(n, m, t, layout) && s32_ok(n, m, t, sms) &&
+        (t == TRI_F64 ? n <= S32_F64_NMAX : n >= 128 && n <= 512))
+        return TRI_VARIANT_SCAN;
     // STREAM (profiles/r01_sweep_stream_f64.jsonl): fp64 contiguous batches with
     // n % 8 == 0 are all taken by SCAN / SCAN_MC above; kept for completeness of
     // the rule list (the paper's fused PCR + p-Thomas, selectable).
@@ -305,6 +335,11 @@ void plan_geometry(tri_plan_s* p) {
     if (p->variant == TRI_VARIANT_SCAN) {
         p->L = n; p->n_pad = n; p->C = m;
         p->sk_S = p->layout == TRI_LAYOUT_STRIDED ? (p->es == 1 ? 1 : 8) : scan_systems(p->layout, m);
+        // many short interleaved systems: one system per lane (32 per window of 8 rows,
+        // 256-byte TMA rows, no lane scans) when a group's (c', d') slots fit the CTA's
+        // shared memory and there are groups for every SM
+        if (p->sk_S == 8 && p->nb == 1 && p->layout == TRI_LAYOUT_INTERLEAVED && s32_ok(n, m, p->dtype, p->sms))
+            p->sk_S = 32;
         p->sk_nc = (int)cdiv(n, SC_W / p->sk_S);
         const int64_t ms = p->ms;
         const int64_t groups = p->sk_S == 1 ? m : cdiv(ms, p->sk_S) * (m / ms);

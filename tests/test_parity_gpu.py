@@ -1196,3 +1196,16 @@ def test_scan_kernels_16_byte_offsets(cuda_ok, dtype, n, m, layout, variant):
     plan.solve(*views, out=x)
     check_parity(n, m, arrs, x.cpu().numpy(), dtype, layout, x_oracle=xo)
     assert torch.isnan(xbuf[:off]).all() and torch.isnan(xbuf[off + n * m:]).all()
+
+
+@pytest.mark.parametrize("dtype,n,m", [("f32", 256, 8192), ("f64", 256, 8192), ("f32", 100, 10000), ("f64", 64, 4800),
+                                       ("f32", 600, 5000), ("f64", 37, 6000)])
+def test_scan_interleaved_32_systems_per_window(cuda_ok, dtype, n, m):
+    """Interleaved SCAN with one system per lane (32 systems x 8 rows per window,
+    256-byte TMA rows, no lane scans) for many short systems: ragged rows and a
+    ragged last group of 32 systems, every element vs the oracle."""
+    arrs = gen(n, m, dtype, 1, "weak", eps=1e-2)
+    plan = tri.Plan(n, m, tri.F64 if dtype == "f64" else tri.F32, 1)
+    plan.variant = tri.VARIANT_SCAN
+    x, _ = gpu_solve(n, m, arrs, dtype, 1, plan=plan)
+    check_parity(n, m, arrs, x, dtype, 1)
