@@ -179,6 +179,12 @@ tri_variant choose_variant(int64_t n, int64_t m, tri_dtype t, tri_layout layout,
     // m = 1 .. 2^20 (fp64 and fp32), except fewer than 128 systems of 32 windows
     // or more, where one CTA per system leaves SMs idle; e.g. n = m = 16384 fp64:
     // 1.84 ms vs 2.92 ms (STREAM).  k = 0 throughout: the paper's M > P rule.
+    // ... except fp32 batches of many systems of 2-4 windows, where the chained
+    // fp32 windows (half the bytes of an fp64 step behind the same chain latency)
+    // lose to the TMA p-Thomas at k = 0 (r02 sweep: n = 512, m = 151552: 395 vs
+    // 539 us; n = 1024, m = 37888: 235 vs 268 us; equal from n = 2048)
+    if (layout == TRI_LAYOUT_CONTIGUOUS && t == TRI_F32 && n > 256 && n <= 1024 && m >= 256 * (int64_t)sms)
+        return TRI_VARIANT_SPLIT;
     if (layout == TRI_LAYOUT_CONTIGUOUS && scan_ok(n, m, t, layout) && (cdiv(n, SC_W) < 32 || m >= 128))
         return TRI_VARIANT_SCAN;
     // SCAN_MC: the remaining contiguous shapes (fewer than 128 systems of 32 windows
@@ -197,8 +203,9 @@ tri_variant choose_variant(int64_t n, int64_t m, tri_dtype t, tri_layout layout,
     // 32-system blocks x <= 8 row pieces of <= 256 rows, one CTA per SM; r02
     // sweep_grid: n = 1024, m = 64: 14.4 us vs 18.4 us ONCHIP; n = 2048, m = 64: 16.4
     // vs 28.7; n <= 256 stays with WARP / ONCHIP, 1.2-1.5x faster there)
-    if (layout == TRI_LAYOUT_INTERLEAVED && n > 256 && scan_ok(n, m, t, layout) && grid_shape_ok(n, m, sms))
-        return TRI_VARIANT_SCAN;
+    if (layout == TRI_LAYOUT_INTERLEAVED && (n > 256 || (n >= 128 && m >= (t == TRI_F64 ? 1024 : 4096))) &&
+        scan_ok(n, m, t, layout) && grid_shape_ok(n, m, sms))
+        return TRI_VARIANT_SCAN;  // (n = 128 .. 256, larger m: fp64 n = 256, m = 4096: 14.4 vs 22.2 us WARP)
     if (layout == TRI_LAYOUT_INTERLEAVED && m >= 256 && n > 256 && scan_ok(n, m, t, layout)) {
         const int64_t N = n * m;
         const bool fits = t == TRI_F64 ? N < ((int64_t)1 << 27) : N < ((int64_t)1 << 28) && m <= 16384;
