@@ -134,6 +134,7 @@ def test_shard_range_partitions(L, m, G):
     ("c5/2", 16384, 8192, "F64", 0, "VARIANT_SCAN", 0),  # one of 2 ranks (strong scaling)
     ("c5/8", 16384, 2048, "F64", 0, "VARIANT_SCAN", 0),  # one of 8 ranks
     ("c5-il", 16384, 16384, "F64", 1, "VARIANT_SPLIT", 0),  # interleaved layout: k = 0 TMA p-Thomas
+    ("c4-il", 256, 1 << 20, "F32", 1, "VARIANT_SCAN", 0),    # interleaved, one system per lane (S = 32)
     ("few-long", 65536, 37, "F64", 0, "VARIANT_SCAN_MC", 0),  # < 128 long systems: chunked SCAN
     ("few-long-il", 65536, 37, "F64", 1, "VARIANT_SPLIT", 8),  # interleaved: deep-k SPLIT
     ("odd-n", 1 << 20, 1, "F64", 0, "VARIANT_SCAN_MC", 0),

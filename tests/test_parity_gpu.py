@@ -872,13 +872,14 @@ def test_chain_interleaved_tma(cuda_ok, dtype, n, m, layout, k):
 @pytest.mark.parametrize("layout", [0, 1])
 def test_c4_auto_plan_sampled(cuda_ok, layout):
     """BASELINE config c4 at full size (n = 256, m = 2^20, fp32) through the auto
-    plan (M > P: k = 0; SCAN on the contiguous layout, TMA-streamed p-Thomas on
-    the interleaved one): sampled systems vs the oracle."""
+    plan (M > P: k = 0; SCAN on both layouts -- the interleaved one with one
+    system per lane, 32 per window, since round 2): sampled systems vs the oracle
+    (every system: test_full_size_every_system)."""
     import trigen
     n, m = 256, 1 << 20
     arrs = gen(n, m, "f32", layout, seed=trigen.SEED_BASE + 4)
     x, plan = gpu_solve(n, m, arrs, "f32", layout)
-    assert plan.variant == (SCAN if layout == 0 else SPLIT) and plan.k == 0
+    assert plan.variant == SCAN and plan.k == 0
     rng = np.random.default_rng(4)
     for q in rng.choice(m, 48, replace=False).tolist() + [0, m - 1]:
         sub = trigen.generate(n, 1, "f32", 0, "dd", seed=trigen.SEED_BASE + 4, q0=q)
