@@ -1,7 +1,7 @@
 # round-2 final validation: every -m gpu test, smoke, bench lines of c1..c5 (+ the
 # reference arm and a 2-rank code-path run), ncu of the c5 kernel, launch lists
 set -u
-O=gpurun_out/final5
+O=gpurun_out/final6
 mkdir -p $O
 timeout 2400 python -m pytest tests -q -m gpu -p no:cacheprovider --timeout 900 > $O/pytest_gpu.log 2>&1; echo "pytest rc=$?" >> $O/pytest_gpu.log
 timeout 300 python -c "import __graft_entry__ as g; g.build(); g.smoke()" > $O/smoke.log 2>&1; echo "smoke rc=$?" >> $O/smoke.log
@@ -15,3 +15,4 @@ python scripts/ncu_summary.py $O/c5_w512.ncu-rep $O/ncu_c5_w512.txt >> $O/ncu_c5
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file $O/launches_c5.csv python bench.py --steps 2 --warmup 1 --no-e2e --no-cpu > $O/ncu_launch_c5.log 2>&1
 rm -f $O/*.ncu-rep
 timeout 300 ncu --cache-control none --clock-control none --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum -k regex:k_scan_mc --launch-skip 3 -c 3 python scripts/prof_one.py 16777216 1 f64 0 0 - 2 > $O/ncu_c3_nocache.log 2>&1
+for c in c4 c5; do timeout 600 python bench.py --config $c --layout 1 --no-e2e --no-cpu > $O/bench_${c}_il.json 2> $O/bench_${c}_il.err; done
