@@ -49,7 +49,6 @@ constexpr int SG_NW = 16;            // warps per CTA
 constexpr int SG_THREADS = 32 * SG_NW;
 constexpr int SG_SR = 4;             // rows per TMA stage
 constexpr int SG_RMAX = 16;          // rows per warp (c', d' kept in registers)
-constexpr int SG_NSTMAX = SG_RMAX / SG_SR;
 constexpr int SG_NBUF = 3;          // TMA stage buffers per warp
 constexpr int SG_QMAX = 8;          // CTAs per block = cluster size (portable)
 
