@@ -282,15 +282,32 @@ __device__ __forceinline__ void sc_patch_tail(int64_t i0, int64_t n_al, int64_t 
 // rows are renormalised in registers by 2^-e (e = exponent of b; exact, a row
 // operation that leaves c', d' unchanged, reading X21), so any |b| in fp64's
 // range works.  Called after sc_fix_rows, on warp-converged code only.
-// fp32 rows are always scaled by 2^-e here (once per load; the product of 8 raw
-// fp32 rows would leave fp32's range beyond |b| ~ 2^16).
+// fp32 rows likewise, with the window's pivots inside 2^+-8 (the product of 8 raw
+// fp32 rows then stays inside 2^+-64; r01 scaled every fp32 row unconditionally,
+// ~14 % of the interleaved kernel's instructions).
 template <typename T>
 __device__ __forceinline__ void sc_range(T (&ra)[SC_R], T (&rb)[SC_R], T (&rc)[SC_R], T (&rd)[SC_R], int* known = nullptr) {
     if constexpr (sizeof(T) == 4) {
+        bool scale;
+        if (known && *known >= 0) {
+            scale = *known != 0;
+        } else {
+            unsigned mx = 0u, mn = 0xffu;  // biased exponents of the pivots
 #pragma unroll
-        for (int u = 0; u < SC_R; ++u) {
-            const T s = sk_exp2_scale(rb[u]);
-            ra[u] *= s; rb[u] *= s; rc[u] *= s; rd[u] *= s;
+            for (int u = 0; u < SC_R; ++u) {
+                const unsigned e = ((unsigned)__float_as_int(rb[u]) >> 23) & 0xffu;
+                mx = max(mx, e);
+                mn = min(mn, e);
+            }
+            scale = __any_sync(0xffffffffu, mx > 127u + 8u || mn < 127u - 8u);
+            if (known) *known = scale ? 1 : 0;
+        }
+        if (scale) {
+#pragma unroll
+            for (int u = 0; u < SC_R; ++u) {
+                const T s = sk_exp2_scale(rb[u]);
+                ra[u] *= s; rb[u] *= s; rc[u] *= s; rd[u] *= s;
+            }
         }
     } else {
         // `known`: the decision of an earlier load of the same rows (-1: not taken yet)
@@ -633,7 +650,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
                 sc_tma4d(buf + 3 * SC_W, &tm.d, y, sq, bt, bar, pol_in);
             }
         } else {  // tensor [nb][n][ms], box [1][WR][S]
-            const int bt = (int)(q / gpb), xq = (int)(q - bt * gpb) * S, y = ww * WR;
+            const int bt = p.nb == 1 ? 0 : (int)(q / gpb), xq = (int)(q - bt * gpb) * S, y = ww * WR;
             sc_tma3d(buf + 0 * SC_W, &tm.a, y, bt, bar, pol_in, xq);
             sc_tma3d(buf + 1 * SC_W, &tm.b, y, bt, bar, pol_in, xq);
             sc_tma3d(buf + 2 * SC_W, &tm.c, y, bt, bar, pol_in, xq);
@@ -812,7 +829,7 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
         const int64_t i0 = (int64_t)cw * WR + seg * SC_R;
         // this lane's system within its batch (S > 1): padding lanes past ms are identity rows
         const int64_t gq = blockIdx.x + (int64_t)cj * gridDim.x;
-        const int64_t qf = S > 1 ? (gq - (gq / gpb) * gpb) * S + ls : 0;
+        const int64_t qf = S > 1 ? (p.nb == 1 ? gq : gq - (gq / gpb) * gpb) * S + ls : 0;
         const bool edge = cw == 0 || (int64_t)(cw + 1) * WR >= n || (S > 1 && qf >= p.ms);  // holds row 0 or row n - 1
         auto load_rows = [&](T (&ra)[SC_R], T (&rb)[SC_R], T (&rc)[SC_R], T (&rd)[SC_R]) {
             if constexpr (S == 1) sc_ld_rows_any(ib, lane, p.w128 != 0, ra, rb, rc, rd);
@@ -915,12 +932,17 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
             if constexpr (S == 1) {
                 sc_store_x(xbase(qb) + xr, n - xr, xv, p.x32 != 0);
             } else {  // INTERLEAVED / BATCHED: x[(batch n + row) ms + s]
-                const int64_t bt = qb / gpb, qx = (qb - bt * gpb) * S + ls;
+                const int64_t bt = p.nb == 1 ? 0 : qb / gpb, qx = (qb - bt * gpb) * S + ls;
                 if (qx < p.ms) {
-                    T* xo = p.x + bt * p.xbat + qx;
+                    const int64_t xel = p.xel;
+                    T* xp = p.x + bt * p.xbat + qx + xr * xel;  // walked one row stride at a time
+                    if (xr + SC_R <= n) {
 #pragma unroll
-                    for (int t = 0; t < SC_R; ++t)
-                        if (xr + t < n) __stcs(xo + (xr + t) * p.xel, xv[t]);
+                        for (int t = 0; t < SC_R; ++t) { __stcs(xp, xv[t]); xp += xel; }
+                    } else {
+#pragma unroll
+                        for (int t = 0; t < SC_R; ++t) { if (xr + t < n) __stcs(xp, xv[t]); xp += xel; }
+                    }
                 }
             }
         }
