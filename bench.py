@@ -378,7 +378,7 @@ def main():
     b2b = None
     if flush and graph is not None and rank == 0:
         try:
-            kk = args.steps
+            kk = int(max(2, min(args.steps, 8e9 // max(1, 5 * n_unknowns * s))))  # <= ~8 GB of copies
             cps = [[t.clone() for t in (a, b, c, d, x)] for _ in range(kk)]
             cap2 = torch.cuda.Stream()
             cap2.wait_stream(stream)
