@@ -104,7 +104,7 @@ struct SCLayout {
     static constexpr int in_bytes = 4 * SC_W * (int)sizeof(T);           // one window, 4 arrays
     static constexpr int in_stride = (in_bytes + 1023) / 1024 * 1024;     // swizzle atoms aligned
     static constexpr int off_in = 0;
-    static constexpr int off_st = off_in + SC_NW * in_stride;             // [NW][<= 32 systems][theta|psi|delta]
+    static constexpr int off_st = off_in + SC_NW * in_stride;             // [theta|psi|delta|-][NW][32 systems]
     static constexpr int off_xh = off_st + SC_NW * 32 * 4 * (int)sizeof(T);   // [NW][<= 32 systems] x handover
     static constexpr int off_bar = (off_xh + SC_NW * 32 * (int)sizeof(T) + 7) / 8 * 8;  // [2][NW] in_full
     static constexpr int off_cnt = off_bar + 2 * SC_NW * 8;               // the slot table follows
@@ -873,9 +873,9 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
         const T xw = (bwd && wb < NC - 1) ? xh[pi * S + ls] : T(0);  // x at the first row of window wb + 1
         T th = T(1), ps = T(0), de = T(0);                  // theta_{-1} = 1, psi_0 = 0, delta_{-1} = 0
         if (fwd && cw > 0) {
-            th = stt[(pi * S + ls) * 4 + 0];
-            ps = stt[(pi * S + ls) * 4 + 1];
-            de = stt[(pi * S + ls) * 4 + 2];
+            th = stt[(0 * SC_NW + pi) * 32 + ls];
+            ps = stt[(1 * SC_NW + pi) * 32 + ls];
+            de = stt[(2 * SC_NW + pi) * 32 + ls];
         }
         const T xs = fma(be, xw, al);  // x at the lane's first row
         const double ot = fma(M.a, (double)th, M.b * (double)ps);
@@ -884,9 +884,9 @@ __global__ void __launch_bounds__(SC_THREADS, 1) k_scan(const __grid_constant__ 
         if (seg == 0) xh[pw * S + ls] = xs;
         if (seg == NSEG - 1) {  // window end: exact power-of-two rescale, hand over
             const double sc = sk_exp2_scale(ot);
-            stt[(pw * S + ls) * 4 + 0] = (T)(ot * sc);
-            stt[(pw * S + ls) * 4 + 1] = (T)(op * sc);
-            stt[(pw * S + ls) * 4 + 2] = (T)(od * sc);
+            stt[(0 * SC_NW + pw) * 32 + ls] = (T)(ot * sc);
+            stt[(1 * SC_NW + pw) * 32 + ls] = (T)(op * sc);
+            stt[(2 * SC_NW + pw) * 32 + ls] = (T)(od * sc);
         }
         if (g + 1 < total && p.dbg != 1)  // arrive -> sync: release / acquire (PTX memory model)
             asm volatile("bar.arrive %0, 64;" ::"r"(1 + pw) : "memory");
