@@ -351,7 +351,11 @@ void plan_geometry(tri_plan_s* p) {
         const int64_t ms = p->ms;
         const int64_t groups = p->sk_S == 1 ? m : cdiv(ms, p->sk_S) * (m / ms);
         p->sk_grid = (int)std::min<int64_t>(groups, p->sms);
-        p->sk_delta = SCAN_DELTA;
+        // the back-substitution lag only matters when a CTA's slots are reused by a
+        // later system: with one system (group) per CTA the backward sweep starts right
+        // after the forward one (c1: no chain of idle steps)
+        const bool one_per_cta = groups <= p->sms;
+        p->sk_delta = one_per_cta ? 0 : SCAN_DELTA;
         const int fixed = SCLayout<double>::smem_bytes(p->sk_nc, p->sk_delta, 0);
         const int fixed32 = SCLayout<float>::smem_bytes(p->sk_nc, p->sk_delta, 0);
         const int slot = p->dtype == TRI_F64 ? SCLayout<double>::slot_bytes : SCLayout<float>::slot_bytes;
@@ -366,7 +370,7 @@ void plan_geometry(tri_plan_s* p) {
             p->n % 16 == 0 && cdiv(n, S5_W) >= 2 && cdiv(n, S5_W) <= SC_NCMAX) {
             p->s5 = 1;
             p->sk_nc = (int)cdiv(n, S5_W);
-            p->sk_delta = S5_DELTA;
+            p->sk_delta = one_per_cta ? 0 : S5_DELTA;
             const int64_t av5 = ((int64_t)p->smem_optin - S5Layout::smem_bytes(p->sk_nc, p->sk_delta, 0)) / S5Layout::slot_bytes;
             p->sk_son = (int)std::max<int64_t>(0, std::min<int64_t>(p->sk_nc + p->sk_delta, av5));
         }
