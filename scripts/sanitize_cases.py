@@ -34,6 +34,10 @@ CASES = {
     # blocks (m % 32), rows past n, 1 / 3 / 4 stages per warp, Q = 1 .. 8
     "scan_grid": [(1024, 40, "f64", 1, V.VARIANT_SCAN, None), (700, 36, "f32", 1, V.VARIANT_SCAN, None),
                   (60, 12, "f64", 1, V.VARIANT_SCAN, None), (2000, 32, "f64", 1, V.VARIANT_SCAN, None)],
+    # k_scan_w512: 512-row fp64 windows (contiguous); several windows, ragged n,
+    # one system per CTA (back-substitution lag 0) and more systems than SMs (lag 8)
+    "scan_w512": [(2048, 3, "f64", 0, V.VARIANT_SCAN, "w512"), (1000, 5, "f64", 0, V.VARIANT_SCAN, "w512"),
+                  (1024, 1, "f64", 0, V.VARIANT_SCAN, "w512"), (1536, 200, "f64", 0, V.VARIANT_SCAN, "w512")],
     "scan_r16": [(256, 40, "f32", 0, V.VARIANT_SCAN, None), (224, 33, "f32", 0, V.VARIANT_SCAN, None)],
     "scan_mc": [(1 << 16, 1, "f64", 0, V.VARIANT_SCAN_MC, None),
                 (40960, 2, "f32", 0, V.VARIANT_SCAN_MC, None),
@@ -70,6 +74,8 @@ def main():
                 plan.k = int(k[5:])
             elif k == "grid0":  # interleaved SCAN through the chained kernel
                 plan.set_option(tri.OPT_SCAN_GRID, 0)
+            elif k == "w512":  # fp64 contiguous SCAN through k_scan_w512
+                plan.set_option(tri.OPT_SCAN_W512, 1)
             elif isinstance(k, str):  # "lbW": SCAN_MC look-back with W-window chunks
                 plan.set_option(tri.OPT_SCAN_MC_LOOKBACK, int(k[2:]))
             elif k is not None:

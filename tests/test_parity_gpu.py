@@ -1212,3 +1212,62 @@ def test_scan_interleaved_32_systems_per_window(cuda_ok, dtype, n, m):
     plan.variant = tri.VARIANT_SCAN
     x, _ = gpu_solve(n, m, arrs, dtype, 1, plan=plan)
     check_parity(n, m, arrs, x, dtype, 1)
+
+
+@pytest.mark.parametrize("dtype,n,m,layout,variant,opt,k", [
+    ("f64", 1024, 1, 0, "SCAN", None, None),             # k_scan_w512, one system (lag 0)
+    ("f64", 1000, 5, 0, "SCAN", ("W512", 1), None),      # k_scan_w512, ragged last window
+    ("f64", 1536, 200, 0, "SCAN", None, None),           # k_scan_w512, more systems than SMs
+    ("f64", 1032, 40, 0, "SCAN", ("W512", 0), None),     # k_scan
+    ("f32", 1000, 7, 0, "SCAN", None, None),             # k_scan fp32, ragged
+    ("f32", 224, 33, 0, "SCAN", None, None),             # k_scan1_r16
+    ("f64", 200, 41, 0, "SCAN", None, None),             # one-window fp64
+    ("f64", 65537, 1, 0, "SCAN_MC", None, None),         # SCAN_MC, ragged n
+    ("f64", 65536, 1, 0, "SCAN_MC", ("LB", 32), None),   # look-back SCAN_MC
+    ("f64", 700, 36, 1, "SCAN", None, None),             # k_scan_grid, ragged block and rows
+    ("f32", 520, 24, 1, "SCAN", ("GRID", 0), None),      # chained interleaved, ragged window
+    ("f64", 4800, 3, 0, "STREAM", None, None),
+    ("f64", 2000, 3, 0, "FUSED", None, None),
+    ("f64", 512, 16, 0, "WARP", None, None),
+    ("f32", 1000, 3, 0, "ONCHIP", None, 4),
+    ("f64", 5003, 3, 0, "SPLIT", None, 9),               # register-tile passes + p-Thomas
+    ("f64", 1000, 37, 1, "SPLIT", None, 7),
+    ("f64", 4096, 2, 0, "SPLIT", ("TMA", 0), 12),        # the paper's sliding window
+])
+def test_guard_bands_and_const_inputs(cuda_ok, dtype, n, m, layout, variant, opt, k):
+    """Every kernel family writes x and nothing else a caller owns: each array
+    sits between 4096-element guard bands of random bits; after the solve the
+    guards of all five buffers and the whole of a, b, c, d (const in tri.h) are
+    bitwise unchanged, and x matches the oracle.  (Our own out-of-bounds check:
+    compute-sanitizer is closed on the GPU pool, profiles/r02_sanitize.)"""
+    import torch
+    arrs = gen(n, m, dtype, layout)
+    xo = oracle.solve_batch(n, m, *arrs, layout=layout)
+    tdt, idt = (torch.float64, torch.int64) if dtype == "f64" else (torch.float32, torch.int32)
+    G, N = 4096, n * m
+    g = torch.Generator().manual_seed(n * 131 + m)
+    bufs, views = [], []
+    for t in list(arrs) + [None]:
+        bits = torch.randint(-2**31, 2**31 - 1, (N + 2 * G,), generator=g, dtype=torch.int64).to(idt)
+        buf = bits.view(tdt).cuda()
+        v = buf[G:G + N]
+        if t is not None:
+            v.copy_(torch.from_numpy(t))
+        bufs.append(buf)
+        views.append(v)
+    before = [b_.view(idt).clone() for b_ in bufs]
+    plan = tri.Plan(n, m, tri.F64 if dtype == "f64" else tri.F32, layout)
+    plan.variant = getattr(tri, "VARIANT_" + variant)
+    if opt is not None:
+        plan.set_option({"W512": tri.OPT_SCAN_W512, "LB": tri.OPT_SCAN_MC_LOOKBACK, "GRID": tri.OPT_SCAN_GRID,
+                         "TMA": tri.OPT_TMA}[opt[0]], opt[1])
+    if k is not None:
+        plan.k = k
+    plan.solve(*views[:4], out=views[4])
+    torch.cuda.synchronize()
+    for i in range(4):
+        assert torch.equal(bufs[i].view(idt), before[i]), f"input {'abcd'[i]} modified [{plan.describe()}]"
+    xb = bufs[4].view(idt)
+    assert torch.equal(xb[:G], before[4][:G]), f"write below x [{plan.describe()}]"
+    assert torch.equal(xb[G + N:], before[4][G + N:]), f"write past x [{plan.describe()}]"
+    check_parity(n, m, arrs, views[4].cpu().numpy(), dtype, layout, x_oracle=xo)
