@@ -1,7 +1,7 @@
 # round-2 final validation: every -m gpu test, smoke, bench lines of c1..c5 (+ the
 # reference arm and a 2-rank code-path run), ncu of the c5 kernel, launch lists
 set -u
-O=gpurun_out/final8
+O=gpurun_out/final9
 mkdir -p $O
 timeout 2400 python -m pytest tests -q -m gpu -p no:cacheprovider --timeout 900 > $O/pytest_gpu.log 2>&1; echo "pytest rc=$?" >> $O/pytest_gpu.log
 timeout 300 python -c "import __graft_entry__ as g; g.build(); g.smoke()" > $O/smoke.log 2>&1; echo "smoke rc=$?" >> $O/smoke.log

@@ -1271,3 +1271,19 @@ def test_guard_bands_and_const_inputs(cuda_ok, dtype, n, m, layout, variant, opt
     assert torch.equal(xb[:G], before[4][:G]), f"write below x [{plan.describe()}]"
     assert torch.equal(xb[G + N:], before[4][G + N:]), f"write past x [{plan.describe()}]"
     check_parity(n, m, arrs, views[4].cpu().numpy(), dtype, layout, x_oracle=xo)
+
+
+@pytest.mark.parametrize("dtype,n,m,w512", [("f64", 65544, 2, 0), ("f64", 65536, 1, 1), ("f32", 1 << 17, 1, 0),
+                                            ("f64", 30000, 150, 0), ("f64", 30208, 150, 1)])
+def test_scan_spilled_slots_lag(cuda_ok, dtype, n, m, w512):
+    """SCAN with more windows than on-chip slots (the spill to global scratch):
+    one system per CTA (no back-substitution lag, the backward sweep reads the
+    last window right after its store) and more systems than SMs (lag 8, slots
+    reused by the CTA's next system) -- every element vs the oracle."""
+    arrs = gen(n, m, dtype, 0, "weak", eps=1e-2)
+    plan = tri.Plan(n, m, tri.F64 if dtype == "f64" else tri.F32, 0)
+    plan.variant = tri.VARIANT_SCAN
+    if dtype == "f64":
+        plan.set_option(tri.OPT_SCAN_W512, w512)
+    x, _ = gpu_solve(n, m, arrs, dtype, 0, plan=plan)
+    check_parity(n, m, arrs, x, dtype, 0)
